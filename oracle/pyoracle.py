@@ -1,0 +1,69 @@
+"""Pure-Python twins of the oracle for tiny inputs -- TEST INFRASTRUCTURE ONLY.
+
+brute(R, Q, L): the MEM definition checked cell by cell:
+    (r, q, lam) with R[r+i] == Q[q+i] for i < lam, lam >= L,
+    (r == 0 or q == 0 or R[r-1] != Q[q-1])        -- left-maximal (end = mismatch, reading R3)
+    (r+lam == |R| or q+lam == |Q| or R[r+lam] != Q[q+lam])  -- right-maximal
+  enumerated over every start cell (r, q): O(|R||Q| * lam). Independent of the
+  C++ brute force (which walks diagonals).
+
+sampled(R, Q, L, ls, step): the paper's method in its own words
+  (index every step-th ls-mer of R, look up every query position, extend both
+  ways, keep >= L, deduplicate) with a dict -- the Python twin of oracle_mems.
+
+homopolymer(n, m, L): closed form for R = A^n, Q = A^m:
+  every MEM touches a sequence start on one side and an end on the other:
+  {(0, q, min(n, m-q)) : q < m} U {(r, 0, min(n-r, m)) : 1 <= r < n}, lam >= L.
+"""
+from __future__ import annotations
+
+
+def _s(x):
+    if isinstance(x, (bytes, bytearray)):
+        x = x.decode("ascii")
+    elif not isinstance(x, str):
+        x = bytes(x).decode("ascii")
+    return x.upper()
+
+
+def brute(R, Q, L):
+    R, Q = _s(R), _s(Q)
+    out = []
+    for r in range(len(R)):
+        for q in range(len(Q)):
+            if r > 0 and q > 0 and R[r - 1] == Q[q - 1]:
+                continue  # not left-maximal
+            lam = 0
+            while r + lam < len(R) and q + lam < len(Q) and R[r + lam] == Q[q + lam]:
+                lam += 1
+            # (r+lam, q+lam) is now an end or a mismatch: right-maximal by construction
+            if lam >= L:
+                out.append((r, q, lam))
+    return sorted(out)
+
+
+def sampled(R, Q, L, ls, step=None):
+    R, Q = _s(R), _s(Q)
+    if step is None:
+        step = L - ls + 1
+    H = {}
+    for p in range(0, len(R) - ls + 1, step):
+        H.setdefault(R[p:p + ls], []).append(p)
+    found = set()
+    for q in range(0, len(Q) - ls + 1):
+        for p in H.get(Q[q:q + ls], ()):
+            a = 0
+            while a < p and a < q and R[p - a - 1] == Q[q - a - 1]:
+                a += 1
+            b = ls
+            while p + b < len(R) and q + b < len(Q) and R[p + b] == Q[q + b]:
+                b += 1
+            if a + b >= L:
+                found.add((p - a, q - a, a + b))
+    return sorted(found)
+
+
+def homopolymer(n, m, L):
+    out = {(0, q, min(n, m - q)) for q in range(m)}
+    out |= {(r, 0, min(n - r, m)) for r in range(1, n)}
+    return sorted(t for t in out if t[2] >= L and t[2] > 0)
