@@ -1,0 +1,167 @@
+/*
+ * include/gpumem.h -- C ABI of libgpumem.so, the B200 (sm_100a) MEM finder.
+ *
+ * Problem (Sec. II): given a reference R, a query Q over
+ * Sigma = {A,C,G,T} (:58) and an integer L, report every maximal exact match
+ * (r, q, len): R[r+i] == Q[q+i] for i < len, len >= L, R[r-1] != Q[q-1] and
+ * R[r+len] != Q[q+len], where a sequence end counts as a mismatch
+ * (reading R3). Positions are 0-based; sequences hold < 2^32 bases
+ * (32-bit locations).
+ *
+ * Method (GPUMEM, Sec. III): index every step-th seed of length
+ * seed_len of R with step = L - seed_len + 1 (Eq. 1, :86-90), look up the seed
+ * at every query position, extend each hit both ways, keep len >= L and report
+ * each MEM once (:151-153, :171-173). Every step runs in hand-written CUDA
+ * kernels on the caller's device; there is no CPU fallback.
+ *
+ * Conventions for every call:
+ *  - Device: the calling thread's current CUDA device (cudaSetDevice). All
+ *    handles passed to one call must live on that device.
+ *  - Streams: `cuda_stream` is a cudaStream_t passed as void* (NULL = the legacy
+ *    default stream). Work is enqueued on it; calls documented "async" return
+ *    before the GPU finishes. Handles are immutable after creation, so several
+ *    streams may read one handle concurrently; the caller orders creation,
+ *    use and gpumem_free across streams (free is enqueued on the handle's
+ *    creation stream).
+ *  - Memory: the library allocates device memory through the allocator hook
+ *    (default: cudaMallocAsync / cudaFreeAsync on the stream, pool kept cached).
+ *    Every handle is owned by the caller and released with gpumem_free.
+ *  - Errors: every call returns gpumem_status. On failure *out is set to NULL,
+ *    nothing leaks, and gpumem_last_error() (thread-local) says why. CUDA
+ *    errors map to GPUMEM_ERR_CUDA with cudaGetErrorString's text. No call
+ *    aborts or exits.
+ */
+#ifndef GPUMEM_H
+#define GPUMEM_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    GPUMEM_OK = 0,
+    GPUMEM_ERR_ARG = 1,         /* bad argument (NULL, ls/L/step out of range, wrong handle type) */
+    GPUMEM_ERR_ALPHABET = 2,    /* a byte outside {A,C,G,T,a,c,g,t} (Sigma; reading R4) */
+    GPUMEM_ERR_RANGE = 3,       /* length >= 2^32, q range outside Q, host buffer too small */
+    GPUMEM_ERR_NOMEM = 4,       /* allocator returned NULL */
+    GPUMEM_ERR_CUDA = 5,        /* a CUDA runtime error (message in gpumem_last_error) */
+    GPUMEM_ERR_UNSUPPORTED = 6  /* no sm_100 device / unsupported request */
+} gpumem_status;
+
+typedef struct gpumem_seq gpumem_seq;     /* 2-bit packed sequence resident on one device        */
+typedef struct gpumem_index gpumem_index; /* ptrs[4^ls+1], locs[n_locs], occupancy bitmap; refs R  */
+typedef struct gpumem_mems gpumem_mems;   /* MEM set sorted by (r, q), device-resident            */
+
+/* One MEM (Table I :34-35): R[r .. r+len) == Q[q .. q+len). 12 bytes, AoS. */
+typedef struct {
+    uint32_t r, q, len;
+} gpumem_triple;
+
+/*
+ * gpumem_pack -- 2-bit encode a sequence (A=00, C=01, G=10, T=11).
+ *  bases            n ASCII bytes; lowercase is folded; anything else is an alphabet error.
+ *  bases_on_device  1: `bases` is a device pointer on the current device (read in place);
+ *                   0: `bases` is host memory, copied to the device inside the call
+ *                      (async if pinned) -- the copy is part of this call's stream work.
+ *  Layout of the result: uint64 words, base i in bits [63-2(i%32), 62-2(i%32)] of
+ *  word i/32 (first base most significant), 2 zero words of padding after the last.
+ *  Async. Alphabet validation runs on the GPU; its verdict is reported by
+ *  gpumem_seq_check() and by gpumem_find_mems() (which synchronises anyway).
+ *  n == 0 is allowed (empty sequence). n >= 2^32 -> GPUMEM_ERR_RANGE.
+ */
+gpumem_status gpumem_pack(const char *bases, uint64_t n, int bases_on_device,
+                          void *cuda_stream, gpumem_seq **out);
+
+/* Synchronises `cuda_stream`; GPUMEM_ERR_ALPHABET (with the first bad position in the
+ * message) if the packed input held a byte outside the alphabet, else GPUMEM_OK. */
+gpumem_status gpumem_seq_check(const gpumem_seq *s, void *cuda_stream);
+
+/* Length in bases and the device pointer to the packed words (borrowed). */
+gpumem_status gpumem_seq_info(const gpumem_seq *s, uint64_t *n_bases, const uint64_t **dev_words,
+                              uint64_t *n_words);
+
+/*
+ * gpumem_index_build -- GPUMEM's lightweight index of R (Sec. III-A, Alg. 1 :102-106).
+ *  seed_len (ls) in [1, 15], min_len (L) >= ls, step = L - ls + 1 (the maximum allowed by
+ *  Eq. 1, :88-90). Indexed locations: p = 0, step, 2*step, ... <= |R| - ls (reading R6).
+ *  Result: ptrs (4^ls + 1 uint32, ptrs[s] = first slot of seed s, ptrs[4^ls] = n_locs, :84)
+ *  and locs (n_locs uint32, sorted ascending inside each seed, Alg. 1 step 4), plus a
+ *  4^ls-bit occupancy bitmap used by the lookup. ptrs alone takes 4*(4^ls+1) bytes
+ *  (268 MB at ls = 13). The index references R: R must outlive it. Async.
+ */
+gpumem_status gpumem_index_build(const gpumem_seq *R, uint32_t seed_len, uint32_t min_len,
+                                 void *cuda_stream, gpumem_index **out);
+
+/* Test-only: same with an explicit step in [1, L - ls + 1] (the MEM set does not depend on it). */
+gpumem_status gpumem_index_build_step(const gpumem_seq *R, uint32_t seed_len, uint32_t min_len,
+                                      uint32_t step, void *cuda_stream, gpumem_index **out);
+
+/* Borrowed device pointers to ptrs (4^ls + 1 entries) and locs (n_locs entries). */
+gpumem_status gpumem_index_view(const gpumem_index *idx, const uint32_t **dev_ptrs,
+                                const uint32_t **dev_locs, uint64_t *n_locs);
+
+/*
+ * gpumem_find_mems -- every MEM of (R, Q, L) whose query start q lies in [q_begin, q_end)
+ *  (q_end clamped to |Q|; 0, UINT64_MAX = all of Q), sorted ascending by (r, q), each
+ *  exactly once (PAPER.md:153 "not to extract a MEM more than once", :185). The set is
+ *  independent of ls and step. q_begin > |Q| -> GPUMEM_ERR_RANGE.
+ *  Synchronises the stream once (the output size is data-dependent) and reports an
+ *  alphabet error of R or Q here. Edge cases: |R| < ls or |Q| < L -> OK with 0 MEMs;
+ *  R == Q includes (0, 0, |R|). Forward strand only.
+ */
+gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uint64_t q_begin,
+                               uint64_t q_end, void *cuda_stream, gpumem_mems **out);
+
+/* Borrowed device pointer to the sorted triples and their count. */
+gpumem_status gpumem_mems_view(const gpumem_mems *m, const gpumem_triple **dev_ptr, uint64_t *count);
+
+/* Copy the triples to host memory (synchronous); capacity < count -> GPUMEM_ERR_RANGE. */
+gpumem_status gpumem_mems_to_host(const gpumem_mems *m, gpumem_triple *host_buf, uint64_t capacity);
+
+/*
+ * gpumem_merge_sorted -- merge n_runs device arrays of triples, each sorted by (r, q), into
+ *  one sorted set (multi-GPU rank-0 merge of query shards; shards are disjoint by the
+ *  ownership rule so no duplicates arise). Runs are read, not modified. Synchronises once.
+ */
+gpumem_status gpumem_merge_sorted(const gpumem_triple *const *dev_runs, const uint64_t *counts,
+                                  int n_runs, void *cuda_stream, gpumem_mems **out);
+
+/* Release any handle above (seq, index, mems). NULL is a no-op. */
+void gpumem_free(void *handle);
+
+/* Thread-local text of the last failure ("" if none). */
+const char *gpumem_last_error(void);
+
+/* Allocator hook (e.g. the torch caching allocator). Both NULL restores the default. */
+gpumem_status gpumem_set_allocator(void *(*alloc_fn)(size_t bytes, void *cuda_stream, void *ctx),
+                                   void (*free_fn)(void *ptr, void *cuda_stream, void *ctx), void *ctx);
+
+/* ---- instrumentation and tuning (not part of the method) ---------------------------- */
+
+/* Tuning knobs; the MEM set never depends on them. Names:
+ *  "find_grid"        CTAs of the find kernel (0 = SMs x occupancy)
+ *  "find_spill"       bucket size above which hits are spilled to the heavy queue
+ *  "out_capacity"     initial output capacity in triples (0 = automatic; small values
+ *                     force the overflow-and-retry path in tests)
+ *  "use_bitmap"       1 (default) probe the occupancy bitmap before ptrs, 0 probe ptrs only */
+gpumem_status gpumem_set_option(const char *name, int64_t value);
+
+/* Per-stage device time: when enabled, CUDA events bracket each stage on its stream.
+ * gpumem_profile_read synchronises those events, writes up to max_stages
+ * (name, total ms, launches) entries and resets the accumulators. */
+gpumem_status gpumem_profile_enable(int on);
+int gpumem_profile_read(const char **names, double *ms, uint64_t *launches, int max_stages);
+
+/* Kernels this library has launched in this process (monotone counter). */
+uint64_t gpumem_launch_count(void);
+
+/* Library version string. */
+const char *gpumem_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* GPUMEM_H */

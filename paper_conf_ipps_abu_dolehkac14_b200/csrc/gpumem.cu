@@ -1,0 +1,622 @@
+// gpumem.cu -- the C ABI of libgpumem.so (include/gpumem.h): handles, allocation,
+// streams, status codes, the overflow-and-retry protocol of find, and stage
+// instrumentation. All compute is in pack.cu / index.cu / radix.cu / find.cu /
+// sort.cu; this file only orchestrates launches.
+#include <atomic>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include "internal.h"
+
+#define GPUMEM_VERSION "0.1.0"
+
+enum : uint32_t { kMagicSeq = 0x47534551u, kMagicIdx = 0x47494458u, kMagicMems = 0x474d454du };
+
+struct gpumem_seq {
+    uint32_t magic;
+    int device;
+    cudaStream_t stream;
+    uint64_t n;
+    uint64_t n_words;
+    uint64_t *words;
+    unsigned long long *bad;  // first invalid position (ULLONG_MAX if none)
+};
+
+struct gpumem_index {
+    uint32_t magic;
+    int device;
+    cudaStream_t stream;
+    const gpumem_seq *R;
+    uint32_t ls, L, step;
+    uint64_t n_locs;
+    uint32_t *ptrs;
+    uint32_t *locs;
+    uint32_t *bitmap;
+};
+
+struct gpumem_mems {
+    uint32_t magic;
+    int device;
+    cudaStream_t stream;
+    uint64_t count;
+    gpumem_triple *dev;
+};
+
+namespace gm {
+
+Options g_opt;
+
+namespace {
+thread_local std::string t_err;
+std::atomic<uint64_t> g_launches{0};
+void *(*g_alloc_fn)(size_t, void *, void *) = nullptr;
+void (*g_free_fn)(void *, void *, void *) = nullptr;
+void *g_alloc_ctx = nullptr;
+std::mutex g_pool_mu;
+uint64_t g_pool_done = 0;  // bitmask of devices whose default pool was configured
+
+struct StageRec {
+    const char *name;
+    cudaEvent_t a, b;
+    uint64_t l0, l1;
+};
+std::mutex g_prof_mu;
+bool g_prof = false;
+std::vector<StageRec> g_recs;
+std::vector<cudaEvent_t> g_ev_free;
+
+cudaEvent_t take_event() {
+    if (!g_ev_free.empty()) {
+        cudaEvent_t e = g_ev_free.back();
+        g_ev_free.pop_back();
+        return e;
+    }
+    cudaEvent_t e = nullptr;
+    cudaEventCreate(&e);
+    return e;
+}
+
+int current_device() {
+    int d = -1;
+    if (cudaGetDevice(&d) != cudaSuccess) {
+        cudaGetLastError();
+        return -1;
+    }
+    return d;
+}
+}  // namespace
+
+gpumem_status fail(gpumem_status st, const char *fmt, ...) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    t_err = buf;
+    return st;
+}
+
+gpumem_status cuda_fail(cudaError_t e, const char *what) {
+    cudaGetLastError();  // clear sticky non-fatal state
+    return fail(GPUMEM_ERR_CUDA, "%s: %s (%s)", what, cudaGetErrorString(e), cudaGetErrorName(e));
+}
+
+void note_launch(int n) { g_launches.fetch_add(uint64_t(n), std::memory_order_relaxed); }
+
+int num_sms() {
+    static int cached[64] = {0};
+    const int d = current_device();
+    if (d < 0) return 148;
+    if (d < 64 && cached[d]) return cached[d];
+    int v = 0;
+    cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, d);
+    if (v <= 0) v = 148;
+    if (d < 64) cached[d] = v;
+    return v;
+}
+
+void *dalloc(size_t bytes, cudaStream_t s) {
+    if (bytes == 0) bytes = 256;
+    bytes = (bytes + 255) & ~size_t(255);
+    if (g_alloc_fn) {
+        void *p = g_alloc_fn(bytes, s, g_alloc_ctx);
+        if (!p) fail(GPUMEM_ERR_NOMEM, "allocator hook returned NULL for %zu bytes", bytes);
+        return p;
+    }
+    const int d = current_device();
+    if (d >= 0 && d < 64) {
+        std::lock_guard<std::mutex> g(g_pool_mu);
+        if (!(g_pool_done >> d & 1)) {  // keep freed memory cached in the pool
+            cudaMemPool_t pool;
+            if (cudaDeviceGetDefaultMemPool(&pool, d) == cudaSuccess) {
+                uint64_t thr = UINT64_MAX;
+                cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+            }
+            cudaGetLastError();
+            g_pool_done |= 1ull << d;
+        }
+    }
+    void *p = nullptr;
+    const cudaError_t e = cudaMallocAsync(&p, bytes, s);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        fail(GPUMEM_ERR_NOMEM, "cudaMallocAsync(%zu bytes): %s", bytes, cudaGetErrorString(e));
+        return nullptr;
+    }
+    return p;
+}
+
+void dfree(void *p, cudaStream_t s) {
+    if (!p) return;
+    if (g_free_fn) {
+        g_free_fn(p, s, g_alloc_ctx);
+        return;
+    }
+    cudaFreeAsync(p, s);
+}
+
+Stage::Stage(const char *name, cudaStream_t st) : slot(-1), s(st) {
+    if (!g_prof) return;
+    std::lock_guard<std::mutex> g(g_prof_mu);
+    StageRec r{name, take_event(), take_event(), g_launches.load(), 0};
+    cudaEventRecord(r.a, s);
+    g_recs.push_back(r);
+    slot = int(g_recs.size()) - 1;
+}
+
+Stage::~Stage() {
+    if (slot < 0) return;
+    std::lock_guard<std::mutex> g(g_prof_mu);
+    if (slot < int(g_recs.size())) {
+        cudaEventRecord(g_recs[slot].b, s);
+        g_recs[slot].l1 = g_launches.load();
+    }
+}
+
+}  // namespace gm
+
+using namespace gm;
+
+namespace {
+
+// RAII bundle of device allocations freed (async) on scope exit unless released.
+struct Scratch {
+    cudaStream_t s;
+    std::vector<void *> ptrs;
+    explicit Scratch(cudaStream_t st) : s(st) {}
+    void *get(size_t bytes) {
+        void *p = dalloc(bytes, s);
+        if (p) ptrs.push_back(p);
+        return p;
+    }
+    void keep(void *p) {
+        for (auto &q : ptrs)
+            if (q == p) q = nullptr;
+    }
+    ~Scratch() {
+        for (void *p : ptrs) dfree(p, s);
+    }
+};
+
+gpumem_status check_device(int *dev) {
+    int n = 0;
+    if (cudaGetDeviceCount(&n) != cudaSuccess || n == 0) {
+        cudaGetLastError();
+        return fail(GPUMEM_ERR_UNSUPPORTED, "no CUDA device visible");
+    }
+    int d = 0;
+    cudaGetDevice(&d);
+    int major = 0, minor = 0;
+    cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, d);
+    cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, d);
+    if (major != 10 || minor != 0)
+        return fail(GPUMEM_ERR_UNSUPPORTED, "libgpumem.so is built for sm_100a (B200); device %d is sm_%d%d", d,
+                    major, minor);
+    *dev = d;
+    return GPUMEM_OK;
+}
+
+#define CK(call, what)                                \
+    do {                                              \
+        const cudaError_t _e = (call);                \
+        if (_e != cudaSuccess) return cuda_fail(_e, what); \
+    } while (0)
+
+unsigned long long *pinned_slots() {  // 8 per thread, never freed
+    thread_local unsigned long long *p = nullptr;
+    if (!p) {
+        if (cudaMallocHost(&p, 8 * sizeof(unsigned long long)) != cudaSuccess) {
+            cudaGetLastError();
+            p = nullptr;
+        }
+    }
+    return p;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char *gpumem_version(void) { return GPUMEM_VERSION; }
+
+const char *gpumem_last_error(void) { return t_err.c_str(); }
+
+uint64_t gpumem_launch_count(void) { return g_launches.load(); }
+
+gpumem_status gpumem_set_allocator(void *(*alloc_fn)(size_t, void *, void *), void (*free_fn)(void *, void *, void *),
+                                   void *ctx) {
+    if ((alloc_fn == nullptr) != (free_fn == nullptr)) return fail(GPUMEM_ERR_ARG, "set both hooks or neither");
+    g_alloc_fn = alloc_fn;
+    g_free_fn = free_fn;
+    g_alloc_ctx = ctx;
+    return GPUMEM_OK;
+}
+
+gpumem_status gpumem_set_option(const char *name, int64_t value) {
+    if (!name) return fail(GPUMEM_ERR_ARG, "NULL option name");
+    if (!strcmp(name, "find_grid")) g_opt.find_grid = value < 0 ? 0 : value;
+    else if (!strcmp(name, "find_spill")) g_opt.find_spill = value < 1 ? 1 : value;
+    else if (!strcmp(name, "out_capacity")) g_opt.out_capacity = value < 0 ? 0 : value;
+    else if (!strcmp(name, "use_bitmap")) g_opt.use_bitmap = value ? 1 : 0;
+    else return fail(GPUMEM_ERR_ARG, "unknown option '%s'", name);
+    return GPUMEM_OK;
+}
+
+gpumem_status gpumem_profile_enable(int on) {
+    std::lock_guard<std::mutex> g(g_prof_mu);
+    g_prof = on != 0;
+    return GPUMEM_OK;
+}
+
+int gpumem_profile_read(const char **names, double *ms, uint64_t *launches, int max_stages) {
+    std::lock_guard<std::mutex> g(g_prof_mu);
+    int n = 0;
+    for (auto &r : g_recs) {
+        float t = 0.f;
+        cudaEventSynchronize(r.b);
+        cudaEventElapsedTime(&t, r.a, r.b);
+        int i = 0;
+        for (; i < n; ++i)
+            if (!strcmp(names[i], r.name)) break;
+        if (i == n) {
+            if (n >= max_stages) continue;
+            names[n] = r.name;
+            ms[n] = 0;
+            launches[n] = 0;
+            ++n;
+        }
+        ms[i] += t;
+        launches[i] += r.l1 - r.l0;
+        g_ev_free.push_back(r.a);
+        g_ev_free.push_back(r.b);
+    }
+    g_recs.clear();
+    cudaGetLastError();
+    return n;
+}
+
+void gpumem_free(void *handle) {
+    if (!handle) return;
+    const uint32_t magic = *static_cast<uint32_t *>(handle);
+    int prev = -1;
+    cudaGetDevice(&prev);
+    if (magic == kMagicSeq) {
+        auto *s = static_cast<gpumem_seq *>(handle);
+        cudaSetDevice(s->device);
+        dfree(s->words, s->stream);
+        dfree(s->bad, s->stream);
+        s->magic = 0;
+        delete s;
+    } else if (magic == kMagicIdx) {
+        auto *x = static_cast<gpumem_index *>(handle);
+        cudaSetDevice(x->device);
+        dfree(x->ptrs, x->stream);
+        dfree(x->locs, x->stream);
+        dfree(x->bitmap, x->stream);
+        x->magic = 0;
+        delete x;
+    } else if (magic == kMagicMems) {
+        auto *m = static_cast<gpumem_mems *>(handle);
+        cudaSetDevice(m->device);
+        dfree(m->dev, m->stream);
+        m->magic = 0;
+        delete m;
+    }
+    if (prev >= 0) cudaSetDevice(prev);
+    cudaGetLastError();
+}
+
+gpumem_status gpumem_pack(const char *bases, uint64_t n, int bases_on_device, void *cuda_stream,
+                          gpumem_seq **out) {
+    if (!out) return fail(GPUMEM_ERR_ARG, "out is NULL");
+    *out = nullptr;
+    if (!bases && n) return fail(GPUMEM_ERR_ARG, "bases is NULL");
+    if (n >= (1ull << 32)) return fail(GPUMEM_ERR_RANGE, "sequence of %llu bases exceeds 2^32-1 (32-bit locations)",
+                                       (unsigned long long)n);
+    int dev;
+    gpumem_status st = check_device(&dev);
+    if (st) return st;
+    cudaStream_t s = static_cast<cudaStream_t>(cuda_stream);
+    Stage stage("pack", s);
+    Scratch sc(s);
+    const uint64_t n_words = (n + 31) / 32 + 2;
+    auto *words = static_cast<uint64_t *>(sc.get(n_words * 8));
+    auto *bad = static_cast<unsigned long long *>(sc.get(8));
+    if (!words || !bad) return GPUMEM_ERR_NOMEM;
+    CK(cudaMemsetAsync(bad, 0xff, 8, s), "memset");
+    const uint8_t *in = reinterpret_cast<const uint8_t *>(bases);
+    if (!bases_on_device && n) {
+        auto *tmp = static_cast<uint8_t *>(sc.get(n));
+        if (!tmp) return GPUMEM_ERR_NOMEM;
+        CK(cudaMemcpyAsync(tmp, bases, n, cudaMemcpyHostToDevice, s), "H2D copy of bases");
+        in = tmp;
+    }
+    CK(launch_pack(in, n, words, n_words, bad, s), "pack kernel");
+    sc.keep(words);
+    sc.keep(bad);
+    auto *h = new gpumem_seq{kMagicSeq, dev, s, n, n_words, words, bad};
+    *out = h;
+    return GPUMEM_OK;
+}
+
+gpumem_status gpumem_seq_check(const gpumem_seq *sq, void *cuda_stream) {
+    if (!sq || sq->magic != kMagicSeq) return fail(GPUMEM_ERR_ARG, "not a gpumem_seq");
+    cudaStream_t s = static_cast<cudaStream_t>(cuda_stream);
+    unsigned long long *h = pinned_slots();
+    if (!h) return fail(GPUMEM_ERR_NOMEM, "pinned host buffer");
+    CK(cudaMemcpyAsync(h, sq->bad, 8, cudaMemcpyDeviceToHost, s), "D2H");
+    CK(cudaStreamSynchronize(s), "sync");
+    if (h[0] != ~0ull)
+        return fail(GPUMEM_ERR_ALPHABET, "byte at position %llu is not in {A,C,G,T,a,c,g,t}", h[0]);
+    return GPUMEM_OK;
+}
+
+gpumem_status gpumem_seq_info(const gpumem_seq *sq, uint64_t *n_bases, const uint64_t **dev_words,
+                              uint64_t *n_words) {
+    if (!sq || sq->magic != kMagicSeq) return fail(GPUMEM_ERR_ARG, "not a gpumem_seq");
+    if (n_bases) *n_bases = sq->n;
+    if (dev_words) *dev_words = sq->words;
+    if (n_words) *n_words = sq->n_words;
+    return GPUMEM_OK;
+}
+
+gpumem_status gpumem_index_build_step(const gpumem_seq *R, uint32_t ls, uint32_t L, uint32_t step,
+                                      void *cuda_stream, gpumem_index **out) {
+    if (!out) return fail(GPUMEM_ERR_ARG, "out is NULL");
+    *out = nullptr;
+    if (!R || R->magic != kMagicSeq) return fail(GPUMEM_ERR_ARG, "R is not a gpumem_seq");
+    if (ls < 1 || ls > 15) return fail(GPUMEM_ERR_ARG, "seed_len %u outside [1, 15]", ls);
+    if (L < ls) return fail(GPUMEM_ERR_ARG, "min_len %u < seed_len %u (Eq. 1 needs ls <= L)", L, ls);
+    if (step < 1 || step > L - ls + 1)
+        return fail(GPUMEM_ERR_ARG, "step %u outside [1, L - ls + 1 = %u] (Eq. 1)", step, L - ls + 1);
+    int dev;
+    gpumem_status st = check_device(&dev);
+    if (st) return st;
+    if (dev != R->device) return fail(GPUMEM_ERR_ARG, "R lives on device %d, current is %d", R->device, dev);
+    cudaStream_t s = static_cast<cudaStream_t>(cuda_stream);
+    const uint64_t nb = 1ull << (2 * ls);
+    const uint64_t n_locs = R->n >= ls ? (R->n - ls) / step + 1 : 0;
+    Scratch sc(s);
+    auto *ptrs = static_cast<uint32_t *>(sc.get((nb + 1) * 4));
+    auto *bitmap = static_cast<uint32_t *>(sc.get(((nb + 31) / 32) * 4));
+    auto *locs0 = static_cast<uint32_t *>(sc.get((n_locs ? n_locs : 1) * 4));
+    if (!ptrs || !bitmap || !locs0) return GPUMEM_ERR_NOMEM;
+    uint32_t *locs = locs0;
+    const uint32_t *codes_sorted = nullptr;
+    if (n_locs) {
+        auto *codes0 = static_cast<uint32_t *>(sc.get(n_locs * 4));
+        auto *codes1 = static_cast<uint32_t *>(sc.get(n_locs * 4));
+        auto *locs1 = static_cast<uint32_t *>(sc.get(n_locs * 4));
+        void *scratch = sc.get(radix_scratch_bytes(n_locs));
+        if (!codes0 || !codes1 || !locs1 || !scratch) return GPUMEM_ERR_NOMEM;
+        {
+            Stage g("index.codes", s);
+            CK(launch_seed_codes(R->words, R->n, ls, step, n_locs, codes0, locs0, s), "seed codes");
+        }
+        bool alt = false;
+        {
+            Stage g("index.sort", s);
+            CK(radix_sort_u32(codes0, locs0, codes1, locs1, n_locs, int(2 * ls), scratch, s, &alt),
+               "seed counting sort");
+        }
+        codes_sorted = alt ? codes1 : codes0;
+        locs = alt ? locs1 : locs0;
+    }
+    {
+        Stage g("index.ptrs", s);
+        CK(launch_ptrs_fill(codes_sorted, n_locs, ls, ptrs, bitmap, s), "ptrs fill");
+    }
+    sc.keep(ptrs);
+    sc.keep(bitmap);
+    sc.keep(locs);
+    auto *h = new gpumem_index{kMagicIdx, dev, s, R, ls, L, step, n_locs, ptrs, locs, bitmap};
+    *out = h;
+    return GPUMEM_OK;
+}
+
+gpumem_status gpumem_index_build(const gpumem_seq *R, uint32_t ls, uint32_t L, void *cuda_stream,
+                                 gpumem_index **out) {
+    if (out) *out = nullptr;
+    if (ls < 1 || ls > 15 || L < ls) {
+        if (!out) return fail(GPUMEM_ERR_ARG, "out is NULL");
+        return fail(GPUMEM_ERR_ARG, "need 1 <= seed_len <= 15 and seed_len <= min_len (got %u, %u)", ls, L);
+    }
+    return gpumem_index_build_step(R, ls, L, L - ls + 1, cuda_stream, out);
+}
+
+gpumem_status gpumem_index_view(const gpumem_index *idx, const uint32_t **dev_ptrs, const uint32_t **dev_locs,
+                                uint64_t *n_locs) {
+    if (!idx || idx->magic != kMagicIdx) return fail(GPUMEM_ERR_ARG, "not a gpumem_index");
+    if (dev_ptrs) *dev_ptrs = idx->ptrs;
+    if (dev_locs) *dev_locs = idx->locs;
+    if (n_locs) *n_locs = idx->n_locs;
+    return GPUMEM_OK;
+}
+
+static gpumem_status sort_into_triples(uint64_t *keys, uint32_t *lens, uint64_t n, uint32_t key_bits,
+                                       uint32_t qbits, int dev, cudaStream_t s, gpumem_mems **out) {
+    Scratch sc(s);
+    auto *trip = static_cast<gpumem_triple *>(sc.get((n ? n : 1) * sizeof(gpumem_triple)));
+    if (!trip) return GPUMEM_ERR_NOMEM;
+    if (n) {
+        Stage g("sort", s);
+        auto *k1 = static_cast<uint64_t *>(sc.get(n * 8));
+        auto *l1 = static_cast<uint32_t *>(sc.get(n * 4));
+        void *scratch = sc.get(radix_scratch_bytes(n));
+        if (!k1 || !l1 || !scratch) return GPUMEM_ERR_NOMEM;
+        bool alt = false;
+        CK(radix_sort_u64(keys, lens, k1, l1, n, int(key_bits), scratch, s, &alt), "triple sort");
+        CK(launch_keys_to_triples(alt ? k1 : keys, alt ? l1 : lens, n, qbits, trip, s), "keys to triples");
+    }
+    sc.keep(trip);
+    *out = new gpumem_mems{kMagicMems, dev, s, n, trip};
+    return GPUMEM_OK;
+}
+
+gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uint64_t q_begin, uint64_t q_end,
+                               void *cuda_stream, gpumem_mems **out) {
+    if (!out) return fail(GPUMEM_ERR_ARG, "out is NULL");
+    *out = nullptr;
+    if (!idx || idx->magic != kMagicIdx) return fail(GPUMEM_ERR_ARG, "idx is not a gpumem_index");
+    if (!Q || Q->magic != kMagicSeq) return fail(GPUMEM_ERR_ARG, "Q is not a gpumem_seq");
+    const gpumem_seq *R = idx->R;
+    if (!R || R->magic != kMagicSeq) return fail(GPUMEM_ERR_ARG, "the index's R was freed");
+    int dev;
+    gpumem_status st = check_device(&dev);
+    if (st) return st;
+    if (Q->device != dev || idx->device != dev) return fail(GPUMEM_ERR_ARG, "handles on another device");
+    const uint64_t nQ = Q->n, nR = R->n;
+    if (q_end > nQ) q_end = nQ;
+    if (q_begin > nQ) return fail(GPUMEM_ERR_RANGE, "q_begin %llu > |Q| = %llu", (unsigned long long)q_begin,
+                                  (unsigned long long)nQ);
+    if (q_begin > q_end) q_end = q_begin;
+    cudaStream_t s = static_cast<cudaStream_t>(cuda_stream);
+    const uint32_t ls = idx->ls, L = idx->L, step = idx->step;
+
+    FindParams P{};
+    P.R = R->words;
+    P.nR = nR;
+    P.Q = Q->words;
+    P.nQ = nQ;
+    P.ptrs = idx->ptrs;
+    P.locs = idx->locs;
+    P.bitmap = idx->bitmap;
+    P.ls = ls;
+    P.L = L;
+    P.step = step;
+    P.qbits = bits_for(nQ);
+    P.own_lo = q_begin;
+    P.own_hi = q_end;
+    P.scan_lo = q_begin;
+    P.scan_hi = q_begin;
+    if (nQ >= ls && nR >= ls && nQ >= L && nR >= L && q_begin < q_end) {
+        const uint64_t hi = q_end + step - 1;  // the canonical seed lies < step right of the MEM start
+        P.scan_hi = hi < nQ - ls + 1 ? hi : nQ - ls + 1;
+        if (P.scan_hi < P.scan_lo) P.scan_hi = P.scan_lo;
+    }
+    const uint64_t span = P.scan_hi - P.scan_lo;
+    const uint64_t tile = find_tile_positions();
+    P.n_tiles = (span + tile - 1) / tile;
+    P.spill_t = uint32_t(g_opt.find_spill);
+    P.use_bitmap = int(g_opt.use_bitmap);
+    uint64_t cap = g_opt.out_capacity ? uint64_t(g_opt.out_capacity) : (span / 8 + 4096);
+
+    Scratch sc(s);
+    auto *ctr = static_cast<unsigned long long *>(sc.get(64));
+    const uint64_t spill_cap = span / 64 + 4096;
+    auto *spill = static_cast<uint4 *>(sc.get(spill_cap * sizeof(uint4)));
+    if (!ctr || !spill) return GPUMEM_ERR_NOMEM;
+    P.out_count = ctr;
+    P.spill_count = ctr + 1;
+    P.tile_ctr = reinterpret_cast<unsigned int *>(ctr + 2);
+    P.spill = spill;
+    P.spill_cap = spill_cap;
+    unsigned long long *h = pinned_slots();
+    if (!h) return fail(GPUMEM_ERR_NOMEM, "pinned host buffer");
+
+    uint64_t count = 0;
+    uint64_t *keys = nullptr;
+    uint32_t *lens = nullptr;
+    for (int attempt = 0; attempt < 2; ++attempt) {
+        keys = static_cast<uint64_t *>(sc.get(cap * 8));
+        lens = static_cast<uint32_t *>(sc.get(cap * 4));
+        if (!keys || !lens) return GPUMEM_ERR_NOMEM;
+        P.out_key = keys;
+        P.out_len = lens;
+        P.capacity = cap;
+        CK(cudaMemsetAsync(ctr, 0, 64, s), "memset counters");
+        {
+            Stage g("find", s);
+            CK(launch_find(P, int(g_opt.find_grid), s), "find kernel");
+        }
+        if (P.n_tiles) {
+            Stage g("find.heavy", s);
+            CK(launch_heavy(P, s), "heavy kernel");
+        }
+        CK(cudaMemcpyAsync(h, ctr, 16, cudaMemcpyDeviceToHost, s), "D2H count");
+        CK(cudaMemcpyAsync(h + 2, R->bad, 8, cudaMemcpyDeviceToHost, s), "D2H flag");
+        CK(cudaMemcpyAsync(h + 3, Q->bad, 8, cudaMemcpyDeviceToHost, s), "D2H flag");
+        CK(cudaStreamSynchronize(s), "find sync");
+        if (h[2] != ~0ull) return fail(GPUMEM_ERR_ALPHABET, "R: byte at position %llu is not in {A,C,G,T,a,c,g,t}", h[2]);
+        if (h[3] != ~0ull) return fail(GPUMEM_ERR_ALPHABET, "Q: byte at position %llu is not in {A,C,G,T,a,c,g,t}", h[3]);
+        count = h[0];
+        if (count <= cap) break;
+        if (attempt == 1) return fail(GPUMEM_ERR_CUDA, "output count changed between runs (%llu > %llu)",
+                                      (unsigned long long)count, (unsigned long long)cap);
+        cap = count;  // overflow: rerun with the exact capacity
+    }
+    const uint32_t key_bits = bits_for(nR) + P.qbits;
+    return sort_into_triples(keys, lens, count, key_bits, P.qbits, dev, s, out);
+}
+
+gpumem_status gpumem_mems_view(const gpumem_mems *m, const gpumem_triple **dev_ptr, uint64_t *count) {
+    if (!m || m->magic != kMagicMems) return fail(GPUMEM_ERR_ARG, "not a gpumem_mems");
+    if (dev_ptr) *dev_ptr = m->dev;
+    if (count) *count = m->count;
+    return GPUMEM_OK;
+}
+
+gpumem_status gpumem_mems_to_host(const gpumem_mems *m, gpumem_triple *host_buf, uint64_t capacity) {
+    if (!m || m->magic != kMagicMems) return fail(GPUMEM_ERR_ARG, "not a gpumem_mems");
+    if (capacity < m->count) return fail(GPUMEM_ERR_RANGE, "host buffer holds %llu < %llu triples",
+                                         (unsigned long long)capacity, (unsigned long long)m->count);
+    if (!m->count) return GPUMEM_OK;
+    if (!host_buf) return fail(GPUMEM_ERR_ARG, "host_buf is NULL");
+    CK(cudaMemcpyAsync(host_buf, m->dev, m->count * sizeof(gpumem_triple), cudaMemcpyDeviceToHost, m->stream),
+       "D2H triples");
+    CK(cudaStreamSynchronize(m->stream), "sync");
+    return GPUMEM_OK;
+}
+
+gpumem_status gpumem_merge_sorted(const gpumem_triple *const *dev_runs, const uint64_t *counts, int n_runs,
+                                  void *cuda_stream, gpumem_mems **out) {
+    if (!out) return fail(GPUMEM_ERR_ARG, "out is NULL");
+    *out = nullptr;
+    if (n_runs < 0 || (n_runs > 0 && (!dev_runs || !counts))) return fail(GPUMEM_ERR_ARG, "bad runs");
+    int dev;
+    gpumem_status st = check_device(&dev);
+    if (st) return st;
+    cudaStream_t s = static_cast<cudaStream_t>(cuda_stream);
+    uint64_t total = 0;
+    for (int i = 0; i < n_runs; ++i) total += counts[i];
+    Scratch sc(s);
+    auto *keys = static_cast<uint64_t *>(sc.get((total ? total : 1) * 8));
+    auto *lens = static_cast<uint32_t *>(sc.get((total ? total : 1) * 4));
+    if (!keys || !lens) return GPUMEM_ERR_NOMEM;
+    {
+        Stage g("merge", s);
+        uint64_t off = 0;
+        for (int i = 0; i < n_runs; ++i) {
+            if (counts[i] && !dev_runs[i]) return fail(GPUMEM_ERR_ARG, "run %d is NULL", i);
+            CK(launch_triples_to_keys(dev_runs[i], counts[i], 32, keys + off, lens + off, s), "merge keys");
+            off += counts[i];
+        }
+    }
+    return sort_into_triples(keys, lens, total, 64, 32, dev, s, out);
+}
+
+}  // extern "C"

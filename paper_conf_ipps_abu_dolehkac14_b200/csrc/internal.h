@@ -1,0 +1,97 @@
+// internal.h -- host-side declarations shared by the .cu files of libgpumem.so.
+// Not part of the ABI (see include/gpumem.h). No torch types anywhere.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "gpumem.h"
+
+namespace gm {
+
+// ---------------------------------------------------------------- runtime
+struct Options {
+    int64_t find_grid = 0;       // 0 = SMs x occupancy
+    int64_t find_spill = 128;    // bucket sizes above this go to the heavy queue
+    int64_t out_capacity = 0;    // 0 = automatic
+    int64_t use_bitmap = 1;      // probe the occupancy bitmap before ptrs
+};
+extern Options g_opt;
+
+void *dalloc(size_t bytes, cudaStream_t s);   // nullptr on failure (error text set)
+void dfree(void *p, cudaStream_t s);
+void note_launch(int n = 1);                  // launch counter
+int num_sms();
+
+gpumem_status fail(gpumem_status st, const char *fmt, ...);
+gpumem_status cuda_fail(cudaError_t e, const char *what);
+
+// Brackets one stage with CUDA events when profiling is enabled.
+struct Stage {
+    Stage(const char *name, cudaStream_t s);
+    ~Stage();
+    int slot;
+    cudaStream_t s;
+};
+
+// ---------------------------------------------------------------- kernels (launchers)
+// K1: ASCII -> 2-bit words (pack.cu). words must hold ceil(n/32) + 2 entries.
+cudaError_t launch_pack(const uint8_t *in, uint64_t n, uint64_t *words, uint64_t n_words_alloc,
+                        unsigned long long *bad_pos, cudaStream_t s);
+
+// Radix sort (radix.cu): stable LSD on the low `bits` bits of the keys, values ride along.
+// Ping-pongs between (k0,v0) and (k1,v1); returns true when the result is in (k1,v1).
+// `scratch` must hold radix_scratch_bytes(n) bytes (digit counts + scan partials).
+cudaError_t radix_sort_u32(uint32_t *k0, uint32_t *v0, uint32_t *k1, uint32_t *v1, uint64_t n, int bits,
+                           void *scratch, cudaStream_t s, bool *in_alt);
+cudaError_t radix_sort_u64(uint64_t *k0, uint32_t *v0, uint64_t *k1, uint32_t *v1, uint64_t n, int bits,
+                           void *scratch, cudaStream_t s, bool *in_alt);
+size_t radix_scratch_bytes(uint64_t n);
+
+// Index (index.cu)
+cudaError_t launch_seed_codes(const uint64_t *R, uint64_t nR, uint32_t ls, uint32_t step, uint64_t n_locs,
+                              uint32_t *codes, uint32_t *locs, cudaStream_t s);
+cudaError_t launch_ptrs_fill(const uint32_t *sorted_codes, uint64_t n_locs, uint32_t ls, uint32_t *ptrs,
+                             uint32_t *bitmap, cudaStream_t s);
+
+// Find (find.cu)
+struct FindParams {
+    const uint64_t *R;
+    uint64_t nR;
+    const uint64_t *Q;
+    uint64_t nQ;
+    const uint32_t *ptrs;
+    const uint32_t *locs;
+    const uint32_t *bitmap;
+    uint32_t ls, L, step, qbits;
+    uint64_t scan_lo, scan_hi;   // query seed positions scanned
+    uint64_t own_lo, own_hi;     // MEM start q kept
+    uint64_t *out_key;           // (r << qbits) | q
+    uint32_t *out_len;
+    uint64_t capacity;
+    unsigned long long *out_count;
+    unsigned int *tile_ctr;
+    uint64_t n_tiles;
+    uint32_t spill_t;
+    uint4 *spill;                // {q, beg, len, 0}
+    uint64_t spill_cap;
+    unsigned long long *spill_count;
+    int use_bitmap;
+};
+uint64_t find_tile_positions();
+cudaError_t launch_find(const FindParams &p, int grid, cudaStream_t s);
+cudaError_t launch_heavy(const FindParams &p, cudaStream_t s);
+int find_default_grid();
+
+// Triples (sort.cu)
+cudaError_t launch_keys_to_triples(const uint64_t *keys, const uint32_t *lens, uint64_t n, uint32_t qbits,
+                                   gpumem_triple *out, cudaStream_t s);
+cudaError_t launch_triples_to_keys(const gpumem_triple *in, uint64_t n, uint32_t qbits, uint64_t *keys,
+                                   uint32_t *lens, cudaStream_t s);
+
+inline uint32_t bits_for(uint64_t n) {  // bits needed to hold values in [0, n)
+    uint32_t b = 0;
+    while (b < 64 && (n >> b) > 0) ++b;
+    return b ? b : 1;
+}
+
+}  // namespace gm

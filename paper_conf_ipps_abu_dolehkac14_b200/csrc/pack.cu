@@ -1,0 +1,79 @@
+// pack.cu -- K1: ASCII -> 2-bit packed words.
+//
+// One thread per output word = 32 input bytes, read as two 128-bit vector loads
+// when the input is 16-byte aligned (scalar bytes otherwise and for the tail).
+// Per 4 bytes (SWAR): code = ((c>>1) ^ (c>>2)) & 3 maps A/a->0 C/c->1 G/g->2
+// T/t->3; validity is checked exactly by rebuilding the expected upper-case
+// byte from the code with one PRMT and comparing. The first invalid position
+// is recorded with atomicMin (alphabet error, reading R4).
+// Algorithmic bytes: 1 B read + 0.25 B written per base (HBM-bound).
+#include "internal.h"
+
+namespace gm {
+namespace {
+
+constexpr int kPackThreads = 256;
+
+// 4 ASCII bytes -> 8 bits of codes (first byte most significant), valid flag.
+__device__ __forceinline__ uint32_t pack4(uint32_t x, bool &ok) {
+    const uint32_t c = ((x >> 1) ^ (x >> 2)) & 0x03030303u;          // per-byte code
+    const uint32_t y = c | (c >> 4);
+    const uint32_t sel = (y & 0xFFu) | ((y >> 8) & 0xFF00u);         // codes -> PRMT nibbles
+    const uint32_t expect = __byte_perm(0x54474341u, 0u, sel);       // 'T''G''C''A'
+    ok = ok && (expect == (x & 0xDFDFDFDFu));                        // exact, upper-cased
+    return (c * 0x40100401u) >> 24;                                  // c0<<6|c1<<4|c2<<2|c3
+}
+
+__global__ void __launch_bounds__(kPackThreads) k_pack(const uint8_t *__restrict__ in, uint64_t n,
+                                                       uint64_t *__restrict__ words, uint64_t n_full,
+                                                       uint64_t n_words_alloc, unsigned long long *bad_pos,
+                                                       int aligned) {
+    const uint64_t w = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+    if (w >= n_words_alloc) return;
+    uint64_t word = 0;
+    bool ok = true;
+    if (w < n_full && aligned) {
+        const uint4 a = __ldcs(reinterpret_cast<const uint4 *>(in) + 2 * w);      // streamed once
+        const uint4 b = __ldcs(reinterpret_cast<const uint4 *>(in) + 2 * w + 1);
+        const uint32_t v[8] = {a.x, a.y, a.z, a.w, b.x, b.y, b.z, b.w};
+#pragma unroll
+        for (int j = 0; j < 8; ++j) word |= uint64_t(pack4(v[j], ok)) << (56 - 8 * j);
+    } else {
+        const uint64_t base = w * 32;
+        for (int i = 0; i < 32; ++i) {
+            const uint64_t pos = base + i;
+            if (pos >= n) break;  // padding bases stay 00
+            const uint32_t ch = in[pos];
+            const uint32_t c = ((ch >> 1) ^ (ch >> 2)) & 3u;
+            const uint32_t up = ch & 0xDFu;
+            if (up != 'A' && up != 'C' && up != 'G' && up != 'T') {
+                atomicMin(bad_pos, (unsigned long long)pos);
+            }
+            word |= uint64_t(c) << (62 - 2 * i);
+        }
+    }
+    if (!ok) {  // locate the first bad byte of this word
+        for (int i = 0; i < 32; ++i) {
+            const uint32_t up = in[w * 32 + i] & 0xDFu;
+            if (up != 'A' && up != 'C' && up != 'G' && up != 'T') {
+                atomicMin(bad_pos, (unsigned long long)(w * 32 + i));
+                break;
+            }
+        }
+    }
+    words[w] = word;
+}
+
+}  // namespace
+
+cudaError_t launch_pack(const uint8_t *in, uint64_t n, uint64_t *words, uint64_t n_words_alloc,
+                        unsigned long long *bad_pos, cudaStream_t s) {
+    const int aligned = (reinterpret_cast<uintptr_t>(in) & 15) == 0;
+    const uint64_t n_full = n / 32;
+    const uint64_t blocks = (n_words_alloc + kPackThreads - 1) / kPackThreads;
+    k_pack<<<unsigned(blocks), kPackThreads, 0, s>>>(in, n, words, n_full, n_words_alloc, bad_pos, aligned);
+    note_launch();
+    return cudaGetLastError();
+}
+
+}  // namespace gm

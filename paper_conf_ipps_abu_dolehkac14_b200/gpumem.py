@@ -1,0 +1,266 @@
+"""Thin Python binding over libgpumem.so (C ABI: include/gpumem.h).
+
+Argument marshalling only: every step of the MEM path runs in the library's
+CUDA kernels. PyTorch is used for device buffers and the current CUDA stream.
+Importing this module fails loudly if the CUDA library has not been built --
+there is no CPU fallback.
+
+    import paper_conf_ipps_abu_dolehkac14_b200.gpumem as gm
+    R = gm.pack(r_bytes)                     # bytes/numpy (host) or uint8 CUDA tensor
+    Q = gm.pack(q_bytes)
+    idx = gm.index_build(R, seed_len=13, min_len=100)
+    mems = gm.find_mems(idx, Q)              # sorted by (r, q)
+    mems.numpy()                             # (N, 3) uint32 [r, q, len] on the host
+    mems.tensor()                            # (N, 3) int64 CUDA tensor (copy)
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "libgpumem.so")
+if not os.path.exists(LIB_PATH):
+    raise ImportError(f"{LIB_PATH} is missing: build it with `python -m paper_conf_ipps_abu_dolehkac14_b200._build` "
+                      "(the MEM path is CUDA-only; there is no CPU fallback)")
+_lib = ctypes.CDLL(LIB_PATH)
+
+_c_u64, _c_u32, _vp = ctypes.c_uint64, ctypes.c_uint32, ctypes.c_void_p
+_P = ctypes.POINTER
+
+SYMBOLS = {
+    # name: (restype, argtypes)
+    "gpumem_pack": (ctypes.c_int, [ctypes.c_void_p, _c_u64, ctypes.c_int, _vp, _P(_vp)]),
+    "gpumem_seq_check": (ctypes.c_int, [_vp, _vp]),
+    "gpumem_seq_info": (ctypes.c_int, [_vp, _P(_c_u64), _P(_vp), _P(_c_u64)]),
+    "gpumem_index_build": (ctypes.c_int, [_vp, _c_u32, _c_u32, _vp, _P(_vp)]),
+    "gpumem_index_build_step": (ctypes.c_int, [_vp, _c_u32, _c_u32, _c_u32, _vp, _P(_vp)]),
+    "gpumem_index_view": (ctypes.c_int, [_vp, _P(_vp), _P(_vp), _P(_c_u64)]),
+    "gpumem_find_mems": (ctypes.c_int, [_vp, _vp, _c_u64, _c_u64, _vp, _P(_vp)]),
+    "gpumem_mems_view": (ctypes.c_int, [_vp, _P(_vp), _P(_c_u64)]),
+    "gpumem_mems_to_host": (ctypes.c_int, [_vp, _vp, _c_u64]),
+    "gpumem_merge_sorted": (ctypes.c_int, [_P(_vp), _P(_c_u64), ctypes.c_int, _vp, _P(_vp)]),
+    "gpumem_free": (None, [_vp]),
+    "gpumem_last_error": (ctypes.c_char_p, []),
+    "gpumem_set_allocator": (ctypes.c_int, [_vp, _vp, _vp]),
+    "gpumem_set_option": (ctypes.c_int, [ctypes.c_char_p, ctypes.c_int64]),
+    "gpumem_profile_enable": (ctypes.c_int, [ctypes.c_int]),
+    "gpumem_profile_read": (ctypes.c_int, [_P(ctypes.c_char_p), _P(ctypes.c_double), _P(_c_u64), ctypes.c_int]),
+    "gpumem_launch_count": (_c_u64, []),
+    "gpumem_version": (ctypes.c_char_p, []),
+}
+for _name, (_res, _args) in SYMBOLS.items():
+    _f = getattr(_lib, _name)
+    _f.restype = _res
+    _f.argtypes = _args
+
+STATUS = {0: "OK", 1: "ERR_ARG", 2: "ERR_ALPHABET", 3: "ERR_RANGE", 4: "ERR_NOMEM", 5: "ERR_CUDA",
+          6: "ERR_UNSUPPORTED"}
+
+
+class GpumemError(RuntimeError):
+    def __init__(self, status, message):
+        super().__init__(f"{STATUS.get(status, status)}: {message}")
+        self.status = status
+        self.name = STATUS.get(status, str(status))
+
+
+def _check(st):
+    if st != 0:
+        raise GpumemError(st, (_lib.gpumem_last_error() or b"").decode())
+
+
+def _stream(stream=None):
+    if stream is not None:
+        return ctypes.c_void_p(int(stream))
+    import torch
+    return ctypes.c_void_p(torch.cuda.current_stream().cuda_stream)
+
+
+class _Handle:
+    __slots__ = ("_h", "_keep", "__weakref__")
+
+    def __init__(self, h, keep=None):
+        self._h = h
+        self._keep = keep
+
+    @property
+    def handle(self):
+        if not self._h:
+            raise GpumemError(1, "handle already freed")
+        return self._h
+
+    def free(self):
+        if self._h:
+            _lib.gpumem_free(self._h)
+            self._h = None
+        self._keep = None
+
+    def __del__(self):
+        try:
+            self.free()
+        except Exception:
+            pass
+
+
+class Seq(_Handle):
+    """A 2-bit packed sequence on the current device."""
+
+    def info(self):
+        n, w, nw = _c_u64(), _vp(), _c_u64()
+        _check(_lib.gpumem_seq_info(self.handle, ctypes.byref(n), ctypes.byref(w), ctypes.byref(nw)))
+        return n.value, w.value, nw.value
+
+    def __len__(self):
+        return self.info()[0]
+
+    def check(self, stream=None):
+        _check(_lib.gpumem_seq_check(self.handle, _stream(stream)))
+
+    def words(self):
+        """Packed words as a uint64 CUDA tensor view (borrowed from the handle)."""
+        n, ptr, nw = self.info()
+        return _device_view(ptr, (nw,), "<u8", self)
+
+
+class Index(_Handle):
+    def view(self):
+        """(ptrs, locs) as uint32 CUDA tensor views (borrowed)."""
+        p, l, n = _vp(), _vp(), _c_u64()
+        _check(_lib.gpumem_index_view(self.handle, ctypes.byref(p), ctypes.byref(l), ctypes.byref(n)))
+        ls = self._keep[1]
+        return (_device_view(p.value, ((1 << (2 * ls)) + 1,), "<u4", self),
+                _device_view(l.value, (n.value,), "<u4", self))
+
+
+class Mems(_Handle):
+    def view(self):
+        ptr, cnt = _vp(), _c_u64()
+        _check(_lib.gpumem_mems_view(self.handle, ctypes.byref(ptr), ctypes.byref(cnt)))
+        return ptr.value, cnt.value
+
+    def __len__(self):
+        return self.view()[1]
+
+    def numpy(self):
+        """(N, 3) uint32 [r, q, len] copied to the host (synchronous)."""
+        _, n = self.view()
+        out = np.empty((n, 3), dtype=np.uint32)
+        _check(_lib.gpumem_mems_to_host(self.handle, out.ctypes.data_as(_vp), n))
+        return out
+
+    def view_u32(self):
+        """(N, 3) uint32 CUDA tensor view (borrowed from the handle)."""
+        ptr, n = self.view()
+        return _device_view(ptr, (n, 3), "<u4", self)
+
+    def tensor(self):
+        """(N, 3) int64 CUDA tensor (copy)."""
+        return self.view_u32().to(dtype=__import__("torch").int64)
+
+
+class _CudaArray:
+    def __init__(self, ptr, shape, typestr, owner):
+        self.__cuda_array_interface__ = {"shape": shape, "typestr": typestr, "data": (ptr or 0, False),
+                                         "version": 3, "strides": None, "stream": None}
+        self._owner = owner
+
+
+def _device_view(ptr, shape, typestr, owner):
+    import torch
+    if int(np.prod(shape)) == 0:
+        dt = {"<u4": torch.uint32, "<u8": torch.uint64}[typestr]
+        return torch.empty(shape, dtype=dt, device="cuda")
+    return torch.as_tensor(_CudaArray(ptr, shape, typestr, owner), device="cuda")
+
+
+def pack(x, stream=None) -> Seq:
+    """2-bit encode `x`: a uint8 CUDA tensor (read in place), or host bytes/str/numpy/CPU tensor."""
+    h = _vp()
+    keep = None
+    try:
+        import torch
+        is_tensor = isinstance(x, torch.Tensor)
+    except ImportError:  # pragma: no cover
+        is_tensor = False
+    if is_tensor and x.is_cuda:
+        if x.dtype != __import__("torch").uint8:
+            raise TypeError("device input must be a uint8 tensor")
+        x = x.contiguous()
+        keep = x
+        _check(_lib.gpumem_pack(_vp(x.data_ptr()), x.numel(), 1, _stream(stream), ctypes.byref(h)))
+    else:
+        if is_tensor:
+            arr = x.contiguous().numpy()
+        elif isinstance(x, str):
+            arr = np.frombuffer(x.encode("ascii"), dtype=np.uint8)
+        elif isinstance(x, (bytes, bytearray, memoryview)):
+            arr = np.frombuffer(bytes(x), dtype=np.uint8)
+        else:
+            arr = np.ascontiguousarray(x, dtype=np.uint8)
+        keep = arr
+        _check(_lib.gpumem_pack(arr.ctypes.data_as(_vp), arr.size, 0, _stream(stream), ctypes.byref(h)))
+    return Seq(h.value, keep)
+
+
+def index_build(R: Seq, seed_len: int, min_len: int, step: int | None = None, stream=None) -> Index:
+    h = _vp()
+    if step is None:
+        _check(_lib.gpumem_index_build(R.handle, seed_len, min_len, _stream(stream), ctypes.byref(h)))
+    else:
+        _check(_lib.gpumem_index_build_step(R.handle, seed_len, min_len, step, _stream(stream), ctypes.byref(h)))
+    return Index(h.value, (R, seed_len))
+
+
+def find_mems(idx: Index, Q: Seq, q_range=None, stream=None) -> Mems:
+    qb, qe = (0, (1 << 64) - 1) if q_range is None else (int(q_range[0]), int(q_range[1]))
+    h = _vp()
+    _check(_lib.gpumem_find_mems(idx.handle, Q.handle, qb, qe, _stream(stream), ctypes.byref(h)))
+    return Mems(h.value, (idx, Q))
+
+
+def merge_sorted(runs, stream=None) -> Mems:
+    """Merge device runs of triples, each sorted by (r, q). `runs`: list of (N_i, 3) uint32/int32 CUDA tensors."""
+    ptrs = (_vp * max(1, len(runs)))(*[_vp(r.data_ptr()) for r in runs])
+    cnts = (_c_u64 * max(1, len(runs)))(*[r.shape[0] for r in runs])
+    h = _vp()
+    _check(_lib.gpumem_merge_sorted(ptrs, cnts, len(runs), _stream(stream), ctypes.byref(h)))
+    return Mems(h.value, list(runs))
+
+
+def set_option(name: str, value: int):
+    _check(_lib.gpumem_set_option(name.encode(), int(value)))
+
+
+def profile_enable(on=True):
+    _check(_lib.gpumem_profile_enable(1 if on else 0))
+
+
+def profile_read(max_stages=32):
+    names = (ctypes.c_char_p * max_stages)()
+    ms = (ctypes.c_double * max_stages)()
+    nl = (_c_u64 * max_stages)()
+    n = _lib.gpumem_profile_read(names, ms, nl, max_stages)
+    return {names[i].decode(): (ms[i], nl[i]) for i in range(n)}
+
+
+def launch_count() -> int:
+    return int(_lib.gpumem_launch_count())
+
+
+def version() -> str:
+    return _lib.gpumem_version().decode()
+
+
+def mems(R_bytes, Q_bytes, min_len, seed_len, q_range=None, stream=None):
+    """Convenience: pack + index + find; returns the host (N, 3) uint32 array."""
+    R = pack(R_bytes, stream)
+    Q = pack(Q_bytes, stream)
+    idx = index_build(R, seed_len, min_len, stream=stream)
+    m = find_mems(idx, Q, q_range, stream=stream)
+    out = m.numpy()
+    for h in (m, idx, Q, R):
+        h.free()
+    return out

@@ -1,0 +1,277 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle, element
+by element, on seeded inputs. Bit-exact: MEMs are integer triples (r, q, len)
+and the set is unique (reading R20), sorted by (r, q)."""
+import numpy as np
+import pytest
+
+import oracle
+from oracle import pyoracle
+from paper_conf_ipps_abu_dolehkac14_b200 import synth
+from tests import invariants
+from tests.conftest import read_golden
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+if not torch.cuda.is_available():  # collected on CPU boxes, skipped there
+    pytest.skip("needs a CUDA device", allow_module_level=True)
+
+from paper_conf_ipps_abu_dolehkac14_b200 import gpumem  # noqa: E402
+
+
+@pytest.fixture(autouse=True)
+def _default_options():
+    yield
+    for k, v in (("find_grid", 0), ("find_spill", 128), ("out_capacity", 0), ("use_bitmap", 1)):
+        gpumem.set_option(k, v)
+
+
+def gpu_mems(R, Q, L, ls, step=None, q_range=None, device_input=False):
+    if device_input:
+        Rt = torch.from_numpy(np.frombuffer(bytes(R), dtype=np.uint8).copy()).cuda()
+        Qt = torch.from_numpy(np.frombuffer(bytes(Q), dtype=np.uint8).copy()).cuda()
+        Rs, Qs = gpumem.pack(Rt), gpumem.pack(Qt)
+    else:
+        Rs, Qs = gpumem.pack(R), gpumem.pack(Q)
+    idx = gpumem.index_build(Rs, ls, L, step)
+    m = gpumem.find_mems(idx, Qs, q_range)
+    out = m.numpy()
+    torch.cuda.synchronize()
+    return out
+
+
+def _b(x):
+    return x.tobytes() if isinstance(x, np.ndarray) else (x.encode() if isinstance(x, str) else bytes(x))
+
+
+# ------------------------------------------------------------------ K1 pack
+def _decode(words, n):
+    w = words.astype(np.uint64)
+    i = np.arange(n, dtype=np.uint64)
+    c = (w[i // 32] >> (np.uint64(62) - np.uint64(2) * (i % np.uint64(32)))) & np.uint64(3)
+    return np.frombuffer(b"ACGT", dtype=np.uint8)[c.astype(np.int64)]
+
+
+def test_pack_known_word():
+    s = gpumem.pack(b"ACGT" * 8)
+    w = s.words().cpu().numpy()
+    assert int(w[0]) == 0x1B1B1B1B1B1B1B1B
+    assert int(w[1]) == 0 and int(w[2]) == 0  # padding
+
+
+@pytest.mark.parametrize("n", [0, 1, 31, 32, 33, 1000, 4097, 100_003])
+@pytest.mark.parametrize("offset", [0, 1, 7, 16])
+def test_pack_roundtrip_device_and_host(n, offset):
+    rng = np.random.default_rng(n + offset)
+    raw = np.frombuffer(b"ACGTacgt", dtype=np.uint8)[rng.integers(0, 8, n + offset)]
+    dev = torch.from_numpy(raw.copy()).cuda()[offset:]
+    for s in (gpumem.pack(dev), gpumem.pack(raw[offset:].tobytes())):
+        s.check()
+        nn, _, nw = s.info()
+        assert nn == n and nw == (n + 31) // 32 + 2
+        w = s.words().cpu().numpy()
+        up = raw[offset:] & 0xDF
+        assert np.array_equal(_decode(w, n), up)
+        if n % 32:
+            last = int(w[n // 32])
+            assert last & ((1 << (64 - 2 * (n % 32))) - 1) == 0  # padding bases are 00
+
+
+@pytest.mark.parametrize("bad", [b"N", b"n", b"-", b"\x00", b"U", b"\xc1", b"B"])
+@pytest.mark.parametrize("pos", [0, 5, 31, 32, 999])
+def test_pack_alphabet_error(bad, pos):
+    s = bytearray(b"ACGT" * 300)
+    s[pos:pos + 1] = bad
+    q = gpumem.pack(bytes(s))
+    with pytest.raises(gpumem.GpumemError) as ei:
+        q.check()
+    assert ei.value.name == "ERR_ALPHABET"
+    assert f"position {pos}" in str(ei.value)
+    # find_mems reports it too
+    R = gpumem.pack(b"ACGT" * 10)
+    idx = gpumem.index_build(R, 4, 8)
+    with pytest.raises(gpumem.GpumemError) as ei:
+        gpumem.find_mems(idx, q)
+    assert ei.value.name == "ERR_ALPHABET"
+
+
+# ------------------------------------------------------------------ K2-K5 index
+def _index_gpu(R, ls, step):
+    s = gpumem.pack(R)
+    idx = gpumem.index_build(s, ls, ls + step - 1, step)
+    p, l = idx.view()
+    out = p.cpu().numpy().copy(), l.cpu().numpy().copy()
+    torch.cuda.synchronize()
+    return out
+
+
+def test_index_golden_w2():
+    g = read_golden("w2_index.txt")
+    p, l = _index_gpu(g["R"], g["ls"], g["step"])
+    assert p.tolist() == g["ptrs"] and l.tolist() == g["locs"]
+
+
+@pytest.mark.parametrize("cfg,ls,step,scale", [("c1", 10, 11, 1.0), ("c1", 1, 1, 0.01), ("c1", 3, 5, 0.2),
+                                                ("c2", 12, 9, 1.0), ("c3", 13, 38, 0.1), ("c4", 13, 8, 0.02),
+                                                ("c4", 15, 1, 0.01), ("c1", 7, 64, 0.5)])
+def test_index_parity_word_for_word(cfg, ls, step, scale):
+    P = synth.make_pair(cfg, scale=scale)
+    p, l = _index_gpu(P.R.tobytes(), ls, step)
+    op, ol = oracle.index(P.R.tobytes(), ls, step)
+    assert np.array_equal(p, op)
+    assert np.array_equal(l, ol)
+
+
+def test_index_short_reference():
+    p, l = _index_gpu(b"ACG", 4, 1)
+    assert len(l) == 0 and not p.any()
+
+
+# ------------------------------------------------------------------ find: small exact cases
+@pytest.mark.parametrize("name", ["w1.txt", "w2.txt", "w3.txt", "w4.txt"])
+def test_golden_examples(name):
+    g = read_golden(name)
+    want = sorted(g["mem"])
+    for ls in range(1, min(g["L"], 15) + 1):
+        for step in range(1, g["L"] - ls + 2):
+            got = gpu_mems(g["R"], g["Q"], g["L"], ls, step)
+            assert [tuple(t) for t in got.tolist()] == want, (ls, step)
+
+
+def test_random_tiny_vs_brute_force():
+    rng = np.random.default_rng(99)
+    alph = [b"A", b"AC", b"ACG", b"ACGT"]
+    for trial in range(300):
+        R, Q = synth.random_pair(rng, int(rng.integers(0, 200)), int(rng.integers(0, 200)), alph[trial % 4])
+        L = int(rng.integers(1, 40))
+        ls = int(rng.integers(1, min(L, 15) + 1))
+        step = int(rng.integers(1, L - ls + 2))
+        want = oracle.brute(R, Q, L)
+        got = gpu_mems(R.tobytes(), Q.tobytes(), L, ls, step)
+        assert np.array_equal(got, want), (trial, len(R), len(Q), L, ls, step)
+
+
+@pytest.mark.parametrize("n,m", [(1, 1), (5, 3), (40, 70), (300, 257), (1000, 64)])
+def test_homopolymer_closed_form(n, m):
+    for L, ls in ((2, 1), (20, 10), (33, 13), (100, 15)):
+        if ls > L:
+            continue
+        want = np.array(pyoracle.homopolymer(n, m, L), dtype=np.uint32).reshape(-1, 3)
+        got = gpu_mems("A" * n, "A" * m, L, ls)
+        assert np.array_equal(got, want), (n, m, L, ls)
+
+
+@pytest.mark.parametrize("L,ls", [(20, 10), (50, 13), (100, 13), (300, 13), (7, 1), (13, 13), (40, 15)])
+def test_adversarial_repeats(L, ls):
+    """Tandem repeats, (AC)^n, multi-word left checks (step > 32, > 64, 288),
+    ls = 1, ls = L (step 1), MEMs touching all four sequence ends."""
+    rng = np.random.default_rng(L * 31 + ls)
+    parts_r = [b"AC" * 200, bytes(synth.to_ascii(rng.integers(0, 4, 500).astype(np.uint8))), b"AAT" * 100,
+               b"G" * 150]
+    R = b"".join(parts_r)
+    Q = R[:400] + b"T" + b"AC" * 150 + bytes(synth.to_ascii(rng.integers(0, 4, 300).astype(np.uint8))) + R[-500:]
+    want = oracle.mems(R, Q, L, ls)
+    got = gpu_mems(R, Q, L, ls)
+    assert np.array_equal(got, want)
+    invariants.check(R, Q, L, got)
+    if len(want):
+        assert np.array_equal(gpu_mems(R, Q, L, ls, device_input=True), want)
+
+
+def test_self_match_and_edges():
+    P = synth.make_pair("c1", scale=0.3)
+    R = P.R.tobytes()
+    got = gpu_mems(R, R, 20, 10)
+    assert (0, 0, len(R)) in {tuple(t) for t in got.tolist()}
+    assert np.array_equal(got, oracle.mems(R, R, 20, 10))
+    assert len(gpu_mems(R, b"ACG", 20, 10)) == 0          # |Q| < ls
+    assert len(gpu_mems(R, b"ACGT" * 4, 20, 10)) == 0     # |Q| < L
+    assert len(gpu_mems(b"", R, 20, 10)) == 0
+    assert len(gpu_mems(R, b"", 20, 10)) == 0
+
+
+def test_overflow_retry_grid_spill_and_bitmap_invariance():
+    P = synth.make_pair("c1")
+    want = oracle.mems(P.R, P.Q, P.L, P.ls)
+    base = gpu_mems(P.R, P.Q, P.L, P.ls)
+    assert np.array_equal(base, want)
+    for opt, vals in (("out_capacity", [1, 100]), ("find_grid", [1, 3, 148]), ("find_spill", [1, 2, 10**9]),
+                      ("use_bitmap", [0])):
+        for v in vals:
+            gpumem.set_option(opt, v)
+            assert np.array_equal(gpu_mems(P.R, P.Q, P.L, P.ls), want), (opt, v)
+        gpumem.set_option(opt, {"out_capacity": 0, "find_grid": 0, "find_spill": 128, "use_bitmap": 1}[opt])
+
+
+def test_seed_length_and_step_invariance():
+    P = synth.make_pair("c1", scale=0.5)
+    want = oracle.mems(P.R, P.Q, 20, 10)
+    for ls, step in ((10, None), (8, None), (12, 5), (1, 3), (15, 6), (13, 1)):
+        assert np.array_equal(gpu_mems(P.R, P.Q, 20, ls, step), want), (ls, step)
+
+
+def test_qrange_shards_union_to_whole():
+    P = synth.make_pair("c2", scale=0.05)
+    whole = gpu_mems(P.R, P.Q, P.L, P.ls)
+    assert np.array_equal(whole, oracle.mems(P.R, P.Q, P.L, P.ls))
+    n = len(P.Q)
+    for G in (2, 3, 8):
+        cuts = [n * g // G for g in range(G + 1)]
+        parts = [gpu_mems(P.R, P.Q, P.L, P.ls, q_range=(a, b)) for a, b in zip(cuts[:-1], cuts[1:])]
+        for (a, b), part in zip(zip(cuts[:-1], cuts[1:]), parts):
+            assert np.array_equal(part, oracle.mems(P.R, P.Q, P.L, P.ls, 0, a, b))
+        cat = np.concatenate(parts)
+        cat = cat[np.lexsort((cat[:, 1], cat[:, 0]))]
+        assert np.array_equal(cat, whole)
+
+
+def test_swap_symmetry():
+    P = synth.make_pair("c1", scale=0.2)
+    a = gpu_mems(P.R, P.Q, 20, 10)
+    b = gpu_mems(P.Q, P.R, 20, 10)[:, [1, 0, 2]]
+    b = b[np.lexsort((b[:, 1], b[:, 0]))]
+    assert np.array_equal(a, b)
+
+
+def test_kernels_are_ours():
+    before = gpumem.launch_count()
+    gpu_mems(b"ACGT" * 100, b"ACGT" * 50, 20, 10)
+    assert gpumem.launch_count() - before >= 5
+
+
+# ------------------------------------------------------------------ configs (scaled and full)
+@pytest.mark.parametrize("cfg,scale", [("c1", 1.0), ("c2", 1.0), ("c3", 0.2), ("c4", 0.04), ("c5_l20", 0.04),
+                                       ("c5_l50", 0.04), ("c5_l300", 0.04)])
+def test_config_parity(cfg, scale):
+    P = synth.make_pair(cfg, scale=scale)
+    want = oracle.mems(P.R, P.Q, P.L, P.ls)
+    got = gpu_mems(P.R, P.Q, P.L, P.ls)
+    assert len(got) == len(want)
+    assert np.array_equal(got, want)
+    invariants.check(P.R, P.Q, P.L, got)
+    s = {tuple(t) for t in got.tolist()}
+    assert all(tuple(t) in s for t in P.planted)
+
+
+@pytest.fixture(scope="module")
+def c4_full():
+    return synth.make_pair("c4")
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("L", [100, 300, 50, 20])
+def test_full_size_c4_c5(c4_full, L):
+    """BASELINE sizes (250 Mbp x 150 Mbp), bit-exact against the full oracle run."""
+    P = c4_full
+    want = oracle.mems(P.R, P.Q, L, 13)
+    got = gpu_mems(P.R, P.Q, L, 13)
+    assert np.array_equal(got, want)
+
+
+@pytest.mark.slow
+def test_full_size_c3():
+    P = synth.make_pair("c3")
+    want = oracle.mems(P.R, P.Q, P.L, P.ls)
+    got = gpu_mems(P.R, P.Q, P.L, P.ls)
+    assert np.array_equal(got, want)
+    invariants.check(P.R, P.Q, P.L, got)
