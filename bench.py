@@ -1,0 +1,318 @@
+#!/usr/bin/env python3
+"""Benchmark: GPUMEM's hot path on B200 -- query Mbp/s (and MEMs/s) incl. index build.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config c4] [--impl ours|reference]
+
+One step = the whole hot path over the configured pair,
+with the ASCII R and Q already resident in HBM: pack R, pack Q, index R, find
+every MEM (lookup, extension, canonical-seed rule, compaction), sort by (r, q);
+for N > 1 also the NCCL gather to rank 0 and rank 0's merge kernel. L2 is
+flushed (a 512 MB write, > 126 MB L2) before every step, outside the timed
+events. `value` = |Q| / (mean step time, max over ranks) in Mbp/s.
+
+--impl reference times the CPU oracle (oracle/, the only reference this paper
+tier has) on the box's host cores, each step a bounded sample of the workload.
+Prints ONE JSON line on rank 0.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from paper_conf_ipps_abu_dolehkac14_b200 import synth  # noqa: E402
+
+METRIC = "query Mbp/s incl. index build (MEM extraction, GPUMEM hot path)"
+WORKLOAD_DESC = {
+    "c1": "C1: 100 kbp random R, Q = R + 1% SNPs + planted repeats, L=20, ls=10",
+    "c2": "C2: 5 Mbp vs 5 Mbp (~5% divergence), L=20, ls=12",
+    "c3": "C3: 50 Mbp vs 50 Mbp with segmental duplications, L=50, ls=13",
+    "c4": "C4: human-chromosome-scale synthetic pair 250 Mbp vs 150 Mbp, L=100, ls=13",
+    "c5_l20": "C5: C4 pair at L=20, ls=13", "c5_l50": "C5: C4 pair at L=50, ls=13",
+    "c5_l100": "C5: C4 pair at L=100, ls=13", "c5_l300": "C5: C4 pair at L=300, ls=13",
+}
+ORACLE_SAMPLE_BP = {"ours": 60_000_000, "reference": 16_000_000}
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=30)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="c4", choices=sorted(WORKLOAD_DESC))
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--e2e-steps", type=int, default=5)
+    return ap.parse_args()
+
+
+# ------------------------------------------------------------------ clocks (NVML, during the timed region)
+_REASONS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap", 0x8: "hw_slowdown",
+            0x10: "sync_boost", 0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown",
+            0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting"}
+
+
+class ClockSampler:
+    def __init__(self, index=0, period=0.005):
+        self.samples, self.reasons, self.max_mhz = [], set(), None
+        self.period = period
+        self._stop = threading.Event()
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+        except Exception as e:  # pragma: no cover
+            self.nv, self.err = None, repr(e)
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                r = self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                for bit, name in _REASONS.items():
+                    if r & bit and bit != 0x1:
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            time.sleep(self.period)
+
+    def __enter__(self):
+        if self.nv:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self.nv:
+            self.t.join()
+
+    def summary(self):
+        if not self.nv:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvml unavailable"]}
+        return {"sm_mhz": statistics.median(self.samples) if self.samples else None, "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+# ------------------------------------------------------------------ CPU oracle timing (cpu_baseline / reference arm)
+def oracle_sample(P, sample_bp):
+    import oracle
+    threads = len(os.sched_getaffinity(0))
+    q_end = min(len(P.Q), sample_bp)
+    t = time.perf_counter()
+    out = oracle.mems(P.R, P.Q, P.L, P.ls, 0, 0, q_end, threads=threads)
+    dt = time.perf_counter() - t
+    return dt, q_end, len(out), oracle.num_threads(threads)
+
+
+def run_reference(args, P):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    sample = min(len(P.Q), ORACLE_SAMPLE_BP["reference"])
+    times = []
+    for i in range(args.warmup + args.steps):
+        dt, q_end, nm, cores = oracle_sample(P, sample)
+        if i >= args.warmup:
+            times.append(dt)
+    t = statistics.mean(times)
+    v = q_end / 1e6 / t
+    desc = (f"full hash index of R ({len(P.R)} bp) + lookup/extension/sort-unique of MEMs starting in "
+            f"Q[0:{q_end}] ({q_end / len(P.Q):.1%} of Q)")
+    line = {"impl": "reference", "metric": METRIC, "value": round(v, 3), "unit": "Mbp/s", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(t * 1e3, 3),
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u8 (ASCII chars)",
+            "data": "synthetic", "config": {"workload": WORKLOAD_DESC[args.config], "sample": desc},
+            "cpu_baseline": {"value": round(v, 3), "unit": "Mbp/s", "cores": cores, "kind": "oracle",
+                             "sample": desc},
+            "e2e": {"value": round(v, 3), "unit": "Mbp/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ------------------------------------------------------------------ roofline bookkeeping
+def algorithmic_bytes(nR, nQ, ls, L, stats, world):
+    """Algorithmic (useful) HBM bytes per step of each stage on one rank (DESIGN.md
+    "Roofline"): what the method must move, not sector over-fetch."""
+    step = L - ls + 1
+    n_locs = (nR - ls) // step + 1 if nR >= ls else 0
+    nb = 1 << (2 * ls)
+    passes = (2 * ls + 7) // 8
+    pos, occ, hits, mems = stats["positions"], stats["occupied"], stats["hits"], stats["mems"]
+    return {
+        # 1 B ASCII read + 0.25 B packed write per base, R and Q
+        "pack": 1.25 * (nR + nQ),
+        # per sampled seed: one 8-byte R window read, code + location written
+        "index.codes": n_locs * (8 + 8),
+        # per radix pass: keys+values read twice (histogram, scatter) and written once
+        "index.sort": passes * n_locs * (16 + 8),
+        # sorted codes read once; ptrs (4^ls + 1 words) and the 4^ls-bit bitmap written
+        "index.ptrs": n_locs * 4 + 4 * (nb + 1) + nb / 8,
+        # per query position: packed Q (0.25 B) + its bitmap bit; per occupied seed the
+        # ptrs pair (8 B); per hit one location (4 B) + one 32-base R word each side
+        # (16 B); per MEM the 12-byte record written
+        "find": 0.25 * pos + pos / 8 + 8 * occ + 20 * hits + 12 * mems,
+        # output sort: 7 passes of (12 B read twice + 12 B written) over 56-bit keys
+        "sort": mems * 36 * ((30 + 30 + 7) // 8),
+    }
+
+
+# ------------------------------------------------------------------ our arm
+def run_ours(args, P):
+    import torch
+    import torch.distributed as dist
+    from paper_conf_ipps_abu_dolehkac14_b200 import gpumem as gm
+    from paper_conf_ipps_abu_dolehkac14_b200.dist import find_mems_sharded
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = torch.device("cuda", local)
+    stream = torch.cuda.current_stream()
+
+    # inputs resident in HBM before timing
+    R_dev = torch.from_numpy(P.R).to(dev)
+    Q_dev = torch.from_numpy(P.Q).to(dev)
+    flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
+    torch.cuda.synchronize()
+
+    def step():
+        merged, local_m = find_mems_sharded(R_dev, Q_dev, P.L, P.ls)
+        return merged, local_m
+
+    for _ in range(args.warmup):
+        flush.zero_()
+        merged, lm = step()
+    torch.cuda.synchronize()
+    n_mems = len(merged) if merged is not None else 0
+    stats = lm.stats()
+    del merged, lm
+
+    gm.profile_enable(True)
+    gm.profile_read()  # drop warm-up records
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    l0 = gm.launch_count()
+    with ClockSampler(local) as clk:
+        for i in range(args.steps):
+            flush.zero_()
+            ev[i][0].record(stream)
+            merged, lm = step()
+            ev[i][1].record(stream)
+        torch.cuda.synchronize()
+    launches = gm.launch_count() - l0
+    if world > 1:
+        dist.barrier()
+    prof = gm.profile_read()
+    gm.profile_enable(False)
+    del merged, lm
+    step_ms = [a.elapsed_time(b) for a, b in ev]
+    tot = torch.tensor([sum(step_ms)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(tot, op=dist.ReduceOp.MAX)
+    ms = tot.item() / args.steps
+    value = len(P.Q) / 1e6 / (ms / 1e3)
+
+    # ---- roofline of the dominant kernel (largest share of the step)
+    kernel_ms = {k: v[0] / args.steps for k, v in prof.items()}
+    dom = max(kernel_ms, key=kernel_ms.get)
+    peaks = {}
+    try:
+        peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        pass
+    peak = peaks.get("hbm_gbs", 6650.0)
+    peak_src = "measured" if "hbm_gbs" in peaks else "fallback"
+    nQ, nR, ls, L = len(P.Q), len(P.R), P.ls, P.L
+    step_ = L - ls + 1
+    alg = algorithmic_bytes(nR, nQ, ls, L, stats, world)
+    roof = None
+    if dom in alg:
+        n_launch = prof[dom][1] / args.steps
+        achieved = alg[dom] / (kernel_ms[dom] / 1e3) / 1e9
+        roof = {"bound": "hbm", "kernel": dom, "achieved": round(achieved, 1), "peak": peak,
+                "peak_source": peak_src, "unit": "GB/s", "frac": round(achieved / peak, 4), "traffic": None,
+                "algorithmic_bytes_per_step": int(alg[dom]), "launches_per_step": n_launch,
+                "ms_per_step": round(kernel_ms[dom], 4)}
+    stage_frac = {k: round(alg[k] / (kernel_ms[k] / 1e3) / 1e9 / peak, 4) for k in alg if k in kernel_ms}
+
+    line = {"metric": METRIC, "value": round(value, 2), "unit": "Mbp/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": round(ms, 4), "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "u64 (2-bit packed bases), u32 positions", "data": "synthetic",
+            "config": {"workload": WORKLOAD_DESC[args.config], "R_bp": nR, "Q_bp": nQ, "L": L, "ls": ls,
+                       "step": step_, "mems": n_mems, "l2": "flushed before every step (512 MB write)",
+                       "parallelism": f"query-sharded dp{world}, index rebuilt per rank, NCCL gather + merge",
+                       "inputs": "ASCII R, Q resident in HBM at t0"},
+            "mems_per_s": round(n_mems / (ms / 1e3), 1),
+            "stage_ms": {k: round(v, 4) for k, v in sorted(kernel_ms.items())},
+            "stage_hbm_frac": stage_frac, "find_stats": stats, "gpu_launches": int(launches),
+            "clocks": clk.summary(), "roofline": roof}
+
+    # ---- end-to-end through the public API with HOST buffers (pinned), H2D + D2H inside
+    if not args.no_e2e and world == 1:
+        R_h = torch.from_numpy(P.R).pin_memory()
+        Q_h = torch.from_numpy(P.Q).pin_memory()
+        times = []
+        nm = 0
+        for i in range(args.e2e_steps + 1):
+            flush.zero_()
+            torch.cuda.synchronize()
+            t = time.perf_counter()
+            Rs = gm.pack(R_h)
+            Qs = gm.pack(Q_h)
+            idx = gm.index_build(Rs, ls, L)
+            m = gm.find_mems(idx, Qs)
+            host = m.numpy()
+            dt = time.perf_counter() - t
+            nm = len(host)
+            for h in (m, idx, Qs, Rs):
+                h.free()
+            if i:
+                times.append(dt)
+        te = statistics.mean(times)
+        line["e2e"] = {"value": round(nQ / 1e6 / te, 2), "unit": "Mbp/s", "h2d_bytes_per_step": nR + nQ,
+                       "d2h_bytes_per_step": 12 * nm + 64, "ms_per_step": round(te * 1e3, 3),
+                       "steps": args.e2e_steps}
+
+    # ---- CPU oracle on a bounded sample (rank 0, N = 1 only)
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        dt, q_end, nm_cpu, cores = oracle_sample(P, ORACLE_SAMPLE_BP["ours"])
+        line["cpu_baseline"] = {
+            "value": round(q_end / 1e6 / dt, 3), "unit": "Mbp/s", "cores": cores, "kind": "oracle",
+            "sample": f"full hash index of R + MEMs starting in Q[0:{q_end}] ({q_end / nQ:.1%} of Q); "
+                      f"{nm_cpu} MEMs in {dt:.2f} s"}
+    if world > 1:
+        dist.barrier()
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def main():
+    args = parse()
+    P = synth.make_pair(args.config)
+    if args.impl == "reference":
+        run_reference(args, P)
+    else:
+        run_ours(args, P)
+
+
+if __name__ == "__main__":
+    main()

@@ -115,6 +115,18 @@ gpumem_status gpumem_index_view(const gpumem_index *idx, const uint32_t **dev_pt
 gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uint64_t q_begin,
                                uint64_t q_end, void *cuda_stream, gpumem_mems **out);
 
+/* Work counters of the find call that produced `m` (diagnostics; the bench derives the
+ * find kernel's algorithmic bytes from them). */
+typedef struct {
+    uint64_t positions;      /* query seed positions scanned                                 */
+    uint64_t occupied;       /* of those, positions whose seed occurs in the index           */
+    uint64_t hits;           /* (sampled r, q) pairs with equal seeds that were examined      */
+    uint64_t spilled_chunks; /* heavy-bucket chunks drained by the heavy kernel               */
+    uint64_t mems;           /* MEMs reported                                                */
+    uint32_t attempts;       /* 1, or 2 after an output-capacity overflow                     */
+} gpumem_find_stats;
+gpumem_status gpumem_mems_stats(const gpumem_mems *m, gpumem_find_stats *out);
+
 /* Borrowed device pointer to the sorted triples and their count. */
 gpumem_status gpumem_mems_view(const gpumem_mems *m, const gpumem_triple **dev_ptr, uint64_t *count);
 

@@ -36,6 +36,7 @@ struct gpumem_index {
     uint32_t *ptrs;
     uint32_t *locs;
     uint32_t *bitmap;
+    uint4 *recs;
 };
 
 struct gpumem_mems {
@@ -44,6 +45,7 @@ struct gpumem_mems {
     cudaStream_t stream;
     uint64_t count;
     gpumem_triple *dev;
+    gpumem_find_stats stats;
 };
 
 namespace gm {
@@ -226,10 +228,10 @@ gpumem_status check_device(int *dev) {
         if (_e != cudaSuccess) return cuda_fail(_e, what); \
     } while (0)
 
-unsigned long long *pinned_slots() {  // 8 per thread, never freed
+unsigned long long *pinned_slots() {  // 16 per thread, never freed
     thread_local unsigned long long *p = nullptr;
     if (!p) {
-        if (cudaMallocHost(&p, 8 * sizeof(unsigned long long)) != cudaSuccess) {
+        if (cudaMallocHost(&p, 16 * sizeof(unsigned long long)) != cudaSuccess) {
             cudaGetLastError();
             p = nullptr;
         }
@@ -317,6 +319,7 @@ void gpumem_free(void *handle) {
         dfree(x->ptrs, x->stream);
         dfree(x->locs, x->stream);
         dfree(x->bitmap, x->stream);
+        dfree(x->recs, x->stream);
         x->magic = 0;
         delete x;
     } else if (magic == kMagicMems) {
@@ -430,10 +433,17 @@ gpumem_status gpumem_index_build_step(const gpumem_seq *R, uint32_t ls, uint32_t
         Stage g("index.ptrs", s);
         CK(launch_ptrs_fill(codes_sorted, n_locs, ls, ptrs, bitmap, s), "ptrs fill");
     }
+    auto *recs = static_cast<uint4 *>(sc.get((n_locs ? n_locs : 1) * sizeof(uint4)));
+    if (!recs) return GPUMEM_ERR_NOMEM;
+    if (n_locs) {
+        Stage g("index.recs", s);
+        CK(launch_seed_recs(R->words, ls, locs, n_locs, recs, s), "seed records");
+    }
     sc.keep(ptrs);
     sc.keep(bitmap);
     sc.keep(locs);
-    auto *h = new gpumem_index{kMagicIdx, dev, s, R, ls, L, step, n_locs, ptrs, locs, bitmap};
+    sc.keep(recs);
+    auto *h = new gpumem_index{kMagicIdx, dev, s, R, ls, L, step, n_locs, ptrs, locs, bitmap, recs};
     *out = h;
     return GPUMEM_OK;
 }
@@ -473,7 +483,8 @@ static gpumem_status sort_into_triples(uint64_t *keys, uint32_t *lens, uint64_t 
         CK(launch_keys_to_triples(alt ? k1 : keys, alt ? l1 : lens, n, qbits, trip, s), "keys to triples");
     }
     sc.keep(trip);
-    *out = new gpumem_mems{kMagicMems, dev, s, n, trip};
+    *out = new gpumem_mems{kMagicMems, dev, s, n, trip, gpumem_find_stats{}};
+    (*out)->stats.mems = n;
     return GPUMEM_OK;
 }
 
@@ -502,8 +513,9 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
     P.nR = nR;
     P.Q = Q->words;
     P.nQ = nQ;
+    P.nQw = Q->n_words;
     P.ptrs = idx->ptrs;
-    P.locs = idx->locs;
+    P.recs = idx->recs;
     P.bitmap = idx->bitmap;
     P.ls = ls;
     P.L = L;
@@ -527,18 +539,20 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
 
     Scratch sc(s);
     auto *ctr = static_cast<unsigned long long *>(sc.get(64));
-    const uint64_t spill_cap = span / 64 + 4096;
+    const uint64_t spill_cap = span / 8 + 4096;
     auto *spill = static_cast<uint4 *>(sc.get(spill_cap * sizeof(uint4)));
     if (!ctr || !spill) return GPUMEM_ERR_NOMEM;
     P.out_count = ctr;
     P.spill_count = ctr + 1;
     P.tile_ctr = reinterpret_cast<unsigned int *>(ctr + 2);
+    P.stats = ctr + 3;
     P.spill = spill;
     P.spill_cap = spill_cap;
     unsigned long long *h = pinned_slots();
     if (!h) return fail(GPUMEM_ERR_NOMEM, "pinned host buffer");
 
     uint64_t count = 0;
+    int attempts = 0;
     uint64_t *keys = nullptr;
     uint32_t *lens = nullptr;
     for (int attempt = 0; attempt < 2; ++attempt) {
@@ -557,26 +571,45 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
             Stage g("find.heavy", s);
             CK(launch_heavy(P, s), "heavy kernel");
         }
-        CK(cudaMemcpyAsync(h, ctr, 16, cudaMemcpyDeviceToHost, s), "D2H count");
-        CK(cudaMemcpyAsync(h + 2, R->bad, 8, cudaMemcpyDeviceToHost, s), "D2H flag");
-        CK(cudaMemcpyAsync(h + 3, Q->bad, 8, cudaMemcpyDeviceToHost, s), "D2H flag");
+        ++attempts;
+        CK(cudaMemcpyAsync(h, ctr, 64, cudaMemcpyDeviceToHost, s), "D2H counters");
+        CK(cudaMemcpyAsync(h + 8, R->bad, 8, cudaMemcpyDeviceToHost, s), "D2H flag");
+        CK(cudaMemcpyAsync(h + 9, Q->bad, 8, cudaMemcpyDeviceToHost, s), "D2H flag");
         CK(cudaStreamSynchronize(s), "find sync");
-        if (h[2] != ~0ull) return fail(GPUMEM_ERR_ALPHABET, "R: byte at position %llu is not in {A,C,G,T,a,c,g,t}", h[2]);
-        if (h[3] != ~0ull) return fail(GPUMEM_ERR_ALPHABET, "Q: byte at position %llu is not in {A,C,G,T,a,c,g,t}", h[3]);
+        if (h[8] != ~0ull) return fail(GPUMEM_ERR_ALPHABET, "R: byte at position %llu is not in {A,C,G,T,a,c,g,t}", h[8]);
+        if (h[9] != ~0ull) return fail(GPUMEM_ERR_ALPHABET, "Q: byte at position %llu is not in {A,C,G,T,a,c,g,t}", h[9]);
         count = h[0];
         if (count <= cap) break;
         if (attempt == 1) return fail(GPUMEM_ERR_CUDA, "output count changed between runs (%llu > %llu)",
                                       (unsigned long long)count, (unsigned long long)cap);
         cap = count;  // overflow: rerun with the exact capacity
     }
+    gpumem_find_stats fs{};
+    fs.positions = span;
+    fs.occupied = h[3] + h[6];
+    fs.hits = h[4] + h[5];
+    fs.spilled_chunks = h[1] < spill_cap ? h[1] : spill_cap;
+    fs.attempts = uint32_t(attempts);
     const uint32_t key_bits = bits_for(nR) + P.qbits;
-    return sort_into_triples(keys, lens, count, key_bits, P.qbits, dev, s, out);
+    const gpumem_status st2 = sort_into_triples(keys, lens, count, key_bits, P.qbits, dev, s, out);
+    if (st2 == GPUMEM_OK) {
+        fs.mems = count;
+        (*out)->stats = fs;
+    }
+    return st2;
 }
 
 gpumem_status gpumem_mems_view(const gpumem_mems *m, const gpumem_triple **dev_ptr, uint64_t *count) {
     if (!m || m->magic != kMagicMems) return fail(GPUMEM_ERR_ARG, "not a gpumem_mems");
     if (dev_ptr) *dev_ptr = m->dev;
     if (count) *count = m->count;
+    return GPUMEM_OK;
+}
+
+gpumem_status gpumem_mems_stats(const gpumem_mems *m, gpumem_find_stats *out) {
+    if (!m || m->magic != kMagicMems) return fail(GPUMEM_ERR_ARG, "not a gpumem_mems");
+    if (!out) return fail(GPUMEM_ERR_ARG, "out is NULL");
+    *out = m->stats;
     return GPUMEM_OK;
 }
 

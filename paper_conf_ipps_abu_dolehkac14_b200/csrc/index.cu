@@ -108,7 +108,31 @@ __global__ void __launch_bounds__(kFillThreads) k_ptrs_fill(const uint32_t *__re
     }
 }
 
+// Seed records (lookup acceleration, not part of the paper's index): for each slot k
+// of locs, {p, bases R[p-16, p) with base p-1 in the low bits (00 before position 0),
+// bases R[p+ls, p+ls+32) first base highest (00 past the end)} -- 16 bytes, one
+// sector, so the find kernel decides a random seed hit without gathering R.
+__global__ void __launch_bounds__(kCodeThreads) k_seed_recs(const uint64_t *__restrict__ R, uint32_t ls,
+                                                            const uint32_t *__restrict__ locs, uint64_t n_locs,
+                                                            uint4 *__restrict__ recs) {
+    const uint64_t k = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+    if (k >= n_locs) return;
+    const uint32_t p = locs[k];
+    const uint32_t left = uint32_t(win_back(R, p));
+    const uint64_t right = win_fwd(R, uint64_t(p) + ls);
+    recs[k] = make_uint4(p, left, uint32_t(right), uint32_t(right >> 32));
+}
+
 }  // namespace
+
+cudaError_t launch_seed_recs(const uint64_t *R, uint32_t ls, const uint32_t *locs, uint64_t n_locs, uint4 *recs,
+                             cudaStream_t s) {
+    if (n_locs == 0) return cudaSuccess;
+    const uint64_t blocks = (n_locs + kCodeThreads - 1) / kCodeThreads;
+    k_seed_recs<<<unsigned(blocks), kCodeThreads, 0, s>>>(R, ls, locs, n_locs, recs);
+    note_launch();
+    return cudaGetLastError();
+}
 
 cudaError_t launch_seed_codes(const uint64_t *R, uint64_t nR, uint32_t ls, uint32_t step, uint64_t n_locs,
                               uint32_t *codes, uint32_t *locs, cudaStream_t s) {

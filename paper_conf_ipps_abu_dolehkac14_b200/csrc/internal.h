@@ -11,7 +11,7 @@ namespace gm {
 // ---------------------------------------------------------------- runtime
 struct Options {
     int64_t find_grid = 0;       // 0 = SMs x occupancy
-    int64_t find_spill = 128;    // bucket sizes above this go to the heavy queue
+    int64_t find_spill = 64;     // bucket sizes above this go to the heavy queue
     int64_t out_capacity = 0;    // 0 = automatic
     int64_t use_bitmap = 1;      // probe the occupancy bitmap before ptrs
 };
@@ -52,6 +52,9 @@ cudaError_t launch_seed_codes(const uint64_t *R, uint64_t nR, uint32_t ls, uint3
                               uint32_t *codes, uint32_t *locs, cudaStream_t s);
 cudaError_t launch_ptrs_fill(const uint32_t *sorted_codes, uint64_t n_locs, uint32_t ls, uint32_t *ptrs,
                              uint32_t *bitmap, cudaStream_t s);
+// Seed records for the lookup: rec[k] = {locs[k], 16 bases left of it, 32 bases right of its seed}.
+cudaError_t launch_seed_recs(const uint64_t *R, uint32_t ls, const uint32_t *locs, uint64_t n_locs, uint4 *recs,
+                             cudaStream_t s);
 
 // Find (find.cu)
 struct FindParams {
@@ -59,8 +62,9 @@ struct FindParams {
     uint64_t nR;
     const uint64_t *Q;
     uint64_t nQ;
+    uint64_t nQw;                // allocated words of Q (incl. padding)
     const uint32_t *ptrs;
-    const uint32_t *locs;
+    const uint4 *recs;           // seed records, parallel to locs: {p, R[p-16,p), R[p+ls,p+ls+32)}
     const uint32_t *bitmap;
     uint32_t ls, L, step, qbits;
     uint64_t scan_lo, scan_hi;   // query seed positions scanned
@@ -75,6 +79,7 @@ struct FindParams {
     uint4 *spill;                // {q, beg, len, 0}
     uint64_t spill_cap;
     unsigned long long *spill_count;
+    unsigned long long *stats;   // [0] entries kept local, [1] hits kept local, [2] hits spilled, [3] entries spilled
     int use_bitmap;
 };
 uint64_t find_tile_positions();

@@ -41,6 +41,7 @@ SYMBOLS = {
     "gpumem_find_mems": (ctypes.c_int, [_vp, _vp, _c_u64, _c_u64, _vp, _P(_vp)]),
     "gpumem_mems_view": (ctypes.c_int, [_vp, _P(_vp), _P(_c_u64)]),
     "gpumem_mems_to_host": (ctypes.c_int, [_vp, _vp, _c_u64]),
+    "gpumem_mems_stats": (ctypes.c_int, [_vp, _vp]),
     "gpumem_merge_sorted": (ctypes.c_int, [_P(_vp), _P(_c_u64), ctypes.c_int, _vp, _P(_vp)]),
     "gpumem_free": (None, [_vp]),
     "gpumem_last_error": (ctypes.c_char_p, []),
@@ -58,6 +59,14 @@ for _name, (_res, _args) in SYMBOLS.items():
 
 STATUS = {0: "OK", 1: "ERR_ARG", 2: "ERR_ALPHABET", 3: "ERR_RANGE", 4: "ERR_NOMEM", 5: "ERR_CUDA",
           6: "ERR_UNSUPPORTED"}
+
+
+class FindStats(ctypes.Structure):
+    _fields_ = [("positions", _c_u64), ("occupied", _c_u64), ("hits", _c_u64), ("spilled_chunks", _c_u64),
+                ("mems", _c_u64), ("attempts", _c_u32)]
+
+    def as_dict(self):
+        return {k: int(getattr(self, k)) for k, _ in self._fields_}
 
 
 class GpumemError(RuntimeError):
@@ -143,6 +152,11 @@ class Mems(_Handle):
 
     def __len__(self):
         return self.view()[1]
+
+    def stats(self):
+        s = FindStats()
+        _check(_lib.gpumem_mems_stats(self.handle, ctypes.byref(s)))
+        return s.as_dict()
 
     def numpy(self):
         """(N, 3) uint32 [r, q, len] copied to the host (synchronous)."""
