@@ -155,10 +155,13 @@ def algorithmic_bytes(nR, nQ, ls, L, stats, world):
         "pack": 1.25 * (nR + nQ),
         # per sampled seed: one 8-byte R window read, code + location written
         "index.codes": n_locs * (8 + 8),
-        # per radix pass: keys+values read twice (histogram, scatter) and written once
-        "index.sort": passes * n_locs * (16 + 8),
+        # counting sort by seed, per 8-bit digit pass: code + location read and written once
+        # (the all-digit histogram adds one read of the codes)
+        "index.sort": passes * n_locs * 16 + n_locs * 4,
         # sorted codes read once; ptrs (4^ls + 1 words) and the 4^ls-bit bitmap written
         "index.ptrs": n_locs * 4 + 4 * (nb + 1) + nb / 8,
+        # per slot: location read, R windows read (2 x 8 B), 16-byte seed record written
+        "index.recs": n_locs * (4 + 16 + 16),
         # per query position: packed Q (0.25 B) + its bitmap bit; per occupied seed the
         # ptrs pair (8 B); per hit one location (4 B) + one 32-base R word each side
         # (16 B); per MEM the 12-byte record written
