@@ -249,8 +249,15 @@ def run_ours(args, P):
     if dom in alg:
         n_launch = prof[dom][1] / args.steps
         achieved = alg[dom] / (kernel_ms[dom] / 1e3) / 1e9
+        traffic = None
+        try:  # dram read+write bytes of that kernel from the committed ncu --set full capture
+            t = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json"))).get(args.config)
+            if t and dom == "find" and world == 1:
+                traffic = int(t["traffic_bytes"])
+        except Exception:
+            pass
         roof = {"bound": "hbm", "kernel": dom, "achieved": round(achieved, 1), "peak": peak,
-                "peak_source": peak_src, "unit": "GB/s", "frac": round(achieved / peak, 4), "traffic": None,
+                "peak_source": peak_src, "unit": "GB/s", "frac": round(achieved / peak, 4), "traffic": traffic,
                 "algorithmic_bytes_per_step": int(alg[dom]), "launches_per_step": n_launch,
                 "ms_per_step": round(kernel_ms[dom], 4)}
     stage_frac = {k: round(alg[k] / (kernel_ms[k] / 1e3) / 1e9 / peak, 4) for k in alg if k in kernel_ms}
