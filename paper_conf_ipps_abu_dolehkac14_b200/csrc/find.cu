@@ -186,15 +186,33 @@ __global__ void __launch_bounds__(kT) k_find(const FindParams P) {
                     occ[j] = qa + j < P.scan_hi;
                 }
                 if (P.use_bitmap) {
+                    // rank-word probe (occupancy bit + rank), then the compact {first, count}
+                    uint32_t rank[kQPT];
 #pragma unroll
-                    for (int j = 0; j < kQPT; ++j)
-                        if (occ[j]) occ[j] = (__ldg(P.bitmap + (code[j] >> 5)) >> (code[j] & 31)) & 1u;
-                }
+                    for (int j = 0; j < kQPT; ++j) {
+                        rank[j] = 0;
+                        if (occ[j]) {
+                            const unsigned long long rw = __ldg(P.rankw + (code[j] >> 5));
+                            const uint32_t bit = code[j] & 31, bits = uint32_t(rw);
+                            occ[j] = (bits >> bit) & 1u;
+                            rank[j] = uint32_t(rw >> 32) + __popc(bits & ((1u << bit) - 1u));
+                        }
+                    }
 #pragma unroll
-                for (int j = 0; j < kQPT; ++j) {
-                    if (occ[j]) {
-                        beg[j] = __ldg(P.ptrs + code[j]);
-                        cnt[j] = __ldg(P.ptrs + code[j] + 1) - beg[j];
+                    for (int j = 0; j < kQPT; ++j) {
+                        if (occ[j]) {
+                            const uint2 b = __ldg(P.buckets + rank[j]);
+                            beg[j] = b.x;
+                            cnt[j] = b.y;
+                        }
+                    }
+                } else {  // the paper's lookup: ptrs[s], ptrs[s+1]
+#pragma unroll
+                    for (int j = 0; j < kQPT; ++j) {
+                        if (occ[j]) {
+                            beg[j] = __ldg(P.ptrs + code[j]);
+                            cnt[j] = __ldg(P.ptrs + code[j] + 1) - beg[j];
+                        }
                     }
                 }
 #pragma unroll

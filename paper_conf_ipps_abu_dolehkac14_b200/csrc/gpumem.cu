@@ -35,7 +35,8 @@ struct gpumem_index {
     uint64_t n_locs;
     uint32_t *ptrs;
     uint32_t *locs;
-    uint32_t *bitmap;
+    unsigned long long *rankw;
+    uint2 *buckets;
     uint4 *recs;
 };
 
@@ -318,7 +319,8 @@ void gpumem_free(void *handle) {
         cudaSetDevice(x->device);
         dfree(x->ptrs, x->stream);
         dfree(x->locs, x->stream);
-        dfree(x->bitmap, x->stream);
+        dfree(x->rankw, x->stream);
+        dfree(x->buckets, x->stream);
         dfree(x->recs, x->stream);
         x->magic = 0;
         delete x;
@@ -405,9 +407,12 @@ gpumem_status gpumem_index_build_step(const gpumem_seq *R, uint32_t ls, uint32_t
     const uint64_t n_locs = R->n >= ls ? (R->n - ls) / step + 1 : 0;
     Scratch sc(s);
     auto *ptrs = static_cast<uint32_t *>(sc.get((nb + 1) * 4));
-    auto *bitmap = static_cast<uint32_t *>(sc.get(((nb + 31) / 32) * 4));
+    auto *rankw = static_cast<unsigned long long *>(sc.get(((nb + 31) / 32) * 8));
+    const uint64_t max_occ = (n_locs < nb ? n_locs : nb) + 1;
+    auto *buckets = static_cast<uint2 *>(sc.get(max_occ * sizeof(uint2)));
+    void *fill_scratch = sc.get(ptrs_fill_scratch_bytes(ls));
     auto *locs0 = static_cast<uint32_t *>(sc.get((n_locs ? n_locs : 1) * 4));
-    if (!ptrs || !bitmap || !locs0) return GPUMEM_ERR_NOMEM;
+    if (!ptrs || !rankw || !buckets || !fill_scratch || !locs0) return GPUMEM_ERR_NOMEM;
     uint32_t *locs = locs0;
     const uint32_t *codes_sorted = nullptr;
     if (n_locs) {
@@ -431,7 +436,7 @@ gpumem_status gpumem_index_build_step(const gpumem_seq *R, uint32_t ls, uint32_t
     }
     {
         Stage g("index.ptrs", s);
-        CK(launch_ptrs_fill(codes_sorted, n_locs, ls, ptrs, bitmap, s), "ptrs fill");
+        CK(launch_ptrs_fill(codes_sorted, n_locs, ls, ptrs, rankw, buckets, fill_scratch, s), "ptrs fill");
     }
     auto *recs = static_cast<uint4 *>(sc.get((n_locs ? n_locs : 1) * sizeof(uint4)));
     if (!recs) return GPUMEM_ERR_NOMEM;
@@ -440,10 +445,11 @@ gpumem_status gpumem_index_build_step(const gpumem_seq *R, uint32_t ls, uint32_t
         CK(launch_seed_recs(R->words, ls, locs, n_locs, recs, s), "seed records");
     }
     sc.keep(ptrs);
-    sc.keep(bitmap);
+    sc.keep(rankw);
+    sc.keep(buckets);
     sc.keep(locs);
     sc.keep(recs);
-    auto *h = new gpumem_index{kMagicIdx, dev, s, R, ls, L, step, n_locs, ptrs, locs, bitmap, recs};
+    auto *h = new gpumem_index{kMagicIdx, dev, s, R, ls, L, step, n_locs, ptrs, locs, rankw, buckets, recs};
     *out = h;
     return GPUMEM_OK;
 }
@@ -516,7 +522,8 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
     P.nQw = Q->n_words;
     P.ptrs = idx->ptrs;
     P.recs = idx->recs;
-    P.bitmap = idx->bitmap;
+    P.rankw = idx->rankw;
+    P.buckets = idx->buckets;
     P.ls = ls;
     P.L = L;
     P.step = step;

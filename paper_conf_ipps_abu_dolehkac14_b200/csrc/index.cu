@@ -11,11 +11,19 @@
 //  k_ptrs_fill   over the 4^ls buckets in chunks of kChunk: per-chunk seed
 //                histogram from the sorted codes (a binary search bounds the
 //                chunk's slice) and a block-wide exclusive scan ->
-//                ptrs[s] = #locations with seed < s (:84), ptrs[4^ls] = n_locs;
-//                the same pass writes the 4^ls-bit occupancy bitmap that the
-//                lookup probes first (an L2-resident filter, 8 MB at ls = 13).
+//                ptrs[s] = #locations with seed < s (:84), ptrs[4^ls] = n_locs.
+//                The same pass writes the lookup structures (not in the paper):
+//                rank words, one u64 per 32 seeds = {occupancy bits, number of
+//                occupied seeds before the word} (16 MB at ls = 13, L2-resident),
+//                and the compact table {ptrs[s], count} of the occupied seeds in
+//                seed order (8 B each). A chunk's first rank comes from a
+//                decoupled look-back over earlier chunks. The lookup then costs
+//                one 8-byte probe per query position plus one 8-byte read per
+//                occupied seed, both L2-resident, instead of two reads of the
+//                HBM-resident 4^ls-entry ptrs.
 // Algorithmic bytes: n_locs * (8 B codes/locs written + 16 B per radix pass read+
-// write) + 4 * (4^ls + 1) B ptrs written + 4^ls / 8 B bitmap written.
+// write) + 4 * (4^ls + 1) B ptrs written + 4^ls / 4 B rank words + 8 B per
+// occupied seed.
 #include "internal.h"
 #include "device.cuh"
 
@@ -47,64 +55,128 @@ __device__ __forceinline__ uint64_t lower_bound(const uint32_t *__restrict__ a, 
     return lo;
 }
 
+constexpr uint64_t kStAgg = 1ull << 62;
+constexpr uint64_t kStInc = 2ull << 62;
+constexpr uint64_t kStMask = (1ull << 62) - 1;
+
+// Exclusive prefix of `agg` over chunks 0..chunk-1 by decoupled look-back (warp 0 only;
+// 32 predecessors per step). Chunks are numbered in launch order by a ticket.
+__device__ __forceinline__ unsigned long long chunk_lookback(unsigned long long *status, uint64_t chunk,
+                                                             unsigned long long agg) {
+    const int lane = threadIdx.x & 31;
+    volatile unsigned long long *st = status;
+    if (chunk == 0) {
+        if (lane == 0) st[0] = kStInc | agg;
+        return 0;
+    }
+    if (lane == 0) st[chunk] = kStAgg | agg;
+    unsigned long long excl = 0;
+    int64_t c = int64_t(chunk) - 1;
+    for (;;) {
+        const int64_t idx = c - lane;
+        const unsigned long long sv = idx >= 0 ? st[idx] : kStInc;
+        const unsigned long long f = sv & ~kStMask;
+        const unsigned inc_m = __ballot_sync(0xffffffffu, f == kStInc);
+        const unsigned zero_m = __ballot_sync(0xffffffffu, f == 0);
+        const int first_inc = inc_m ? __ffs(int(inc_m)) - 1 : 32;
+        const unsigned need = first_inc >= 31 ? 0xffffffffu : ((2u << first_inc) - 1u);
+        if (zero_m & need) continue;  // a predecessor has not published yet
+        unsigned long long part = (lane <= first_inc) ? (sv & kStMask) : 0ull;
+#pragma unroll
+        for (int o = 16; o; o >>= 1) part += __shfl_down_sync(0xffffffffu, part, o);
+        excl += __shfl_sync(0xffffffffu, part, 0);
+        if (first_inc < 32) break;
+        c -= 32;
+    }
+    if (lane == 0) st[chunk] = kStInc | (excl + agg);
+    return excl;
+}
+
 __global__ void __launch_bounds__(kFillThreads) k_ptrs_fill(const uint32_t *__restrict__ codes, uint64_t n,
                                                             uint64_t n_buckets, uint32_t *__restrict__ ptrs,
-                                                            uint32_t *__restrict__ bitmap) {
+                                                            unsigned long long *__restrict__ rankw,
+                                                            uint2 *__restrict__ buckets,
+                                                            unsigned long long *status, unsigned int *ticket) {
     __shared__ uint32_t cnt[kChunk + kChunk / 32];   // one pad word per 32: conflict-free rows
     __shared__ uint64_t range[2];
     __shared__ uint32_t wsum[kFillThreads / 32];
+    __shared__ uint32_t wocc[kFillThreads / 32];
+    __shared__ unsigned long long s_rank0;
+    __shared__ unsigned int s_chunk;
     const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
-    for (uint64_t s0 = uint64_t(blockIdx.x) * kChunk; s0 < n_buckets; s0 += uint64_t(gridDim.x) * kChunk) {
+    if (tid == 0) s_chunk = atomicAdd(ticket, 1u);
+    __syncthreads();
+    {
+        const uint64_t s0 = uint64_t(s_chunk) * kChunk;
         for (int i = tid; i < kChunk + kChunk / 32; i += kFillThreads) cnt[i] = 0;
         if (tid == 0) range[0] = lower_bound(codes, n, s0);
         if (tid == 32) range[1] = lower_bound(codes, n, s0 + kChunk);
         __syncthreads();
         const uint64_t lo = range[0], hi = range[1];
-        // Alg. 1 step 1 for this chunk: seed counts (sorted input: equal runs aggregate per warp)
-        for (uint64_t b = lo; b < hi; b += kFillThreads) {
-            const uint64_t i = b + tid;
-            const bool valid = i < hi;
-            const unsigned act = __ballot_sync(0xffffffffu, valid);
-            if (valid) {
-                const uint32_t d = uint32_t(codes[i] - s0);
-                const unsigned peers = __match_any_sync(act, d);
-                if (lane == __ffs(peers) - 1) atomicAdd(&cnt[d + (d >> 5)], __popc(peers));
-            }
+        // Alg. 1 step 1 for this chunk: seed counts
+        for (uint64_t i = lo + tid; i < hi; i += kFillThreads) {
+            const uint32_t d = uint32_t(codes[i] - s0);
+            atomicAdd(&cnt[d + (d >> 5)], 1u);
         }
         __syncthreads();
         // Alg. 1 step 2: block-wide exclusive scan; thread t owns buckets [32t, 32t+32)
-        uint32_t v[kPer];
         uint32_t sum = 0, occ = 0;
 #pragma unroll
         for (int j = 0; j < kPer; ++j) {
-            v[j] = cnt[tid * (kPer + 1) + j];
-            sum += v[j];
-            occ |= (v[j] ? 1u : 0u) << j;
+            const uint32_t c = cnt[tid * (kPer + 1) + j];
+            sum += c;
+            occ |= (c ? 1u : 0u) << j;
         }
-        uint32_t inc = sum;
+        // block scans of (counts, occupied buckets) per thread
+        const uint32_t nocc = __popc(occ);
+        uint32_t inc = sum, inco = nocc;
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
             const uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
-            if (lane >= o) inc += y;
+            const uint32_t z = __shfl_up_sync(0xffffffffu, inco, o);
+            if (lane >= o) {
+                inc += y;
+                inco += z;
+            }
         }
-        if (lane == 31) wsum[w] = inc;
+        if (lane == 31) {
+            wsum[w] = inc;
+            wocc[w] = inco;
+        }
         __syncthreads();
-        uint32_t pre = uint32_t(lo);
-        for (int i = 0; i < w; ++i) pre += wsum[i];
-        pre += inc - sum;
-#pragma unroll
-        for (int j = 0; j < kPer; ++j) {
-            cnt[tid * (kPer + 1) + j] = pre;
-            pre += v[j];
+        uint32_t pre = uint32_t(lo), preo = 0, tot_occ = 0;
+        for (int i = 0; i < kFillThreads / 32; ++i) {
+            if (i < w) {
+                pre += wsum[i];
+                preo += wocc[i];
+            }
+            tot_occ += wocc[i];
         }
-        const uint64_t bw = (s0 >> 5) + tid;                     // bitmap word of my 32 buckets
-        if (s0 + uint64_t(tid) * kPer < n_buckets) bitmap[bw] = occ;
+        pre += inc - sum;
+        preo += inco - nocc;
+        // rank of the chunk's first occupied bucket among all occupied buckets
+        if (w == 0) {
+            const unsigned long long r0 = chunk_lookback(status, s_chunk, tot_occ);
+            if (lane == 0) s_rank0 = r0;
+        }
+        __syncthreads();
+        // counts -> ptrs (in place), rank words {occupancy bits, occupied buckets before
+        // this word} and the compact {first slot, count} table, in bucket order
+        const uint64_t rank = s_rank0 + preo;
+        uint64_t r = rank;
+#pragma unroll 4
+        for (int j = 0; j < kPer; ++j) {
+            const uint32_t c = cnt[tid * (kPer + 1) + j];
+            cnt[tid * (kPer + 1) + j] = pre;
+            if (c) buckets[r++] = make_uint2(pre, c);
+            pre += c;
+        }
+        if (s0 + uint64_t(tid) * kPer < n_buckets) rankw[(s0 >> 5) + tid] = (rank << 32) | occ;
         __syncthreads();
         // coalesced write-out of the chunk's ptrs
         const uint64_t lim = n_buckets - s0 < uint64_t(kChunk) ? n_buckets - s0 : uint64_t(kChunk);
         for (int i = tid; i < int(lim); i += kFillThreads) ptrs[s0 + i] = cnt[i + (i >> 5)];
-        if (blockIdx.x == 0 && tid == 0 && s0 == 0) ptrs[n_buckets] = uint32_t(n);
-        __syncthreads();
+        if (s0 == 0 && tid == 0) ptrs[n_buckets] = uint32_t(n);
     }
 }
 
@@ -144,12 +216,21 @@ cudaError_t launch_seed_codes(const uint64_t *R, uint64_t nR, uint32_t ls, uint3
     return cudaGetLastError();
 }
 
+size_t ptrs_fill_scratch_bytes(uint32_t ls) {
+    const uint64_t nb = 1ull << (2 * ls);
+    return ((nb + kChunk - 1) / kChunk) * 8 + 64;
+}
+
 cudaError_t launch_ptrs_fill(const uint32_t *sorted_codes, uint64_t n_locs, uint32_t ls, uint32_t *ptrs,
-                             uint32_t *bitmap, cudaStream_t s) {
+                             unsigned long long *rankw, uint2 *buckets, void *scratch, cudaStream_t s) {
     const uint64_t nb = 1ull << (2 * ls);
     const uint64_t chunks = (nb + kChunk - 1) / kChunk;
-    const int grid = int(chunks < 65535ull ? chunks : 65535ull);
-    k_ptrs_fill<<<grid, kFillThreads, 0, s>>>(sorted_codes, n_locs, nb, ptrs, bitmap);
+    cudaError_t e = cudaMemsetAsync(scratch, 0, ptrs_fill_scratch_bytes(ls), s);
+    if (e != cudaSuccess) return e;
+    auto *status = static_cast<unsigned long long *>(scratch);
+    auto *ticket = reinterpret_cast<unsigned int *>(status + chunks);
+    k_ptrs_fill<<<unsigned(chunks), kFillThreads, 0, s>>>(sorted_codes, n_locs, nb, ptrs, rankw, buckets, status,
+                                                         ticket);
     note_launch();
     return cudaGetLastError();
 }

@@ -13,7 +13,7 @@ struct Options {
     int64_t find_grid = 0;       // 0 = SMs x occupancy
     int64_t find_spill = 64;     // bucket sizes above this go to the heavy queue
     int64_t out_capacity = 0;    // 0 = automatic
-    int64_t use_bitmap = 1;      // probe the occupancy bitmap before ptrs
+    int64_t use_bitmap = 1;      // 1: rank-word probe + compact bucket table; 0: read the dense ptrs
 };
 extern Options g_opt;
 
@@ -50,8 +50,9 @@ size_t radix_scratch_bytes(uint64_t n);
 // Index (index.cu)
 cudaError_t launch_seed_codes(const uint64_t *R, uint64_t nR, uint32_t ls, uint32_t step, uint64_t n_locs,
                               uint32_t *codes, uint32_t *locs, cudaStream_t s);
+size_t ptrs_fill_scratch_bytes(uint32_t ls);
 cudaError_t launch_ptrs_fill(const uint32_t *sorted_codes, uint64_t n_locs, uint32_t ls, uint32_t *ptrs,
-                             uint32_t *bitmap, cudaStream_t s);
+                             unsigned long long *rankw, uint2 *buckets, void *scratch, cudaStream_t s);
 // Seed records for the lookup: rec[k] = {locs[k], 16 bases left of it, 32 bases right of its seed}.
 cudaError_t launch_seed_recs(const uint64_t *R, uint32_t ls, const uint32_t *locs, uint64_t n_locs, uint4 *recs,
                              cudaStream_t s);
@@ -65,7 +66,8 @@ struct FindParams {
     uint64_t nQw;                // allocated words of Q (incl. padding)
     const uint32_t *ptrs;
     const uint4 *recs;           // seed records, parallel to locs: {p, R[p-16,p), R[p+ls,p+ls+32)}
-    const uint32_t *bitmap;
+    const unsigned long long *rankw;  // per 32 seeds: {occupancy bits (low 32), occupied seeds before (high 32)}
+    const uint2 *buckets;        // per occupied seed, in seed order: {first slot in locs, count}
     uint32_t ls, L, step, qbits;
     uint64_t scan_lo, scan_hi;   // query seed positions scanned
     uint64_t own_lo, own_hi;     // MEM start q kept
