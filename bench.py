@@ -197,12 +197,16 @@ def run_ours(args, P):
         merged, local_m = find_mems_sharded(R_dev, Q_dev, P.L, P.ls)
         return merged, local_m
 
+    n_mems, stats = 0, None
     for _ in range(args.warmup):
         flush.zero_()
         merged, lm = step()
-    torch.cuda.synchronize()
-    n_mems = len(merged) if merged is not None else 0
-    stats = lm.stats()
+        torch.cuda.synchronize()
+        n_mems = len(merged) if merged is not None else 0
+        stats = lm.stats()
+        for h in (merged, lm):
+            if h is not None:
+                h.free()
     del merged, lm
 
     gm.profile_enable(True)
@@ -218,13 +222,15 @@ def run_ours(args, P):
             ev[i][0].record(stream)
             merged, lm = step()
             ev[i][1].record(stream)
+            for h in (merged, lm):  # release this step's handles (async frees, stream-ordered)
+                if h is not None:
+                    h.free()
         torch.cuda.synchronize()
     launches = gm.launch_count() - l0
     if world > 1:
         dist.barrier()
     prof = gm.profile_read()
     gm.profile_enable(False)
-    del merged, lm
     step_ms = [a.elapsed_time(b) for a, b in ev]
     tot = torch.tensor([sum(step_ms)], dtype=torch.float64, device=dev)
     if world > 1:

@@ -144,6 +144,11 @@ gpumem_status gpumem_merge_sorted(const gpumem_triple *const *dev_runs, const ui
 /* Release any handle above (seq, index, mems). NULL is a no-op. */
 void gpumem_free(void *handle);
 
+/* Temporaries (find buffers, sort and index scratch) live in a grow-only workspace per
+ * (device, stream) so repeated calls do not allocate. gpumem_trim synchronises those
+ * streams and releases every workspace. Handles are unaffected. */
+gpumem_status gpumem_trim(void);
+
 /* Thread-local text of the last failure ("" if none). */
 const char *gpumem_last_error(void);
 

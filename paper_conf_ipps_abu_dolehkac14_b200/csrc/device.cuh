@@ -33,6 +33,8 @@ __device__ __forceinline__ uint32_t lead_eq(uint64_t x) { return x ? uint32_t(__
 // Number of equal trailing bases of two backward windows (32 if identical).
 __device__ __forceinline__ uint32_t trail_eq(uint64_t x) { return x ? uint32_t(__ffsll(x) - 1) >> 1 : 32u; }
 
+__device__ __forceinline__ int lane_id() { return int(threadIdx.x & 31); }
+
 __device__ __forceinline__ uint32_t lanemask_lt() {
     uint32_t m;
     asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));

@@ -27,6 +27,9 @@
 //  A9      keep len = e + ls + f >= L (:53-56), maximal by construction;
 //  A10     ballot/popc into a per-warp shared buffer, flushed 32+ at a time with
 //          one atomicAdd; writes past `capacity` are counted, not stored.
+// Extensions past the record run per lane up to kLaneCap bases; longer ones (R == Q,
+// long repeats) are queued and finished by k_coop with the whole warp, 1024 bases
+// per step, so no single lane walks a megabase-long match.
 // Compares are 2-bit packed words: XOR, then clz (rightwards) / ffs (leftwards)
 // finds the first mismatching base exactly (reading R11).
 #include "internal.h"
@@ -43,6 +46,8 @@ constexpr uint32_t kGrab = 4;             // chunks per scheduler grab
 constexpr int kQW = kChunk / 32 + 6;      // staged Q words (chunk + left/right halo)
 constexpr uint32_t kSpillHits = 32;       // hits per heavy-queue piece (one per lane)
 constexpr int kOutBuf = 64;
+constexpr uint32_t kUnresolved = 0xffffffffu;
+constexpr uint32_t kLaneCap = 4096;       // bases one lane extends before the warp takes over
 
 struct WarpSmem {
     uint64_t qw[kQW];
@@ -74,31 +79,37 @@ struct Hit {
     uint32_t len;
 };
 
+enum : int { kDrop = 0, kDefer = 1, kEmit = 2 };
+
 // Decide one hit: seed of R at p equals seed of Q at q. rleft = R[p-16, p) (base p-1
 // lowest), rright = R[p+ls, p+ls+32) (first base highest); qleft/qright likewise for Q.
-__device__ __forceinline__ bool decide(const FindParams &P, uint32_t p, uint32_t rleft, uint64_t rright,
-                                       uint32_t q, uint32_t qleft, uint64_t qright, Hit &out) {
+// Extensions beyond the record use global windows, at most kLaneCap bases per lane;
+// a longer one returns kDefer and goes to the coop queue (k_coop).
+__device__ __forceinline__ int decide(const FindParams &P, uint32_t p, uint32_t rleft, uint64_t rright,
+                                      uint32_t q, uint32_t qleft, uint64_t qright, Hit &out) {
     // A7: left extension, capped at step
     const uint32_t lim = min(P.step, min(p, q));
     const uint32_t xl = rleft ^ qleft;
     uint32_t e = xl ? uint32_t(__ffs(int(xl)) - 1) >> 1 : 16u;
     if (e == 16) {
         while (e < lim) {
+            if (e >= kLaneCap) return kDefer;
             const uint32_t run = trail_eq(win_back(P.R, p - e) ^ win_back(P.Q, q - e));
             e += run;
             if (run < 32) break;
         }
     }
     e = min(e, lim);
-    if (e == P.step) return false;                         // not the canonical (leftmost) seed
+    if (e == P.step) return kDrop;                         // not the canonical (leftmost) seed
     const uint32_t qs = q - e;
-    if (qs < P.own_lo || qs >= P.own_hi) return false;     // another shard owns it
+    if (qs < P.own_lo || qs >= P.own_hi) return kDrop;     // another shard owns it
     // A8: right extension from the end of the seed
     const uint32_t a = p + P.ls, b = q + P.ls;
     const uint32_t lim_r = min(uint32_t(P.nR) - a, uint32_t(P.nQ) - b);
     uint32_t f = lead_eq(rright ^ qright);
     if (f == 32) {
         while (f < lim_r) {
+            if (f >= kLaneCap) return kDefer;
             const uint32_t run = lead_eq(win_fwd(P.R, uint64_t(a) + f) ^ win_fwd(P.Q, uint64_t(b) + f));
             f += run;
             if (run < 32) break;
@@ -106,10 +117,128 @@ __device__ __forceinline__ bool decide(const FindParams &P, uint32_t p, uint32_t
     }
     f = min(f, lim_r);
     const uint32_t lam = e + P.ls + f;
-    if (lam < P.L) return false;                           // A9
+    if (lam < P.L) return kDrop;                           // A9
+    out.key = (uint64_t(p - e) << P.qbits) | qs;
+    out.len = lam;
+    return kEmit;
+}
+
+// Warp-cooperative extensions (uniform arguments): lane i compares the i-th 32-base
+// window, 1024 bases per step; the first mismatching window decides.
+__device__ __forceinline__ uint32_t warp_ext_right(const FindParams &P, uint64_t a, uint64_t b, uint32_t f,
+                                                   uint32_t lim) {
+    const int lane = threadIdx.x & 31;
+    while (f < lim) {
+        const uint32_t o = f + 32u * lane;
+        const bool in = o < lim;
+        const uint64_t x = in ? (win_fwd(P.R, a + o) ^ win_fwd(P.Q, b + o)) : 0ull;
+        const unsigned bad = __ballot_sync(0xffffffffu, !in || x != 0);
+        if (bad) {
+            const int first = __ffs(int(bad)) - 1;
+            const uint32_t run = __shfl_sync(0xffffffffu, in ? lead_eq(x) : 0u, first);
+            return min(f + 32u * first + run, lim);
+        }
+        f += 1024;
+    }
+    return min(f, lim);
+}
+
+__device__ __forceinline__ uint32_t warp_ext_left(const FindParams &P, uint64_t a, uint64_t b, uint32_t e,
+                                                  uint32_t lim) {
+    const int lane = threadIdx.x & 31;
+    while (e < lim) {
+        const uint32_t o = e + 32u * lane;
+        const bool in = o < lim;
+        const uint64_t x = in ? (win_back(P.R, a - o) ^ win_back(P.Q, b - o)) : 0ull;
+        const unsigned bad = __ballot_sync(0xffffffffu, !in || x != 0);
+        if (bad) {
+            const int first = __ffs(int(bad)) - 1;
+            const uint32_t run = __shfl_sync(0xffffffffu, in ? trail_eq(x) : 0u, first);
+            return min(e + 32u * first + run, lim);
+        }
+        e += 1024;
+    }
+    return min(e, lim);
+}
+
+// Resolve deferred hits, one per lane (all 32 lanes call it; `valid` marks real ones):
+// the full decision again from global windows, per lane up to kLaneCap bases per
+// direction, longer extensions handed to the whole warp.
+__device__ __forceinline__ bool resolve_deferred(const FindParams &P, bool valid, uint32_t p, uint32_t q,
+                                              uint32_t es, Hit &out) {
+    // ---- left
+    const uint32_t lim = valid ? min(P.step, min(p, q)) : 0u;
+    uint32_t e = 0;
+    bool need = false;
+    if (valid) {
+        if (es == kUnresolved) {
+            e = 0;  // recomputed from the sequences (rare path)
+            const uint32_t cap = min(lim, kLaneCap);
+            bool done = false;
+            while (e < cap) {
+                const uint32_t run = trail_eq(win_back(P.R, p - e) ^ win_back(P.Q, q - e));
+                e += run;
+                if (run < 32) {
+                    done = true;
+                    break;
+                }
+            }
+            need = !done && e < lim;
+        } else {
+            e = es;
+        }
+    }
+    for (unsigned m = __ballot_sync(0xffffffffu, need); m; m &= m - 1) {
+        const int src = __ffs(int(m)) - 1;
+        const uint32_t sp = __shfl_sync(0xffffffffu, p, src), sq = __shfl_sync(0xffffffffu, q, src);
+        const uint32_t se = __shfl_sync(0xffffffffu, e, src), sl = __shfl_sync(0xffffffffu, lim, src);
+        const uint32_t r = warp_ext_left(P, sp, sq, se, sl);
+        if (lane_id() == src) e = r;
+    }
+    e = min(e, lim);
+    bool alive = valid && e != P.step;
+    const uint32_t qs = q - e;
+    alive = alive && qs >= P.own_lo && qs < P.own_hi;
+    // ---- right
+    const uint32_t a = p + P.ls, b = q + P.ls;
+    const uint32_t lim_r = alive ? min(uint32_t(P.nR) - a, uint32_t(P.nQ) - b) : 0u;
+    uint32_t f = 0;
+    need = false;
+    if (alive) {
+        const uint32_t cap = min(lim_r, kLaneCap);
+        bool done = false;
+        while (f < cap) {
+            const uint32_t run = lead_eq(win_fwd(P.R, uint64_t(a) + f) ^ win_fwd(P.Q, uint64_t(b) + f));
+            f += run;
+            if (run < 32) {
+                done = true;
+                break;
+            }
+        }
+        need = !done && f < lim_r;
+    }
+    for (unsigned m = __ballot_sync(0xffffffffu, need); m; m &= m - 1) {
+        const int src = __ffs(int(m)) - 1;
+        const uint32_t sa = __shfl_sync(0xffffffffu, a, src), sb = __shfl_sync(0xffffffffu, b, src);
+        const uint32_t sf = __shfl_sync(0xffffffffu, f, src), sl = __shfl_sync(0xffffffffu, lim_r, src);
+        const uint32_t r = warp_ext_right(P, sa, sb, sf, sl);
+        if (lane_id() == src) f = r;
+    }
+    f = min(f, lim_r);
+    const uint32_t lam = e + P.ls + f;
+    if (!alive || lam < P.L) return false;
     out.key = (uint64_t(p - e) << P.qbits) | qs;
     out.len = lam;
     return true;
+}
+
+// Deferred hits (extension longer than kLaneCap) go to the coop queue, drained by
+// k_coop after the find kernels; rare, so one atomic per hit is fine.
+__device__ __forceinline__ void push_coop(const FindParams &P, int &verdict, uint32_t p, uint32_t q) {
+    if (verdict != kDefer) return;
+    verdict = kDrop;
+    const unsigned long long slot = atomicAdd(P.coop_count, 1ull);
+    if (slot < P.coop_cap) P.coopq[slot] = make_uint2(p, q);
 }
 
 // A10: warp-aggregated append into the warp's buffer; flush when >= 32 are pending.
@@ -271,21 +400,23 @@ __global__ void __launch_bounds__(kT) k_find(const FindParams P) {
                 // ---- A6-A10: hits dealt 32 at a time
                 for (uint32_t hb = 0; hb < H; hb += 32) {
                     const uint32_t h = hb + lane;
-                    bool emit = false;
+                    int verdict = kDrop;
                     Hit out{0, 0};
+                    uint32_t p = 0, q = 0;
                     if (h < H) {
                         uint32_t lo = 0, hi = E;  // largest entry i with e_off[i] <= h
                         while (hi - lo > 1) {
                             const uint32_t mid = (lo + hi) >> 1;
                             if (s.e_off[mid] <= h) lo = mid; else hi = mid;
                         }
-                        const uint32_t q = q0 + s.e_q[lo];
-                        uint32_t p, rl;
+                        q = q0 + s.e_q[lo];
+                        uint32_t rl;
                         uint64_t rr;
                         load_rec(P.recs, s.e_beg[lo] + (h - s.e_off[lo]), p, rl, rr);
-                        emit = decide(P, p, rl, rr, q, qs.back16(q), qs.fwd(q + P.ls), out);
+                        verdict = decide(P, p, rl, rr, q, qs.back16(q), qs.fwd(q + P.ls), out);
                     }
-                    warp_emit(P, s, nbuf, emit, out, false);
+                    push_coop(P, verdict, p, q);
+                    warp_emit(P, s, nbuf, verdict == kEmit, out, false);
                 }
             }
             __syncwarp();
@@ -310,16 +441,40 @@ __global__ void __launch_bounds__(kT) k_heavy(const FindParams P) {
     const unsigned long long nw = (unsigned long long)gridDim.x * kWarps;
     for (unsigned long long c = gw; c < n; c += nw) {
         const uint4 piece = P.spill[c];
-        bool emit = false;
+        int verdict = kDrop;
         Hit out{0, 0};
+        uint32_t p = 0;
+        const uint32_t q = piece.x;
         if (uint32_t(lane) < piece.z) {
-            uint32_t p, rl;
+            uint32_t rl;
             uint64_t rr;
             load_rec(P.recs, piece.y + lane, p, rl, rr);
-            const uint32_t q = piece.x;
-            emit = decide(P, p, rl, rr, q, uint32_t(win_back(P.Q, q)), win_fwd(P.Q, uint64_t(q) + P.ls), out);
+            verdict = decide(P, p, rl, rr, q, uint32_t(win_back(P.Q, q)), win_fwd(P.Q, uint64_t(q) + P.ls), out);
         }
-        warp_emit(P, s, nbuf, emit, out, false);
+        push_coop(P, verdict, p, q);
+        warp_emit(P, s, nbuf, verdict == kEmit, out, false);
+    }
+    warp_emit(P, s, nbuf, false, Hit{0, 0}, true);
+}
+
+// Drain the coop queue: 32 deferred hits per warp iteration, decided from scratch
+// with per-lane extension up to kLaneCap and warp-cooperative extension beyond.
+__global__ void __launch_bounds__(kT) k_coop(const FindParams P) {
+    __shared__ WarpSmem smem[kWarps];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    WarpSmem &s = smem[wid];
+    uint32_t nbuf = 0;
+    const unsigned long long cc = *P.coop_count;
+    const unsigned long long n = cc < P.coop_cap ? cc : P.coop_cap;
+    const unsigned long long gw = (unsigned long long)blockIdx.x * kWarps + wid;
+    const unsigned long long nw = (unsigned long long)gridDim.x * kWarps;
+    for (unsigned long long base = gw * 32; base < n; base += nw * 32) {
+        const unsigned long long i = base + lane;
+        const bool valid = i < n;
+        const uint2 x = valid ? P.coopq[i] : make_uint2(0u, 0u);
+        Hit h{0, 0};
+        const bool em = resolve_deferred(P, valid, x.x, x.y, kUnresolved, h);
+        warp_emit(P, s, nbuf, em, h, false);
     }
     warp_emit(P, s, nbuf, false, Hit{0, 0}, true);
 }
@@ -347,6 +502,12 @@ cudaError_t launch_find(const FindParams &p, int grid, cudaStream_t s) {
     if (uint64_t(grid) * kWarps > max_useful) grid = int((max_useful + kWarps - 1) / kWarps);
     if (grid < 1) grid = 1;
     k_find<<<grid, kT, 0, s>>>(p);
+    note_launch();
+    return cudaGetLastError();
+}
+
+cudaError_t launch_coop(const FindParams &p, cudaStream_t s) {
+    k_coop<<<num_sms() * 2, kT, 0, s>>>(p);
     note_launch();
     return cudaGetLastError();
 }

@@ -229,6 +229,40 @@ gpumem_status check_device(int *dev) {
         if (_e != cudaSuccess) return cuda_fail(_e, what); \
     } while (0)
 
+// Per-(device, stream) grow-only workspace for temporaries: successive calls on one
+// stream are ordered, so a slot can be reused without synchronisation, and the hot
+// loop does no allocation at all once warm. gpumem_trim() releases everything.
+enum WsSlot {
+    kWsCtr, kWsSpill, kWsKeys, kWsLens, kWsSortK, kWsSortL, kWsSortScratch, kWsCodes0, kWsCodes1,
+    kWsRadix, kWsFill, kWsMergeK, kWsMergeL, kWsPackTmp, kWsCoop, kWsCount
+};
+struct Workspace {
+    void *p[kWsCount] = {};
+    size_t sz[kWsCount] = {};
+};
+std::mutex g_ws_mu;
+std::vector<std::pair<std::pair<int, cudaStream_t>, Workspace *>> g_ws;
+
+void *ws_get(int slot, size_t bytes, cudaStream_t s) {
+    int d = 0;
+    cudaGetDevice(&d);
+    std::lock_guard<std::mutex> g(g_ws_mu);
+    Workspace *w = nullptr;
+    for (auto &e : g_ws)
+        if (e.first.first == d && e.first.second == s) w = e.second;
+    if (!w) {
+        w = new Workspace();
+        g_ws.push_back({{d, s}, w});
+    }
+    if (w->sz[slot] < bytes) {
+        if (w->p[slot]) dfree(w->p[slot], s);
+        const size_t want = bytes + bytes / 8 + 4096;
+        w->p[slot] = dalloc(want, s);
+        w->sz[slot] = w->p[slot] ? want : 0;
+    }
+    return w->p[slot];
+}
+
 unsigned long long *pinned_slots() {  // 16 per thread, never freed
     thread_local unsigned long long *p = nullptr;
     if (!p) {
@@ -247,6 +281,24 @@ extern "C" {
 const char *gpumem_version(void) { return GPUMEM_VERSION; }
 
 const char *gpumem_last_error(void) { return t_err.c_str(); }
+
+gpumem_status gpumem_trim(void) {
+    std::lock_guard<std::mutex> g(g_ws_mu);
+    int prev = -1;
+    cudaGetDevice(&prev);
+    for (auto &e : g_ws) {
+        cudaSetDevice(e.first.first);
+        cudaStreamSynchronize(e.first.second);
+        for (int i = 0; i < kWsCount; ++i)
+            if (e.second->p[i]) dfree(e.second->p[i], e.first.second);
+        cudaStreamSynchronize(e.first.second);
+        delete e.second;
+    }
+    g_ws.clear();
+    if (prev >= 0) cudaSetDevice(prev);
+    const cudaError_t err = cudaGetLastError();
+    return err == cudaSuccess ? GPUMEM_OK : cuda_fail(err, "trim");
+}
 
 uint64_t gpumem_launch_count(void) { return g_launches.load(); }
 
@@ -355,7 +407,7 @@ gpumem_status gpumem_pack(const char *bases, uint64_t n, int bases_on_device, vo
     CK(cudaMemsetAsync(bad, 0xff, 8, s), "memset");
     const uint8_t *in = reinterpret_cast<const uint8_t *>(bases);
     if (!bases_on_device && n) {
-        auto *tmp = static_cast<uint8_t *>(sc.get(n));
+        auto *tmp = static_cast<uint8_t *>(ws_get(kWsPackTmp, n, s));
         if (!tmp) return GPUMEM_ERR_NOMEM;
         CK(cudaMemcpyAsync(tmp, bases, n, cudaMemcpyHostToDevice, s), "H2D copy of bases");
         in = tmp;
@@ -410,16 +462,16 @@ gpumem_status gpumem_index_build_step(const gpumem_seq *R, uint32_t ls, uint32_t
     auto *rankw = static_cast<unsigned long long *>(sc.get(((nb + 31) / 32) * 8));
     const uint64_t max_occ = (n_locs < nb ? n_locs : nb) + 1;
     auto *buckets = static_cast<uint2 *>(sc.get(max_occ * sizeof(uint2)));
-    void *fill_scratch = sc.get(ptrs_fill_scratch_bytes(ls));
+    void *fill_scratch = ws_get(kWsFill, ptrs_fill_scratch_bytes(ls), s);
     auto *locs0 = static_cast<uint32_t *>(sc.get((n_locs ? n_locs : 1) * 4));
     if (!ptrs || !rankw || !buckets || !fill_scratch || !locs0) return GPUMEM_ERR_NOMEM;
     uint32_t *locs = locs0;
     const uint32_t *codes_sorted = nullptr;
     if (n_locs) {
-        auto *codes0 = static_cast<uint32_t *>(sc.get(n_locs * 4));
-        auto *codes1 = static_cast<uint32_t *>(sc.get(n_locs * 4));
+        auto *codes0 = static_cast<uint32_t *>(ws_get(kWsCodes0, n_locs * 4, s));
+        auto *codes1 = static_cast<uint32_t *>(ws_get(kWsCodes1, n_locs * 4, s));
         auto *locs1 = static_cast<uint32_t *>(sc.get(n_locs * 4));
-        void *scratch = sc.get(radix_scratch_bytes(n_locs));
+        void *scratch = ws_get(kWsRadix, radix_scratch_bytes(n_locs), s);
         if (!codes0 || !codes1 || !locs1 || !scratch) return GPUMEM_ERR_NOMEM;
         {
             Stage g("index.codes", s);
@@ -480,9 +532,9 @@ static gpumem_status sort_into_triples(uint64_t *keys, uint32_t *lens, uint64_t 
     if (!trip) return GPUMEM_ERR_NOMEM;
     if (n) {
         Stage g("sort", s);
-        auto *k1 = static_cast<uint64_t *>(sc.get(n * 8));
-        auto *l1 = static_cast<uint32_t *>(sc.get(n * 4));
-        void *scratch = sc.get(radix_scratch_bytes(n));
+        auto *k1 = static_cast<uint64_t *>(ws_get(kWsSortK, n * 8, s));
+        auto *l1 = static_cast<uint32_t *>(ws_get(kWsSortL, n * 4, s));
+        void *scratch = ws_get(kWsSortScratch, radix_scratch_bytes(n), s);
         if (!k1 || !l1 || !scratch) return GPUMEM_ERR_NOMEM;
         bool alt = false;
         CK(radix_sort_u64(keys, lens, k1, l1, n, int(key_bits), scratch, s, &alt), "triple sort");
@@ -545,14 +597,16 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
     uint64_t cap = g_opt.out_capacity ? uint64_t(g_opt.out_capacity) : (span / 8 + 4096);
 
     Scratch sc(s);
-    auto *ctr = static_cast<unsigned long long *>(sc.get(64));
+    auto *ctr = static_cast<unsigned long long *>(ws_get(kWsCtr, 64, s));
     const uint64_t spill_cap = span / 8 + 4096;
-    auto *spill = static_cast<uint4 *>(sc.get(spill_cap * sizeof(uint4)));
+    auto *spill = static_cast<uint4 *>(ws_get(kWsSpill, spill_cap * sizeof(uint4), s));
+    uint64_t coop_cap = span / 64 + 4096;
     if (!ctr || !spill) return GPUMEM_ERR_NOMEM;
     P.out_count = ctr;
     P.spill_count = ctr + 1;
     P.tile_ctr = reinterpret_cast<unsigned int *>(ctr + 2);
     P.stats = ctr + 3;
+    P.coop_count = ctr + 7;
     P.spill = spill;
     P.spill_cap = spill_cap;
     unsigned long long *h = pinned_slots();
@@ -563,12 +617,15 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
     uint64_t *keys = nullptr;
     uint32_t *lens = nullptr;
     for (int attempt = 0; attempt < 2; ++attempt) {
-        keys = static_cast<uint64_t *>(sc.get(cap * 8));
-        lens = static_cast<uint32_t *>(sc.get(cap * 4));
+        keys = static_cast<uint64_t *>(ws_get(kWsKeys, cap * 8, s));
+        lens = static_cast<uint32_t *>(ws_get(kWsLens, cap * 4, s));
         if (!keys || !lens) return GPUMEM_ERR_NOMEM;
         P.out_key = keys;
         P.out_len = lens;
         P.capacity = cap;
+        P.coopq = static_cast<uint2 *>(ws_get(kWsCoop, coop_cap * sizeof(uint2), s));
+        P.coop_cap = coop_cap;
+        if (!P.coopq) return GPUMEM_ERR_NOMEM;
         CK(cudaMemsetAsync(ctr, 0, 64, s), "memset counters");
         {
             Stage g("find", s);
@@ -577,6 +634,7 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
         if (P.n_tiles) {
             Stage g("find.heavy", s);
             CK(launch_heavy(P, s), "heavy kernel");
+            CK(launch_coop(P, s), "coop kernel");
         }
         ++attempts;
         CK(cudaMemcpyAsync(h, ctr, 64, cudaMemcpyDeviceToHost, s), "D2H counters");
@@ -586,10 +644,11 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
         if (h[8] != ~0ull) return fail(GPUMEM_ERR_ALPHABET, "R: byte at position %llu is not in {A,C,G,T,a,c,g,t}", h[8]);
         if (h[9] != ~0ull) return fail(GPUMEM_ERR_ALPHABET, "Q: byte at position %llu is not in {A,C,G,T,a,c,g,t}", h[9]);
         count = h[0];
-        if (count <= cap) break;
+        if (count <= cap && h[7] <= coop_cap) break;
         if (attempt == 1) return fail(GPUMEM_ERR_CUDA, "output count changed between runs (%llu > %llu)",
                                       (unsigned long long)count, (unsigned long long)cap);
-        cap = count;  // overflow: rerun with the exact capacity
+        if (count > cap) cap = count;            // overflow: rerun with the exact capacity
+        if (h[7] > coop_cap) coop_cap = h[7];    // coop queue overflow: likewise
     }
     gpumem_find_stats fs{};
     fs.positions = span;
@@ -644,8 +703,8 @@ gpumem_status gpumem_merge_sorted(const gpumem_triple *const *dev_runs, const ui
     uint64_t total = 0;
     for (int i = 0; i < n_runs; ++i) total += counts[i];
     Scratch sc(s);
-    auto *keys = static_cast<uint64_t *>(sc.get((total ? total : 1) * 8));
-    auto *lens = static_cast<uint32_t *>(sc.get((total ? total : 1) * 4));
+    auto *keys = static_cast<uint64_t *>(ws_get(kWsMergeK, (total ? total : 1) * 8, s));
+    auto *lens = static_cast<uint32_t *>(ws_get(kWsMergeL, (total ? total : 1) * 4, s));
     if (!keys || !lens) return GPUMEM_ERR_NOMEM;
     {
         Stage g("merge", s);

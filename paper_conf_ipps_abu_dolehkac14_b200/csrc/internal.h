@@ -82,11 +82,15 @@ struct FindParams {
     uint64_t spill_cap;
     unsigned long long *spill_count;
     unsigned long long *stats;   // [0] entries kept local, [1] hits kept local, [2] hits spilled, [3] entries spilled
+    uint2 *coopq;                // hits whose extension exceeds kLaneCap: {p, q}
+    uint64_t coop_cap;
+    unsigned long long *coop_count;
     int use_bitmap;
 };
 uint64_t find_tile_positions();
 cudaError_t launch_find(const FindParams &p, int grid, cudaStream_t s);
 cudaError_t launch_heavy(const FindParams &p, cudaStream_t s);
+cudaError_t launch_coop(const FindParams &p, cudaStream_t s);
 int find_default_grid();
 
 // Triples (sort.cu)

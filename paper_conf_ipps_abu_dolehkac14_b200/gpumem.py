@@ -44,6 +44,7 @@ SYMBOLS = {
     "gpumem_mems_stats": (ctypes.c_int, [_vp, _vp]),
     "gpumem_merge_sorted": (ctypes.c_int, [_P(_vp), _P(_c_u64), ctypes.c_int, _vp, _P(_vp)]),
     "gpumem_free": (None, [_vp]),
+    "gpumem_trim": (ctypes.c_int, []),
     "gpumem_last_error": (ctypes.c_char_p, []),
     "gpumem_set_allocator": (ctypes.c_int, [_vp, _vp, _vp]),
     "gpumem_set_option": (ctypes.c_int, [ctypes.c_char_p, ctypes.c_int64]),
@@ -258,6 +259,11 @@ def profile_read(max_stages=32):
     nl = (_c_u64 * max_stages)()
     n = _lib.gpumem_profile_read(names, ms, nl, max_stages)
     return {names[i].decode(): (ms[i], nl[i]) for i in range(n)}
+
+
+def trim():
+    """Release the library's per-stream workspaces (synchronises those streams)."""
+    _check(_lib.gpumem_trim())
 
 
 def launch_count() -> int:
