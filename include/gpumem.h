@@ -75,6 +75,13 @@ typedef struct {
 gpumem_status gpumem_pack(const char *bases, uint64_t n, int bases_on_device,
                           void *cuda_stream, gpumem_seq **out);
 
+/* Reverse complement of a packed sequence (NEXT-F4; the paper's problem is forward-only,
+ * reading R17): base i of the result is the complement of base n-1-i (A<->T, C<->G).
+ * MEMs on the reverse strand are gpumem_find_mems(idx, revcomp(Q)); their q is a position
+ * in the reverse-complemented query (the forward-strand interval is [|Q|-q-len, |Q|-q)).
+ * The alphabet verdict of the input is carried over. Async. */
+gpumem_status gpumem_revcomp(const gpumem_seq *in, void *cuda_stream, gpumem_seq **out);
+
 /* Synchronises `cuda_stream`; GPUMEM_ERR_ALPHABET (with the first bad position in the
  * message) if the packed input held a byte outside the alphabet, else GPUMEM_OK. */
 gpumem_status gpumem_seq_check(const gpumem_seq *s, void *cuda_stream);
@@ -98,6 +105,19 @@ gpumem_status gpumem_index_build(const gpumem_seq *R, uint32_t seed_len, uint32_
 /* Test-only: same with an explicit step in [1, L - ls + 1] (the MEM set does not depend on it). */
 gpumem_status gpumem_index_build_step(const gpumem_seq *R, uint32_t seed_len, uint32_t min_len,
                                       uint32_t step, void *cuda_stream, gpumem_index **out);
+
+/*
+ * gpumem_index_build_range -- partial index of one band of R (the paper's tile-row
+ *  index: "only a partial index is created for l_tile base pairs of
+ *  reference"): only sampled locations p with r_begin <= p < r_end are indexed (same
+ *  stride, same phase as the whole index, reading R6). Extensions still read the whole
+ *  of R, so gpumem_find_mems on a band index returns exactly the MEMs whose canonical
+ *  (leftmost sampled) seed lies in the band; the bands of a partition of [0, |R|) give
+ *  disjoint MEM sets whose union is the whole set. r_begin > r_end -> GPUMEM_ERR_RANGE.
+ */
+gpumem_status gpumem_index_build_range(const gpumem_seq *R, uint32_t seed_len, uint32_t min_len,
+                                       uint64_t r_begin, uint64_t r_end, void *cuda_stream,
+                                       gpumem_index **out);
 
 /* Borrowed device pointers to ptrs (4^ls + 1 entries) and locs (n_locs entries). */
 gpumem_status gpumem_index_view(const gpumem_index *idx, const uint32_t **dev_ptrs,
@@ -126,6 +146,15 @@ typedef struct {
     uint32_t attempts;       /* 1, or 2 after an output-capacity overflow                     */
 } gpumem_find_stats;
 gpumem_status gpumem_mems_stats(const gpumem_mems *m, gpumem_find_stats *out);
+
+/*
+ * gpumem_mums -- maximal unique matches (NEXT-F3; PAPER.md:23 defines a MUM, :286 lists
+ *  it as future work): the MEMs of `m` whose string occurs exactly once in R and once in
+ *  Q (reading R21), in the same (r, q) order. `m` must be a complete MEM set of
+ *  (R, Q, L) (a q-range or band subset is not enough to decide uniqueness).
+ *  Synchronises once (the result size is data-dependent).
+ */
+gpumem_status gpumem_mums(const gpumem_mems *m, void *cuda_stream, gpumem_mems **out);
 
 /* Borrowed device pointer to the sorted triples and their count. */
 gpumem_status gpumem_mems_view(const gpumem_mems *m, const gpumem_triple **dev_ptr, uint64_t *count);

@@ -10,6 +10,7 @@ shared module and holds no method arithmetic).
                              C++ oracle O1 (mem_oracle.cpp: oracle_mems)
   brute(R, Q, L)          -> same, by the O(|R||Q|) definition (brute_mems)
   index(R, ls, step)      -> (ptrs, locs) by Algorithm 1 (oracle_index)
+  mums(R, Q, L, ls)       -> MUMs: MEMs unique in both sequences (oracle_mums)
   pyoracle                -> pure-Python twins for tiny inputs
 
 See mem_oracle.cpp's header for the PAPER.md passages each function follows
@@ -59,6 +60,9 @@ def _load():
             lib.oracle_index.argtypes = [ctypes.c_char_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_uint32,
                                          P(ctypes.c_uint32), P(ctypes.c_uint32)]
             lib.oracle_index.restype = ctypes.c_int64
+            lib.oracle_mums.argtypes = [ctypes.c_char_p, ctypes.c_uint64, ctypes.c_char_p, ctypes.c_uint64,
+                                        ctypes.c_uint32, ctypes.c_uint32, ctypes.c_int, u32pp]
+            lib.oracle_mums.restype = ctypes.c_int64
             lib.oracle_free.argtypes = [ctypes.c_void_p]
             lib.oracle_num_threads.argtypes = [ctypes.c_int]
             lib.oracle_num_threads.restype = ctypes.c_int
@@ -115,6 +119,15 @@ def brute(R, Q, L, threads=0):
     Rb, Qb = _bytes(R), _bytes(Q)
     out = ctypes.POINTER(ctypes.c_uint32)()
     n = lib.brute_mems(Rb, len(Rb), Qb, len(Qb), int(L), int(threads), ctypes.byref(out))
+    return _take(n, out)
+
+
+def mums(R, Q, L, ls, threads=0):
+    """MUMs: MEMs whose string occurs exactly once in R and once in Q (oracle_mums)."""
+    lib = _load()
+    Rb, Qb = _bytes(R), _bytes(Q)
+    out = ctypes.POINTER(ctypes.c_uint32)()
+    n = lib.oracle_mums(Rb, len(Rb), Qb, len(Qb), int(L), int(ls), int(threads), ctypes.byref(out))
     return _take(n, out)
 
 

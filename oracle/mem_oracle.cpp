@@ -243,3 +243,32 @@ int64_t oracle_index(const char* Rs, uint64_t nR, uint32_t ls, uint32_t step,
 }
 
 }  // extern "C"
+
+// MUMs (a match that "appears only once in both sequences ... and cannot be
+// extended to either directions"): the MEMs of oracle_mems whose string occurs exactly
+// once in R and exactly once in Q, counted by plain substring search (std::string::find,
+// overlapping occurrences). Pinned by the hand-worked W2 MUM fixture and the Python twin.
+extern "C" int64_t oracle_mums(const char* Rs, uint64_t nR, const char* Qs, uint64_t nQ, uint32_t L,
+                               uint32_t ls, int threads, uint32_t** out) {
+    uint32_t* mem = nullptr;
+    const int64_t n = oracle_mems(Rs, nR, Qs, nQ, L, ls, 0, 0, nQ, threads, &mem);
+    *out = nullptr;
+    if (n < 0) return n;
+    std::string R, Q;
+    normalise(Rs, nR, R);
+    normalise(Qs, nQ, Q);
+    auto occurs_once = [](const std::string& T, const std::string& S) {
+        size_t pos = T.find(S);
+        if (pos == std::string::npos) return false;
+        return T.find(S, pos + 1) == std::string::npos;
+    };
+    std::vector<Triple> keep;
+    for (int64_t i = 0; i < n; ++i) {
+        const Triple t{mem[3 * i], mem[3 * i + 1], mem[3 * i + 2]};
+        const std::string S = R.substr(t.r, t.len);
+        if (occurs_once(R, S) && occurs_once(Q, S)) keep.push_back(t);
+    }
+    std::free(mem);
+    *out = export_triples(keep);
+    return *out ? int64_t(keep.size()) : -3;
+}

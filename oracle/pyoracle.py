@@ -67,3 +67,13 @@ def homopolymer(n, m, L):
     out = {(0, q, min(n, m - q)) for q in range(m)}
     out |= {(r, 0, min(n - r, m)) for r in range(1, n)}
     return sorted(t for t in out if t[2] >= L and t[2] > 0)
+
+
+def mums(R, Q, L):
+    """MEMs (by the definition) whose string occurs exactly once in R and in Q."""
+    R, Q = _s(R), _s(Q)
+
+    def count(T, S):
+        return sum(1 for i in range(len(T) - len(S) + 1) if T[i:i + len(S)] == S)
+
+    return [t for t in brute(R, Q, L) if count(R, R[t[0]:t[0] + t[2]]) == 1 and count(Q, R[t[0]:t[0] + t[2]]) == 1]

@@ -234,7 +234,7 @@ gpumem_status check_device(int *dev) {
 // loop does no allocation at all once warm. gpumem_trim() releases everything.
 enum WsSlot {
     kWsCtr, kWsSpill, kWsKeys, kWsLens, kWsSortK, kWsSortL, kWsSortScratch, kWsCodes0, kWsCodes1,
-    kWsRadix, kWsFill, kWsMergeK, kWsMergeL, kWsPackTmp, kWsCoop, kWsCount
+    kWsRadix, kWsFill, kWsMergeK, kWsMergeL, kWsPackTmp, kWsCoop, kWsMums, kWsCount
 };
 struct Workspace {
     void *p[kWsCount] = {};
@@ -420,6 +420,27 @@ gpumem_status gpumem_pack(const char *bases, uint64_t n, int bases_on_device, vo
     return GPUMEM_OK;
 }
 
+gpumem_status gpumem_revcomp(const gpumem_seq *in, void *cuda_stream, gpumem_seq **out) {
+    if (!out) return fail(GPUMEM_ERR_ARG, "out is NULL");
+    *out = nullptr;
+    if (!in || in->magic != kMagicSeq) return fail(GPUMEM_ERR_ARG, "not a gpumem_seq");
+    int dev;
+    gpumem_status st = check_device(&dev);
+    if (st) return st;
+    cudaStream_t s = static_cast<cudaStream_t>(cuda_stream);
+    Stage stage("revcomp", s);
+    Scratch sc(s);
+    auto *words = static_cast<uint64_t *>(sc.get(in->n_words * 8));
+    auto *bad = static_cast<unsigned long long *>(sc.get(8));
+    if (!words || !bad) return GPUMEM_ERR_NOMEM;
+    CK(cudaMemcpyAsync(bad, in->bad, 8, cudaMemcpyDeviceToDevice, s), "copy flag");
+    CK(launch_revcomp(in->words, in->n, words, in->n_words, s), "revcomp kernel");
+    sc.keep(words);
+    sc.keep(bad);
+    *out = new gpumem_seq{kMagicSeq, dev, s, in->n, in->n_words, words, bad};
+    return GPUMEM_OK;
+}
+
 gpumem_status gpumem_seq_check(const gpumem_seq *sq, void *cuda_stream) {
     if (!sq || sq->magic != kMagicSeq) return fail(GPUMEM_ERR_ARG, "not a gpumem_seq");
     cudaStream_t s = static_cast<cudaStream_t>(cuda_stream);
@@ -441,8 +462,25 @@ gpumem_status gpumem_seq_info(const gpumem_seq *sq, uint64_t *n_bases, const uin
     return GPUMEM_OK;
 }
 
+static gpumem_status index_build_impl(const gpumem_seq *R, uint32_t ls, uint32_t L, uint32_t step,
+                                      uint64_t r_begin, uint64_t r_end, void *cuda_stream, gpumem_index **out);
+
 gpumem_status gpumem_index_build_step(const gpumem_seq *R, uint32_t ls, uint32_t L, uint32_t step,
                                       void *cuda_stream, gpumem_index **out) {
+    return index_build_impl(R, ls, L, step, 0, UINT64_MAX, cuda_stream, out);
+}
+
+gpumem_status gpumem_index_build_range(const gpumem_seq *R, uint32_t ls, uint32_t L, uint64_t r_begin,
+                                       uint64_t r_end, void *cuda_stream, gpumem_index **out) {
+    if (ls < 1 || ls > 15 || L < ls) {
+        if (out) *out = nullptr;
+        return fail(GPUMEM_ERR_ARG, "need 1 <= seed_len <= 15 and seed_len <= min_len (got %u, %u)", ls, L);
+    }
+    return index_build_impl(R, ls, L, L - ls + 1, r_begin, r_end, cuda_stream, out);
+}
+
+static gpumem_status index_build_impl(const gpumem_seq *R, uint32_t ls, uint32_t L, uint32_t step,
+                                      uint64_t r_begin, uint64_t r_end, void *cuda_stream, gpumem_index **out) {
     if (!out) return fail(GPUMEM_ERR_ARG, "out is NULL");
     *out = nullptr;
     if (!R || R->magic != kMagicSeq) return fail(GPUMEM_ERR_ARG, "R is not a gpumem_seq");
@@ -456,7 +494,13 @@ gpumem_status gpumem_index_build_step(const gpumem_seq *R, uint32_t ls, uint32_t
     if (dev != R->device) return fail(GPUMEM_ERR_ARG, "R lives on device %d, current is %d", R->device, dev);
     cudaStream_t s = static_cast<cudaStream_t>(cuda_stream);
     const uint64_t nb = 1ull << (2 * ls);
-    const uint64_t n_locs = R->n >= ls ? (R->n - ls) / step + 1 : 0;
+    // sampled locations p = k * step with r_begin <= p < r_end and p <= |R| - ls
+    if (r_begin > r_end) return fail(GPUMEM_ERR_RANGE, "r_begin > r_end");
+    const uint64_t k_all = R->n >= ls ? (R->n - ls) / step + 1 : 0;
+    const uint64_t k0 = (r_begin + step - 1) / step;
+    const uint64_t k1_band = r_end >= UINT64_MAX - step ? UINT64_MAX : (r_end + step - 1) / step;
+    const uint64_t k1 = k1_band < k_all ? k1_band : k_all;
+    const uint64_t n_locs = k1 > k0 ? k1 - k0 : 0;
     Scratch sc(s);
     auto *ptrs = static_cast<uint32_t *>(sc.get((nb + 1) * 4));
     auto *rankw = static_cast<unsigned long long *>(sc.get(((nb + 31) / 32) * 8));
@@ -475,7 +519,7 @@ gpumem_status gpumem_index_build_step(const gpumem_seq *R, uint32_t ls, uint32_t
         if (!codes0 || !codes1 || !locs1 || !scratch) return GPUMEM_ERR_NOMEM;
         {
             Stage g("index.codes", s);
-            CK(launch_seed_codes(R->words, R->n, ls, step, n_locs, codes0, locs0, s), "seed codes");
+            CK(launch_seed_codes(R->words, ls, step, k0, n_locs, codes0, locs0, s), "seed codes");
         }
         bool alt = false;
         {
@@ -663,6 +707,30 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
         (*out)->stats = fs;
     }
     return st2;
+}
+
+gpumem_status gpumem_mums(const gpumem_mems *m, void *cuda_stream, gpumem_mems **out) {
+    if (!out) return fail(GPUMEM_ERR_ARG, "out is NULL");
+    *out = nullptr;
+    if (!m || m->magic != kMagicMems) return fail(GPUMEM_ERR_ARG, "not a gpumem_mems");
+    int dev;
+    gpumem_status st = check_device(&dev);
+    if (st) return st;
+    cudaStream_t s = static_cast<cudaStream_t>(cuda_stream);
+    Stage g("mums", s);
+    Scratch sc(s);
+    auto *res = static_cast<gpumem_triple *>(sc.get((m->count ? m->count : 1) * sizeof(gpumem_triple)));
+    void *scratch = ws_get(kWsMums, mum_scratch_bytes(m->count), s);
+    auto *dcount = static_cast<unsigned long long *>(ws_get(kWsCtr, 64, s));
+    unsigned long long *h = pinned_slots();
+    if (!res || !scratch || !dcount || !h) return GPUMEM_ERR_NOMEM;
+    CK(mum_filter(m->dev, m->count, res, dcount, scratch, s), "MUM filter");
+    CK(cudaMemcpyAsync(h, dcount, 8, cudaMemcpyDeviceToHost, s), "D2H count");
+    CK(cudaStreamSynchronize(s), "sync");
+    sc.keep(res);
+    *out = new gpumem_mems{kMagicMems, dev, s, h[0], res, m->stats};
+    (*out)->stats.mems = h[0];
+    return GPUMEM_OK;
 }
 
 gpumem_status gpumem_mems_view(const gpumem_mems *m, const gpumem_triple **dev_ptr, uint64_t *count) {

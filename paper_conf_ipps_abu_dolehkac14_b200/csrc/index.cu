@@ -36,12 +36,12 @@ constexpr int kChunk = 8192;                    // buckets per CTA in k_ptrs_fil
 constexpr int kPer = kChunk / kFillThreads;     // 32 consecutive buckets per thread
 
 __global__ void __launch_bounds__(kCodeThreads) k_seed_codes(const uint64_t *__restrict__ R, uint32_t ls,
-                                                             uint32_t step, uint64_t n_locs,
+                                                             uint32_t step, uint64_t k0, uint64_t n_locs,
                                                              uint32_t *__restrict__ codes,
                                                              uint32_t *__restrict__ locs) {
     const uint64_t k = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
     if (k >= n_locs) return;
-    const uint64_t p = k * step;
+    const uint64_t p = (k0 + k) * step;
     codes[k] = uint32_t(win_fwd(R, p) >> (64 - 2 * ls));
     locs[k] = uint32_t(p);
 }
@@ -206,12 +206,11 @@ cudaError_t launch_seed_recs(const uint64_t *R, uint32_t ls, const uint32_t *loc
     return cudaGetLastError();
 }
 
-cudaError_t launch_seed_codes(const uint64_t *R, uint64_t nR, uint32_t ls, uint32_t step, uint64_t n_locs,
+cudaError_t launch_seed_codes(const uint64_t *R, uint32_t ls, uint32_t step, uint64_t k0, uint64_t n_locs,
                               uint32_t *codes, uint32_t *locs, cudaStream_t s) {
-    (void)nR;
     if (n_locs == 0) return cudaSuccess;
     const uint64_t blocks = (n_locs + kCodeThreads - 1) / kCodeThreads;
-    k_seed_codes<<<unsigned(blocks), kCodeThreads, 0, s>>>(R, ls, step, n_locs, codes, locs);
+    k_seed_codes<<<unsigned(blocks), kCodeThreads, 0, s>>>(R, ls, step, k0, n_locs, codes, locs);
     note_launch();
     return cudaGetLastError();
 }

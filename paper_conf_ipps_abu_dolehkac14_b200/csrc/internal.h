@@ -38,6 +38,9 @@ struct Stage {
 cudaError_t launch_pack(const uint8_t *in, uint64_t n, uint64_t *words, uint64_t n_words_alloc,
                         unsigned long long *bad_pos, cudaStream_t s);
 
+// Reverse complement of packed words (pack.cu).
+cudaError_t launch_revcomp(const uint64_t *in, uint64_t n, uint64_t *out, uint64_t n_words_alloc, cudaStream_t s);
+
 // Radix sort (radix.cu): stable LSD on the low `bits` bits of the keys, values ride along.
 // Ping-pongs between (k0,v0) and (k1,v1); returns true when the result is in (k1,v1).
 // `scratch` must hold radix_scratch_bytes(n) bytes (digit counts + scan partials).
@@ -48,7 +51,8 @@ cudaError_t radix_sort_u64(uint64_t *k0, uint32_t *v0, uint64_t *k1, uint32_t *v
 size_t radix_scratch_bytes(uint64_t n);
 
 // Index (index.cu)
-cudaError_t launch_seed_codes(const uint64_t *R, uint64_t nR, uint32_t ls, uint32_t step, uint64_t n_locs,
+// sampled locations p = (k0 + k) * step for k in [0, n_locs)
+cudaError_t launch_seed_codes(const uint64_t *R, uint32_t ls, uint32_t step, uint64_t k0, uint64_t n_locs,
                               uint32_t *codes, uint32_t *locs, cudaStream_t s);
 size_t ptrs_fill_scratch_bytes(uint32_t ls);
 cudaError_t launch_ptrs_fill(const uint32_t *sorted_codes, uint64_t n_locs, uint32_t ls, uint32_t *ptrs,
@@ -92,6 +96,12 @@ cudaError_t launch_find(const FindParams &p, int grid, cudaStream_t s);
 cudaError_t launch_heavy(const FindParams &p, cudaStream_t s);
 cudaError_t launch_coop(const FindParams &p, cudaStream_t s);
 int find_default_grid();
+
+// MUM filter (variants.cu): the MEMs whose string is unique in R and in Q, order kept;
+// the kept count is written to *d_count (device).
+size_t mum_scratch_bytes(uint64_t n);
+cudaError_t mum_filter(const gpumem_triple *in, uint64_t n, gpumem_triple *out, unsigned long long *d_count,
+                       void *scratch, cudaStream_t s);
 
 // Triples (sort.cu)
 cudaError_t launch_keys_to_triples(const uint64_t *keys, const uint32_t *lens, uint64_t n, uint32_t qbits,

@@ -64,7 +64,43 @@ __global__ void __launch_bounds__(kPackThreads) k_pack(const uint8_t *__restrict
     words[w] = word;
 }
 
+// Reverse complement of a packed sequence (NEXT-F4): rc[i] = 3 - s[n-1-i] (A<->T, C<->G
+// is XOR 3 in the A0 C1 G2 T3 code). Output word w holds rc bases [32w, 32w+32): the
+// 32 bases of s ending at n - 32w, reversed pairwise, complemented, tail kept 00.
+__global__ void __launch_bounds__(kPackThreads) k_revcomp(const uint64_t *__restrict__ in, uint64_t n,
+                                                          uint64_t *__restrict__ out, uint64_t n_words_alloc) {
+    const uint64_t w = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+    if (w >= n_words_alloc) return;
+    const uint64_t first = w * 32;
+    if (first >= n) {
+        out[w] = 0;
+        return;
+    }
+    const uint64_t end = n - first;  // s bases [end-32, end) -> rc bases [first, first+32)
+    uint64_t x;
+    if (end >= 32) {
+        const uint64_t a = end - 32, wi = a >> 5;
+        const uint32_t sh = uint32_t(a & 31) * 2;
+        x = sh ? (in[wi] << sh) | (in[wi + 1] >> (64 - sh)) : in[wi];
+    } else {
+        x = in[0] >> (64 - 2 * end);  // s bases [0, end) in the low bits
+    }
+    uint64_t y = __brevll(x);                                                  // bit order reversed
+    y = ((y >> 1) & 0x5555555555555555ull) | ((y & 0x5555555555555555ull) << 1);  // fix pairs
+    y = ~y;                                                                    // complement (XOR 3)
+    const uint64_t valid = end >= 32 ? 32 : end;
+    if (valid < 32) y &= ~0ull << (64 - 2 * valid);                            // padding stays 00
+    out[w] = y;
+}
+
 }  // namespace
+
+cudaError_t launch_revcomp(const uint64_t *in, uint64_t n, uint64_t *out, uint64_t n_words_alloc, cudaStream_t s) {
+    const uint64_t blocks = (n_words_alloc + kPackThreads - 1) / kPackThreads;
+    k_revcomp<<<unsigned(blocks), kPackThreads, 0, s>>>(in, n, out, n_words_alloc);
+    note_launch();
+    return cudaGetLastError();
+}
 
 cudaError_t launch_pack(const uint8_t *in, uint64_t n, uint64_t *words, uint64_t n_words_alloc,
                         unsigned long long *bad_pos, cudaStream_t s) {

@@ -34,14 +34,17 @@ SYMBOLS = {
     # name: (restype, argtypes)
     "gpumem_pack": (ctypes.c_int, [ctypes.c_void_p, _c_u64, ctypes.c_int, _vp, _P(_vp)]),
     "gpumem_seq_check": (ctypes.c_int, [_vp, _vp]),
+    "gpumem_revcomp": (ctypes.c_int, [_vp, _vp, _P(_vp)]),
     "gpumem_seq_info": (ctypes.c_int, [_vp, _P(_c_u64), _P(_vp), _P(_c_u64)]),
     "gpumem_index_build": (ctypes.c_int, [_vp, _c_u32, _c_u32, _vp, _P(_vp)]),
     "gpumem_index_build_step": (ctypes.c_int, [_vp, _c_u32, _c_u32, _c_u32, _vp, _P(_vp)]),
+    "gpumem_index_build_range": (ctypes.c_int, [_vp, _c_u32, _c_u32, _c_u64, _c_u64, _vp, _P(_vp)]),
     "gpumem_index_view": (ctypes.c_int, [_vp, _P(_vp), _P(_vp), _P(_c_u64)]),
     "gpumem_find_mems": (ctypes.c_int, [_vp, _vp, _c_u64, _c_u64, _vp, _P(_vp)]),
     "gpumem_mems_view": (ctypes.c_int, [_vp, _P(_vp), _P(_c_u64)]),
     "gpumem_mems_to_host": (ctypes.c_int, [_vp, _vp, _c_u64]),
     "gpumem_mems_stats": (ctypes.c_int, [_vp, _vp]),
+    "gpumem_mums": (ctypes.c_int, [_vp, _vp, _P(_vp)]),
     "gpumem_merge_sorted": (ctypes.c_int, [_P(_vp), _P(_c_u64), ctypes.c_int, _vp, _P(_vp)]),
     "gpumem_free": (None, [_vp]),
     "gpumem_trim": (ctypes.c_int, []),
@@ -220,9 +223,23 @@ def pack(x, stream=None) -> Seq:
     return Seq(h.value, keep)
 
 
-def index_build(R: Seq, seed_len: int, min_len: int, step: int | None = None, stream=None) -> Index:
+def revcomp(S: Seq, stream=None) -> Seq:
+    """Packed reverse complement of S (for reverse-strand MEMs)."""
     h = _vp()
-    if step is None:
+    _check(_lib.gpumem_revcomp(S.handle, _stream(stream), ctypes.byref(h)))
+    return Seq(h.value, S)
+
+
+def index_build(R: Seq, seed_len: int, min_len: int, step: int | None = None, stream=None,
+                r_range=None) -> Index:
+    """Index of R (Alg. 1). r_range=(r_begin, r_end) builds the partial index of one band."""
+    h = _vp()
+    if r_range is not None:
+        if step is not None:
+            raise ValueError("step and r_range are exclusive")
+        _check(_lib.gpumem_index_build_range(R.handle, seed_len, min_len, int(r_range[0]), int(r_range[1]),
+                                             _stream(stream), ctypes.byref(h)))
+    elif step is None:
         _check(_lib.gpumem_index_build(R.handle, seed_len, min_len, _stream(stream), ctypes.byref(h)))
     else:
         _check(_lib.gpumem_index_build_step(R.handle, seed_len, min_len, step, _stream(stream), ctypes.byref(h)))
@@ -234,6 +251,13 @@ def find_mems(idx: Index, Q: Seq, q_range=None, stream=None) -> Mems:
     h = _vp()
     _check(_lib.gpumem_find_mems(idx.handle, Q.handle, qb, qe, _stream(stream), ctypes.byref(h)))
     return Mems(h.value, (idx, Q))
+
+
+def mums(m: Mems, stream=None) -> Mems:
+    """Maximal unique matches: the MEMs of `m` unique in both sequences (order kept)."""
+    h = _vp()
+    _check(_lib.gpumem_mums(m.handle, _stream(stream), ctypes.byref(h)))
+    return Mems(h.value, m)
 
 
 def merge_sorted(runs, stream=None) -> Mems:

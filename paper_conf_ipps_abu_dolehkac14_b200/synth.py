@@ -213,9 +213,9 @@ def make_c3(scale=1.0, seed=3):
     fam_b = random_symbols(rng, 6000, 0.41)
     overwrite_copies(rng, R, fam_a, _sc(5000, scale), 0.12)
     overwrite_copies(rng, R, fam_b, _sc(300, scale), 0.08)
-    segmental_dups(rng, R, _sc(200, scale), 10_000, 100_000 if n > 1_000_000 else 2_000, 0.01, 0.04)
+    segmental_dups(rng, R, _sc(200, scale), 10_000 if n > 1_000_000 else 500, 100_000 if n > 1_000_000 else 2_000, 0.01, 0.04)
     Q = mutate(rng, R, 0.01, 0.001)
-    segmental_dups(rng, Q, _sc(50, scale), 10_000, 100_000 if n > 1_000_000 else 2_000, 0.01, 0.04)
+    segmental_dups(rng, Q, _sc(50, scale), 10_000 if n > 1_000_000 else 500, 100_000 if n > 1_000_000 else 2_000, 0.01, 0.04)
     return R, Q, [], dict(n=n, gc=0.41, fam=[(300, 5000, 0.12), (6000, 300, 0.08)], sd=200, snp=0.01,
                           indel=0.001, q_sd=50)
 

@@ -51,7 +51,8 @@ def test_library_holds_sm100a_code(lib_path):
     assert "sm_100a" in out
     sass = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "-sass", lib_path], capture_output=True,
                           text=True).stdout
-    for k in ("k_pack", "k_find", "k_heavy", "k_seed_codes", "k_ptrs_fill", "k_scatter", "k_hist"):
+    for k in ("k_pack", "k_find", "k_heavy", "k_coop", "k_seed_codes", "k_ptrs_fill", "k_seed_recs",
+              "k_onesweep", "k_hist_all", "k_revcomp", "k_contained"):
         assert k in sass, k
 
 

@@ -268,6 +268,69 @@ def test_full_size_c4_c5(c4_full, L):
     assert np.array_equal(got, want)
 
 
+# ------------------------------------------------------------------ NEXT rows
+def _rc(b):
+    return bytes(b)[::-1].translate(bytes.maketrans(b"ACGTacgt", b"TGCAtgca"))
+
+
+@pytest.mark.parametrize("cfg,scale,bands", [("c1", 1.0, 3), ("c2", 0.1, 5), ("c4", 0.02, 7)])
+def test_band_index_union_is_whole(cfg, scale, bands):
+    """F2: partial index per band of R: bands partition the MEM set."""
+    P = synth.make_pair(cfg, scale=scale)
+    Rs, Qs = gpumem.pack(P.R), gpumem.pack(P.Q)
+    whole = gpumem.find_mems(gpumem.index_build(Rs, P.ls, P.L), Qs).numpy()
+    n = len(P.R)
+    cuts = [n * b // bands for b in range(bands + 1)]
+    parts = [gpumem.find_mems(gpumem.index_build(Rs, P.ls, P.L, r_range=(a, b)), Qs).numpy()
+             for a, b in zip(cuts[:-1], cuts[1:])]
+    cat = np.concatenate(parts)
+    cat = cat[np.lexsort((cat[:, 1], cat[:, 0]))]
+    assert np.array_equal(cat, whole)                       # disjoint, complete
+    assert np.array_equal(whole, oracle.mems(P.R, P.Q, P.L, P.ls))
+
+
+@pytest.mark.parametrize("n", [1, 31, 32, 33, 100, 4097])
+def test_revcomp_words(n):
+    rng = np.random.default_rng(n)
+    s = synth.to_ascii(rng.integers(0, 4, n).astype(np.uint8)).tobytes()
+    rc = gpumem.revcomp(gpumem.pack(s))
+    direct = gpumem.pack(_rc(s))
+    assert np.array_equal(rc.words().cpu().numpy(), direct.words().cpu().numpy())
+
+
+@pytest.mark.parametrize("cfg,scale", [("c1", 1.0), ("c4", 0.02)])
+def test_reverse_strand_mems(cfg, scale):
+    """F4: MEMs between R and the reverse complement of Q."""
+    P = synth.make_pair(cfg, scale=scale)
+    Q_rc = _rc(P.Q.tobytes())
+    idx = gpumem.index_build(gpumem.pack(P.R), P.ls, P.L)
+    got = gpumem.find_mems(idx, gpumem.revcomp(gpumem.pack(P.Q))).numpy()
+    assert np.array_equal(got, oracle.mems(P.R, Q_rc, P.L, P.ls))
+
+
+@pytest.mark.parametrize("cfg,scale,L", [("c1", 1.0, 20), ("c1", 0.3, 12), ("c3", 0.01, 50), ("c4", 0.01, 40)])
+def test_mums(cfg, scale, L):
+    """F3: MUMs = MEMs unique in both sequences, vs the substring-count oracle."""
+    P = synth.make_pair(cfg, scale=scale)
+    ls = min(P.ls, L)
+    m = gpumem.find_mems(gpumem.index_build(gpumem.pack(P.R), ls, L), gpumem.pack(P.Q))
+    got = gpumem.mums(m).numpy()
+    want = oracle.mums(P.R, P.Q, L, ls)
+    assert np.array_equal(got, want)
+    assert len(want) > 0
+
+
+def test_mums_tiny_random():
+    rng = np.random.default_rng(5)
+    for trial in range(80):
+        R, Q = synth.random_pair(rng, int(rng.integers(2, 150)), int(rng.integers(2, 150)),
+                                 [b"AC", b"ACG", b"ACGT"][trial % 3])
+        L = int(rng.integers(2, 12))
+        ls = int(rng.integers(1, L + 1))
+        m = gpumem.find_mems(gpumem.index_build(gpumem.pack(R.tobytes()), min(ls, 15), L), gpumem.pack(Q.tobytes()))
+        assert np.array_equal(gpumem.mums(m).numpy(), oracle.mums(R, Q, L, min(ls, 15))), trial
+
+
 @pytest.mark.slow
 def test_full_size_c3():
     P = synth.make_pair("c3")

@@ -199,3 +199,21 @@ def test_c1_full_vs_brute_force_and_planted():
         assert tuple(t) in s
     assert np.array_equal(oracle.mems(P.R, P.Q, P.L, 8), got)
     assert np.array_equal(oracle.mems(P.R, P.Q, P.L, 12, step=5), got)
+
+
+def test_golden_mums_w2():
+    g = read_golden("w2_mums.txt")
+    want = set(g["mem"])
+    assert set(pyoracle.mums(g["R"], g["Q"], g["L"])) == want
+    for ls in (1, 2, 3):
+        assert as_set(oracle.mums(g["R"], g["Q"], g["L"], ls)) == want
+    assert len(oracle.mums("ACGTACGT", "ACGT", 2, 2)) == 0  # W1: "ACGT" twice in R
+
+
+def test_mums_random_vs_python_twin():
+    rng = np.random.default_rng(77)
+    for trial in range(60):
+        R, Q = synth.random_pair(rng, int(rng.integers(5, 120)), int(rng.integers(5, 120)), ALPHABETS[trial % 4])
+        L = int(rng.integers(2, 10))
+        want = set(pyoracle.mums(R.tobytes(), Q.tobytes(), L))
+        assert as_set(oracle.mums(R, Q, L, min(L, 3))) == want
