@@ -276,6 +276,7 @@ __device__ __forceinline__ void load_rec(const uint4 *recs, uint32_t k, uint32_t
     right = (uint64_t(r.w) << 32) | r.z;
 }
 
+template <bool kStatic>
 __global__ void __launch_bounds__(kT) k_find(const FindParams P) {
     __shared__ WarpSmem smem[kWarps];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
@@ -398,12 +399,23 @@ __global__ void __launch_bounds__(kT) k_find(const FindParams P) {
                 st_e += E;
                 st_h += H;
                 // ---- A6-A10: hits dealt 32 at a time
-                for (uint32_t hb = 0; hb < H; hb += 32) {
-                    const uint32_t h = hb + lane;
+                // default: hits dealt 32 per round across the warp (A6). static_lb (the
+                // Fig. 7 ablation, "without load balancing"): every lane walks
+                // the hits of its own query positions, rounds = the warp's largest count.
+                uint32_t rounds = (H + 31) / 32;
+                const uint32_t h0 = ih - n_h;
+                if (kStatic) {
+                    rounds = n_h;
+#pragma unroll
+                    for (int o = 16; o; o >>= 1) rounds = max(rounds, __shfl_xor_sync(0xffffffffu, rounds, o));
+                }
+                for (uint32_t rd = 0; rd < rounds; ++rd) {
+                    const uint32_t h = kStatic ? h0 + rd : rd * 32 + lane;
+                    const bool has = kStatic ? rd < n_h : h < H;
                     int verdict = kDrop;
                     Hit out{0, 0};
                     uint32_t p = 0, q = 0;
-                    if (h < H) {
+                    if (has) {
                         uint32_t lo = 0, hi = E;  // largest entry i with e_off[i] <= h
                         while (hi - lo > 1) {
                             const uint32_t mid = (lo + hi) >> 1;
@@ -488,7 +500,7 @@ uint64_t find_tile_positions() { return kChunk; }
 int find_default_grid() {
     if (!g_default_grid) {
         int per_sm = 0;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_find, kT, 0);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_find<false>, kT, 0);
         if (per_sm < 1) per_sm = 1;
         g_default_grid = per_sm * num_sms();
     }
@@ -501,7 +513,8 @@ cudaError_t launch_find(const FindParams &p, int grid, cudaStream_t s) {
     const uint64_t max_useful = (p.n_tiles + kGrab - 1) / kGrab;
     if (uint64_t(grid) * kWarps > max_useful) grid = int((max_useful + kWarps - 1) / kWarps);
     if (grid < 1) grid = 1;
-    k_find<<<grid, kT, 0, s>>>(p);
+    if (p.static_lb) k_find<true><<<grid, kT, 0, s>>>(p);
+    else k_find<false><<<grid, kT, 0, s>>>(p);
     note_launch();
     return cudaGetLastError();
 }

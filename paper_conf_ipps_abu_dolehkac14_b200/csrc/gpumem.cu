@@ -317,6 +317,7 @@ gpumem_status gpumem_set_option(const char *name, int64_t value) {
     else if (!strcmp(name, "find_spill")) g_opt.find_spill = value < 1 ? 1 : value;
     else if (!strcmp(name, "out_capacity")) g_opt.out_capacity = value < 0 ? 0 : value;
     else if (!strcmp(name, "use_bitmap")) g_opt.use_bitmap = value ? 1 : 0;
+    else if (!strcmp(name, "static_lb")) g_opt.static_lb = value ? 1 : 0;
     else return fail(GPUMEM_ERR_ARG, "unknown option '%s'", name);
     return GPUMEM_OK;
 }
@@ -638,6 +639,7 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
     P.n_tiles = (span + tile - 1) / tile;
     P.spill_t = uint32_t(g_opt.find_spill);
     P.use_bitmap = int(g_opt.use_bitmap);
+    P.static_lb = int(g_opt.static_lb);
     uint64_t cap = g_opt.out_capacity ? uint64_t(g_opt.out_capacity) : (span / 8 + 4096);
 
     Scratch sc(s);

@@ -14,6 +14,7 @@ struct Options {
     int64_t find_spill = 64;     // bucket sizes above this go to the heavy queue
     int64_t out_capacity = 0;    // 0 = automatic
     int64_t use_bitmap = 1;      // 1: rank-word probe + compact bucket table; 0: read the dense ptrs
+    int64_t static_lb = 0;       // 1: each lane processes its own positions' hits (LB ablation)
 };
 extern Options g_opt;
 
@@ -90,6 +91,7 @@ struct FindParams {
     uint64_t coop_cap;
     unsigned long long *coop_count;
     int use_bitmap;
+    int static_lb;               // ablation: no hit redistribution across lanes
 };
 uint64_t find_tile_positions();
 cudaError_t launch_find(const FindParams &p, int grid, cudaStream_t s);
