@@ -40,7 +40,7 @@ WORKLOAD_DESC = {
     "c5_l20": "C5: C4 pair at L=20, ls=13", "c5_l50": "C5: C4 pair at L=50, ls=13",
     "c5_l100": "C5: C4 pair at L=100, ls=13", "c5_l300": "C5: C4 pair at L=300, ls=13",
 }
-ORACLE_SAMPLE_BP = {"ours": 60_000_000, "reference": 16_000_000}
+ORACLE_SAMPLE_BP = {"ours": 40_000_000, "reference": 40_000_000}  # same bounded sample in both legs
 
 
 def parse():

@@ -318,6 +318,7 @@ gpumem_status gpumem_set_option(const char *name, int64_t value) {
     else if (!strcmp(name, "out_capacity")) g_opt.out_capacity = value < 0 ? 0 : value;
     else if (!strcmp(name, "use_bitmap")) g_opt.use_bitmap = value ? 1 : 0;
     else if (!strcmp(name, "static_lb")) g_opt.static_lb = value ? 1 : 0;
+    else if (!strcmp(name, "sort_impl")) g_opt.sort_impl = value ? 1 : 0;
     else return fail(GPUMEM_ERR_ARG, "unknown option '%s'", name);
     return GPUMEM_OK;
 }
@@ -525,8 +526,18 @@ static gpumem_status index_build_impl(const gpumem_seq *R, uint32_t ls, uint32_t
         bool alt = false;
         {
             Stage g("index.sort", s);
-            CK(radix_sort_u32(codes0, locs0, codes1, locs1, n_locs, int(2 * ls), scratch, s, &alt),
-               "seed counting sort");
+            if (g_opt.sort_impl == 0) {  // MSD sort of the unique keys (code << 32 | p)
+                auto *keys = static_cast<uint64_t *>(ws_get(kWsSortK, n_locs * 8, s));
+                void *ms = ws_get(kWsSortScratch, msd_scratch_bytes(n_locs), s);
+                if (!keys || !ms) return GPUMEM_ERR_NOMEM;
+                CK(launch_join_keys(codes0, locs0, n_locs, keys, s), "join keys");
+                CK(msd_sort(keys, nullptr, n_locs, int(2 * ls) + 32, ms, s), "seed sort");
+                CK(launch_split_keys(keys, n_locs, codes1, locs1, s), "split keys");
+                alt = true;
+            } else {
+                CK(radix_sort_u32(codes0, locs0, codes1, locs1, n_locs, int(2 * ls), scratch, s, &alt),
+                   "seed counting sort");
+            }
         }
         codes_sorted = alt ? codes1 : codes0;
         locs = alt ? locs1 : locs0;
@@ -577,13 +588,20 @@ static gpumem_status sort_into_triples(uint64_t *keys, uint32_t *lens, uint64_t 
     if (!trip) return GPUMEM_ERR_NOMEM;
     if (n) {
         Stage g("sort", s);
-        auto *k1 = static_cast<uint64_t *>(ws_get(kWsSortK, n * 8, s));
-        auto *l1 = static_cast<uint32_t *>(ws_get(kWsSortL, n * 4, s));
-        void *scratch = ws_get(kWsSortScratch, radix_scratch_bytes(n), s);
-        if (!k1 || !l1 || !scratch) return GPUMEM_ERR_NOMEM;
-        bool alt = false;
-        CK(radix_sort_u64(keys, lens, k1, l1, n, int(key_bits), scratch, s, &alt), "triple sort");
-        CK(launch_keys_to_triples(alt ? k1 : keys, alt ? l1 : lens, n, qbits, trip, s), "keys to triples");
+        if (g_opt.sort_impl == 0) {  // MSD bucket sort (keys are unique)
+            void *scratch = ws_get(kWsSortScratch, msd_scratch_bytes(n), s);
+            if (!scratch) return GPUMEM_ERR_NOMEM;
+            CK(msd_sort(keys, lens, n, int(key_bits), scratch, s), "triple sort");
+            CK(launch_keys_to_triples(keys, lens, n, qbits, trip, s), "keys to triples");
+        } else {  // stable LSD onesweep radix
+            auto *k1 = static_cast<uint64_t *>(ws_get(kWsSortK, n * 8, s));
+            auto *l1 = static_cast<uint32_t *>(ws_get(kWsSortL, n * 4, s));
+            void *scratch = ws_get(kWsSortScratch, radix_scratch_bytes(n), s);
+            if (!k1 || !l1 || !scratch) return GPUMEM_ERR_NOMEM;
+            bool alt = false;
+            CK(radix_sort_u64(keys, lens, k1, l1, n, int(key_bits), scratch, s, &alt), "triple sort");
+            CK(launch_keys_to_triples(alt ? k1 : keys, alt ? l1 : lens, n, qbits, trip, s), "keys to triples");
+        }
     }
     sc.keep(trip);
     *out = new gpumem_mems{kMagicMems, dev, s, n, trip, gpumem_find_stats{}};

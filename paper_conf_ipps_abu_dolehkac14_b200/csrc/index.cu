@@ -55,6 +55,17 @@ __device__ __forceinline__ uint64_t lower_bound(const uint32_t *__restrict__ a, 
     return lo;
 }
 
+// chunk_first[c] = first index i of the sorted codes with codes[i] >= c * kChunk, for
+// c in [0, n_chunks]; written by the element at each chunk boundary (no searches).
+__global__ void __launch_bounds__(kCodeThreads) k_chunk_bounds(const uint32_t *__restrict__ codes, uint64_t n,
+                                                               uint64_t n_chunks, uint32_t *__restrict__ first) {
+    const uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+    if (i > n) return;
+    const uint64_t c_prev = i == 0 ? 0 : uint64_t(codes[i - 1]) / kChunk + 1;  // chunks after codes[i-1]'s
+    const uint64_t c_this = i == n ? n_chunks : uint64_t(codes[i]) / kChunk;    // ... up to codes[i]'s
+    for (uint64_t c = (i == 0 ? 0 : c_prev); c <= c_this && c <= n_chunks; ++c) first[c] = uint32_t(i);
+}
+
 constexpr uint64_t kStAgg = 1ull << 62;
 constexpr uint64_t kStInc = 2ull << 62;
 constexpr uint64_t kStMask = (1ull << 62) - 1;
@@ -96,6 +107,7 @@ __global__ void __launch_bounds__(kFillThreads) k_ptrs_fill(const uint32_t *__re
                                                             uint64_t n_buckets, uint32_t *__restrict__ ptrs,
                                                             unsigned long long *__restrict__ rankw,
                                                             uint2 *__restrict__ buckets,
+                                                            const uint32_t *__restrict__ chunk_first,
                                                             unsigned long long *status, unsigned int *ticket) {
     __shared__ uint32_t cnt[kChunk + kChunk / 32];   // one pad word per 32: conflict-free rows
     __shared__ uint64_t range[2];
@@ -109,8 +121,8 @@ __global__ void __launch_bounds__(kFillThreads) k_ptrs_fill(const uint32_t *__re
     {
         const uint64_t s0 = uint64_t(s_chunk) * kChunk;
         for (int i = tid; i < kChunk + kChunk / 32; i += kFillThreads) cnt[i] = 0;
-        if (tid == 0) range[0] = lower_bound(codes, n, s0);
-        if (tid == 32) range[1] = lower_bound(codes, n, s0 + kChunk);
+        if (tid == 0) range[0] = chunk_first[s_chunk];
+        if (tid == 32) range[1] = chunk_first[s_chunk + 1];
         __syncthreads();
         const uint64_t lo = range[0], hi = range[1];
         // Alg. 1 step 1 for this chunk: seed counts
@@ -217,20 +229,24 @@ cudaError_t launch_seed_codes(const uint64_t *R, uint32_t ls, uint32_t step, uin
 
 size_t ptrs_fill_scratch_bytes(uint32_t ls) {
     const uint64_t nb = 1ull << (2 * ls);
-    return ((nb + kChunk - 1) / kChunk) * 8 + 64;
+    const uint64_t chunks = (nb + kChunk - 1) / kChunk;
+    return chunks * 8 + 64 + (chunks + 1) * 4 + 256;
 }
 
 cudaError_t launch_ptrs_fill(const uint32_t *sorted_codes, uint64_t n_locs, uint32_t ls, uint32_t *ptrs,
                              unsigned long long *rankw, uint2 *buckets, void *scratch, cudaStream_t s) {
     const uint64_t nb = 1ull << (2 * ls);
     const uint64_t chunks = (nb + kChunk - 1) / kChunk;
-    cudaError_t e = cudaMemsetAsync(scratch, 0, ptrs_fill_scratch_bytes(ls), s);
+    cudaError_t e = cudaMemsetAsync(scratch, 0, chunks * 8 + 64, s);
     if (e != cudaSuccess) return e;
     auto *status = static_cast<unsigned long long *>(scratch);
     auto *ticket = reinterpret_cast<unsigned int *>(status + chunks);
-    k_ptrs_fill<<<unsigned(chunks), kFillThreads, 0, s>>>(sorted_codes, n_locs, nb, ptrs, rankw, buckets, status,
-                                                         ticket);
-    note_launch();
+    auto *first = reinterpret_cast<uint32_t *>(reinterpret_cast<char *>(scratch) + chunks * 8 + 64);
+    k_chunk_bounds<<<unsigned((n_locs + 1 + kCodeThreads - 1) / kCodeThreads), kCodeThreads, 0, s>>>(
+        sorted_codes, n_locs, chunks, first);
+    k_ptrs_fill<<<unsigned(chunks), kFillThreads, 0, s>>>(sorted_codes, n_locs, nb, ptrs, rankw, buckets, first,
+                                                         status, ticket);
+    note_launch(2);
     return cudaGetLastError();
 }
 

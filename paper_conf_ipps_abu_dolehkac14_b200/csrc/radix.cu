@@ -36,7 +36,7 @@ template <>
 struct Cfg<uint64_t> {
     static constexpr int kItems = 8;
 };
-constexpr int kLookWin = 4;  // predecessors read per look-back step
+constexpr int kLookWin = 16;  // predecessors read per look-back step
 
 // Lanes of the warp holding the same digit (among lanes with valid == true), built
 // from one ballot per digit bit -- full-rate, unlike __match_any_sync.

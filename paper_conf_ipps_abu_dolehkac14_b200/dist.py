@@ -29,6 +29,9 @@ def gather_to_root(local: torch.Tensor, group=None):
     Works with any backend that has all_gather/send/recv (NCCL, gloo)."""
     world = dist.get_world_size(group)
     rank = dist.get_rank(group)
+    if local.is_cuda and dist.get_backend(group) == "gloo":  # gloo moves host tensors only
+        runs = gather_to_root(local.cpu(), group)
+        return None if runs is None else [r.to(local.device) for r in runs]
     dev = local.device
     cnt = torch.tensor([local.shape[0]], dtype=torch.int64, device=dev)
     counts = [torch.zeros_like(cnt) for _ in range(world)]
