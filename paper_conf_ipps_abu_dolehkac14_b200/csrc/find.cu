@@ -8,8 +8,10 @@
 // never waits on other warps (no CTA barriers). Per chunk:
 //  stage   the chunk's packed Q words (+ halo) go to the warp's shared memory;
 //  A5      each lane cuts kQPT consecutive seeds out of one 64-bit window, probes
-//          the 4^ls-bit occupancy bitmap (L2-resident) and, for occupied seeds,
-//          reads the bucket range [ptrs[s], ptrs[s+1]). Buckets of
+//          the rank word of each seed (occupancy bit + running rank, 16 MB,
+//          L2-resident) and, for occupied seeds, reads {first slot, count} of the
+//          bucket from the compact table -- the same range as [ptrs[s], ptrs[s+1])
+//          (PAPER.md:84); use_bitmap = 0 reads the dense ptrs instead. Buckets of
 //          more than spill_t hits are cut into kSpillHits-hit pieces and pushed to
 //          a global queue drained by k_heavy (reference-axis tiles of the hot
 //          seeds, Fig. 6 :268-270); the rest become (q, bucket) entries with a
