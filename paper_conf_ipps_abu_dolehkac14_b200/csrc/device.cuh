@@ -35,6 +35,38 @@ __device__ __forceinline__ uint32_t trail_eq(uint64_t x) { return x ? uint32_t(_
 
 __device__ __forceinline__ int lane_id() { return int(threadIdx.x & 31); }
 
+// Loads with an L2 eviction priority (PTX createpolicy + ld.L2::cache_hint): the small,
+// hot lookup tables stay (evict_last) while one-pass streams go first (evict_first).
+// The policy is created inside each asm block so it never occupies a live register.
+#define GM_LD_HINT(PRIO, TYPE, MOD, OUTS, ...)                                                     \
+    asm("{ .reg .b64 pol; createpolicy.fractional.L2::" PRIO ".b64 pol, 1.0;\n\t"                 \
+        "ld.global.nc" MOD ".L2::cache_hint" TYPE " " OUTS ", pol; }" __VA_ARGS__)
+__device__ __forceinline__ unsigned long long ld_last_u64(const unsigned long long *a) {
+    unsigned long long v;
+    GM_LD_HINT("evict_last", ".u64", "", "%0, [%1]", : "=l"(v) : "l"(a));
+    return v;
+}
+__device__ __forceinline__ unsigned long long ld_first_u64(const unsigned long long *a) {
+    unsigned long long v;
+    GM_LD_HINT("evict_first", ".u64", "", "%0, [%1]", : "=l"(v) : "l"(a));
+    return v;
+}
+__device__ __forceinline__ uint2 ld_last_u2(const uint2 *a) {
+    uint2 v;
+    GM_LD_HINT("evict_last", ".v2.u32", "", "{%0, %1}, [%2]", : "=r"(v.x), "=r"(v.y) : "l"(a));
+    return v;
+}
+__device__ __forceinline__ uint4 ld_hint_u4(const uint4 *a, bool stream) {
+    uint4 v;
+    if (stream)
+        GM_LD_HINT("evict_first", ".v4.u32", ".L1::no_allocate", "{%0, %1, %2, %3}, [%4]",
+                   : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(a));
+    else
+        GM_LD_HINT("evict_last", ".v4.u32", ".L1::no_allocate", "{%0, %1, %2, %3}, [%4]",
+                   : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(a));
+    return v;
+}
+
 __device__ __forceinline__ uint32_t lanemask_lt() {
     uint32_t m;
     asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));

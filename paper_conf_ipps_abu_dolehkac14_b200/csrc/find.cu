@@ -271,14 +271,14 @@ __device__ __forceinline__ void warp_emit(const FindParams &P, WarpSmem &s, uint
 }
 
 __device__ __forceinline__ void load_rec(const uint4 *recs, uint32_t k, uint32_t &p, uint32_t &left,
-                                         uint64_t &right) {
-    const uint4 r = __ldg(recs + k);
+                                         uint64_t &right, int stream) {
+    const uint4 r = stream < 0 ? __ldg(recs + k) : ld_hint_u4(recs + k, stream != 0);
     p = r.x;
     left = r.y;
     right = (uint64_t(r.w) << 32) | r.z;
 }
 
-template <bool kStatic>
+template <bool kStatic, bool kHints>
 __global__ void __launch_bounds__(kT) k_find(const FindParams P) {
     __shared__ WarpSmem smem[kWarps];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
@@ -287,6 +287,8 @@ __global__ void __launch_bounds__(kT) k_find(const FindParams P) {
     uint32_t nbuf = 0;
     unsigned long long st_e = 0, st_h = 0;
     QStage qs{s.qw, 0};
+    // L2 priorities: lookup tables stay, streamed data goes first (records only when
+    // they cannot stay resident anyway, P.recs_stream)
 
     for (;;) {
         uint32_t grab = 0;
@@ -300,7 +302,11 @@ __global__ void __launch_bounds__(kT) k_find(const FindParams P) {
             // ---- stage the chunk's Q words (+ halo) in shared memory
             const uint32_t wb = (q0 >> 5) ? (q0 >> 5) - 1 : 0;
             qs.wbase = wb;
-            if (lane < kQW) s.qw[lane] = (wb + lane < P.nQw) ? __ldg(P.Q + wb + lane) : 0ull;
+            if (lane < kQW)
+                s.qw[lane] = (wb + lane < P.nQw)
+                                 ? (kHints ? ld_first_u64(reinterpret_cast<const unsigned long long *>(P.Q) + wb + lane)
+                                          : __ldg(P.Q + wb + lane))
+                                 : 0ull;
             __syncwarp();
 
             // ---- A5: seeds -> bitmap -> bucket ranges
@@ -324,7 +330,8 @@ __global__ void __launch_bounds__(kT) k_find(const FindParams P) {
                     for (int j = 0; j < kQPT; ++j) {
                         rank[j] = 0;
                         if (occ[j]) {
-                            const unsigned long long rw = __ldg(P.rankw + (code[j] >> 5));
+                            const unsigned long long rw = kHints ? ld_last_u64(P.rankw + (code[j] >> 5))
+                                                                      : __ldg(P.rankw + (code[j] >> 5));
                             const uint32_t bit = code[j] & 31, bits = uint32_t(rw);
                             occ[j] = (bits >> bit) & 1u;
                             rank[j] = uint32_t(rw >> 32) + __popc(bits & ((1u << bit) - 1u));
@@ -333,7 +340,7 @@ __global__ void __launch_bounds__(kT) k_find(const FindParams P) {
 #pragma unroll
                     for (int j = 0; j < kQPT; ++j) {
                         if (occ[j]) {
-                            const uint2 b = __ldg(P.buckets + rank[j]);
+                            const uint2 b = kHints ? ld_last_u2(P.buckets + rank[j]) : __ldg(P.buckets + rank[j]);
                             beg[j] = b.x;
                             cnt[j] = b.y;
                         }
@@ -426,7 +433,7 @@ __global__ void __launch_bounds__(kT) k_find(const FindParams P) {
                         q = q0 + s.e_q[lo];
                         uint32_t rl;
                         uint64_t rr;
-                        load_rec(P.recs, s.e_beg[lo] + (h - s.e_off[lo]), p, rl, rr);
+                        load_rec(P.recs, s.e_beg[lo] + (h - s.e_off[lo]), p, rl, rr, kHints ? 1 : -1);
                         verdict = decide(P, p, rl, rr, q, qs.back16(q), qs.fwd(q + P.ls), out);
                     }
                     push_coop(P, verdict, p, q);
@@ -462,7 +469,7 @@ __global__ void __launch_bounds__(kT) k_heavy(const FindParams P) {
         if (uint32_t(lane) < piece.z) {
             uint32_t rl;
             uint64_t rr;
-            load_rec(P.recs, piece.y + lane, p, rl, rr);
+            load_rec(P.recs, piece.y + lane, p, rl, rr, P.recs_stream);
             verdict = decide(P, p, rl, rr, q, uint32_t(win_back(P.Q, q)), win_fwd(P.Q, uint64_t(q) + P.ls), out);
         }
         push_coop(P, verdict, p, q);
@@ -502,7 +509,7 @@ uint64_t find_tile_positions() { return kChunk; }
 int find_default_grid() {
     if (!g_default_grid) {
         int per_sm = 0;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_find<false>, kT, 0);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_find<false, false>, kT, 0);
         if (per_sm < 1) per_sm = 1;
         g_default_grid = per_sm * num_sms();
     }
@@ -515,8 +522,11 @@ cudaError_t launch_find(const FindParams &p, int grid, cudaStream_t s) {
     const uint64_t max_useful = (p.n_tiles + kGrab - 1) / kGrab;
     if (uint64_t(grid) * kWarps > max_useful) grid = int((max_useful + kWarps - 1) / kWarps);
     if (grid < 1) grid = 1;
-    if (p.static_lb) k_find<true><<<grid, kT, 0, s>>>(p);
-    else k_find<false><<<grid, kT, 0, s>>>(p);
+    // kHints: the seed records exceed half of L2 -> cache-policy loads (lookup tables
+    // evict_last, streams evict_first); otherwise plain loads (measured faster there)
+    if (p.static_lb) k_find<true, false><<<grid, kT, 0, s>>>(p);
+    else if (p.recs_stream) k_find<false, true><<<grid, kT, 0, s>>>(p);
+    else k_find<false, false><<<grid, kT, 0, s>>>(p);
     note_launch();
     return cudaGetLastError();
 }

@@ -658,6 +658,11 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
     P.spill_t = uint32_t(g_opt.find_spill);
     P.use_bitmap = int(g_opt.use_bitmap);
     P.static_lb = int(g_opt.static_lb);
+    {  // records that cannot share L2 with the lookup tables are streamed
+        int l2 = 0;
+        cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, dev);
+        P.recs_stream = idx->n_locs * 16 > uint64_t(l2) / 2 ? 1 : 0;
+    }
     uint64_t cap = g_opt.out_capacity ? uint64_t(g_opt.out_capacity) : (span / 8 + 4096);
 
     Scratch sc(s);

@@ -100,6 +100,7 @@ struct FindParams {
     unsigned long long *coop_count;
     int use_bitmap;
     int static_lb;               // ablation: no hit redistribution across lanes
+    int recs_stream;             // seed records too large to stay in L2: load them evict_first
 };
 uint64_t find_tile_positions();
 cudaError_t launch_find(const FindParams &p, int grid, cudaStream_t s);
