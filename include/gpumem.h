@@ -192,7 +192,12 @@ gpumem_status gpumem_set_allocator(void *(*alloc_fn)(size_t bytes, void *cuda_st
  *  "find_spill"       bucket size above which hits are spilled to the heavy queue
  *  "out_capacity"     initial output capacity in triples (0 = automatic; small values
  *                     force the overflow-and-retry path in tests)
- *  "use_bitmap"       1 (default) probe the occupancy bitmap before ptrs, 0 probe ptrs only */
+ *  "use_bitmap"       1 (default) probe the rank words + bucket table, 0 probe ptrs only
+ *  "static_lb"        1: no hit redistribution across lanes (load-balancing ablation)
+ *  "sort_impl"        1 (default) stable LSD onesweep radix sort, 0 MSD bucket sort
+ *  "radix_bits"       LSD digit width: 0 (default) = 9 bits when that saves a pass, else 8;
+ *                     or pinned to 8, 9, 10; anything else is GPUMEM_ERR_ARG
+ * Unknown names are GPUMEM_ERR_ARG. */
 gpumem_status gpumem_set_option(const char *name, int64_t value);
 
 /* Per-stage device time: when enabled, CUDA events bracket each stage on its stream.

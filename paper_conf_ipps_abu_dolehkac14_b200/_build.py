@@ -35,12 +35,12 @@ def _headers():
                   + glob.glob(os.path.join(INCLUDE, "*.h")))
 
 
-def _compile(src, verbose):
-    obj = os.path.join(OBJDIR, os.path.basename(src) + ".o")
+def _compile(src, verbose, objdir=OBJDIR, defines=()):
+    obj = os.path.join(objdir, os.path.basename(src) + ".o")
     newest_dep = max([os.path.getmtime(src)] + [os.path.getmtime(h) for h in _headers()])
     if os.path.exists(obj) and os.path.getmtime(obj) >= newest_dep:
         return obj, ""
-    cmd = [NVCC, *FLAGS, "-c", src, "-o", obj]
+    cmd = [NVCC, *FLAGS, *defines, "-c", src, "-o", obj]
     if verbose:
         cmd.insert(1, "-Xptxas=-v")
     r = subprocess.run(cmd, capture_output=True, text=True)
@@ -49,14 +49,17 @@ def _compile(src, verbose):
     return obj, r.stdout + r.stderr
 
 
-def build(verbose=False, force=False):
-    os.makedirs(OBJDIR, exist_ok=True)
+def build(verbose=False, force=False, lib=LIB, objdir=OBJDIR, defines=()):
+    """Compile csrc/*.cu and link `lib`. `defines` (-DNAME=V) select compile-time tuning
+    variants; they build into their own objdir and library (tools/variants.py)."""
+    LIB = lib
+    os.makedirs(objdir, exist_ok=True)
     if force:
-        for f in glob.glob(os.path.join(OBJDIR, "*.o")):
+        for f in glob.glob(os.path.join(objdir, "*.o")):
             os.remove(f)
     srcs = _sources()
     with concurrent.futures.ThreadPoolExecutor(max_workers=min(8, len(srcs))) as ex:
-        results = list(ex.map(lambda s: _compile(s, verbose), srcs))
+        results = list(ex.map(lambda s: _compile(s, verbose, objdir, tuple(defines)), srcs))
     objs = [o for o, _ in results]
     if verbose:
         for _, log in results:

@@ -319,6 +319,10 @@ gpumem_status gpumem_set_option(const char *name, int64_t value) {
     else if (!strcmp(name, "use_bitmap")) g_opt.use_bitmap = value ? 1 : 0;
     else if (!strcmp(name, "static_lb")) g_opt.static_lb = value ? 1 : 0;
     else if (!strcmp(name, "sort_impl")) g_opt.sort_impl = value ? 1 : 0;
+    else if (!strcmp(name, "radix_bits")) {
+        if (value != 0 && (value < 8 || value > 10)) return fail(GPUMEM_ERR_ARG, "radix_bits must be 0 or 8..10");
+        g_opt.radix_bits = value;
+    }
     else return fail(GPUMEM_ERR_ARG, "unknown option '%s'", name);
     return GPUMEM_OK;
 }

@@ -16,6 +16,7 @@ struct Options {
     int64_t use_bitmap = 1;      // 1: rank-word probe + compact bucket table; 0: read the dense ptrs
     int64_t static_lb = 0;       // 1: each lane processes its own positions' hits (LB ablation)
     int64_t sort_impl = 1;       // 0: MSD bucket sort (unique keys; measured slower), 1: stable LSD onesweep radix
+    int64_t radix_bits = 0;      // LSD digit width: 0 = 9 bits if that saves a pass else 8; or pinned 8, 9, 10
 };
 extern Options g_opt;
 

@@ -1,4 +1,5 @@
-// radix.cu -- stable LSD radix sort, onesweep style (counting sort per 8-bit digit).
+// radix.cu -- stable LSD radix sort (counting sort per 8-, 9- or 10-bit digit), one
+// contiguous chunk of the input per resident CTA.
 // Used twice on the hot path:
 //  * index build: the counting sort of sampled seeds over 4^ls buckets (Alg. 1
 //    steps 1-3) done digit by digit; stability leaves every
@@ -6,44 +7,60 @@
 //    per-seed sort) achieves, without a per-bucket sort;
 //  * output: MEM triples into (r, q) order.
 //
-// Launches per sort: one memset, k_hist_all (histograms of every digit in one
-// read of the keys), k_hist_scan (exclusive scan of each digit histogram), then
-// one k_onesweep per digit: the tile's stable local ranks (per-warp running
-// counters + __match_any_sync peers), its digit counts published to a status
-// array and the global prefix found by decoupled look-back over earlier tiles,
-// then a reorder through shared memory so each digit run is written out
-// contiguously (coalesced).
+// Per digit pass, three launches:
+//  k_chunk_hist  -- one CTA per chunk (a contiguous run of tiles; as many chunks as the
+//                   GPU holds resident scatter CTAs) counts the chunk's digits into
+//                   counts[d][c] and adds them to the pass's digit totals;
+//  k_chunk_scan  -- exact global offsets of every (digit, chunk):
+//                   offs[d][c] = sum_{d'<d} total[d'] + sum_{c'<c} counts[d][c'];
+//  k_scatter     -- same grid; CTA c walks its chunk's tiles in order with the next
+//                   tile's keys/values already in flight (TMA bulk copy into the second
+//                   shared-memory stage), ranks each tile stably (per-warp running digit
+//                   counters + ballot peers), reorders it through shared memory and
+//                   writes every digit run contiguously at its running chunk offset.
+// No CTA ever waits on another (no look-back chain); the cost is one extra read of
+// the keys per pass for the chunk histogram.
 #include "internal.h"
 #include "device.cuh"
 
 namespace gm {
 namespace {
 
-constexpr int kT = 256;                 // threads per CTA
+constexpr int kT = 256;  // threads per CTA
 constexpr int kWarps = kT / 32;
-constexpr int kBins = 256;
-constexpr uint32_t kFlagAgg = 1u << 30;
-constexpr uint32_t kFlagInc = 2u << 30;
-constexpr uint32_t kValMask = (1u << 30) - 1;
 
+#ifndef GM_RADIX_ITEMS32
+#define GM_RADIX_ITEMS32 16
+#endif
+#ifndef GM_RADIX_ITEMS64
+#define GM_RADIX_ITEMS64 16
+#endif
+#ifndef GM_RADIX_MINB
+#define GM_RADIX_MINB 2
+#endif
 template <class K>
 struct Cfg;
 template <>
 struct Cfg<uint32_t> {
-    static constexpr int kItems = 12;
+    static constexpr int kItems = GM_RADIX_ITEMS32;
 };
 template <>
 struct Cfg<uint64_t> {
-    static constexpr int kItems = 8;
+    static constexpr int kItems = GM_RADIX_ITEMS64;
 };
-constexpr int kLookWin = 16;  // predecessors read per look-back step
+
+template <class K>
+constexpr uint64_t tile_items() {
+    return uint64_t(kT) * Cfg<K>::kItems;
+}
 
 // Lanes of the warp holding the same digit (among lanes with valid == true), built
 // from one ballot per digit bit -- full-rate, unlike __match_any_sync.
+template <int RB>
 __device__ __forceinline__ unsigned match_digit(uint32_t d, bool valid, int bits) {
     unsigned peers = __ballot_sync(0xffffffffu, valid);
 #pragma unroll
-    for (int b = 0; b < 8; ++b) {
+    for (int b = 0; b < RB; ++b) {
         if (b < bits) {
             const bool bit = (d >> b) & 1u;
             const unsigned m = __ballot_sync(0xffffffffu, bit);
@@ -53,190 +70,351 @@ __device__ __forceinline__ unsigned match_digit(uint32_t d, bool valid, int bits
     return peers;
 }
 
-// Histograms of every digit position in one read of the keys. Each warp owns
-// private counters (no shared-memory atomics, which serialise per lane): the
-// leader of each group of equal digits adds the group's size.
-constexpr int kHT = 128;
-constexpr int kHWarps = kHT / 32;
-
-template <class K>
-__global__ void __launch_bounds__(kHT) k_hist_all(const K *__restrict__ keys, uint64_t n, int passes,
-                                                  uint32_t *__restrict__ hist) {
-    __shared__ uint32_t h[kHWarps][8][kBins];  // 32 KB
-    for (int i = threadIdx.x; i < kHWarps * 8 * kBins; i += kHT) (&h[0][0][0])[i] = 0;
-    __syncthreads();
-    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-    const uint64_t stride = uint64_t(gridDim.x) * kHT;
-    for (uint64_t base = uint64_t(blockIdx.x) * kHT + uint64_t(w) * 32; base < n; base += stride) {
-        const uint64_t idx = base + lane;
-        const bool valid = idx < n;
-        const K k = valid ? keys[idx] : K(0);
-        if (valid) {
-            for (int p = 0; p < passes; ++p) atomicAdd(&h[w][p][uint32_t(k >> (8 * p)) & (kBins - 1)], 1u);
-        }
+// Chunk c of a pass: tiles [c * tpc, min((c + 1) * tpc, tiles)).
+struct Chunking {
+    uint64_t n, tiles, tpc;
+    uint32_t chunks;
+    __host__ __device__ uint64_t begin(uint32_t c, uint64_t tile) const {
+        const uint64_t b = uint64_t(c) * tpc * tile;
+        return b < n ? b : n;
     }
-    __syncthreads();
-    for (int i = threadIdx.x; i < passes * kBins; i += kHT) {
-        uint32_t c = 0;
-#pragma unroll
-        for (int ww = 0; ww < kHWarps; ++ww) c += (&h[ww][0][0])[i];
-        if (c) atomicAdd(hist + i, c);
+    __host__ __device__ uint64_t end(uint32_t c, uint64_t tile) const {
+        const uint64_t e = (uint64_t(c) + 1) * tpc * tile;
+        return e < n ? e : n;
     }
-}
-
-__global__ void __launch_bounds__(kT) k_hist_scan(uint32_t *hist, int passes) {
-    __shared__ uint32_t ws[kWarps];
-    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-    for (int p = 0; p < passes; ++p) {
-        const uint32_t x = hist[p * kBins + threadIdx.x];
-        uint32_t inc = x;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            const uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
-            if (lane >= o) inc += y;
-        }
-        if (lane == 31) ws[w] = inc;
-        __syncthreads();
-        uint32_t pre = 0;
-        for (int i = 0; i < w; ++i) pre += ws[i];
-        hist[p * kBins + threadIdx.x] = pre + inc - x;  // exclusive
-        __syncthreads();
-    }
-}
-
-template <class K, class V>
-struct alignas(16) SweepSmem {
-    K k[kT * Cfg<K>::kItems];
-    V v[kT * Cfg<K>::kItems];
-    uint32_t wcnt[kWarps][kBins];
-    uint32_t local_excl[kBins];
-    uint32_t global_base[kBins];
-    uint32_t ws[kWarps];
-    uint32_t tile;
 };
 
-template <class K, class V>
-__global__ void __launch_bounds__(kT, 3) k_onesweep(const K *__restrict__ kin, const V *__restrict__ vin,
-                                                 K *__restrict__ kout, V *__restrict__ vout, uint64_t n,
-                                                 int shift, int bits, const uint32_t *__restrict__ digit_off,
-                                                 uint32_t *status, unsigned int *tile_ctr) {
-    constexpr int kItems = Cfg<K>::kItems;
-    constexpr int kTile = kT * kItems;
-    extern __shared__ __align__(16) unsigned char smem_raw[];
-    SweepSmem<K, V> &S = *reinterpret_cast<SweepSmem<K, V> *>(smem_raw);
-    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+template <class K, int RB>
+__global__ void __launch_bounds__(kT) k_chunk_hist(const K *__restrict__ keys, Chunking ch, int shift, int bits,
+                                                   uint32_t *__restrict__ counts, uint32_t *__restrict__ totals) {
+    constexpr int kBins = 1 << RB;
+    constexpr int DPT = kBins / kT;
+    __shared__ uint32_t h[kWarps][kBins];
+    const int tid = threadIdx.x, w = tid >> 5;
     const uint32_t dmask = (1u << bits) - 1;
-    if (tid == 0) S.tile = atomicAdd(tile_ctr, 1u);
-    for (int i = tid; i < kWarps * kBins; i += kT) (&S.wcnt[0][0])[i] = 0;
+    for (int i = tid; i < kWarps * kBins; i += kT) (&h[0][0])[i] = 0;
     __syncthreads();
-    const uint32_t tile = S.tile;
-    const uint64_t base = uint64_t(tile) * kTile;
-    const uint32_t tile_n = uint32_t(min(uint64_t(kTile), n - base));
-
-    // ---- load (warp-striped rounds keep input order = (warp, round, lane)) and rank
-    K k[kItems];
-    V v[kItems];
-    uint32_t rank[kItems];
-    const uint64_t wbase = base + uint64_t(w) * 32 * kItems;
-#pragma unroll
-    for (int j = 0; j < kItems; ++j) {
-        const uint64_t idx = wbase + uint64_t(j) * 32 + lane;
-        const bool valid = idx < n;
-        k[j] = valid ? kin[idx] : K(0);
-        v[j] = valid ? vin[idx] : 0u;
-        const uint32_t d = uint32_t(k[j] >> shift) & dmask;
-        const unsigned peers = match_digit(d, valid, bits);
-        const uint32_t b0 = valid ? S.wcnt[w][d] : 0u;
-        rank[j] = b0 + __popc(peers & lanemask_lt());
-        __syncwarp();
-        if (valid && lane == __ffs(peers) - 1) S.wcnt[w][d] = b0 + __popc(peers);
-        __syncwarp();
-    }
+    const uint32_t c = blockIdx.x;
+    const uint64_t b = ch.begin(c, tile_items<K>()), e = ch.end(c, tile_items<K>());
+    for (uint64_t i = b + tid; i < e; i += kT) atomicAdd(&h[w][uint32_t(keys[i] >> shift) & dmask], 1u);
     __syncthreads();
-
-    // ---- per digit: tile count, warp offsets, publish + decoupled look-back
-    const uint32_t d = tid;  // kT == kBins
-    uint32_t cnt = 0;
 #pragma unroll
-    for (int ww = 0; ww < kWarps; ++ww) {
-        const uint32_t c = S.wcnt[ww][d];
-        S.wcnt[ww][d] = cnt;
-        cnt += c;
+    for (int dd = 0; dd < DPT; ++dd) {
+        const int d = dd * kT + tid;
+        uint32_t s = 0;
+#pragma unroll
+        for (int ww = 0; ww < kWarps; ++ww) s += h[ww][d];
+        counts[uint64_t(d) * ch.chunks + c] = s;  // digit-major
+        if (s) atomicAdd(totals + d, s);
     }
-    volatile uint32_t *st = status;
-    if (tile == 0) {
-        st[d] = kFlagInc | cnt;
-        S.global_base[d] = digit_off[d];
-    } else {
-        st[uint64_t(tile) * kBins + d] = kFlagAgg | cnt;
-        // decoupled look-back in windows of kLookWin predecessors (independent loads)
-        uint32_t excl = 0;
-        int64_t t = int64_t(tile) - 1;
-        for (bool done = false; !done;) {
-            uint32_t s[kLookWin];
+}
+
+// offs[d][c] = sum_{d' < d} totals[d'] + sum_{c' < c} counts[d][c']: every CTA scans the
+// (small) digit totals, then each warp scans one digit's row of chunk counts.
+template <int RB>
+__global__ void __launch_bounds__(kT) k_chunk_scan(const uint32_t *__restrict__ counts,
+                                                   const uint32_t *__restrict__ totals, uint32_t chunks,
+                                                   uint32_t *__restrict__ offs) {
+    constexpr int kBins = 1 << RB;
+    constexpr int DPT = kBins / kT;
+    __shared__ uint32_t dbase[kBins];
+    __shared__ uint32_t ws[kWarps * DPT];
+    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+    uint32_t tot[DPT], inc[DPT];
 #pragma unroll
-            for (int i = 0; i < kLookWin; ++i)
-                s[i] = (t - i >= 0) ? st[uint64_t(t - i) * kBins + d] : uint32_t(2u << 30);
-            int i = 0;
+    for (int dd = 0; dd < DPT; ++dd) tot[dd] = inc[dd] = totals[dd * kT + tid];
 #pragma unroll
-            for (int ii = 0; ii < kLookWin; ++ii) {
-                if (i != ii || done) continue;
-                const uint32_t f = s[ii] & ~kValMask;
-                if (f == 0) continue;  // not published yet: re-poll from here
-                excl += s[ii] & kValMask;
-                if (f == kFlagInc) done = true; else ++i;
-            }
-            t -= i;
+    for (int o = 1; o < 32; o <<= 1) {
+#pragma unroll
+        for (int dd = 0; dd < DPT; ++dd) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, inc[dd], o);
+            if (lane >= o) inc[dd] += y;
         }
-        st[uint64_t(tile) * kBins + d] = kFlagInc | (excl + cnt);
-        S.global_base[d] = digit_off[d] + excl;
     }
-    {  // tile-local exclusive digit offsets (block scan over the 256 digits)
-        uint32_t inc = cnt;
+    if (lane == 31) {
+#pragma unroll
+        for (int dd = 0; dd < DPT; ++dd) ws[dd * kWarps + w] = inc[dd];
+    }
+    __syncthreads();
+    uint32_t carry = 0;
+#pragma unroll
+    for (int dd = 0; dd < DPT; ++dd) {
+        uint32_t pre = 0, seg = 0;
+#pragma unroll
+        for (int i = 0; i < kWarps; ++i) {
+            const uint32_t x = ws[dd * kWarps + i];
+            pre += i < w ? x : 0u;
+            seg += x;
+        }
+        dbase[dd * kT + tid] = carry + pre + inc[dd] - tot[dd];
+        carry += seg;
+    }
+    __syncthreads();
+    const uint32_t d = blockIdx.x * kWarps + w;
+    const uint32_t *row = counts + uint64_t(d) * chunks;
+    uint32_t *orow = offs + uint64_t(d) * chunks;
+    uint32_t run = dbase[d];
+    for (uint32_t c0 = 0; c0 < chunks; c0 += 32) {
+        const uint32_t c = c0 + lane;
+        const uint32_t x = c < chunks ? row[c] : 0u;
+        uint32_t s = x;
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
-            const uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
-            if (lane >= o) inc += y;
+            const uint32_t y = __shfl_up_sync(0xffffffffu, s, o);
+            if (lane >= o) s += y;
         }
-        if (lane == 31) S.ws[w] = inc;
-        __syncthreads();
-        uint32_t pre = 0;
-        for (int i = 0; i < w; ++i) pre += S.ws[i];
-        S.local_excl[d] = pre + inc - cnt;
+        if (c < chunks) orow[c] = run + s - x;
+        run += __shfl_sync(0xffffffffu, s, 31);
     }
-    __syncthreads();
+}
 
-    // ---- reorder into digit order in shared memory
+// Shared memory of k_scatter: two stage buffers, each first the TMA destination of
+// one tile's keys/values and then, once they sit in registers, that tile's reorder
+// buffer.
+template <class K, class V, int RB>
+struct alignas(128) ScatterSmem {
+    K k[2][kT * Cfg<K>::kItems];
+    V v[2][kT * Cfg<K>::kItems];
+    uint32_t wcnt[kWarps][1 << RB];
+    uint32_t gofs[1 << RB];  // per digit: global position of the tile's slot 0 (mod 2^32)
+    uint32_t ws[kWarps * ((1 << RB) / kT)];
+    unsigned long long bar[2];
+};
+
+__device__ __forceinline__ uint32_t smem_u32(const void *p) {
+    return uint32_t(__cvta_generic_to_shared(p));
+}
+
+// One thread: bulk-copy `bytes` (multiple of 16) from global to shared, completing on `bar`.
+__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes, unsigned long long *bar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                 :: "r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)) : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait(unsigned long long *bar, uint32_t parity) {
+    uint32_t ok = 0;
+    while (!ok)
+        asm volatile("{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
+                     : "=r"(ok) : "r"(smem_u32(bar)), "r"(parity) : "memory");
+}
+
+template <class K, class V, int RB>
+__global__ void __launch_bounds__(kT, GM_RADIX_MINB) k_scatter(const K *__restrict__ kin, const V *__restrict__ vin,
+                                                  K *__restrict__ kout, V *__restrict__ vout, Chunking ch,
+                                                  int shift, int bits, const uint32_t *__restrict__ offs) {
+    constexpr int kBins = 1 << RB;
+    constexpr int DPT = kBins / kT;  // digits owned per thread: tid, tid + kT, ...
+    constexpr int kItems = Cfg<K>::kItems;
+    constexpr int kTile = kT * kItems;
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    ScatterSmem<K, V, RB> &S = *reinterpret_cast<ScatterSmem<K, V, RB> *>(smem_raw);
+    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+    const uint32_t dmask = (1u << bits) - 1;
+    const uint32_t c = blockIdx.x;
+    const uint64_t cb = ch.begin(c, kTile), ce = ch.end(c, kTile);
+    const uint32_t n_t = uint32_t((ce - cb + kTile - 1) / kTile);
+    const uint32_t n_full = uint32_t((ce - cb) / kTile);  // tiles moved by TMA; a ragged tail is loaded directly
+
+    auto issue = [&](uint32_t t, int stage) {  // thread 0
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;"
+                     :: "r"(smem_u32(&S.bar[stage])), "r"(uint32_t(kTile * (sizeof(K) + sizeof(V)))) : "memory");
+        bulk_g2s(S.k[stage], kin + cb + uint64_t(t) * kTile, kTile * sizeof(K), &S.bar[stage]);
+        bulk_g2s(S.v[stage], vin + cb + uint64_t(t) * kTile, kTile * sizeof(V), &S.bar[stage]);
+    };
+    if (tid == 0) {
+        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" :: "r"(smem_u32(&S.bar[0])) : "memory");
+        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" :: "r"(smem_u32(&S.bar[1])) : "memory");
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        if (n_full > 0) issue(0, 0);
+    }
+    uint32_t gbase[DPT];  // running global offset of each owned digit in this chunk
 #pragma unroll
-    for (int j = 0; j < kItems; ++j) {
-        const uint64_t idx = wbase + uint64_t(j) * 32 + lane;
-        if (idx < n) {
-            const uint32_t dd = uint32_t(k[j] >> shift) & dmask;
-            const uint32_t lp = S.local_excl[dd] + S.wcnt[w][dd] + rank[j];
-            S.k[lp] = k[j];
-            S.v[lp] = v[j];
-        }
-    }
+    for (int dd = 0; dd < DPT; ++dd) gbase[dd] = offs[uint64_t(dd * kT + tid) * ch.chunks + c];
     __syncthreads();
-    // ---- coalesced write-out: consecutive slots of one digit go to consecutive addresses
-    for (uint32_t i = tid; i < tile_n; i += kT) {
-        const K kk = S.k[i];
-        const uint32_t dd = uint32_t(kk >> shift) & dmask;
-        const uint64_t g = uint64_t(S.global_base[dd]) + (i - S.local_excl[dd]);
-        kout[g] = kk;
-        vout[g] = S.v[i];
+
+    for (uint32_t t = 0; t < n_t; ++t) {
+        const int sg = t & 1;
+        if (tid == 0 && t + 1 < n_full) issue(t + 1, sg ^ 1);  // buffer sg^1 was released at the end of tile t-1
+        for (int i = tid; i < kWarps * kBins; i += kT) (&S.wcnt[0][0])[i] = 0;
+        const uint64_t base = cb + uint64_t(t) * kTile;
+        const uint32_t tile_n = uint32_t(min(uint64_t(kTile), ce - base));
+
+        // ---- items into registers (warp-striped rounds keep input order = (warp, round, lane))
+        K k[kItems];
+        V v[kItems];
+        uint32_t rank[kItems];
+        const uint32_t wofs = uint32_t(w) * 32 * kItems;
+        if (t < n_full) {
+            mbar_wait(&S.bar[sg], (t >> 1) & 1);
+#pragma unroll
+            for (int j = 0; j < kItems; ++j) {
+                k[j] = S.k[sg][wofs + j * 32 + lane];
+                v[j] = S.v[sg][wofs + j * 32 + lane];
+            }
+        } else {
+#pragma unroll
+            for (int j = 0; j < kItems; ++j) {
+                const uint32_t li = wofs + j * 32 + lane;
+                k[j] = li < tile_n ? kin[base + li] : K(0);
+                v[j] = li < tile_n ? vin[base + li] : V(0);
+            }
+        }
+        __syncthreads();  // wcnt zeroed
+
+        // ---- stable ranks: per-warp running digit counters + ballot peers (all ballots
+        //      first: they are independent, only the counter updates are sequential)
+        unsigned peers[kItems];
+#pragma unroll
+        for (int j = 0; j < kItems; ++j)
+            peers[j] = match_digit<RB>(uint32_t(k[j] >> shift) & dmask, wofs + j * 32 + lane < tile_n, bits);
+#pragma unroll
+        for (int j = 0; j < kItems; ++j) {
+            const bool valid = wofs + j * 32 + lane < tile_n;
+            const uint32_t d = uint32_t(k[j] >> shift) & dmask;
+            const uint32_t b0 = valid ? S.wcnt[w][d] : 0u;
+            rank[j] = b0 + __popc(peers[j] & lanemask_lt());
+            __syncwarp();
+            if (valid && lane == __ffs(peers[j]) - 1) S.wcnt[w][d] = b0 + __popc(peers[j]);
+            __syncwarp();
+        }
+        __syncthreads();
+
+        // ---- per digit: tile count, tile-local exclusive offset (block scan); then each
+        //      warp's slot base in the reorder buffer and the tile-to-global offset
+        uint32_t cnt[DPT], inc[DPT], xw[DPT][kWarps];
+#pragma unroll
+        for (int dd = 0; dd < DPT; ++dd) {
+            uint32_t c0 = 0;
+#pragma unroll
+            for (int ww = 0; ww < kWarps; ++ww) {
+                xw[dd][ww] = S.wcnt[ww][dd * kT + tid];
+                c0 += xw[dd][ww];
+            }
+            cnt[dd] = inc[dd] = c0;
+        }
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+#pragma unroll
+            for (int dd = 0; dd < DPT; ++dd) {
+                const uint32_t y = __shfl_up_sync(0xffffffffu, inc[dd], o);
+                if (lane >= o) inc[dd] += y;
+            }
+        }
+        if (lane == 31) {
+#pragma unroll
+            for (int dd = 0; dd < DPT; ++dd) S.ws[dd * kWarps + w] = inc[dd];
+        }
+        __syncthreads();
+        {
+            uint32_t carry = 0;
+#pragma unroll
+            for (int dd = 0; dd < DPT; ++dd) {
+                uint32_t pre = 0, seg = 0;
+#pragma unroll
+                for (int i = 0; i < kWarps; ++i) {
+                    const uint32_t x = S.ws[dd * kWarps + i];
+                    pre += i < w ? x : 0u;
+                    seg += x;
+                }
+                const uint32_t excl = carry + pre + inc[dd] - cnt[dd];
+                carry += seg;
+                const uint32_t d = dd * kT + tid;
+                uint32_t run = excl;
+#pragma unroll
+                for (int ww = 0; ww < kWarps; ++ww) {
+                    S.wcnt[ww][d] = run;
+                    run += xw[dd][ww];
+                }
+                S.gofs[d] = gbase[dd] - excl;  // slot i of digit d goes to gofs[d] + i (mod 2^32)
+                gbase[dd] += cnt[dd];
+            }
+        }
+        __syncthreads();
+
+        // ---- reorder into digit order through this tile's (consumed) stage buffer
+        K *rk = S.k[sg];
+        V *rv = S.v[sg];
+#pragma unroll
+        for (int j = 0; j < kItems; ++j) {
+            if (wofs + j * 32 + lane < tile_n) {
+                const uint32_t lp = S.wcnt[w][uint32_t(k[j] >> shift) & dmask] + rank[j];
+                rk[lp] = k[j];
+                rv[lp] = v[j];
+            }
+        }
+        __syncthreads();
+        // ---- coalesced write-out: consecutive slots of one digit go to consecutive addresses
+        auto put = [&](uint32_t i) {
+            const K kk = rk[i];
+            const uint32_t g = S.gofs[uint32_t(kk >> shift) & dmask] + i;
+            kout[g] = kk;
+            vout[g] = rv[i];
+        };
+        if (tile_n == kTile) {
+#pragma unroll
+            for (int j = 0; j < kItems; ++j) put(j * kT + tid);
+        } else {
+            for (uint32_t i = tid; i < tile_n; i += kT) put(i);
+        }
+        __syncthreads();  // buffer sg, wcnt and gofs free for the next tiles
     }
 }
 
-template <class K>
-constexpr uint64_t tile_items() {
-    return uint64_t(kT) * Cfg<K>::kItems;
+// Digit width: 9 bits when that saves a pass over 8 (26-bit seed codes: 3 passes
+// instead of 4), else 8; 10-bit digits measured slower (more ballots, shorter digit
+// runs per tile) and are used only when g_opt.radix_bits pins them.
+int pick_digit_bits(int bits) {
+    if (g_opt.radix_bits >= 8 && g_opt.radix_bits <= 10) return int(g_opt.radix_bits);
+    return (bits + 8) / 9 < (bits + 7) / 8 ? 9 : 8;
 }
 
-template <class K>
-size_t scratch_bytes(uint64_t n, int passes) {
-    const uint64_t tiles = (n + tile_items<K>() - 1) / tile_items<K>();
-    return (size_t(passes) * kBins + 16 + size_t(passes) * tiles * kBins) * sizeof(uint32_t);
+constexpr int kMaxChunks = 148 * 8;  // >= SMs x resident scatter CTAs
+
+template <class K, int RB>
+cudaError_t radix_sort_rb(K *k0, uint32_t *v0, K *k1, uint32_t *v1, uint64_t n, int bits, void *scratch,
+                          cudaStream_t s, bool *in_alt) {
+    constexpr int kBins = 1 << RB;
+    const int passes = (bits + RB - 1) / RB;
+    const size_t smem = sizeof(ScatterSmem<K, uint32_t, RB>);
+    static int grid_cap = 0;  // per instantiation: resident scatter CTAs on the whole GPU
+    cudaError_t e;
+    if (!grid_cap) {
+        e = cudaFuncSetAttribute(k_scatter<K, uint32_t, RB>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+        if (e != cudaSuccess) return e;
+        e = cudaFuncSetAttribute(k_scatter<K, uint32_t, RB>, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+        if (e != cudaSuccess) return e;
+        int per_sm = 0;
+        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_scatter<K, uint32_t, RB>, kT, smem);
+        if (e != cudaSuccess) return e;
+        grid_cap = (per_sm > 0 ? per_sm : 1) * num_sms();
+        if (grid_cap > kMaxChunks) grid_cap = kMaxChunks;
+    }
+    Chunking ch;
+    ch.n = n;
+    ch.tiles = (n + tile_items<K>() - 1) / tile_items<K>();
+    ch.chunks = uint32_t(ch.tiles < uint64_t(grid_cap) ? ch.tiles : uint64_t(grid_cap));
+    ch.tpc = (ch.tiles + ch.chunks - 1) / ch.chunks;
+    ch.chunks = uint32_t((ch.tiles + ch.tpc - 1) / ch.tpc);  // no empty chunk
+    uint32_t *totals = static_cast<uint32_t *>(scratch);  // [passes][kBins]
+    uint32_t *counts = totals + size_t(passes) * kBins;     // [kBins][chunks]
+    uint32_t *offs = counts + size_t(ch.chunks) * kBins;    // [kBins][chunks]
+    e = cudaMemsetAsync(totals, 0, size_t(passes) * kBins * sizeof(uint32_t), s);
+    if (e != cudaSuccess) return e;
+    K *ka = k0, *kb = k1;
+    uint32_t *va = v0, *vb = v1;
+    for (int p = 0; p < passes; ++p) {
+        const int dbits = (p == passes - 1) ? bits - RB * p : RB;
+        uint32_t *tot = totals + size_t(p) * kBins;
+        k_chunk_hist<K, RB><<<ch.chunks, kT, 0, s>>>(ka, ch, RB * p, dbits, counts, tot);
+        k_chunk_scan<RB><<<kBins / kWarps, kT, 0, s>>>(counts, tot, ch.chunks, offs);
+        k_scatter<K, uint32_t, RB><<<ch.chunks, kT, smem, s>>>(ka, va, kb, vb, ch, RB * p, dbits, offs);
+        note_launch(3);
+        std::swap(ka, kb);
+        std::swap(va, vb);
+        *in_alt = !*in_alt;
+    }
+    return cudaGetLastError();
 }
 
 template <class K>
@@ -246,46 +424,19 @@ cudaError_t radix_sort(K *k0, uint32_t *v0, K *k1, uint32_t *v1, uint64_t n, int
     if (n <= 1 || bits <= 0) return cudaSuccess;
     if (!scratch) return cudaErrorInvalidValue;
     if (bits > int(8 * sizeof(K))) bits = int(8 * sizeof(K));
-    const int passes = (bits + 7) / 8;
-    const uint64_t tiles = (n + tile_items<K>() - 1) / tile_items<K>();
-    uint32_t *hist = static_cast<uint32_t *>(scratch);
-    unsigned int *ctr = hist + passes * kBins;  // one tile counter per pass
-    uint32_t *status = ctr + 16;
-    cudaError_t e = cudaMemsetAsync(scratch, 0, scratch_bytes<K>(n, passes), s);
-    if (e != cudaSuccess) return e;
-    const uint64_t hblocks = (n + kHT * 8 - 1) / (kHT * 8);  // >= 8 items per thread
-    const int hgrid = int(hblocks < uint64_t(num_sms() * 6) ? hblocks : uint64_t(num_sms() * 6));
-    k_hist_all<K><<<hgrid, kHT, 0, s>>>(k0, n, passes, hist);
-    k_hist_scan<<<1, kT, 0, s>>>(hist, passes);
-    note_launch(2);
-    const size_t smem = sizeof(SweepSmem<K, uint32_t>);
-    static bool attr_set = false;  // per instantiation
-    if (!attr_set) {
-        e = cudaFuncSetAttribute(k_onesweep<K, uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
-        if (e != cudaSuccess) return e;
-        e = cudaFuncSetAttribute(k_onesweep<K, uint32_t>, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
-        if (e != cudaSuccess) return e;
-        attr_set = true;
+    if (uint64_t(n) >= (uint64_t(1) << 32)) return cudaErrorInvalidValue;  // 32-bit offsets
+    switch (pick_digit_bits(bits)) {
+        case 9: return radix_sort_rb<K, 9>(k0, v0, k1, v1, n, bits, scratch, s, in_alt);
+        case 10: return radix_sort_rb<K, 10>(k0, v0, k1, v1, n, bits, scratch, s, in_alt);
+        default: return radix_sort_rb<K, 8>(k0, v0, k1, v1, n, bits, scratch, s, in_alt);
     }
-    K *ka = k0, *kb = k1;
-    uint32_t *va = v0, *vb = v1;
-    for (int p = 0; p < passes; ++p) {
-        const int dbits = (p == passes - 1) ? bits - 8 * p : 8;
-        k_onesweep<K, uint32_t><<<unsigned(tiles), kT, smem, s>>>(ka, va, kb, vb, n, 8 * p, dbits, hist + p * kBins,
-                                                                  status + uint64_t(p) * tiles * kBins, ctr + p);
-        note_launch();
-        std::swap(ka, kb);
-        std::swap(va, vb);
-        *in_alt = !*in_alt;
-    }
-    return cudaGetLastError();
 }
 
 }  // namespace
 
-size_t radix_scratch_bytes(uint64_t n) {
-    const size_t a = scratch_bytes<uint32_t>(n, 8), b = scratch_bytes<uint64_t>(n, 8);
-    return a > b ? a : b;
+size_t radix_scratch_bytes(uint64_t n) {  // totals of every pass + counts + offsets, at the widest digit
+    (void)n;
+    return size_t(8 * 1024 + 2 * size_t(kMaxChunks) * 1024) * sizeof(uint32_t);
 }
 
 cudaError_t radix_sort_u32(uint32_t *k0, uint32_t *v0, uint32_t *k1, uint32_t *v1, uint64_t n, int bits,

@@ -21,7 +21,8 @@ import os
 import numpy as np
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "libgpumem.so")
+# GPUMEM_LIB: an alternative build of the same library (tuning experiments, tools/variants.py)
+LIB_PATH = os.environ.get("GPUMEM_LIB") or os.path.join(_PKG, "libgpumem.so")
 if not os.path.exists(LIB_PATH):
     raise ImportError(f"{LIB_PATH} is missing: build it with `python -m paper_conf_ipps_abu_dolehkac14_b200._build` "
                       "(the MEM path is CUDA-only; there is no CPU fallback)")

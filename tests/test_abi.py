@@ -52,7 +52,7 @@ def test_library_holds_sm100a_code(lib_path):
     sass = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "-sass", lib_path], capture_output=True,
                           text=True).stdout
     for k in ("k_pack", "k_find", "k_heavy", "k_coop", "k_seed_codes", "k_ptrs_fill", "k_seed_recs",
-              "k_onesweep", "k_hist_all", "k_revcomp", "k_contained"):
+              "k_chunk_hist", "k_chunk_scan", "k_scatter", "k_revcomp", "k_contained"):
         assert k in sass, k
 
 
@@ -84,5 +84,7 @@ def test_errors_without_gpu_are_clean(lib_path):
     assert lib.gpumem_find_mems(None, None, 0, 0, None, ctypes.byref(out)) == 1
     assert lib.gpumem_set_option(b"nope", 1) == 1
     assert lib.gpumem_set_option(b"find_spill", 64) == 0
+    assert lib.gpumem_set_option(b"radix_bits", 7) == 1 and lib.gpumem_set_option(b"radix_bits", 11) == 1
+    assert lib.gpumem_set_option(b"radix_bits", 0) == 0
     lib.gpumem_free(None)
     assert gpumem.version()

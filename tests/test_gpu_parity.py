@@ -23,7 +23,7 @@ from paper_conf_ipps_abu_dolehkac14_b200 import gpumem  # noqa: E402
 def _default_options():
     yield
     for k, v in (("find_grid", 0), ("find_spill", 64), ("out_capacity", 0), ("use_bitmap", 1), ("static_lb", 0),
-                 ("sort_impl", 1)):
+                 ("sort_impl", 1), ("radix_bits", 0)):
         gpumem.set_option(k, v)
 
 
@@ -197,12 +197,12 @@ def test_overflow_retry_grid_spill_and_bitmap_invariance():
     base = gpu_mems(P.R, P.Q, P.L, P.ls)
     assert np.array_equal(base, want)
     for opt, vals in (("out_capacity", [1, 100]), ("find_grid", [1, 3, 148]), ("find_spill", [1, 2, 10**9]),
-                      ("use_bitmap", [0]), ("static_lb", [1]), ("sort_impl", [0])):
+                      ("use_bitmap", [0]), ("static_lb", [1]), ("sort_impl", [0]), ("radix_bits", [8, 9, 10])):
         for v in vals:
             gpumem.set_option(opt, v)
             assert np.array_equal(gpu_mems(P.R, P.Q, P.L, P.ls), want), (opt, v)
         gpumem.set_option(opt, {"out_capacity": 0, "find_grid": 0, "find_spill": 64, "use_bitmap": 1,
-                                "static_lb": 0, "sort_impl": 1}[opt])
+                                "static_lb": 0, "sort_impl": 1, "radix_bits": 0}[opt])
 
 
 def test_seed_length_and_step_invariance():
