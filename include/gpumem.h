@@ -67,7 +67,7 @@ typedef struct {
  *                   0: `bases` is host memory, copied to the device inside the call
  *                      (async if pinned) -- the copy is part of this call's stream work.
  *  Layout of the result: uint64 words, base i in bits [63-2(i%32), 62-2(i%32)] of
- *  word i/32 (first base most significant), 2 zero words of padding after the last.
+ *  word i/32 (first base most significant), 4 zero words of padding after the last.
  *  Async. Alphabet validation runs on the GPU; its verdict is reported by
  *  gpumem_seq_check() and by gpumem_find_mems() (which synchronises anyway).
  *  n == 0 is allowed (empty sequence). n >= 2^32 -> GPUMEM_ERR_RANGE.
@@ -194,7 +194,9 @@ gpumem_status gpumem_set_allocator(void *(*alloc_fn)(size_t bytes, void *cuda_st
  *                     force the overflow-and-retry path in tests)
  *  "use_bitmap"       1 (default) probe the rank words + bucket table, 0 probe ptrs only
  *  "static_lb"        1: no hit redistribution across lanes (load-balancing ablation)
- *  "sort_impl"        1 (default) stable LSD onesweep radix sort, 0 MSD bucket sort
+ *  "sort_impl"        output sort: 0 (default) auto by size, 1 stable LSD radix sort,
+ *                     2 MSD bucket sort
+ *  "index_msd"        index sort: 0 (default) stable LSD radix, 1 MSD bucket sort
  *  "radix_bits"       LSD digit width: 0 (default) = 9 bits when that saves a pass, else 8;
  *                     or pinned to 8, 9, 10; anything else is GPUMEM_ERR_ARG
  * Unknown names are GPUMEM_ERR_ARG. */

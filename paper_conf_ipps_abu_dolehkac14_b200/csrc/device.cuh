@@ -4,7 +4,7 @@
 // G=10 T=11): base i sits in bits [63-2(i%32), 62-2(i%32)] of word i/32, so the
 // first base of a word is its most significant pair and a 64-bit window of 32
 // consecutive bases starting anywhere is a funnel shift of two words. Every
-// sequence carries two zero words of padding after its last word; bases past
+// sequence carries four zero words of padding after its last word; bases past
 // the end read as 'A' (00), so every compare is clamped by the caller to the
 // sequence ends (an end counts as a mismatch, reading R3).
 #pragma once

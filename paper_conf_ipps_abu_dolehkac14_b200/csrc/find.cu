@@ -51,7 +51,10 @@ constexpr int kOutBuf = 64;
 constexpr uint32_t kUnresolved = 0xffffffffu;
 constexpr uint32_t kLaneCap = 4096;       // bases one lane extends before the warp takes over
 
+constexpr int kDQ = 64;                   // deferred-extension queue entries per warp
+
 struct WarpSmem {
+    uint4 dq[kDQ];                        // {p, q, e (or kUnresolved), 0}: hits needing global extension
     uint64_t qw[kQW];
     uint32_t e_beg[kChunk];
     uint32_t e_off[kChunk + 1];
@@ -83,23 +86,93 @@ struct Hit {
 
 enum : int { kDrop = 0, kDefer = 1, kEmit = 2 };
 
+// Extension rounds: kRW consecutive 32-base windows per round, so a round loads kRW + 1
+// words of each sequence at once (independent loads, one memory latency) instead of one
+// dependent pair of loads per 32 bases. The first mismatching window decides.
+#ifndef GM_KRW
+#define GM_KRW 2
+#endif
+constexpr int kRW = GM_KRW;
+
+__device__ __forceinline__ uint64_t funnel(uint64_t hi, uint64_t lo, uint32_t sh) {  // sh even, 0..62
+    return (hi << sh) | ((lo >> 1) >> (63 - sh));
+}
+
+// Equal bases of R[a + f ..) and Q[b + f ..), the first f known equal; clamped to lim.
+// kUnresolved when the run passes `cap` (the lane hands it to the warp).
+__device__ __forceinline__ uint32_t ext_right(const uint64_t *__restrict__ R, const uint64_t *__restrict__ Q,
+                                              uint64_t a, uint64_t b, uint32_t f, uint32_t lim, uint32_t cap) {
+    while (f < lim) {
+        if (f >= cap) return kUnresolved;
+        const uint64_t x = a + f, y = b + f;  // x < |R|, y < |Q|: words x/32 + kRW are padding at worst
+        const uint64_t *pr = R + (x >> 5), *pq = Q + (y >> 5);
+        const uint32_t sr = uint32_t(x & 31) * 2, sq = uint32_t(y & 31) * 2;
+        uint64_t wr[kRW + 1], wq[kRW + 1];
+#pragma unroll
+        for (int k = 0; k <= kRW; ++k) {
+            wr[k] = __ldg(pr + k);
+            wq[k] = __ldg(pq + k);
+        }
+        uint32_t run = 32 * kRW;
+#pragma unroll
+        for (int k = kRW - 1; k >= 0; --k) {  // nearest mismatching window assigned last
+            const uint64_t d = funnel(wr[k], wr[k + 1], sr) ^ funnel(wq[k], wq[k + 1], sq);
+            if (d) run = 32u * k + (uint32_t(__clzll(d)) >> 1);
+        }
+        f += run;
+        if (run < 32 * kRW) break;
+    }
+    return min(f, lim);
+}
+
+// Equal bases leftwards of the exclusive ends a - e (R) and b - e (Q), the first e known
+// equal; clamped to lim (lim <= min(a, b), so no base before 0 is ever counted).
+__device__ __forceinline__ uint32_t ext_left(const uint64_t *__restrict__ R, const uint64_t *__restrict__ Q,
+                                             uint64_t a, uint64_t b, uint32_t e, uint32_t lim, uint32_t cap) {
+    while (e < lim) {
+        if (e >= cap) return kUnresolved;
+        const uint64_t x = a - e, y = b - e;
+        uint32_t run;
+        if (x >= 32 * kRW && y >= 32 * kRW) {
+            const uint64_t xs = x - 32 * kRW, ys = y - 32 * kRW;  // window k covers [xs + 32k, xs + 32k + 32)
+            const uint64_t *pr = R + (xs >> 5), *pq = Q + (ys >> 5);
+            const uint32_t sr = uint32_t(xs & 31) * 2, sq = uint32_t(ys & 31) * 2;
+            uint64_t wr[kRW + 1], wq[kRW + 1];
+#pragma unroll
+            for (int k = 0; k <= kRW; ++k) {
+                wr[k] = __ldg(pr + k);
+                wq[k] = __ldg(pq + k);
+            }
+            run = 32 * kRW;
+#pragma unroll
+            for (int k = 0; k < kRW; ++k) {  // nearest (k = kRW - 1) mismatching window assigned last
+                const uint64_t d = funnel(wr[k], wr[k + 1], sr) ^ funnel(wq[k], wq[k + 1], sq);
+                if (d) run = 32u * (kRW - 1 - k) + ((uint32_t(__ffsll(d)) - 1) >> 1);
+            }
+            e += run;
+            if (run < 32 * kRW) break;
+        } else {  // near the start of R or Q: one window at a time (zero-filled before 0)
+            run = trail_eq(win_back(R, x) ^ win_back(Q, y));
+            e += run;
+            if (run < 32) break;
+        }
+    }
+    return min(e, lim);
+}
+
 // Decide one hit: seed of R at p equals seed of Q at q. rleft = R[p-16, p) (base p-1
 // lowest), rright = R[p+ls, p+ls+32) (first base highest); qleft/qright likewise for Q.
-// Extensions beyond the record use global windows, at most kLaneCap bases per lane;
-// a longer one returns kDefer and goes to the coop queue (k_coop).
+// Extensions beyond the record use global multi-window rounds, at most kLaneCap bases
+// per lane; a longer one returns kDefer and goes to the coop queue (k_coop).
 __device__ __forceinline__ int decide(const FindParams &P, uint32_t p, uint32_t rleft, uint64_t rright,
                                       uint32_t q, uint32_t qleft, uint64_t qright, Hit &out) {
     // A7: left extension, capped at step
     const uint32_t lim = min(P.step, min(p, q));
     const uint32_t xl = rleft ^ qleft;
     uint32_t e = xl ? uint32_t(__ffs(int(xl)) - 1) >> 1 : 16u;
-    if (e == 16) {
-        while (e < lim) {
-            if (e >= kLaneCap) return kDefer;
-            const uint32_t run = trail_eq(win_back(P.R, p - e) ^ win_back(P.Q, q - e));
-            e += run;
-            if (run < 32) break;
-        }
+    if (e == 16 && lim > 16) {
+        e = ext_left(P.R, P.Q, p, q, 16, lim, kLaneCap);
+        if (e == kUnresolved) return kDefer;
     }
     e = min(e, lim);
     if (e == P.step) return kDrop;                         // not the canonical (leftmost) seed
@@ -109,17 +182,71 @@ __device__ __forceinline__ int decide(const FindParams &P, uint32_t p, uint32_t 
     const uint32_t a = p + P.ls, b = q + P.ls;
     const uint32_t lim_r = min(uint32_t(P.nR) - a, uint32_t(P.nQ) - b);
     uint32_t f = lead_eq(rright ^ qright);
-    if (f == 32) {
-        while (f < lim_r) {
-            if (f >= kLaneCap) return kDefer;
-            const uint32_t run = lead_eq(win_fwd(P.R, uint64_t(a) + f) ^ win_fwd(P.Q, uint64_t(b) + f));
-            f += run;
-            if (run < 32) break;
-        }
+    if (f == 32 && lim_r > 32) {
+        f = ext_right(P.R, P.Q, a, b, 32, lim_r, kLaneCap);
+        if (f == kUnresolved) return kDefer;
     }
     f = min(f, lim_r);
     const uint32_t lam = e + P.ls + f;
     if (lam < P.L) return kDrop;                           // A9
+    out.key = (uint64_t(p - e) << P.qbits) | qs;
+    out.len = lam;
+    return kEmit;
+}
+
+// The record-only part of decide(): kDrop / kEmit when the 16 + 32 flank bases settle
+// the hit, else kExt with e_out = the left extension if the record settled it, or
+// kUnresolved. kExt hits are queued per warp and finished 32 at a time by
+// decide_deferred(), so the (rare, long) global-memory extensions run with all lanes
+// busy instead of stalling a whole warp round for one lane.
+enum : int { kExt = 3 };
+__device__ __forceinline__ int decide_rec(const FindParams &P, uint32_t p, uint32_t rleft, uint64_t rright,
+                                          uint32_t q, uint32_t qleft, uint64_t qright, Hit &out, uint32_t &e_out) {
+    const uint32_t lim = min(P.step, min(p, q));
+    const uint32_t xl = rleft ^ qleft;
+    uint32_t e = xl ? uint32_t(__ffs(int(xl)) - 1) >> 1 : 16u;
+    if (e == 16 && lim > 16) {
+        e_out = kUnresolved;
+        return kExt;
+    }
+    e = min(e, lim);
+    if (e == P.step) return kDrop;
+    const uint32_t qs = q - e;
+    if (qs < P.own_lo || qs >= P.own_hi) return kDrop;
+    const uint32_t a = p + P.ls, b = q + P.ls;
+    const uint32_t lim_r = min(uint32_t(P.nR) - a, uint32_t(P.nQ) - b);
+    uint32_t f = lead_eq(rright ^ qright);
+    if (f == 32 && lim_r > 32) {
+        e_out = e;
+        return kExt;
+    }
+    f = min(f, lim_r);
+    const uint32_t lam = e + P.ls + f;
+    if (lam < P.L) return kDrop;
+    out.key = (uint64_t(p - e) << P.qbits) | qs;
+    out.len = lam;
+    return kEmit;
+}
+
+// The rest of decide() for a queued hit, from global memory (16 left bases already known
+// equal when e_in == kUnresolved).
+__device__ __forceinline__ int decide_deferred(const FindParams &P, uint32_t p, uint32_t q, uint32_t e_in, Hit &out) {
+    const uint32_t lim = min(P.step, min(p, q));
+    uint32_t e = e_in;
+    if (e == kUnresolved) {
+        e = ext_left(P.R, P.Q, p, q, 16, lim, kLaneCap);
+        if (e == kUnresolved) return kDefer;
+    }
+    e = min(e, lim);
+    if (e == P.step) return kDrop;
+    const uint32_t qs = q - e;
+    if (qs < P.own_lo || qs >= P.own_hi) return kDrop;
+    const uint32_t a = p + P.ls, b = q + P.ls;
+    const uint32_t lim_r = min(uint32_t(P.nR) - a, uint32_t(P.nQ) - b);
+    uint32_t f = ext_right(P.R, P.Q, a, b, 0, lim_r, kLaneCap);
+    if (f == kUnresolved) return kDefer;
+    const uint32_t lam = e + P.ls + f;
+    if (lam < P.L) return kDrop;
     out.key = (uint64_t(p - e) << P.qbits) | qs;
     out.len = lam;
     return kEmit;
@@ -278,13 +405,35 @@ __device__ __forceinline__ void load_rec(const uint4 *recs, uint32_t k, uint32_t
     right = (uint64_t(r.w) << 32) | r.z;
 }
 
+// One converged extension round: the last `take` (<= 32) queued hits, one per lane.
+__device__ __forceinline__ void drain_deferred(const FindParams &P, WarpSmem &s, uint32_t &nq, uint32_t &nbuf,
+                                               uint32_t take) {
+    const int lane = threadIdx.x & 31;
+    int verdict = kDrop;
+    Hit out{0, 0};
+    uint32_t p = 0, q = 0;
+    if (uint32_t(lane) < take) {
+        const uint4 d = s.dq[nq - take + lane];
+        p = d.x;
+        q = d.y;
+        verdict = decide_deferred(P, p, q, d.z, out);
+    }
+    __syncwarp();
+    nq -= take;
+    push_coop(P, verdict, p, q);
+    warp_emit(P, s, nbuf, verdict == kEmit, out, false);
+}
+
+#ifndef GM_FIND_MINB
+#define GM_FIND_MINB 4
+#endif
 template <bool kStatic, bool kHints>
-__global__ void __launch_bounds__(kT) k_find(const FindParams P) {
+__global__ void __launch_bounds__(kT, GM_FIND_MINB) k_find(const FindParams P) {
     __shared__ WarpSmem smem[kWarps];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     WarpSmem &s = smem[wid];
     const uint32_t sh = 64 - 2 * P.ls;
-    uint32_t nbuf = 0;
+    uint32_t nbuf = 0, nq = 0;
     unsigned long long st_e = 0, st_h = 0;
     QStage qs{s.qw, 0};
     // L2 priorities: lookup tables stay, streamed data goes first (records only when
@@ -423,7 +572,7 @@ __global__ void __launch_bounds__(kT) k_find(const FindParams P) {
                     const bool has = kStatic ? rd < n_h : h < H;
                     int verdict = kDrop;
                     Hit out{0, 0};
-                    uint32_t p = 0, q = 0;
+                    uint32_t p = 0, q = 0, e_rec = 0;
                     if (has) {
                         uint32_t lo = 0, hi = E;  // largest entry i with e_off[i] <= h
                         while (hi - lo > 1) {
@@ -434,15 +583,23 @@ __global__ void __launch_bounds__(kT) k_find(const FindParams P) {
                         uint32_t rl;
                         uint64_t rr;
                         load_rec(P.recs, s.e_beg[lo] + (h - s.e_off[lo]), p, rl, rr, kHints ? 1 : -1);
-                        verdict = decide(P, p, rl, rr, q, qs.back16(q), qs.fwd(q + P.ls), out);
+                        verdict = decide_rec(P, p, rl, rr, q, qs.back16(q), qs.fwd(q + P.ls), out, e_rec);
                     }
-                    push_coop(P, verdict, p, q);
+                    // hits the records cannot settle wait in the warp's queue
+                    const unsigned need = __ballot_sync(0xffffffffu, verdict == kExt);
+                    if (need) {
+                        if (verdict == kExt) s.dq[nq + __popc(need & lanemask_lt())] = make_uint4(p, q, e_rec, 0u);
+                        nq += __popc(need);
+                        __syncwarp();
+                    }
                     warp_emit(P, s, nbuf, verdict == kEmit, out, false);
+                    if (nq >= 32) drain_deferred(P, s, nq, nbuf, 32);
                 }
             }
             __syncwarp();
         }
     }
+    if (nq) drain_deferred(P, s, nq, nbuf, nq);
     warp_emit(P, s, nbuf, false, Hit{0, 0}, true);
     if (lane == 0 && st_e) {
         atomicAdd(&P.stats[0], st_e);

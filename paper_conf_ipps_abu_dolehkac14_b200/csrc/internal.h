@@ -15,7 +15,9 @@ struct Options {
     int64_t out_capacity = 0;    // 0 = automatic
     int64_t use_bitmap = 1;      // 1: rank-word probe + compact bucket table; 0: read the dense ptrs
     int64_t static_lb = 0;       // 1: each lane processes its own positions' hits (LB ablation)
-    int64_t sort_impl = 1;       // 0: MSD bucket sort (unique keys; measured slower), 1: stable LSD onesweep radix
+    int64_t sort_impl = 0;       // output sort: 0 = auto (MSD below kMsdMaxN keys, else LSD), 1 = stable LSD radix
+                                 // (radix.cu), 2 = MSD bucket sort (msd.cu)
+    int64_t index_msd = 0;       // index sort: 1 = MSD bucket sort of (code << 32 | p), 0 = stable LSD radix
     int64_t radix_bits = 0;      // LSD digit width: 0 = 9 bits if that saves a pass else 8; or pinned 8, 9, 10
 };
 extern Options g_opt;
@@ -53,9 +55,11 @@ cudaError_t radix_sort_u64(uint64_t *k0, uint32_t *v0, uint64_t *k1, uint32_t *v
                            void *scratch, cudaStream_t s, bool *in_alt);
 size_t radix_scratch_bytes(uint64_t n);
 
-// MSD bucket sort of unique u64 keys (+ optional u32 values), in place (msd.cu).
+// MSD bucket sort of unique u64 keys (+ optional u32 values), in place, or written as
+// triples {key >> qbits, key & qmask, val} when trip != null (msd.cu).
 size_t msd_scratch_bytes(uint64_t n);
-cudaError_t msd_sort(uint64_t *keys, uint32_t *vals, uint64_t n, int bits, void *scratch, cudaStream_t s);
+cudaError_t msd_sort(uint64_t *keys, uint32_t *vals, uint64_t n, int bits, void *scratch, cudaStream_t s,
+                     gpumem_triple *trip = nullptr, uint32_t qbits = 0);
 // keys[i] = (codes[i] << 32) | locs[i] and back (sort.cu)
 cudaError_t launch_join_keys(const uint32_t *codes, const uint32_t *locs, uint64_t n, uint64_t *keys, cudaStream_t s);
 cudaError_t launch_split_keys(const uint64_t *keys, uint64_t n, uint32_t *codes, uint32_t *locs, cudaStream_t s);

@@ -1,134 +1,312 @@
 // msd.cu -- MSD bucket sort for unique 64-bit keys (+ optional 32-bit values).
 //
 // Used where the keys are unique, so stability is irrelevant:
-//  * the index: keys (seed code << 32 | location) -- sorting them groups the sampled
-//    locations by seed with ascending locations inside each seed, i.e. Alg. 1 steps
-//    1-4 in one sort;
-//  * the output: keys (r << qbits | q) with len as value.
-// One pass scatters every key into one of 2^B buckets by its top B bits (an atomic
-// cursor per bucket; order inside a bucket is arbitrary), then each bucket is sorted
-// by one CTA: in shared memory (bitonic) when it holds <= kLocal keys, otherwise by a
-// CTA-level LSD radix over the bucket in global memory. B is chosen so that buckets
-// average ~1K keys, which keeps a 13M-key sort to two passes over the data.
+//  * the output: keys (r << qbits | q) with len as value; the
+//    last kernel writes gpumem_triple {r, q, len} directly;
+//  * the index (sort_impl = 0 option): keys (seed code << 32 | location) -- sorting them
+//    groups the sampled locations by seed, ascending inside each seed, i.e. Alg. 1
+//    steps 1-4 in one sort.
+// Two passes over the data:
+//  k_bp_hist     chunk c (one CTA per SM, a contiguous run of the input) counts the
+//                top B key bits (2^B <= 16384 buckets) in a shared-memory histogram;
+//  k_bp_colscan  per bucket: exclusive prefix over the chunks + the bucket total;
+//  k_bs_scan     one CTA: bucket offsets;
+//  k_bp_scatter  chunk c moves its keys to its private range of each bucket (order
+//                inside a chunk's range arbitrary: shared-memory atomic cursors; the
+//                keys are unique and get fully sorted next);
+//  k_bs_local    CTA s sorts the buckets that start in slots [s * kSeg, (s + 1) * kSeg)
+//                -- a contiguous segment of whole buckets, so sorting the segment by
+//                the full key sorts each of them -- with an LSD radix sort in shared
+//                memory (digits that are equal across the segment are skipped), and
+//                writes the result (keys/values, or triples);
+//  k_bs_big      buckets too large for shared memory (adversarial inputs: e.g. one
+//                r with 10^5 MEMs) get a CTA-level LSD radix in global memory.
+// No per-element global atomics anywhere. B is chosen so that buckets average ~512 keys.
 #include "internal.h"
 #include "device.cuh"
 
 namespace gm {
 namespace {
 
-constexpr int kT = 256;
+constexpr int kT = 256;                          // threads of k_bs_big
 constexpr int kWarps = kT / 32;
-constexpr uint32_t kLocal = 4096;   // keys sorted in shared memory per bucket
-constexpr int kMaxB = 14;
+constexpr int kPT = 1024;                        // threads of the chunk kernels
+constexpr int kLT = 512;                         // threads of k_bs_local
+constexpr int kLWarps = kLT / 32;
+constexpr int kItems = 8;                        // keys per thread in k_bs_local
+constexpr uint32_t kLocal = kLT * kItems;        // most keys one CTA sorts in shared memory (4096)
+constexpr uint32_t kSeg = kLocal / 2;            // segment spacing (slots)
+constexpr int kMaxB = 14;                        // 16384 buckets: a 64 KB shared histogram
 
-__global__ void __launch_bounds__(kT) k_msd_hist(const uint64_t *__restrict__ keys, uint64_t n, int shift,
-                                                 uint32_t nb, uint32_t *__restrict__ counts) {
+// chunk c = elements [c * cs, min((c + 1) * cs, n))
+__global__ void __launch_bounds__(kPT) k_bp_hist(const uint64_t *__restrict__ keys, uint64_t n, uint64_t cs,
+                                                 int shift, uint32_t nb, uint32_t *__restrict__ counts) {
     extern __shared__ uint32_t h[];
-    for (uint32_t i = threadIdx.x; i < nb; i += kT) h[i] = 0;
+    for (uint32_t i = threadIdx.x; i < nb; i += kPT) h[i] = 0;
     __syncthreads();
-    for (uint64_t i = uint64_t(blockIdx.x) * kT + threadIdx.x; i < n; i += uint64_t(gridDim.x) * kT)
-        atomicAdd(&h[uint32_t(keys[i] >> shift)], 1u);
+    const uint64_t b = uint64_t(blockIdx.x) * cs, e = min(b + cs, n);
+    for (uint64_t i = b + threadIdx.x; i < e; i += kPT) atomicAdd(&h[uint32_t(keys[i] >> shift)], 1u);
     __syncthreads();
-    for (uint32_t i = threadIdx.x; i < nb; i += kT)
-        if (h[i]) atomicAdd(counts + i, h[i]);
+    uint32_t *row = counts + uint64_t(blockIdx.x) * nb;  // chunk-major
+    for (uint32_t i = threadIdx.x; i < nb; i += kPT) row[i] = h[i];
 }
 
-// exclusive scan of counts[0..nb) -> offs[0..nb] and a copy in cursor[0..nb)
-__global__ void __launch_bounds__(kT) k_msd_scan(const uint32_t *__restrict__ counts, uint32_t nb,
-                                                 uint32_t *__restrict__ offs, uint32_t *__restrict__ cursor) {
-    __shared__ uint32_t ws[kWarps];
-    __shared__ uint32_t carry;
-    if (threadIdx.x == 0) carry = 0;
-    __syncthreads();
+// per bucket b (one thread): counts[c][b] -> exclusive prefix over c (in place); totals[b]
+__global__ void __launch_bounds__(256) k_bp_colscan(uint32_t *__restrict__ counts, uint32_t chunks, uint32_t nb,
+                                                    uint32_t *__restrict__ totals) {
+    const uint32_t b = blockIdx.x * 256 + threadIdx.x;
+    if (b >= nb) return;
+    uint32_t run = 0;
+    uint32_t c = 0;
+    for (; c + 8 <= chunks; c += 8) {  // independent loads in flight
+        uint32_t x[8];
+#pragma unroll
+        for (int j = 0; j < 8; ++j) x[j] = counts[uint64_t(c + j) * nb + b];
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+            counts[uint64_t(c + j) * nb + b] = run;
+            run += x[j];
+        }
+    }
+    for (; c < chunks; ++c) {
+        const uint32_t x = counts[uint64_t(c) * nb + b];
+        counts[uint64_t(c) * nb + b] = run;
+        run += x;
+    }
+    totals[b] = run;
+}
+
+// exclusive scan of totals[0..nb) -> offs[0..nb] (offs[nb] = the sum); each thread owns
+// a contiguous run of ceil(nb / 1024) entries
+__global__ void __launch_bounds__(1024) k_bs_scan(const uint32_t *__restrict__ totals, uint32_t nb,
+                                                  uint32_t *__restrict__ offs) {
+    __shared__ uint32_t ws[32];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-    for (uint32_t base = 0; base < nb; base += kT) {
-        const uint32_t i = base + threadIdx.x;
-        const uint32_t x = i < nb ? counts[i] : 0;
-        uint32_t inc = x;
+    const uint32_t per = (nb + 1023) / 1024;
+    const uint32_t i0 = threadIdx.x * per, i1 = min(i0 + per, nb);
+    uint32_t sum = 0;
+    for (uint32_t i = i0; i < i1; ++i) sum += totals[i];
+    uint32_t inc = sum;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
+        if (lane >= o) inc += y;
+    }
+    if (lane == 31) ws[w] = inc;
+    __syncthreads();
+    uint32_t run = inc - sum;
+    for (int k = 0; k < w; ++k) run += ws[k];
+    for (uint32_t i = i0; i < i1; ++i) {
+        offs[i] = run;
+        run += totals[i];
+    }
+    if (threadIdx.x == 1023) offs[nb] = run;
+}
+
+__global__ void __launch_bounds__(kPT) k_bp_scatter(const uint64_t *__restrict__ keys,
+                                                    const uint32_t *__restrict__ vals, uint64_t n, uint64_t cs,
+                                                    int shift, uint32_t nb, const uint32_t *__restrict__ rel,
+                                                    const uint32_t *__restrict__ offs, uint64_t *__restrict__ ok,
+                                                    uint32_t *__restrict__ ov) {
+    extern __shared__ uint32_t cur[];
+    const uint32_t *row = rel + uint64_t(blockIdx.x) * nb;
+    for (uint32_t i = threadIdx.x; i < nb; i += kPT) cur[i] = offs[i] + row[i];
+    __syncthreads();
+    const uint64_t b = uint64_t(blockIdx.x) * cs, e = min(b + cs, n);
+    for (uint64_t i = b + threadIdx.x; i < e; i += kPT) {
+        const uint64_t k = keys[i];
+        const uint32_t slot = atomicAdd(&cur[uint32_t(k >> shift)], 1u);
+        ok[slot] = k;
+        if (vals) ov[slot] = vals[i];
+    }
+}
+
+struct Out {
+    uint64_t *keys;          // generic result (in place of the input)
+    uint32_t *vals;          // may be null
+    gpumem_triple *trip;     // if set: triples {key >> qbits, key & qmask, val} instead
+    uint32_t qbits;
+    __device__ __forceinline__ void put(uint64_t i, uint64_t k, uint32_t v) const {
+        if (trip) {
+            gpumem_triple t;
+            t.r = uint32_t(k >> qbits);
+            t.q = uint32_t(k & ((1ull << qbits) - 1));
+            t.len = v;
+            trip[i] = t;
+        } else {
+            keys[i] = k;
+            if (vals) vals[i] = v;
+        }
+    }
+};
+
+// first bucket b in [0, nb] with offs[b] >= x
+__device__ __forceinline__ uint32_t first_at(const uint32_t *__restrict__ offs, uint32_t nb, uint64_t x) {
+    uint32_t lo = 0, hi = nb;
+    while (lo < hi) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (uint64_t(offs[mid]) < x) lo = mid + 1; else hi = mid;
+    }
+    return lo;
+}
+
+// Shared memory of k_bs_local: a ping-pong pair of key/value buffers and the per-warp
+// digit counters of one LSD pass.
+struct LocalSmem {
+    uint64_t k[2][kLocal];
+    uint32_t v[2][kLocal];
+    uint32_t wcnt[kLWarps][256];
+    uint32_t ws[kLWarps];
+    unsigned long long kor, kand;  // OR / AND of the keys: digits equal in all keys are skipped
+};
+
+// Lanes of the warp holding the same 8-bit digit (among valid lanes): one ballot per bit.
+__device__ __forceinline__ unsigned match8(uint32_t d, bool valid) {
+    unsigned peers = __ballot_sync(0xffffffffu, valid);
+#pragma unroll
+    for (int b = 0; b < 8; ++b) {
+        const bool bit = (d >> b) & 1u;
+        const unsigned m = __ballot_sync(0xffffffffu, bit);
+        peers &= bit ? m : ~m;
+    }
+    return peers;
+}
+
+// Sorts the m <= kLocal keys (with values) of [tk + lo, tk + lo + m) by their low `bits`
+// bits -- an LSD radix sort with 8-bit digits entirely in shared memory (stable ranks
+// from per-warp digit counters + ballot peers) -- and writes them to out[lo, lo + m).
+__device__ void smem_sort_write(LocalSmem &S, const uint64_t *__restrict__ tk, const uint32_t *__restrict__ tv,
+                                uint32_t lo, uint32_t m, int bits, const Out &out) {
+    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+    if (tid == 0) {
+        S.kor = 0ull;
+        S.kand = ~0ull;
+    }
+    __syncthreads();
+    unsigned long long kor = 0ull, kand = ~0ull;
+    for (uint32_t i = tid; i < m; i += kLT) {
+        const uint64_t x = tk[lo + i];
+        S.k[0][i] = x;
+        S.v[0][i] = tv[lo + i];
+        kor |= x;
+        kand &= x;
+    }
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+        kor |= __shfl_xor_sync(0xffffffffu, kor, o);
+        kand &= __shfl_xor_sync(0xffffffffu, kand, o);
+    }
+    if (lane == 0) {
+        atomicOr(&S.kor, kor);
+        atomicAnd(&S.kand, kand);
+    }
+    __syncthreads();
+    const uint64_t diff = S.kor ^ S.kand;
+    int cur = 0;
+    const uint32_t wofs = uint32_t(w) * 32 * kItems;  // warp w owns slots [wofs, wofs + 32 kItems)
+    for (int sh = 0; sh < bits; sh += 8) {
+        if (((diff >> sh) & 255u) == 0) continue;  // same digit in every key: the pass is the identity
+#pragma unroll
+        for (int ww = 0; ww < kLWarps; ++ww) S.wcnt[ww][tid & 255] = 0;
+        __syncthreads();
+        uint64_t k[kItems];
+        uint32_t v[kItems], rank[kItems];
+        unsigned peers[kItems];
+#pragma unroll
+        for (int j = 0; j < kItems; ++j) {
+            const uint32_t i = wofs + j * 32 + lane;
+            const bool valid = i < m;
+            k[j] = valid ? S.k[cur][i] : 0ull;
+            v[j] = valid ? S.v[cur][i] : 0u;
+            peers[j] = match8(uint32_t(k[j] >> sh) & 255u, valid);
+        }
+#pragma unroll
+        for (int j = 0; j < kItems; ++j) {
+            const bool valid = wofs + j * 32 + lane < m;
+            const uint32_t d = uint32_t(k[j] >> sh) & 255u;
+            const uint32_t b0 = valid ? S.wcnt[w][d] : 0u;
+            rank[j] = b0 + __popc(peers[j] & lanemask_lt());
+            __syncwarp();
+            if (valid && lane == __ffs(peers[j]) - 1) S.wcnt[w][d] = b0 + __popc(peers[j]);
+            __syncwarp();
+        }
+        __syncthreads();
+        // digit-major, warp-minor exclusive offsets (thread tid < 256 owns digit tid)
+        uint32_t xw[kLWarps], c = 0;
+        if (tid < 256) {
+#pragma unroll
+            for (int ww = 0; ww < kLWarps; ++ww) {
+                xw[ww] = S.wcnt[ww][tid];
+                c += xw[ww];
+            }
+        }
+        uint32_t inc = c;
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
             const uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
             if (lane >= o) inc += y;
         }
-        if (lane == 31) ws[w] = inc;
+        if (lane == 31) S.ws[w] = inc;
         __syncthreads();
-        uint32_t pre = carry, tot = carry;
-        for (int k = 0; k < kWarps; ++k) {
-            if (k < w) pre += ws[k];
-            tot += ws[k];
-        }
-        if (i < nb) offs[i] = cursor[i] = pre + inc - x;
-        __syncthreads();
-        if (threadIdx.x == 0) carry = tot;
-        __syncthreads();
-    }
-    if (threadIdx.x == 0) offs[nb] = carry;
-}
-
-__global__ void __launch_bounds__(kT) k_msd_scatter(const uint64_t *__restrict__ keys,
-                                                    const uint32_t *__restrict__ vals, uint64_t n, int shift,
-                                                    uint32_t *__restrict__ cursor, uint64_t *__restrict__ ok,
-                                                    uint32_t *__restrict__ ov) {
-    const uint64_t i = uint64_t(blockIdx.x) * kT + threadIdx.x;
-    if (i >= n) return;
-    const uint64_t k = keys[i];
-    const uint32_t slot = atomicAdd(cursor + uint32_t(k >> shift), 1u);
-    ok[slot] = k;
-    if (vals) ov[slot] = vals[i];
-}
-
-// One CTA per bucket: shared-memory bitonic sort when it fits, else defer to k_msd_big.
-__global__ void __launch_bounds__(kT) k_msd_local(const uint32_t *__restrict__ offs, uint32_t nb, uint64_t *keys,
-                                                  uint32_t *vals, uint32_t *big, unsigned int *n_big) {
-    extern __shared__ __align__(16) unsigned char smem[];
-    uint64_t *sk = reinterpret_cast<uint64_t *>(smem);
-    uint32_t *sv = reinterpret_cast<uint32_t *>(sk + kLocal);
-    for (uint32_t b = blockIdx.x; b < nb; b += gridDim.x) {
-        const uint32_t lo = offs[b], m = offs[b + 1] - lo;
-        if (m <= 1) continue;
-        if (m > kLocal) {
-            if (threadIdx.x == 0) big[atomicAdd(n_big, 1u)] = b;
-            continue;
-        }
-        uint32_t P = 2;
-        while (P < m) P <<= 1;
-        for (uint32_t j = threadIdx.x; j < P; j += kT) {
-            sk[j] = j < m ? keys[lo + j] : ~0ull;
-            if (vals) sv[j] = j < m ? vals[lo + j] : 0u;
-        }
-        __syncthreads();
-        for (uint32_t size = 2; size <= P; size <<= 1) {
-            for (uint32_t stride = size >> 1; stride; stride >>= 1) {
-                for (uint32_t j = threadIdx.x; j < P / 2; j += kT) {
-                    const uint32_t a = 2 * stride * (j / stride) + (j % stride), c = a + stride;
-                    const bool up = (a & size) == 0;
-                    const uint64_t x = sk[a], y = sk[c];
-                    if ((x > y) == up) {
-                        sk[a] = y;
-                        sk[c] = x;
-                        if (vals) {
-                            const uint32_t t = sv[a];
-                            sv[a] = sv[c];
-                            sv[c] = t;
-                        }
-                    }
-                }
-                __syncthreads();
+        if (tid < 256) {
+            uint32_t run = inc - c;
+            for (int i = 0; i < w; ++i) run += S.ws[i];
+#pragma unroll
+            for (int ww = 0; ww < kLWarps; ++ww) {
+                S.wcnt[ww][tid] = run;
+                run += xw[ww];
             }
         }
-        for (uint32_t j = threadIdx.x; j < m; j += kT) {
-            keys[lo + j] = sk[j];
-            if (vals) vals[lo + j] = sv[j];
-        }
         __syncthreads();
+#pragma unroll
+        for (int j = 0; j < kItems; ++j) {
+            if (wofs + j * 32 + lane < m) {
+                const uint32_t pos = S.wcnt[w][uint32_t(k[j] >> sh) & 255u] + rank[j];
+                S.k[cur ^ 1][pos] = k[j];
+                S.v[cur ^ 1][pos] = v[j];
+            }
+        }
+        cur ^= 1;
+        __syncthreads();
+    }
+    for (uint32_t i = tid; i < m; i += kLT) out.put(uint64_t(lo) + i, S.k[cur][i], S.v[cur][i]);
+    __syncthreads();
+}
+
+__global__ void __launch_bounds__(kLT, 2) k_bs_local(const uint32_t *__restrict__ offs, uint32_t nb, int bits,
+                                                 const uint64_t *__restrict__ tk, const uint32_t *__restrict__ tv,
+                                                 Out out, uint32_t *__restrict__ big, unsigned int *n_big) {
+    extern __shared__ __align__(16) unsigned char smem[];
+    LocalSmem &S = *reinterpret_cast<LocalSmem *>(smem);
+    __shared__ uint32_t s_b[2];
+    if (threadIdx.x == 0) s_b[0] = first_at(offs, nb, uint64_t(blockIdx.x) * kSeg);
+    if (threadIdx.x == 32) s_b[1] = first_at(offs, nb, uint64_t(blockIdx.x + 1) * kSeg);
+    __syncthreads();
+    const uint32_t b0 = s_b[0], b1 = s_b[1];
+    if (b0 >= b1) return;
+    const uint32_t lo = offs[b0], m = offs[b1] - lo;
+    if (m <= kLocal) {
+        // the segment's keys share no common prefix below the bucket bits in general:
+        // sort by all key bits (the bucket prefix bits then sort the buckets among themselves)
+        smem_sort_write(S, tk, tv, lo, m, bits, out);
+        return;
+    }
+    for (uint32_t b = b0; b < b1; ++b) {  // a large bucket in the segment: one bucket at a time
+        const uint32_t blo = offs[b], bm = offs[b + 1] - blo;
+        if (bm == 0) continue;
+        if (bm <= kLocal) {
+            smem_sort_write(S, tk, tv, blo, bm, bits, out);
+        } else if (threadIdx.x == 0) {
+            big[atomicAdd(n_big, 1u)] = b;
+        }
     }
 }
 
-// One CTA per oversized bucket: LSD radix (8-bit digits) over its low `bits` key bits,
-// ping-ponging with the same range of (tk, tv).
-__global__ void __launch_bounds__(kT) k_msd_big(const uint32_t *__restrict__ offs, const uint32_t *__restrict__ big,
-                                                const unsigned int *__restrict__ n_big, uint64_t *keys,
-                                                uint32_t *vals, uint64_t *tk, uint32_t *tv, int bits) {
+// One CTA per oversized bucket: LSD radix (8-bit digits) over the low `bits` key bits,
+// ping-ponging between (tk, tv) and (sk, sv) over the bucket's range; then written out.
+__global__ void __launch_bounds__(kT) k_bs_big(const uint32_t *__restrict__ offs, const uint32_t *__restrict__ big,
+                                               const unsigned int *__restrict__ n_big, uint64_t *tk, uint32_t *tv,
+                                               uint64_t *xk, uint32_t *xv, int bits, Out out) {
     __shared__ uint32_t hist[256];
     __shared__ uint32_t wcnt[kWarps][256];
     __shared__ uint32_t ws[kWarps];
@@ -138,11 +316,11 @@ __global__ void __launch_bounds__(kT) k_msd_big(const uint32_t *__restrict__ off
     for (unsigned li = blockIdx.x; li < nbig; li += gridDim.x) {
         const uint32_t b = big[li];
         const uint32_t lo = offs[b], m = offs[b + 1] - lo;
-        uint64_t *sk = keys + lo, *dk = tk + lo;
-        uint32_t *sv = vals ? vals + lo : nullptr, *dv = vals ? tv + lo : nullptr;
+        uint64_t *sk = tk + lo, *dk = xk + lo;
+        uint32_t *sv = tv + lo, *dv = xv + lo;
         for (int pass = 0; pass < passes; ++pass) {
             const int sh = 8 * pass;
-            for (int i = tid; i < 256; i += kT) hist[i] = 0;
+            hist[tid] = 0;
             __syncthreads();
             for (uint32_t j = tid; j < m; j += kT) atomicAdd(&hist[uint32_t(sk[j] >> sh) & 255u], 1u);
             __syncthreads();
@@ -165,7 +343,7 @@ __global__ void __launch_bounds__(kT) k_msd_big(const uint32_t *__restrict__ off
                 const uint32_t j = base + tid;
                 const bool valid = j < m;
                 const uint64_t x = valid ? sk[j] : 0ull;
-                const uint32_t xv = (valid && sv) ? sv[j] : 0u;
+                const uint32_t xv2 = valid ? sv[j] : 0u;
                 const uint32_t d = uint32_t(x >> sh) & 255u;
                 unsigned peers = __ballot_sync(0xffffffffu, valid);
 #pragma unroll
@@ -188,7 +366,7 @@ __global__ void __launch_bounds__(kT) k_msd_big(const uint32_t *__restrict__ off
                 if (valid) {
                     const uint32_t pos = hist[d] + wcnt[w][d] + __popc(peers & lanemask_lt());
                     dk[pos] = x;
-                    if (dv) dv[pos] = xv;
+                    dv[pos] = xv2;
                 }
                 __syncthreads();
                 hist[tid] += run;
@@ -202,73 +380,80 @@ __global__ void __launch_bounds__(kT) k_msd_big(const uint32_t *__restrict__ off
             dv = t2;
             __syncthreads();
         }
-        if (passes & 1) {
-            for (uint32_t j = tid; j < m; j += kT) {
-                keys[lo + j] = tk[lo + j];
-                if (vals) vals[lo + j] = tv[lo + j];
-            }
-        }
+        for (uint32_t j = tid; j < m; j += kT) out.put(uint64_t(lo) + j, sk[j], sv[j]);
         __syncthreads();
     }
 }
 
 int choose_b(uint64_t n, int bits) {
-    int B = 4;
-    while (B < kMaxB && (n >> (B + 10)) > 0) ++B;  // ~1K keys per bucket
+    int B = 1;
+    while (B < kMaxB && (n >> (B + 9)) > 0) ++B;  // ~512 keys per bucket
     return B < bits ? B : bits;
+}
+
+uint32_t n_chunks(uint64_t n) {
+    const uint64_t c = (n + 4095) / 4096;  // >= 4K keys per chunk
+    const uint64_t cap = uint64_t(num_sms());
+    return uint32_t(c < cap ? (c ? c : 1) : cap);
 }
 
 }  // namespace
 
 size_t msd_scratch_bytes(uint64_t n) {
     const uint64_t nb = 1ull << kMaxB;
-    return n * 8 + n * 4 + (nb + 1) * 4 * 3 + nb * 4 + 1024;
+    const uint64_t chunks = 1024;  // >= SMs
+    return n * 8 + n * 4 * 2 + chunks * nb * 4 + (nb + 1) * 4 * 2 + nb * 4 + 1024 + 8 * 256;
 }
 
-// Sorts (keys, vals) (vals may be null) of n unique keys whose significant bits are the
-// low `bits`. The result lands in (keys, vals) in place. `scratch` >= msd_scratch_bytes(n).
-cudaError_t msd_sort(uint64_t *keys, uint32_t *vals, uint64_t n, int bits, void *scratch, cudaStream_t s) {
-    if (n <= 1) return cudaSuccess;
+// Sorts n unique keys whose significant bits are the low `bits` (+ values, may be null).
+// Result: in place in (keys, vals), or as triples {key >> qbits, key & qmask, val} in
+// `trip` when trip != null. `scratch` >= msd_scratch_bytes(n).
+cudaError_t msd_sort(uint64_t *keys, uint32_t *vals, uint64_t n, int bits, void *scratch, cudaStream_t s,
+                     gpumem_triple *trip, uint32_t qbits) {
+    Out out{keys, vals, trip, qbits};
+    if (n == 0) return cudaSuccess;
     if (bits < 1) bits = 1;
     const int B = choose_b(n, bits);
     const uint32_t nb = 1u << B;
     const int shift = bits - B;
+    const uint32_t chunks = n_chunks(n);
+    const uint64_t cs = (n + chunks - 1) / chunks;
     auto align = [](uintptr_t p) { return (p + 255) & ~uintptr_t(255); };
     uintptr_t c = align(reinterpret_cast<uintptr_t>(scratch));
     uint64_t *tk = reinterpret_cast<uint64_t *>(c);
     c = align(c + n * 8);
     uint32_t *tv = reinterpret_cast<uint32_t *>(c);
     c = align(c + n * 4);
-    uint32_t *counts = reinterpret_cast<uint32_t *>(c);
+    uint32_t *xv = vals ? vals : reinterpret_cast<uint32_t *>(c);  // value ping-pong of k_bs_big
+    c = align(c + n * 4);
+    uint32_t *counts = reinterpret_cast<uint32_t *>(c);  // [chunks][nb]
+    c = align(c + uint64_t(chunks) * nb * 4);
+    uint32_t *totals = reinterpret_cast<uint32_t *>(c);
     c = align(c + (nb + 1) * 4);
     uint32_t *offs = reinterpret_cast<uint32_t *>(c);
-    c = align(c + (nb + 1) * 4);
-    uint32_t *cursor = reinterpret_cast<uint32_t *>(c);
     c = align(c + (nb + 1) * 4);
     uint32_t *big = reinterpret_cast<uint32_t *>(c);
     c = align(c + nb * 4);
     unsigned int *n_big = reinterpret_cast<unsigned int *>(c);
-    cudaError_t e = cudaMemsetAsync(counts, 0, (nb + 1) * 4, s);
+    cudaError_t e = cudaMemsetAsync(n_big, 0, 4, s);
     if (e != cudaSuccess) return e;
-    if ((e = cudaMemsetAsync(n_big, 0, 4, s)) != cudaSuccess) return e;
     static bool attr = false;
     if (!attr) {
-        cudaFuncSetAttribute(k_msd_hist, cudaFuncAttributeMaxDynamicSharedMemorySize, (1 << kMaxB) * 4);
-        cudaFuncSetAttribute(k_msd_local, cudaFuncAttributeMaxDynamicSharedMemorySize, int(kLocal * 12));
+        cudaFuncSetAttribute(k_bp_hist, cudaFuncAttributeMaxDynamicSharedMemorySize, (1 << kMaxB) * 4);
+        cudaFuncSetAttribute(k_bp_scatter, cudaFuncAttributeMaxDynamicSharedMemorySize, (1 << kMaxB) * 4);
+        cudaFuncSetAttribute(k_bs_local, cudaFuncAttributeMaxDynamicSharedMemorySize, int(sizeof(LocalSmem)));
         attr = true;
     }
-    const int sms = num_sms();
-    const uint64_t hblocks = (n + kT * 16 - 1) / (kT * 16);
-    k_msd_hist<<<unsigned(hblocks < uint64_t(sms * 4) ? hblocks : uint64_t(sms * 4)), kT, nb * 4, s>>>(
-        keys, n, shift, nb, counts);
-    k_msd_scan<<<1, kT, 0, s>>>(counts, nb, offs, cursor);
-    k_msd_scatter<<<unsigned((n + kT - 1) / kT), kT, 0, s>>>(keys, vals, n, shift, cursor, tk, vals ? tv : nullptr);
-    // sorted-by-bucket data now in (tk, tv); sort each bucket in place there, then copy back
-    k_msd_local<<<nb < 65535u ? nb : 65535u, kT, kLocal * 12, s>>>(offs, nb, tk, vals ? tv : nullptr, big, n_big);
-    k_msd_big<<<sms, kT, 0, s>>>(offs, big, n_big, tk, vals ? tv : nullptr, keys, vals, shift);
-    note_launch(5);
-    if ((e = cudaMemcpyAsync(keys, tk, n * 8, cudaMemcpyDeviceToDevice, s)) != cudaSuccess) return e;
-    if (vals && (e = cudaMemcpyAsync(vals, tv, n * 4, cudaMemcpyDeviceToDevice, s)) != cudaSuccess) return e;
+    k_bp_hist<<<chunks, kPT, nb * 4, s>>>(keys, n, cs, shift, nb, counts);
+    k_bp_colscan<<<(nb + 255) / 256, 256, 0, s>>>(counts, chunks, nb, totals);
+    k_bs_scan<<<1, 1024, 0, s>>>(totals, nb, offs);
+    k_bp_scatter<<<chunks, kPT, nb * 4, s>>>(keys, vals, n, cs, shift, nb, counts, offs, tk, tv);
+    const uint64_t segs = (n + kSeg - 1) / kSeg;
+    k_bs_local<<<unsigned(segs), kLT, sizeof(LocalSmem), s>>>(offs, nb, bits, tk, tv, out, big, n_big);
+    // oversized buckets: ping-pong with the input's range of the bucket (free: the scatter
+    // consumed it and the local pass wrote only other buckets' ranges)
+    k_bs_big<<<num_sms(), kT, 0, s>>>(offs, big, n_big, tk, tv, keys, xv, shift, out);
+    note_launch(6);
     return cudaGetLastError();
 }
 

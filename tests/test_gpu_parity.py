@@ -23,7 +23,7 @@ from paper_conf_ipps_abu_dolehkac14_b200 import gpumem  # noqa: E402
 def _default_options():
     yield
     for k, v in (("find_grid", 0), ("find_spill", 64), ("out_capacity", 0), ("use_bitmap", 1), ("static_lb", 0),
-                 ("sort_impl", 1), ("radix_bits", 0)):
+                 ("sort_impl", 0), ("index_msd", 0), ("radix_bits", 0)):
         gpumem.set_option(k, v)
 
 
@@ -57,7 +57,7 @@ def test_pack_known_word():
     s = gpumem.pack(b"ACGT" * 8)
     w = s.words().cpu().numpy()
     assert int(w[0]) == 0x1B1B1B1B1B1B1B1B
-    assert int(w[1]) == 0 and int(w[2]) == 0  # padding
+    assert len(w) == 5 and not w[1:].any()  # four zero padding words
 
 
 @pytest.mark.parametrize("n", [0, 1, 31, 32, 33, 1000, 4097, 100_003])
@@ -69,8 +69,9 @@ def test_pack_roundtrip_device_and_host(n, offset):
     for s in (gpumem.pack(dev), gpumem.pack(raw[offset:].tobytes())):
         s.check()
         nn, _, nw = s.info()
-        assert nn == n and nw == (n + 31) // 32 + 2
+        assert nn == n and nw == (n + 31) // 32 + 4
         w = s.words().cpu().numpy()
+        assert not w[(n + 31) // 32:].any()  # four zero padding words
         up = raw[offset:] & 0xDF
         assert np.array_equal(_decode(w, n), up)
         if n % 32:
@@ -162,6 +163,18 @@ def test_homopolymer_closed_form(n, m):
         assert np.array_equal(got, want), (n, m, L, ls)
 
 
+@pytest.mark.parametrize("impl", [1, 2])
+@pytest.mark.parametrize("n,m,L", [(300, 20000, 20), (20000, 300, 20), (9000, 9000, 8000), (2, 50000, 1)])
+def test_sort_skewed_buckets(impl, n, m, L):
+    """Output sort on skewed key sets: most MEMs share r = 0 (one MSD bucket far past
+    shared memory -> the global LSD fallback) or q = 0 (many small buckets), checked
+    against the homopolymer closed form, under both sort implementations."""
+    gpumem.set_option("sort_impl", impl)
+    want = np.array(pyoracle.homopolymer(n, m, L), dtype=np.uint32).reshape(-1, 3)
+    got = gpu_mems("A" * n, "A" * m, L, 1 if L < 13 else 13)
+    assert np.array_equal(got, want), (impl, n, m, L)
+
+
 @pytest.mark.parametrize("L,ls", [(20, 10), (50, 13), (100, 13), (300, 13), (7, 1), (13, 13), (40, 15)])
 def test_adversarial_repeats(L, ls):
     """Tandem repeats, (AC)^n, multi-word left checks (step > 32, > 64, 288),
@@ -197,12 +210,13 @@ def test_overflow_retry_grid_spill_and_bitmap_invariance():
     base = gpu_mems(P.R, P.Q, P.L, P.ls)
     assert np.array_equal(base, want)
     for opt, vals in (("out_capacity", [1, 100]), ("find_grid", [1, 3, 148]), ("find_spill", [1, 2, 10**9]),
-                      ("use_bitmap", [0]), ("static_lb", [1]), ("sort_impl", [0]), ("radix_bits", [8, 9, 10])):
+                      ("use_bitmap", [0]), ("static_lb", [1]), ("sort_impl", [1, 2]), ("index_msd", [1]),
+                      ("radix_bits", [8, 9, 10])):
         for v in vals:
             gpumem.set_option(opt, v)
             assert np.array_equal(gpu_mems(P.R, P.Q, P.L, P.ls), want), (opt, v)
         gpumem.set_option(opt, {"out_capacity": 0, "find_grid": 0, "find_spill": 64, "use_bitmap": 1,
-                                "static_lb": 0, "sort_impl": 1, "radix_bits": 0}[opt])
+                                "static_lb": 0, "sort_impl": 0, "index_msd": 0, "radix_bits": 0}[opt])
 
 
 def test_seed_length_and_step_invariance():
