@@ -197,6 +197,8 @@ gpumem_status gpumem_set_allocator(void *(*alloc_fn)(size_t bytes, void *cuda_st
  *  "sort_impl"        output sort: 0 (default) auto by size, 1 stable LSD radix sort,
  *                     2 MSD bucket sort
  *  "index_msd"        index sort: 0 (default) stable LSD radix, 1 MSD bucket sort
+ *  "small_sort"       1: single-launch cooperative radix sorts (index and output) when
+ *                     the input fits in shared memory; 0 (default): multi-launch
  *  "radix_bits"       LSD digit width: 0 (default) = 9 bits when that saves a pass, else 8;
  *                     or pinned to 8, 9, 10; anything else is GPUMEM_ERR_ARG
  * Unknown names are GPUMEM_ERR_ARG. */

@@ -234,7 +234,7 @@ gpumem_status check_device(int *dev) {
 // loop does no allocation at all once warm. gpumem_trim() releases everything.
 enum WsSlot {
     kWsCtr, kWsSpill, kWsKeys, kWsLens, kWsSortK, kWsSortL, kWsSortScratch, kWsCodes0, kWsCodes1,
-    kWsRadix, kWsFill, kWsMergeK, kWsMergeL, kWsPackTmp, kWsCoop, kWsMums, kWsCount
+    kWsRadix, kWsFill, kWsMergeK, kWsMergeL, kWsPackTmp, kWsCoop, kWsMums, kWsSmall, kWsCount
 };
 struct Workspace {
     void *p[kWsCount] = {};
@@ -323,6 +323,7 @@ gpumem_status gpumem_set_option(const char *name, int64_t value) {
         g_opt.sort_impl = value;
     }
     else if (!strcmp(name, "index_msd")) g_opt.index_msd = value ? 1 : 0;
+    else if (!strcmp(name, "small_sort")) g_opt.small_sort = value ? 1 : 0;
     else if (!strcmp(name, "radix_bits")) {
         if (value != 0 && (value < 8 || value > 10)) return fail(GPUMEM_ERR_ARG, "radix_bits must be 0 or 8..10");
         g_opt.radix_bits = value;
@@ -521,7 +522,21 @@ static gpumem_status index_build_impl(const gpumem_seq *R, uint32_t ls, uint32_t
     if (!ptrs || !rankw || !buckets || !fill_scratch || !locs0) return GPUMEM_ERR_NOMEM;
     uint32_t *locs = locs0;
     const uint32_t *codes_sorted = nullptr;
-    if (n_locs) {
+    auto *recs = static_cast<uint4 *>(sc.get((n_locs ? n_locs : 1) * sizeof(uint4)));
+    if (!recs) return GPUMEM_ERR_NOMEM;
+    bool recs_done = false;
+    if (n_locs && !g_opt.index_msd && g_opt.small_sort && n_locs <= small_sort_max_n(4)) {
+        // one cooperative launch: seed codes from R, stable sort, codes + locs + records
+        auto *codes1 = static_cast<uint32_t *>(ws_get(kWsCodes1, n_locs * 4, s));
+        void *scratch = ws_get(kWsSmall, small_sort_scratch_bytes(n_locs, 4), s);
+        if (!codes1 || !scratch) return GPUMEM_ERR_NOMEM;
+        {
+            Stage g("index.sort", s);
+            CK(small_sort_index(R->words, ls, step, k0, n_locs, codes1, locs0, recs, scratch, s), "seed sort");
+        }
+        codes_sorted = codes1;
+        recs_done = true;
+    } else if (n_locs) {
         auto *codes0 = static_cast<uint32_t *>(ws_get(kWsCodes0, n_locs * 4, s));
         auto *codes1 = static_cast<uint32_t *>(ws_get(kWsCodes1, n_locs * 4, s));
         auto *locs1 = static_cast<uint32_t *>(sc.get(n_locs * 4));
@@ -554,9 +569,7 @@ static gpumem_status index_build_impl(const gpumem_seq *R, uint32_t ls, uint32_t
         Stage g("index.ptrs", s);
         CK(launch_ptrs_fill(codes_sorted, n_locs, ls, ptrs, rankw, buckets, fill_scratch, s), "ptrs fill");
     }
-    auto *recs = static_cast<uint4 *>(sc.get((n_locs ? n_locs : 1) * sizeof(uint4)));
-    if (!recs) return GPUMEM_ERR_NOMEM;
-    if (n_locs) {
+    if (n_locs && !recs_done) {
         Stage g("index.recs", s);
         CK(launch_seed_recs(R->words, ls, locs, n_locs, recs, s), "seed records");
     }
@@ -599,7 +612,11 @@ static gpumem_status sort_into_triples(uint64_t *keys, uint32_t *lens, uint64_t 
         // MSD bucket sort (keys are unique): two passes over the data; measured faster than
         // the 7-pass LSD radix up to a few million keys, slower beyond (its 16K-way scatter)
         constexpr uint64_t kMsdMaxN = 4u << 20;
-        if (g_opt.sort_impl == 2 || (g_opt.sort_impl == 0 && n <= kMsdMaxN)) {
+        if (g_opt.sort_impl == 0 && g_opt.small_sort && n <= small_sort_max_n(8)) {
+            void *scratch = ws_get(kWsSmall, small_sort_scratch_bytes(n, 8), s);
+            if (!scratch) return GPUMEM_ERR_NOMEM;
+            CK(small_sort_triples(keys, lens, n, int(key_bits), qbits, trip, scratch, s), "triple sort");
+        } else if (g_opt.sort_impl == 2 || (g_opt.sort_impl == 0 && n <= kMsdMaxN)) {
             void *scratch = ws_get(kWsSortScratch, msd_scratch_bytes(n), s);
             if (!scratch) return GPUMEM_ERR_NOMEM;
             CK(msd_sort(keys, lens, n, int(key_bits), scratch, s, trip, qbits), "triple sort");

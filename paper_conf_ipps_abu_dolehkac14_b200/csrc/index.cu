@@ -31,8 +31,8 @@ namespace gm {
 namespace {
 
 constexpr int kCodeThreads = 256;
-constexpr int kFillThreads = 256;
-constexpr int kChunk = 8192;                    // buckets per CTA in k_ptrs_fill
+constexpr int kFillThreads = 512;
+constexpr int kChunk = 16384;                   // buckets per CTA in k_ptrs_fill
 constexpr int kPer = kChunk / kFillThreads;     // 32 consecutive buckets per thread
 
 __global__ void __launch_bounds__(kCodeThreads) k_seed_codes(const uint64_t *__restrict__ R, uint32_t ls,
@@ -46,15 +46,6 @@ __global__ void __launch_bounds__(kCodeThreads) k_seed_codes(const uint64_t *__r
     locs[k] = uint32_t(p);
 }
 
-__device__ __forceinline__ uint64_t lower_bound(const uint32_t *__restrict__ a, uint64_t n, uint64_t x) {
-    uint64_t lo = 0, hi = n;
-    while (lo < hi) {
-        const uint64_t mid = (lo + hi) >> 1;
-        if (uint64_t(a[mid]) < x) lo = mid + 1; else hi = mid;
-    }
-    return lo;
-}
-
 // chunk_first[c] = first index i of the sorted codes with codes[i] >= c * kChunk, for
 // c in [0, n_chunks]; written by the element at each chunk boundary (no searches).
 __global__ void __launch_bounds__(kCodeThreads) k_chunk_bounds(const uint32_t *__restrict__ codes, uint64_t n,
@@ -66,41 +57,50 @@ __global__ void __launch_bounds__(kCodeThreads) k_chunk_bounds(const uint32_t *_
     for (uint64_t c = (i == 0 ? 0 : c_prev); c <= c_this && c <= n_chunks; ++c) first[c] = uint32_t(i);
 }
 
-constexpr uint64_t kStAgg = 1ull << 62;
-constexpr uint64_t kStInc = 2ull << 62;
-constexpr uint64_t kStMask = (1ull << 62) - 1;
-
-// Exclusive prefix of `agg` over chunks 0..chunk-1 by decoupled look-back (warp 0 only;
-// 32 predecessors per step). Chunks are numbered in launch order by a ticket.
-__device__ __forceinline__ unsigned long long chunk_lookback(unsigned long long *status, uint64_t chunk,
-                                                             unsigned long long agg) {
-    const int lane = threadIdx.x & 31;
-    volatile unsigned long long *st = status;
-    if (chunk == 0) {
-        if (lane == 0) st[0] = kStInc | agg;
-        return 0;
-    }
-    if (lane == 0) st[chunk] = kStAgg | agg;
-    unsigned long long excl = 0;
-    int64_t c = int64_t(chunk) - 1;
-    for (;;) {
-        const int64_t idx = c - lane;
-        const unsigned long long sv = idx >= 0 ? st[idx] : kStInc;
-        const unsigned long long f = sv & ~kStMask;
-        const unsigned inc_m = __ballot_sync(0xffffffffu, f == kStInc);
-        const unsigned zero_m = __ballot_sync(0xffffffffu, f == 0);
-        const int first_inc = inc_m ? __ffs(int(inc_m)) - 1 : 32;
-        const unsigned need = first_inc >= 31 ? 0xffffffffu : ((2u << first_inc) - 1u);
-        if (zero_m & need) continue;  // a predecessor has not published yet
-        unsigned long long part = (lane <= first_inc) ? (sv & kStMask) : 0ull;
+// occ[c] = number of distinct codes in chunk c (one CTA per chunk, block reduction of
+// the run heads; no global atomics -- sorted codes would hammer a few counters)
+__global__ void __launch_bounds__(kCodeThreads) k_occ_count(const uint32_t *__restrict__ codes,
+                                                            const uint32_t *__restrict__ first,
+                                                            uint32_t *__restrict__ occ) {
+    __shared__ uint32_t ws[kCodeThreads / 32];
+    const uint32_t c = blockIdx.x;
+    const uint64_t lo = first[c], hi = first[c + 1];
+    uint32_t h = 0;
+    for (uint64_t i = lo + threadIdx.x; i < hi; i += kCodeThreads) h += (i == 0 || codes[i - 1] != codes[i]) ? 1u : 0u;
 #pragma unroll
-        for (int o = 16; o; o >>= 1) part += __shfl_down_sync(0xffffffffu, part, o);
-        excl += __shfl_sync(0xffffffffu, part, 0);
-        if (first_inc < 32) break;
-        c -= 32;
+    for (int o = 16; o; o >>= 1) h += __shfl_xor_sync(0xffffffffu, h, o);
+    if ((threadIdx.x & 31) == 0) ws[threadIdx.x >> 5] = h;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        uint32_t t = 0;
+        for (int k = 0; k < kCodeThreads / 32; ++k) t += ws[k];
+        occ[c] = t;
     }
-    if (lane == 0) st[chunk] = kStInc | (excl + agg);
-    return excl;
+}
+
+// rank0[c] = exclusive prefix of occ over the chunks (one CTA, contiguous runs per thread)
+__global__ void __launch_bounds__(1024) k_occ_scan(const uint32_t *__restrict__ occ, uint32_t n,
+                                                   uint32_t *__restrict__ rank0) {
+    __shared__ uint32_t ws[32];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const uint32_t per = (n + 1023) / 1024;
+    const uint32_t i0 = threadIdx.x * per, i1 = min(i0 + per, n);
+    uint32_t sum = 0;
+    for (uint32_t i = i0; i < i1; ++i) sum += occ[i];
+    uint32_t inc = sum;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
+        if (lane >= o) inc += y;
+    }
+    if (lane == 31) ws[w] = inc;
+    __syncthreads();
+    uint32_t run = inc - sum;
+    for (int k = 0; k < w; ++k) run += ws[k];
+    for (uint32_t i = i0; i < i1; ++i) {
+        rank0[i] = run;
+        run += occ[i];
+    }
 }
 
 __global__ void __launch_bounds__(kFillThreads) k_ptrs_fill(const uint32_t *__restrict__ codes, uint64_t n,
@@ -108,88 +108,91 @@ __global__ void __launch_bounds__(kFillThreads) k_ptrs_fill(const uint32_t *__re
                                                             unsigned long long *__restrict__ rankw,
                                                             uint2 *__restrict__ buckets,
                                                             const uint32_t *__restrict__ chunk_first,
-                                                            unsigned long long *status, unsigned int *ticket) {
-    __shared__ uint32_t cnt[kChunk + kChunk / 32];   // one pad word per 32: conflict-free rows
-    __shared__ uint64_t range[2];
+                                                            const uint32_t *__restrict__ rank0) {
+    extern __shared__ uint32_t cnt[];                // kChunk + kChunk / 32: a pad word per 32 (conflict-free rows)
     __shared__ uint32_t wsum[kFillThreads / 32];
     __shared__ uint32_t wocc[kFillThreads / 32];
-    __shared__ unsigned long long s_rank0;
-    __shared__ unsigned int s_chunk;
     const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
-    if (tid == 0) s_chunk = atomicAdd(ticket, 1u);
+    const uint32_t c = blockIdx.x;
+    const uint64_t s0 = uint64_t(c) * kChunk;
+    for (int i = tid; i < kChunk + kChunk / 32; i += kFillThreads) cnt[i] = 0;
+    const uint64_t lo = chunk_first[c], hi = chunk_first[c + 1];
     __syncthreads();
-    {
-        const uint64_t s0 = uint64_t(s_chunk) * kChunk;
-        for (int i = tid; i < kChunk + kChunk / 32; i += kFillThreads) cnt[i] = 0;
-        if (tid == 0) range[0] = chunk_first[s_chunk];
-        if (tid == 32) range[1] = chunk_first[s_chunk + 1];
-        __syncthreads();
-        const uint64_t lo = range[0], hi = range[1];
-        // Alg. 1 step 1 for this chunk: seed counts
-        for (uint64_t i = lo + tid; i < hi; i += kFillThreads) {
-            const uint32_t d = uint32_t(codes[i] - s0);
-            atomicAdd(&cnt[d + (d >> 5)], 1u);
+    // Alg. 1 step 1 for this chunk: seed counts. The codes are sorted, so equal codes are
+    // runs of lanes: one shared atomic per run (a hot seed, e.g. poly-A, would otherwise
+    // serialise thousands of atomics on one counter)
+    for (uint64_t base = lo; base < hi; base += kFillThreads) {
+        const uint64_t i = base + tid;
+        const bool valid = i < hi;
+        const uint32_t code = valid ? codes[i] : 0xffffffffu;
+        const uint32_t prev = __shfl_up_sync(0xffffffffu, code, 1);
+        const bool start = valid && (lane == 0 || prev != code);
+        const unsigned starts = __ballot_sync(0xffffffffu, start), vmask = __ballot_sync(0xffffffffu, valid);
+        if (start) {
+            const unsigned later = starts & ~((2u << lane) - 1u);
+            const unsigned run = (later ? ((1u << (__ffs(int(later)) - 1)) - 1u) : 0xffffffffu) & ~((1u << lane) - 1u);
+            const uint32_t d = code - uint32_t(s0);
+            atomicAdd(&cnt[d + (d >> 5)], uint32_t(__popc(run & vmask)));
         }
-        __syncthreads();
-        // Alg. 1 step 2: block-wide exclusive scan; thread t owns buckets [32t, 32t+32)
-        uint32_t sum = 0, occ = 0;
-#pragma unroll
-        for (int j = 0; j < kPer; ++j) {
-            const uint32_t c = cnt[tid * (kPer + 1) + j];
-            sum += c;
-            occ |= (c ? 1u : 0u) << j;
-        }
-        // block scans of (counts, occupied buckets) per thread
-        const uint32_t nocc = __popc(occ);
-        uint32_t inc = sum, inco = nocc;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            const uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
-            const uint32_t z = __shfl_up_sync(0xffffffffu, inco, o);
-            if (lane >= o) {
-                inc += y;
-                inco += z;
-            }
-        }
-        if (lane == 31) {
-            wsum[w] = inc;
-            wocc[w] = inco;
-        }
-        __syncthreads();
-        uint32_t pre = uint32_t(lo), preo = 0, tot_occ = 0;
-        for (int i = 0; i < kFillThreads / 32; ++i) {
-            if (i < w) {
-                pre += wsum[i];
-                preo += wocc[i];
-            }
-            tot_occ += wocc[i];
-        }
-        pre += inc - sum;
-        preo += inco - nocc;
-        // rank of the chunk's first occupied bucket among all occupied buckets
-        if (w == 0) {
-            const unsigned long long r0 = chunk_lookback(status, s_chunk, tot_occ);
-            if (lane == 0) s_rank0 = r0;
-        }
-        __syncthreads();
-        // counts -> ptrs (in place), rank words {occupancy bits, occupied buckets before
-        // this word} and the compact {first slot, count} table, in bucket order
-        const uint64_t rank = s_rank0 + preo;
-        uint64_t r = rank;
-#pragma unroll 4
-        for (int j = 0; j < kPer; ++j) {
-            const uint32_t c = cnt[tid * (kPer + 1) + j];
-            cnt[tid * (kPer + 1) + j] = pre;
-            if (c) buckets[r++] = make_uint2(pre, c);
-            pre += c;
-        }
-        if (s0 + uint64_t(tid) * kPer < n_buckets) rankw[(s0 >> 5) + tid] = (rank << 32) | occ;
-        __syncthreads();
-        // coalesced write-out of the chunk's ptrs
-        const uint64_t lim = n_buckets - s0 < uint64_t(kChunk) ? n_buckets - s0 : uint64_t(kChunk);
-        for (int i = tid; i < int(lim); i += kFillThreads) ptrs[s0 + i] = cnt[i + (i >> 5)];
-        if (s0 == 0 && tid == 0) ptrs[n_buckets] = uint32_t(n);
     }
+    __syncthreads();
+    // Alg. 1 step 2: block-wide exclusive scan; thread t owns buckets [32t, 32t+32)
+    uint32_t sum = 0, occ = 0;
+#pragma unroll
+    for (int j = 0; j < kPer; ++j) {
+        const uint32_t x = cnt[tid * (kPer + 1) + j];
+        sum += x;
+        occ |= (x ? 1u : 0u) << j;
+    }
+    const uint32_t nocc = __popc(occ);
+    uint32_t inc = sum, inco = nocc;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
+        const uint32_t z = __shfl_up_sync(0xffffffffu, inco, o);
+        if (lane >= o) {
+            inc += y;
+            inco += z;
+        }
+    }
+    if (lane == 31) {
+        wsum[w] = inc;
+        wocc[w] = inco;
+    }
+    __syncthreads();
+    uint32_t pre = uint32_t(lo), preo = 0;
+    for (int i = 0; i < w; ++i) {
+        pre += wsum[i];
+        preo += wocc[i];
+    }
+    pre += inc - sum;
+    preo += inco - nocc;
+    // counts -> ptrs (in place), rank words {occupancy bits, occupied buckets before this
+    // word} and the compact {first slot, count} table, in bucket order
+    const uint64_t rank = uint64_t(rank0[c]) + preo;
+    uint64_t r = rank;
+#pragma unroll 4
+    for (int j = 0; j < kPer; ++j) {
+        const uint32_t x = cnt[tid * (kPer + 1) + j];
+        cnt[tid * (kPer + 1) + j] = pre;
+        if (x) buckets[r++] = make_uint2(pre, x);
+        pre += x;
+    }
+    if (s0 + uint64_t(tid) * kPer < n_buckets) rankw[(s0 >> 5) + tid] = (rank << 32) | occ;
+    __syncthreads();
+    // coalesced write-out of the chunk's ptrs, 16 bytes per store
+    const uint64_t lim = n_buckets - s0 < uint64_t(kChunk) ? n_buckets - s0 : uint64_t(kChunk);
+    if (lim == uint64_t(kChunk)) {
+        uint4 *dst = reinterpret_cast<uint4 *>(ptrs + s0);
+        for (int i = tid; i < kChunk / 4; i += kFillThreads) {
+            const int b = 4 * i;  // 4 | 32: the four buckets share one padded row
+            const int sp = b + (b >> 5);
+            dst[i] = make_uint4(cnt[sp], cnt[sp + 1], cnt[sp + 2], cnt[sp + 3]);
+        }
+    } else {
+        for (int i = tid; i < int(lim); i += kFillThreads) ptrs[s0 + i] = cnt[i + (i >> 5)];
+    }
+    if (s0 == 0 && tid == 0) ptrs[n_buckets] = uint32_t(n);
 }
 
 // Seed records (lookup acceleration, not part of the paper's index): for each slot k
@@ -202,8 +205,21 @@ __global__ void __launch_bounds__(kCodeThreads) k_seed_recs(const uint64_t *__re
     const uint64_t k = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
     if (k >= n_locs) return;
     const uint32_t p = locs[k];
-    const uint32_t left = uint32_t(win_back(R, p));
-    const uint64_t right = win_fwd(R, uint64_t(p) + ls);
+    uint32_t left;
+    uint64_t right;
+    if (p >= 16) {  // bases [p - 16, p + ls + 32) lie in the 3 words from (p - 16) / 32: one gather
+        const uint64_t x = p - 16, w = x >> 5;
+        const uint64_t w0 = __ldg(R + w), w1 = __ldg(R + w + 1), w2 = __ldg(R + w + 2);
+        const uint32_t sx = uint32_t(x & 31) * 2;
+        left = uint32_t(((w0 << sx) | ((w1 >> 1) >> (63 - sx))) >> 32);
+        const uint32_t o = uint32_t(x & 31) + 16 + ls;  // right window start, bases from word w
+        const uint32_t so = (o & 31) * 2;
+        const uint64_t a = o < 32 ? w0 : w1, b = o < 32 ? w1 : w2;
+        right = (a << so) | ((b >> 1) >> (63 - so));
+    } else {
+        left = uint32_t(win_back(R, p));
+        right = win_fwd(R, uint64_t(p) + ls);
+    }
     recs[k] = make_uint4(p, left, uint32_t(right), uint32_t(right >> 32));
 }
 
@@ -230,23 +246,35 @@ cudaError_t launch_seed_codes(const uint64_t *R, uint32_t ls, uint32_t step, uin
 size_t ptrs_fill_scratch_bytes(uint32_t ls) {
     const uint64_t nb = 1ull << (2 * ls);
     const uint64_t chunks = (nb + kChunk - 1) / kChunk;
-    return chunks * 8 + 64 + (chunks + 1) * 4 + 256;
+    return (chunks + 1) * 4 * 3 + 3 * 256;
 }
 
 cudaError_t launch_ptrs_fill(const uint32_t *sorted_codes, uint64_t n_locs, uint32_t ls, uint32_t *ptrs,
                              unsigned long long *rankw, uint2 *buckets, void *scratch, cudaStream_t s) {
     const uint64_t nb = 1ull << (2 * ls);
     const uint64_t chunks = (nb + kChunk - 1) / kChunk;
-    cudaError_t e = cudaMemsetAsync(scratch, 0, chunks * 8 + 64, s);
-    if (e != cudaSuccess) return e;
-    auto *status = static_cast<unsigned long long *>(scratch);
-    auto *ticket = reinterpret_cast<unsigned int *>(status + chunks);
-    auto *first = reinterpret_cast<uint32_t *>(reinterpret_cast<char *>(scratch) + chunks * 8 + 64);
+    auto align = [](uintptr_t p) { return (p + 255) & ~uintptr_t(255); };
+    uintptr_t a = align(reinterpret_cast<uintptr_t>(scratch));
+    auto *first = reinterpret_cast<uint32_t *>(a);
+    a = align(a + (chunks + 1) * 4);
+    auto *occ = reinterpret_cast<uint32_t *>(a);
+    a = align(a + (chunks + 1) * 4);
+    auto *rank0 = reinterpret_cast<uint32_t *>(a);
+    cudaError_t e = cudaSuccess;
     k_chunk_bounds<<<unsigned((n_locs + 1 + kCodeThreads - 1) / kCodeThreads), kCodeThreads, 0, s>>>(
         sorted_codes, n_locs, chunks, first);
-    k_ptrs_fill<<<unsigned(chunks), kFillThreads, 0, s>>>(sorted_codes, n_locs, nb, ptrs, rankw, buckets, first,
-                                                         status, ticket);
-    note_launch(2);
+    k_occ_count<<<unsigned(chunks), kCodeThreads, 0, s>>>(sorted_codes, first, occ);
+    k_occ_scan<<<1, 1024, 0, s>>>(occ, uint32_t(chunks), rank0);
+    constexpr int smem = (kChunk + kChunk / 32) * 4;
+    static bool attr = false;
+    if (!attr) {
+        e = cudaFuncSetAttribute(k_ptrs_fill, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+        if (e != cudaSuccess) return e;
+        attr = true;
+    }
+    k_ptrs_fill<<<unsigned(chunks), kFillThreads, smem, s>>>(sorted_codes, n_locs, nb, ptrs, rankw, buckets, first,
+                                                         rank0);
+    note_launch(4);
     return cudaGetLastError();
 }
 

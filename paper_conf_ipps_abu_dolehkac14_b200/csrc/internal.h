@@ -17,6 +17,8 @@ struct Options {
     int64_t static_lb = 0;       // 1: each lane processes its own positions' hits (LB ablation)
     int64_t sort_impl = 0;       // output sort: 0 = auto (MSD below kMsdMaxN keys, else LSD), 1 = stable LSD radix
                                  // (radix.cu), 2 = MSD bucket sort (msd.cu)
+    int64_t small_sort = 0;      // 1: single-launch cooperative sorts when the input fits (small_sort.cu;
+                                 // measured slower at C4: its scattered global writes are not coalesced)
     int64_t index_msd = 0;       // index sort: 1 = MSD bucket sort of (code << 32 | p), 0 = stable LSD radix
     int64_t radix_bits = 0;      // LSD digit width: 0 = 9 bits if that saves a pass else 8; or pinned 8, 9, 10
 };
@@ -54,6 +56,16 @@ cudaError_t radix_sort_u32(uint32_t *k0, uint32_t *v0, uint32_t *k1, uint32_t *v
 cudaError_t radix_sort_u64(uint64_t *k0, uint32_t *v0, uint64_t *k1, uint32_t *v1, uint64_t n, int bits,
                            void *scratch, cudaStream_t s, bool *in_alt);
 size_t radix_scratch_bytes(uint64_t n);
+
+// Single-launch (cooperative) stable LSD radix sorts for small inputs (small_sort.cu):
+// n <= small_sort_max_n(key bytes). The index variant computes the seed codes of the
+// sampled locations from packed R itself and writes sorted codes, locs and seed records.
+uint64_t small_sort_max_n(int key_bytes);
+size_t small_sort_scratch_bytes(uint64_t n, int key_bytes);
+cudaError_t small_sort_index(const uint64_t *R, uint32_t ls, uint32_t step, uint64_t k0, uint64_t n_locs,
+                             uint32_t *codes, uint32_t *locs, uint4 *recs, void *scratch, cudaStream_t s);
+cudaError_t small_sort_triples(const uint64_t *keys, const uint32_t *lens, uint64_t n, int bits, uint32_t qbits,
+                               gpumem_triple *out, void *scratch, cudaStream_t s);
 
 // MSD bucket sort of unique u64 keys (+ optional u32 values), in place, or written as
 // triples {key >> qbits, key & qmask, val} when trip != null (msd.cu).

@@ -23,7 +23,7 @@ from paper_conf_ipps_abu_dolehkac14_b200 import gpumem  # noqa: E402
 def _default_options():
     yield
     for k, v in (("find_grid", 0), ("find_spill", 64), ("out_capacity", 0), ("use_bitmap", 1), ("static_lb", 0),
-                 ("sort_impl", 0), ("index_msd", 0), ("radix_bits", 0)):
+                 ("sort_impl", 0), ("index_msd", 0), ("small_sort", 0), ("radix_bits", 0)):
         gpumem.set_option(k, v)
 
 
@@ -124,6 +124,18 @@ def test_index_parity_word_for_word(cfg, ls, step, scale):
     assert np.array_equal(l, ol)
 
 
+@pytest.mark.parametrize("opts", [{"small_sort": 1}, {"radix_bits": 8}, {"index_msd": 1}])
+def test_index_sort_paths(opts):
+    """Every index sort path (single-launch cooperative, multi-launch LSD, MSD) gives
+    Alg. 1's ptrs/locs word for word."""
+    P = synth.make_pair("c3", scale=0.05)
+    op, ol = oracle.index(P.R.tobytes(), 13, 38)
+    for k, v in opts.items():
+        gpumem.set_option(k, v)
+    p, l = _index_gpu(P.R.tobytes(), 13, 38)
+    assert np.array_equal(p, op) and np.array_equal(l, ol)
+
+
 def test_index_short_reference():
     p, l = _index_gpu(b"ACG", 4, 1)
     assert len(l) == 0 and not p.any()
@@ -163,13 +175,15 @@ def test_homopolymer_closed_form(n, m):
         assert np.array_equal(got, want), (n, m, L, ls)
 
 
-@pytest.mark.parametrize("impl", [1, 2])
+@pytest.mark.parametrize("impl", [0, 1, 2, 3])
 @pytest.mark.parametrize("n,m,L", [(300, 20000, 20), (20000, 300, 20), (9000, 9000, 8000), (2, 50000, 1)])
 def test_sort_skewed_buckets(impl, n, m, L):
     """Output sort on skewed key sets: most MEMs share r = 0 (one MSD bucket far past
     shared memory -> the global LSD fallback) or q = 0 (many small buckets), checked
-    against the homopolymer closed form, under both sort implementations."""
-    gpumem.set_option("sort_impl", impl)
+    against the homopolymer closed form, under every output sort path (auto, LSD, MSD,
+    single-launch)."""
+    gpumem.set_option("sort_impl", impl % 3)
+    gpumem.set_option("small_sort", int(impl == 3))
     want = np.array(pyoracle.homopolymer(n, m, L), dtype=np.uint32).reshape(-1, 3)
     got = gpu_mems("A" * n, "A" * m, L, 1 if L < 13 else 13)
     assert np.array_equal(got, want), (impl, n, m, L)
@@ -210,13 +224,14 @@ def test_overflow_retry_grid_spill_and_bitmap_invariance():
     base = gpu_mems(P.R, P.Q, P.L, P.ls)
     assert np.array_equal(base, want)
     for opt, vals in (("out_capacity", [1, 100]), ("find_grid", [1, 3, 148]), ("find_spill", [1, 2, 10**9]),
-                      ("use_bitmap", [0]), ("static_lb", [1]), ("sort_impl", [1, 2]), ("index_msd", [1]),
+                      ("use_bitmap", [0]), ("static_lb", [1]), ("sort_impl", [1, 2]), ("index_msd", [1]), ("small_sort", [1]),
                       ("radix_bits", [8, 9, 10])):
         for v in vals:
             gpumem.set_option(opt, v)
             assert np.array_equal(gpu_mems(P.R, P.Q, P.L, P.ls), want), (opt, v)
         gpumem.set_option(opt, {"out_capacity": 0, "find_grid": 0, "find_spill": 64, "use_bitmap": 1,
-                                "static_lb": 0, "sort_impl": 0, "index_msd": 0, "radix_bits": 0}[opt])
+                                "static_lb": 0, "sort_impl": 0, "index_msd": 0, "small_sort": 0,
+                                "radix_bits": 0}[opt])
 
 
 def test_seed_length_and_step_invariance():
