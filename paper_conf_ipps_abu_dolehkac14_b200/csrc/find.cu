@@ -8,10 +8,15 @@
 // never waits on other warps (no CTA barriers). Per chunk:
 //  stage   the chunk's packed Q words (+ halo) go to the warp's shared memory;
 //  A5      each lane cuts kQPT consecutive seeds out of one 64-bit window, probes
-//          the rank word of each seed (occupancy bit + running rank, 16 MB,
-//          L2-resident) and, for occupied seeds, reads {first slot, count} of the
-//          bucket from the compact table -- the same range as [ptrs[s], ptrs[s+1])
-//          (PAPER.md:84); use_bitmap = 0 reads the dense ptrs instead. Buckets of
+//          the rank word of each seed (occupancy bit + running rank, 8 B per 32
+//          seeds, 16 MB at ls = 13, L2-resident) and, for occupied seeds, reads
+//          {first slot, count} of the bucket from the compact table -- the range
+//          [ptrs[s], ptrs[s+1]). When that table is too large to stay
+//          in L2 (many sampled seeds: C5 L = 20, 50) the index carries rank sectors
+//          instead (16 B per 32 seeds: records and occupied seeds before the group +
+//          a 2-bit saturating count per seed), which alone give {first, count}
+//          unless a count in the group up to the seed saturates; only then is the
+//          compact table read. use_bitmap = 0 reads the dense ptrs. Buckets of
 //          more than spill_t hits are cut into kSpillHits-hit pieces and pushed to
 //          a global queue drained by k_heavy (reference-axis tiles of the hot
 //          seeds, Fig. 6 :268-270); the rest become (q, bucket) entries with a
@@ -427,7 +432,7 @@ __device__ __forceinline__ void drain_deferred(const FindParams &P, WarpSmem &s,
 #ifndef GM_FIND_MINB
 #define GM_FIND_MINB 4
 #endif
-template <bool kStatic, bool kHints>
+template <bool kStatic, bool kHints, bool kSect>
 __global__ void __launch_bounds__(kT, GM_FIND_MINB) k_find(const FindParams P) {
     __shared__ WarpSmem smem[kWarps];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
@@ -472,7 +477,7 @@ __global__ void __launch_bounds__(kT, GM_FIND_MINB) k_find(const FindParams P) {
                     code[j] = uint32_t((win << (2 * j)) >> sh);
                     occ[j] = qa + j < P.scan_hi;
                 }
-                if (P.use_bitmap) {
+                if (P.use_bitmap && !kSect) {
                     // rank-word probe (occupancy bit + rank), then the compact {first, count}
                     uint32_t rank[kQPT];
 #pragma unroll
@@ -489,6 +494,39 @@ __global__ void __launch_bounds__(kT, GM_FIND_MINB) k_find(const FindParams P) {
 #pragma unroll
                     for (int j = 0; j < kQPT; ++j) {
                         if (occ[j]) {
+                            const uint2 b = kHints ? ld_last_u2(P.buckets + rank[j]) : __ldg(P.buckets + rank[j]);
+                            beg[j] = b.x;
+                            cnt[j] = b.y;
+                        }
+                    }
+                } else if (P.use_bitmap) {
+                    // rank-sector probe: {records before the group, occupied seeds before
+                    // the group, 2-bit saturating count per seed}. Counts <= 2 all the way
+                    // up to the seed give {first, count} directly; otherwise the compact
+                    // {first, count} table is read at the seed's rank.
+                    uint32_t rank[kQPT];
+                    bool need[kQPT];
+#pragma unroll
+                    for (int j = 0; j < kQPT; ++j) {
+                        need[j] = false;
+                        rank[j] = 0;
+                        if (occ[j]) {
+                            const uint4 rs = kHints ? ld_last_u4(P.rsect + (code[j] >> 5)) : __ldg(P.rsect + (code[j] >> 5));
+                            const uint32_t b = code[j] & 31;
+                            const uint64_t c2 = (uint64_t(rs.w) << 32) | rs.z;
+                            const uint32_t f = uint32_t(c2 >> (2 * b)) & 3u;
+                            const uint64_t below = c2 & ((1ull << (2 * b)) - 1ull);
+                            constexpr uint64_t kLo = 0x5555555555555555ull;
+                            occ[j] = f != 0;
+                            need[j] = f != 0 && (f == 3u || (below & (below >> 1) & kLo) != 0);
+                            beg[j] = rs.x + __popcll(below & kLo) + 2 * __popcll(below & ~kLo);
+                            cnt[j] = occ[j] ? f : 0u;
+                            rank[j] = rs.y + __popcll((below | (below >> 1)) & kLo);
+                        }
+                    }
+#pragma unroll
+                    for (int j = 0; j < kQPT; ++j) {
+                        if (need[j]) {
                             const uint2 b = kHints ? ld_last_u2(P.buckets + rank[j]) : __ldg(P.buckets + rank[j]);
                             beg[j] = b.x;
                             cnt[j] = b.y;
@@ -666,7 +704,7 @@ uint64_t find_tile_positions() { return kChunk; }
 int find_default_grid() {
     if (!g_default_grid) {
         int per_sm = 0;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_find<false, false>, kT, 0);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_find<false, false, false>, kT, 0);
         if (per_sm < 1) per_sm = 1;
         g_default_grid = per_sm * num_sms();
     }
@@ -681,9 +719,17 @@ cudaError_t launch_find(const FindParams &p, int grid, cudaStream_t s) {
     if (grid < 1) grid = 1;
     // kHints: the seed records exceed half of L2 -> cache-policy loads (lookup tables
     // evict_last, streams evict_first); otherwise plain loads (measured faster there)
-    if (p.static_lb) k_find<true, false><<<grid, kT, 0, s>>>(p);
-    else if (p.recs_stream) k_find<false, true><<<grid, kT, 0, s>>>(p);
-    else k_find<false, false><<<grid, kT, 0, s>>>(p);
+    const bool sect = p.rsect != nullptr;
+    if (p.static_lb) {
+        if (sect) k_find<true, false, true><<<grid, kT, 0, s>>>(p);
+        else k_find<true, false, false><<<grid, kT, 0, s>>>(p);
+    } else if (p.recs_stream) {
+        if (sect) k_find<false, true, true><<<grid, kT, 0, s>>>(p);
+        else k_find<false, true, false><<<grid, kT, 0, s>>>(p);
+    } else {
+        if (sect) k_find<false, false, true><<<grid, kT, 0, s>>>(p);
+        else k_find<false, false, false><<<grid, kT, 0, s>>>(p);
+    }
     note_launch();
     return cudaGetLastError();
 }

@@ -35,7 +35,8 @@ struct gpumem_index {
     uint64_t n_locs;
     uint32_t *ptrs;
     uint32_t *locs;
-    unsigned long long *rankw;
+    unsigned long long *rankw;   // rank words, 8 B per 32 seeds, or
+    uint4 *rsect;                // rank sectors, 16 B per 32 seeds (index.cu); one of the two is null
     uint2 *buckets;
     uint4 *recs;
 };
@@ -324,6 +325,7 @@ gpumem_status gpumem_set_option(const char *name, int64_t value) {
     }
     else if (!strcmp(name, "index_msd")) g_opt.index_msd = value ? 1 : 0;
     else if (!strcmp(name, "small_sort")) g_opt.small_sort = value ? 1 : 0;
+    else if (!strcmp(name, "rank_sectors")) g_opt.rank_sectors = value < 0 ? -1 : (value ? 1 : 0);
     else if (!strcmp(name, "radix_bits")) {
         if (value != 0 && (value < 8 || value > 10)) return fail(GPUMEM_ERR_ARG, "radix_bits must be 0 or 8..10");
         g_opt.radix_bits = value;
@@ -383,6 +385,7 @@ void gpumem_free(void *handle) {
         dfree(x->ptrs, x->stream);
         dfree(x->locs, x->stream);
         dfree(x->rankw, x->stream);
+        dfree(x->rsect, x->stream);
         dfree(x->buckets, x->stream);
         dfree(x->recs, x->stream);
         x->magic = 0;
@@ -514,12 +517,20 @@ static gpumem_status index_build_impl(const gpumem_seq *R, uint32_t ls, uint32_t
     const uint64_t n_locs = k1 > k0 ? k1 - k0 : 0;
     Scratch sc(s);
     auto *ptrs = static_cast<uint32_t *>(sc.get((nb + 1) * 4));
-    auto *rankw = static_cast<unsigned long long *>(sc.get(((nb + 31) / 32) * 8));
+    // lookup directory: rank sectors when the compact table {first, count} (<= 8 B per
+    // sampled seed) would not stay in L2 next to the rest, else the smaller rank words
+    int l2 = 0;
+    cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, dev);
+    const bool use_sect = g_opt.rank_sectors < 0 ? n_locs * 8 > uint64_t(l2) / 4 : g_opt.rank_sectors != 0;
+    unsigned long long *rankw = nullptr;
+    uint4 *rsect = nullptr;
+    if (use_sect) rsect = static_cast<uint4 *>(sc.get(((nb + 31) / 32) * 16));
+    else rankw = static_cast<unsigned long long *>(sc.get(((nb + 31) / 32) * 8));
     const uint64_t max_occ = (n_locs < nb ? n_locs : nb) + 1;
     auto *buckets = static_cast<uint2 *>(sc.get(max_occ * sizeof(uint2)));
     void *fill_scratch = ws_get(kWsFill, ptrs_fill_scratch_bytes(ls), s);
     auto *locs0 = static_cast<uint32_t *>(sc.get((n_locs ? n_locs : 1) * 4));
-    if (!ptrs || !rankw || !buckets || !fill_scratch || !locs0) return GPUMEM_ERR_NOMEM;
+    if (!ptrs || !(rsect || rankw) || !buckets || !fill_scratch || !locs0) return GPUMEM_ERR_NOMEM;
     uint32_t *locs = locs0;
     const uint32_t *codes_sorted = nullptr;
     auto *recs = static_cast<uint4 *>(sc.get((n_locs ? n_locs : 1) * sizeof(uint4)));
@@ -567,18 +578,19 @@ static gpumem_status index_build_impl(const gpumem_seq *R, uint32_t ls, uint32_t
     }
     {
         Stage g("index.ptrs", s);
-        CK(launch_ptrs_fill(codes_sorted, n_locs, ls, ptrs, rankw, buckets, fill_scratch, s), "ptrs fill");
+        CK(launch_ptrs_fill(codes_sorted, n_locs, ls, ptrs, rankw, rsect, buckets, fill_scratch, s), "ptrs fill");
     }
     if (n_locs && !recs_done) {
         Stage g("index.recs", s);
         CK(launch_seed_recs(R->words, ls, locs, n_locs, recs, s), "seed records");
     }
     sc.keep(ptrs);
-    sc.keep(rankw);
+    if (rankw) sc.keep(rankw);
+    if (rsect) sc.keep(rsect);
     sc.keep(buckets);
     sc.keep(locs);
     sc.keep(recs);
-    auto *h = new gpumem_index{kMagicIdx, dev, s, R, ls, L, step, n_locs, ptrs, locs, rankw, buckets, recs};
+    auto *h = new gpumem_index{kMagicIdx, dev, s, R, ls, L, step, n_locs, ptrs, locs, rankw, rsect, buckets, recs};
     *out = h;
     return GPUMEM_OK;
 }
@@ -665,6 +677,7 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
     P.ptrs = idx->ptrs;
     P.recs = idx->recs;
     P.rankw = idx->rankw;
+    P.rsect = idx->rsect;
     P.buckets = idx->buckets;
     P.ls = ls;
     P.L = L;

@@ -12,17 +12,21 @@
 //                histogram from the sorted codes (a binary search bounds the
 //                chunk's slice) and a block-wide exclusive scan ->
 //                ptrs[s] = #locations with seed < s (:84), ptrs[4^ls] = n_locs.
-//                The same pass writes the lookup structures (not in the paper):
-//                rank words, one u64 per 32 seeds = {occupancy bits, number of
-//                occupied seeds before the word} (16 MB at ls = 13, L2-resident),
-//                and the compact table {ptrs[s], count} of the occupied seeds in
-//                seed order (8 B each). A chunk's first rank comes from a
-//                decoupled look-back over earlier chunks. The lookup then costs
-//                one 8-byte probe per query position plus one 8-byte read per
-//                occupied seed, both L2-resident, instead of two reads of the
-//                HBM-resident 4^ls-entry ptrs.
+//                The same pass writes the lookup structures (not in the paper): the
+//                compact table {ptrs[s], count} of the occupied seeds in seed order
+//                (8 B each) and a directory over the 4^ls seeds, either
+//                rank words, 8 B per 32 seeds = {occupancy bits, occupied seeds before}
+//                (16 MB at ls = 13) -- the lookup is one 8-byte probe per query
+//                position + one 8-byte table read per occupied seed, both L2-resident
+//                when the table is small -- or, when the compact table would not stay
+//                in L2, rank sectors, 16 B per 32 seeds = {records before the group,
+//                occupied seeds before the group, a 2-bit saturating count per seed}:
+//                the probe alone gives {first, count} unless a count in the group up
+//                to the seed saturates (>= 3), so most HBM table reads disappear.
+//                A chunk's first rank comes from a scan of the per-chunk occupancy
+//                counts. Either replaces two reads of the HBM-resident 4^ls-entry ptrs.
 // Algorithmic bytes: n_locs * (8 B codes/locs written + 16 B per radix pass read+
-// write) + 4 * (4^ls + 1) B ptrs written + 4^ls / 4 B rank words + 8 B per
+// write) + 4 * (4^ls + 1) B ptrs written + 4^ls / 2 B rank sectors + 8 B per
 // occupied seed.
 #include "internal.h"
 #include "device.cuh"
@@ -103,9 +107,11 @@ __global__ void __launch_bounds__(1024) k_occ_scan(const uint32_t *__restrict__ 
     }
 }
 
+template <bool kSect>
 __global__ void __launch_bounds__(kFillThreads) k_ptrs_fill(const uint32_t *__restrict__ codes, uint64_t n,
                                                             uint64_t n_buckets, uint32_t *__restrict__ ptrs,
                                                             unsigned long long *__restrict__ rankw,
+                                                            uint4 *__restrict__ rsect,
                                                             uint2 *__restrict__ buckets,
                                                             const uint32_t *__restrict__ chunk_first,
                                                             const uint32_t *__restrict__ rank0) {
@@ -171,14 +177,20 @@ __global__ void __launch_bounds__(kFillThreads) k_ptrs_fill(const uint32_t *__re
     // word} and the compact {first slot, count} table, in bucket order
     const uint64_t rank = uint64_t(rank0[c]) + preo;
     uint64_t r = rank;
+    const uint32_t group_first = pre;
+    uint64_t c2 = 0;  // 2-bit saturating count per seed of the group
 #pragma unroll 4
     for (int j = 0; j < kPer; ++j) {
         const uint32_t x = cnt[tid * (kPer + 1) + j];
         cnt[tid * (kPer + 1) + j] = pre;
         if (x) buckets[r++] = make_uint2(pre, x);
+        if (kSect) c2 |= uint64_t(x < 3 ? x : 3u) << (2 * j);
         pre += x;
     }
-    if (s0 + uint64_t(tid) * kPer < n_buckets) rankw[(s0 >> 5) + tid] = (rank << 32) | occ;
+    if (s0 + uint64_t(tid) * kPer < n_buckets) {
+        if (kSect) rsect[(s0 >> 5) + tid] = make_uint4(group_first, uint32_t(rank), uint32_t(c2), uint32_t(c2 >> 32));
+        else rankw[(s0 >> 5) + tid] = (rank << 32) | occ;
+    }
     __syncthreads();
     // coalesced write-out of the chunk's ptrs, 16 bytes per store
     const uint64_t lim = n_buckets - s0 < uint64_t(kChunk) ? n_buckets - s0 : uint64_t(kChunk);
@@ -250,7 +262,8 @@ size_t ptrs_fill_scratch_bytes(uint32_t ls) {
 }
 
 cudaError_t launch_ptrs_fill(const uint32_t *sorted_codes, uint64_t n_locs, uint32_t ls, uint32_t *ptrs,
-                             unsigned long long *rankw, uint2 *buckets, void *scratch, cudaStream_t s) {
+                             unsigned long long *rankw, uint4 *rsect, uint2 *buckets, void *scratch,
+                             cudaStream_t s) {
     const uint64_t nb = 1ull << (2 * ls);
     const uint64_t chunks = (nb + kChunk - 1) / kChunk;
     auto align = [](uintptr_t p) { return (p + 255) & ~uintptr_t(255); };
@@ -268,12 +281,18 @@ cudaError_t launch_ptrs_fill(const uint32_t *sorted_codes, uint64_t n_locs, uint
     constexpr int smem = (kChunk + kChunk / 32) * 4;
     static bool attr = false;
     if (!attr) {
-        e = cudaFuncSetAttribute(k_ptrs_fill, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+        e = cudaFuncSetAttribute(k_ptrs_fill<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+        if (e != cudaSuccess) return e;
+        e = cudaFuncSetAttribute(k_ptrs_fill<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
         if (e != cudaSuccess) return e;
         attr = true;
     }
-    k_ptrs_fill<<<unsigned(chunks), kFillThreads, smem, s>>>(sorted_codes, n_locs, nb, ptrs, rankw, buckets, first,
-                                                         rank0);
+    if (rsect)
+        k_ptrs_fill<true><<<unsigned(chunks), kFillThreads, smem, s>>>(sorted_codes, n_locs, nb, ptrs, rankw, rsect,
+                                                                       buckets, first, rank0);
+    else
+        k_ptrs_fill<false><<<unsigned(chunks), kFillThreads, smem, s>>>(sorted_codes, n_locs, nb, ptrs, rankw, rsect,
+                                                                        buckets, first, rank0);
     note_launch(4);
     return cudaGetLastError();
 }

@@ -19,7 +19,9 @@ struct Options {
                                  // (radix.cu), 2 = MSD bucket sort (msd.cu)
     int64_t small_sort = 0;      // 1: single-launch cooperative sorts when the input fits (small_sort.cu;
                                  // measured slower at C4: its scattered global writes are not coalesced)
-    int64_t index_msd = 0;       // index sort: 1 = MSD bucket sort of (code << 32 | p), 0 = stable LSD radix
+    int64_t index_msd = 0;
+    int64_t rank_sectors = -1;   // lookup directory: -1 auto (sectors when the compact table exceeds L2/4),
+                                 // 0 rank words, 1 rank sectors       // index sort: 1 = MSD bucket sort of (code << 32 | p), 0 = stable LSD radix
     int64_t radix_bits = 0;      // LSD digit width: 0 = 9 bits if that saves a pass else 8; or pinned 8, 9, 10
 };
 extern Options g_opt;
@@ -82,7 +84,8 @@ cudaError_t launch_seed_codes(const uint64_t *R, uint32_t ls, uint32_t step, uin
                               uint32_t *codes, uint32_t *locs, cudaStream_t s);
 size_t ptrs_fill_scratch_bytes(uint32_t ls);
 cudaError_t launch_ptrs_fill(const uint32_t *sorted_codes, uint64_t n_locs, uint32_t ls, uint32_t *ptrs,
-                             unsigned long long *rankw, uint2 *buckets, void *scratch, cudaStream_t s);
+                             unsigned long long *rankw, uint4 *rsect, uint2 *buckets, void *scratch,
+                             cudaStream_t s);
 // Seed records for the lookup: rec[k] = {locs[k], 16 bases left of it, 32 bases right of its seed}.
 cudaError_t launch_seed_recs(const uint64_t *R, uint32_t ls, const uint32_t *locs, uint64_t n_locs, uint4 *recs,
                              cudaStream_t s);
@@ -97,6 +100,8 @@ struct FindParams {
     const uint32_t *ptrs;
     const uint4 *recs;           // seed records, parallel to locs: {p, R[p-16,p), R[p+ls,p+ls+32)}
     const unsigned long long *rankw;  // per 32 seeds: {occupancy bits (low 32), occupied seeds before (high 32)}
+    const uint4 *rsect;          // or (large indexes) per 32 seeds: {records before, occupied seeds before,
+                                 // 2-bit saturating counts lo, hi}; exactly one of rankw / rsect is set
     const uint2 *buckets;        // per occupied seed, in seed order: {first slot in locs, count}
     uint32_t ls, L, step, qbits;
     uint64_t scan_lo, scan_hi;   // query seed positions scanned

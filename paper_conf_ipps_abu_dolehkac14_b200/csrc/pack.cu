@@ -1,7 +1,7 @@
 // pack.cu -- K1: ASCII -> 2-bit packed words.
 //
-// One thread per output word = 32 input bytes, read as two 128-bit vector loads
-// when the input is 16-byte aligned (scalar bytes otherwise and for the tail).
+// One thread per kWPT output words = 32 input bytes each, read as two 128-bit vector
+// loads when the input is 16-byte aligned (scalar bytes otherwise and for the tail).
 // Per 4 bytes (SWAR): code = ((c>>1) ^ (c>>2)) & 3 maps A/a->0 C/c->1 G/g->2
 // T/t->3; validity is checked exactly by rebuilding the expected upper-case
 // byte from the code with one PRMT and comparing. The first invalid position
@@ -24,44 +24,70 @@ __device__ __forceinline__ uint32_t pack4(uint32_t x, bool &ok) {
     return (c * 0x40100401u) >> 24;                                  // c0<<6|c1<<4|c2<<2|c3
 }
 
+#ifndef GM_PACK_WPT
+#define GM_PACK_WPT 4
+#endif
+constexpr int kWPT = GM_PACK_WPT;  // output words per thread (all input loads issued first)
+
+// word w from 32 ASCII bytes (the scalar path handles unaligned input and the tail)
+__device__ __forceinline__ uint64_t pack_word_scalar(const uint8_t *__restrict__ in, uint64_t n, uint64_t w,
+                                                     unsigned long long *bad_pos) {
+    uint64_t word = 0;
+    const uint64_t base = w * 32;
+    for (int i = 0; i < 32; ++i) {
+        const uint64_t pos = base + i;
+        if (pos >= n) break;  // padding bases stay 00
+        const uint32_t ch = in[pos];
+        const uint32_t c = ((ch >> 1) ^ (ch >> 2)) & 3u;
+        const uint32_t up = ch & 0xDFu;
+        if (up != 'A' && up != 'C' && up != 'G' && up != 'T') atomicMin(bad_pos, (unsigned long long)pos);
+        word |= uint64_t(c) << (62 - 2 * i);
+    }
+    return word;
+}
+
+__device__ __noinline__ void report_bad(const uint8_t *__restrict__ in, uint64_t w, unsigned long long *bad_pos) {
+    for (int i = 0; i < 32; ++i) {  // locate the first bad byte of this word
+        const uint32_t up = in[w * 32 + i] & 0xDFu;
+        if (up != 'A' && up != 'C' && up != 'G' && up != 'T') {
+            atomicMin(bad_pos, (unsigned long long)(w * 32 + i));
+            break;
+        }
+    }
+}
+
+// Thread t packs words t, t + T, ..., t + (kWPT - 1) T of its CTA's span (T = threads):
+// every load of the thread is in flight before the first word is assembled.
 __global__ void __launch_bounds__(kPackThreads) k_pack(const uint8_t *__restrict__ in, uint64_t n,
                                                        uint64_t *__restrict__ words, uint64_t n_full,
                                                        uint64_t n_words_alloc, unsigned long long *bad_pos,
                                                        int aligned) {
-    const uint64_t w = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
-    if (w >= n_words_alloc) return;
-    uint64_t word = 0;
-    bool ok = true;
-    if (w < n_full && aligned) {
-        const uint4 a = __ldcs(reinterpret_cast<const uint4 *>(in) + 2 * w);      // streamed once
-        const uint4 b = __ldcs(reinterpret_cast<const uint4 *>(in) + 2 * w + 1);
-        const uint32_t v[8] = {a.x, a.y, a.z, a.w, b.x, b.y, b.z, b.w};
+    const uint64_t w0 = uint64_t(blockIdx.x) * kPackThreads * kWPT + threadIdx.x;
+    uint4 a[kWPT], b[kWPT];
 #pragma unroll
-        for (int j = 0; j < 8; ++j) word |= uint64_t(pack4(v[j], ok)) << (56 - 8 * j);
-    } else {
-        const uint64_t base = w * 32;
-        for (int i = 0; i < 32; ++i) {
-            const uint64_t pos = base + i;
-            if (pos >= n) break;  // padding bases stay 00
-            const uint32_t ch = in[pos];
-            const uint32_t c = ((ch >> 1) ^ (ch >> 2)) & 3u;
-            const uint32_t up = ch & 0xDFu;
-            if (up != 'A' && up != 'C' && up != 'G' && up != 'T') {
-                atomicMin(bad_pos, (unsigned long long)pos);
-            }
-            word |= uint64_t(c) << (62 - 2 * i);
+    for (int k = 0; k < kWPT; ++k) {
+        const uint64_t w = w0 + uint64_t(k) * kPackThreads;
+        if (aligned && w < n_full) {
+            a[k] = __ldcs(reinterpret_cast<const uint4 *>(in) + 2 * w);  // streamed once
+            b[k] = __ldcs(reinterpret_cast<const uint4 *>(in) + 2 * w + 1);
         }
     }
-    if (!ok) {  // locate the first bad byte of this word
-        for (int i = 0; i < 32; ++i) {
-            const uint32_t up = in[w * 32 + i] & 0xDFu;
-            if (up != 'A' && up != 'C' && up != 'G' && up != 'T') {
-                atomicMin(bad_pos, (unsigned long long)(w * 32 + i));
-                break;
-            }
+#pragma unroll
+    for (int k = 0; k < kWPT; ++k) {
+        const uint64_t w = w0 + uint64_t(k) * kPackThreads;
+        if (w >= n_words_alloc) break;
+        uint64_t word = 0;
+        if (aligned && w < n_full) {
+            bool ok = true;
+            const uint32_t v[8] = {a[k].x, a[k].y, a[k].z, a[k].w, b[k].x, b[k].y, b[k].z, b[k].w};
+#pragma unroll
+            for (int j = 0; j < 8; ++j) word |= uint64_t(pack4(v[j], ok)) << (56 - 8 * j);
+            if (!ok) report_bad(in, w, bad_pos);
+        } else {
+            word = pack_word_scalar(in, n, w, bad_pos);
         }
+        words[w] = word;
     }
-    words[w] = word;
 }
 
 // Reverse complement of a packed sequence (NEXT-F4): rc[i] = 3 - s[n-1-i] (A<->T, C<->G
@@ -106,7 +132,7 @@ cudaError_t launch_pack(const uint8_t *in, uint64_t n, uint64_t *words, uint64_t
                         unsigned long long *bad_pos, cudaStream_t s) {
     const int aligned = (reinterpret_cast<uintptr_t>(in) & 15) == 0;
     const uint64_t n_full = n / 32;
-    const uint64_t blocks = (n_words_alloc + kPackThreads - 1) / kPackThreads;
+    const uint64_t blocks = (n_words_alloc + uint64_t(kPackThreads) * kWPT - 1) / (uint64_t(kPackThreads) * kWPT);
     k_pack<<<unsigned(blocks), kPackThreads, 0, s>>>(in, n, words, n_full, n_words_alloc, bad_pos, aligned);
     note_launch();
     return cudaGetLastError();
