@@ -26,8 +26,13 @@
 namespace gm {
 namespace {
 
-constexpr int kT = 256;  // threads per CTA
+constexpr int kT = 256;  // threads per CTA of the histogram / scan kernels
 constexpr int kWarps = kT / 32;
+#ifndef GM_RADIX_ST
+#define GM_RADIX_ST 256
+#endif
+constexpr int kST = GM_RADIX_ST;  // threads per CTA of k_scatter (512 x 8 items measured slower)
+constexpr int kSW = kST / 32;
 
 #ifndef GM_RADIX_ITEMS32
 #define GM_RADIX_ITEMS32 16
@@ -51,7 +56,7 @@ struct Cfg<uint64_t> {
 
 template <class K>
 constexpr uint64_t tile_items() {
-    return uint64_t(kT) * Cfg<K>::kItems;
+    return uint64_t(kST) * Cfg<K>::kItems;  // one k_scatter tile
 }
 
 // Lanes of the warp holding the same digit (among lanes with valid == true), built
@@ -173,11 +178,11 @@ __global__ void __launch_bounds__(kT) k_chunk_scan(const uint32_t *__restrict__ 
 // buffer.
 template <class K, class V, int RB>
 struct alignas(128) ScatterSmem {
-    K k[2][kT * Cfg<K>::kItems];
-    V v[2][kT * Cfg<K>::kItems];
-    uint32_t wcnt[kWarps][1 << RB];
+    K k[2][kST * Cfg<K>::kItems];
+    V v[2][kST * Cfg<K>::kItems];
+    uint32_t wcnt[kSW][1 << RB];
     uint32_t gofs[1 << RB];  // per digit: global position of the tile's slot 0 (mod 2^32)
-    uint32_t ws[kWarps * ((1 << RB) / kT)];
+    uint32_t ws[kSW * (((1 << RB) + kST - 1) / kST)];
     unsigned long long bar[2];
 };
 
@@ -199,13 +204,13 @@ __device__ __forceinline__ void mbar_wait(unsigned long long *bar, uint32_t pari
 }
 
 template <class K, class V, int RB>
-__global__ void __launch_bounds__(kT, GM_RADIX_MINB) k_scatter(const K *__restrict__ kin, const V *__restrict__ vin,
+__global__ void __launch_bounds__(kST, GM_RADIX_MINB) k_scatter(const K *__restrict__ kin, const V *__restrict__ vin,
                                                   K *__restrict__ kout, V *__restrict__ vout, Chunking ch,
                                                   int shift, int bits, const uint32_t *__restrict__ offs) {
     constexpr int kBins = 1 << RB;
-    constexpr int DPT = kBins / kT;  // digits owned per thread: tid, tid + kT, ...
+    constexpr int DPT = (kBins + kST - 1) / kST;  // digits owned per thread: tid, tid + kST, ... (< kBins)
     constexpr int kItems = Cfg<K>::kItems;
-    constexpr int kTile = kT * kItems;
+    constexpr int kTile = kST * kItems;
     extern __shared__ __align__(128) unsigned char smem_raw[];
     ScatterSmem<K, V, RB> &S = *reinterpret_cast<ScatterSmem<K, V, RB> *>(smem_raw);
     const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
@@ -230,13 +235,14 @@ __global__ void __launch_bounds__(kT, GM_RADIX_MINB) k_scatter(const K *__restri
     }
     uint32_t gbase[DPT];  // running global offset of each owned digit in this chunk
 #pragma unroll
-    for (int dd = 0; dd < DPT; ++dd) gbase[dd] = offs[uint64_t(dd * kT + tid) * ch.chunks + c];
+    for (int dd = 0; dd < DPT; ++dd)
+        gbase[dd] = dd * kST + tid < kBins ? offs[uint64_t(dd * kST + tid) * ch.chunks + c] : 0u;
     __syncthreads();
 
     for (uint32_t t = 0; t < n_t; ++t) {
         const int sg = t & 1;
         if (tid == 0 && t + 1 < n_full) issue(t + 1, sg ^ 1);  // buffer sg^1 was released at the end of tile t-1
-        for (int i = tid; i < kWarps * kBins; i += kT) (&S.wcnt[0][0])[i] = 0;
+        for (int i = tid; i < kSW * kBins; i += kST) (&S.wcnt[0][0])[i] = 0;
         const uint64_t base = cb + uint64_t(t) * kTile;
         const uint32_t tile_n = uint32_t(min(uint64_t(kTile), ce - base));
 
@@ -282,14 +288,13 @@ __global__ void __launch_bounds__(kT, GM_RADIX_MINB) k_scatter(const K *__restri
 
         // ---- per digit: tile count, tile-local exclusive offset (block scan); then each
         //      warp's slot base in the reorder buffer and the tile-to-global offset
-        uint32_t cnt[DPT], inc[DPT], xw[DPT][kWarps];
+        uint32_t cnt[DPT], inc[DPT];
 #pragma unroll
         for (int dd = 0; dd < DPT; ++dd) {
             uint32_t c0 = 0;
+            if (dd * kST + tid < kBins) {
 #pragma unroll
-            for (int ww = 0; ww < kWarps; ++ww) {
-                xw[dd][ww] = S.wcnt[ww][dd * kT + tid];
-                c0 += xw[dd][ww];
+                for (int ww = 0; ww < kSW; ++ww) c0 += S.wcnt[ww][dd * kST + tid];
             }
             cnt[dd] = inc[dd] = c0;
         }
@@ -303,7 +308,7 @@ __global__ void __launch_bounds__(kT, GM_RADIX_MINB) k_scatter(const K *__restri
         }
         if (lane == 31) {
 #pragma unroll
-            for (int dd = 0; dd < DPT; ++dd) S.ws[dd * kWarps + w] = inc[dd];
+            for (int dd = 0; dd < DPT; ++dd) S.ws[dd * kSW + w] = inc[dd];
         }
         __syncthreads();
         {
@@ -312,22 +317,25 @@ __global__ void __launch_bounds__(kT, GM_RADIX_MINB) k_scatter(const K *__restri
             for (int dd = 0; dd < DPT; ++dd) {
                 uint32_t pre = 0, seg = 0;
 #pragma unroll
-                for (int i = 0; i < kWarps; ++i) {
-                    const uint32_t x = S.ws[dd * kWarps + i];
+                for (int i = 0; i < kSW; ++i) {
+                    const uint32_t x = S.ws[dd * kSW + i];
                     pre += i < w ? x : 0u;
                     seg += x;
                 }
                 const uint32_t excl = carry + pre + inc[dd] - cnt[dd];
                 carry += seg;
-                const uint32_t d = dd * kT + tid;
-                uint32_t run = excl;
+                const uint32_t d = dd * kST + tid;
+                if (d < kBins) {
+                    uint32_t run = excl;
 #pragma unroll
-                for (int ww = 0; ww < kWarps; ++ww) {
-                    S.wcnt[ww][d] = run;
-                    run += xw[dd][ww];
+                    for (int ww = 0; ww < kSW; ++ww) {
+                        const uint32_t x = S.wcnt[ww][d];
+                        S.wcnt[ww][d] = run;
+                        run += x;
+                    }
+                    S.gofs[d] = gbase[dd] - excl;  // slot i of digit d goes to gofs[d] + i (mod 2^32)
+                    gbase[dd] += cnt[dd];
                 }
-                S.gofs[d] = gbase[dd] - excl;  // slot i of digit d goes to gofs[d] + i (mod 2^32)
-                gbase[dd] += cnt[dd];
             }
         }
         __syncthreads();
@@ -353,9 +361,9 @@ __global__ void __launch_bounds__(kT, GM_RADIX_MINB) k_scatter(const K *__restri
         };
         if (tile_n == kTile) {
 #pragma unroll
-            for (int j = 0; j < kItems; ++j) put(j * kT + tid);
+            for (int j = 0; j < kItems; ++j) put(j * kST + tid);
         } else {
-            for (uint32_t i = tid; i < tile_n; i += kT) put(i);
+            for (uint32_t i = tid; i < tile_n; i += kST) put(i);
         }
         __syncthreads();  // buffer sg, wcnt and gofs free for the next tiles
     }
@@ -385,7 +393,7 @@ cudaError_t radix_sort_rb(K *k0, uint32_t *v0, K *k1, uint32_t *v1, uint64_t n, 
         e = cudaFuncSetAttribute(k_scatter<K, uint32_t, RB>, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
         if (e != cudaSuccess) return e;
         int per_sm = 0;
-        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_scatter<K, uint32_t, RB>, kT, smem);
+        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_scatter<K, uint32_t, RB>, kST, smem);
         if (e != cudaSuccess) return e;
         grid_cap = (per_sm > 0 ? per_sm : 1) * num_sms();
         if (grid_cap > kMaxChunks) grid_cap = kMaxChunks;
@@ -408,7 +416,7 @@ cudaError_t radix_sort_rb(K *k0, uint32_t *v0, K *k1, uint32_t *v1, uint64_t n, 
         uint32_t *tot = totals + size_t(p) * kBins;
         k_chunk_hist<K, RB><<<ch.chunks, kT, 0, s>>>(ka, ch, RB * p, dbits, counts, tot);
         k_chunk_scan<RB><<<kBins / kWarps, kT, 0, s>>>(counts, tot, ch.chunks, offs);
-        k_scatter<K, uint32_t, RB><<<ch.chunks, kT, smem, s>>>(ka, va, kb, vb, ch, RB * p, dbits, offs);
+        k_scatter<K, uint32_t, RB><<<ch.chunks, kST, smem, s>>>(ka, va, kb, vb, ch, RB * p, dbits, offs);
         note_launch(3);
         std::swap(ka, kb);
         std::swap(va, vb);
