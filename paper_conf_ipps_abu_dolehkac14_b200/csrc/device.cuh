@@ -61,6 +61,14 @@ __device__ __forceinline__ uint4 ld_last_u4(const uint4 *a) {
     GM_LD_HINT("evict_last", ".v4.u32", "", "{%0, %1, %2, %3}, [%4]", : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(a));
     return v;
 }
+__device__ __forceinline__ uint2 ld_hint_u2(const uint2 *a, bool stream) {
+    uint2 v;
+    if (stream)
+        GM_LD_HINT("evict_first", ".v2.u32", ".L1::no_allocate", "{%0, %1}, [%2]", : "=r"(v.x), "=r"(v.y) : "l"(a));
+    else
+        GM_LD_HINT("evict_last", ".v2.u32", ".L1::no_allocate", "{%0, %1}, [%2]", : "=r"(v.x), "=r"(v.y) : "l"(a));
+    return v;
+}
 __device__ __forceinline__ uint4 ld_hint_u4(const uint4 *a, bool stream) {
     uint4 v;
     if (stream)

@@ -59,7 +59,7 @@ constexpr uint32_t kLaneCap = 4096;       // bases one lane extends before the w
 constexpr int kDQ = 64;                   // deferred-extension queue entries per warp
 
 struct WarpSmem {
-    uint4 dq[kDQ];                        // {p, q, e (or kUnresolved), 0}: hits needing global extension
+    uint4 dq[kDQ];                        // {p, q, e (or kUnresolved), known right}: hits needing global extension
     uint64_t qw[kQW];
     uint32_t e_beg[kChunk];
     uint32_t e_off[kChunk + 1];
@@ -165,53 +165,24 @@ __device__ __forceinline__ uint32_t ext_left(const uint64_t *__restrict__ R, con
     return min(e, lim);
 }
 
-// Decide one hit: seed of R at p equals seed of Q at q. rleft = R[p-16, p) (base p-1
-// lowest), rright = R[p+ls, p+ls+32) (first base highest); qleft/qright likewise for Q.
-// Extensions beyond the record use global multi-window rounds, at most kLaneCap bases
-// per lane; a longer one returns kDefer and goes to the coop queue (k_coop).
-__device__ __forceinline__ int decide(const FindParams &P, uint32_t p, uint32_t rleft, uint64_t rright,
-                                      uint32_t q, uint32_t qleft, uint64_t qright, Hit &out) {
-    // A7: left extension, capped at step
-    const uint32_t lim = min(P.step, min(p, q));
-    const uint32_t xl = rleft ^ qleft;
-    uint32_t e = xl ? uint32_t(__ffs(int(xl)) - 1) >> 1 : 16u;
-    if (e == 16 && lim > 16) {
-        e = ext_left(P.R, P.Q, p, q, 16, lim, kLaneCap);
-        if (e == kUnresolved) return kDefer;
-    }
-    e = min(e, lim);
-    if (e == P.step) return kDrop;                         // not the canonical (leftmost) seed
-    const uint32_t qs = q - e;
-    if (qs < P.own_lo || qs >= P.own_hi) return kDrop;     // another shard owns it
-    // A8: right extension from the end of the seed
-    const uint32_t a = p + P.ls, b = q + P.ls;
-    const uint32_t lim_r = min(uint32_t(P.nR) - a, uint32_t(P.nQ) - b);
-    uint32_t f = lead_eq(rright ^ qright);
-    if (f == 32 && lim_r > 32) {
-        f = ext_right(P.R, P.Q, a, b, 32, lim_r, kLaneCap);
-        if (f == kUnresolved) return kDefer;
-    }
-    f = min(f, lim_r);
-    const uint32_t lam = e + P.ls + f;
-    if (lam < P.L) return kDrop;                           // A9
-    out.key = (uint64_t(p - e) << P.qbits) | qs;
-    out.len = lam;
-    return kEmit;
-}
-
-// The record-only part of decide(): kDrop / kEmit when the 16 + 32 flank bases settle
-// the hit, else kExt with e_out = the left extension if the record settled it, or
-// kUnresolved. kExt hits are queued per warp and finished 32 at a time by
-// decide_deferred(), so the (rare, long) global-memory extensions run with all lanes
-// busy instead of stalling a whole warp round for one lane.
+// The record-only part of decide(): kDrop / kEmit when the kL + kR flank bases of the
+// record (16 + 32 for 16-byte records, 8 + 8 for 8-byte records) settle the hit, else
+// kExt with e_out = the left extension if the record settled it, or kUnresolved. kExt
+// hits are queued per warp and finished 32 at a time by decide_deferred(), so the
+// (rare, long) global-memory extensions run with all lanes busy instead of stalling a
+// whole warp round for one lane.
 enum : int { kExt = 3 };
+template <int kL, int kR>
 __device__ __forceinline__ int decide_rec(const FindParams &P, uint32_t p, uint32_t rleft, uint64_t rright,
-                                          uint32_t q, uint32_t qleft, uint64_t qright, Hit &out, uint32_t &e_out) {
+                                          uint32_t q, uint32_t qleft, uint64_t qright, Hit &out, uint32_t &e_out,
+                                          uint32_t &f_out) {
     const uint32_t lim = min(P.step, min(p, q));
-    const uint32_t xl = rleft ^ qleft;
-    uint32_t e = xl ? uint32_t(__ffs(int(xl)) - 1) >> 1 : 16u;
-    if (e == 16 && lim > 16) {
+    const uint32_t lmask = kL >= 16 ? 0xffffffffu : ((1u << (2 * kL)) - 1u);  // kL bases, base p-1 lowest
+    const uint32_t xl = (rleft ^ qleft) & lmask;
+    uint32_t e = xl ? uint32_t(__ffs(int(xl)) - 1) >> 1 : uint32_t(kL);
+    if (e == kL && lim > kL) {
         e_out = kUnresolved;
+        f_out = 0;
         return kExt;
     }
     e = min(e, lim);
@@ -220,9 +191,12 @@ __device__ __forceinline__ int decide_rec(const FindParams &P, uint32_t p, uint3
     if (qs < P.own_lo || qs >= P.own_hi) return kDrop;
     const uint32_t a = p + P.ls, b = q + P.ls;
     const uint32_t lim_r = min(uint32_t(P.nR) - a, uint32_t(P.nQ) - b);
-    uint32_t f = lead_eq(rright ^ qright);
-    if (f == 32 && lim_r > 32) {
+    const uint64_t rmask = kR >= 32 ? ~0ull : ~(~0ull >> (2 * kR));  // kR bases, first base highest
+    const uint64_t xr = (rright ^ qright) & rmask;
+    uint32_t f = xr ? uint32_t(__clzll(xr)) >> 1 : uint32_t(kR);
+    if (f == kR && lim_r > kR) {
         e_out = e;
+        f_out = kR;  // the record's right flank matched: the global extension starts past it
         return kExt;
     }
     f = min(f, lim_r);
@@ -233,13 +207,15 @@ __device__ __forceinline__ int decide_rec(const FindParams &P, uint32_t p, uint3
     return kEmit;
 }
 
-// The rest of decide() for a queued hit, from global memory (16 left bases already known
-// equal when e_in == kUnresolved).
-__device__ __forceinline__ int decide_deferred(const FindParams &P, uint32_t p, uint32_t q, uint32_t e_in, Hit &out) {
+// The rest of decide() for a queued hit, from global memory (kL left bases already known
+// equal when e_in == kUnresolved; f0 right bases known equal).
+template <int kL>
+__device__ __forceinline__ int decide_deferred(const FindParams &P, uint32_t p, uint32_t q, uint32_t e_in, uint32_t f0,
+                                               Hit &out) {
     const uint32_t lim = min(P.step, min(p, q));
     uint32_t e = e_in;
     if (e == kUnresolved) {
-        e = ext_left(P.R, P.Q, p, q, 16, lim, kLaneCap);
+        e = ext_left(P.R, P.Q, p, q, kL, lim, kLaneCap);
         if (e == kUnresolved) return kDefer;
     }
     e = min(e, lim);
@@ -248,7 +224,7 @@ __device__ __forceinline__ int decide_deferred(const FindParams &P, uint32_t p, 
     if (qs < P.own_lo || qs >= P.own_hi) return kDrop;
     const uint32_t a = p + P.ls, b = q + P.ls;
     const uint32_t lim_r = min(uint32_t(P.nR) - a, uint32_t(P.nQ) - b);
-    uint32_t f = ext_right(P.R, P.Q, a, b, 0, lim_r, kLaneCap);
+    uint32_t f = ext_right(P.R, P.Q, a, b, f0, lim_r, kLaneCap);
     if (f == kUnresolved) return kDefer;
     const uint32_t lam = e + P.ls + f;
     if (lam < P.L) return kDrop;
@@ -402,15 +378,29 @@ __device__ __forceinline__ void warp_emit(const FindParams &P, WarpSmem &s, uint
     }
 }
 
-__device__ __forceinline__ void load_rec(const uint4 *recs, uint32_t k, uint32_t &p, uint32_t &left,
+// Seed record k: 16-byte {p, R[p-16, p), R[p+ls, p+ls+32)} or, for 8-byte records,
+// {p, R[p-8, p) | R[p+ls, p+ls+8) << 16}; left flank base p-1 lowest, right flank first
+// base highest (the layout decide_rec<kL, kR> expects).
+template <bool kRec8>
+__device__ __forceinline__ void load_rec(const FindParams &P, uint64_t k, uint32_t &p, uint32_t &left,
                                          uint64_t &right, int stream) {
-    const uint4 r = stream < 0 ? __ldg(recs + k) : ld_hint_u4(recs + k, stream != 0);
-    p = r.x;
-    left = r.y;
-    right = (uint64_t(r.w) << 32) | r.z;
+    if (kRec8) {
+        const uint2 *r8 = reinterpret_cast<const uint2 *>(P.recs);
+        const uint2 r = stream < 0 ? __ldg(r8 + k) : ld_hint_u2(r8 + k, stream != 0);
+        p = r.x;
+        left = r.y & 0xffffu;
+        right = uint64_t(r.y >> 16) << 48;
+    } else {
+        const uint4 *r16 = reinterpret_cast<const uint4 *>(P.recs);
+        const uint4 r = stream < 0 ? __ldg(r16 + k) : ld_hint_u4(r16 + k, stream != 0);
+        p = r.x;
+        left = r.y;
+        right = (uint64_t(r.w) << 32) | r.z;
+    }
 }
 
 // One converged extension round: the last `take` (<= 32) queued hits, one per lane.
+template <int kL>
 __device__ __forceinline__ void drain_deferred(const FindParams &P, WarpSmem &s, uint32_t &nq, uint32_t &nbuf,
                                                uint32_t take) {
     const int lane = threadIdx.x & 31;
@@ -421,7 +411,7 @@ __device__ __forceinline__ void drain_deferred(const FindParams &P, WarpSmem &s,
         const uint4 d = s.dq[nq - take + lane];
         p = d.x;
         q = d.y;
-        verdict = decide_deferred(P, p, q, d.z, out);
+        verdict = decide_deferred<kL>(P, p, q, d.z, d.w, out);
     }
     __syncwarp();
     nq -= take;
@@ -432,8 +422,9 @@ __device__ __forceinline__ void drain_deferred(const FindParams &P, WarpSmem &s,
 #ifndef GM_FIND_MINB
 #define GM_FIND_MINB 4
 #endif
-template <bool kStatic, bool kHints, bool kSect>
+template <bool kStatic, bool kHints, bool kSect, bool kRec8>
 __global__ void __launch_bounds__(kT, GM_FIND_MINB) k_find(const FindParams P) {
+    constexpr int kL = kRec8 ? 8 : 16, kR = kRec8 ? 8 : 32;  // record flank widths (bases)
     __shared__ WarpSmem smem[kWarps];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     WarpSmem &s = smem[wid];
@@ -610,7 +601,7 @@ __global__ void __launch_bounds__(kT, GM_FIND_MINB) k_find(const FindParams P) {
                     const bool has = kStatic ? rd < n_h : h < H;
                     int verdict = kDrop;
                     Hit out{0, 0};
-                    uint32_t p = 0, q = 0, e_rec = 0;
+                    uint32_t p = 0, q = 0, e_rec = 0, f_rec = 0;
                     if (has) {
                         uint32_t lo = 0, hi = E;  // largest entry i with e_off[i] <= h
                         while (hi - lo > 1) {
@@ -620,24 +611,25 @@ __global__ void __launch_bounds__(kT, GM_FIND_MINB) k_find(const FindParams P) {
                         q = q0 + s.e_q[lo];
                         uint32_t rl;
                         uint64_t rr;
-                        load_rec(P.recs, s.e_beg[lo] + (h - s.e_off[lo]), p, rl, rr, kHints ? 1 : -1);
-                        verdict = decide_rec(P, p, rl, rr, q, qs.back16(q), qs.fwd(q + P.ls), out, e_rec);
+                        load_rec<kRec8>(P, s.e_beg[lo] + (h - s.e_off[lo]), p, rl, rr, kHints ? 1 : -1);
+                        verdict = decide_rec<kL, kR>(P, p, rl, rr, q, qs.back16(q), qs.fwd(q + P.ls), out, e_rec,
+                                                     f_rec);
                     }
                     // hits the records cannot settle wait in the warp's queue
                     const unsigned need = __ballot_sync(0xffffffffu, verdict == kExt);
                     if (need) {
-                        if (verdict == kExt) s.dq[nq + __popc(need & lanemask_lt())] = make_uint4(p, q, e_rec, 0u);
+                        if (verdict == kExt) s.dq[nq + __popc(need & lanemask_lt())] = make_uint4(p, q, e_rec, f_rec);
                         nq += __popc(need);
                         __syncwarp();
                     }
                     warp_emit(P, s, nbuf, verdict == kEmit, out, false);
-                    if (nq >= 32) drain_deferred(P, s, nq, nbuf, 32);
+                    if (nq >= 32) drain_deferred<kL>(P, s, nq, nbuf, 32);
                 }
             }
             __syncwarp();
         }
     }
-    if (nq) drain_deferred(P, s, nq, nbuf, nq);
+    if (nq) drain_deferred<kL>(P, s, nq, nbuf, nq);
     warp_emit(P, s, nbuf, false, Hit{0, 0}, true);
     if (lane == 0 && st_e) {
         atomicAdd(&P.stats[0], st_e);
@@ -646,7 +638,9 @@ __global__ void __launch_bounds__(kT, GM_FIND_MINB) k_find(const FindParams P) {
 }
 
 // K7: drain the heavy-bucket queue, one 32-hit piece per warp iteration.
+template <bool kRec8>
 __global__ void __launch_bounds__(kT) k_heavy(const FindParams P) {
+    constexpr int kL = kRec8 ? 8 : 16, kR = kRec8 ? 8 : 32;
     __shared__ WarpSmem smem[kWarps];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     WarpSmem &s = smem[wid];
@@ -662,10 +656,12 @@ __global__ void __launch_bounds__(kT) k_heavy(const FindParams P) {
         uint32_t p = 0;
         const uint32_t q = piece.x;
         if (uint32_t(lane) < piece.z) {
-            uint32_t rl;
+            uint32_t rl, e_rec = 0, f_rec = 0;
             uint64_t rr;
-            load_rec(P.recs, piece.y + lane, p, rl, rr, P.recs_stream);
-            verdict = decide(P, p, rl, rr, q, uint32_t(win_back(P.Q, q)), win_fwd(P.Q, uint64_t(q) + P.ls), out);
+            load_rec<kRec8>(P, piece.y + lane, p, rl, rr, P.recs_stream);
+            verdict = decide_rec<kL, kR>(P, p, rl, rr, q, uint32_t(win_back(P.Q, q)), win_fwd(P.Q, uint64_t(q) + P.ls),
+                                         out, e_rec, f_rec);
+            if (verdict == kExt) verdict = decide_deferred<kL>(P, p, q, e_rec, f_rec, out);
         }
         push_coop(P, verdict, p, q);
         warp_emit(P, s, nbuf, verdict == kEmit, out, false);
@@ -704,7 +700,7 @@ uint64_t find_tile_positions() { return kChunk; }
 int find_default_grid() {
     if (!g_default_grid) {
         int per_sm = 0;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_find<false, false, false>, kT, 0);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_find<false, false, false, false>, kT, 0);
         if (per_sm < 1) per_sm = 1;
         g_default_grid = per_sm * num_sms();
     }
@@ -720,16 +716,20 @@ cudaError_t launch_find(const FindParams &p, int grid, cudaStream_t s) {
     // kHints: the seed records exceed half of L2 -> cache-policy loads (lookup tables
     // evict_last, streams evict_first); otherwise plain loads (measured faster there)
     const bool sect = p.rsect != nullptr;
-    if (p.static_lb) {
-        if (sect) k_find<true, false, true><<<grid, kT, 0, s>>>(p);
-        else k_find<true, false, false><<<grid, kT, 0, s>>>(p);
-    } else if (p.recs_stream) {
-        if (sect) k_find<false, true, true><<<grid, kT, 0, s>>>(p);
-        else k_find<false, true, false><<<grid, kT, 0, s>>>(p);
-    } else {
-        if (sect) k_find<false, false, true><<<grid, kT, 0, s>>>(p);
-        else k_find<false, false, false><<<grid, kT, 0, s>>>(p);
-    }
+#define GM_FIND_LAUNCH(ST, HI)                                                              \
+    do {                                                                                    \
+        if (sect) {                                                                         \
+            if (p.rec8) k_find<ST, HI, true, true><<<grid, kT, 0, s>>>(p);                  \
+            else k_find<ST, HI, true, false><<<grid, kT, 0, s>>>(p);                        \
+        } else {                                                                            \
+            if (p.rec8) k_find<ST, HI, false, true><<<grid, kT, 0, s>>>(p);                 \
+            else k_find<ST, HI, false, false><<<grid, kT, 0, s>>>(p);                       \
+        }                                                                                   \
+    } while (0)
+    if (p.static_lb) GM_FIND_LAUNCH(true, false);
+    else if (p.recs_stream) GM_FIND_LAUNCH(false, true);
+    else GM_FIND_LAUNCH(false, false);
+#undef GM_FIND_LAUNCH
     note_launch();
     return cudaGetLastError();
 }
@@ -741,7 +741,8 @@ cudaError_t launch_coop(const FindParams &p, cudaStream_t s) {
 }
 
 cudaError_t launch_heavy(const FindParams &p, cudaStream_t s) {
-    k_heavy<<<num_sms() * 4, kT, 0, s>>>(p);
+    if (p.rec8) k_heavy<true><<<num_sms() * 4, kT, 0, s>>>(p);
+    else k_heavy<false><<<num_sms() * 4, kT, 0, s>>>(p);
     note_launch();
     return cudaGetLastError();
 }

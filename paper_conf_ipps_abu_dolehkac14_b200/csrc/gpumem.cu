@@ -38,7 +38,8 @@ struct gpumem_index {
     unsigned long long *rankw;   // rank words, 8 B per 32 seeds, or
     uint4 *rsect;                // rank sectors, 16 B per 32 seeds (index.cu); one of the two is null
     uint2 *buckets;
-    uint4 *recs;
+    void *recs;                  // uint4 records, or uint2 when rec8
+    int rec8;
 };
 
 struct gpumem_mems {
@@ -325,6 +326,7 @@ gpumem_status gpumem_set_option(const char *name, int64_t value) {
     }
     else if (!strcmp(name, "index_msd")) g_opt.index_msd = value ? 1 : 0;
     else if (!strcmp(name, "small_sort")) g_opt.small_sort = value ? 1 : 0;
+    else if (!strcmp(name, "rec8")) g_opt.rec8 = value < 0 ? -1 : (value ? 1 : 0);
     else if (!strcmp(name, "rank_sectors")) g_opt.rank_sectors = value < 0 ? -1 : (value ? 1 : 0);
     else if (!strcmp(name, "radix_bits")) {
         if (value != 0 && (value < 8 || value > 10)) return fail(GPUMEM_ERR_ARG, "radix_bits must be 0 or 8..10");
@@ -533,17 +535,19 @@ static gpumem_status index_build_impl(const gpumem_seq *R, uint32_t ls, uint32_t
     if (!ptrs || !(rsect || rankw) || !buckets || !fill_scratch || !locs0) return GPUMEM_ERR_NOMEM;
     uint32_t *locs = locs0;
     const uint32_t *codes_sorted = nullptr;
-    auto *recs = static_cast<uint4 *>(sc.get((n_locs ? n_locs : 1) * sizeof(uint4)));
+    // 8-byte seed records when the left extension is capped at <= 8 bases (step <= 8)
+    const int rec8 = g_opt.rec8 < 0 ? (step <= 8 ? 1 : 0) : int(g_opt.rec8 != 0);
+    void *recs = sc.get((n_locs ? n_locs : 1) * (rec8 ? sizeof(uint2) : sizeof(uint4)));
     if (!recs) return GPUMEM_ERR_NOMEM;
     bool recs_done = false;
-    if (n_locs && !g_opt.index_msd && g_opt.small_sort && n_locs <= small_sort_max_n(4)) {
+    if (n_locs && !rec8 && !g_opt.index_msd && g_opt.small_sort && n_locs <= small_sort_max_n(4)) {
         // one cooperative launch: seed codes from R, stable sort, codes + locs + records
         auto *codes1 = static_cast<uint32_t *>(ws_get(kWsCodes1, n_locs * 4, s));
         void *scratch = ws_get(kWsSmall, small_sort_scratch_bytes(n_locs, 4), s);
         if (!codes1 || !scratch) return GPUMEM_ERR_NOMEM;
         {
             Stage g("index.sort", s);
-            CK(small_sort_index(R->words, ls, step, k0, n_locs, codes1, locs0, recs, scratch, s), "seed sort");
+            CK(small_sort_index(R->words, ls, step, k0, n_locs, codes1, locs0, static_cast<uint4 *>(recs), scratch, s), "seed sort");
         }
         codes_sorted = codes1;
         recs_done = true;
@@ -582,7 +586,7 @@ static gpumem_status index_build_impl(const gpumem_seq *R, uint32_t ls, uint32_t
     }
     if (n_locs && !recs_done) {
         Stage g("index.recs", s);
-        CK(launch_seed_recs(R->words, ls, locs, n_locs, recs, s), "seed records");
+        CK(launch_seed_recs(R->words, ls, locs, n_locs, recs, rec8, s), "seed records");
     }
     sc.keep(ptrs);
     if (rankw) sc.keep(rankw);
@@ -590,7 +594,7 @@ static gpumem_status index_build_impl(const gpumem_seq *R, uint32_t ls, uint32_t
     sc.keep(buckets);
     sc.keep(locs);
     sc.keep(recs);
-    auto *h = new gpumem_index{kMagicIdx, dev, s, R, ls, L, step, n_locs, ptrs, locs, rankw, rsect, buckets, recs};
+    auto *h = new gpumem_index{kMagicIdx, dev, s, R, ls, L, step, n_locs, ptrs, locs, rankw, rsect, buckets, recs, rec8};
     *out = h;
     return GPUMEM_OK;
 }
@@ -676,6 +680,7 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
     P.nQw = Q->n_words;
     P.ptrs = idx->ptrs;
     P.recs = idx->recs;
+    P.rec8 = idx->rec8;
     P.rankw = idx->rankw;
     P.rsect = idx->rsect;
     P.buckets = idx->buckets;
@@ -701,7 +706,7 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
     {  // records that cannot share L2 with the lookup tables are streamed
         int l2 = 0;
         cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, dev);
-        P.recs_stream = idx->n_locs * 16 > uint64_t(l2) / 2 ? 1 : 0;
+        P.recs_stream = idx->n_locs * (idx->rec8 ? 8 : 16) > uint64_t(l2) / 2 ? 1 : 0;
     }
     uint64_t cap = g_opt.out_capacity ? uint64_t(g_opt.out_capacity) : (span / 8 + 4096);
 

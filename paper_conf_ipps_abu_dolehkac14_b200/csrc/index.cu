@@ -210,10 +210,13 @@ __global__ void __launch_bounds__(kFillThreads) k_ptrs_fill(const uint32_t *__re
 // Seed records (lookup acceleration, not part of the paper's index): for each slot k
 // of locs, {p, bases R[p-16, p) with base p-1 in the low bits (00 before position 0),
 // bases R[p+ls, p+ls+32) first base highest (00 past the end)} -- 16 bytes, one
-// sector, so the find kernel decides a random seed hit without gathering R.
+// sector, so the find kernel decides a random seed hit without gathering R. With
+// step <= 8 the left extension never passes 8 bases, and 8-byte records {p, R[p-8, p)
+// | R[p+ls, p+ls+8) << 16} halve the record traffic of the (then numerous) hits.
+template <bool kRec8>
 __global__ void __launch_bounds__(kCodeThreads) k_seed_recs(const uint64_t *__restrict__ R, uint32_t ls,
                                                             const uint32_t *__restrict__ locs, uint64_t n_locs,
-                                                            uint4 *__restrict__ recs) {
+                                                            void *__restrict__ recs) {
     const uint64_t k = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
     if (k >= n_locs) return;
     const uint32_t p = locs[k];
@@ -232,16 +235,18 @@ __global__ void __launch_bounds__(kCodeThreads) k_seed_recs(const uint64_t *__re
         left = uint32_t(win_back(R, p));
         right = win_fwd(R, uint64_t(p) + ls);
     }
-    recs[k] = make_uint4(p, left, uint32_t(right), uint32_t(right >> 32));
+    if (kRec8) static_cast<uint2 *>(recs)[k] = make_uint2(p, (left & 0xffffu) | uint32_t(right >> 48) << 16);
+    else static_cast<uint4 *>(recs)[k] = make_uint4(p, left, uint32_t(right), uint32_t(right >> 32));
 }
 
 }  // namespace
 
-cudaError_t launch_seed_recs(const uint64_t *R, uint32_t ls, const uint32_t *locs, uint64_t n_locs, uint4 *recs,
-                             cudaStream_t s) {
+cudaError_t launch_seed_recs(const uint64_t *R, uint32_t ls, const uint32_t *locs, uint64_t n_locs, void *recs,
+                             int rec8, cudaStream_t s) {
     if (n_locs == 0) return cudaSuccess;
     const uint64_t blocks = (n_locs + kCodeThreads - 1) / kCodeThreads;
-    k_seed_recs<<<unsigned(blocks), kCodeThreads, 0, s>>>(R, ls, locs, n_locs, recs);
+    if (rec8) k_seed_recs<true><<<unsigned(blocks), kCodeThreads, 0, s>>>(R, ls, locs, n_locs, recs);
+    else k_seed_recs<false><<<unsigned(blocks), kCodeThreads, 0, s>>>(R, ls, locs, n_locs, recs);
     note_launch();
     return cudaGetLastError();
 }

@@ -20,6 +20,7 @@ struct Options {
     int64_t small_sort = 0;      // 1: single-launch cooperative sorts when the input fits (small_sort.cu;
                                  // measured slower at C4: its scattered global writes are not coalesced)
     int64_t index_msd = 0;
+    int64_t rec8 = -1;           // seed records: -1 auto (8-byte when step <= 8), 0 16-byte, 1 8-byte
     int64_t rank_sectors = -1;   // lookup directory: -1 auto (sectors when the compact table exceeds L2/4),
                                  // 0 rank words, 1 rank sectors       // index sort: 1 = MSD bucket sort of (code << 32 | p), 0 = stable LSD radix
     int64_t radix_bits = 0;      // LSD digit width: 0 = 9 bits if that saves a pass else 8; or pinned 8, 9, 10
@@ -86,9 +87,10 @@ size_t ptrs_fill_scratch_bytes(uint32_t ls);
 cudaError_t launch_ptrs_fill(const uint32_t *sorted_codes, uint64_t n_locs, uint32_t ls, uint32_t *ptrs,
                              unsigned long long *rankw, uint4 *rsect, uint2 *buckets, void *scratch,
                              cudaStream_t s);
-// Seed records for the lookup: rec[k] = {locs[k], 16 bases left of it, 32 bases right of its seed}.
-cudaError_t launch_seed_recs(const uint64_t *R, uint32_t ls, const uint32_t *locs, uint64_t n_locs, uint4 *recs,
-                             cudaStream_t s);
+// Seed records for the lookup: rec[k] = {locs[k], 16 bases left of it, 32 bases right of its seed}
+// (uint4), or with rec8 {locs[k], 8 bases left | 8 bases right << 16} (uint2).
+cudaError_t launch_seed_recs(const uint64_t *R, uint32_t ls, const uint32_t *locs, uint64_t n_locs, void *recs,
+                             int rec8, cudaStream_t s);
 
 // Find (find.cu)
 struct FindParams {
@@ -98,7 +100,8 @@ struct FindParams {
     uint64_t nQ;
     uint64_t nQw;                // allocated words of Q (incl. padding)
     const uint32_t *ptrs;
-    const uint4 *recs;           // seed records, parallel to locs: {p, R[p-16,p), R[p+ls,p+ls+32)}
+    const void *recs;            // seed records, parallel to locs: uint4 {p, R[p-16,p), R[p+ls,p+ls+32)}, or
+    int rec8;                    // (rec8) uint2 {p, R[p-8,p) | R[p+ls,p+ls+8) << 16}
     const unsigned long long *rankw;  // per 32 seeds: {occupancy bits (low 32), occupied seeds before (high 32)}
     const uint4 *rsect;          // or (large indexes) per 32 seeds: {records before, occupied seeds before,
                                  // 2-bit saturating counts lo, hi}; exactly one of rankw / rsect is set

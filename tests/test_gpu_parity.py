@@ -24,7 +24,7 @@ def _default_options():
     yield
     for k, v in (("find_grid", 0), ("find_spill", 64), ("out_capacity", 0), ("use_bitmap", 1), ("static_lb", 0),
                  ("sort_impl", 0), ("index_msd", 0), ("small_sort", 0), ("radix_bits", 0),
-                 ("rank_sectors", -1)):
+                 ("rank_sectors", -1), ("rec8", -1)):
         gpumem.set_option(k, v)
 
 
@@ -203,10 +203,13 @@ def test_adversarial_repeats(L, ls):
     got = gpu_mems(R, Q, L, ls)
     assert np.array_equal(got, want)
     invariants.check(R, Q, L, got)
-    for mode in (0, 1):  # both lookup directories (rank sectors: saturated repeat counts)
-        gpumem.set_option("rank_sectors", mode)
-        assert np.array_equal(gpu_mems(R, Q, L, ls), want), mode
+    for sect in (0, 1):  # both lookup directories (rank sectors: saturated repeat counts)
+        for rec8 in (0, 1):  # both record widths
+            gpumem.set_option("rank_sectors", sect)
+            gpumem.set_option("rec8", rec8)
+            assert np.array_equal(gpu_mems(R, Q, L, ls), want), (sect, rec8)
     gpumem.set_option("rank_sectors", -1)
+    gpumem.set_option("rec8", -1)
     if len(want):
         assert np.array_equal(gpu_mems(R, Q, L, ls, device_input=True), want)
 
@@ -230,13 +233,13 @@ def test_overflow_retry_grid_spill_and_bitmap_invariance():
     assert np.array_equal(base, want)
     for opt, vals in (("out_capacity", [1, 100]), ("find_grid", [1, 3, 148]), ("find_spill", [1, 2, 10**9]),
                       ("use_bitmap", [0]), ("static_lb", [1]), ("sort_impl", [1, 2]), ("index_msd", [1]), ("small_sort", [1]),
-                      ("rank_sectors", [0, 1]),
+                      ("rank_sectors", [0, 1]), ("rec8", [0, 1]),
                       ("radix_bits", [8, 9, 10])):
         for v in vals:
             gpumem.set_option(opt, v)
             assert np.array_equal(gpu_mems(P.R, P.Q, P.L, P.ls), want), (opt, v)
         gpumem.set_option(opt, {"out_capacity": 0, "find_grid": 0, "find_spill": 64, "use_bitmap": 1,
-                                "static_lb": 0, "sort_impl": 0, "index_msd": 0, "small_sort": 0, "rank_sectors": -1,
+                                "static_lb": 0, "sort_impl": 0, "index_msd": 0, "small_sort": 0, "rank_sectors": -1, "rec8": -1,
                                 "radix_bits": 0}[opt])
 
 
