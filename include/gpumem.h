@@ -197,6 +197,8 @@ gpumem_status gpumem_set_allocator(void *(*alloc_fn)(size_t bytes, void *cuda_st
  *  "sort_impl"        output sort: 0 (default) auto by size, 1 stable LSD radix sort,
  *                     2 MSD bucket sort
  *  "index_msd"        index sort: 0 (default) stable LSD radix, 1 MSD bucket sort
+ *  "index_fused"      1 (ls >= 9): group radix passes + one fused counting/placement
+ *                     kernel; 0 (default): full radix sort, ptrs fill and record gather
  *  "rec8"             seed records: -1 (default) auto (8-byte when step <= 8), 0 16-byte, 1 8-byte
  *  "rank_sectors"     lookup directory: -1 (default) auto, 0 rank words, 1 rank sectors
  *  "small_sort"       1: single-launch cooperative radix sorts (index and output) when

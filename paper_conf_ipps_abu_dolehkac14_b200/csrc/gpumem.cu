@@ -236,7 +236,7 @@ gpumem_status check_device(int *dev) {
 // loop does no allocation at all once warm. gpumem_trim() releases everything.
 enum WsSlot {
     kWsCtr, kWsSpill, kWsKeys, kWsLens, kWsSortK, kWsSortL, kWsSortScratch, kWsCodes0, kWsCodes1,
-    kWsRadix, kWsFill, kWsMergeK, kWsMergeL, kWsPackTmp, kWsCoop, kWsMums, kWsSmall, kWsCount
+    kWsRadix, kWsFill, kWsMergeK, kWsMergeL, kWsPackTmp, kWsCoop, kWsMums, kWsSmall, kWsLocsTmp, kWsSlot, kWsCount
 };
 struct Workspace {
     void *p[kWsCount] = {};
@@ -325,6 +325,7 @@ gpumem_status gpumem_set_option(const char *name, int64_t value) {
         g_opt.sort_impl = value;
     }
     else if (!strcmp(name, "index_msd")) g_opt.index_msd = value ? 1 : 0;
+    else if (!strcmp(name, "index_fused")) g_opt.index_fused = value ? 1 : 0;
     else if (!strcmp(name, "small_sort")) g_opt.small_sort = value ? 1 : 0;
     else if (!strcmp(name, "rec8")) g_opt.rec8 = value < 0 ? -1 : (value ? 1 : 0);
     else if (!strcmp(name, "rank_sectors")) g_opt.rank_sectors = value < 0 ? -1 : (value ? 1 : 0);
@@ -539,8 +540,46 @@ static gpumem_status index_build_impl(const gpumem_seq *R, uint32_t ls, uint32_t
     const int rec8 = g_opt.rec8 < 0 ? (step <= 8 ? 1 : 0) : int(g_opt.rec8 != 0);
     void *recs = sc.get((n_locs ? n_locs : 1) * (rec8 ? sizeof(uint2) : sizeof(uint4)));
     if (!recs) return GPUMEM_ERR_NOMEM;
-    bool recs_done = false;
-    if (n_locs && !rec8 && !g_opt.index_msd && g_opt.small_sort && n_locs <= small_sort_max_n(4)) {
+    bool recs_done = false, fill_done = false;
+    if (n_locs && ls >= 9 && g_opt.index_fused && !g_opt.index_msd && !g_opt.small_sort) {
+        // radix passes over the code bits above the 1024-seed groups, then one fused
+        // kernel: counts, ptrs, stable placement of locs + records, rank directory
+        auto *codes0 = static_cast<uint32_t *>(ws_get(kWsCodes0, n_locs * 4, s));
+        auto *codes1 = static_cast<uint32_t *>(ws_get(kWsCodes1, n_locs * 4, s));
+        auto *locs1 = static_cast<uint32_t *>(ws_get(kWsLocsTmp, n_locs * 4, s));
+        void *scratch = ws_get(kWsRadix, radix_scratch_bytes(n_locs), s);
+        void *lscratch = ws_get(kWsFill, index_local_scratch_bytes(ls), s);
+        if (!codes0 || !codes1 || !locs1 || !scratch || !lscratch) return GPUMEM_ERR_NOMEM;
+        {
+            Stage g("index.codes", s);
+            CK(launch_seed_codes(R->words, ls, step, k0, n_locs, codes0, locs1, s), "seed codes");
+        }
+        bool alt = false;
+        {
+            Stage g("index.sort", s);
+            CK(radix_sort_u32(codes0, locs1, codes1, locs0, n_locs, int(2 * ls), scratch, s, &alt, 10),
+               "seed group sort");
+        }
+        // the pairs are in (codes0, locs1) or, after an odd number of passes, (codes1, locs0);
+        // the final locs go to whichever of locs0 / locs1 is free, and that one is kept
+        const uint32_t *gc = alt ? codes1 : codes0;
+        const uint32_t *gp = alt ? locs0 : locs1;
+        uint32_t *out_locs = locs0;
+        if (alt) {  // locs0 holds the input: write into a fresh kept buffer
+            out_locs = static_cast<uint32_t *>(sc.get(n_locs * 4));
+            if (!out_locs) return GPUMEM_ERR_NOMEM;
+        }
+        {
+            Stage g("index.ptrs", s);
+            auto *slot = static_cast<uint32_t *>(ws_get(kWsSlot, index_local_slot_bytes(n_locs), s));
+            if (!slot) return GPUMEM_ERR_NOMEM;
+            CK(launch_index_local(gc, gp, n_locs, ls, R->words, ptrs, rankw, rsect, buckets, out_locs, recs, rec8,
+                                  slot, lscratch, s),
+               "index local");
+        }
+        locs = out_locs;
+        recs_done = fill_done = true;
+    } else if (n_locs && !rec8 && !g_opt.index_msd && g_opt.small_sort && n_locs <= small_sort_max_n(4)) {
         // one cooperative launch: seed codes from R, stable sort, codes + locs + records
         auto *codes1 = static_cast<uint32_t *>(ws_get(kWsCodes1, n_locs * 4, s));
         void *scratch = ws_get(kWsSmall, small_sort_scratch_bytes(n_locs, 4), s);
@@ -580,7 +619,7 @@ static gpumem_status index_build_impl(const gpumem_seq *R, uint32_t ls, uint32_t
         codes_sorted = alt ? codes1 : codes0;
         locs = alt ? locs1 : locs0;
     }
-    {
+    if (!fill_done) {
         Stage g("index.ptrs", s);
         CK(launch_ptrs_fill(codes_sorted, n_locs, ls, ptrs, rankw, rsect, buckets, fill_scratch, s), "ptrs fill");
     }

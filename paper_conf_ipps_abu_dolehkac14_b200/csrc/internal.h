@@ -20,6 +20,9 @@ struct Options {
     int64_t small_sort = 0;      // 1: single-launch cooperative sorts when the input fits (small_sort.cu;
                                  // measured slower at C4: its scattered global writes are not coalesced)
     int64_t index_msd = 0;
+    int64_t index_fused = 0;     // 1: radix passes over the code bits above 1024-seed groups + the fused
+                                 // local kernel (ls >= 9; measured slower: 0.25 vs 0.20 ms at C4);
+                                 // 0: full radix sort + ptrs fill + record gather
     int64_t rec8 = -1;           // seed records: -1 auto (8-byte when step <= 8), 0 16-byte, 1 8-byte
     int64_t rank_sectors = -1;   // lookup directory: -1 auto (sectors when the compact table exceeds L2/4),
                                  // 0 rank words, 1 rank sectors       // index sort: 1 = MSD bucket sort of (code << 32 | p), 0 = stable LSD radix
@@ -51,11 +54,11 @@ cudaError_t launch_pack(const uint8_t *in, uint64_t n, uint64_t *words, uint64_t
 // Reverse complement of packed words (pack.cu).
 cudaError_t launch_revcomp(const uint64_t *in, uint64_t n, uint64_t *out, uint64_t n_words_alloc, cudaStream_t s);
 
-// Radix sort (radix.cu): stable LSD on the low `bits` bits of the keys, values ride along.
+// Radix sort (radix.cu): stable LSD on bits [lo, bits) of the keys, values ride along.
 // Ping-pongs between (k0,v0) and (k1,v1); returns true when the result is in (k1,v1).
 // `scratch` must hold radix_scratch_bytes(n) bytes (digit counts + scan partials).
 cudaError_t radix_sort_u32(uint32_t *k0, uint32_t *v0, uint32_t *k1, uint32_t *v1, uint64_t n, int bits,
-                           void *scratch, cudaStream_t s, bool *in_alt);
+                           void *scratch, cudaStream_t s, bool *in_alt, int lo = 0);
 cudaError_t radix_sort_u64(uint64_t *k0, uint32_t *v0, uint64_t *k1, uint32_t *v1, uint64_t n, int bits,
                            void *scratch, cudaStream_t s, bool *in_alt);
 size_t radix_scratch_bytes(uint64_t n);
@@ -87,6 +90,14 @@ size_t ptrs_fill_scratch_bytes(uint32_t ls);
 cudaError_t launch_ptrs_fill(const uint32_t *sorted_codes, uint64_t n_locs, uint32_t ls, uint32_t *ptrs,
                              unsigned long long *rankw, uint4 *rsect, uint2 *buckets, void *scratch,
                              cudaStream_t s);
+// Fused last step of the index (index.cu): (code, p) pairs sorted stably by code bits
+// [10, 2 ls) -> ptrs, rank directory, compact table, final locs and seed records.
+size_t index_local_scratch_bytes(uint32_t ls);
+size_t index_local_slot_bytes(uint64_t n_locs);
+cudaError_t launch_index_local(const uint32_t *codes, const uint32_t *ps, uint64_t n_locs, uint32_t ls,
+                               const uint64_t *R, uint32_t *ptrs, unsigned long long *rankw, uint4 *rsect,
+                               uint2 *buckets, uint32_t *locs, void *recs, int rec8, uint32_t *slot, void *scratch,
+                               cudaStream_t s);
 // Seed records for the lookup: rec[k] = {locs[k], 16 bases left of it, 32 bases right of its seed}
 // (uint4), or with rec8 {locs[k], 8 bases left | 8 bases right << 16} (uint2).
 cudaError_t launch_seed_recs(const uint64_t *R, uint32_t ls, const uint32_t *locs, uint64_t n_locs, void *recs,

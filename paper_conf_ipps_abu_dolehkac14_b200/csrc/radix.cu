@@ -380,10 +380,10 @@ int pick_digit_bits(int bits) {
 constexpr int kMaxChunks = 148 * 8;  // >= SMs x resident scatter CTAs
 
 template <class K, int RB>
-cudaError_t radix_sort_rb(K *k0, uint32_t *v0, K *k1, uint32_t *v1, uint64_t n, int bits, void *scratch,
+cudaError_t radix_sort_rb(K *k0, uint32_t *v0, K *k1, uint32_t *v1, uint64_t n, int lo, int bits, void *scratch,
                           cudaStream_t s, bool *in_alt) {
     constexpr int kBins = 1 << RB;
-    const int passes = (bits + RB - 1) / RB;
+    const int passes = (bits - lo + RB - 1) / RB;
     const size_t smem = sizeof(ScatterSmem<K, uint32_t, RB>);
     static int grid_cap = 0;  // per instantiation: resident scatter CTAs on the whole GPU
     cudaError_t e;
@@ -412,11 +412,12 @@ cudaError_t radix_sort_rb(K *k0, uint32_t *v0, K *k1, uint32_t *v1, uint64_t n, 
     K *ka = k0, *kb = k1;
     uint32_t *va = v0, *vb = v1;
     for (int p = 0; p < passes; ++p) {
-        const int dbits = (p == passes - 1) ? bits - RB * p : RB;
+        const int sh = lo + RB * p;
+        const int dbits = (p == passes - 1) ? bits - sh : RB;
         uint32_t *tot = totals + size_t(p) * kBins;
-        k_chunk_hist<K, RB><<<ch.chunks, kT, 0, s>>>(ka, ch, RB * p, dbits, counts, tot);
+        k_chunk_hist<K, RB><<<ch.chunks, kT, 0, s>>>(ka, ch, sh, dbits, counts, tot);
         k_chunk_scan<RB><<<kBins / kWarps, kT, 0, s>>>(counts, tot, ch.chunks, offs);
-        k_scatter<K, uint32_t, RB><<<ch.chunks, kST, smem, s>>>(ka, va, kb, vb, ch, RB * p, dbits, offs);
+        k_scatter<K, uint32_t, RB><<<ch.chunks, kST, smem, s>>>(ka, va, kb, vb, ch, sh, dbits, offs);
         note_launch(3);
         std::swap(ka, kb);
         std::swap(va, vb);
@@ -426,17 +427,17 @@ cudaError_t radix_sort_rb(K *k0, uint32_t *v0, K *k1, uint32_t *v1, uint64_t n, 
 }
 
 template <class K>
-cudaError_t radix_sort(K *k0, uint32_t *v0, K *k1, uint32_t *v1, uint64_t n, int bits, void *scratch,
+cudaError_t radix_sort(K *k0, uint32_t *v0, K *k1, uint32_t *v1, uint64_t n, int lo, int bits, void *scratch,
                        cudaStream_t s, bool *in_alt) {
     *in_alt = false;
-    if (n <= 1 || bits <= 0) return cudaSuccess;
-    if (!scratch) return cudaErrorInvalidValue;
     if (bits > int(8 * sizeof(K))) bits = int(8 * sizeof(K));
+    if (n <= 1 || bits <= lo) return cudaSuccess;
+    if (!scratch) return cudaErrorInvalidValue;
     if (uint64_t(n) >= (uint64_t(1) << 32)) return cudaErrorInvalidValue;  // 32-bit offsets
-    switch (pick_digit_bits(bits)) {
-        case 9: return radix_sort_rb<K, 9>(k0, v0, k1, v1, n, bits, scratch, s, in_alt);
-        case 10: return radix_sort_rb<K, 10>(k0, v0, k1, v1, n, bits, scratch, s, in_alt);
-        default: return radix_sort_rb<K, 8>(k0, v0, k1, v1, n, bits, scratch, s, in_alt);
+    switch (pick_digit_bits(bits - lo)) {
+        case 9: return radix_sort_rb<K, 9>(k0, v0, k1, v1, n, lo, bits, scratch, s, in_alt);
+        case 10: return radix_sort_rb<K, 10>(k0, v0, k1, v1, n, lo, bits, scratch, s, in_alt);
+        default: return radix_sort_rb<K, 8>(k0, v0, k1, v1, n, lo, bits, scratch, s, in_alt);
     }
 }
 
@@ -448,13 +449,13 @@ size_t radix_scratch_bytes(uint64_t n) {  // totals of every pass + counts + off
 }
 
 cudaError_t radix_sort_u32(uint32_t *k0, uint32_t *v0, uint32_t *k1, uint32_t *v1, uint64_t n, int bits,
-                           void *scratch, cudaStream_t s, bool *in_alt) {
-    return radix_sort<uint32_t>(k0, v0, k1, v1, n, bits, scratch, s, in_alt);
+                           void *scratch, cudaStream_t s, bool *in_alt, int lo) {
+    return radix_sort<uint32_t>(k0, v0, k1, v1, n, lo, bits, scratch, s, in_alt);
 }
 
 cudaError_t radix_sort_u64(uint64_t *k0, uint32_t *v0, uint64_t *k1, uint32_t *v1, uint64_t n, int bits,
                            void *scratch, cudaStream_t s, bool *in_alt) {
-    return radix_sort<uint64_t>(k0, v0, k1, v1, n, bits, scratch, s, in_alt);
+    return radix_sort<uint64_t>(k0, v0, k1, v1, n, 0, bits, scratch, s, in_alt);
 }
 
 }  // namespace gm

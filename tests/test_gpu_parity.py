@@ -24,7 +24,7 @@ def _default_options():
     yield
     for k, v in (("find_grid", 0), ("find_spill", 64), ("out_capacity", 0), ("use_bitmap", 1), ("static_lb", 0),
                  ("sort_impl", 0), ("index_msd", 0), ("small_sort", 0), ("radix_bits", 0),
-                 ("rank_sectors", -1), ("rec8", -1)):
+                 ("rank_sectors", -1), ("rec8", -1), ("index_fused", 0)):
         gpumem.set_option(k, v)
 
 
@@ -125,7 +125,8 @@ def test_index_parity_word_for_word(cfg, ls, step, scale):
     assert np.array_equal(l, ol)
 
 
-@pytest.mark.parametrize("opts", [{"small_sort": 1}, {"radix_bits": 8}, {"index_msd": 1}])
+@pytest.mark.parametrize("opts", [{"small_sort": 1}, {"radix_bits": 8}, {"index_msd": 1}, {"index_fused": 1},
+                                  {"index_fused": 1, "rank_sectors": 1, "rec8": 1}])
 def test_index_sort_paths(opts):
     """Every index sort path (single-launch cooperative, multi-launch LSD, MSD) gives
     Alg. 1's ptrs/locs word for word."""
@@ -233,13 +234,14 @@ def test_overflow_retry_grid_spill_and_bitmap_invariance():
     assert np.array_equal(base, want)
     for opt, vals in (("out_capacity", [1, 100]), ("find_grid", [1, 3, 148]), ("find_spill", [1, 2, 10**9]),
                       ("use_bitmap", [0]), ("static_lb", [1]), ("sort_impl", [1, 2]), ("index_msd", [1]), ("small_sort", [1]),
-                      ("rank_sectors", [0, 1]), ("rec8", [0, 1]),
+                      ("rank_sectors", [0, 1]), ("rec8", [0, 1]), ("index_fused", [1]),
                       ("radix_bits", [8, 9, 10])):
         for v in vals:
             gpumem.set_option(opt, v)
             assert np.array_equal(gpu_mems(P.R, P.Q, P.L, P.ls), want), (opt, v)
         gpumem.set_option(opt, {"out_capacity": 0, "find_grid": 0, "find_spill": 64, "use_bitmap": 1,
-                                "static_lb": 0, "sort_impl": 0, "index_msd": 0, "small_sort": 0, "rank_sectors": -1, "rec8": -1,
+                                "static_lb": 0, "sort_impl": 0, "index_msd": 0, "small_sort": 0, "rank_sectors": -1,
+                                "rec8": -1, "index_fused": 0,
                                 "radix_bits": 0}[opt])
 
 
