@@ -89,6 +89,8 @@ class ClockSampler:
             time.sleep(self.period)
 
     def __enter__(self):
+        if os.environ.get("GM_BENCH_NOCLK"):  # diagnostics: no sampler thread
+            self.nv = None
         if self.nv:
             self.t = threading.Thread(target=self._run, daemon=True)
             self.t.start()
@@ -143,31 +145,34 @@ def run_reference(args, P):
 
 # ------------------------------------------------------------------ roofline bookkeeping
 def algorithmic_bytes(nR, nQ, ls, L, stats, world):
-    """Algorithmic (useful) HBM bytes per step of each stage on one rank (DESIGN.md
-    "Roofline"): what the method must move, not sector over-fetch."""
+    """Algorithmic (useful) HBM bytes per step of each stage on one rank:
+    what the method must move, not sector over-fetch."""
     step = L - ls + 1
     n_locs = (nR - ls) // step + 1 if nR >= ls else 0
     nb = 1 << (2 * ls)
-    passes = (2 * ls + 7) // 8
+    passes = (2 * ls + 8) // 9                # LSD passes of 9-bit digits over the 2*ls-bit codes
+    rec = 8 if step <= 8 else 16              # seed record bytes (index.cu)
     pos, occ, hits, mems = stats["positions"], stats["occupied"], stats["hits"], stats["mems"]
     return {
         # 1 B ASCII read + 0.25 B packed write per base, R and Q
         "pack": 1.25 * (nR + nQ),
         # per sampled seed: one 8-byte R window read, code + location written
         "index.codes": n_locs * (8 + 8),
-        # counting sort by seed, per 8-bit digit pass: code + location read and written once
-        # (the all-digit histogram adds one read of the codes)
-        "index.sort": passes * n_locs * 16 + n_locs * 4,
-        # sorted codes read once; ptrs (4^ls + 1 words) and the 4^ls-bit bitmap written
-        "index.ptrs": n_locs * 4 + 4 * (nb + 1) + nb / 8,
-        # per slot: location read, R windows read (2 x 8 B), 16-byte seed record written
-        "index.recs": n_locs * (4 + 16 + 16),
-        # per query position: packed Q (0.25 B) + its bitmap bit; per occupied seed the
-        # ptrs pair (8 B); per hit one location (4 B) + one 32-base R word each side
-        # (16 B); per MEM the 12-byte record written
-        "find": 0.25 * pos + pos / 8 + 8 * occ + 20 * hits + 12 * mems,
-        # output sort: 7 passes of (12 B read twice + 12 B written) over 56-bit keys
-        "sort": mems * 36 * ((30 + 30 + 7) // 8),
+        # stable counting sort by seed code: per digit pass the (code, location) pair is
+        # read and written once, plus one code read for the chunk histogram
+        "index.sort": passes * n_locs * (16 + 4),
+        # sorted codes read once; ptrs (4^ls + 1 words), the rank directory (8 B per 32
+        # seeds) and the compact {first, count} table (8 B per occupied seed) written
+        "index.ptrs": n_locs * 4 + 4 * (nb + 1) + nb / 4 + 8 * min(n_locs, nb),
+        # per slot: location read, 3 words of R read, the seed record written
+        "index.recs": n_locs * (4 + 24 + rec),
+        # per query position: packed Q (0.25 B) + its occupancy bit (1/8 B); per occupied
+        # position the {first, count} entry (8 B); per hit one seed record; per MEM the
+        # 12-byte (key, len) record written
+        "find": 0.25 * pos + pos / 8 + 8 * occ + rec * hits + 12 * mems,
+        # output MSD sort: key read (histogram), key + len read and written (scatter),
+        # read again and written as a triple (local sort): 8 + 24 + 24 B per MEM
+        "sort": mems * 56,
     }
 
 
@@ -176,7 +181,7 @@ def run_ours(args, P):
     import torch
     import torch.distributed as dist
     from paper_conf_ipps_abu_dolehkac14_b200 import gpumem as gm
-    from paper_conf_ipps_abu_dolehkac14_b200.dist import find_mems_sharded
+    from paper_conf_ipps_abu_dolehkac14_b200.dist import ShardedPipeline
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -193,44 +198,49 @@ def run_ours(args, P):
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
     torch.cuda.synchronize()
 
-    def step():
-        merged, local_m = find_mems_sharded(R_dev, Q_dev, P.L, P.ls)
-        return merged, local_m
-
+    # the step: one CUDA-graph launch of the whole path per rank (pack R, pack Q, index,
+    # find over the rank's shard, output sort); for N > 1 also the gather + rank-0 merge
+    sp = ShardedPipeline(len(P.R), len(P.Q), P.L, P.ls)
     n_mems, stats = 0, None
     for _ in range(args.warmup):
         flush.zero_()
-        merged, lm = step()
-        torch.cuda.synchronize()
-        n_mems = len(merged) if merged is not None else 0
-        stats = lm.stats()
-        for h in (merged, lm):
-            if h is not None:
-                h.free()
-    del merged, lm
+        sp.run(R_dev, Q_dev)
+        n_mems = sp.finish() or 0
+        stats = sp.pl.stats()
+    torch.cuda.synchronize()
 
-    gm.profile_enable(True)
-    gm.profile_read()  # drop warm-up records
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    prof = {}
+    fallbacks = 0
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
     l0 = gm.launch_count()
+    host_ms = []
     with ClockSampler(local) as clk:
         for i in range(args.steps):
             flush.zero_()
             ev[i][0].record(stream)
-            merged, lm = step()
-            ev[i][1].record(stream)
-            for h in (merged, lm):  # release this step's handles (async frees, stream-ordered)
-                if h is not None:
-                    h.free()
+            th = time.perf_counter()
+            sp.run(R_dev, Q_dev)
+            if world > 1:  # the exchange needs the counts: result, gather, merge inside the step
+                sp.finish()
+                ev[i][1].record(stream)
+            else:
+                ev[i][1].record(stream)
+                sp.finish()  # sync + capacity check outside the step's events
+                if sp.pl.stats()["attempts"] > 1:  # overflow rerun ran after ev[i][1]: time it too
+                    fallbacks += 1
+                    ev[i] = (ev[i][0], torch.cuda.Event(enable_timing=True))
+                    ev[i][1].record(stream)
+            host_ms.append(1e3 * (time.perf_counter() - th))
+            for k, (t, nl) in sp.pl.profile().items():  # stage events inside this launch
+                a0 = prof.get(k, (0.0, 0))
+                prof[k] = (a0[0] + t, a0[1] + nl)
         torch.cuda.synchronize()
     launches = gm.launch_count() - l0
     if world > 1:
         dist.barrier()
-    prof = gm.profile_read()
-    gm.profile_enable(False)
     step_ms = [a.elapsed_time(b) for a, b in ev]
     tot = torch.tensor([sum(step_ms)], dtype=torch.float64, device=dev)
     if world > 1:
@@ -278,7 +288,10 @@ def run_ours(args, P):
             "mems_per_s": round(n_mems / (ms / 1e3), 1),
             "stage_ms": {k: round(v, 4) for k, v in sorted(kernel_ms.items())},
             "stage_hbm_frac": stage_frac, "find_stats": stats, "gpu_launches": int(launches),
-            "clocks": clk.summary(), "roofline": roof}
+            "clocks": clk.summary(), "roofline": roof,
+            "host_ms_per_step": round(statistics.mean(host_ms), 4), "capacity_fallbacks": fallbacks,
+            "launch_mode": "one CUDA graph per step (gpumem_pipeline_run)",
+            "step_ms_minmax": [round(min(step_ms), 4), round(max(step_ms), 4)]}
 
     # ---- end-to-end through the public API with HOST buffers (pinned), H2D + D2H inside
     if not args.no_e2e and world == 1:

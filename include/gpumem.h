@@ -54,6 +54,7 @@ typedef enum {
 typedef struct gpumem_seq gpumem_seq;     /* 2-bit packed sequence resident on one device        */
 typedef struct gpumem_index gpumem_index; /* ptrs[4^ls+1], locs[n_locs], occupancy bitmap; refs R  */
 typedef struct gpumem_mems gpumem_mems;   /* MEM set sorted by (r, q), device-resident            */
+typedef struct gpumem_pipeline gpumem_pipeline; /* the whole path captured as one CUDA graph        */
 
 /* One MEM (Table I :34-35): R[r .. r+len) == Q[q .. q+len). 12 bytes, AoS. */
 typedef struct {
@@ -170,7 +171,48 @@ gpumem_status gpumem_mems_to_host(const gpumem_mems *m, gpumem_triple *host_buf,
 gpumem_status gpumem_merge_sorted(const gpumem_triple *const *dev_runs, const uint64_t *counts,
                                   int n_runs, void *cuda_stream, gpumem_mems **out);
 
-/* Release any handle above (seq, index, mems). NULL is a no-op. */
+/*
+ * Pipeline: the whole path (pack R, pack Q, index R, find, sort -- the same kernels
+ * and the same result as gpumem_pack + gpumem_index_build + gpumem_find_mems) for
+ * fixed sizes, captured once as a CUDA graph and replayed with one launch and no host
+ * round trip in between (find's output count stays on the device; the output sort is
+ * sized by it there). Intended for repeated work of one shape (benchmarks, batches of
+ * equally long queries) where host launch latency would otherwise show between stages.
+ *
+ * gpumem_pipeline_create -- sizes |R| = r_len, |Q| = q_len, seed_len (ls), min_len (L)
+ *  and the MEM start range [q_begin, q_end) as in gpumem_find_mems (0, UINT64_MAX = all).
+ *  Argument rules as gpumem_index_build / gpumem_find_mems. Stream: every run is
+ *  enqueued on `cuda_stream` (the pipeline's workspaces belong to it). Allocates only a
+ *  pinned 128-byte counter buffer; device memory (one arena holding the packed
+ *  sequences, the index and the result) is allocated at the first run.
+ *
+ * gpumem_pipeline_run -- async. r_bases_dev / q_bases_dev: device pointers to r_len and
+ *  q_len ASCII bases (read, not modified; must stay valid until the run completes).
+ *  The first call, and any call with different input pointers, measures and captures
+ *  the graph (one ordinary synchronous pass + capture); later calls are one
+ *  cudaGraphLaunch. The previous run's result is invalidated.
+ *
+ * gpumem_pipeline_result -- synchronises the stream, then checks the alphabet flags
+ *  (GPUMEM_ERR_ALPHABET as gpumem_find_mems) and the output capacity: on overflow the
+ *  MEMs are recomputed with gpumem_find_mems on the pipeline's packed sequences and
+ *  index (stats.attempts > 1). *dev_ptr / *count: the sorted triples, borrowed, valid
+ *  until the next run or gpumem_free(pl).
+ *
+ * gpumem_pipeline_stats -- find statistics of the last result.
+ * gpumem_pipeline_profile -- per-stage device time of the last completed run (the
+ *  stage events are part of the graph), aggregated by name as gpumem_profile_read;
+ *  synchronises those events. Returns the number of entries written.
+ * gpumem_free(pl) synchronises the stream and releases everything.
+ */
+gpumem_status gpumem_pipeline_create(uint64_t r_len, uint64_t q_len, uint32_t seed_len, uint32_t min_len,
+                                     uint64_t q_begin, uint64_t q_end, void *cuda_stream, gpumem_pipeline **out);
+gpumem_status gpumem_pipeline_run(gpumem_pipeline *pl, const char *r_bases_dev, const char *q_bases_dev);
+gpumem_status gpumem_pipeline_result(gpumem_pipeline *pl, const gpumem_triple **dev_ptr, uint64_t *count);
+gpumem_status gpumem_pipeline_stats(const gpumem_pipeline *pl, gpumem_find_stats *out);
+int gpumem_pipeline_profile(const gpumem_pipeline *pl, const char **names, double *ms, uint64_t *launches,
+                            int max_stages);
+
+/* Release any handle above (seq, index, mems, pipeline). NULL is a no-op. */
 void gpumem_free(void *handle);
 
 /* Temporaries (find buffers, sort and index scratch) live in a grow-only workspace per
@@ -195,7 +237,9 @@ gpumem_status gpumem_set_allocator(void *(*alloc_fn)(size_t bytes, void *cuda_st
  *  "use_bitmap"       1 (default) probe the rank words + bucket table, 0 probe ptrs only
  *  "static_lb"        1: no hit redistribution across lanes (load-balancing ablation)
  *  "sort_impl"        output sort: 0 (default) auto by size, 1 stable LSD radix sort,
- *                     2 MSD bucket sort
+ *                     2 MSD bucket sort, 3 hybrid (LSD passes over the top 16 key bits,
+ *                     then shared-memory sorts of the equal-prefix runs); in a pipeline
+ *                     0 picks MSD or LSD by the MEM count of its measuring run
  *  "index_msd"        index sort: 0 (default) stable LSD radix, 1 MSD bucket sort
  *  "index_fused"      1 (ls >= 9): group radix passes + one fused counting/placement
  *                     kernel; 0 (default): full radix sort, ptrs fill and record gather

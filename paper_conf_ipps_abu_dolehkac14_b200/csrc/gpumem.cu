@@ -14,7 +14,12 @@
 
 #define GPUMEM_VERSION "0.1.0"
 
-enum : uint32_t { kMagicSeq = 0x47534551u, kMagicIdx = 0x47494458u, kMagicMems = 0x474d454du };
+// output sort: the MSD bucket sort up to this many MEMs, the LSD radix sort beyond
+// (measured: MSD faster below a few million keys, its 16K-way scatter slower above)
+constexpr uint64_t kMsdMaxN = 4u << 20;
+
+enum : uint32_t { kMagicSeq = 0x47534551u, kMagicIdx = 0x47494458u, kMagicMems = 0x474d454du,
+                  kMagicPipe = 0x47504950u };
 
 struct gpumem_seq {
     uint32_t magic;
@@ -74,6 +79,36 @@ bool g_prof = false;
 std::vector<StageRec> g_recs;
 std::vector<cudaEvent_t> g_ev_free;
 
+// Pipeline capture context (gpumem_pipeline_*). mode 1 = measuring run: real
+// allocations, their bytes summed; mode 2 = capture: handle/scratch allocations are
+// bump-allocated from the pipeline's arena (frees of arena memory are no-ops), so the
+// captured graph holds no allocation nodes and can be relaunched. `deferred` makes
+// find_mems skip its host synchronisation: the output sort reads the MEM count from
+// device memory and the counters are copied to pinned host memory at the end.
+// One step of a pipeline run: a captured graph segment, or a stage event recorded
+// between segments (so stage times are ordinary stream events on the launching stream).
+struct PipeItem {
+    cudaGraph_t g;
+    cudaGraphExec_t x;
+    cudaEvent_t ev;
+};
+
+struct CapCtx {
+    int mode = 0;
+    std::vector<PipeItem> *items = nullptr;  // capture: segments cut at every stage boundary
+    cudaError_t err = cudaSuccess;
+    char *arena = nullptr;
+    size_t off = 0, cap = 0, need = 0;
+    bool deferred = false;
+    std::vector<StageRec> *recs = nullptr;
+    unsigned long long *host = nullptr;   // pinned: [0, 8) find counters, [8] R flag, [9] Q flag
+    uint64_t out_cap = 0, coop_cap = 0, spill_cap = 0, span = 0;
+    uint64_t expect_n = 0;                // capture: the measuring run's MEM count (sort choice)
+    gpumem_mems *mems = nullptr;
+};
+thread_local CapCtx *t_cap = nullptr;
+thread_local bool t_ws_alloc = false;     // workspace growth: never from the arena
+
 cudaEvent_t take_event() {
     if (!g_ev_free.empty()) {
         cudaEvent_t e = g_ev_free.back();
@@ -127,6 +162,19 @@ int num_sms() {
 void *dalloc(size_t bytes, cudaStream_t s) {
     if (bytes == 0) bytes = 256;
     bytes = (bytes + 255) & ~size_t(255);
+    if (t_cap && !t_ws_alloc) {
+        if (t_cap->mode == 2) {
+            if (t_cap->off + bytes > t_cap->cap) {
+                fail(GPUMEM_ERR_NOMEM, "pipeline arena exhausted (%zu + %zu > %zu bytes)", t_cap->off, bytes,
+                     t_cap->cap);
+                return nullptr;
+            }
+            void *p = t_cap->arena + t_cap->off;
+            t_cap->off += bytes;
+            return p;
+        }
+        t_cap->need += bytes;
+    }
     if (g_alloc_fn) {
         void *p = g_alloc_fn(bytes, s, g_alloc_ctx);
         if (!p) fail(GPUMEM_ERR_NOMEM, "allocator hook returned NULL for %zu bytes", bytes);
@@ -157,6 +205,9 @@ void *dalloc(size_t bytes, cudaStream_t s) {
 
 void dfree(void *p, cudaStream_t s) {
     if (!p) return;
+    if (t_cap && t_cap->mode == 2 && static_cast<char *>(p) >= t_cap->arena &&
+        static_cast<char *>(p) < t_cap->arena + t_cap->cap)
+        return;  // arena memory lives as long as the pipeline
     if (g_free_fn) {
         g_free_fn(p, s, g_alloc_ctx);
         return;
@@ -164,21 +215,48 @@ void dfree(void *p, cudaStream_t s) {
     cudaFreeAsync(p, s);
 }
 
-Stage::Stage(const char *name, cudaStream_t st) : slot(-1), s(st) {
-    if (!g_prof) return;
+// Capture: close the current graph segment, append it and then `ev` (if any) to the
+// pipeline's run list, and open the next segment.
+static void cap_cut(cudaStream_t s, cudaEvent_t ev) {
+    CapCtx &c = *t_cap;
+    cudaGraph_t g = nullptr;
+    cudaError_t e = cudaStreamEndCapture(s, &g);
+    if (e == cudaSuccess && g) {
+        size_t nodes = 0;
+        cudaGraphGetNodes(g, nullptr, &nodes);
+        if (nodes) {
+            cudaGraphExec_t x = nullptr;
+            e = cudaGraphInstantiate(&x, g, 0);
+            if (e == cudaSuccess) c.items->push_back(PipeItem{g, x, nullptr});
+        } else {
+            cudaGraphDestroy(g);
+        }
+    }
+    if (ev) c.items->push_back(PipeItem{nullptr, nullptr, ev});
+    const cudaError_t e2 = cudaStreamBeginCapture(s, cudaStreamCaptureModeRelaxed);
+    if (c.err == cudaSuccess) c.err = e != cudaSuccess ? e : e2;
+}
+
+Stage::Stage(const char *name, cudaStream_t st) : slot(-1), s(st), vec(nullptr) {
+    std::vector<StageRec> *v = (t_cap && t_cap->recs) ? t_cap->recs : (g_prof ? &g_recs : nullptr);
+    if (!v) return;
     std::lock_guard<std::mutex> g(g_prof_mu);
     StageRec r{name, take_event(), take_event(), g_launches.load(), 0};
-    cudaEventRecord(r.a, s);
-    g_recs.push_back(r);
-    slot = int(g_recs.size()) - 1;
+    if (t_cap && t_cap->items) cap_cut(s, r.a);
+    else cudaEventRecord(r.a, s);
+    v->push_back(r);
+    slot = int(v->size()) - 1;
+    vec = v;
 }
 
 Stage::~Stage() {
     if (slot < 0) return;
     std::lock_guard<std::mutex> g(g_prof_mu);
-    if (slot < int(g_recs.size())) {
-        cudaEventRecord(g_recs[slot].b, s);
-        g_recs[slot].l1 = g_launches.load();
+    auto &v = *static_cast<std::vector<StageRec> *>(vec);
+    if (slot < int(v.size())) {
+        if (t_cap && t_cap->items) cap_cut(s, v[slot].b);
+        else cudaEventRecord(v[slot].b, s);
+        v[slot].l1 = g_launches.load();
     }
 }
 
@@ -257,12 +335,33 @@ void *ws_get(int slot, size_t bytes, cudaStream_t s) {
         g_ws.push_back({{d, s}, w});
     }
     if (w->sz[slot] < bytes) {
+        if (t_cap && t_cap->mode == 2) {  // the measuring run sized every workspace
+            fail(GPUMEM_ERR_NOMEM, "workspace %d would grow during a pipeline capture", slot);
+            return nullptr;
+        }
+        t_ws_alloc = true;
         if (w->p[slot]) dfree(w->p[slot], s);
         const size_t want = bytes + bytes / 8 + 4096;
         w->p[slot] = dalloc(want, s);
         w->sz[slot] = w->p[slot] ? want : 0;
+        t_ws_alloc = false;
     }
     return w->p[slot];
+}
+
+// Free one stream's workspace (the stream is about to be destroyed).
+void ws_release_stream(int d, cudaStream_t s) {
+    std::lock_guard<std::mutex> g(g_ws_mu);
+    for (size_t i = 0; i < g_ws.size(); ++i) {
+        if (g_ws[i].first.first != d || g_ws[i].first.second != s) continue;
+        cudaStreamSynchronize(s);
+        for (int k = 0; k < kWsCount; ++k)
+            if (g_ws[i].second->p[k]) dfree(g_ws[i].second->p[k], s);
+        cudaStreamSynchronize(s);
+        delete g_ws[i].second;
+        g_ws.erase(g_ws.begin() + long(i));
+        return;
+    }
 }
 
 unsigned long long *pinned_slots() {  // 16 per thread, never freed
@@ -274,6 +373,136 @@ unsigned long long *pinned_slots() {  // 16 per thread, never freed
         }
     }
     return p;
+}
+
+}  // namespace
+
+// ---------------------------------------------------------------- pipeline (CUDA graph)
+struct gpumem_pipeline {
+    uint32_t magic;
+    int device;
+    cudaStream_t user;                     // the caller's stream (runs are ordered on it by events)
+    cudaStream_t stream;                   // the pipeline's own stream: capture, launches, fallback
+    cudaEvent_t ev_in, ev_out;
+    uint64_t nR, nQ, q_begin, q_end;
+    uint32_t ls, L;
+    const char *inR, *inQ;                 // the device inputs the graph was captured with
+    char *arena;
+    size_t arena_bytes;
+    std::vector<PipeItem> items;           // graph segments and stage events, in run order
+    gpumem_seq *R, *Q;
+    gpumem_index *idx;
+    gpumem_mems *mems;                     // the graph's result buffer (count set by _result)
+    gpumem_mems *fallback;                 // overflow rerun through gpumem_find_mems
+    unsigned long long *host;              // pinned counters written by the graph
+    uint64_t out_cap, coop_cap, spill_cap, span;
+    std::vector<StageRec> recs;
+    uint64_t launches;                     // kernels per graph launch
+    int ran;
+    gpumem_find_stats stats;
+};
+
+namespace {
+
+// The whole path on the pipeline's stream: pack R, pack Q, index R, find (deferred).
+gpumem_status pipeline_path(gpumem_pipeline *pl, const char *R, const char *Q, gpumem_seq **hR, gpumem_seq **hQ,
+                            gpumem_index **hI, gpumem_mems **hM) {
+    *hR = *hQ = nullptr;
+    *hI = nullptr;
+    *hM = nullptr;
+    gpumem_status st = gpumem_pack(R, pl->nR, 1, pl->stream, hR);
+    if (!st) st = gpumem_pack(Q, pl->nQ, 1, pl->stream, hQ);
+    if (!st) st = gpumem_index_build(*hR, pl->ls, pl->L, pl->stream, hI);
+    if (!st) st = gpumem_find_mems(*hI, *hQ, pl->q_begin, pl->q_end, pl->stream, hM);
+    return st;
+}
+
+void pipeline_release(gpumem_pipeline *pl) {  // graph, arena and the arena-backed handles
+    for (auto &it : pl->items) {
+        if (it.x) cudaGraphExecDestroy(it.x);
+        if (it.g) cudaGraphDestroy(it.g);
+    }
+    pl->items.clear();
+    if (pl->R) { pl->R->magic = 0; delete pl->R; }
+    if (pl->Q) { pl->Q->magic = 0; delete pl->Q; }
+    if (pl->idx) { pl->idx->magic = 0; delete pl->idx; }
+    if (pl->mems) { pl->mems->magic = 0; delete pl->mems; }
+    pl->R = pl->Q = nullptr;
+    pl->idx = nullptr;
+    pl->mems = nullptr;
+    if (pl->arena) cudaFree(pl->arena);
+    pl->arena = nullptr;
+    pl->arena_bytes = 0;
+    {
+        std::lock_guard<std::mutex> g(g_prof_mu);
+        for (auto &r : pl->recs) {
+            g_ev_free.push_back(r.a);
+            g_ev_free.push_back(r.b);
+        }
+    }
+    pl->recs.clear();
+    pl->inR = pl->inQ = nullptr;
+    cudaGetLastError();
+}
+
+gpumem_status pipeline_capture(gpumem_pipeline *pl, const char *R, const char *Q) {
+    cudaStream_t s = pl->stream;
+    CK(cudaStreamSynchronize(s), "sync");
+    pipeline_release(pl);
+    // 1) measuring run: sizes every workspace, sums the handle/scratch bytes
+    CapCtx m;
+    m.mode = 1;
+    m.deferred = true;
+    m.host = pl->host;
+    gpumem_seq *hR, *hQ;
+    gpumem_index *hI;
+    gpumem_mems *hM;
+    t_cap = &m;
+    gpumem_status st = pipeline_path(pl, R, Q, &hR, &hQ, &hI, &hM);
+    t_cap = nullptr;
+    const cudaError_t se = cudaStreamSynchronize(s);
+    for (void *h : {(void *)hM, (void *)hI, (void *)hQ, (void *)hR}) gpumem_free(h);
+    if (st) return st;
+    CK(se, "measuring run");
+    CK(cudaStreamSynchronize(s), "sync");
+    // 2) capture into the arena
+    pl->arena_bytes = m.need + (1u << 20);
+    CK(cudaMalloc(&pl->arena, pl->arena_bytes), "pipeline arena");
+    CapCtx c;
+    c.mode = 2;
+    c.arena = pl->arena;
+    c.cap = pl->arena_bytes;
+    c.deferred = true;
+    c.host = pl->host;
+    c.recs = &pl->recs;
+    c.items = &pl->items;
+    c.expect_n = pl->host[0];
+    CK(cudaStreamBeginCapture(s, cudaStreamCaptureModeRelaxed), "begin capture");
+    const uint64_t l0 = g_launches.load();
+    t_cap = &c;
+    st = pipeline_path(pl, R, Q, &pl->R, &pl->Q, &pl->idx, &pl->mems);
+    if (!st) cap_cut(s, nullptr);  // the last segment (a fresh capture is left open)
+    t_cap = nullptr;
+    pl->launches = g_launches.load() - l0;
+    g_launches.fetch_sub(pl->launches);      // captured, not launched
+    cudaGraph_t rest = nullptr;
+    const cudaError_t ce = cudaStreamEndCapture(s, &rest);
+    if (rest) cudaGraphDestroy(rest);
+    if (st) {
+        pipeline_release(pl);
+        return st;
+    }
+    if (c.err != cudaSuccess || ce != cudaSuccess) {
+        pipeline_release(pl);
+        return cuda_fail(c.err != cudaSuccess ? c.err : ce, "pipeline capture");
+    }
+    pl->out_cap = c.out_cap;
+    pl->coop_cap = c.coop_cap;
+    pl->spill_cap = c.spill_cap;
+    pl->span = c.span;
+    pl->inR = R;
+    pl->inQ = Q;
+    return GPUMEM_OK;
 }
 
 }  // namespace
@@ -321,7 +550,7 @@ gpumem_status gpumem_set_option(const char *name, int64_t value) {
     else if (!strcmp(name, "use_bitmap")) g_opt.use_bitmap = value ? 1 : 0;
     else if (!strcmp(name, "static_lb")) g_opt.static_lb = value ? 1 : 0;
     else if (!strcmp(name, "sort_impl")) {
-        if (value < 0 || value > 2) return fail(GPUMEM_ERR_ARG, "sort_impl must be 0, 1 or 2");
+        if (value < 0 || value > 3) return fail(GPUMEM_ERR_ARG, "sort_impl must be 0, 1, 2 or 3");
         g_opt.sort_impl = value;
     }
     else if (!strcmp(name, "index_msd")) g_opt.index_msd = value ? 1 : 0;
@@ -393,6 +622,20 @@ void gpumem_free(void *handle) {
         dfree(x->recs, x->stream);
         x->magic = 0;
         delete x;
+    } else if (magic == kMagicPipe) {
+        auto *pl = static_cast<gpumem_pipeline *>(handle);
+        cudaSetDevice(pl->device);
+        cudaStreamSynchronize(pl->stream);
+        if (pl->fallback) gpumem_free(pl->fallback);
+        pipeline_release(pl);
+        cudaStreamSynchronize(pl->stream);
+        cudaFreeHost(pl->host);
+        cudaEventDestroy(pl->ev_in);
+        cudaEventDestroy(pl->ev_out);
+        ws_release_stream(pl->device, pl->stream);
+        cudaStreamDestroy(pl->stream);
+        pl->magic = 0;
+        delete pl;
     } else if (magic == kMagicMems) {
         auto *m = static_cast<gpumem_mems *>(handle);
         cudaSetDevice(m->device);
@@ -666,11 +909,17 @@ static gpumem_status sort_into_triples(uint64_t *keys, uint32_t *lens, uint64_t 
         Stage g("sort", s);
         // MSD bucket sort (keys are unique): two passes over the data; measured faster than
         // the 7-pass LSD radix up to a few million keys, slower beyond (its 16K-way scatter)
-        constexpr uint64_t kMsdMaxN = 4u << 20;
         if (g_opt.sort_impl == 0 && g_opt.small_sort && n <= small_sort_max_n(8)) {
             void *scratch = ws_get(kWsSmall, small_sort_scratch_bytes(n, 8), s);
             if (!scratch) return GPUMEM_ERR_NOMEM;
             CK(small_sort_triples(keys, lens, n, int(key_bits), qbits, trip, scratch, s), "triple sort");
+        } else if (g_opt.sort_impl == 3) {  // hybrid: 2 LSD passes on the top 16 bits + local sorts
+            auto *k1 = static_cast<uint64_t *>(ws_get(kWsSortK, n * 8, s));
+            auto *l1 = static_cast<uint32_t *>(ws_get(kWsSortL, n * 4, s));
+            void *scratch = ws_get(kWsSortScratch, hybrid_scratch_bytes(), s);
+            if (!k1 || !l1 || !scratch) return GPUMEM_ERR_NOMEM;
+            CK(hybrid_sort_triples(keys, lens, k1, l1, nullptr, n, int(key_bits), scratch, s, trip, qbits),
+               "triple sort");
         } else if (g_opt.sort_impl == 2 || (g_opt.sort_impl == 0 && n <= kMsdMaxN)) {
             void *scratch = ws_get(kWsSortScratch, msd_scratch_bytes(n), s);
             if (!scratch) return GPUMEM_ERR_NOMEM;
@@ -765,6 +1014,67 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
     unsigned long long *h = pinned_slots();
     if (!h) return fail(GPUMEM_ERR_NOMEM, "pinned host buffer");
 
+    if (t_cap && t_cap->deferred) {
+        // pipeline: one pass with the automatic capacity, no host round trip. The sort
+        // takes the MEM count from the device counter; the counters and alphabet flags go
+        // to the pipeline's pinned buffer, checked by gpumem_pipeline_result (which reruns
+        // this call the ordinary way in the rare overflow case).
+        auto *keys = static_cast<uint64_t *>(ws_get(kWsKeys, cap * 8, s));
+        auto *lens = static_cast<uint32_t *>(ws_get(kWsLens, cap * 4, s));
+        P.coopq = static_cast<uint2 *>(ws_get(kWsCoop, coop_cap * sizeof(uint2), s));
+        // output sort by the device-resident count; which one: sort_impl if pinned, else by
+        // the MEM count of the pipeline's measuring run (MSD up to kMsdMaxN, LSD beyond)
+        int impl = int(g_opt.sort_impl);
+        if (impl == 0) impl = (t_cap->mode == 2 && t_cap->expect_n > kMsdMaxN) ? 1 : 2;
+        size_t sbytes = msd_scratch_bytes(cap);
+        if (hybrid_scratch_bytes() > sbytes) sbytes = hybrid_scratch_bytes();
+        if (radix_scratch_bytes(cap) > sbytes) sbytes = radix_scratch_bytes(cap);
+        void *scratch = ws_get(kWsSortScratch, sbytes, s);  // sized for every choice: the measuring
+        auto *k1 = static_cast<uint64_t *>(ws_get(kWsSortK, cap * 8, s));  // run and the capture agree
+        auto *l1 = static_cast<uint32_t *>(ws_get(kWsSortL, cap * 4, s));
+        auto *trip = static_cast<gpumem_triple *>(sc.get(cap * sizeof(gpumem_triple)));
+        if (!keys || !lens || !P.coopq || !scratch || !trip || !k1 || !l1) return GPUMEM_ERR_NOMEM;
+        P.out_key = keys;
+        P.out_len = lens;
+        P.capacity = cap;
+        P.coop_cap = coop_cap;
+        CK(cudaMemsetAsync(ctr, 0, 64, s), "memset counters");
+        {
+            Stage g("find", s);
+            CK(launch_find(P, int(g_opt.find_grid), s), "find kernel");
+        }
+        if (P.n_tiles) {
+            Stage g("find.heavy", s);
+            CK(launch_heavy(P, s), "heavy kernel");
+            CK(launch_coop(P, s), "coop kernel");
+        }
+        {
+            Stage g("sort", s);
+            const int kb = int(bits_for(nR) + P.qbits);
+            if (impl == 3) {
+                CK(hybrid_sort_triples(keys, lens, k1, l1, ctr, cap, kb, scratch, s, trip, P.qbits), "triple sort");
+            } else if (impl == 2) {
+                CK(msd_sort_dev(keys, lens, ctr, cap, kb, scratch, s, trip, P.qbits), "triple sort");
+            } else {
+                bool alt = false;
+                CK(radix_sort_u64(keys, lens, k1, l1, cap, kb, scratch, s, &alt, 0, ctr), "triple sort");
+                CK(launch_keys_to_triples(alt ? k1 : keys, alt ? l1 : lens, cap, P.qbits, trip, s, ctr),
+                   "keys to triples");
+            }
+        }
+        CK(cudaMemcpyAsync(t_cap->host, ctr, 64, cudaMemcpyDeviceToHost, s), "D2H counters");
+        CK(cudaMemcpyAsync(t_cap->host + 8, R->bad, 8, cudaMemcpyDeviceToHost, s), "D2H flag");
+        CK(cudaMemcpyAsync(t_cap->host + 9, Q->bad, 8, cudaMemcpyDeviceToHost, s), "D2H flag");
+        sc.keep(trip);
+        *out = new gpumem_mems{kMagicMems, dev, s, 0, trip, gpumem_find_stats{}};
+        t_cap->out_cap = cap;
+        t_cap->coop_cap = coop_cap;
+        t_cap->spill_cap = spill_cap;
+        t_cap->span = span;
+        t_cap->mems = *out;
+        return GPUMEM_OK;
+    }
+
     uint64_t count = 0;
     int attempts = 0;
     uint64_t *keys = nullptr;
@@ -816,6 +1126,144 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
         (*out)->stats = fs;
     }
     return st2;
+}
+
+gpumem_status gpumem_pipeline_create(uint64_t r_len, uint64_t q_len, uint32_t seed_len, uint32_t min_len,
+                                     uint64_t q_begin, uint64_t q_end, void *cuda_stream, gpumem_pipeline **out) {
+    if (!out) return fail(GPUMEM_ERR_ARG, "out is NULL");
+    *out = nullptr;
+    if (seed_len < 1 || seed_len > 15 || min_len < seed_len)
+        return fail(GPUMEM_ERR_ARG, "need 1 <= seed_len <= 15 and seed_len <= min_len (got %u, %u)", seed_len,
+                    min_len);
+    if (r_len >= (1ull << 32) || q_len >= (1ull << 32))
+        return fail(GPUMEM_ERR_RANGE, "sequences must be shorter than 2^32 bases");
+    if (q_begin > q_len) return fail(GPUMEM_ERR_RANGE, "q_begin > |Q|");
+    int dev;
+    gpumem_status st = check_device(&dev);
+    if (st) return st;
+    auto *pl = new gpumem_pipeline{};
+    pl->magic = kMagicPipe;
+    pl->device = dev;
+    pl->user = static_cast<cudaStream_t>(cuda_stream);
+    // the legacy default stream cannot be captured: the graph runs on a stream of its
+    // own, ordered after / before the caller's stream by events
+    if (cudaStreamCreateWithFlags(&pl->stream, cudaStreamNonBlocking) != cudaSuccess ||
+        cudaEventCreateWithFlags(&pl->ev_in, cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreateWithFlags(&pl->ev_out, cudaEventDisableTiming) != cudaSuccess) {
+        const cudaError_t e = cudaGetLastError();
+        delete pl;
+        return cuda_fail(e, "pipeline stream");
+    }
+    pl->nR = r_len;
+    pl->nQ = q_len;
+    pl->q_begin = q_begin;
+    pl->q_end = q_end;
+    pl->ls = seed_len;
+    pl->L = min_len;
+    if (cudaMallocHost(&pl->host, 16 * sizeof(unsigned long long)) != cudaSuccess) {
+        cudaGetLastError();
+        delete pl;
+        return fail(GPUMEM_ERR_NOMEM, "pinned host buffer");
+    }
+    *out = pl;
+    return GPUMEM_OK;
+}
+
+gpumem_status gpumem_pipeline_run(gpumem_pipeline *pl, const char *r_bases_dev, const char *q_bases_dev) {
+    if (!pl || pl->magic != kMagicPipe) return fail(GPUMEM_ERR_ARG, "not a gpumem_pipeline");
+    if ((!r_bases_dev && pl->nR) || (!q_bases_dev && pl->nQ)) return fail(GPUMEM_ERR_ARG, "NULL input");
+    int dev = -1;
+    cudaGetDevice(&dev);
+    if (dev != pl->device) return fail(GPUMEM_ERR_ARG, "pipeline lives on device %d, current is %d", pl->device, dev);
+    if (pl->fallback) {
+        gpumem_free(pl->fallback);
+        pl->fallback = nullptr;
+    }
+    CK(cudaEventRecord(pl->ev_in, pl->user), "event");  // inputs written on the caller's stream
+    CK(cudaStreamWaitEvent(pl->stream, pl->ev_in, 0), "wait");
+    if (pl->items.empty() || pl->inR != r_bases_dev || pl->inQ != q_bases_dev) {
+        const gpumem_status st = pipeline_capture(pl, r_bases_dev, q_bases_dev);
+        if (st) return st;
+    }
+    for (const auto &it : pl->items) {
+        if (it.x) CK(cudaGraphLaunch(it.x, pl->stream), "graph launch");
+        else CK(cudaEventRecord(it.ev, pl->stream), "stage event");
+    }
+    note_launch(int(pl->launches));
+    CK(cudaEventRecord(pl->ev_out, pl->stream), "event");  // the caller's later work sees the result
+    CK(cudaStreamWaitEvent(pl->user, pl->ev_out, 0), "wait");
+    pl->ran = 1;
+    return GPUMEM_OK;
+}
+
+gpumem_status gpumem_pipeline_result(gpumem_pipeline *pl, const gpumem_triple **dev_ptr, uint64_t *count) {
+    if (!pl || pl->magic != kMagicPipe) return fail(GPUMEM_ERR_ARG, "not a gpumem_pipeline");
+    if (!pl->ran) return fail(GPUMEM_ERR_ARG, "gpumem_pipeline_run has not been called");
+    CK(cudaStreamSynchronize(pl->stream), "pipeline sync");
+    const unsigned long long *h = pl->host;
+    if (h[8] != ~0ull) return fail(GPUMEM_ERR_ALPHABET, "R: byte at position %llu is not in {A,C,G,T,a,c,g,t}", h[8]);
+    if (h[9] != ~0ull) return fail(GPUMEM_ERR_ALPHABET, "Q: byte at position %llu is not in {A,C,G,T,a,c,g,t}", h[9]);
+    gpumem_find_stats fs{};
+    fs.positions = pl->span;
+    fs.occupied = h[3] + h[6];
+    fs.hits = h[4] + h[5];
+    fs.spilled_chunks = h[1] < pl->spill_cap ? h[1] : pl->spill_cap;
+    fs.attempts = 1;
+    const gpumem_mems *res = pl->mems;
+    uint64_t n = h[0];
+    if (!pl->fallback && (h[0] > pl->out_cap || h[7] > pl->coop_cap)) {
+        // output or coop queue overflow: the ordinary call (exact-capacity retry) on the
+        // pipeline's packed sequences and index
+        const gpumem_status st = gpumem_find_mems(pl->idx, pl->Q, pl->q_begin, pl->q_end, pl->stream, &pl->fallback);
+        if (st) return st;
+        fs.attempts = 2;
+        CK(cudaEventRecord(pl->ev_out, pl->stream), "event");
+        CK(cudaStreamWaitEvent(pl->user, pl->ev_out, 0), "wait");
+    }
+    if (pl->fallback) {
+        res = pl->fallback;
+        n = pl->fallback->count;
+        fs = pl->fallback->stats;
+        fs.attempts += 1;
+    } else {
+        pl->mems->count = n;
+    }
+    fs.mems = n;
+    pl->stats = fs;
+    if (dev_ptr) *dev_ptr = res->dev;
+    if (count) *count = n;
+    return GPUMEM_OK;
+}
+
+gpumem_status gpumem_pipeline_stats(const gpumem_pipeline *pl, gpumem_find_stats *out) {
+    if (!pl || pl->magic != kMagicPipe || !out) return fail(GPUMEM_ERR_ARG, "not a gpumem_pipeline");
+    *out = pl->stats;
+    return GPUMEM_OK;
+}
+
+int gpumem_pipeline_profile(const gpumem_pipeline *pl, const char **names, double *ms, uint64_t *launches,
+                            int max_stages) {
+    if (!pl || pl->magic != kMagicPipe) return 0;
+    int n = 0;
+    for (auto &r : pl->recs) {
+        float t = 0.f;
+        cudaEventSynchronize(r.b);
+        cudaEventElapsedTime(&t, r.a, r.b);
+        int i = 0;
+        for (; i < n; ++i)
+            if (!strcmp(names[i], r.name)) break;
+        if (i == n) {
+            if (n >= max_stages) continue;
+            names[n] = r.name;
+            ms[n] = 0;
+            launches[n] = 0;
+            ++n;
+        }
+        ms[i] += t;
+        launches[i] += r.l1 - r.l0;
+    }
+    cudaGetLastError();
+    return n;
 }
 
 gpumem_status gpumem_mums(const gpumem_mems *m, void *cuda_stream, gpumem_mems **out) {

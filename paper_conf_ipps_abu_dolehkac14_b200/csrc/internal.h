@@ -16,7 +16,7 @@ struct Options {
     int64_t use_bitmap = 1;      // 1: rank-word probe + compact bucket table; 0: read the dense ptrs
     int64_t static_lb = 0;       // 1: each lane processes its own positions' hits (LB ablation)
     int64_t sort_impl = 0;       // output sort: 0 = auto (MSD below kMsdMaxN keys, else LSD), 1 = stable LSD radix
-                                 // (radix.cu), 2 = MSD bucket sort (msd.cu)
+                                 // (radix.cu), 2 = MSD bucket sort (msd.cu), 3 = hybrid (msd.cu)
     int64_t small_sort = 0;      // 1: single-launch cooperative sorts when the input fits (small_sort.cu;
                                  // measured slower at C4: its scattered global writes are not coalesced)
     int64_t index_msd = 0;
@@ -39,11 +39,14 @@ gpumem_status fail(gpumem_status st, const char *fmt, ...);
 gpumem_status cuda_fail(cudaError_t e, const char *what);
 
 // Brackets one stage with CUDA events when profiling is enabled.
+// Inside a pipeline capture the events go to the pipeline instead (re-recorded by
+// every graph launch).
 struct Stage {
     Stage(const char *name, cudaStream_t s);
     ~Stage();
     int slot;
     cudaStream_t s;
+    void *vec;
 };
 
 // ---------------------------------------------------------------- kernels (launchers)
@@ -59,8 +62,10 @@ cudaError_t launch_revcomp(const uint64_t *in, uint64_t n, uint64_t *out, uint64
 // `scratch` must hold radix_scratch_bytes(n) bytes (digit counts + scan partials).
 cudaError_t radix_sort_u32(uint32_t *k0, uint32_t *v0, uint32_t *k1, uint32_t *v1, uint64_t n, int bits,
                            void *scratch, cudaStream_t s, bool *in_alt, int lo = 0);
+// radix_sort_u64 with dn != null: n is a capacity, the count is min(*dn, n) on the device.
 cudaError_t radix_sort_u64(uint64_t *k0, uint32_t *v0, uint64_t *k1, uint32_t *v1, uint64_t n, int bits,
-                           void *scratch, cudaStream_t s, bool *in_alt);
+                           void *scratch, cudaStream_t s, bool *in_alt, int lo = 0,
+                           const unsigned long long *dn = nullptr);
 size_t radix_scratch_bytes(uint64_t n);
 
 // Single-launch (cooperative) stable LSD radix sorts for small inputs (small_sort.cu):
@@ -78,6 +83,16 @@ cudaError_t small_sort_triples(const uint64_t *keys, const uint32_t *lens, uint6
 size_t msd_scratch_bytes(uint64_t n);
 cudaError_t msd_sort(uint64_t *keys, uint32_t *vals, uint64_t n, int bits, void *scratch, cudaStream_t s,
                      gpumem_triple *trip = nullptr, uint32_t qbits = 0);
+// The same with the key count in device memory (n = min(*d_n, cap)); capturable.
+cudaError_t msd_sort_dev(uint64_t *keys, uint32_t *vals, const unsigned long long *d_n, uint64_t cap, int bits,
+                         void *scratch, cudaStream_t s, gpumem_triple *trip, uint32_t qbits);
+// Output sort for large key sets: stable LSD passes over the top 16 key bits, then
+// every run of equal 16-bit prefix sorted in shared memory and written as triples
+// (msd.cu). (k1, v1): ping-pong buffers of cap entries. d_n: device count or null.
+size_t hybrid_scratch_bytes();
+cudaError_t hybrid_sort_triples(uint64_t *keys, uint32_t *vals, uint64_t *k1, uint32_t *v1,
+                                const unsigned long long *d_n, uint64_t cap, int bits, void *scratch,
+                                cudaStream_t s, gpumem_triple *trip, uint32_t qbits);
 // keys[i] = (codes[i] << 32) | locs[i] and back (sort.cu)
 cudaError_t launch_join_keys(const uint32_t *codes, const uint32_t *locs, uint64_t n, uint64_t *keys, cudaStream_t s);
 cudaError_t launch_split_keys(const uint64_t *keys, uint64_t n, uint32_t *codes, uint32_t *locs, cudaStream_t s);
@@ -152,7 +167,7 @@ cudaError_t mum_filter(const gpumem_triple *in, uint64_t n, gpumem_triple *out, 
 
 // Triples (sort.cu)
 cudaError_t launch_keys_to_triples(const uint64_t *keys, const uint32_t *lens, uint64_t n, uint32_t qbits,
-                                   gpumem_triple *out, cudaStream_t s);
+                                   gpumem_triple *out, cudaStream_t s, const unsigned long long *dn = nullptr);
 cudaError_t launch_triples_to_keys(const gpumem_triple *in, uint64_t n, uint32_t qbits, uint64_t *keys,
                                    uint32_t *lens, cudaStream_t s);
 

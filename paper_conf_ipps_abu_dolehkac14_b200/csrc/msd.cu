@@ -22,6 +22,10 @@
 //  k_bs_big      buckets too large for shared memory (adversarial inputs: e.g. one
 //                r with 10^5 MEMs) get a CTA-level LSD radix in global memory.
 // No per-element global atomics anywhere. B is chosen so that buckets average ~512 keys.
+// The key count n may live in device memory (msd_sort_dev: the find kernel's output
+// counter, so a captured CUDA graph needs no host round trip): every kernel derives n,
+// B, the bucket count and its chunk bounds from it on the device; grids are sized for
+// the capacity and idle blocks exit (k_bs_local loops over segments).
 #include "internal.h"
 #include "device.cuh"
 
@@ -38,10 +42,34 @@ constexpr uint32_t kLocal = kLT * kItems;        // most keys one CTA sorts in s
 constexpr uint32_t kSeg = kLocal / 2;            // segment spacing (slots)
 constexpr int kMaxB = 14;                        // 16384 buckets: a 64 KB shared histogram
 
+__host__ __device__ __forceinline__ int choose_b(uint64_t n, int bits) {
+    int B = 1;
+    while (B < kMaxB && (n >> (B + 9)) > 0) ++B;  // ~512 keys per bucket
+    return B < bits ? B : bits;
+}
+
+// The number of keys: *dn clamped to cap when the count is device-resident, else cap.
+struct NSpec {
+    const unsigned long long *dn;
+    uint64_t cap;
+    int bits;                                    // significant key bits
+    int fixed_b;                                 // bucket = the top fixed_b bits (hybrid sort), else chosen by n
+    __device__ __forceinline__ int B(uint64_t n) const { return fixed_b ? fixed_b : choose_b(n, bits); }
+    __device__ __forceinline__ uint64_t n() const {
+        if (!dn) return cap;
+        const unsigned long long x = *dn;
+        return x < cap ? x : cap;
+    }
+};
+
 // chunk c = elements [c * cs, min((c + 1) * cs, n))
-__global__ void __launch_bounds__(kPT) k_bp_hist(const uint64_t *__restrict__ keys, uint64_t n, uint64_t cs,
-                                                 int shift, uint32_t nb, uint32_t *__restrict__ counts) {
+__global__ void __launch_bounds__(kPT) k_bp_hist(const uint64_t *__restrict__ keys, NSpec ns,
+                                                 uint32_t *__restrict__ counts) {
     extern __shared__ uint32_t h[];
+    const uint64_t n = ns.n();
+    const int B = choose_b(n, ns.bits), shift = ns.bits - B;
+    const uint32_t nb = 1u << B;
+    const uint64_t cs = (n + gridDim.x - 1) / gridDim.x;
     for (uint32_t i = threadIdx.x; i < nb; i += kPT) h[i] = 0;
     __syncthreads();
     const uint64_t b = uint64_t(blockIdx.x) * cs, e = min(b + cs, n);
@@ -52,8 +80,9 @@ __global__ void __launch_bounds__(kPT) k_bp_hist(const uint64_t *__restrict__ ke
 }
 
 // per bucket b (one thread): counts[c][b] -> exclusive prefix over c (in place); totals[b]
-__global__ void __launch_bounds__(256) k_bp_colscan(uint32_t *__restrict__ counts, uint32_t chunks, uint32_t nb,
+__global__ void __launch_bounds__(256) k_bp_colscan(uint32_t *__restrict__ counts, uint32_t chunks, NSpec ns,
                                                     uint32_t *__restrict__ totals) {
+    const uint32_t nb = 1u << choose_b(ns.n(), ns.bits);
     const uint32_t b = blockIdx.x * 256 + threadIdx.x;
     if (b >= nb) return;
     uint32_t run = 0;
@@ -78,9 +107,10 @@ __global__ void __launch_bounds__(256) k_bp_colscan(uint32_t *__restrict__ count
 
 // exclusive scan of totals[0..nb) -> offs[0..nb] (offs[nb] = the sum); each thread owns
 // a contiguous run of ceil(nb / 1024) entries
-__global__ void __launch_bounds__(1024) k_bs_scan(const uint32_t *__restrict__ totals, uint32_t nb,
+__global__ void __launch_bounds__(1024) k_bs_scan(const uint32_t *__restrict__ totals, NSpec ns,
                                                   uint32_t *__restrict__ offs) {
     __shared__ uint32_t ws[32];
+    const uint32_t nb = 1u << choose_b(ns.n(), ns.bits);
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     const uint32_t per = (nb + 1023) / 1024;
     const uint32_t i0 = threadIdx.x * per, i1 = min(i0 + per, nb);
@@ -104,11 +134,15 @@ __global__ void __launch_bounds__(1024) k_bs_scan(const uint32_t *__restrict__ t
 }
 
 __global__ void __launch_bounds__(kPT) k_bp_scatter(const uint64_t *__restrict__ keys,
-                                                    const uint32_t *__restrict__ vals, uint64_t n, uint64_t cs,
-                                                    int shift, uint32_t nb, const uint32_t *__restrict__ rel,
+                                                    const uint32_t *__restrict__ vals, NSpec ns,
+                                                    const uint32_t *__restrict__ rel,
                                                     const uint32_t *__restrict__ offs, uint64_t *__restrict__ ok,
                                                     uint32_t *__restrict__ ov) {
     extern __shared__ uint32_t cur[];
+    const uint64_t n = ns.n();
+    const int B = choose_b(n, ns.bits), shift = ns.bits - B;
+    const uint32_t nb = 1u << B;
+    const uint64_t cs = (n + gridDim.x - 1) / gridDim.x;
     const uint32_t *row = rel + uint64_t(blockIdx.x) * nb;
     for (uint32_t i = threadIdx.x; i < nb; i += kPT) cur[i] = offs[i] + row[i];
     __syncthreads();
@@ -273,31 +307,37 @@ __device__ void smem_sort_write(LocalSmem &S, const uint64_t *__restrict__ tk, c
     __syncthreads();
 }
 
-__global__ void __launch_bounds__(kLT, 2) k_bs_local(const uint32_t *__restrict__ offs, uint32_t nb, int bits,
+__global__ void __launch_bounds__(kLT, 2) k_bs_local(const uint32_t *__restrict__ offs, NSpec ns,
                                                  const uint64_t *__restrict__ tk, const uint32_t *__restrict__ tv,
                                                  Out out, uint32_t *__restrict__ big, unsigned int *n_big) {
     extern __shared__ __align__(16) unsigned char smem[];
     LocalSmem &S = *reinterpret_cast<LocalSmem *>(smem);
     __shared__ uint32_t s_b[2];
-    if (threadIdx.x == 0) s_b[0] = first_at(offs, nb, uint64_t(blockIdx.x) * kSeg);
-    if (threadIdx.x == 32) s_b[1] = first_at(offs, nb, uint64_t(blockIdx.x + 1) * kSeg);
-    __syncthreads();
-    const uint32_t b0 = s_b[0], b1 = s_b[1];
-    if (b0 >= b1) return;
-    const uint32_t lo = offs[b0], m = offs[b1] - lo;
-    if (m <= kLocal) {
-        // the segment's keys share no common prefix below the bucket bits in general:
-        // sort by all key bits (the bucket prefix bits then sort the buckets among themselves)
-        smem_sort_write(S, tk, tv, lo, m, bits, out);
-        return;
-    }
-    for (uint32_t b = b0; b < b1; ++b) {  // a large bucket in the segment: one bucket at a time
-        const uint32_t blo = offs[b], bm = offs[b + 1] - blo;
-        if (bm == 0) continue;
-        if (bm <= kLocal) {
-            smem_sort_write(S, tk, tv, blo, bm, bits, out);
-        } else if (threadIdx.x == 0) {
-            big[atomicAdd(n_big, 1u)] = b;
+    const uint64_t n = ns.n();
+    const int bits = ns.bits;
+    const uint32_t nb = 1u << ns.B(n);
+    for (uint64_t seg = blockIdx.x; seg * kSeg < n; seg += gridDim.x) {
+        __syncthreads();  // the previous segment's readers of s_b are done
+        if (threadIdx.x == 0) s_b[0] = first_at(offs, nb, seg * kSeg);
+        if (threadIdx.x == 32) s_b[1] = first_at(offs, nb, (seg + 1) * kSeg);
+        __syncthreads();
+        const uint32_t b0 = s_b[0], b1 = s_b[1];
+        if (b0 >= b1) continue;
+        const uint32_t lo = offs[b0], m = offs[b1] - lo;
+        if (m <= kLocal) {
+            // the segment's keys share no common prefix below the bucket bits in general:
+            // sort by all key bits (the bucket prefix bits then sort the buckets among themselves)
+            smem_sort_write(S, tk, tv, lo, m, bits, out);
+            continue;
+        }
+        for (uint32_t b = b0; b < b1; ++b) {  // a large bucket in the segment: one bucket at a time
+            const uint32_t blo = offs[b], bm = offs[b + 1] - blo;
+            if (bm == 0) continue;
+            if (bm <= kLocal) {
+                smem_sort_write(S, tk, tv, blo, bm, bits, out);
+            } else if (threadIdx.x == 0) {
+                big[atomicAdd(n_big, 1u)] = b;
+            }
         }
     }
 }
@@ -306,12 +346,13 @@ __global__ void __launch_bounds__(kLT, 2) k_bs_local(const uint32_t *__restrict_
 // ping-ponging between (tk, tv) and (sk, sv) over the bucket's range; then written out.
 __global__ void __launch_bounds__(kT) k_bs_big(const uint32_t *__restrict__ offs, const uint32_t *__restrict__ big,
                                                const unsigned int *__restrict__ n_big, uint64_t *tk, uint32_t *tv,
-                                               uint64_t *xk, uint32_t *xv, int bits, Out out) {
+                                               uint64_t *xk, uint32_t *xv, NSpec ns, Out out) {
     __shared__ uint32_t hist[256];
     __shared__ uint32_t wcnt[kWarps][256];
     __shared__ uint32_t ws[kWarps];
     const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
     const unsigned nbig = *n_big;
+    const int bits = ns.bits - ns.B(ns.n());  // the bits below the bucket prefix
     const int passes = (bits + 7) / 8;
     for (unsigned li = blockIdx.x; li < nbig; li += gridDim.x) {
         const uint32_t b = big[li];
@@ -385,12 +426,6 @@ __global__ void __launch_bounds__(kT) k_bs_big(const uint32_t *__restrict__ offs
     }
 }
 
-int choose_b(uint64_t n, int bits) {
-    int B = 1;
-    while (B < kMaxB && (n >> (B + 9)) > 0) ++B;  // ~512 keys per bucket
-    return B < bits ? B : bits;
-}
-
 uint32_t n_chunks(uint64_t n) {
     const uint64_t c = (n + 4095) / 4096;  // >= 4K keys per chunk
     const uint64_t cap = uint64_t(num_sms());
@@ -405,35 +440,28 @@ size_t msd_scratch_bytes(uint64_t n) {
     return n * 8 + n * 4 * 2 + chunks * nb * 4 + (nb + 1) * 4 * 2 + nb * 4 + 1024 + 8 * 256;
 }
 
-// Sorts n unique keys whose significant bits are the low `bits` (+ values, may be null).
-// Result: in place in (keys, vals), or as triples {key >> qbits, key & qmask, val} in
-// `trip` when trip != null. `scratch` >= msd_scratch_bytes(n).
-cudaError_t msd_sort(uint64_t *keys, uint32_t *vals, uint64_t n, int bits, void *scratch, cudaStream_t s,
-                     gpumem_triple *trip, uint32_t qbits) {
+static cudaError_t msd_run(uint64_t *keys, uint32_t *vals, NSpec ns, void *scratch, cudaStream_t s,
+                           gpumem_triple *trip, uint32_t qbits) {
     Out out{keys, vals, trip, qbits};
-    if (n == 0) return cudaSuccess;
-    if (bits < 1) bits = 1;
-    const int B = choose_b(n, bits);
-    const uint32_t nb = 1u << B;
-    const int shift = bits - B;
-    const uint32_t chunks = n_chunks(n);
-    const uint64_t cs = (n + chunks - 1) / chunks;
+    const uint64_t cap = ns.cap;
+    const uint32_t nb_max = 1u << choose_b(ns.dn ? (1ull << 62) : cap, ns.bits);  // device count: any B
+    const uint32_t chunks = n_chunks(cap);
     auto align = [](uintptr_t p) { return (p + 255) & ~uintptr_t(255); };
     uintptr_t c = align(reinterpret_cast<uintptr_t>(scratch));
     uint64_t *tk = reinterpret_cast<uint64_t *>(c);
-    c = align(c + n * 8);
+    c = align(c + cap * 8);
     uint32_t *tv = reinterpret_cast<uint32_t *>(c);
-    c = align(c + n * 4);
+    c = align(c + cap * 4);
     uint32_t *xv = vals ? vals : reinterpret_cast<uint32_t *>(c);  // value ping-pong of k_bs_big
-    c = align(c + n * 4);
+    c = align(c + cap * 4);
     uint32_t *counts = reinterpret_cast<uint32_t *>(c);  // [chunks][nb]
-    c = align(c + uint64_t(chunks) * nb * 4);
+    c = align(c + uint64_t(chunks) * nb_max * 4);
     uint32_t *totals = reinterpret_cast<uint32_t *>(c);
-    c = align(c + (nb + 1) * 4);
+    c = align(c + (nb_max + 1) * 4);
     uint32_t *offs = reinterpret_cast<uint32_t *>(c);
-    c = align(c + (nb + 1) * 4);
+    c = align(c + (nb_max + 1) * 4);
     uint32_t *big = reinterpret_cast<uint32_t *>(c);
-    c = align(c + nb * 4);
+    c = align(c + nb_max * 4);
     unsigned int *n_big = reinterpret_cast<unsigned int *>(c);
     cudaError_t e = cudaMemsetAsync(n_big, 0, 4, s);
     if (e != cudaSuccess) return e;
@@ -444,16 +472,96 @@ cudaError_t msd_sort(uint64_t *keys, uint32_t *vals, uint64_t n, int bits, void 
         cudaFuncSetAttribute(k_bs_local, cudaFuncAttributeMaxDynamicSharedMemorySize, int(sizeof(LocalSmem)));
         attr = true;
     }
-    k_bp_hist<<<chunks, kPT, nb * 4, s>>>(keys, n, cs, shift, nb, counts);
-    k_bp_colscan<<<(nb + 255) / 256, 256, 0, s>>>(counts, chunks, nb, totals);
-    k_bs_scan<<<1, 1024, 0, s>>>(totals, nb, offs);
-    k_bp_scatter<<<chunks, kPT, nb * 4, s>>>(keys, vals, n, cs, shift, nb, counts, offs, tk, tv);
-    const uint64_t segs = (n + kSeg - 1) / kSeg;
-    k_bs_local<<<unsigned(segs), kLT, sizeof(LocalSmem), s>>>(offs, nb, bits, tk, tv, out, big, n_big);
+    k_bp_hist<<<chunks, kPT, nb_max * 4, s>>>(keys, ns, counts);
+    k_bp_colscan<<<(nb_max + 255) / 256, 256, 0, s>>>(counts, chunks, ns, totals);
+    k_bs_scan<<<1, 1024, 0, s>>>(totals, ns, offs);
+    k_bp_scatter<<<chunks, kPT, nb_max * 4, s>>>(keys, vals, ns, counts, offs, tk, tv);
+    uint64_t segs = (cap + kSeg - 1) / kSeg;
+    if (ns.dn && segs > uint64_t(2 * num_sms())) segs = 2 * num_sms();  // blocks loop over the segments
+    k_bs_local<<<unsigned(segs ? segs : 1), kLT, sizeof(LocalSmem), s>>>(offs, ns, tk, tv, out, big, n_big);
     // oversized buckets: ping-pong with the input's range of the bucket (free: the scatter
     // consumed it and the local pass wrote only other buckets' ranges)
-    k_bs_big<<<num_sms(), kT, 0, s>>>(offs, big, n_big, tk, tv, keys, xv, shift, out);
+    k_bs_big<<<num_sms(), kT, 0, s>>>(offs, big, n_big, tk, tv, keys, xv, ns, out);
     note_launch(6);
+    return cudaGetLastError();
+}
+
+// Sorts n unique keys whose significant bits are the low `bits` (+ values, may be null).
+// Result: in place in (keys, vals), or as triples {key >> qbits, key & qmask, val} in
+// `trip` when trip != null. `scratch` >= msd_scratch_bytes(n).
+cudaError_t msd_sort(uint64_t *keys, uint32_t *vals, uint64_t n, int bits, void *scratch, cudaStream_t s,
+                     gpumem_triple *trip, uint32_t qbits) {
+    if (n == 0) return cudaSuccess;
+    return msd_run(keys, vals, NSpec{nullptr, n, bits < 1 ? 1 : bits, 0}, scratch, s, trip, qbits);
+}
+
+// The same with the key count in device memory: n = min(*d_n, cap); nothing is read on
+// the host, so the launch sequence is fixed (CUDA-graph capturable).
+cudaError_t msd_sort_dev(uint64_t *keys, uint32_t *vals, const unsigned long long *d_n, uint64_t cap, int bits,
+                         void *scratch, cudaStream_t s, gpumem_triple *trip, uint32_t qbits) {
+    if (cap == 0) return cudaSuccess;
+    return msd_run(keys, vals, NSpec{d_n, cap, bits < 1 ? 1 : bits, 0}, scratch, s, trip, qbits);
+}
+
+// offs[b] = the first slot whose key prefix (key >> shift) is >= b, b in [0, nb] (keys
+// already ordered by that prefix): one binary search per bucket.
+__global__ void __launch_bounds__(256) k_prefix_bounds(const uint64_t *__restrict__ keys, NSpec ns, int shift,
+                                                       uint32_t nb, uint32_t *__restrict__ offs) {
+    const uint64_t n = ns.n();
+    for (uint32_t b = blockIdx.x * 256 + threadIdx.x; b <= nb; b += gridDim.x * 256) {
+        uint64_t lo = 0, hi = n;
+        while (lo < hi) {
+            const uint64_t mid = (lo + hi) >> 1;
+            if ((keys[mid] >> shift) < b) lo = mid + 1; else hi = mid;
+        }
+        offs[b] = uint32_t(lo);
+    }
+}
+
+size_t hybrid_scratch_bytes() { return radix_scratch_bytes(0) + (1u << 16) * 8 + 4096; }
+
+// Hybrid sort for large outputs: two stable LSD passes (8-bit
+// digits, radix.cu: coalesced tile-reordered scatter) order the keys by their top 16
+// bits; each run of equal prefix (65536 buckets, ~200 keys each at 1.3e7 MEMs) is then
+// a contiguous segment sorted in shared memory by k_bs_local and written as triples.
+// Three passes over the data instead of the LSD sort's seven, and no 16K-way scatter.
+cudaError_t hybrid_sort_triples(uint64_t *keys, uint32_t *vals, uint64_t *k1, uint32_t *v1,
+                                const unsigned long long *d_n, uint64_t cap, int bits, void *scratch,
+                                cudaStream_t s, gpumem_triple *trip, uint32_t qbits) {
+    if (cap == 0) return cudaSuccess;
+    if (bits < 1) bits = 1;
+    const int T = bits < 16 ? bits : 16;
+    const int lo = bits - T;
+    const uint32_t nb = 1u << T;
+    auto align = [](uintptr_t p) { return (p + 255) & ~uintptr_t(255); };
+    uintptr_t c = align(reinterpret_cast<uintptr_t>(scratch));
+    void *rscratch = reinterpret_cast<void *>(c);
+    c = align(c + radix_scratch_bytes(0));
+    uint32_t *offs = reinterpret_cast<uint32_t *>(c);
+    c = align(c + (nb + 1) * 4);
+    uint32_t *big = reinterpret_cast<uint32_t *>(c);
+    c = align(c + nb * 4);
+    unsigned int *n_big = reinterpret_cast<unsigned int *>(c);
+    bool alt = false;
+    cudaError_t e = radix_sort_u64(keys, vals, k1, v1, cap, bits, rscratch, s, &alt, lo, d_n);
+    if (e != cudaSuccess) return e;
+    uint64_t *tk = alt ? k1 : keys, *xk = alt ? keys : k1;
+    uint32_t *tv = alt ? v1 : vals, *xv = alt ? vals : v1;
+    const NSpec ns{d_n, cap, bits, T};
+    e = cudaMemsetAsync(n_big, 0, 4, s);
+    if (e != cudaSuccess) return e;
+    static bool attr = false;
+    if (!attr) {
+        cudaFuncSetAttribute(k_bs_local, cudaFuncAttributeMaxDynamicSharedMemorySize, int(sizeof(LocalSmem)));
+        attr = true;
+    }
+    k_prefix_bounds<<<(nb + 256) / 256, 256, 0, s>>>(tk, ns, lo, nb, offs);
+    uint64_t segs = (cap + kSeg - 1) / kSeg;
+    if (segs > uint64_t(2 * num_sms())) segs = 2 * num_sms();  // blocks loop over the segments
+    Out out{keys, vals, trip, qbits};
+    k_bs_local<<<unsigned(segs), kLT, sizeof(LocalSmem), s>>>(offs, ns, tk, tv, out, big, n_big);
+    k_bs_big<<<num_sms(), kT, 0, s>>>(offs, big, n_big, tk, tv, xk, xv, ns, out);
+    note_launch(3);
     return cudaGetLastError();
 }
 

@@ -75,10 +75,24 @@ __device__ __forceinline__ unsigned match_digit(uint32_t d, bool valid, int bits
     return peers;
 }
 
-// Chunk c of a pass: tiles [c * tpc, min((c + 1) * tpc, tiles)).
+// Chunk c of a pass: tiles [c * tpc, min((c + 1) * tpc, tiles)). With a device-resident
+// count (dn != null: the sort inside a captured pipeline) n is the capacity on the host
+// and live() re-derives n, tiles and tiles-per-chunk from min(*dn, capacity) on the
+// device; the chunk count (the grid) stays fixed and trailing chunks may be empty.
 struct Chunking {
     uint64_t n, tiles, tpc;
     uint32_t chunks;
+    const unsigned long long *dn;
+    __device__ Chunking live(uint64_t tile) const {
+        if (!dn) return *this;
+        Chunking c = *this;
+        const unsigned long long x = *dn;
+        c.n = x < n ? x : n;
+        c.tiles = (c.n + tile - 1) / tile;
+        c.tpc = (c.tiles + chunks - 1) / chunks;
+        if (!c.tpc) c.tpc = 1;
+        return c;
+    }
     __host__ __device__ uint64_t begin(uint32_t c, uint64_t tile) const {
         const uint64_t b = uint64_t(c) * tpc * tile;
         return b < n ? b : n;
@@ -90,7 +104,7 @@ struct Chunking {
 };
 
 template <class K, int RB>
-__global__ void __launch_bounds__(kT) k_chunk_hist(const K *__restrict__ keys, Chunking ch, int shift, int bits,
+__global__ void __launch_bounds__(kT) k_chunk_hist(const K *__restrict__ keys, Chunking ch0, int shift, int bits,
                                                    uint32_t *__restrict__ counts, uint32_t *__restrict__ totals) {
     constexpr int kBins = 1 << RB;
     constexpr int DPT = kBins / kT;
@@ -100,6 +114,7 @@ __global__ void __launch_bounds__(kT) k_chunk_hist(const K *__restrict__ keys, C
     for (int i = tid; i < kWarps * kBins; i += kT) (&h[0][0])[i] = 0;
     __syncthreads();
     const uint32_t c = blockIdx.x;
+    const Chunking ch = ch0.live(tile_items<K>());
     const uint64_t b = ch.begin(c, tile_items<K>()), e = ch.end(c, tile_items<K>());
     for (uint64_t i = b + tid; i < e; i += kT) atomicAdd(&h[w][uint32_t(keys[i] >> shift) & dmask], 1u);
     __syncthreads();
@@ -205,7 +220,7 @@ __device__ __forceinline__ void mbar_wait(unsigned long long *bar, uint32_t pari
 
 template <class K, class V, int RB>
 __global__ void __launch_bounds__(kST, GM_RADIX_MINB) k_scatter(const K *__restrict__ kin, const V *__restrict__ vin,
-                                                  K *__restrict__ kout, V *__restrict__ vout, Chunking ch,
+                                                  K *__restrict__ kout, V *__restrict__ vout, Chunking ch0,
                                                   int shift, int bits, const uint32_t *__restrict__ offs) {
     constexpr int kBins = 1 << RB;
     constexpr int DPT = (kBins + kST - 1) / kST;  // digits owned per thread: tid, tid + kST, ... (< kBins)
@@ -216,6 +231,7 @@ __global__ void __launch_bounds__(kST, GM_RADIX_MINB) k_scatter(const K *__restr
     const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
     const uint32_t dmask = (1u << bits) - 1;
     const uint32_t c = blockIdx.x;
+    const Chunking ch = ch0.live(kTile);
     const uint64_t cb = ch.begin(c, kTile), ce = ch.end(c, kTile);
     const uint32_t n_t = uint32_t((ce - cb + kTile - 1) / kTile);
     const uint32_t n_full = uint32_t((ce - cb) / kTile);  // tiles moved by TMA; a ragged tail is loaded directly
@@ -381,7 +397,7 @@ constexpr int kMaxChunks = 148 * 8;  // >= SMs x resident scatter CTAs
 
 template <class K, int RB>
 cudaError_t radix_sort_rb(K *k0, uint32_t *v0, K *k1, uint32_t *v1, uint64_t n, int lo, int bits, void *scratch,
-                          cudaStream_t s, bool *in_alt) {
+                          cudaStream_t s, bool *in_alt, const unsigned long long *dn) {
     constexpr int kBins = 1 << RB;
     const int passes = (bits - lo + RB - 1) / RB;
     const size_t smem = sizeof(ScatterSmem<K, uint32_t, RB>);
@@ -399,6 +415,7 @@ cudaError_t radix_sort_rb(K *k0, uint32_t *v0, K *k1, uint32_t *v1, uint64_t n, 
         if (grid_cap > kMaxChunks) grid_cap = kMaxChunks;
     }
     Chunking ch;
+    ch.dn = dn;
     ch.n = n;
     ch.tiles = (n + tile_items<K>() - 1) / tile_items<K>();
     ch.chunks = uint32_t(ch.tiles < uint64_t(grid_cap) ? ch.tiles : uint64_t(grid_cap));
@@ -428,16 +445,16 @@ cudaError_t radix_sort_rb(K *k0, uint32_t *v0, K *k1, uint32_t *v1, uint64_t n, 
 
 template <class K>
 cudaError_t radix_sort(K *k0, uint32_t *v0, K *k1, uint32_t *v1, uint64_t n, int lo, int bits, void *scratch,
-                       cudaStream_t s, bool *in_alt) {
+                       cudaStream_t s, bool *in_alt, const unsigned long long *dn = nullptr) {
     *in_alt = false;
     if (bits > int(8 * sizeof(K))) bits = int(8 * sizeof(K));
-    if (n <= 1 || bits <= lo) return cudaSuccess;
+    if ((n <= 1 && !dn) || n == 0 || bits <= lo) return cudaSuccess;
     if (!scratch) return cudaErrorInvalidValue;
     if (uint64_t(n) >= (uint64_t(1) << 32)) return cudaErrorInvalidValue;  // 32-bit offsets
     switch (pick_digit_bits(bits - lo)) {
-        case 9: return radix_sort_rb<K, 9>(k0, v0, k1, v1, n, lo, bits, scratch, s, in_alt);
-        case 10: return radix_sort_rb<K, 10>(k0, v0, k1, v1, n, lo, bits, scratch, s, in_alt);
-        default: return radix_sort_rb<K, 8>(k0, v0, k1, v1, n, lo, bits, scratch, s, in_alt);
+        case 9: return radix_sort_rb<K, 9>(k0, v0, k1, v1, n, lo, bits, scratch, s, in_alt, dn);
+        case 10: return radix_sort_rb<K, 10>(k0, v0, k1, v1, n, lo, bits, scratch, s, in_alt, dn);
+        default: return radix_sort_rb<K, 8>(k0, v0, k1, v1, n, lo, bits, scratch, s, in_alt, dn);
     }
 }
 
@@ -454,8 +471,8 @@ cudaError_t radix_sort_u32(uint32_t *k0, uint32_t *v0, uint32_t *k1, uint32_t *v
 }
 
 cudaError_t radix_sort_u64(uint64_t *k0, uint32_t *v0, uint64_t *k1, uint32_t *v1, uint64_t n, int bits,
-                           void *scratch, cudaStream_t s, bool *in_alt) {
-    return radix_sort<uint64_t>(k0, v0, k1, v1, n, 0, bits, scratch, s, in_alt);
+                           void *scratch, cudaStream_t s, bool *in_alt, int lo, const unsigned long long *dn) {
+    return radix_sort<uint64_t>(k0, v0, k1, v1, n, lo, bits, scratch, s, in_alt, dn);
 }
 
 }  // namespace gm

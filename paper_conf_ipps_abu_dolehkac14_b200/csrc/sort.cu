@@ -10,8 +10,13 @@ constexpr int kT = 256;
 
 __global__ void __launch_bounds__(kT) k_keys_to_triples(const uint64_t *__restrict__ keys,
                                                         const uint32_t *__restrict__ lens, uint64_t n,
-                                                        uint32_t qbits, gpumem_triple *__restrict__ out) {
+                                                        uint32_t qbits, gpumem_triple *__restrict__ out,
+                                                        const unsigned long long *__restrict__ dn) {
     const uint64_t i = uint64_t(blockIdx.x) * kT + threadIdx.x;
+    if (dn) {  // device-resident count, n is the capacity
+        const unsigned long long x = *dn;
+        if (x < n) n = x;
+    }
     if (i >= n) return;
     const uint64_t k = keys[i];
     const uint64_t qmask = (1ull << qbits) - 1;
@@ -64,9 +69,9 @@ cudaError_t launch_split_keys(const uint64_t *keys, uint64_t n, uint32_t *codes,
 }
 
 cudaError_t launch_keys_to_triples(const uint64_t *keys, const uint32_t *lens, uint64_t n, uint32_t qbits,
-                                   gpumem_triple *out, cudaStream_t s) {
+                                   gpumem_triple *out, cudaStream_t s, const unsigned long long *dn) {
     if (!n) return cudaSuccess;
-    k_keys_to_triples<<<unsigned((n + kT - 1) / kT), kT, 0, s>>>(keys, lens, n, qbits, out);
+    k_keys_to_triples<<<unsigned((n + kT - 1) / kT), kT, 0, s>>>(keys, lens, n, qbits, out, dn);
     note_launch();
     return cudaGetLastError();
 }

@@ -68,3 +68,45 @@ def find_mems_sharded(R_dev: torch.Tensor, Q_dev: torch.Tensor, min_len: int, se
     if rank == 0:
         return gm.merge_sorted(runs), local
     return None, local
+
+
+class ShardedPipeline:
+    """This rank's share of the whole step as a CUDA-graph pipeline (gpumem_pipeline_*):
+    pack, index, find over the rank's MEM-start range [a_g, b_g) and the output sort in
+    one graph launch; `finish` checks the result and, for world > 1, gathers the sorted
+    runs to rank 0 and merges them there (the only exchange, as in find_mems_sharded)."""
+
+    def __init__(self, n_r: int, n_q: int, min_len: int, seed_len: int, group=None):
+        from . import gpumem as gm
+        self.gm = gm
+        self.group = group
+        self.world = dist.get_world_size(group) if dist.is_initialized() else 1
+        self.rank = dist.get_rank(group) if dist.is_initialized() else 0
+        self.q_range = shard_range(n_q, self.rank, self.world)
+        self.pl = gm.Pipeline(n_r, n_q, seed_len, min_len, self.q_range)
+        self.merged = None
+
+    def run(self, R_dev: torch.Tensor, Q_dev: torch.Tensor):
+        """Async: one graph launch on the current stream's pipeline."""
+        if self.merged is not None:
+            self.merged.free()
+            self.merged = None
+        self.pl.run(R_dev, Q_dev)
+
+    def finish(self):
+        """Synchronise, check (alphabet, capacity fallback), gather + merge for world > 1.
+        Returns the number of MEMs on rank 0 (this rank's count when world == 1), None
+        on other ranks."""
+        n = self.pl.result()
+        if self.world == 1:
+            return n
+        runs = gather_to_root(self.pl.view_u32().view(torch.int32), self.group)
+        if self.rank == 0:
+            self.merged = self.gm.merge_sorted(runs)
+            return len(self.merged)
+        return None
+
+    def free(self):
+        if self.merged is not None:
+            self.merged.free()
+        self.pl.free()

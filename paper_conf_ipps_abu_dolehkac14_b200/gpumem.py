@@ -47,6 +47,12 @@ SYMBOLS = {
     "gpumem_mems_stats": (ctypes.c_int, [_vp, _vp]),
     "gpumem_mums": (ctypes.c_int, [_vp, _vp, _P(_vp)]),
     "gpumem_merge_sorted": (ctypes.c_int, [_P(_vp), _P(_c_u64), ctypes.c_int, _vp, _P(_vp)]),
+    "gpumem_pipeline_create": (ctypes.c_int, [_c_u64, _c_u64, _c_u32, _c_u32, _c_u64, _c_u64, _vp, _P(_vp)]),
+    "gpumem_pipeline_run": (ctypes.c_int, [_vp, _vp, _vp]),
+    "gpumem_pipeline_result": (ctypes.c_int, [_vp, _P(_vp), _P(_c_u64)]),
+    "gpumem_pipeline_stats": (ctypes.c_int, [_vp, _vp]),
+    "gpumem_pipeline_profile": (ctypes.c_int, [_vp, _P(ctypes.c_char_p), _P(ctypes.c_double), _P(_c_u64),
+                                               ctypes.c_int]),
     "gpumem_free": (None, [_vp]),
     "gpumem_trim": (ctypes.c_int, []),
     "gpumem_last_error": (ctypes.c_char_p, []),
@@ -268,6 +274,69 @@ def merge_sorted(runs, stream=None) -> Mems:
     h = _vp()
     _check(_lib.gpumem_merge_sorted(ptrs, cnts, len(runs), _stream(stream), ctypes.byref(h)))
     return Mems(h.value, list(runs))
+
+
+class Pipeline(_Handle):
+    """The whole path for fixed sizes as one CUDA graph (gpumem_pipeline_*).
+
+        pl = gm.Pipeline(len(R), len(Q), seed_len=13, min_len=100)
+        pl.run(R_dev, Q_dev)      # async: one graph launch (captured on the first call)
+        n = pl.result()           # sync; MEM count (same set as find_mems)
+        pl.view_u32()             # (n, 3) uint32 CUDA view, valid until the next run
+    """
+
+    def __init__(self, r_len, q_len, seed_len, min_len, q_range=None, stream=None):
+        qb, qe = (0, (1 << 64) - 1) if q_range is None else (int(q_range[0]), int(q_range[1]))
+        h = _vp()
+        _check(_lib.gpumem_pipeline_create(int(r_len), int(q_len), seed_len, min_len, qb, qe, _stream(stream),
+                                           ctypes.byref(h)))
+        super().__init__(h.value)
+        self._inputs = None
+        self._ptr, self._n = None, 0
+
+    def run(self, R_dev, Q_dev):
+        """R_dev, Q_dev: uint8 CUDA tensors of the sizes given at creation (kept alive
+        until the next run)."""
+        import torch
+        for x in (R_dev, Q_dev):
+            if not (isinstance(x, torch.Tensor) and x.is_cuda and x.dtype == torch.uint8 and x.is_contiguous()):
+                raise TypeError("pipeline inputs must be contiguous uint8 CUDA tensors")
+        self._inputs = (R_dev, Q_dev)
+        self._ptr = None
+        _check(_lib.gpumem_pipeline_run(self.handle, _vp(R_dev.data_ptr()), _vp(Q_dev.data_ptr())))
+
+    def result(self):
+        ptr, n = _vp(), _c_u64()
+        _check(_lib.gpumem_pipeline_result(self.handle, ctypes.byref(ptr), ctypes.byref(n)))
+        self._ptr, self._n = ptr.value, n.value
+        return self._n
+
+    def __len__(self):
+        if self._ptr is None:
+            self.result()
+        return self._n
+
+    def view_u32(self):
+        """(N, 3) uint32 CUDA view of the last result (borrowed; valid until the next run)."""
+        if self._ptr is None:
+            self.result()
+        return _device_view(self._ptr, (self._n, 3), "<u4", self)
+
+    def numpy(self):
+        return self.view_u32().cpu().numpy()
+
+    def stats(self):
+        s = FindStats()
+        _check(_lib.gpumem_pipeline_stats(self.handle, ctypes.byref(s)))
+        return s.as_dict()
+
+    def profile(self, max_stages=32):
+        """Per-stage device ms of the last completed run: {name: (ms, launches)}."""
+        names = (ctypes.c_char_p * max_stages)()
+        ms = (ctypes.c_double * max_stages)()
+        nl = (_c_u64 * max_stages)()
+        n = _lib.gpumem_pipeline_profile(self.handle, names, ms, nl, max_stages)
+        return {names[i].decode(): (ms[i], nl[i]) for i in range(n)}
 
 
 def set_option(name: str, value: int):

@@ -177,15 +177,15 @@ def test_homopolymer_closed_form(n, m):
         assert np.array_equal(got, want), (n, m, L, ls)
 
 
-@pytest.mark.parametrize("impl", [0, 1, 2, 3])
+@pytest.mark.parametrize("impl", [0, 1, 2, 3, 4])
 @pytest.mark.parametrize("n,m,L", [(300, 20000, 20), (20000, 300, 20), (9000, 9000, 8000), (2, 50000, 1)])
 def test_sort_skewed_buckets(impl, n, m, L):
     """Output sort on skewed key sets: most MEMs share r = 0 (one MSD bucket far past
     shared memory -> the global LSD fallback) or q = 0 (many small buckets), checked
     against the homopolymer closed form, under every output sort path (auto, LSD, MSD,
-    single-launch)."""
-    gpumem.set_option("sort_impl", impl % 3)
-    gpumem.set_option("small_sort", int(impl == 3))
+    hybrid, single-launch)."""
+    gpumem.set_option("sort_impl", impl % 4)
+    gpumem.set_option("small_sort", int(impl == 4))
     want = np.array(pyoracle.homopolymer(n, m, L), dtype=np.uint32).reshape(-1, 3)
     got = gpu_mems("A" * n, "A" * m, L, 1 if L < 13 else 13)
     assert np.array_equal(got, want), (impl, n, m, L)
@@ -233,7 +233,7 @@ def test_overflow_retry_grid_spill_and_bitmap_invariance():
     base = gpu_mems(P.R, P.Q, P.L, P.ls)
     assert np.array_equal(base, want)
     for opt, vals in (("out_capacity", [1, 100]), ("find_grid", [1, 3, 148]), ("find_spill", [1, 2, 10**9]),
-                      ("use_bitmap", [0]), ("static_lb", [1]), ("sort_impl", [1, 2]), ("index_msd", [1]), ("small_sort", [1]),
+                      ("use_bitmap", [0]), ("static_lb", [1]), ("sort_impl", [1, 2, 3]), ("index_msd", [1]), ("small_sort", [1]),
                       ("rank_sectors", [0, 1]), ("rec8", [0, 1]), ("index_fused", [1]),
                       ("radix_bits", [8, 9, 10])):
         for v in vals:
@@ -308,6 +308,14 @@ def test_full_size_c4_c5(c4_full, L):
     want = oracle.mems(P.R, P.Q, L, 13)
     got = gpu_mems(P.R, P.Q, L, 13)
     assert np.array_equal(got, want)
+    # the launch configuration bench.py times: the CUDA-graph pipeline, relaunched
+    Rt, Qt = torch.from_numpy(P.R).cuda(), torch.from_numpy(P.Q).cuda()
+    pl = gpumem.Pipeline(len(P.R), len(P.Q), 13, L)
+    for _ in range(2):
+        pl.run(Rt, Qt)
+        assert pl.result() == len(want)
+        assert np.array_equal(pl.numpy(), want)
+    pl.free()
 
 
 # ------------------------------------------------------------------ NEXT rows

@@ -1,0 +1,133 @@
+"""GPU parity of the CUDA-graph pipeline (gpumem_pipeline_*, the launch configuration
+bench.py times): the same kernels as pack + index_build + find_mems, captured once
+and replayed, with the output sort sized by the device-resident MEM count. Checked
+bit-exact against the CPU oracle (and brute force on tiny inputs), across relaunches,
+recaptures, q ranges, the overflow fallback and alphabet errors."""
+import numpy as np
+import pytest
+
+import oracle
+from paper_conf_ipps_abu_dolehkac14_b200 import synth
+from tests import invariants
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+if not torch.cuda.is_available():  # collected on CPU boxes, skipped there
+    pytest.skip("needs a CUDA device", allow_module_level=True)
+
+from paper_conf_ipps_abu_dolehkac14_b200 import gpumem  # noqa: E402
+
+
+@pytest.fixture(autouse=True)
+def _default_options():
+    yield
+    gpumem.set_option("out_capacity", 0)
+    gpumem.set_option("sort_impl", 0)
+
+
+def _dev(x):
+    b = x.tobytes() if isinstance(x, np.ndarray) else (x.encode() if isinstance(x, str) else bytes(x))
+    if not b:
+        return torch.empty(0, dtype=torch.uint8, device="cuda")
+    return torch.from_numpy(np.frombuffer(b, dtype=np.uint8).copy()).cuda()
+
+
+def pipe_mems(R, Q, L, ls, q_range=None, runs=1):
+    Rt, Qt = _dev(R), _dev(Q)
+    pl = gpumem.Pipeline(Rt.numel(), Qt.numel(), ls, L, q_range)
+    outs = []
+    for _ in range(runs):
+        pl.run(Rt, Qt)
+        pl.result()
+        outs.append(pl.numpy())
+    for o in outs[1:]:
+        assert np.array_equal(o, outs[0])  # graph relaunch: identical
+    st = pl.stats()
+    pl.free()
+    return outs[0], st
+
+
+@pytest.mark.parametrize("cfg,scale", [("c1", 1.0), ("c2", 0.3), ("c3", 0.05), ("c4", 0.02), ("c5_l20", 0.02),
+                                       ("c5_l300", 0.02)])
+def test_pipeline_config_parity(cfg, scale):
+    P = synth.make_pair(cfg, scale=scale)
+    want = oracle.mems(P.R, P.Q, P.L, P.ls)
+    got, st = pipe_mems(P.R, P.Q, P.L, P.ls, runs=3)
+    assert np.array_equal(got, want)
+    assert st["mems"] == len(want) and st["attempts"] == 1
+    invariants.check(P.R, P.Q, P.L, got)
+
+
+@pytest.mark.parametrize("impl", [0, 1, 2, 3])
+@pytest.mark.parametrize("n,m,L", [(300, 20000, 20), (20000, 300, 20), (2, 50000, 1)])
+def test_pipeline_sort_skewed(impl, n, m, L):
+    """Device-count output sorts (auto, LSD, MSD, hybrid) on skewed keys: one r with 20 000 MEMs
+    (a prefix run far past shared memory -> the global fallback), or many small runs."""
+    from oracle import pyoracle
+    gpumem.set_option("sort_impl", impl)
+    want = np.array(pyoracle.homopolymer(n, m, L), dtype=np.uint32).reshape(-1, 3)
+    got, _ = pipe_mems("A" * n, "A" * m, L, 1 if L < 13 else 13)
+    assert np.array_equal(got, want)
+
+
+def test_pipeline_random_tiny_vs_brute_force():
+    rng = np.random.default_rng(7)
+    alph = [b"A", b"AC", b"ACGT"]
+    for trial in range(40):
+        R, Q = synth.random_pair(rng, int(rng.integers(1, 300)), int(rng.integers(1, 300)), alph[trial % 3])
+        L = int(rng.integers(1, 30))
+        ls = int(rng.integers(1, min(L, 15) + 1))
+        got, _ = pipe_mems(R, Q, L, ls)
+        assert np.array_equal(got, oracle.brute(R, Q, L)), trial
+
+
+def test_pipeline_qrange_and_recapture():
+    P = synth.make_pair("c2", scale=0.05)
+    n = len(P.Q)
+    for a, b in ((0, n // 3), (n // 3, n), (n // 2, n // 2)):
+        got, _ = pipe_mems(P.R, P.Q, P.L, P.ls, q_range=(a, b))
+        assert np.array_equal(got, oracle.mems(P.R, P.Q, P.L, P.ls, 0, a, b)), (a, b)
+    # new input buffers (other contents, same sizes) -> recapture on the same pipeline
+    Rt, Qt = _dev(P.R), _dev(P.Q)
+    pl = gpumem.Pipeline(len(P.R), n, P.ls, P.L)
+    pl.run(Rt, Qt)
+    first = (pl.result(), pl.numpy())
+    Q2 = P.Q.copy()
+    Q2[: n // 2] = P.R[: n // 2]
+    Qt2 = _dev(Q2)
+    pl.run(Rt, Qt2)
+    pl.result()
+    assert np.array_equal(pl.numpy(), oracle.mems(P.R, Q2, P.L, P.ls))
+    pl.run(Rt, Qt)
+    assert pl.result() == first[0] and np.array_equal(pl.numpy(), first[1])
+    prof = pl.profile()
+    assert {"pack", "find", "sort"} <= set(prof) and all(v[0] > 0 for k, v in prof.items() if k in ("find", "sort"))
+    pl.free()
+
+
+def test_pipeline_overflow_fallback():
+    P = synth.make_pair("c1")
+    want = oracle.mems(P.R, P.Q, P.L, P.ls)
+    gpumem.set_option("out_capacity", 100)  # fewer than the MEMs: the graph's output overflows
+    got, st = pipe_mems(P.R, P.Q, P.L, P.ls, runs=2)
+    assert np.array_equal(got, want)
+    assert st["attempts"] >= 2
+
+
+def test_pipeline_edges_and_alphabet():
+    R = synth.make_pair("c1", scale=0.2).R.tobytes()
+    got, _ = pipe_mems(R, R, 20, 10)
+    assert (0, 0, len(R)) in {tuple(t) for t in got.tolist()}
+    assert np.array_equal(got, oracle.mems(R, R, 20, 10))
+    assert len(pipe_mems(R, b"ACGT" * 4, 20, 10)[0]) == 0
+    assert len(pipe_mems(R, b"", 20, 10)[0]) == 0
+    bad = bytearray(R[:5000])
+    bad[1234] = ord("N")
+    Rt, Qt = _dev(bytes(bad)), _dev(R[:3000])
+    pl = gpumem.Pipeline(Rt.numel(), Qt.numel(), 10, 20)
+    pl.run(Rt, Qt)
+    with pytest.raises(gpumem.GpumemError) as ei:
+        pl.result()
+    assert ei.value.name == "ERR_ALPHABET" and "1234" in str(ei.value)
+    pl.free()
