@@ -52,7 +52,7 @@ typedef enum {
 } gpumem_status;
 
 typedef struct gpumem_seq gpumem_seq;     /* 2-bit packed sequence resident on one device        */
-typedef struct gpumem_index gpumem_index; /* ptrs[4^ls+1], locs[n_locs], occupancy bitmap; refs R  */
+typedef struct gpumem_index gpumem_index; /* locs[n_locs] + lookup directory (ptrs on demand); refs R */
 typedef struct gpumem_mems gpumem_mems;   /* MEM set sorted by (r, q), device-resident            */
 typedef struct gpumem_pipeline gpumem_pipeline; /* the whole path captured as one CUDA graph        */
 
@@ -95,10 +95,13 @@ gpumem_status gpumem_seq_info(const gpumem_seq *s, uint64_t *n_bases, const uint
  * gpumem_index_build -- GPUMEM's lightweight index of R (Sec. III-A, Alg. 1 :102-106).
  *  seed_len (ls) in [1, 15], min_len (L) >= ls, step = L - ls + 1 (the maximum allowed by
  *  Eq. 1, :88-90). Indexed locations: p = 0, step, 2*step, ... <= |R| - ls (reading R6).
- *  Result: ptrs (4^ls + 1 uint32, ptrs[s] = first slot of seed s, ptrs[4^ls] = n_locs, :84)
- *  and locs (n_locs uint32, sorted ascending inside each seed, Alg. 1 step 4), plus a
- *  4^ls-bit occupancy bitmap used by the lookup. ptrs alone takes 4*(4^ls+1) bytes
- *  (268 MB at ls = 13). The index references R: R must outlive it. Async.
+ *  Result: locs (n_locs uint32, sorted ascending inside each seed, Alg. 1 step 4) and the
+ *  lookup directory: per 32 seeds an occupancy/rank word (or rank sector), plus the
+ *  compact table {first slot, count} of the occupied seeds -- an exact, compressed form
+ *  of the paper's ptrs (4^ls + 1 uint32, ptrs[s] = first slot of seed s, ptrs[4^ls] =
+ *  n_locs, :84; 268 MB at ls = 13), which is expanded from it only on demand
+ *  (gpumem_index_view, or find with option use_bitmap = 0). The index references R: R
+ *  must outlive it. Async.
  */
 gpumem_status gpumem_index_build(const gpumem_seq *R, uint32_t seed_len, uint32_t min_len,
                                  void *cuda_stream, gpumem_index **out);
@@ -120,7 +123,8 @@ gpumem_status gpumem_index_build_range(const gpumem_seq *R, uint32_t seed_len, u
                                        uint64_t r_begin, uint64_t r_end, void *cuda_stream,
                                        gpumem_index **out);
 
-/* Borrowed device pointers to ptrs (4^ls + 1 entries) and locs (n_locs entries). */
+/* Borrowed device pointers to ptrs (4^ls + 1 entries) and locs (n_locs entries). The first
+ * request for ptrs expands it on the index's stream and synchronises that stream. */
 gpumem_status gpumem_index_view(const gpumem_index *idx, const uint32_t **dev_ptrs,
                                 const uint32_t **dev_locs, uint64_t *n_locs);
 

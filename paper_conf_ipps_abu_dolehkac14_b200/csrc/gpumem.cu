@@ -762,7 +762,7 @@ static gpumem_status index_build_impl(const gpumem_seq *R, uint32_t ls, uint32_t
     const uint64_t k1 = k1_band < k_all ? k1_band : k_all;
     const uint64_t n_locs = k1 > k0 ? k1 - k0 : 0;
     Scratch sc(s);
-    auto *ptrs = static_cast<uint32_t *>(sc.get((nb + 1) * 4));
+    uint32_t *ptrs = nullptr;  // the dense ptrs table is expanded on demand (index_ptrs)
     // lookup directory: rank sectors when the compact table {first, count} (<= 8 B per
     // sampled seed) would not stay in L2 next to the rest, else the smaller rank words
     int l2 = 0;
@@ -776,7 +776,7 @@ static gpumem_status index_build_impl(const gpumem_seq *R, uint32_t ls, uint32_t
     auto *buckets = static_cast<uint2 *>(sc.get(max_occ * sizeof(uint2)));
     void *fill_scratch = ws_get(kWsFill, ptrs_fill_scratch_bytes(ls), s);
     auto *locs0 = static_cast<uint32_t *>(sc.get((n_locs ? n_locs : 1) * 4));
-    if (!ptrs || !(rsect || rankw) || !buckets || !fill_scratch || !locs0) return GPUMEM_ERR_NOMEM;
+    if (!(rsect || rankw) || !buckets || !fill_scratch || !locs0) return GPUMEM_ERR_NOMEM;
     uint32_t *locs = locs0;
     const uint32_t *codes_sorted = nullptr;
     // 8-byte seed records when the left extension is capped at <= 8 bases (step <= 8)
@@ -870,7 +870,6 @@ static gpumem_status index_build_impl(const gpumem_seq *R, uint32_t ls, uint32_t
         Stage g("index.recs", s);
         CK(launch_seed_recs(R->words, ls, locs, n_locs, recs, rec8, s), "seed records");
     }
-    sc.keep(ptrs);
     if (rankw) sc.keep(rankw);
     if (rsect) sc.keep(rsect);
     sc.keep(buckets);
@@ -891,9 +890,38 @@ gpumem_status gpumem_index_build(const gpumem_seq *R, uint32_t ls, uint32_t L, v
     return gpumem_index_build_step(R, ls, L, L - ls + 1, cuda_stream, out);
 }
 
+// The paper's dense ptrs[4^ls + 1], expanded once from the rank directory
+// and the compact table on first use (index_view, or find with use_bitmap = 0), on
+// stream s. The fast lookup never reads it, so the index build does not write it.
+static std::mutex g_ptrs_mu;
+static gpumem_status index_ptrs(const gpumem_index *cidx, cudaStream_t s) {
+    auto *idx = const_cast<gpumem_index *>(cidx);
+    std::lock_guard<std::mutex> g(g_ptrs_mu);
+    if (idx->ptrs) return GPUMEM_OK;
+    const uint64_t nb = 1ull << (2 * idx->ls);
+    auto *p = static_cast<uint32_t *>(dalloc((nb + 1) * 4, s));
+    if (!p) return GPUMEM_ERR_NOMEM;
+    const cudaError_t e = launch_ptrs_expand(idx->rankw, idx->rsect, idx->buckets, idx->ls, idx->n_locs, p, s);
+    if (e != cudaSuccess) {
+        dfree(p, s);
+        return cuda_fail(e, "ptrs expand");
+    }
+    if (s != idx->stream && !(t_cap && t_cap->mode == 2)) {  // freed on the index's stream later
+        const cudaError_t e2 = cudaStreamSynchronize(s);
+        if (e2 != cudaSuccess) return cuda_fail(e2, "ptrs expand");
+    }
+    idx->ptrs = p;
+    return GPUMEM_OK;
+}
+
 gpumem_status gpumem_index_view(const gpumem_index *idx, const uint32_t **dev_ptrs, const uint32_t **dev_locs,
                                 uint64_t *n_locs) {
     if (!idx || idx->magic != kMagicIdx) return fail(GPUMEM_ERR_ARG, "not a gpumem_index");
+    if (dev_ptrs) {
+        gpumem_status st = index_ptrs(idx, idx->stream);
+        if (st) return st;
+        CK(cudaStreamSynchronize(idx->stream), "ptrs expand");
+    }
     if (dev_ptrs) *dev_ptrs = idx->ptrs;
     if (dev_locs) *dev_locs = idx->locs;
     if (n_locs) *n_locs = idx->n_locs;
@@ -966,6 +994,10 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
     P.Q = Q->words;
     P.nQ = nQ;
     P.nQw = Q->n_words;
+    if (!g_opt.use_bitmap) {  // the paper's lookup reads the dense ptrs
+        st = index_ptrs(idx, s);
+        if (st) return st;
+    }
     P.ptrs = idx->ptrs;
     P.recs = idx->recs;
     P.rec8 = idx->rec8;

@@ -28,6 +28,8 @@
 // Algorithmic bytes: n_locs * (8 B codes/locs written + 16 B per radix pass read+
 // write) + 4 * (4^ls + 1) B ptrs written + 4^ls / 2 B rank sectors + 8 B per
 // occupied seed.
+#include <algorithm>
+
 #include "internal.h"
 #include "device.cuh"
 
@@ -192,7 +194,10 @@ __global__ void __launch_bounds__(kFillThreads) k_ptrs_fill(const uint32_t *__re
         else rankw[(s0 >> 5) + tid] = (rank << 32) | occ;
     }
     __syncthreads();
-    // coalesced write-out of the chunk's ptrs, 16 bytes per store
+    // coalesced write-out of the chunk's ptrs, 16 bytes per store (skipped when the dense
+    // table is not wanted: the lookup uses the rank directory + compact table, and
+    // gpumem_index_view expands ptrs from them on demand, k_ptrs_expand)
+    if (!ptrs) return;
     const uint64_t lim = n_buckets - s0 < uint64_t(kChunk) ? n_buckets - s0 : uint64_t(kChunk);
     if (lim == uint64_t(kChunk)) {
         uint4 *dst = reinterpret_cast<uint4 *>(ptrs + s0);
@@ -388,9 +393,10 @@ __global__ void __launch_bounds__(kFillThreads) k_index_local(
     if ((tid & 31) == 0) gstart[w] = first_pre;  // group w = seeds [1024 w, 1024 w + 1024) starts here
     if (tid == 0) gstart[kFillThreads / 32] = uint32_t(hi);
     __syncthreads();
-    // ptrs out, 16 bytes per store
+    // ptrs out, 16 bytes per store (skipped without a dense table)
     const uint64_t lim = n_buckets - s0 < uint64_t(kChunk) ? n_buckets - s0 : uint64_t(kChunk);
-    if (lim == uint64_t(kChunk)) {
+    if (!ptrs) {
+    } else if (lim == uint64_t(kChunk)) {
         uint4 *dst = reinterpret_cast<uint4 *>(ptrs + s0);
         for (int i = tid; i < kChunk / 4; i += kFillThreads) {
             const int b = 4 * i;
@@ -400,7 +406,7 @@ __global__ void __launch_bounds__(kFillThreads) k_index_local(
     } else {
         for (int i = tid; i < int(lim); i += kFillThreads) ptrs[s0 + i] = cnt[i + (i >> 5)];
     }
-    if (s0 == 0 && tid == 0) ptrs[n_buckets] = uint32_t(n);
+    if (ptrs && s0 == 0 && tid == 0) ptrs[n_buckets] = uint32_t(n);
     __syncthreads();
     // place: warp w walks group w in p order; counters advance as cursors. Only the
     // slots are computed here (shared memory only, so a hot group's long walk stays
@@ -466,6 +472,53 @@ cudaError_t launch_seed_codes(const uint64_t *R, uint32_t ls, uint32_t step, uin
     if (n_locs == 0) return cudaSuccess;
     const uint64_t blocks = (n_locs + kCodeThreads - 1) / kCodeThreads;
     k_seed_codes<<<unsigned(blocks), kCodeThreads, 0, s>>>(R, ls, step, k0, n_locs, codes, locs);
+    note_launch();
+    return cudaGetLastError();
+}
+
+// The paper's dense ptrs (ptrs[s] = number of sampled locations with seed
+// < s, ptrs[4^ls] = n_locs) expanded from the rank directory and the compact table:
+// ptrs[s] = first slot of the first occupied seed >= s = buckets[rank(s)].first, where
+// rank(s) = occupied seeds below s, or n_locs past the last occupied seed.
+template <bool kSect>
+__global__ void __launch_bounds__(256) k_ptrs_expand(const unsigned long long *__restrict__ rankw,
+                                                     const uint4 *__restrict__ rsect,
+                                                     const uint2 *__restrict__ buckets, uint64_t nb, uint64_t n_locs,
+                                                     uint32_t *__restrict__ ptrs) {
+    constexpr uint64_t kLo = 0x5555555555555555ull;
+    auto rank_of = [&](uint64_t s, bool &in) -> uint64_t {  // occupied seeds in [0, s) (+ s's own occupancy)
+        const uint32_t b = uint32_t(s & 31);
+        if (kSect) {
+            const uint4 r = rsect[s >> 5];
+            const uint64_t c2 = (uint64_t(r.w) << 32) | r.z;
+            const uint64_t below = b ? c2 & ((1ull << (2 * b)) - 1ull) : 0ull;
+            in = ((c2 >> (2 * b)) & 3u) != 0;
+            return r.y + __popcll((below | (below >> 1)) & kLo);
+        }
+        const unsigned long long r = rankw[s >> 5];
+        const uint32_t bits = uint32_t(r);
+        in = (bits >> b) & 1u;
+        return uint32_t(r >> 32) + __popc(bits & ((1u << b) - 1u));
+    };
+    bool in_last = false;
+    const uint64_t n_occ = nb ? rank_of(nb - 1, in_last) + (in_last ? 1 : 0) : 0;
+    for (uint64_t s = uint64_t(blockIdx.x) * 256 + threadIdx.x; s <= nb; s += uint64_t(gridDim.x) * 256) {
+        uint32_t v = uint32_t(n_locs);
+        if (s < nb) {
+            bool in = false;
+            const uint64_t r = rank_of(s, in);
+            if (r < n_occ) v = buckets[r].x;
+        }
+        ptrs[s] = v;
+    }
+}
+
+cudaError_t launch_ptrs_expand(const unsigned long long *rankw, const uint4 *rsect, const uint2 *buckets, uint32_t ls,
+                               uint64_t n_locs, uint32_t *ptrs, cudaStream_t s) {
+    const uint64_t nb = 1ull << (2 * ls);
+    const unsigned grid = unsigned(std::min<uint64_t>((nb + 1 + 255) / 256, uint64_t(num_sms()) * 16));
+    if (rsect) k_ptrs_expand<true><<<grid, 256, 0, s>>>(rankw, rsect, buckets, nb, n_locs, ptrs);
+    else k_ptrs_expand<false><<<grid, 256, 0, s>>>(rankw, rsect, buckets, nb, n_locs, ptrs);
     note_launch();
     return cudaGetLastError();
 }

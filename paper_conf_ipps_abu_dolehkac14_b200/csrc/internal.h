@@ -105,6 +105,9 @@ size_t ptrs_fill_scratch_bytes(uint32_t ls);
 cudaError_t launch_ptrs_fill(const uint32_t *sorted_codes, uint64_t n_locs, uint32_t ls, uint32_t *ptrs,
                              unsigned long long *rankw, uint4 *rsect, uint2 *buckets, void *scratch,
                              cudaStream_t s);
+// Dense ptrs[0 .. 4^ls] from the rank directory (rankw or rsect) + compact table (index.cu).
+cudaError_t launch_ptrs_expand(const unsigned long long *rankw, const uint4 *rsect, const uint2 *buckets, uint32_t ls,
+                               uint64_t n_locs, uint32_t *ptrs, cudaStream_t s);
 // Fused last step of the index (index.cu): (code, p) pairs sorted stably by code bits
 // [10, 2 ls) -> ptrs, rank directory, compact table, final locs and seed records.
 size_t index_local_scratch_bytes(uint32_t ls);
