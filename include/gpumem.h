@@ -196,6 +196,12 @@ gpumem_status gpumem_merge_sorted(const gpumem_triple *const *dev_runs, const ui
  *  the graph (one ordinary synchronous pass + capture); later calls are one
  *  cudaGraphLaunch. The previous run's result is invalidated.
  *
+ * gpumem_pipeline_run_host -- the same from host memory (pinned for full speed): R and Q
+ *  are copied on a copy stream into pipeline-owned device buffers (allocated on the
+ *  first call), R first; the graph packs and indexes R while Q is still in flight and
+ *  each segment waits only for the copy it reads. Async: the host buffers must stay
+ *  valid and unmodified until the run completes (gpumem_pipeline_result).
+ *
  * gpumem_pipeline_result -- synchronises the stream, then checks the alphabet flags
  *  (GPUMEM_ERR_ALPHABET as gpumem_find_mems) and the output capacity: on overflow the
  *  MEMs are recomputed with gpumem_find_mems on the pipeline's packed sequences and
@@ -211,6 +217,7 @@ gpumem_status gpumem_merge_sorted(const gpumem_triple *const *dev_runs, const ui
 gpumem_status gpumem_pipeline_create(uint64_t r_len, uint64_t q_len, uint32_t seed_len, uint32_t min_len,
                                      uint64_t q_begin, uint64_t q_end, void *cuda_stream, gpumem_pipeline **out);
 gpumem_status gpumem_pipeline_run(gpumem_pipeline *pl, const char *r_bases_dev, const char *q_bases_dev);
+gpumem_status gpumem_pipeline_run_host(gpumem_pipeline *pl, const char *r_bases_host, const char *q_bases_host);
 gpumem_status gpumem_pipeline_result(gpumem_pipeline *pl, const gpumem_triple **dev_ptr, uint64_t *count);
 gpumem_status gpumem_pipeline_stats(const gpumem_pipeline *pl, gpumem_find_stats *out);
 int gpumem_pipeline_profile(const gpumem_pipeline *pl, const char **names, double *ms, uint64_t *launches,

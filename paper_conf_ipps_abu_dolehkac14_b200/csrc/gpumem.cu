@@ -91,6 +91,7 @@ struct PipeItem {
     cudaGraph_t g;
     cudaGraphExec_t x;
     cudaEvent_t ev;
+    int wait;   // 1 / 2: wait for the host copy of R / Q (host-input runs only)
 };
 
 struct CapCtx {
@@ -227,12 +228,12 @@ static void cap_cut(cudaStream_t s, cudaEvent_t ev) {
         if (nodes) {
             cudaGraphExec_t x = nullptr;
             e = cudaGraphInstantiate(&x, g, 0);
-            if (e == cudaSuccess) c.items->push_back(PipeItem{g, x, nullptr});
+            if (e == cudaSuccess) c.items->push_back(PipeItem{g, x, nullptr, 0});
         } else {
             cudaGraphDestroy(g);
         }
     }
-    if (ev) c.items->push_back(PipeItem{nullptr, nullptr, ev});
+    if (ev) c.items->push_back(PipeItem{nullptr, nullptr, ev, 0});
     const cudaError_t e2 = cudaStreamBeginCapture(s, cudaStreamCaptureModeRelaxed);
     if (c.err == cudaSuccess) c.err = e != cudaSuccess ? e : e2;
 }
@@ -390,6 +391,9 @@ struct gpumem_pipeline {
     char *arena;
     size_t arena_bytes;
     std::vector<PipeItem> items;           // graph segments and stage events, in run order
+    char *stage;                           // host-input runs: device copies of R and Q (nR + nQ bytes)
+    cudaStream_t copy;                     // ... copied on this stream
+    cudaEvent_t ev_r, ev_q;                // R / Q copied
     gpumem_seq *R, *Q;
     gpumem_index *idx;
     gpumem_mems *mems;                     // the graph's result buffer (count set by _result)
@@ -405,14 +409,24 @@ struct gpumem_pipeline {
 namespace {
 
 // The whole path on the pipeline's stream: pack R, pack Q, index R, find (deferred).
+// Capture: mark where a host-input run must wait for the copy of R (1) or Q (2).
+void pipeline_wait_mark(cudaStream_t s, int which) {
+    if (!(t_cap && t_cap->items)) return;
+    cap_cut(s, nullptr);
+    t_cap->items->push_back(PipeItem{nullptr, nullptr, nullptr, which});
+}
+
 gpumem_status pipeline_path(gpumem_pipeline *pl, const char *R, const char *Q, gpumem_seq **hR, gpumem_seq **hQ,
                             gpumem_index **hI, gpumem_mems **hM) {
     *hR = *hQ = nullptr;
     *hI = nullptr;
     *hM = nullptr;
+    // R's part first: with host inputs the index is built while Q is still crossing PCIe
+    pipeline_wait_mark(pl->stream, 1);
     gpumem_status st = gpumem_pack(R, pl->nR, 1, pl->stream, hR);
-    if (!st) st = gpumem_pack(Q, pl->nQ, 1, pl->stream, hQ);
     if (!st) st = gpumem_index_build(*hR, pl->ls, pl->L, pl->stream, hI);
+    if (!st) pipeline_wait_mark(pl->stream, 2);
+    if (!st) st = gpumem_pack(Q, pl->nQ, 1, pl->stream, hQ);
     if (!st) st = gpumem_find_mems(*hI, *hQ, pl->q_begin, pl->q_end, pl->stream, hM);
     return st;
 }
@@ -503,6 +517,19 @@ gpumem_status pipeline_capture(gpumem_pipeline *pl, const char *R, const char *Q
     pl->inR = R;
     pl->inQ = Q;
     return GPUMEM_OK;
+}
+
+// One run: the graph segments and stage events in order; with host inputs the
+// segments that read R / Q first wait for their copy.
+cudaError_t pipeline_launch(gpumem_pipeline *pl, bool host_inputs) {
+    for (const auto &it : pl->items) {
+        cudaError_t e = cudaSuccess;
+        if (it.x) e = cudaGraphLaunch(it.x, pl->stream);
+        else if (it.ev) e = cudaEventRecord(it.ev, pl->stream);
+        else if (host_inputs) e = cudaStreamWaitEvent(pl->stream, it.wait == 1 ? pl->ev_r : pl->ev_q, 0);
+        if (e != cudaSuccess) return e;
+    }
+    return cudaSuccess;
 }
 
 }  // namespace
@@ -632,6 +659,13 @@ void gpumem_free(void *handle) {
         cudaFreeHost(pl->host);
         cudaEventDestroy(pl->ev_in);
         cudaEventDestroy(pl->ev_out);
+        if (pl->stage) {
+            cudaStreamSynchronize(pl->copy);
+            cudaFree(pl->stage);
+            cudaEventDestroy(pl->ev_r);
+            cudaEventDestroy(pl->ev_q);
+            cudaStreamDestroy(pl->copy);
+        }
         ws_release_stream(pl->device, pl->stream);
         cudaStreamDestroy(pl->stream);
         pl->magic = 0;
@@ -1217,12 +1251,49 @@ gpumem_status gpumem_pipeline_run(gpumem_pipeline *pl, const char *r_bases_dev, 
         const gpumem_status st = pipeline_capture(pl, r_bases_dev, q_bases_dev);
         if (st) return st;
     }
-    for (const auto &it : pl->items) {
-        if (it.x) CK(cudaGraphLaunch(it.x, pl->stream), "graph launch");
-        else CK(cudaEventRecord(it.ev, pl->stream), "stage event");
-    }
+    CK(pipeline_launch(pl, false), "graph launch");
     note_launch(int(pl->launches));
     CK(cudaEventRecord(pl->ev_out, pl->stream), "event");  // the caller's later work sees the result
+    CK(cudaStreamWaitEvent(pl->user, pl->ev_out, 0), "wait");
+    pl->ran = 1;
+    return GPUMEM_OK;
+}
+
+gpumem_status gpumem_pipeline_run_host(gpumem_pipeline *pl, const char *r_bases_host, const char *q_bases_host) {
+    if (!pl || pl->magic != kMagicPipe) return fail(GPUMEM_ERR_ARG, "not a gpumem_pipeline");
+    if ((!r_bases_host && pl->nR) || (!q_bases_host && pl->nQ)) return fail(GPUMEM_ERR_ARG, "NULL input");
+    int dev = -1;
+    cudaGetDevice(&dev);
+    if (dev != pl->device) return fail(GPUMEM_ERR_ARG, "pipeline lives on device %d, current is %d", pl->device, dev);
+    if (pl->fallback) {
+        gpumem_free(pl->fallback);
+        pl->fallback = nullptr;
+    }
+    if (!pl->stage) {
+        CK(cudaMalloc(&pl->stage, pl->nR + pl->nQ + 256), "input staging");
+        CK(cudaStreamCreateWithFlags(&pl->copy, cudaStreamNonBlocking), "copy stream");
+        CK(cudaEventCreateWithFlags(&pl->ev_r, cudaEventDisableTiming), "event");
+        CK(cudaEventCreateWithFlags(&pl->ev_q, cudaEventDisableTiming), "event");
+    }
+    char *dR = pl->stage, *dQ = pl->stage + pl->nR;
+    // the copies start after the caller's prior work and after the previous run (which
+    // read the staging buffers); R, then Q, each announced by an event
+    CK(cudaEventRecord(pl->ev_in, pl->user), "event");
+    CK(cudaStreamWaitEvent(pl->copy, pl->ev_in, 0), "wait");
+    CK(cudaStreamWaitEvent(pl->copy, pl->ev_out, 0), "wait");
+    if (pl->nR) CK(cudaMemcpyAsync(dR, r_bases_host, pl->nR, cudaMemcpyHostToDevice, pl->copy), "H2D R");
+    CK(cudaEventRecord(pl->ev_r, pl->copy), "event");
+    if (pl->nQ) CK(cudaMemcpyAsync(dQ, q_bases_host, pl->nQ, cudaMemcpyHostToDevice, pl->copy), "H2D Q");
+    CK(cudaEventRecord(pl->ev_q, pl->copy), "event");
+    CK(cudaStreamWaitEvent(pl->stream, pl->ev_in, 0), "wait");
+    if (pl->items.empty() || pl->inR != dR || pl->inQ != dQ) {
+        CK(cudaStreamWaitEvent(pl->stream, pl->ev_q, 0), "wait");  // the measuring run reads both
+        const gpumem_status st = pipeline_capture(pl, dR, dQ);
+        if (st) return st;
+    }
+    CK(pipeline_launch(pl, true), "graph launch");
+    note_launch(int(pl->launches));
+    CK(cudaEventRecord(pl->ev_out, pl->stream), "event");
     CK(cudaStreamWaitEvent(pl->user, pl->ev_out, 0), "wait");
     pl->ran = 1;
     return GPUMEM_OK;

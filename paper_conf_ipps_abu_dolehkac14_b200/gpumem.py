@@ -49,6 +49,7 @@ SYMBOLS = {
     "gpumem_merge_sorted": (ctypes.c_int, [_P(_vp), _P(_c_u64), ctypes.c_int, _vp, _P(_vp)]),
     "gpumem_pipeline_create": (ctypes.c_int, [_c_u64, _c_u64, _c_u32, _c_u32, _c_u64, _c_u64, _vp, _P(_vp)]),
     "gpumem_pipeline_run": (ctypes.c_int, [_vp, _vp, _vp]),
+    "gpumem_pipeline_run_host": (ctypes.c_int, [_vp, _vp, _vp]),
     "gpumem_pipeline_result": (ctypes.c_int, [_vp, _P(_vp), _P(_c_u64)]),
     "gpumem_pipeline_stats": (ctypes.c_int, [_vp, _vp]),
     "gpumem_pipeline_profile": (ctypes.c_int, [_vp, _P(ctypes.c_char_p), _P(ctypes.c_double), _P(_c_u64),
@@ -304,6 +305,24 @@ class Pipeline(_Handle):
         self._inputs = (R_dev, Q_dev)
         self._ptr = None
         _check(_lib.gpumem_pipeline_run(self.handle, _vp(R_dev.data_ptr()), _vp(Q_dev.data_ptr())))
+
+    def run_host(self, R_host, Q_host):
+        """R_host, Q_host: host uint8 buffers (numpy arrays or CPU tensors; pinned for full
+        PCIe speed) of the sizes given at creation, kept alive until the next run. The
+        copies overlap the R half of the path (pack + index)."""
+        import torch
+        keep = []
+        for x in (R_host, Q_host):
+            if isinstance(x, torch.Tensor):
+                if x.is_cuda or x.dtype != torch.uint8 or not x.is_contiguous():
+                    raise TypeError("host inputs must be contiguous uint8 CPU tensors or numpy arrays")
+                keep.append((x, x.data_ptr()))
+            else:
+                a = np.ascontiguousarray(x, dtype=np.uint8)
+                keep.append((a, a.ctypes.data))
+        self._inputs = tuple(k[0] for k in keep)
+        self._ptr = None
+        _check(_lib.gpumem_pipeline_run_host(self.handle, _vp(keep[0][1]), _vp(keep[1][1])))
 
     def result(self):
         ptr, n = _vp(), _c_u64()

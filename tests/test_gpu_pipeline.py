@@ -131,3 +131,23 @@ def test_pipeline_edges_and_alphabet():
         pl.result()
     assert ei.value.name == "ERR_ALPHABET" and "1234" in str(ei.value)
     pl.free()
+
+
+def test_pipeline_host_inputs():
+    """run_host: H2D copies overlapped with the R half of the graph; same MEM set, and
+    switching between host and device inputs recaptures correctly."""
+    P = synth.make_pair("c2", scale=0.2)
+    want = oracle.mems(P.R, P.Q, P.L, P.ls)
+    Rh = torch.from_numpy(P.R).pin_memory()
+    Qh = torch.from_numpy(P.Q).pin_memory()
+    pl = gpumem.Pipeline(len(P.R), len(P.Q), P.ls, P.L)
+    for src in ("host", "host", "dev", "host", "numpy"):
+        if src == "host":
+            pl.run_host(Rh, Qh)
+        elif src == "numpy":
+            pl.run_host(P.R, P.Q)
+        else:
+            pl.run(_dev(P.R), _dev(P.Q))
+        assert pl.result() == len(want), src
+        assert np.array_equal(pl.numpy(), want), src
+    pl.free()
