@@ -212,6 +212,134 @@ __global__ void __launch_bounds__(kFillThreads) k_ptrs_fill(const uint32_t *__re
     if (s0 == 0 && tid == 0) ptrs[n_buckets] = uint32_t(n);
 }
 
+// The lookup directory of one chunk (kChunk seeds = kGroups groups of 32) driven by
+// the chunk's sorted codes instead of its seeds: work O(elements + groups) per CTA
+// rather than O(kChunk), so a sparse index (C4: ~700 sampled seeds per 16K-seed chunk)
+// is not dominated by zeroing and scanning 16K empty counters (k_ptrs_fill).
+//  elements  run heads (first of each distinct code) get their in-chunk rank by a
+//            block scan; a run's length is the distance to the next head (runs never
+//            cross a chunk), the last run of a block is finished by the next block
+//            (or the chunk end). Each run -> buckets[rank0 + rank] = {first, count},
+//            its occupancy bit, its 2-bit saturating count (rank sectors) and its
+//            element count per group (records before the group, rank sectors);
+//  groups    a block scan over the chunk's kGroups groups gives occupied seeds (and
+//            records) before each group -> one rank word / rank sector per group.
+constexpr int kGroups = kChunk / 32;           // 512
+constexpr int kDirThreads = 512;
+static_assert(kGroups == kDirThreads, "one group per thread in the group phase");
+
+template <bool kSect>
+__global__ void __launch_bounds__(kDirThreads) k_dir_fill(const uint32_t *__restrict__ codes, uint64_t n_buckets,
+                                                          unsigned long long *__restrict__ rankw,
+                                                          uint4 *__restrict__ rsect, uint2 *__restrict__ buckets,
+                                                          const uint32_t *__restrict__ chunk_first,
+                                                          const uint32_t *__restrict__ rank0) {
+    __shared__ uint32_t occ[kGroups], ecnt[kGroups], c2lo[kGroups], c2hi[kGroups];
+    __shared__ uint32_t hpos[kDirThreads + 1];
+    __shared__ uint32_t wsum[kDirThreads / 32];
+    __shared__ uint32_t s_carry, s_pend_first, s_pend_code, s_pend_rank, s_pend;
+    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+    const uint32_t c = blockIdx.x;
+    const uint64_t s0 = uint64_t(c) * kChunk;
+    const uint32_t lo = chunk_first[c], hi = chunk_first[c + 1];
+    const uint32_t r0 = rank0[c];
+    occ[tid] = 0;
+    ecnt[tid] = 0;
+    if (kSect) {
+        c2lo[tid] = 0;
+        c2hi[tid] = 0;
+    }
+    if (tid == 0) {
+        s_carry = 0;
+        s_pend = 0;
+    }
+    __syncthreads();
+    // one finished run (code, first slot, count, in-chunk rank) into every structure
+    auto run_out = [&](uint32_t code, uint32_t first, uint32_t count, uint32_t rank) {
+        buckets[r0 + rank] = make_uint2(first, count);
+        const uint32_t sd = code - uint32_t(s0), g = sd >> 5, b = sd & 31;
+        atomicOr(&occ[g], 1u << b);
+        if (kSect) {
+            atomicAdd(&ecnt[g], count);
+            const uint32_t sat = count < 3 ? count : 3u;
+            if (b < 16) atomicOr(&c2lo[g], sat << (2 * b));
+            else atomicOr(&c2hi[g], sat << (2 * (b - 16)));
+        }
+    };
+    for (uint32_t base = lo; base < hi; base += kDirThreads) {
+        const uint32_t i = base + tid;
+        const bool valid = i < hi;
+        const uint32_t code = valid ? codes[i] : 0u;
+        const bool head = valid && (i == 0 || codes[i - 1] != code);
+        const unsigned hb = __ballot_sync(0xffffffffu, head);
+        if (lane == 0) wsum[w] = __popc(hb);
+        __syncthreads();
+        uint32_t before = 0, total = 0;
+        for (int k = 0; k < kDirThreads / 32; ++k) {
+            const uint32_t x = wsum[k];
+            before += k < w ? x : 0u;
+            total += x;
+        }
+        const uint32_t hr = before + __popc(hb & ((1u << lane) - 1u));  // head rank in this block
+        if (head) hpos[hr] = i;
+        if (tid == 0) hpos[total] = base + kDirThreads < hi ? 0xffffffffu : hi;  // block end sentinel
+        __syncthreads();
+        const uint32_t carry = s_carry;
+        // the previous block's last run ends at this block's first head (or the chunk end)
+        if (tid == 0 && s_pend) {
+            const uint32_t end = total ? hpos[0] : (base + kDirThreads < hi ? 0xffffffffu : hi);
+            if (end != 0xffffffffu) {
+                run_out(s_pend_code, s_pend_first, end - s_pend_first, s_pend_rank);
+                s_pend = 0;
+            }
+        }
+        __syncthreads();  // the old pending run is settled before a new one is recorded
+        if (head) {
+            const uint32_t nxt = hpos[hr + 1];
+            if (nxt != 0xffffffffu) run_out(code, i, nxt - i, carry + hr);
+            else {  // the last head of a non-final block: finished later
+                s_pend = 1;
+                s_pend_code = code;
+                s_pend_first = i;
+                s_pend_rank = carry + hr;
+            }
+        }
+        __syncthreads();
+        if (tid == 0) s_carry = carry + total;
+        __syncthreads();
+    }
+    if (tid == 0 && s_pend) run_out(s_pend_code, s_pend_first, hi - s_pend_first, s_pend_rank);
+    __syncthreads();
+    // group phase: thread tid owns group tid of the chunk
+    const uint32_t o = occ[tid], no = __popc(o), ne = kSect ? ecnt[tid] : 0u;
+    uint32_t inc = no, ince = ne;
+#pragma unroll
+    for (int k = 1; k < 32; k <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, inc, k);
+        const uint32_t z = __shfl_up_sync(0xffffffffu, ince, k);
+        if (lane >= k) {
+            inc += y;
+            ince += z;
+        }
+    }
+    __shared__ uint32_t wo[kDirThreads / 32], we[kDirThreads / 32];
+    if (lane == 31) {
+        wo[w] = inc;
+        we[w] = ince;
+    }
+    __syncthreads();
+    uint32_t po = inc - no, pe = ince - ne;
+    for (int k = 0; k < w; ++k) {
+        po += wo[k];
+        pe += we[k];
+    }
+    if (s0 + uint64_t(tid) * 32 < n_buckets) {
+        const uint64_t g = (s0 >> 5) + tid;
+        if (kSect) rsect[g] = make_uint4(lo + pe, r0 + po, c2lo[tid], c2hi[tid]);
+        else rankw[g] = (uint64_t(r0 + po) << 32) | o;
+    }
+}
+
 // Seed records (lookup acceleration, not part of the paper's index): for each slot k
 // of locs, {p, bases R[p-16, p) with base p-1 in the low bits (00 before position 0),
 // bases R[p+ls, p+ls+32) first base highest (00 past the end)} -- 16 bytes, one
@@ -555,12 +683,23 @@ cudaError_t launch_ptrs_fill(const uint32_t *sorted_codes, uint64_t n_locs, uint
         if (e != cudaSuccess) return e;
         attr = true;
     }
-    if (rsect)
+    // directory + compact table only (the default): element-driven while the index is
+    // sparse (C4: 0.086 -> 0.053 ms); a dense one (C5 at L = 20: 7.6K seeds per chunk,
+    // 0.33 vs 0.46 ms) keeps the seed-driven fill with its ptrs write-out skipped
+    if (!ptrs && n_locs * 4 < nb) {
+        if (rsect)
+            k_dir_fill<true><<<unsigned(chunks), kDirThreads, 0, s>>>(sorted_codes, nb, rankw, rsect, buckets, first,
+                                                                      rank0);
+        else
+            k_dir_fill<false><<<unsigned(chunks), kDirThreads, 0, s>>>(sorted_codes, nb, rankw, rsect, buckets, first,
+                                                                       rank0);
+    } else if (rsect) {
         k_ptrs_fill<true><<<unsigned(chunks), kFillThreads, smem, s>>>(sorted_codes, n_locs, nb, ptrs, rankw, rsect,
                                                                        buckets, first, rank0);
-    else
+    } else {
         k_ptrs_fill<false><<<unsigned(chunks), kFillThreads, smem, s>>>(sorted_codes, n_locs, nb, ptrs, rankw, rsect,
                                                                         buckets, first, rank0);
+    }
     note_launch(4);
     return cudaGetLastError();
 }

@@ -118,11 +118,27 @@ def test_index_golden_w2():
                                                 ("c2", 12, 9, 1.0), ("c3", 13, 38, 0.1), ("c4", 13, 8, 0.02),
                                                 ("c4", 15, 1, 0.01), ("c1", 7, 64, 0.5)])
 def test_index_parity_word_for_word(cfg, ls, step, scale):
+    """ptrs (expanded from the lookup directory + compact table, both directory kinds)
+    and locs word for word against Alg. 1."""
     P = synth.make_pair(cfg, scale=scale)
-    p, l = _index_gpu(P.R.tobytes(), ls, step)
     op, ol = oracle.index(P.R.tobytes(), ls, step)
-    assert np.array_equal(p, op)
-    assert np.array_equal(l, ol)
+    for sect in (-1, 0, 1):
+        gpumem.set_option("rank_sectors", sect)
+        p, l = _index_gpu(P.R.tobytes(), ls, step)
+        assert np.array_equal(p, op), sect
+        assert np.array_equal(l, ol), sect
+
+
+def test_index_hot_seed_chunks():
+    """Directory build on runs far longer than a block (poly-A / (AC)^n seeds: one code
+    with tens of thousands of sampled locations), every block/run boundary case."""
+    R = b"A" * 70000 + b"AC" * 20000 + b"ACGT" * 3000 + b"T" * 1500
+    for ls, step in ((13, 1), (12, 3), (5, 2)):
+        op, ol = oracle.index(R, ls, step)
+        for sect in (0, 1):
+            gpumem.set_option("rank_sectors", sect)
+            p, l = _index_gpu(R, ls, step)
+            assert np.array_equal(p, op) and np.array_equal(l, ol), (ls, step, sect)
 
 
 @pytest.mark.parametrize("opts", [{"small_sort": 1}, {"radix_bits": 8}, {"index_msd": 1}, {"index_fused": 1},
