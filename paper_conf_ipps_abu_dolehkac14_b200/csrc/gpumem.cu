@@ -91,12 +91,14 @@ struct PipeItem {
     cudaGraph_t g;
     cudaGraphExec_t x;
     cudaEvent_t ev;
-    int wait;   // 1 / 2: wait for the host copy of R / Q (host-input runs only)
+    int wait;   // 1 / 2: wait for the host copy of R / Q (host-input runs only); 3: join the side stream
+    int sid;    // 0: the pipeline's stream, 1: its side stream (pack Q, concurrent with the index build)
 };
 
 struct CapCtx {
     int mode = 0;
     std::vector<PipeItem> *items = nullptr;  // capture: segments cut at every stage boundary
+    int sid = 0;                             // stream the segments being captured will run on
     cudaError_t err = cudaSuccess;
     char *arena = nullptr;
     size_t off = 0, cap = 0, need = 0;
@@ -228,12 +230,12 @@ static void cap_cut(cudaStream_t s, cudaEvent_t ev) {
         if (nodes) {
             cudaGraphExec_t x = nullptr;
             e = cudaGraphInstantiate(&x, g, 0);
-            if (e == cudaSuccess) c.items->push_back(PipeItem{g, x, nullptr, 0});
+            if (e == cudaSuccess) c.items->push_back(PipeItem{g, x, nullptr, 0, c.sid});
         } else {
             cudaGraphDestroy(g);
         }
     }
-    if (ev) c.items->push_back(PipeItem{nullptr, nullptr, ev, 0});
+    if (ev) c.items->push_back(PipeItem{nullptr, nullptr, ev, 0, c.sid});
     const cudaError_t e2 = cudaStreamBeginCapture(s, cudaStreamCaptureModeRelaxed);
     if (c.err == cudaSuccess) c.err = e != cudaSuccess ? e : e2;
 }
@@ -384,7 +386,8 @@ struct gpumem_pipeline {
     int device;
     cudaStream_t user;                     // the caller's stream (runs are ordered on it by events)
     cudaStream_t stream;                   // the pipeline's own stream: capture, launches, fallback
-    cudaEvent_t ev_in, ev_out;
+    cudaStream_t side;                     // runs pack Q next to the index build
+    cudaEvent_t ev_in, ev_out, ev_join;
     uint64_t nR, nQ, q_begin, q_end;
     uint32_t ls, L;
     const char *inR, *inQ;                 // the device inputs the graph was captured with
@@ -413,7 +416,16 @@ namespace {
 void pipeline_wait_mark(cudaStream_t s, int which) {
     if (!(t_cap && t_cap->items)) return;
     cap_cut(s, nullptr);
-    t_cap->items->push_back(PipeItem{nullptr, nullptr, nullptr, which});
+    t_cap->items->push_back(PipeItem{nullptr, nullptr, nullptr, which, t_cap->sid});
+}
+
+// Capture: the following segments run on the side stream (1) / back on the main stream
+// after joining the side stream (0).
+void pipeline_side(cudaStream_t s, int sid) {
+    if (!(t_cap && t_cap->items)) return;
+    cap_cut(s, nullptr);
+    if (sid == 0) t_cap->items->push_back(PipeItem{nullptr, nullptr, nullptr, 3, 0});
+    t_cap->sid = sid;
 }
 
 gpumem_status pipeline_path(gpumem_pipeline *pl, const char *R, const char *Q, gpumem_seq **hR, gpumem_seq **hQ,
@@ -422,11 +434,14 @@ gpumem_status pipeline_path(gpumem_pipeline *pl, const char *R, const char *Q, g
     *hI = nullptr;
     *hM = nullptr;
     // R's part first: with host inputs the index is built while Q is still crossing PCIe
+    // pack Q runs on the side stream, concurrently with the (latency-bound) index build
     pipeline_wait_mark(pl->stream, 1);
     gpumem_status st = gpumem_pack(R, pl->nR, 1, pl->stream, hR);
     if (!st) st = gpumem_index_build(*hR, pl->ls, pl->L, pl->stream, hI);
+    if (!st) pipeline_side(pl->stream, 1);
     if (!st) pipeline_wait_mark(pl->stream, 2);
     if (!st) st = gpumem_pack(Q, pl->nQ, 1, pl->stream, hQ);
+    if (!st) pipeline_side(pl->stream, 0);
     if (!st) st = gpumem_find_mems(*hI, *hQ, pl->q_begin, pl->q_end, pl->stream, hM);
     return st;
 }
@@ -522,11 +537,18 @@ gpumem_status pipeline_capture(gpumem_pipeline *pl, const char *R, const char *Q
 // One run: the graph segments and stage events in order; with host inputs the
 // segments that read R / Q first wait for their copy.
 cudaError_t pipeline_launch(gpumem_pipeline *pl, bool host_inputs) {
+    cudaError_t e = cudaStreamWaitEvent(pl->side, pl->ev_in, 0);  // fork: the side stream starts with the run
+    if (e != cudaSuccess) return e;
     for (const auto &it : pl->items) {
-        cudaError_t e = cudaSuccess;
-        if (it.x) e = cudaGraphLaunch(it.x, pl->stream);
-        else if (it.ev) e = cudaEventRecord(it.ev, pl->stream);
-        else if (host_inputs) e = cudaStreamWaitEvent(pl->stream, it.wait == 1 ? pl->ev_r : pl->ev_q, 0);
+        cudaStream_t st = it.sid ? pl->side : pl->stream;
+        if (it.x) e = cudaGraphLaunch(it.x, st);
+        else if (it.ev) e = cudaEventRecord(it.ev, st);
+        else if (it.wait == 3) {  // join
+            e = cudaEventRecord(pl->ev_join, pl->side);
+            if (e == cudaSuccess) e = cudaStreamWaitEvent(pl->stream, pl->ev_join, 0);
+        } else if (host_inputs) {
+            e = cudaStreamWaitEvent(st, it.wait == 1 ? pl->ev_r : pl->ev_q, 0);
+        }
         if (e != cudaSuccess) return e;
     }
     return cudaSuccess;
@@ -667,6 +689,9 @@ void gpumem_free(void *handle) {
             cudaStreamDestroy(pl->copy);
         }
         ws_release_stream(pl->device, pl->stream);
+        cudaStreamSynchronize(pl->side);
+        cudaStreamDestroy(pl->side);
+        cudaEventDestroy(pl->ev_join);
         cudaStreamDestroy(pl->stream);
         pl->magic = 0;
         delete pl;
@@ -1214,6 +1239,8 @@ gpumem_status gpumem_pipeline_create(uint64_t r_len, uint64_t q_len, uint32_t se
     // the legacy default stream cannot be captured: the graph runs on a stream of its
     // own, ordered after / before the caller's stream by events
     if (cudaStreamCreateWithFlags(&pl->stream, cudaStreamNonBlocking) != cudaSuccess ||
+        cudaStreamCreateWithFlags(&pl->side, cudaStreamNonBlocking) != cudaSuccess ||
+        cudaEventCreateWithFlags(&pl->ev_join, cudaEventDisableTiming) != cudaSuccess ||
         cudaEventCreateWithFlags(&pl->ev_in, cudaEventDisableTiming) != cudaSuccess ||
         cudaEventCreateWithFlags(&pl->ev_out, cudaEventDisableTiming) != cudaSuccess) {
         const cudaError_t e = cudaGetLastError();
