@@ -15,8 +15,9 @@
 #define GPUMEM_VERSION "0.1.0"
 
 // output sort: the MSD bucket sort up to this many MEMs, the LSD radix sort beyond
-// (measured: MSD faster below a few million keys, its 16K-way scatter slower above)
-constexpr uint64_t kMsdMaxN = 4u << 20;
+// (measured in the pipeline: MSD 0.115 vs LSD 0.173 ms at 0.81 M keys (C4), 0.50 vs 0.31 ms
+// at 2.98 M (C5 L = 50): its shared-memory segment sorts grow with the key count)
+constexpr uint64_t kMsdMaxN = 2u << 20;
 
 enum : uint32_t { kMagicSeq = 0x47534551u, kMagicIdx = 0x47494458u, kMagicMems = 0x474d454du,
                   kMagicPipe = 0x47504950u };
@@ -85,20 +86,8 @@ std::vector<cudaEvent_t> g_ev_free;
 // captured graph holds no allocation nodes and can be relaunched. `deferred` makes
 // find_mems skip its host synchronisation: the output sort reads the MEM count from
 // device memory and the counters are copied to pinned host memory at the end.
-// One step of a pipeline run: a captured graph segment, or a stage event recorded
-// between segments (so stage times are ordinary stream events on the launching stream).
-struct PipeItem {
-    cudaGraph_t g;
-    cudaGraphExec_t x;
-    cudaEvent_t ev;
-    int wait;   // 1 / 2: wait for the host copy of R / Q (host-input runs only); 3: join the side stream
-    int sid;    // 0: the pipeline's stream, 1: its side stream (pack Q, concurrent with the index build)
-};
-
 struct CapCtx {
     int mode = 0;
-    std::vector<PipeItem> *items = nullptr;  // capture: segments cut at every stage boundary
-    int sid = 0;                             // stream the segments being captured will run on
     cudaError_t err = cudaSuccess;
     char *arena = nullptr;
     size_t off = 0, cap = 0, need = 0;
@@ -218,34 +207,13 @@ void dfree(void *p, cudaStream_t s) {
     cudaFreeAsync(p, s);
 }
 
-// Capture: close the current graph segment, append it and then `ev` (if any) to the
-// pipeline's run list, and open the next segment.
-static void cap_cut(cudaStream_t s, cudaEvent_t ev) {
-    CapCtx &c = *t_cap;
-    cudaGraph_t g = nullptr;
-    cudaError_t e = cudaStreamEndCapture(s, &g);
-    if (e == cudaSuccess && g) {
-        size_t nodes = 0;
-        cudaGraphGetNodes(g, nullptr, &nodes);
-        if (nodes) {
-            cudaGraphExec_t x = nullptr;
-            e = cudaGraphInstantiate(&x, g, 0);
-            if (e == cudaSuccess) c.items->push_back(PipeItem{g, x, nullptr, 0, c.sid});
-        } else {
-            cudaGraphDestroy(g);
-        }
-    }
-    if (ev) c.items->push_back(PipeItem{nullptr, nullptr, ev, 0, c.sid});
-    const cudaError_t e2 = cudaStreamBeginCapture(s, cudaStreamCaptureModeRelaxed);
-    if (c.err == cudaSuccess) c.err = e != cudaSuccess ? e : e2;
-}
-
 Stage::Stage(const char *name, cudaStream_t st) : slot(-1), s(st), vec(nullptr) {
     std::vector<StageRec> *v = (t_cap && t_cap->recs) ? t_cap->recs : (g_prof ? &g_recs : nullptr);
     if (!v) return;
     std::lock_guard<std::mutex> g(g_prof_mu);
     StageRec r{name, take_event(), take_event(), g_launches.load(), 0};
-    if (t_cap && t_cap->items) cap_cut(s, r.a);
+    // in a capture: an event record node of the graph (timed on every launch)
+    if (t_cap && t_cap->recs) cudaEventRecordWithFlags(r.a, s, cudaEventRecordExternal);
     else cudaEventRecord(r.a, s);
     v->push_back(r);
     slot = int(v->size()) - 1;
@@ -257,7 +225,7 @@ Stage::~Stage() {
     std::lock_guard<std::mutex> g(g_prof_mu);
     auto &v = *static_cast<std::vector<StageRec> *>(vec);
     if (slot < int(v.size())) {
-        if (t_cap && t_cap->items) cap_cut(s, v[slot].b);
+        if (t_cap && t_cap->recs) cudaEventRecordWithFlags(v[slot].b, s, cudaEventRecordExternal);
         else cudaEventRecord(v[slot].b, s);
         v[slot].l1 = g_launches.load();
     }
@@ -393,7 +361,9 @@ struct gpumem_pipeline {
     const char *inR, *inQ;                 // the device inputs the graph was captured with
     char *arena;
     size_t arena_bytes;
-    std::vector<PipeItem> items;           // graph segments and stage events, in run order
+    cudaGraph_t graph;                     // the captured path (one launch per run)
+    cudaGraphExec_t exec;
+    cudaEvent_t ev_fork;                   // side-stream fork inside the graph
     char *stage;                           // host-input runs: device copies of R and Q (nR + nQ bytes)
     cudaStream_t copy;                     // ... copied on this stream
     cudaEvent_t ev_r, ev_q;                // R / Q copied
@@ -412,20 +382,11 @@ struct gpumem_pipeline {
 namespace {
 
 // The whole path on the pipeline's stream: pack R, pack Q, index R, find (deferred).
-// Capture: mark where a host-input run must wait for the copy of R (1) or Q (2).
-void pipeline_wait_mark(cudaStream_t s, int which) {
-    if (!(t_cap && t_cap->items)) return;
-    cap_cut(s, nullptr);
-    t_cap->items->push_back(PipeItem{nullptr, nullptr, nullptr, which, t_cap->sid});
-}
-
-// Capture: the following segments run on the side stream (1) / back on the main stream
-// after joining the side stream (0).
-void pipeline_side(cudaStream_t s, int sid) {
-    if (!(t_cap && t_cap->items)) return;
-    cap_cut(s, nullptr);
-    if (sid == 0) t_cap->items->push_back(PipeItem{nullptr, nullptr, nullptr, 3, 0});
-    t_cap->sid = sid;
+// Where the path waits for the host copy of R (1) or Q (2): an external event wait
+// node in the captured graph (device-input runs record both events just before the
+// launch, so the waits are free). Nothing to do outside a capture.
+void pipeline_wait_mark(gpumem_pipeline *pl, cudaStream_t s, int which) {
+    if (t_cap && t_cap->recs) cudaStreamWaitEvent(s, which == 1 ? pl->ev_r : pl->ev_q, cudaEventWaitExternal);
 }
 
 gpumem_status pipeline_path(gpumem_pipeline *pl, const char *R, const char *Q, gpumem_seq **hR, gpumem_seq **hQ,
@@ -435,23 +396,25 @@ gpumem_status pipeline_path(gpumem_pipeline *pl, const char *R, const char *Q, g
     *hM = nullptr;
     // R's part first: with host inputs the index is built while Q is still crossing PCIe
     // pack Q runs on the side stream, concurrently with the (latency-bound) index build
-    pipeline_wait_mark(pl->stream, 1);
-    gpumem_status st = gpumem_pack(R, pl->nR, 1, pl->stream, hR);
+    gpumem_status st = GPUMEM_OK;
+    if (cudaEventRecord(pl->ev_fork, pl->stream) != cudaSuccess) st = cuda_fail(cudaGetLastError(), "fork");
+    if (!st && cudaStreamWaitEvent(pl->side, pl->ev_fork, 0) != cudaSuccess) st = cuda_fail(cudaGetLastError(), "fork");
+    if (!st) pipeline_wait_mark(pl, pl->side, 2);
+    if (!st) st = gpumem_pack(Q, pl->nQ, 1, pl->side, hQ);
+    if (!st && cudaEventRecord(pl->ev_join, pl->side) != cudaSuccess) st = cuda_fail(cudaGetLastError(), "join");
+    if (!st) pipeline_wait_mark(pl, pl->stream, 1);
+    if (!st) st = gpumem_pack(R, pl->nR, 1, pl->stream, hR);
     if (!st) st = gpumem_index_build(*hR, pl->ls, pl->L, pl->stream, hI);
-    if (!st) pipeline_side(pl->stream, 1);
-    if (!st) pipeline_wait_mark(pl->stream, 2);
-    if (!st) st = gpumem_pack(Q, pl->nQ, 1, pl->stream, hQ);
-    if (!st) pipeline_side(pl->stream, 0);
+    if (!st && cudaStreamWaitEvent(pl->stream, pl->ev_join, 0) != cudaSuccess) st = cuda_fail(cudaGetLastError(), "join");
     if (!st) st = gpumem_find_mems(*hI, *hQ, pl->q_begin, pl->q_end, pl->stream, hM);
     return st;
 }
 
 void pipeline_release(gpumem_pipeline *pl) {  // graph, arena and the arena-backed handles
-    for (auto &it : pl->items) {
-        if (it.x) cudaGraphExecDestroy(it.x);
-        if (it.g) cudaGraphDestroy(it.g);
-    }
-    pl->items.clear();
+    if (pl->exec) cudaGraphExecDestroy(pl->exec);
+    if (pl->graph) cudaGraphDestroy(pl->graph);
+    pl->exec = nullptr;
+    pl->graph = nullptr;
     if (pl->R) { pl->R->magic = 0; delete pl->R; }
     if (pl->Q) { pl->Q->magic = 0; delete pl->Q; }
     if (pl->idx) { pl->idx->magic = 0; delete pl->idx; }
@@ -504,26 +467,27 @@ gpumem_status pipeline_capture(gpumem_pipeline *pl, const char *R, const char *Q
     c.deferred = true;
     c.host = pl->host;
     c.recs = &pl->recs;
-    c.items = &pl->items;
     c.expect_n = pl->host[0];
     CK(cudaStreamBeginCapture(s, cudaStreamCaptureModeRelaxed), "begin capture");
     const uint64_t l0 = g_launches.load();
     t_cap = &c;
     st = pipeline_path(pl, R, Q, &pl->R, &pl->Q, &pl->idx, &pl->mems);
-    if (!st) cap_cut(s, nullptr);  // the last segment (a fresh capture is left open)
     t_cap = nullptr;
     pl->launches = g_launches.load() - l0;
     g_launches.fetch_sub(pl->launches);      // captured, not launched
-    cudaGraph_t rest = nullptr;
-    const cudaError_t ce = cudaStreamEndCapture(s, &rest);
-    if (rest) cudaGraphDestroy(rest);
+    const cudaError_t ce = cudaStreamEndCapture(s, &pl->graph);
     if (st) {
         pipeline_release(pl);
         return st;
     }
-    if (c.err != cudaSuccess || ce != cudaSuccess) {
+    if (ce != cudaSuccess) {
         pipeline_release(pl);
-        return cuda_fail(c.err != cudaSuccess ? c.err : ce, "pipeline capture");
+        return cuda_fail(ce, "pipeline capture");
+    }
+    const cudaError_t ie = cudaGraphInstantiate(&pl->exec, pl->graph, 0);
+    if (ie != cudaSuccess) {
+        pipeline_release(pl);
+        return cuda_fail(ie, "graph instantiate");
     }
     pl->out_cap = c.out_cap;
     pl->coop_cap = c.coop_cap;
@@ -534,24 +498,16 @@ gpumem_status pipeline_capture(gpumem_pipeline *pl, const char *R, const char *Q
     return GPUMEM_OK;
 }
 
-// One run: the graph segments and stage events in order; with host inputs the
-// segments that read R / Q first wait for their copy.
+// One run = one graph launch. Device-input runs record the copy events first so the
+// graph's external waits on them are satisfied at once.
 cudaError_t pipeline_launch(gpumem_pipeline *pl, bool host_inputs) {
-    cudaError_t e = cudaStreamWaitEvent(pl->side, pl->ev_in, 0);  // fork: the side stream starts with the run
-    if (e != cudaSuccess) return e;
-    for (const auto &it : pl->items) {
-        cudaStream_t st = it.sid ? pl->side : pl->stream;
-        if (it.x) e = cudaGraphLaunch(it.x, st);
-        else if (it.ev) e = cudaEventRecord(it.ev, st);
-        else if (it.wait == 3) {  // join
-            e = cudaEventRecord(pl->ev_join, pl->side);
-            if (e == cudaSuccess) e = cudaStreamWaitEvent(pl->stream, pl->ev_join, 0);
-        } else if (host_inputs) {
-            e = cudaStreamWaitEvent(st, it.wait == 1 ? pl->ev_r : pl->ev_q, 0);
-        }
+    cudaError_t e = cudaSuccess;
+    if (!host_inputs) {
+        e = cudaEventRecord(pl->ev_r, pl->stream);
+        if (e == cudaSuccess) e = cudaEventRecord(pl->ev_q, pl->stream);
         if (e != cudaSuccess) return e;
     }
-    return cudaSuccess;
+    return cudaGraphLaunch(pl->exec, pl->stream);
 }
 
 }  // namespace
@@ -684,10 +640,11 @@ void gpumem_free(void *handle) {
         if (pl->stage) {
             cudaStreamSynchronize(pl->copy);
             cudaFree(pl->stage);
-            cudaEventDestroy(pl->ev_r);
-            cudaEventDestroy(pl->ev_q);
             cudaStreamDestroy(pl->copy);
         }
+        cudaEventDestroy(pl->ev_r);
+        cudaEventDestroy(pl->ev_q);
+        cudaEventDestroy(pl->ev_fork);
         ws_release_stream(pl->device, pl->stream);
         cudaStreamSynchronize(pl->side);
         cudaStreamDestroy(pl->side);
@@ -1241,6 +1198,9 @@ gpumem_status gpumem_pipeline_create(uint64_t r_len, uint64_t q_len, uint32_t se
     if (cudaStreamCreateWithFlags(&pl->stream, cudaStreamNonBlocking) != cudaSuccess ||
         cudaStreamCreateWithFlags(&pl->side, cudaStreamNonBlocking) != cudaSuccess ||
         cudaEventCreateWithFlags(&pl->ev_join, cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreateWithFlags(&pl->ev_fork, cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreateWithFlags(&pl->ev_r, cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreateWithFlags(&pl->ev_q, cudaEventDisableTiming) != cudaSuccess ||
         cudaEventCreateWithFlags(&pl->ev_in, cudaEventDisableTiming) != cudaSuccess ||
         cudaEventCreateWithFlags(&pl->ev_out, cudaEventDisableTiming) != cudaSuccess) {
         const cudaError_t e = cudaGetLastError();
@@ -1274,7 +1234,7 @@ gpumem_status gpumem_pipeline_run(gpumem_pipeline *pl, const char *r_bases_dev, 
     }
     CK(cudaEventRecord(pl->ev_in, pl->user), "event");  // inputs written on the caller's stream
     CK(cudaStreamWaitEvent(pl->stream, pl->ev_in, 0), "wait");
-    if (pl->items.empty() || pl->inR != r_bases_dev || pl->inQ != q_bases_dev) {
+    if (!pl->exec || pl->inR != r_bases_dev || pl->inQ != q_bases_dev) {
         const gpumem_status st = pipeline_capture(pl, r_bases_dev, q_bases_dev);
         if (st) return st;
     }
@@ -1299,8 +1259,6 @@ gpumem_status gpumem_pipeline_run_host(gpumem_pipeline *pl, const char *r_bases_
     if (!pl->stage) {
         CK(cudaMalloc(&pl->stage, pl->nR + pl->nQ + 256), "input staging");
         CK(cudaStreamCreateWithFlags(&pl->copy, cudaStreamNonBlocking), "copy stream");
-        CK(cudaEventCreateWithFlags(&pl->ev_r, cudaEventDisableTiming), "event");
-        CK(cudaEventCreateWithFlags(&pl->ev_q, cudaEventDisableTiming), "event");
     }
     char *dR = pl->stage, *dQ = pl->stage + pl->nR;
     // the copies start after the caller's prior work and after the previous run (which
@@ -1313,7 +1271,7 @@ gpumem_status gpumem_pipeline_run_host(gpumem_pipeline *pl, const char *r_bases_
     if (pl->nQ) CK(cudaMemcpyAsync(dQ, q_bases_host, pl->nQ, cudaMemcpyHostToDevice, pl->copy), "H2D Q");
     CK(cudaEventRecord(pl->ev_q, pl->copy), "event");
     CK(cudaStreamWaitEvent(pl->stream, pl->ev_in, 0), "wait");
-    if (pl->items.empty() || pl->inR != dR || pl->inQ != dQ) {
+    if (!pl->exec || pl->inR != dR || pl->inQ != dQ) {
         CK(cudaStreamWaitEvent(pl->stream, pl->ev_q, 0), "wait");  // the measuring run reads both
         const gpumem_status st = pipeline_capture(pl, dR, dQ);
         if (st) return st;
