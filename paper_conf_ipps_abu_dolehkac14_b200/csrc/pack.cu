@@ -24,11 +24,6 @@ __device__ __forceinline__ uint32_t pack4(uint32_t x, bool &ok) {
     return (c * 0x40100401u) >> 24;                                  // c0<<6|c1<<4|c2<<2|c3
 }
 
-#ifndef GM_PACK_WPT
-#define GM_PACK_WPT 4
-#endif
-constexpr int kWPT = GM_PACK_WPT;  // output words per thread (all input loads issued first)
-
 // word w from 32 ASCII bytes (the scalar path handles unaligned input and the tail)
 __device__ __forceinline__ uint64_t pack_word_scalar(const uint8_t *__restrict__ in, uint64_t n, uint64_t w,
                                                      unsigned long long *bad_pos) {
@@ -56,38 +51,53 @@ __device__ __noinline__ void report_bad(const uint8_t *__restrict__ in, uint64_t
     }
 }
 
-// Thread t packs words t, t + T, ..., t + (kWPT - 1) T of its CTA's span (T = threads):
-// every load of the thread is in flight before the first word is assembled.
+// Aligned input: thread t of a CTA takes the 16-byte halves t, t + T, ... (T = threads;
+// kHPT of them, all loads in flight first), so every warp load instruction reads 512
+// contiguous bytes; a half packs to 32 bits and the even lane of each pair assembles
+// the 64-bit word with its odd neighbour's half (one shuffle) and stores it -- each
+// input sector is requested exactly once. Words from n_full on (the partial last word
+// and the zero padding) and unaligned inputs take the scalar path.
+#ifndef GM_PACK_HPT
+#define GM_PACK_HPT 8
+#endif
+constexpr int kHPT = GM_PACK_HPT;  // halves per thread
+
+__device__ __forceinline__ uint32_t pack16(const uint4 v, bool &ok) {
+    return (pack4(v.x, ok) << 24) | (pack4(v.y, ok) << 16) | (pack4(v.z, ok) << 8) | pack4(v.w, ok);
+}
+
 __global__ void __launch_bounds__(kPackThreads) k_pack(const uint8_t *__restrict__ in, uint64_t n,
                                                        uint64_t *__restrict__ words, uint64_t n_full,
                                                        uint64_t n_words_alloc, unsigned long long *bad_pos,
                                                        int aligned) {
-    const uint64_t w0 = uint64_t(blockIdx.x) * kPackThreads * kWPT + threadIdx.x;
-    uint4 a[kWPT], b[kWPT];
+    const int lane = threadIdx.x & 31;
+    if (aligned) {
+        const uint64_t n_halves = 2 * n_full;
+        const uint64_t h0 = uint64_t(blockIdx.x) * kPackThreads * kHPT + threadIdx.x;
+        uint4 v[kHPT];
 #pragma unroll
-    for (int k = 0; k < kWPT; ++k) {
-        const uint64_t w = w0 + uint64_t(k) * kPackThreads;
-        if (aligned && w < n_full) {
-            a[k] = __ldcs(reinterpret_cast<const uint4 *>(in) + 2 * w);  // streamed once
-            b[k] = __ldcs(reinterpret_cast<const uint4 *>(in) + 2 * w + 1);
+        for (int k = 0; k < kHPT; ++k) {
+            const uint64_t h = h0 + uint64_t(k) * kPackThreads;
+            if (h < n_halves) v[k] = __ldcs(reinterpret_cast<const uint4 *>(in) + h);  // streamed once
         }
-    }
 #pragma unroll
-    for (int k = 0; k < kWPT; ++k) {
-        const uint64_t w = w0 + uint64_t(k) * kPackThreads;
-        if (w >= n_words_alloc) break;
-        uint64_t word = 0;
-        if (aligned && w < n_full) {
+        for (int k = 0; k < kHPT; ++k) {
+            const uint64_t h = h0 + uint64_t(k) * kPackThreads;  // h's parity = the lane's parity
             bool ok = true;
-            const uint32_t v[8] = {a[k].x, a[k].y, a[k].z, a[k].w, b[k].x, b[k].y, b[k].z, b[k].w};
-#pragma unroll
-            for (int j = 0; j < 8; ++j) word |= uint64_t(pack4(v[j], ok)) << (56 - 8 * j);
-            if (!ok) report_bad(in, w, bad_pos);
-        } else {
-            word = pack_word_scalar(in, n, w, bad_pos);
+            const uint32_t half = h < n_halves ? pack16(v[k], ok) : 0u;
+            const uint32_t odd = __shfl_down_sync(0xffffffffu, half, 1);
+            if (h < n_halves) {
+                if (!ok) report_bad(in, h >> 1, bad_pos);  // the word's first bad byte (either half)
+                if (!(lane & 1)) words[h >> 1] = (uint64_t(half) << 32) | odd;
+            }
         }
-        words[w] = word;
     }
+    // scalar words: [n_full, n_words_alloc) always, all words for unaligned input
+    const uint64_t first = aligned ? n_full : 0;
+    const uint64_t tail = n_words_alloc - first;
+    const uint64_t per_cta = uint64_t(kPackThreads);
+    for (uint64_t i = uint64_t(blockIdx.x) * per_cta + threadIdx.x; i < tail; i += uint64_t(gridDim.x) * per_cta)
+        words[first + i] = pack_word_scalar(in, n, first + i, bad_pos);
 }
 
 // Reverse complement of a packed sequence (NEXT-F4): rc[i] = 3 - s[n-1-i] (A<->T, C<->G
@@ -132,7 +142,9 @@ cudaError_t launch_pack(const uint8_t *in, uint64_t n, uint64_t *words, uint64_t
                         unsigned long long *bad_pos, cudaStream_t s) {
     const int aligned = (reinterpret_cast<uintptr_t>(in) & 15) == 0;
     const uint64_t n_full = n / 32;
-    const uint64_t blocks = (n_words_alloc + uint64_t(kPackThreads) * kWPT - 1) / (uint64_t(kPackThreads) * kWPT);
+    const uint64_t per = uint64_t(kPackThreads) * kHPT;  // halves per CTA
+    uint64_t blocks = aligned ? (2 * n_full + per - 1) / per : (n_words_alloc + kPackThreads - 1) / kPackThreads;
+    if (blocks == 0) blocks = 1;
     k_pack<<<unsigned(blocks), kPackThreads, 0, s>>>(in, n, words, n_full, n_words_alloc, bad_pos, aligned);
     note_launch();
     return cudaGetLastError();

@@ -26,7 +26,7 @@ def _port():
     return p
 
 
-def _worker(rank, world, port, cfg, scale, q):
+def _worker(rank, world, port, cfg, scale, q, mode="direct"):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
@@ -35,12 +35,24 @@ def _worker(rank, world, port, cfg, scale, q):
         from paper_conf_ipps_abu_dolehkac14_b200 import synth
         from paper_conf_ipps_abu_dolehkac14_b200.dist import find_mems_sharded
         P = synth.make_pair(cfg, scale=scale)
-        merged, local = find_mems_sharded(torch.from_numpy(P.R).cuda(), torch.from_numpy(P.Q).cuda(), P.L, P.ls)
+        Rt, Qt = torch.from_numpy(P.R).cuda(), torch.from_numpy(P.Q).cuda()
+        if mode == "pipeline":  # the launch configuration bench.py times at N > 1
+            from paper_conf_ipps_abu_dolehkac14_b200.dist import ShardedPipeline
+            sp = ShardedPipeline(len(P.R), len(P.Q), P.L, P.ls)
+            for _ in range(2):
+                sp.run(Rt, Qt)
+                n = sp.finish()
+            merged, n_local = sp.merged, len(sp.pl)
+        else:
+            merged, local = find_mems_sharded(Rt, Qt, P.L, P.ls)
+            n_local = len(local)
         if rank == 0:
             import oracle
             got = merged.numpy()
             want = oracle.mems(P.R, P.Q, P.L, P.ls)
-            q.put(("ok", bool(np.array_equal(got, want)), len(want), len(local)))
+            if mode == "pipeline":
+                assert n == len(want)
+            q.put(("ok", bool(np.array_equal(got, want)), len(want), n_local))
     except Exception as e:  # pragma: no cover
         q.put(("err", repr(e)))
         raise
@@ -48,12 +60,13 @@ def _worker(rank, world, port, cfg, scale, q):
         dist.destroy_process_group()
 
 
+@pytest.mark.parametrize("mode", ["direct", "pipeline"])
 @pytest.mark.parametrize("world,cfg,scale", [(2, "c1", 1.0), (3, "c2", 0.2)])
-def test_sharded_find_gather_merge(world, cfg, scale):
+def test_sharded_find_gather_merge(world, cfg, scale, mode):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _port()
-    procs = [ctx.Process(target=_worker, args=(r, world, port, cfg, scale, q)) for r in range(world)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, cfg, scale, q, mode)) for r in range(world)]
     for p in procs:
         p.start()
     for p in procs:
