@@ -265,17 +265,25 @@ def run_ours(args, P):
     if dom in alg:
         n_launch = prof[dom][1] / args.steps
         achieved = alg[dom] / (kernel_ms[dom] / 1e3) / 1e9
-        traffic = None
+        traffic, sectors = None, None
         try:  # dram read+write bytes of that kernel from the committed ncu --set full capture
             t = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json"))).get(args.config)
             if t and dom == "find" and world == 1:
                 traffic = int(t["traffic_bytes"])
+                sectors = t.get("l1_ld_sectors")
         except Exception:
             pass
         roof = {"bound": "hbm", "kernel": dom, "achieved": round(achieved, 1), "peak": peak,
                 "peak_source": peak_src, "unit": "GB/s", "frac": round(achieved / peak, 4), "traffic": traffic,
                 "algorithmic_bytes_per_step": int(alg[dom]), "launches_per_step": n_launch,
                 "ms_per_step": round(kernel_ms[dom], 4)}
+        if sectors:  # what bounds k_find: 32-byte sector requests L1 -> L2, ceiling
+            # ~1 sector per SM clock; ncu's sector count over the live kernel time and SM clock
+            clk_mhz = (clk.summary().get("sm_mhz") or 1965.0)
+            rate = sectors / (torch.cuda.get_device_properties(dev).multi_processor_count * clk_mhz * 1e6
+                              * kernel_ms[dom] / 1e3 / n_launch)
+            roof["l1_sectors_per_launch"] = int(sectors)
+            roof["l1_sector_rate_per_sm_clk"] = round(rate, 3)
     stage_frac = {k: round(alg[k] / (kernel_ms[k] / 1e3) / 1e9 / peak, 4) for k in alg if k in kernel_ms}
 
     line = {"metric": METRIC, "value": round(value, 2), "unit": "Mbp/s", "n_gpus": world, "steps": args.steps,

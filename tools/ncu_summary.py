@@ -87,7 +87,8 @@ def full(path, out, traffic_json=None, config=None):
                     d = json.load(open(traffic_json))
                 except Exception:
                     d = {}
-                d[config] = {"kernel": "k_find", "traffic_bytes": t, "source": path}
+                sec = float(r[h.index("l1tex__t_sectors_pipe_lsu_mem_global_op_ld.sum")].replace(",", ""))
+                d[config] = {"kernel": "k_find", "traffic_bytes": t, "l1_ld_sectors": sec, "source": path}
                 json.dump(d, open(traffic_json, "w"), indent=1)
 
 
