@@ -49,7 +49,10 @@ constexpr int kT = 256;                   // threads per CTA
 constexpr int kWarps = kT / 32;
 constexpr int kQPT = 8;                   // query positions per lane per chunk
 constexpr int kChunk = 32 * kQPT;         // 256 positions per warp chunk
-constexpr uint32_t kGrab = 4;             // chunks per scheduler grab
+#ifndef GM_FIND_GRAB
+#define GM_FIND_GRAB 2
+#endif
+constexpr uint32_t kGrab = GM_FIND_GRAB;  // chunks per scheduler grab
 constexpr int kQW = kChunk / 32 + 6;      // staged Q words (chunk + left/right halo)
 constexpr uint32_t kSpillHits = 32;       // hits per heavy-queue piece (one per lane)
 constexpr int kOutBuf = 64;

@@ -39,7 +39,12 @@ constexpr int kLT = 512;                         // threads of k_bs_local
 constexpr int kLWarps = kLT / 32;
 constexpr int kItems = 8;                        // keys per thread in k_bs_local
 constexpr uint32_t kLocal = kLT * kItems;        // most keys one CTA sorts in shared memory (4096)
-constexpr uint32_t kSeg = kLocal / 2;            // segment spacing (slots)
+constexpr uint32_t kSeg = kLocal / 2;            // segment spacing (slots) for the grid size
+#ifndef GM_MSD_SEGMAX
+#define GM_MSD_SEGMAX (kLocal * 7 / 8)           // largest segment spacing k_bs_local picks (measured
+                                                 // 2048 / 3072 / 3584 / 4096: C4 0.149 / 0.113 / 0.113 / 0.113 ms,
+                                                 // C5 L = 50 0.437 / 0.400 / 0.380 / 0.381 ms)
+#endif
 constexpr int kMaxB = 14;                        // 16384 buckets: a 64 KB shared histogram
 
 __host__ __device__ __forceinline__ int choose_b(uint64_t n, int bits) {
@@ -79,30 +84,35 @@ __global__ void __launch_bounds__(kPT) k_bp_hist(const uint64_t *__restrict__ ke
     for (uint32_t i = threadIdx.x; i < nb; i += kPT) row[i] = h[i];
 }
 
-// per bucket b (one thread): counts[c][b] -> exclusive prefix over c (in place); totals[b]
+// per bucket b (one warp): counts[c][b] -> exclusive prefix over c (in place); totals[b].
+// Lane l owns a contiguous run of chunks; a warp scan joins the runs.
 __global__ void __launch_bounds__(256) k_bp_colscan(uint32_t *__restrict__ counts, uint32_t chunks, NSpec ns,
                                                     uint32_t *__restrict__ totals) {
     const uint32_t nb = 1u << choose_b(ns.n(), ns.bits);
-    const uint32_t b = blockIdx.x * 256 + threadIdx.x;
+    const uint32_t b = blockIdx.x * 8 + (threadIdx.x >> 5);
+    const int lane = threadIdx.x & 31;
     if (b >= nb) return;
-    uint32_t run = 0;
-    uint32_t c = 0;
-    for (; c + 8 <= chunks; c += 8) {  // independent loads in flight
-        uint32_t x[8];
+    const uint32_t per = (chunks + 31) / 32;
+    const uint32_t c0 = min(uint32_t(lane) * per, chunks), c1 = min(c0 + per, chunks);
+    uint32_t x[8], sum = 0;  // per <= 8 (chunks <= 256)
 #pragma unroll
-        for (int j = 0; j < 8; ++j) x[j] = counts[uint64_t(c + j) * nb + b];
+    for (int j = 0; j < 8; ++j) {
+        x[j] = c0 + j < c1 ? counts[uint64_t(c0 + j) * nb + b] : 0u;
+        sum += x[j];
+    }
+    uint32_t inc = sum;
 #pragma unroll
-        for (int j = 0; j < 8; ++j) {
-            counts[uint64_t(c + j) * nb + b] = run;
-            run += x[j];
-        }
+    for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
+        if (lane >= o) inc += y;
     }
-    for (; c < chunks; ++c) {
-        const uint32_t x = counts[uint64_t(c) * nb + b];
-        counts[uint64_t(c) * nb + b] = run;
-        run += x;
+    uint32_t run = inc - sum;
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+        if (c0 + j < c1) counts[uint64_t(c0 + j) * nb + b] = run;
+        run += x[j];
     }
-    totals[b] = run;
+    if (lane == 31) totals[b] = inc;
 }
 
 // exclusive scan of totals[0..nb) -> offs[0..nb] (offs[nb] = the sum); each thread owns
@@ -316,10 +326,18 @@ __global__ void __launch_bounds__(kLT, 2) k_bs_local(const uint32_t *__restrict_
     const uint64_t n = ns.n();
     const int bits = ns.bits;
     const uint32_t nb = 1u << ns.B(n);
-    for (uint64_t seg = blockIdx.x; seg * kSeg < n; seg += gridDim.x) {
+    // segment spacing: an even share of n over the grid in as few rounds as possible, a
+    // segment's cost being nearly independent of its size (every thread walks kItems
+    // slots per pass): up to kSegMax slots, leaving room below kLocal for the whole
+    // buckets that start in the segment (C4: 0.81 M keys over 296 blocks -> one round of
+    // 2.7 K-slot segments instead of 1-2 rounds of 2 K)
+    constexpr uint64_t kSegMax = GM_MSD_SEGMAX;
+    const uint64_t rounds = (n + uint64_t(gridDim.x) * kSegMax - 1) / (uint64_t(gridDim.x) * kSegMax);
+    const uint64_t seg_w = rounds ? (n + uint64_t(gridDim.x) * rounds - 1) / (uint64_t(gridDim.x) * rounds) : kSeg;
+    for (uint64_t seg = blockIdx.x; seg * seg_w < n; seg += gridDim.x) {
         __syncthreads();  // the previous segment's readers of s_b are done
-        if (threadIdx.x == 0) s_b[0] = first_at(offs, nb, seg * kSeg);
-        if (threadIdx.x == 32) s_b[1] = first_at(offs, nb, (seg + 1) * kSeg);
+        if (threadIdx.x == 0) s_b[0] = first_at(offs, nb, seg * seg_w);
+        if (threadIdx.x == 32) s_b[1] = first_at(offs, nb, (seg + 1) * seg_w);
         __syncthreads();
         const uint32_t b0 = s_b[0], b1 = s_b[1];
         if (b0 >= b1) continue;
@@ -330,14 +348,20 @@ __global__ void __launch_bounds__(kLT, 2) k_bs_local(const uint32_t *__restrict_
             smem_sort_write(S, tk, tv, lo, m, bits, out);
             continue;
         }
-        for (uint32_t b = b0; b < b1; ++b) {  // a large bucket in the segment: one bucket at a time
-            const uint32_t blo = offs[b], bm = offs[b + 1] - blo;
-            if (bm == 0) continue;
-            if (bm <= kLocal) {
-                smem_sort_write(S, tk, tv, blo, bm, bits, out);
-            } else if (threadIdx.x == 0) {
-                big[atomicAdd(n_big, 1u)] = b;
+        // a large bucket in the segment: runs of consecutive buckets of <= kLocal keys in
+        // all, each sorted as one (buckets are ordered by their prefix); a bucket past
+        // kLocal alone goes to k_bs_big
+        for (uint32_t b = b0; b < b1;) {
+            const uint32_t blo = offs[b];
+            if (offs[b + 1] - blo > kLocal) {
+                if (threadIdx.x == 0) big[atomicAdd(n_big, 1u)] = b;
+                ++b;
+                continue;
             }
+            uint32_t e = b + 1;
+            while (e < b1 && offs[e + 1] - blo <= kLocal) ++e;
+            if (offs[e] > blo) smem_sort_write(S, tk, tv, blo, offs[e] - blo, bits, out);
+            b = e;
         }
     }
 }
@@ -473,11 +497,11 @@ static cudaError_t msd_run(uint64_t *keys, uint32_t *vals, NSpec ns, void *scrat
         attr = true;
     }
     k_bp_hist<<<chunks, kPT, nb_max * 4, s>>>(keys, ns, counts);
-    k_bp_colscan<<<(nb_max + 255) / 256, 256, 0, s>>>(counts, chunks, ns, totals);
+    k_bp_colscan<<<(nb_max + 7) / 8, 256, 0, s>>>(counts, chunks, ns, totals);
     k_bs_scan<<<1, 1024, 0, s>>>(totals, ns, offs);
     k_bp_scatter<<<chunks, kPT, nb_max * 4, s>>>(keys, vals, ns, counts, offs, tk, tv);
     uint64_t segs = (cap + kSeg - 1) / kSeg;
-    if (ns.dn && segs > uint64_t(2 * num_sms())) segs = 2 * num_sms();  // blocks loop over the segments
+    if (segs > uint64_t(2 * num_sms())) segs = 2 * num_sms();  // blocks loop over the segments
     k_bs_local<<<unsigned(segs ? segs : 1), kLT, sizeof(LocalSmem), s>>>(offs, ns, tk, tv, out, big, n_big);
     // oversized buckets: ping-pong with the input's range of the bucket (free: the scatter
     // consumed it and the local pass wrote only other buckets' ranges)
