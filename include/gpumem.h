@@ -258,6 +258,9 @@ gpumem_status gpumem_set_allocator(void *(*alloc_fn)(size_t bytes, void *cuda_st
  *  "rank_sectors"     lookup directory: -1 (default) auto, 0 rank words, 1 rank sectors
  *  "small_sort"       1: single-launch cooperative radix sorts (index and output) when
  *                     the input fits in shared memory; 0 (default): multi-launch
+ *  "pdl"              1 (default): programmatic dependent launch between consecutive
+ *                     kernels (each waits for its predecessor with griddepcontrol.wait);
+ *                     0: ordinary launches
  *  "radix_bits"       LSD digit width: 0 (default) = 9 bits when that saves a pass, else 8;
  *                     or pinned to 8, 9, 10; anything else is GPUMEM_ERR_ARG
  * Unknown names are GPUMEM_ERR_ARG. */

@@ -427,6 +427,7 @@ __device__ __forceinline__ void drain_deferred(const FindParams &P, WarpSmem &s,
 #endif
 template <bool kStatic, bool kHints, bool kSect, bool kRec8>
 __global__ void __launch_bounds__(kT, GM_FIND_MINB) k_find(const FindParams P) {
+    pdl_wait();
     constexpr int kL = kRec8 ? 8 : 16, kR = kRec8 ? 8 : 32;  // record flank widths (bases)
     __shared__ WarpSmem smem[kWarps];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
@@ -643,6 +644,7 @@ __global__ void __launch_bounds__(kT, GM_FIND_MINB) k_find(const FindParams P) {
 // K7: drain the heavy-bucket queue, one 32-hit piece per warp iteration.
 template <bool kRec8>
 __global__ void __launch_bounds__(kT) k_heavy(const FindParams P) {
+    pdl_wait();
     constexpr int kL = kRec8 ? 8 : 16, kR = kRec8 ? 8 : 32;
     __shared__ WarpSmem smem[kWarps];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
@@ -675,6 +677,7 @@ __global__ void __launch_bounds__(kT) k_heavy(const FindParams P) {
 // Drain the coop queue: 32 deferred hits per warp iteration, decided from scratch
 // with per-lane extension up to kLaneCap and warp-cooperative extension beyond.
 __global__ void __launch_bounds__(kT) k_coop(const FindParams P) {
+    pdl_wait();
     __shared__ WarpSmem smem[kWarps];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     WarpSmem &s = smem[wid];
@@ -722,11 +725,11 @@ cudaError_t launch_find(const FindParams &p, int grid, cudaStream_t s) {
 #define GM_FIND_LAUNCH(ST, HI)                                                              \
     do {                                                                                    \
         if (sect) {                                                                         \
-            if (p.rec8) k_find<ST, HI, true, true><<<grid, kT, 0, s>>>(p);                  \
-            else k_find<ST, HI, true, false><<<grid, kT, 0, s>>>(p);                        \
+            if (p.rec8) pdl_launch(k_find<ST, HI, true, true>, grid, kT, 0, s, p);                  \
+            else pdl_launch(k_find<ST, HI, true, false>, grid, kT, 0, s, p);                        \
         } else {                                                                            \
-            if (p.rec8) k_find<ST, HI, false, true><<<grid, kT, 0, s>>>(p);                 \
-            else k_find<ST, HI, false, false><<<grid, kT, 0, s>>>(p);                       \
+            if (p.rec8) pdl_launch(k_find<ST, HI, false, true>, grid, kT, 0, s, p);                 \
+            else pdl_launch(k_find<ST, HI, false, false>, grid, kT, 0, s, p);                       \
         }                                                                                   \
     } while (0)
     if (p.static_lb) GM_FIND_LAUNCH(true, false);
@@ -738,14 +741,14 @@ cudaError_t launch_find(const FindParams &p, int grid, cudaStream_t s) {
 }
 
 cudaError_t launch_coop(const FindParams &p, cudaStream_t s) {
-    k_coop<<<num_sms() * 2, kT, 0, s>>>(p);
+    pdl_launch(k_coop, num_sms() * 2, kT, 0, s, p);
     note_launch();
     return cudaGetLastError();
 }
 
 cudaError_t launch_heavy(const FindParams &p, cudaStream_t s) {
-    if (p.rec8) k_heavy<true><<<num_sms() * 4, kT, 0, s>>>(p);
-    else k_heavy<false><<<num_sms() * 4, kT, 0, s>>>(p);
+    if (p.rec8) pdl_launch(k_heavy<true>, num_sms() * 4, kT, 0, s, p);
+    else pdl_launch(k_heavy<false>, num_sms() * 4, kT, 0, s, p);
     note_launch();
     return cudaGetLastError();
 }

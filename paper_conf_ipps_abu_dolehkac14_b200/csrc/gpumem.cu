@@ -559,6 +559,7 @@ gpumem_status gpumem_set_option(const char *name, int64_t value) {
         g_opt.sort_impl = value;
     }
     else if (!strcmp(name, "index_msd")) g_opt.index_msd = value ? 1 : 0;
+    else if (!strcmp(name, "pdl")) g_opt.pdl = value ? 1 : 0;
     else if (!strcmp(name, "index_fused")) g_opt.index_fused = value ? 1 : 0;
     else if (!strcmp(name, "small_sort")) g_opt.small_sort = value ? 1 : 0;
     else if (!strcmp(name, "rec8")) g_opt.rec8 = value < 0 ? -1 : (value ? 1 : 0);

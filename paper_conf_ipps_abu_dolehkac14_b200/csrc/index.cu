@@ -45,6 +45,7 @@ __global__ void __launch_bounds__(kCodeThreads) k_seed_codes(const uint64_t *__r
                                                              uint32_t step, uint64_t k0, uint64_t n_locs,
                                                              uint32_t *__restrict__ codes,
                                                              uint32_t *__restrict__ locs) {
+    pdl_wait();
     const uint64_t k = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
     if (k >= n_locs) return;
     const uint64_t p = (k0 + k) * step;
@@ -56,6 +57,7 @@ __global__ void __launch_bounds__(kCodeThreads) k_seed_codes(const uint64_t *__r
 // c in [0, n_chunks]; written by the element at each chunk boundary (no searches).
 __global__ void __launch_bounds__(kCodeThreads) k_chunk_bounds(const uint32_t *__restrict__ codes, uint64_t n,
                                                                uint64_t n_chunks, uint32_t *__restrict__ first) {
+    pdl_wait();
     const uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
     if (i > n) return;
     const uint64_t c_prev = i == 0 ? 0 : uint64_t(codes[i - 1]) / kChunk + 1;  // chunks after codes[i-1]'s
@@ -68,6 +70,7 @@ __global__ void __launch_bounds__(kCodeThreads) k_chunk_bounds(const uint32_t *_
 __global__ void __launch_bounds__(kCodeThreads) k_occ_count(const uint32_t *__restrict__ codes,
                                                             const uint32_t *__restrict__ first,
                                                             uint32_t *__restrict__ occ) {
+    pdl_wait();
     __shared__ uint32_t ws[kCodeThreads / 32];
     const uint32_t c = blockIdx.x;
     const uint64_t lo = first[c], hi = first[c + 1];
@@ -87,6 +90,7 @@ __global__ void __launch_bounds__(kCodeThreads) k_occ_count(const uint32_t *__re
 // rank0[c] = exclusive prefix of occ over the chunks (one CTA, contiguous runs per thread)
 __global__ void __launch_bounds__(1024) k_occ_scan(const uint32_t *__restrict__ occ, uint32_t n,
                                                    uint32_t *__restrict__ rank0) {
+    pdl_wait();
     __shared__ uint32_t ws[32];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     const uint32_t per = (n + 1023) / 1024;
@@ -117,6 +121,7 @@ __global__ void __launch_bounds__(kFillThreads) k_ptrs_fill(const uint32_t *__re
                                                             uint2 *__restrict__ buckets,
                                                             const uint32_t *__restrict__ chunk_first,
                                                             const uint32_t *__restrict__ rank0) {
+    pdl_wait();
     extern __shared__ uint32_t cnt[];                // kChunk + kChunk / 32: a pad word per 32 (conflict-free rows)
     __shared__ uint32_t wsum[kFillThreads / 32];
     __shared__ uint32_t wocc[kFillThreads / 32];
@@ -234,6 +239,7 @@ __global__ void __launch_bounds__(kDirThreads) k_dir_fill(const uint32_t *__rest
                                                           uint4 *__restrict__ rsect, uint2 *__restrict__ buckets,
                                                           const uint32_t *__restrict__ chunk_first,
                                                           const uint32_t *__restrict__ rank0) {
+    pdl_wait();
     __shared__ uint32_t occ[kGroups], ecnt[kGroups], c2lo[kGroups], c2hi[kGroups];
     __shared__ uint32_t hpos[kDirThreads + 1];
     __shared__ uint32_t wsum[kDirThreads / 32];
@@ -350,6 +356,7 @@ template <bool kRec8>
 __global__ void __launch_bounds__(kCodeThreads) k_seed_recs(const uint64_t *__restrict__ R, uint32_t ls,
                                                             const uint32_t *__restrict__ locs, uint64_t n_locs,
                                                             void *__restrict__ recs) {
+    pdl_wait();
     const uint64_t k = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
     if (k >= n_locs) return;
     const uint32_t p = locs[k];
@@ -455,6 +462,7 @@ __global__ void __launch_bounds__(kFillThreads) k_index_local(
     unsigned long long *__restrict__ rankw, uint4 *__restrict__ rsect, uint2 *__restrict__ buckets,
     uint32_t *__restrict__ locs, void *__restrict__ recs, uint32_t *__restrict__ slot, unsigned long long *status,
     unsigned int *ticket) {
+    pdl_wait();
     extern __shared__ uint32_t cnt[];                // kChunk + kChunk / 32 (a pad word per 32 counters)
     __shared__ uint32_t wsum[kFillThreads / 32];
     __shared__ uint32_t wocc[kFillThreads / 32];
@@ -589,8 +597,8 @@ cudaError_t launch_seed_recs(const uint64_t *R, uint32_t ls, const uint32_t *loc
                              int rec8, cudaStream_t s) {
     if (n_locs == 0) return cudaSuccess;
     const uint64_t blocks = (n_locs + kCodeThreads - 1) / kCodeThreads;
-    if (rec8) k_seed_recs<true><<<unsigned(blocks), kCodeThreads, 0, s>>>(R, ls, locs, n_locs, recs);
-    else k_seed_recs<false><<<unsigned(blocks), kCodeThreads, 0, s>>>(R, ls, locs, n_locs, recs);
+    if (rec8) pdl_launch(k_seed_recs<true>, unsigned(blocks), kCodeThreads, 0, s, R, ls, locs, n_locs, recs);
+    else pdl_launch(k_seed_recs<false>, unsigned(blocks), kCodeThreads, 0, s, R, ls, locs, n_locs, recs);
     note_launch();
     return cudaGetLastError();
 }
@@ -599,7 +607,7 @@ cudaError_t launch_seed_codes(const uint64_t *R, uint32_t ls, uint32_t step, uin
                               uint32_t *codes, uint32_t *locs, cudaStream_t s) {
     if (n_locs == 0) return cudaSuccess;
     const uint64_t blocks = (n_locs + kCodeThreads - 1) / kCodeThreads;
-    k_seed_codes<<<unsigned(blocks), kCodeThreads, 0, s>>>(R, ls, step, k0, n_locs, codes, locs);
+    pdl_launch(k_seed_codes, unsigned(blocks), kCodeThreads, 0, s, R, ls, step, k0, n_locs, codes, locs);
     note_launch();
     return cudaGetLastError();
 }
@@ -613,6 +621,7 @@ __global__ void __launch_bounds__(256) k_ptrs_expand(const unsigned long long *_
                                                      const uint4 *__restrict__ rsect,
                                                      const uint2 *__restrict__ buckets, uint64_t nb, uint64_t n_locs,
                                                      uint32_t *__restrict__ ptrs) {
+    pdl_wait();
     constexpr uint64_t kLo = 0x5555555555555555ull;
     auto rank_of = [&](uint64_t s, bool &in) -> uint64_t {  // occupied seeds in [0, s) (+ s's own occupancy)
         const uint32_t b = uint32_t(s & 31);
@@ -645,8 +654,8 @@ cudaError_t launch_ptrs_expand(const unsigned long long *rankw, const uint4 *rse
                                uint64_t n_locs, uint32_t *ptrs, cudaStream_t s) {
     const uint64_t nb = 1ull << (2 * ls);
     const unsigned grid = unsigned(std::min<uint64_t>((nb + 1 + 255) / 256, uint64_t(num_sms()) * 16));
-    if (rsect) k_ptrs_expand<true><<<grid, 256, 0, s>>>(rankw, rsect, buckets, nb, n_locs, ptrs);
-    else k_ptrs_expand<false><<<grid, 256, 0, s>>>(rankw, rsect, buckets, nb, n_locs, ptrs);
+    if (rsect) pdl_launch(k_ptrs_expand<true>, grid, 256, 0, s, rankw, rsect, buckets, nb, n_locs, ptrs);
+    else pdl_launch(k_ptrs_expand<false>, grid, 256, 0, s, rankw, rsect, buckets, nb, n_locs, ptrs);
     note_launch();
     return cudaGetLastError();
 }
@@ -670,10 +679,10 @@ cudaError_t launch_ptrs_fill(const uint32_t *sorted_codes, uint64_t n_locs, uint
     a = align(a + (chunks + 1) * 4);
     auto *rank0 = reinterpret_cast<uint32_t *>(a);
     cudaError_t e = cudaSuccess;
-    k_chunk_bounds<<<unsigned((n_locs + 1 + kCodeThreads - 1) / kCodeThreads), kCodeThreads, 0, s>>>(
+    pdl_launch(k_chunk_bounds, unsigned((n_locs + 1 + kCodeThreads - 1) / kCodeThreads), kCodeThreads, 0, s, 
         sorted_codes, n_locs, chunks, first);
-    k_occ_count<<<unsigned(chunks), kCodeThreads, 0, s>>>(sorted_codes, first, occ);
-    k_occ_scan<<<1, 1024, 0, s>>>(occ, uint32_t(chunks), rank0);
+    pdl_launch(k_occ_count, unsigned(chunks), kCodeThreads, 0, s, sorted_codes, first, occ);
+    pdl_launch(k_occ_scan, 1, 1024, 0, s, occ, uint32_t(chunks), rank0);
     constexpr int smem = (kChunk + kChunk / 32) * 4;
     static bool attr = false;
     if (!attr) {
@@ -688,16 +697,16 @@ cudaError_t launch_ptrs_fill(const uint32_t *sorted_codes, uint64_t n_locs, uint
     // 0.33 vs 0.46 ms) keeps the seed-driven fill with its ptrs write-out skipped
     if (!ptrs && n_locs * 4 < nb) {
         if (rsect)
-            k_dir_fill<true><<<unsigned(chunks), kDirThreads, 0, s>>>(sorted_codes, nb, rankw, rsect, buckets, first,
+            pdl_launch(k_dir_fill<true>, unsigned(chunks), kDirThreads, 0, s, sorted_codes, nb, rankw, rsect, buckets, first,
                                                                       rank0);
         else
-            k_dir_fill<false><<<unsigned(chunks), kDirThreads, 0, s>>>(sorted_codes, nb, rankw, rsect, buckets, first,
+            pdl_launch(k_dir_fill<false>, unsigned(chunks), kDirThreads, 0, s, sorted_codes, nb, rankw, rsect, buckets, first,
                                                                        rank0);
     } else if (rsect) {
-        k_ptrs_fill<true><<<unsigned(chunks), kFillThreads, smem, s>>>(sorted_codes, n_locs, nb, ptrs, rankw, rsect,
+        pdl_launch(k_ptrs_fill<true>, unsigned(chunks), kFillThreads, smem, s, sorted_codes, n_locs, nb, ptrs, rankw, rsect,
                                                                        buckets, first, rank0);
     } else {
-        k_ptrs_fill<false><<<unsigned(chunks), kFillThreads, smem, s>>>(sorted_codes, n_locs, nb, ptrs, rankw, rsect,
+        pdl_launch(k_ptrs_fill<false>, unsigned(chunks), kFillThreads, smem, s, sorted_codes, n_locs, nb, ptrs, rankw, rsect,
                                                                         buckets, first, rank0);
     }
     note_launch(4);
@@ -728,7 +737,7 @@ cudaError_t launch_index_local(const uint32_t *codes, const uint32_t *ps, uint64
     auto *ticket = reinterpret_cast<unsigned int *>(a);
     cudaError_t e = cudaMemsetAsync(status, 0, (chunks * 8 + 255) / 256 * 256 + 4, s);
     if (e != cudaSuccess) return e;
-    k_chunk_bounds<<<unsigned((n_locs + 1 + kCodeThreads - 1) / kCodeThreads), kCodeThreads, 0, s>>>(codes, n_locs,
+    pdl_launch(k_chunk_bounds, unsigned((n_locs + 1 + kCodeThreads - 1) / kCodeThreads), kCodeThreads, 0, s, codes, n_locs,
                                                                                                     chunks, first);
     constexpr int smem = (kChunk + kChunk / 32) * 4;
     static bool attr = false;
@@ -742,7 +751,7 @@ cudaError_t launch_index_local(const uint32_t *codes, const uint32_t *ps, uint64
     }
     auto kern = rsect ? (rec8 ? k_index_local<true, true> : k_index_local<true, false>)
                       : (rec8 ? k_index_local<false, true> : k_index_local<false, false>);
-    kern<<<unsigned(chunks), kFillThreads, smem, s>>>(codes, ps, n_locs, nb, R, ls, first, ptrs, rankw, rsect, buckets,
+    pdl_launch(kern, unsigned(chunks), kFillThreads, smem, s, codes, ps, n_locs, nb, R, ls, first, ptrs, rankw, rsect, buckets,
                                                      locs, recs, slot, status, ticket);
     note_launch(2);
     return cudaGetLastError();

@@ -2,6 +2,7 @@
 // Not part of the ABI (see include/gpumem.h). No torch types anywhere.
 #pragma once
 #include <cstdint>
+#include <utility>
 #include <cuda_runtime.h>
 
 #include "gpumem.h"
@@ -27,8 +28,34 @@ struct Options {
     int64_t rank_sectors = -1;   // lookup directory: -1 auto (sectors when the compact table exceeds L2/4),
                                  // 0 rank words, 1 rank sectors       // index sort: 1 = MSD bucket sort of (code << 32 | p), 0 = stable LSD radix
     int64_t radix_bits = 0;      // LSD digit width: 0 = 9 bits if that saves a pass else 8; or pinned 8, 9, 10
+    int64_t pdl = 1;             // programmatic dependent launch between consecutive kernels
 };
 extern Options g_opt;
+
+// Kernel launch with programmatic dependent launch (PDL): the next kernel on the stream
+// may be scheduled while this one drains (its CTAs fill the SMs freed by finished
+// ones); every kernel of the library begins with pdl_wait() (griddepcontrol.wait),
+// which blocks until the preceding grid has completed and its writes are visible, so
+// the overlap covers only launch latency and CTA ramp-up. In a captured graph the
+// attribute becomes a programmatic dependency edge. g_opt.pdl = 0: ordinary launches.
+template <typename... KArgs, typename... Args>
+inline cudaError_t pdl_launch(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t s,
+                              Args &&...args) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = g_opt.pdl ? 1 : 0;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, kernel, std::forward<Args>(args)...);
+}
+#ifdef __CUDACC__
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+#endif
 
 void *dalloc(size_t bytes, cudaStream_t s);   // nullptr on failure (error text set)
 void dfree(void *p, cudaStream_t s);

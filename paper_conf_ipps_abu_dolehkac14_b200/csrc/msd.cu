@@ -70,6 +70,7 @@ struct NSpec {
 // chunk c = elements [c * cs, min((c + 1) * cs, n))
 __global__ void __launch_bounds__(kPT) k_bp_hist(const uint64_t *__restrict__ keys, NSpec ns,
                                                  uint32_t *__restrict__ counts) {
+    pdl_wait();
     extern __shared__ uint32_t h[];
     const uint64_t n = ns.n();
     const int B = choose_b(n, ns.bits), shift = ns.bits - B;
@@ -88,6 +89,7 @@ __global__ void __launch_bounds__(kPT) k_bp_hist(const uint64_t *__restrict__ ke
 // Lane l owns a contiguous run of chunks; a warp scan joins the runs.
 __global__ void __launch_bounds__(256) k_bp_colscan(uint32_t *__restrict__ counts, uint32_t chunks, NSpec ns,
                                                     uint32_t *__restrict__ totals) {
+    pdl_wait();
     const uint32_t nb = 1u << choose_b(ns.n(), ns.bits);
     const uint32_t b = blockIdx.x * 8 + (threadIdx.x >> 5);
     const int lane = threadIdx.x & 31;
@@ -119,6 +121,7 @@ __global__ void __launch_bounds__(256) k_bp_colscan(uint32_t *__restrict__ count
 // a contiguous run of ceil(nb / 1024) entries
 __global__ void __launch_bounds__(1024) k_bs_scan(const uint32_t *__restrict__ totals, NSpec ns,
                                                   uint32_t *__restrict__ offs) {
+    pdl_wait();
     __shared__ uint32_t ws[32];
     const uint32_t nb = 1u << choose_b(ns.n(), ns.bits);
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
@@ -148,6 +151,7 @@ __global__ void __launch_bounds__(kPT) k_bp_scatter(const uint64_t *__restrict__
                                                     const uint32_t *__restrict__ rel,
                                                     const uint32_t *__restrict__ offs, uint64_t *__restrict__ ok,
                                                     uint32_t *__restrict__ ov) {
+    pdl_wait();
     extern __shared__ uint32_t cur[];
     const uint64_t n = ns.n();
     const int B = choose_b(n, ns.bits), shift = ns.bits - B;
@@ -320,6 +324,7 @@ __device__ void smem_sort_write(LocalSmem &S, const uint64_t *__restrict__ tk, c
 __global__ void __launch_bounds__(kLT, 2) k_bs_local(const uint32_t *__restrict__ offs, NSpec ns,
                                                  const uint64_t *__restrict__ tk, const uint32_t *__restrict__ tv,
                                                  Out out, uint32_t *__restrict__ big, unsigned int *n_big) {
+    pdl_wait();
     extern __shared__ __align__(16) unsigned char smem[];
     LocalSmem &S = *reinterpret_cast<LocalSmem *>(smem);
     __shared__ uint32_t s_b[2];
@@ -371,6 +376,7 @@ __global__ void __launch_bounds__(kLT, 2) k_bs_local(const uint32_t *__restrict_
 __global__ void __launch_bounds__(kT) k_bs_big(const uint32_t *__restrict__ offs, const uint32_t *__restrict__ big,
                                                const unsigned int *__restrict__ n_big, uint64_t *tk, uint32_t *tv,
                                                uint64_t *xk, uint32_t *xv, NSpec ns, Out out) {
+    pdl_wait();
     __shared__ uint32_t hist[256];
     __shared__ uint32_t wcnt[kWarps][256];
     __shared__ uint32_t ws[kWarps];
@@ -496,16 +502,16 @@ static cudaError_t msd_run(uint64_t *keys, uint32_t *vals, NSpec ns, void *scrat
         cudaFuncSetAttribute(k_bs_local, cudaFuncAttributeMaxDynamicSharedMemorySize, int(sizeof(LocalSmem)));
         attr = true;
     }
-    k_bp_hist<<<chunks, kPT, nb_max * 4, s>>>(keys, ns, counts);
-    k_bp_colscan<<<(nb_max + 7) / 8, 256, 0, s>>>(counts, chunks, ns, totals);
-    k_bs_scan<<<1, 1024, 0, s>>>(totals, ns, offs);
-    k_bp_scatter<<<chunks, kPT, nb_max * 4, s>>>(keys, vals, ns, counts, offs, tk, tv);
+    pdl_launch(k_bp_hist, chunks, kPT, nb_max * 4, s, keys, ns, counts);
+    pdl_launch(k_bp_colscan, (nb_max + 7) / 8, 256, 0, s, counts, chunks, ns, totals);
+    pdl_launch(k_bs_scan, 1, 1024, 0, s, totals, ns, offs);
+    pdl_launch(k_bp_scatter, chunks, kPT, nb_max * 4, s, keys, vals, ns, counts, offs, tk, tv);
     uint64_t segs = (cap + kSeg - 1) / kSeg;
     if (segs > uint64_t(2 * num_sms())) segs = 2 * num_sms();  // blocks loop over the segments
-    k_bs_local<<<unsigned(segs ? segs : 1), kLT, sizeof(LocalSmem), s>>>(offs, ns, tk, tv, out, big, n_big);
+    pdl_launch(k_bs_local, unsigned(segs ? segs : 1), kLT, sizeof(LocalSmem), s, offs, ns, tk, tv, out, big, n_big);
     // oversized buckets: ping-pong with the input's range of the bucket (free: the scatter
     // consumed it and the local pass wrote only other buckets' ranges)
-    k_bs_big<<<num_sms(), kT, 0, s>>>(offs, big, n_big, tk, tv, keys, xv, ns, out);
+    pdl_launch(k_bs_big, num_sms(), kT, 0, s, offs, big, n_big, tk, tv, keys, xv, ns, out);
     note_launch(6);
     return cudaGetLastError();
 }
@@ -531,6 +537,7 @@ cudaError_t msd_sort_dev(uint64_t *keys, uint32_t *vals, const unsigned long lon
 // already ordered by that prefix): one binary search per bucket.
 __global__ void __launch_bounds__(256) k_prefix_bounds(const uint64_t *__restrict__ keys, NSpec ns, int shift,
                                                        uint32_t nb, uint32_t *__restrict__ offs) {
+    pdl_wait();
     const uint64_t n = ns.n();
     for (uint32_t b = blockIdx.x * 256 + threadIdx.x; b <= nb; b += gridDim.x * 256) {
         uint64_t lo = 0, hi = n;
@@ -579,12 +586,12 @@ cudaError_t hybrid_sort_triples(uint64_t *keys, uint32_t *vals, uint64_t *k1, ui
         cudaFuncSetAttribute(k_bs_local, cudaFuncAttributeMaxDynamicSharedMemorySize, int(sizeof(LocalSmem)));
         attr = true;
     }
-    k_prefix_bounds<<<(nb + 256) / 256, 256, 0, s>>>(tk, ns, lo, nb, offs);
+    pdl_launch(k_prefix_bounds, (nb + 256) / 256, 256, 0, s, tk, ns, lo, nb, offs);
     uint64_t segs = (cap + kSeg - 1) / kSeg;
     if (segs > uint64_t(2 * num_sms())) segs = 2 * num_sms();  // blocks loop over the segments
     Out out{keys, vals, trip, qbits};
-    k_bs_local<<<unsigned(segs), kLT, sizeof(LocalSmem), s>>>(offs, ns, tk, tv, out, big, n_big);
-    k_bs_big<<<num_sms(), kT, 0, s>>>(offs, big, n_big, tk, tv, xk, xv, ns, out);
+    pdl_launch(k_bs_local, unsigned(segs), kLT, sizeof(LocalSmem), s, offs, ns, tk, tv, out, big, n_big);
+    pdl_launch(k_bs_big, num_sms(), kT, 0, s, offs, big, n_big, tk, tv, xk, xv, ns, out);
     note_launch(3);
     return cudaGetLastError();
 }

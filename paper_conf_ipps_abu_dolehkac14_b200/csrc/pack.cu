@@ -70,6 +70,7 @@ __global__ void __launch_bounds__(kPackThreads) k_pack(const uint8_t *__restrict
                                                        uint64_t *__restrict__ words, uint64_t n_full,
                                                        uint64_t n_words_alloc, unsigned long long *bad_pos,
                                                        int aligned) {
+    pdl_wait();
     const int lane = threadIdx.x & 31;
     if (aligned) {
         const uint64_t n_halves = 2 * n_full;
@@ -105,6 +106,7 @@ __global__ void __launch_bounds__(kPackThreads) k_pack(const uint8_t *__restrict
 // 32 bases of s ending at n - 32w, reversed pairwise, complemented, tail kept 00.
 __global__ void __launch_bounds__(kPackThreads) k_revcomp(const uint64_t *__restrict__ in, uint64_t n,
                                                           uint64_t *__restrict__ out, uint64_t n_words_alloc) {
+    pdl_wait();
     const uint64_t w = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
     if (w >= n_words_alloc) return;
     const uint64_t first = w * 32;
@@ -133,7 +135,7 @@ __global__ void __launch_bounds__(kPackThreads) k_revcomp(const uint64_t *__rest
 
 cudaError_t launch_revcomp(const uint64_t *in, uint64_t n, uint64_t *out, uint64_t n_words_alloc, cudaStream_t s) {
     const uint64_t blocks = (n_words_alloc + kPackThreads - 1) / kPackThreads;
-    k_revcomp<<<unsigned(blocks), kPackThreads, 0, s>>>(in, n, out, n_words_alloc);
+    pdl_launch(k_revcomp, unsigned(blocks), kPackThreads, 0, s, in, n, out, n_words_alloc);
     note_launch();
     return cudaGetLastError();
 }
@@ -145,7 +147,7 @@ cudaError_t launch_pack(const uint8_t *in, uint64_t n, uint64_t *words, uint64_t
     const uint64_t per = uint64_t(kPackThreads) * kHPT;  // halves per CTA
     uint64_t blocks = aligned ? (2 * n_full + per - 1) / per : (n_words_alloc + kPackThreads - 1) / kPackThreads;
     if (blocks == 0) blocks = 1;
-    k_pack<<<unsigned(blocks), kPackThreads, 0, s>>>(in, n, words, n_full, n_words_alloc, bad_pos, aligned);
+    pdl_launch(k_pack, unsigned(blocks), kPackThreads, 0, s, in, n, words, n_full, n_words_alloc, bad_pos, aligned);
     note_launch();
     return cudaGetLastError();
 }

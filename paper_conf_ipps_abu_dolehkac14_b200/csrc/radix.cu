@@ -106,6 +106,7 @@ struct Chunking {
 template <class K, int RB>
 __global__ void __launch_bounds__(kT) k_chunk_hist(const K *__restrict__ keys, Chunking ch0, int shift, int bits,
                                                    uint32_t *__restrict__ counts, uint32_t *__restrict__ totals) {
+    pdl_wait();
     constexpr int kBins = 1 << RB;
     constexpr int DPT = kBins / kT;
     __shared__ uint32_t h[kWarps][kBins];
@@ -135,6 +136,7 @@ template <int RB>
 __global__ void __launch_bounds__(kT) k_chunk_scan(const uint32_t *__restrict__ counts,
                                                    const uint32_t *__restrict__ totals, uint32_t chunks,
                                                    uint32_t *__restrict__ offs) {
+    pdl_wait();
     constexpr int kBins = 1 << RB;
     constexpr int DPT = kBins / kT;
     __shared__ uint32_t dbase[kBins];
@@ -222,6 +224,7 @@ template <class K, class V, int RB>
 __global__ void __launch_bounds__(kST, GM_RADIX_MINB) k_scatter(const K *__restrict__ kin, const V *__restrict__ vin,
                                                   K *__restrict__ kout, V *__restrict__ vout, Chunking ch0,
                                                   int shift, int bits, const uint32_t *__restrict__ offs) {
+    pdl_wait();
     constexpr int kBins = 1 << RB;
     constexpr int DPT = (kBins + kST - 1) / kST;  // digits owned per thread: tid, tid + kST, ... (< kBins)
     constexpr int kItems = Cfg<K>::kItems;
@@ -438,9 +441,9 @@ cudaError_t radix_sort_rb(K *k0, uint32_t *v0, K *k1, uint32_t *v1, uint64_t n, 
         const int sh = lo + RB * p;
         const int dbits = (p == passes - 1) ? bits - sh : RB;
         uint32_t *tot = totals + size_t(p) * kBins;
-        k_chunk_hist<K, RB><<<ch.chunks, kT, 0, s>>>(ka, ch, sh, dbits, counts, tot);
-        k_chunk_scan<RB><<<kBins / kWarps, kT, 0, s>>>(counts, tot, ch.chunks, offs);
-        k_scatter<K, uint32_t, RB><<<ch.chunks, kST, smem, s>>>(ka, va, kb, vb, ch, sh, dbits, offs);
+        pdl_launch(k_chunk_hist<K, RB>, ch.chunks, kT, 0, s, ka, ch, sh, dbits, counts, tot);
+        pdl_launch(k_chunk_scan<RB>, kBins / kWarps, kT, 0, s, counts, tot, ch.chunks, offs);
+        pdl_launch(k_scatter<K, uint32_t, RB>, ch.chunks, kST, smem, s, ka, va, kb, vb, ch, sh, dbits, offs);
         note_launch(3);
         std::swap(ka, kb);
         std::swap(va, vb);

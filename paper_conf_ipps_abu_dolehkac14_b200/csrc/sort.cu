@@ -12,6 +12,7 @@ __global__ void __launch_bounds__(kT) k_keys_to_triples(const uint64_t *__restri
                                                         const uint32_t *__restrict__ lens, uint64_t n,
                                                         uint32_t qbits, gpumem_triple *__restrict__ out,
                                                         const unsigned long long *__restrict__ dn) {
+    pdl_wait();
     const uint64_t i = uint64_t(blockIdx.x) * kT + threadIdx.x;
     if (dn) {  // device-resident count, n is the capacity
         const unsigned long long x = *dn;
@@ -30,6 +31,7 @@ __global__ void __launch_bounds__(kT) k_keys_to_triples(const uint64_t *__restri
 __global__ void __launch_bounds__(kT) k_triples_to_keys(const gpumem_triple *__restrict__ in, uint64_t n,
                                                         uint32_t qbits, uint64_t *__restrict__ keys,
                                                         uint32_t *__restrict__ lens) {
+    pdl_wait();
     const uint64_t i = uint64_t(blockIdx.x) * kT + threadIdx.x;
     if (i >= n) return;
     const gpumem_triple t = in[i];
@@ -39,12 +41,14 @@ __global__ void __launch_bounds__(kT) k_triples_to_keys(const gpumem_triple *__r
 
 __global__ void __launch_bounds__(kT) k_join(const uint32_t *__restrict__ codes, const uint32_t *__restrict__ locs,
                                              uint64_t n, uint64_t *__restrict__ keys) {
+    pdl_wait();
     const uint64_t i = uint64_t(blockIdx.x) * kT + threadIdx.x;
     if (i < n) keys[i] = (uint64_t(codes[i]) << 32) | locs[i];
 }
 
 __global__ void __launch_bounds__(kT) k_split(const uint64_t *__restrict__ keys, uint64_t n,
                                               uint32_t *__restrict__ codes, uint32_t *__restrict__ locs) {
+    pdl_wait();
     const uint64_t i = uint64_t(blockIdx.x) * kT + threadIdx.x;
     if (i >= n) return;
     const uint64_t k = keys[i];
@@ -56,14 +60,14 @@ __global__ void __launch_bounds__(kT) k_split(const uint64_t *__restrict__ keys,
 
 cudaError_t launch_join_keys(const uint32_t *codes, const uint32_t *locs, uint64_t n, uint64_t *keys, cudaStream_t s) {
     if (!n) return cudaSuccess;
-    k_join<<<unsigned((n + kT - 1) / kT), kT, 0, s>>>(codes, locs, n, keys);
+    pdl_launch(k_join, unsigned((n + kT - 1) / kT), kT, 0, s, codes, locs, n, keys);
     note_launch();
     return cudaGetLastError();
 }
 
 cudaError_t launch_split_keys(const uint64_t *keys, uint64_t n, uint32_t *codes, uint32_t *locs, cudaStream_t s) {
     if (!n) return cudaSuccess;
-    k_split<<<unsigned((n + kT - 1) / kT), kT, 0, s>>>(keys, n, codes, locs);
+    pdl_launch(k_split, unsigned((n + kT - 1) / kT), kT, 0, s, keys, n, codes, locs);
     note_launch();
     return cudaGetLastError();
 }
@@ -71,7 +75,7 @@ cudaError_t launch_split_keys(const uint64_t *keys, uint64_t n, uint32_t *codes,
 cudaError_t launch_keys_to_triples(const uint64_t *keys, const uint32_t *lens, uint64_t n, uint32_t qbits,
                                    gpumem_triple *out, cudaStream_t s, const unsigned long long *dn) {
     if (!n) return cudaSuccess;
-    k_keys_to_triples<<<unsigned((n + kT - 1) / kT), kT, 0, s>>>(keys, lens, n, qbits, out, dn);
+    pdl_launch(k_keys_to_triples, unsigned((n + kT - 1) / kT), kT, 0, s, keys, lens, n, qbits, out, dn);
     note_launch();
     return cudaGetLastError();
 }
@@ -79,7 +83,7 @@ cudaError_t launch_keys_to_triples(const uint64_t *keys, const uint32_t *lens, u
 cudaError_t launch_triples_to_keys(const gpumem_triple *in, uint64_t n, uint32_t qbits, uint64_t *keys,
                                    uint32_t *lens, cudaStream_t s) {
     if (!n) return cudaSuccess;
-    k_triples_to_keys<<<unsigned((n + kT - 1) / kT), kT, 0, s>>>(in, n, qbits, keys, lens);
+    pdl_launch(k_triples_to_keys, unsigned((n + kT - 1) / kT), kT, 0, s, in, n, qbits, keys, lens);
     note_launch();
     return cudaGetLastError();
 }

@@ -30,6 +30,7 @@ constexpr int kBlock = kT * kPer;  // items per CTA in the scans
 
 __global__ void __launch_bounds__(kT) k_interval_keys(const gpumem_triple *__restrict__ t, uint64_t n, int axis,
                                                       uint64_t *__restrict__ keys, uint32_t *__restrict__ vals) {
+    pdl_wait();
     const uint64_t i = uint64_t(blockIdx.x) * kT + threadIdx.x;
     if (i >= n) return;
     const gpumem_triple x = t[i];
@@ -44,6 +45,7 @@ __device__ __forceinline__ uint64_t end_of(uint64_t key) {
 
 __global__ void __launch_bounds__(kT) k_block_max(const uint64_t *__restrict__ keys, uint64_t n,
                                                   uint64_t *__restrict__ bmax) {
+    pdl_wait();
     __shared__ uint64_t ws[kT / 32];
     const uint64_t base = uint64_t(blockIdx.x) * kBlock;
     uint64_t m = 0;
@@ -64,6 +66,7 @@ __global__ void __launch_bounds__(kT) k_block_max(const uint64_t *__restrict__ k
 
 // exclusive running maximum of bmax[0..m) in place (single CTA, sequential over chunks)
 __global__ void __launch_bounds__(kT) k_scan_max(uint64_t *bmax, uint64_t m) {
+    pdl_wait();
     __shared__ uint64_t ws[kT / 32];
     __shared__ uint64_t carry;
     if (threadIdx.x == 0) carry = 0;
@@ -96,6 +99,7 @@ __global__ void __launch_bounds__(kT) k_scan_max(uint64_t *bmax, uint64_t m) {
 __global__ void __launch_bounds__(kT) k_contained(const uint64_t *__restrict__ keys, const uint32_t *__restrict__ vals,
                                                   uint64_t n, const uint64_t *__restrict__ bprefix,
                                                   uint8_t *__restrict__ flags) {
+    pdl_wait();
     __shared__ uint64_t ws[kT / 32];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     const uint64_t base = uint64_t(blockIdx.x) * kBlock + uint64_t(threadIdx.x) * kPer;  // blocked
@@ -132,6 +136,7 @@ __global__ void __launch_bounds__(kT) k_contained(const uint64_t *__restrict__ k
 
 __global__ void __launch_bounds__(kT) k_count_kept(const uint8_t *__restrict__ fq, const uint8_t *__restrict__ fr,
                                                    uint64_t n, uint32_t *__restrict__ counts) {
+    pdl_wait();
     __shared__ uint32_t ws[kT / 32];
     const uint64_t base = uint64_t(blockIdx.x) * kBlock;
     uint32_t c = 0;
@@ -152,6 +157,7 @@ __global__ void __launch_bounds__(kT) k_count_kept(const uint8_t *__restrict__ f
 
 // exclusive sum of counts[0..m) in place; total -> *total
 __global__ void __launch_bounds__(kT) k_scan_sum(uint32_t *counts, uint64_t m, unsigned long long *total) {
+    pdl_wait();
     __shared__ uint32_t ws[kT / 32];
     __shared__ unsigned long long carry;
     if (threadIdx.x == 0) carry = 0;
@@ -185,6 +191,7 @@ __global__ void __launch_bounds__(kT) k_scan_sum(uint32_t *counts, uint64_t m, u
 __global__ void __launch_bounds__(kT) k_compact(const gpumem_triple *__restrict__ in, const uint8_t *__restrict__ fq,
                                                 const uint8_t *__restrict__ fr, uint64_t n,
                                                 const uint32_t *__restrict__ offs, gpumem_triple *__restrict__ out) {
+    pdl_wait();
     __shared__ uint32_t ws[kT / 32];
     __shared__ uint32_t s_base;
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
@@ -242,19 +249,19 @@ cudaError_t mum_filter(const gpumem_triple *in, uint64_t n, gpumem_triple *out, 
     void *rs = reinterpret_cast<void *>(c);
     if ((e = cudaMemsetAsync(flags, 0, n * 2, s)) != cudaSuccess) return e;
     for (int axis = 0; axis < 2; ++axis) {  // 0: query intervals (uniqueness in R), 1: reference (in Q)
-        k_interval_keys<<<nblk(n, kT), kT, 0, s>>>(in, n, axis, k0, v0);
+        pdl_launch(k_interval_keys, nblk(n, kT), kT, 0, s, in, n, axis, k0, v0);
         bool alt = false;
         if ((e = radix_sort_u64(k0, v0, k1, v1, n, 64, rs, s, &alt)) != cudaSuccess) return e;
         const uint64_t *ks = alt ? k1 : k0;
         const uint32_t *vs = alt ? v1 : v0;
-        k_block_max<<<unsigned(nb), kT, 0, s>>>(ks, n, bmax);
-        k_scan_max<<<1, kT, 0, s>>>(bmax, nb);
-        k_contained<<<unsigned(nb), kT, 0, s>>>(ks, vs, n, bmax, flags + uint64_t(axis) * n);
+        pdl_launch(k_block_max, unsigned(nb), kT, 0, s, ks, n, bmax);
+        pdl_launch(k_scan_max, 1, kT, 0, s, bmax, nb);
+        pdl_launch(k_contained, unsigned(nb), kT, 0, s, ks, vs, n, bmax, flags + uint64_t(axis) * n);
         note_launch(4);
     }
-    k_count_kept<<<unsigned(nb), kT, 0, s>>>(flags, flags + n, n, counts);
-    k_scan_sum<<<1, kT, 0, s>>>(counts, nb, d_count);
-    k_compact<<<unsigned(nb), kT, 0, s>>>(in, flags, flags + n, n, counts, out);
+    pdl_launch(k_count_kept, unsigned(nb), kT, 0, s, flags, flags + n, n, counts);
+    pdl_launch(k_scan_sum, 1, kT, 0, s, counts, nb, d_count);
+    pdl_launch(k_compact, unsigned(nb), kT, 0, s, in, flags, flags + n, n, counts, out);
     note_launch(3);
     return cudaGetLastError();
 }

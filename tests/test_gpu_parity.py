@@ -24,7 +24,7 @@ def _default_options():
     yield
     for k, v in (("find_grid", 0), ("find_spill", 64), ("out_capacity", 0), ("use_bitmap", 1), ("static_lb", 0),
                  ("sort_impl", 0), ("index_msd", 0), ("small_sort", 0), ("radix_bits", 0),
-                 ("rank_sectors", -1), ("rec8", -1), ("index_fused", 0)):
+                 ("rank_sectors", -1), ("rec8", -1), ("index_fused", 0), ("pdl", 1)):
         gpumem.set_option(k, v)
 
 
@@ -251,14 +251,14 @@ def test_overflow_retry_grid_spill_and_bitmap_invariance():
     for opt, vals in (("out_capacity", [1, 100]), ("find_grid", [1, 3, 148]), ("find_spill", [1, 2, 10**9]),
                       ("use_bitmap", [0]), ("static_lb", [1]), ("sort_impl", [1, 2, 3]), ("index_msd", [1]), ("small_sort", [1]),
                       ("rank_sectors", [0, 1]), ("rec8", [0, 1]), ("index_fused", [1]),
-                      ("radix_bits", [8, 9, 10])):
+                      ("radix_bits", [8, 9, 10]), ("pdl", [0])):
         for v in vals:
             gpumem.set_option(opt, v)
             assert np.array_equal(gpu_mems(P.R, P.Q, P.L, P.ls), want), (opt, v)
         gpumem.set_option(opt, {"out_capacity": 0, "find_grid": 0, "find_spill": 64, "use_bitmap": 1,
                                 "static_lb": 0, "sort_impl": 0, "index_msd": 0, "small_sort": 0, "rank_sectors": -1,
                                 "rec8": -1, "index_fused": 0,
-                                "radix_bits": 0}[opt])
+                                "radix_bits": 0, "pdl": 1}[opt])
 
 
 def test_seed_length_and_step_invariance():
