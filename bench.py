@@ -284,6 +284,21 @@ def run_ours(args, P):
                               * kernel_ms[dom] / 1e3 / n_launch)
             roof["l1_sectors_per_launch"] = int(sectors)
             roof["l1_sector_rate_per_sm_clk"] = round(rate, 3)
+            # the same number of random 8-byte probes into an L2-resident table the size of
+            # the rank directory, nothing else (gpumem_gather_ceiling), measured here: the
+            # practical peak of k_find's access pattern on this GPU
+            try:
+                table = (1 << (2 * ls)) // 32 * 8
+                ceil_ms = gm.gather_ceiling(int(sectors), table)
+                find_ms = kernel_ms[dom] / n_launch
+                roof["note"] = ("at C4 k_find is bound by random 32-B sector requests to L2, not HBM "
+                                "bandwidth: see gather_ceiling (DESIGN.md §7)")
+                roof["gather_ceiling"] = {
+                    "what": f"{int(sectors)} random 8-B loads into a {table >> 20} MB table, 8 per thread",
+                    "unit": "Gsector/s", "peak": round(sectors / ceil_ms / 1e6, 1),
+                    "achieved": round(sectors / find_ms / 1e6, 1), "frac": round(ceil_ms / find_ms, 3)}
+            except Exception as e:  # pragma: no cover
+                roof["gather_ceiling"] = {"error": repr(e)}
     stage_frac = {k: round(alg[k] / (kernel_ms[k] / 1e3) / 1e9 / peak, 4) for k in alg if k in kernel_ms}
 
     line = {"metric": METRIC, "value": round(value, 2), "unit": "Mbp/s", "n_gpus": world, "steps": args.steps,

@@ -272,6 +272,13 @@ gpumem_status gpumem_set_option(const char *name, int64_t value);
 gpumem_status gpumem_profile_enable(int on);
 int gpumem_profile_read(const char **names, double *ms, uint64_t *launches, int max_stages);
 
+/* The ceiling of k_find's access pattern on this GPU (not part of the method):
+ * *ms = best time of n_probes random 8-byte loads into a device table of table_bytes
+ * (rounded down to a power of two; L2-resident when small), 8 independent loads per
+ * thread as the find kernel issues its probes. Synchronous; allocates and frees its
+ * own table. bench.py sets k_find's sector rate against it. */
+gpumem_status gpumem_gather_ceiling(uint64_t n_probes, uint64_t table_bytes, void *cuda_stream, double *ms);
+
 /* Kernels this library has launched in this process (monotone counter). */
 uint64_t gpumem_launch_count(void);
 

@@ -538,6 +538,17 @@ gpumem_status gpumem_trim(void) {
 
 uint64_t gpumem_launch_count(void) { return g_launches.load(); }
 
+gpumem_status gpumem_gather_ceiling(uint64_t n_probes, uint64_t table_bytes, void *cuda_stream, double *ms) {
+    if (!ms || n_probes == 0 || table_bytes < 16) return fail(GPUMEM_ERR_ARG, "need ms, n_probes > 0, table >= 16 B");
+    int dev;
+    gpumem_status st = check_device(&dev);
+    if (st) return st;
+    float best = 0.f;
+    CK(gather_ceiling(n_probes, table_bytes, static_cast<cudaStream_t>(cuda_stream), &best), "gather ceiling");
+    *ms = best;
+    return GPUMEM_OK;
+}
+
 gpumem_status gpumem_set_allocator(void *(*alloc_fn)(size_t, void *, void *), void (*free_fn)(void *, void *, void *),
                                    void *ctx) {
     if ((alloc_fn == nullptr) != (free_fn == nullptr)) return fail(GPUMEM_ERR_ARG, "set both hooks or neither");

@@ -189,6 +189,10 @@ cudaError_t launch_heavy(const FindParams &p, cudaStream_t s);
 cudaError_t launch_coop(const FindParams &p, cudaStream_t s);
 int find_default_grid();
 
+// Instrumentation (diag.cu): best-of-4 time of n random 8-byte probes into a table of
+// table_bytes (rounded down to a power of two), 8 independent probes per thread.
+cudaError_t gather_ceiling(uint64_t n_probes, uint64_t table_bytes, cudaStream_t s, float *best_ms);
+
 // MUM filter (variants.cu): the MEMs whose string is unique in R and in Q, order kept;
 // the kept count is written to *d_count (device).
 size_t mum_scratch_bytes(uint64_t n);

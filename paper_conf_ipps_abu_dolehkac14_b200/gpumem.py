@@ -62,6 +62,7 @@ SYMBOLS = {
     "gpumem_profile_enable": (ctypes.c_int, [ctypes.c_int]),
     "gpumem_profile_read": (ctypes.c_int, [_P(ctypes.c_char_p), _P(ctypes.c_double), _P(_c_u64), ctypes.c_int]),
     "gpumem_launch_count": (_c_u64, []),
+    "gpumem_gather_ceiling": (ctypes.c_int, [_c_u64, _c_u64, _vp, _P(ctypes.c_double)]),
     "gpumem_version": (ctypes.c_char_p, []),
 }
 for _name, (_res, _args) in SYMBOLS.items():
@@ -377,6 +378,13 @@ def profile_read(max_stages=32):
 def trim():
     """Release the library's per-stream workspaces (synchronises those streams)."""
     _check(_lib.gpumem_trim())
+
+
+def gather_ceiling(n_probes: int, table_bytes: int, stream=None) -> float:
+    """ms for n_probes random 8-byte loads into a table_bytes device table (k_find's ceiling)."""
+    ms = ctypes.c_double()
+    _check(_lib.gpumem_gather_ceiling(int(n_probes), int(table_bytes), _stream(stream), ctypes.byref(ms)))
+    return ms.value
 
 
 def launch_count() -> int:
