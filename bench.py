@@ -116,6 +116,7 @@ def oracle_sample(P, sample_bp):
     t = time.perf_counter()
     out = oracle.mems(P.R, P.Q, P.L, P.ls, 0, 0, q_end, threads=threads)
     dt = time.perf_counter() - t
+    oracle_sample.last = out
     return dt, q_end, len(out), oracle.num_threads(threads)
 
 
@@ -239,6 +240,7 @@ def run_ours(args, P):
                 prof[k] = (a0[0] + t, a0[1] + nl)
         torch.cuda.synchronize()
     launches = gm.launch_count() - l0
+    gpu_result = sp.pl.numpy() if world == 1 else None  # the last timed step's MEMs
     if world > 1:
         dist.barrier()
     step_ms = [a.elapsed_time(b) for a, b in ev]
@@ -354,6 +356,17 @@ def run_ours(args, P):
             "value": round(q_end / 1e6 / dt, 3), "unit": "Mbp/s", "cores": cores, "kind": "oracle",
             "sample": f"full hash index of R + MEMs starting in Q[0:{q_end}] ({q_end / nQ:.1%} of Q); "
                       f"{nm_cpu} MEMs in {dt:.2f} s"}
+        # parity on the same sample: the timed pipeline's last result restricted to MEM
+        # starts q < q_end (sorted by (r, q), so the restriction keeps the order) against
+        # the oracle's triples, element by element
+        import hashlib
+        want = np.ascontiguousarray(oracle_sample.last, dtype=np.uint32)
+        got = gpu_result[gpu_result[:, 1] < q_end] if gpu_result is not None else np.zeros((0, 3), np.uint32)
+        got = np.ascontiguousarray(got, dtype=np.uint32)
+        line["parity_sample"] = {"q_range": [0, int(q_end)], "mems_gpu": int(len(got)), "mems_oracle": int(len(want)),
+                                 "equal": bool(got.shape == want.shape and np.array_equal(got, want)),
+                                 "sha256_gpu": hashlib.sha256(got.tobytes()).hexdigest()[:16],
+                                 "sha256_oracle": hashlib.sha256(want.tobytes()).hexdigest()[:16]}
     if world > 1:
         dist.barrier()
     if rank == 0:
