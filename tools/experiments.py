@@ -7,8 +7,9 @@
         on C2/C3/C4 at several L
   tab34 index-build and extraction times per config (Table III/IV analogues, :230-258)
 
-Times are CUDA-event device times (mean of --steps after --warmup, L2 flushed before
-each step), per stage from the library's stage events. Writes a JSON file and a
+Times are CUDA-event device times of one pipeline (CUDA-graph) run per step (mean of
+--steps after --warmup, L2 flushed before each step), per stage from the graph's
+event nodes (pack R and pack Q run concurrently: the 'index' column includes both packs). Writes a JSON file and a
 markdown summary. The paper's numbers are on a K20c with real genomes: context only.
 
     python tools/experiments.py --out profiles/r1_experiments [--steps 5]
@@ -28,35 +29,31 @@ from paper_conf_ipps_abu_dolehkac14_b200 import gpumem as gm, synth  # noqa: E40
 
 
 def run(R_dev, Q_dev, L, ls, steps, warmup, q_range=None, opts=None):
+    """The path as bench.py times it: one gpumem_pipeline_run per step (CUDA graph),
+    stage times from the graph's own event nodes."""
     opts = opts or {}
     for k, v in opts.items():
         gm.set_option(k, v)
     flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
     stream = torch.cuda.current_stream()
+    pl = gm.Pipeline(R_dev.numel(), Q_dev.numel(), ls, L, q_range)  # captured with these options
     tot, prof_acc, n_mems = 0.0, {}, 0
     for i in range(warmup + steps):
         flush.zero_()
-        torch.cuda.synchronize()
-        if i == warmup:
-            gm.profile_enable(True)
-            gm.profile_read()
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a.record(stream)
-        Rs, Qs = gm.pack(R_dev), gm.pack(Q_dev)
-        idx = gm.index_build(Rs, ls, L)
-        m = gm.find_mems(idx, Qs, q_range)
+        pl.run(R_dev, Q_dev)
         b.record(stream)
-        torch.cuda.synchronize()
-        n_mems = len(m)
-        for h in (m, idx, Qs, Rs):
-            h.free()
+        n_mems = pl.result()
+        b.synchronize()
         if i >= warmup:
             tot += a.elapsed_time(b)
-    prof = gm.profile_read()
-    gm.profile_enable(False)
+            for k, (t, _) in pl.profile().items():
+                prof_acc[k] = prof_acc.get(k, 0.0) + t
+    pl.free()
     for k in opts:
         gm.set_option(k, {"find_spill": 64, "static_lb": 0}.get(k, 0))
-    stage = {k: v[0] / steps for k, v in prof.items()}
+    stage = {k: v / steps for k, v in prof_acc.items()}
     index_ms = sum(v for k, v in stage.items() if k.startswith("index") or k == "pack")
     extract_ms = sum(v for k, v in stage.items() if k.startswith("find") or k == "sort")
     return {"ms": tot / steps, "mems": n_mems, "index_ms": index_ms, "extract_ms": extract_ms, "stage_ms": stage}
