@@ -47,7 +47,10 @@ namespace {
 
 constexpr int kT = 256;                   // threads per CTA
 constexpr int kWarps = kT / 32;
-constexpr int kQPT = 8;                   // query positions per lane per chunk
+#ifndef GM_FIND_QPT
+#define GM_FIND_QPT 8
+#endif
+constexpr int kQPT = GM_FIND_QPT;         // query positions per lane per chunk
 constexpr int kChunk = 32 * kQPT;         // 256 positions per warp chunk
 #ifndef GM_FIND_GRAB
 #define GM_FIND_GRAB 2

@@ -362,7 +362,14 @@ __global__ void __launch_bounds__(kCodeThreads) k_seed_recs(const uint64_t *__re
     const uint32_t p = locs[k];
     uint32_t left;
     uint64_t right;
-    if (p >= 16) {  // bases [p - 16, p + ls + 32) lie in the 3 words from (p - 16) / 32: one gather
+    if (kRec8 && p >= 8) {  // bases [p - 8, p + ls + 8) (<= 31 bases) lie in the 2 words from (p - 8) / 32
+        const uint64_t x = p - 8, w = x >> 5;
+        const uint64_t w0 = __ldg(R + w), w1 = __ldg(R + w + 1);
+        const uint32_t sx = uint32_t(x & 31) * 2;
+        const uint64_t win = sx ? (w0 << sx) | (w1 >> (64 - sx)) : w0;  // bases [p - 8, p + 24)
+        left = uint32_t(win >> 48);                                       // R[p - 8, p), base p-1 lowest
+        right = (win << (2 * (8 + ls))) & 0xffff000000000000ull;          // R[p + ls, p + ls + 8) on top
+    } else if (p >= 16) {  // bases [p - 16, p + ls + 32) lie in the 3 words from (p - 16) / 32: one gather
         const uint64_t x = p - 16, w = x >> 5;
         const uint64_t w0 = __ldg(R + w), w1 = __ldg(R + w + 1), w2 = __ldg(R + w + 2);
         const uint32_t sx = uint32_t(x & 31) * 2;
