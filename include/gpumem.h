@@ -185,21 +185,24 @@ gpumem_status gpumem_merge_sorted(const gpumem_triple *const *dev_runs, const ui
  *
  * gpumem_pipeline_create -- sizes |R| = r_len, |Q| = q_len, seed_len (ls), min_len (L)
  *  and the MEM start range [q_begin, q_end) as in gpumem_find_mems (0, UINT64_MAX = all).
- *  Argument rules as gpumem_index_build / gpumem_find_mems. Stream: every run is
- *  enqueued on `cuda_stream` (the pipeline's workspaces belong to it). Allocates only a
- *  pinned 128-byte counter buffer; device memory (one arena holding the packed
+ *  Argument rules as gpumem_index_build / gpumem_find_mems. Stream: runs are ordered
+ *  after the caller's prior work on `cuda_stream` and before its later work (events);
+ *  the graph itself runs on streams the pipeline owns (a captured graph cannot live on
+ *  the legacy default stream), which also own its workspaces. Allocates those streams
+ *  and a pinned 128-byte counter buffer; device memory (one arena holding the packed
  *  sequences, the index and the result) is allocated at the first run.
  *
  * gpumem_pipeline_run -- async. r_bases_dev / q_bases_dev: device pointers to r_len and
  *  q_len ASCII bases (read, not modified; must stay valid until the run completes).
  *  The first call, and any call with different input pointers, measures and captures
- *  the graph (one ordinary synchronous pass + capture); later calls are one
- *  cudaGraphLaunch. The previous run's result is invalidated.
+ *  the graph (one ordinary synchronous pass + capture; option settings are taken at
+ *  capture time); later calls are one cudaGraphLaunch. The previous run's result is
+ *  invalidated.
  *
  * gpumem_pipeline_run_host -- the same from host memory (pinned for full speed): R and Q
  *  are copied on a copy stream into pipeline-owned device buffers (allocated on the
- *  first call), R first; the graph packs and indexes R while Q is still in flight and
- *  each segment waits only for the copy it reads. Async: the host buffers must stay
+ *  first call), R first; the graph packs and indexes R while Q is still in flight (its
+ *  external event-wait nodes make each branch wait only for the copy it reads). Async: the host buffers must stay
  *  valid and unmodified until the run completes (gpumem_pipeline_result).
  *
  * gpumem_pipeline_result -- synchronises the stream, then checks the alphabet flags
@@ -210,7 +213,8 @@ gpumem_status gpumem_merge_sorted(const gpumem_triple *const *dev_runs, const ui
  *
  * gpumem_pipeline_stats -- find statistics of the last result.
  * gpumem_pipeline_profile -- per-stage device time of the last completed run (the
- *  stage events are part of the graph), aggregated by name as gpumem_profile_read;
+ *  stage events are event-record nodes of the graph), aggregated by name as
+ *  gpumem_profile_read;
  *  synchronises those events. Returns the number of entries written.
  * gpumem_free(pl) synchronises the stream and releases everything.
  */
