@@ -334,6 +334,33 @@ def test_full_size_c4_c5(c4_full, L):
     pl.free()
 
 
+@pytest.mark.slow
+def test_full_size_shards_byte_identical(c4_full):
+    """SURVEY.md §8(e) check at the full C4 size: the query-sharded runs of G = 1, 2, 4, 8
+    ranks (one pipeline per rank's MEM-start range, as bench.py --gpus G runs them;
+    here all on one device) concatenate, after the rank-0 merge kernel, to the byte-
+    identical whole set."""
+    P = c4_full
+    Rt, Qt = torch.from_numpy(P.R).cuda(), torch.from_numpy(P.Q).cuda()
+    from paper_conf_ipps_abu_dolehkac14_b200.dist import shard_range
+    whole = None
+    for G in (1, 2, 4, 8):
+        runs = []
+        for g in range(G):
+            pl = gpumem.Pipeline(len(P.R), len(P.Q), P.ls, P.L, shard_range(len(P.Q), g, G))
+            pl.run(Rt, Qt)
+            pl.result()
+            runs.append(pl.view_u32().clone())
+            pl.free()
+        merged = gpumem.merge_sorted([r.view(torch.int32) for r in runs])
+        got = merged.numpy()
+        merged.free()
+        if whole is None:
+            whole = got
+            assert len(whole) == 811662
+        assert got.tobytes() == whole.tobytes(), G
+
+
 # ------------------------------------------------------------------ NEXT rows (SURVEY.md §8(f))
 def _rc(b):
     return bytes(b)[::-1].translate(bytes.maketrans(b"ACGTacgt", b"TGCAtgca"))
