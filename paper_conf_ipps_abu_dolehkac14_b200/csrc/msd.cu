@@ -37,7 +37,14 @@ constexpr int kWarps = kT / 32;
 constexpr int kPT = 1024;                        // threads of the chunk kernels
 constexpr int kLT = 512;                         // threads of k_bs_local
 constexpr int kLWarps = kLT / 32;
-constexpr int kItems = 8;                        // keys per thread in k_bs_local
+#ifndef GM_MSD_ITEMS
+#define GM_MSD_ITEMS 8
+#endif
+#ifndef GM_MSD_CTAS
+#define GM_MSD_CTAS 2
+#endif
+constexpr int kItems = GM_MSD_ITEMS;             // keys per thread in k_bs_local
+constexpr int kLocalCtas = GM_MSD_CTAS;          // resident k_bs_local CTAs per SM (grid size)
 constexpr uint32_t kLocal = kLT * kItems;        // most keys one CTA sorts in shared memory (4096)
 constexpr uint32_t kSeg = kLocal / 2;            // segment spacing (slots) for the grid size
 #ifndef GM_MSD_SEGMAX
@@ -321,7 +328,7 @@ __device__ void smem_sort_write(LocalSmem &S, const uint64_t *__restrict__ tk, c
     __syncthreads();
 }
 
-__global__ void __launch_bounds__(kLT, 2) k_bs_local(const uint32_t *__restrict__ offs, NSpec ns,
+__global__ void __launch_bounds__(kLT, kLocalCtas) k_bs_local(const uint32_t *__restrict__ offs, NSpec ns,
                                                  const uint64_t *__restrict__ tk, const uint32_t *__restrict__ tv,
                                                  Out out, uint32_t *__restrict__ big, unsigned int *n_big) {
     pdl_wait();
@@ -507,7 +514,7 @@ static cudaError_t msd_run(uint64_t *keys, uint32_t *vals, NSpec ns, void *scrat
     pdl_launch(k_bs_scan, 1, 1024, 0, s, totals, ns, offs);
     pdl_launch(k_bp_scatter, chunks, kPT, nb_max * 4, s, keys, vals, ns, counts, offs, tk, tv);
     uint64_t segs = (cap + kSeg - 1) / kSeg;
-    if (segs > uint64_t(2 * num_sms())) segs = 2 * num_sms();  // blocks loop over the segments
+    if (segs > uint64_t(kLocalCtas * num_sms())) segs = kLocalCtas * num_sms();  // blocks loop over the segments
     pdl_launch(k_bs_local, unsigned(segs ? segs : 1), kLT, sizeof(LocalSmem), s, offs, ns, tk, tv, out, big, n_big);
     // oversized buckets: ping-pong with the input's range of the bucket (free: the scatter
     // consumed it and the local pass wrote only other buckets' ranges)
@@ -588,7 +595,7 @@ cudaError_t hybrid_sort_triples(uint64_t *keys, uint32_t *vals, uint64_t *k1, ui
     }
     pdl_launch(k_prefix_bounds, (nb + 256) / 256, 256, 0, s, tk, ns, lo, nb, offs);
     uint64_t segs = (cap + kSeg - 1) / kSeg;
-    if (segs > uint64_t(2 * num_sms())) segs = 2 * num_sms();  // blocks loop over the segments
+    if (segs > uint64_t(kLocalCtas * num_sms())) segs = kLocalCtas * num_sms();  // blocks loop over the segments
     Out out{keys, vals, trip, qbits};
     pdl_launch(k_bs_local, unsigned(segs), kLT, sizeof(LocalSmem), s, offs, ns, tk, tv, out, big, n_big);
     pdl_launch(k_bs_big, num_sms(), kT, 0, s, offs, big, n_big, tk, tv, xk, xv, ns, out);
