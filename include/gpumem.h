@@ -262,6 +262,10 @@ gpumem_status gpumem_set_allocator(void *(*alloc_fn)(size_t bytes, void *cuda_st
  *  "rank_sectors"     lookup directory: -1 (default) auto, 0 rank words, 1 rank sectors
  *  "small_sort"       1: single-launch cooperative radix sorts (index and output) when
  *                     the input fits in shared memory; 0 (default): multi-launch
+ *  "index_alg1"       1: PAPER.md Alg. 1 as written (atomic counts, prefix sums,
+ *                     placement, per-bucket sort) instead of the stable radix sort;
+ *                     -1: only for dense indexes (n_locs >= 4^ls / 4); 0 (default): never
+ *                     (measured slower: random atomics/stores into the 4^ls table)
  *  "pdl"              1 (default): programmatic dependent launch between consecutive
  *                     kernels (each waits for its predecessor with griddepcontrol.wait);
  *                     0: ordinary launches

@@ -285,7 +285,8 @@ gpumem_status check_device(int *dev) {
 // loop does no allocation at all once warm. gpumem_trim() releases everything.
 enum WsSlot {
     kWsCtr, kWsSpill, kWsKeys, kWsLens, kWsSortK, kWsSortL, kWsSortScratch, kWsCodes0, kWsCodes1,
-    kWsRadix, kWsFill, kWsMergeK, kWsMergeL, kWsPackTmp, kWsCoop, kWsMums, kWsSmall, kWsLocsTmp, kWsSlot, kWsCount
+    kWsRadix, kWsFill, kWsMergeK, kWsMergeL, kWsPackTmp, kWsCoop, kWsMums, kWsSmall, kWsLocsTmp, kWsSlot, kWsAlg1,
+    kWsCount
 };
 struct Workspace {
     void *p[kWsCount] = {};
@@ -571,6 +572,7 @@ gpumem_status gpumem_set_option(const char *name, int64_t value) {
     }
     else if (!strcmp(name, "index_msd")) g_opt.index_msd = value ? 1 : 0;
     else if (!strcmp(name, "pdl")) g_opt.pdl = value ? 1 : 0;
+    else if (!strcmp(name, "index_alg1")) g_opt.index_alg1 = value < 0 ? -1 : (value ? 1 : 0);
     else if (!strcmp(name, "index_fused")) g_opt.index_fused = value ? 1 : 0;
     else if (!strcmp(name, "small_sort")) g_opt.small_sort = value ? 1 : 0;
     else if (!strcmp(name, "rec8")) g_opt.rec8 = value < 0 ? -1 : (value ? 1 : 0);
@@ -861,6 +863,17 @@ static gpumem_status index_build_impl(const gpumem_seq *R, uint32_t ls, uint32_t
         }
         codes_sorted = codes1;
         recs_done = true;
+    } else if (n_locs && !g_opt.index_msd &&
+               (g_opt.index_alg1 > 0 || (g_opt.index_alg1 < 0 && n_locs * 4 >= nb))) {
+        // dense index: Alg. 1 literally (atomic counts, prefix sums, placement, bucket sort)
+        void *scratch = ws_get(kWsAlg1, alg1_scratch_bytes(ls, n_locs), s);
+        if (!scratch) return GPUMEM_ERR_NOMEM;
+        {
+            Stage g("index.alg1", s);
+            CK(launch_index_alg1(R->words, ls, step, k0, n_locs, rankw, rsect, buckets, locs0, scratch, s),
+               "index (Alg. 1)");
+        }
+        fill_done = true;
     } else if (n_locs) {
         auto *codes0 = static_cast<uint32_t *>(ws_get(kWsCodes0, n_locs * 4, s));
         auto *codes1 = static_cast<uint32_t *>(ws_get(kWsCodes1, n_locs * 4, s));

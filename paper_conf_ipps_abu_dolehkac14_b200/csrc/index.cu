@@ -113,7 +113,9 @@ __global__ void __launch_bounds__(1024) k_occ_scan(const uint32_t *__restrict__ 
     }
 }
 
-template <bool kSect>
+// kCounts: `codes` is instead the dense per-seed count array (Alg. 1 step 1 done with
+// atomics by k_alg1_count) and chunk_first the records before each chunk.
+template <bool kSect, bool kCounts = false>
 __global__ void __launch_bounds__(kFillThreads) k_ptrs_fill(const uint32_t *__restrict__ codes, uint64_t n,
                                                             uint64_t n_buckets, uint32_t *__restrict__ ptrs,
                                                             unsigned long long *__restrict__ rankw,
@@ -128,8 +130,13 @@ __global__ void __launch_bounds__(kFillThreads) k_ptrs_fill(const uint32_t *__re
     const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
     const uint32_t c = blockIdx.x;
     const uint64_t s0 = uint64_t(c) * kChunk;
-    for (int i = tid; i < kChunk + kChunk / 32; i += kFillThreads) cnt[i] = 0;
-    const uint64_t lo = chunk_first[c], hi = chunk_first[c + 1];
+    const uint64_t lo = chunk_first[c], hi = kCounts ? lo : chunk_first[c + 1];
+    if (kCounts) {  // the chunk's counts, coalesced
+        for (int i = tid; i < kChunk; i += kFillThreads)
+            cnt[i + (i >> 5)] = s0 + uint64_t(i) < n_buckets ? codes[s0 + i] : 0u;
+    } else {
+        for (int i = tid; i < kChunk + kChunk / 32; i += kFillThreads) cnt[i] = 0;
+    }
     __syncthreads();
     // Alg. 1 step 1 for this chunk: seed counts. The codes are sorted, so equal codes are
     // runs of lanes: one shared atomic per run (a hot seed, e.g. poly-A, would otherwise
@@ -343,6 +350,193 @@ __global__ void __launch_bounds__(kDirThreads) k_dir_fill(const uint32_t *__rest
         const uint64_t g = (s0 >> 5) + tid;
         if (kSect) rsect[g] = make_uint4(lo + pe, r0 + po, c2lo[tid], c2hi[tid]);
         else rankw[g] = (uint64_t(r0 + po) << 32) | o;
+    }
+}
+
+// ---------------------------------------------------------------- Alg. 1 for dense indexes
+// PAPER.md Alg. 1 (:102-106) as written -- per-seed counts by atomics (step 1), prefix
+// sums (step 2), placement through per-seed cursors (step 3), a sort of every bucket
+// (step 4). Option index_alg1; measured slower than the radix path even where the index
+// is dense (C5 L = 20: 2.9 vs 1.4 ms; the counting atomics and the placement stores go
+// to random 4-byte cells of the DRAM-resident 4^ls table / locs, ~1 ms each), so it is
+// not the default. The arrival order of the atomics is made deterministic by step 4
+// (most buckets hold 1-3 locations; a bucket over kFixMax goes to k_bucket_big).
+// code(R, p) for the sampled location k; warp-aggregated atomics per equal code (hot
+// seeds -- poly-A, (AC)^n -- come in runs of consecutive k).
+__global__ void __launch_bounds__(kCodeThreads) k_alg1_count(const uint64_t *__restrict__ R, uint32_t ls, uint32_t step,
+                                                             uint64_t k0, uint64_t n_locs, uint32_t *__restrict__ cnt,
+                                                             uint32_t *__restrict__ codes, uint32_t *__restrict__ arr) {
+    pdl_wait();
+    const uint64_t k = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+    const bool valid = k < n_locs;
+    const uint32_t code = valid ? uint32_t(win_fwd(R, (k0 + k) * step) >> (64 - 2 * ls)) : 0xffffffffu;
+    const unsigned active = __ballot_sync(0xffffffffu, valid);
+    if (!valid) return;
+    const unsigned peers = __match_any_sync(active, code);
+    const int leader = __ffs(int(peers)) - 1;
+    uint32_t base = 0;
+    if ((threadIdx.x & 31) == leader) base = atomicAdd(cnt + code, uint32_t(__popc(peers)));
+    base = __shfl_sync(peers, base, leader);
+    codes[k] = code;
+    arr[k] = base + __popc(peers & lanemask_lt());
+}
+
+// per chunk of kChunk seeds: records and occupied seeds (one CTA per chunk)
+__global__ void __launch_bounds__(kCodeThreads) k_cnt_chunk_sums(const uint32_t *__restrict__ cnt, uint64_t nb,
+                                                                 uint32_t *__restrict__ rec, uint32_t *__restrict__ occ) {
+    pdl_wait();
+    __shared__ uint32_t ws[2][kCodeThreads / 32];
+    const uint64_t s0 = uint64_t(blockIdx.x) * kChunk;
+    uint32_t r = 0, o = 0;
+    for (uint64_t i = s0 + threadIdx.x; i < s0 + kChunk && i < nb; i += kCodeThreads) {
+        const uint32_t x = cnt[i];
+        r += x;
+        o += x ? 1u : 0u;
+    }
+#pragma unroll
+    for (int d = 16; d; d >>= 1) {
+        r += __shfl_xor_sync(0xffffffffu, r, d);
+        o += __shfl_xor_sync(0xffffffffu, o, d);
+    }
+    if ((threadIdx.x & 31) == 0) {
+        ws[0][threadIdx.x >> 5] = r;
+        ws[1][threadIdx.x >> 5] = o;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        uint32_t tr = 0, to = 0;
+        for (int k = 0; k < kCodeThreads / 32; ++k) {
+            tr += ws[0][k];
+            to += ws[1][k];
+        }
+        rec[blockIdx.x] = tr;
+        occ[blockIdx.x] = to;
+    }
+}
+
+// Alg. 1 step 3: locs[first(code) + arrival rank] = p, first(code) from the directory
+// just built (rank sector: records before the group + the 2-bit counts below the seed,
+// exact unless one saturates; rank word / saturation: the compact table).
+template <bool kSect>
+__global__ void __launch_bounds__(kCodeThreads) k_alg1_place(const uint32_t *__restrict__ codes,
+                                                             const uint32_t *__restrict__ arr, uint64_t n_locs,
+                                                             uint64_t k0, uint32_t step,
+                                                             const unsigned long long *__restrict__ rankw,
+                                                             const uint4 *__restrict__ rsect,
+                                                             const uint2 *__restrict__ buckets,
+                                                             uint32_t *__restrict__ locs) {
+    pdl_wait();
+    const uint64_t k = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+    if (k >= n_locs) return;
+    const uint32_t code = codes[k], b = code & 31;
+    uint32_t first;
+    if (kSect) {
+        constexpr uint64_t kLo = 0x5555555555555555ull;
+        const uint4 rs = __ldg(rsect + (code >> 5));
+        const uint64_t c2 = (uint64_t(rs.w) << 32) | rs.z;
+        const uint64_t below = b ? c2 & ((1ull << (2 * b)) - 1ull) : 0ull;
+        if ((below & (below >> 1) & kLo) == 0) {  // no saturated count below: exact from the sector
+            first = rs.x + uint32_t(__popcll(below & kLo) + 2 * __popcll(below & ~kLo));
+        } else {
+            first = __ldg(buckets + rs.y + __popcll((below | (below >> 1)) & kLo)).x;
+        }
+    } else {
+        const unsigned long long rw = __ldg(rankw + (code >> 5));
+        const uint32_t rank = uint32_t(rw >> 32) + __popc(uint32_t(rw) & ((1u << b) - 1u));
+        first = __ldg(buckets + rank).x;
+    }
+    locs[first + arr[k]] = uint32_t((k0 + k) * step);
+}
+
+// Alg. 1 step 4: each bucket ascending. One thread per occupied seed: insertion sort up
+// to kFixMax locations (nearly all); larger buckets are listed for k_bucket_big.
+constexpr uint32_t kFixMax = 32;
+__global__ void __launch_bounds__(kCodeThreads) k_bucket_fix(const uint2 *__restrict__ buckets,
+                                                             const unsigned long long *__restrict__ rankw,
+                                                             const uint4 *__restrict__ rsect, uint64_t nb,
+                                                             uint32_t *__restrict__ locs, uint32_t *__restrict__ big,
+                                                             unsigned int *__restrict__ n_big) {
+    pdl_wait();
+    // occupied seeds in total, from the last directory group
+    const uint64_t g = (nb - 1) >> 5;
+    uint64_t n_occ;
+    if (rsect) {
+        const uint4 rs = rsect[g];
+        const uint64_t c2 = (uint64_t(rs.w) << 32) | rs.z;
+        n_occ = rs.y + __popcll((c2 | (c2 >> 1)) & 0x5555555555555555ull);
+    } else {
+        const unsigned long long rw = rankw[g];
+        n_occ = uint32_t(rw >> 32) + __popc(uint32_t(rw));
+    }
+    for (uint64_t r = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; r < n_occ; r += uint64_t(gridDim.x) * blockDim.x) {
+        const uint2 bk = buckets[r];
+        if (bk.y < 2) continue;
+        if (bk.y > kFixMax) {
+            big[atomicAdd(n_big, 1u)] = uint32_t(r);
+            continue;
+        }
+        uint32_t *a = locs + bk.x;
+        for (uint32_t x = 1; x < bk.y; ++x) {
+            const uint32_t v = a[x];
+            uint32_t y = x;
+            while (y > 0 && a[y - 1] > v) {
+                a[y] = a[y - 1];
+                --y;
+            }
+            a[y] = v;
+        }
+    }
+}
+
+// One CTA per listed bucket: a bitonic-type sorting network with ascending
+// compare-exchanges only (the first stage of every merge pairs i with the mirror
+// element), so indices past the bucket act as +infinity and need no padding. In shared
+// memory up to kBigSmem locations, in place in global memory beyond.
+constexpr uint32_t kBigSmem = 16384;
+__device__ __forceinline__ void cmpswap(uint32_t *a, uint32_t i, uint32_t j) {
+    const uint32_t x = a[i], y = a[j];
+    if (x > y) {
+        a[i] = y;
+        a[j] = x;
+    }
+}
+__device__ void net_sort(uint32_t *a, uint32_t n) {
+    uint32_t N = 1;
+    while (N < n) N <<= 1;
+    for (uint32_t k = 2; k <= N; k <<= 1) {
+        for (uint32_t t = threadIdx.x; t < N / 2; t += blockDim.x) {  // mirror stage
+            const uint32_t blk = t / (k / 2), j = t % (k / 2);
+            const uint32_t i0 = blk * k + j, i1 = blk * k + k - 1 - j;
+            if (i1 < n) cmpswap(a, i0, i1);
+        }
+        __syncthreads();
+        for (uint32_t d = k / 4; d >= 1; d >>= 1) {  // half-cleaners
+            for (uint32_t t = threadIdx.x; t < N / 2; t += blockDim.x) {
+                const uint32_t blk = t / d, j = t % d;
+                const uint32_t i0 = blk * 2 * d + j, i1 = i0 + d;
+                if (i1 < n) cmpswap(a, i0, i1);
+            }
+            __syncthreads();
+        }
+    }
+}
+__global__ void __launch_bounds__(1024) k_bucket_big(const uint2 *__restrict__ buckets, const uint32_t *__restrict__ big,
+                                                     const unsigned int *__restrict__ n_big, uint32_t *__restrict__ locs) {
+    pdl_wait();
+    extern __shared__ uint32_t sm[];
+    const unsigned nbig = *n_big;
+    for (unsigned li = blockIdx.x; li < nbig; li += gridDim.x) {
+        const uint2 bk = buckets[big[li]];
+        uint32_t *a = locs + bk.x;
+        if (bk.y <= kBigSmem) {
+            for (uint32_t i = threadIdx.x; i < bk.y; i += blockDim.x) sm[i] = a[i];
+            __syncthreads();
+            net_sort(sm, bk.y);
+            for (uint32_t i = threadIdx.x; i < bk.y; i += blockDim.x) a[i] = sm[i];
+        } else {
+            net_sort(a, bk.y);  // global memory: visible to the block after each barrier
+        }
+        __syncthreads();
     }
 }
 
@@ -664,6 +858,69 @@ cudaError_t launch_ptrs_expand(const unsigned long long *rankw, const uint4 *rse
     if (rsect) pdl_launch(k_ptrs_expand<true>, grid, 256, 0, s, rankw, rsect, buckets, nb, n_locs, ptrs);
     else pdl_launch(k_ptrs_expand<false>, grid, 256, 0, s, rankw, rsect, buckets, nb, n_locs, ptrs);
     note_launch();
+    return cudaGetLastError();
+}
+
+size_t alg1_scratch_bytes(uint32_t ls, uint64_t n_locs) {
+    const uint64_t nb = 1ull << (2 * ls);
+    const uint64_t chunks = (nb + kChunk - 1) / kChunk;
+    return nb * 4 + n_locs * 8 + (chunks + 1) * 4 * 4 + (n_locs / kFixMax + 1) * 4 + 16 * 256;
+}
+
+// Alg. 1 on packed R: codes + counts, directory + compact table (+ chunk sums and
+// scans), placement, per-bucket sort. locs out; scratch >= alg1_scratch_bytes.
+cudaError_t launch_index_alg1(const uint64_t *R, uint32_t ls, uint32_t step, uint64_t k0, uint64_t n_locs,
+                              unsigned long long *rankw, uint4 *rsect, uint2 *buckets, uint32_t *locs, void *scratch,
+                              cudaStream_t s) {
+    const uint64_t nb = 1ull << (2 * ls);
+    const uint64_t chunks = (nb + kChunk - 1) / kChunk;
+    auto align = [](uintptr_t p) { return (p + 255) & ~uintptr_t(255); };
+    uintptr_t a = align(reinterpret_cast<uintptr_t>(scratch));
+    auto *cnt = reinterpret_cast<uint32_t *>(a);
+    a = align(a + nb * 4);
+    auto *codes = reinterpret_cast<uint32_t *>(a);
+    a = align(a + n_locs * 4);
+    auto *arr = reinterpret_cast<uint32_t *>(a);
+    a = align(a + n_locs * 4);
+    auto *rec = reinterpret_cast<uint32_t *>(a);
+    a = align(a + (chunks + 1) * 4);
+    auto *occ = reinterpret_cast<uint32_t *>(a);
+    a = align(a + (chunks + 1) * 4);
+    auto *first = reinterpret_cast<uint32_t *>(a);
+    a = align(a + (chunks + 1) * 4);
+    auto *rank0 = reinterpret_cast<uint32_t *>(a);
+    a = align(a + (chunks + 1) * 4);
+    auto *n_big = reinterpret_cast<unsigned int *>(a);
+    a = align(a + 256);
+    auto *big = reinterpret_cast<uint32_t *>(a);  // occupied seeds over kFixMax (<= n_locs / kFixMax)
+    cudaError_t e = cudaMemsetAsync(cnt, 0, nb * 4, s);
+    if (e == cudaSuccess) e = cudaMemsetAsync(n_big, 0, 4, s);
+    if (e != cudaSuccess) return e;
+    const unsigned grid_k = unsigned((n_locs + kCodeThreads - 1) / kCodeThreads);
+    pdl_launch(k_alg1_count, grid_k, kCodeThreads, 0, s, R, ls, step, k0, n_locs, cnt, codes, arr);
+    pdl_launch(k_cnt_chunk_sums, unsigned(chunks), kCodeThreads, 0, s, cnt, nb, rec, occ);
+    pdl_launch(k_occ_scan, 1, 1024, 0, s, rec, uint32_t(chunks), first);
+    pdl_launch(k_occ_scan, 1, 1024, 0, s, occ, uint32_t(chunks), rank0);
+    constexpr int smem = (kChunk + kChunk / 32) * 4;
+    static bool attr = false;
+    if (!attr) {
+        e = cudaFuncSetAttribute(k_ptrs_fill<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+        if (e == cudaSuccess) e = cudaFuncSetAttribute(k_ptrs_fill<true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+        if (e == cudaSuccess) e = cudaFuncSetAttribute(k_bucket_big, cudaFuncAttributeMaxDynamicSharedMemorySize, int(kBigSmem * 4));
+        if (e != cudaSuccess) return e;
+        attr = true;
+    }
+    if (rsect)
+        pdl_launch(k_ptrs_fill<true, true>, unsigned(chunks), kFillThreads, smem, s, cnt, n_locs, nb, (uint32_t *)nullptr,
+                   rankw, rsect, buckets, first, rank0);
+    else
+        pdl_launch(k_ptrs_fill<false, true>, unsigned(chunks), kFillThreads, smem, s, cnt, n_locs, nb, (uint32_t *)nullptr,
+                   rankw, rsect, buckets, first, rank0);
+    if (rsect) pdl_launch(k_alg1_place<true>, grid_k, kCodeThreads, 0, s, codes, arr, n_locs, k0, step, rankw, rsect, buckets, locs);
+    else pdl_launch(k_alg1_place<false>, grid_k, kCodeThreads, 0, s, codes, arr, n_locs, k0, step, rankw, rsect, buckets, locs);
+    pdl_launch(k_bucket_fix, unsigned(num_sms() * 8), kCodeThreads, 0, s, buckets, rankw, rsect, nb, locs, big, n_big);
+    pdl_launch(k_bucket_big, unsigned(num_sms()), 1024, size_t(kBigSmem * 4), s, buckets, big, n_big, locs);
+    note_launch(9);
     return cudaGetLastError();
 }
 

@@ -29,6 +29,9 @@ struct Options {
                                  // 0 rank words, 1 rank sectors       // index sort: 1 = MSD bucket sort of (code << 32 | p), 0 = stable LSD radix
     int64_t radix_bits = 0;      // LSD digit width: 0 = 9 bits if that saves a pass else 8; or pinned 8, 9, 10
     int64_t pdl = 1;             // programmatic dependent launch between consecutive kernels
+    int64_t index_alg1 = 0;      // Alg. 1 literally (atomic counts, scan, placement, bucket sort): 1 always,
+                                 // -1 for dense indexes (n_locs >= 4^ls / 4), 0 never (default: measured
+                                 // slower everywhere -- C5 L = 20 2.9 vs 1.4 ms, C4 0.40 vs 0.21 ms)
 };
 extern Options g_opt;
 
@@ -129,6 +132,12 @@ cudaError_t launch_split_keys(const uint64_t *keys, uint64_t n, uint32_t *codes,
 cudaError_t launch_seed_codes(const uint64_t *R, uint32_t ls, uint32_t step, uint64_t k0, uint64_t n_locs,
                               uint32_t *codes, uint32_t *locs, cudaStream_t s);
 size_t ptrs_fill_scratch_bytes(uint32_t ls);
+// Alg. 1 as written for dense indexes (index.cu): counts by atomics, prefix sums +
+// directory, placement, per-bucket sort -> locs, directory, compact table.
+size_t alg1_scratch_bytes(uint32_t ls, uint64_t n_locs);
+cudaError_t launch_index_alg1(const uint64_t *R, uint32_t ls, uint32_t step, uint64_t k0, uint64_t n_locs,
+                              unsigned long long *rankw, uint4 *rsect, uint2 *buckets, uint32_t *locs, void *scratch,
+                              cudaStream_t s);
 cudaError_t launch_ptrs_fill(const uint32_t *sorted_codes, uint64_t n_locs, uint32_t ls, uint32_t *ptrs,
                              unsigned long long *rankw, uint4 *rsect, uint2 *buckets, void *scratch,
                              cudaStream_t s);

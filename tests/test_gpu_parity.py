@@ -24,7 +24,7 @@ def _default_options():
     yield
     for k, v in (("find_grid", 0), ("find_spill", 64), ("out_capacity", 0), ("use_bitmap", 1), ("static_lb", 0),
                  ("sort_impl", 0), ("index_msd", 0), ("small_sort", 0), ("radix_bits", 0),
-                 ("rank_sectors", -1), ("rec8", -1), ("index_fused", 0), ("pdl", 1)):
+                 ("rank_sectors", -1), ("rec8", -1), ("index_fused", 0), ("pdl", 1), ("index_alg1", 0)):
         gpumem.set_option(k, v)
 
 
@@ -136,12 +136,15 @@ def test_index_hot_seed_chunks():
     for ls, step in ((13, 1), (12, 3), (5, 2)):
         op, ol = oracle.index(R, ls, step)
         for sect in (0, 1):
-            gpumem.set_option("rank_sectors", sect)
-            p, l = _index_gpu(R, ls, step)
-            assert np.array_equal(p, op) and np.array_equal(l, ol), (ls, step, sect)
+            for alg1 in (0, 1):  # Alg. 1 path: buckets of 70 000 (global sorting network), 20 000, ...
+                gpumem.set_option("rank_sectors", sect)
+                gpumem.set_option("index_alg1", alg1)
+                p, l = _index_gpu(R, ls, step)
+                assert np.array_equal(p, op) and np.array_equal(l, ol), (ls, step, sect, alg1)
 
 
 @pytest.mark.parametrize("opts", [{"small_sort": 1}, {"radix_bits": 8}, {"index_msd": 1}, {"index_fused": 1},
+                                  {"index_alg1": 1}, {"index_alg1": 1, "rank_sectors": 1}, {"index_alg1": 0},
                                   {"index_fused": 1, "rank_sectors": 1, "rec8": 1}])
 def test_index_sort_paths(opts):
     """Every index sort path (single-launch cooperative, multi-launch LSD, MSD) gives
@@ -251,14 +254,14 @@ def test_overflow_retry_grid_spill_and_bitmap_invariance():
     for opt, vals in (("out_capacity", [1, 100]), ("find_grid", [1, 3, 148]), ("find_spill", [1, 2, 10**9]),
                       ("use_bitmap", [0]), ("static_lb", [1]), ("sort_impl", [1, 2, 3]), ("index_msd", [1]), ("small_sort", [1]),
                       ("rank_sectors", [0, 1]), ("rec8", [0, 1]), ("index_fused", [1]),
-                      ("radix_bits", [8, 9, 10]), ("pdl", [0])):
+                      ("radix_bits", [8, 9, 10]), ("pdl", [0]), ("index_alg1", [1, -1])):
         for v in vals:
             gpumem.set_option(opt, v)
             assert np.array_equal(gpu_mems(P.R, P.Q, P.L, P.ls), want), (opt, v)
         gpumem.set_option(opt, {"out_capacity": 0, "find_grid": 0, "find_spill": 64, "use_bitmap": 1,
                                 "static_lb": 0, "sort_impl": 0, "index_msd": 0, "small_sort": 0, "rank_sectors": -1,
                                 "rec8": -1, "index_fused": 0,
-                                "radix_bits": 0, "pdl": 1}[opt])
+                                "radix_bits": 0, "pdl": 1, "index_alg1": 0}[opt])
 
 
 def test_seed_length_and_step_invariance():

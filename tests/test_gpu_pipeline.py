@@ -24,6 +24,7 @@ def _default_options():
     yield
     gpumem.set_option("out_capacity", 0)
     gpumem.set_option("sort_impl", 0)
+    gpumem.set_option("index_alg1", 0)
 
 
 def _dev(x):
@@ -69,6 +70,16 @@ def test_pipeline_sort_skewed(impl, n, m, L):
     want = np.array(pyoracle.homopolymer(n, m, L), dtype=np.uint32).reshape(-1, 3)
     got, _ = pipe_mems("A" * n, "A" * m, L, 1 if L < 13 else 13)
     assert np.array_equal(got, want)
+
+
+@pytest.mark.parametrize("alg1", [0, 1])
+def test_pipeline_index_paths(alg1):
+    """Both index builds (stable radix sort / Alg. 1 as written) under the captured graph."""
+    gpumem.set_option("index_alg1", alg1)
+    for cfg, scale in (("c5_l20", 0.02), ("c1", 1.0)):
+        P = synth.make_pair(cfg, scale=scale)
+        got, _ = pipe_mems(P.R, P.Q, P.L, P.ls, runs=2)
+        assert np.array_equal(got, oracle.mems(P.R, P.Q, P.L, P.ls)), (cfg, alg1)
 
 
 def test_pipeline_random_tiny_vs_brute_force():
