@@ -52,6 +52,9 @@ constexpr int kWarps = kT / 32;
 #endif
 constexpr int kQPT = GM_FIND_QPT;         // query positions per lane per chunk
 constexpr int kChunk = 32 * kQPT;         // 256 positions per warp chunk
+#ifndef GM_HEAVY_CTAS
+#define GM_HEAVY_CTAS 8  // k_heavy CTAs per SM (8 vs 4: C5 L = 20 0.517 vs 0.536 ms)
+#endif
 #ifndef GM_FIND_GRAB
 #define GM_FIND_GRAB 2
 #endif
@@ -603,17 +606,38 @@ __global__ void __launch_bounds__(kT, GM_FIND_MINB) k_find(const FindParams P) {
 #pragma unroll
                     for (int o = 16; o; o >>= 1) rounds = max(rounds, __shfl_xor_sync(0xffffffffu, rounds, o));
                 }
+                uint32_t ent0 = 0;  // entry holding the round's first hit (entries hold >= 1 hit each)
                 for (uint32_t rd = 0; rd < rounds; ++rd) {
                     const uint32_t h = kStatic ? h0 + rd : rd * 32 + lane;
                     const bool has = kStatic ? rd < n_h : h < H;
                     int verdict = kDrop;
                     Hit out{0, 0};
                     uint32_t p = 0, q = 0, e_rec = 0, f_rec = 0;
+                    uint32_t ent = 0;
+                    if (!kStatic) {
+                        // the entries starting inside this round's 32 hits are among the next
+                        // 32: one shared load per lane, an OR-reduction of their start bits,
+                        // and each lane's entry is ent0 + the starts at or before it
+                        const uint32_t hb = rd * 32, cand = ent0 + 1 + lane;
+                        uint32_t bit = 0;
+                        if (cand < E) {
+                            const uint32_t off = s.e_off[cand];
+                            if (off < hb + 32) bit = 1u << (off - hb);
+                        }
+                        const uint32_t starts = __reduce_or_sync(0xffffffffu, bit);
+                        ent = ent0 + __popc(starts & ((2u << lane) - 1u));
+                        const uint32_t last = ent0 + __popc(starts);  // entry of hit hb + 31
+                        ent0 = (last + 1 < E && s.e_off[last + 1] <= hb + 32) ? last + 1 : last;
+                    }
                     if (has) {
-                        uint32_t lo = 0, hi = E;  // largest entry i with e_off[i] <= h
-                        while (hi - lo > 1) {
-                            const uint32_t mid = (lo + hi) >> 1;
-                            if (s.e_off[mid] <= h) lo = mid; else hi = mid;
+                        uint32_t lo = ent;
+                        if (kStatic) {
+                            uint32_t lo2 = 0, hi = E;  // largest entry i with e_off[i] <= h
+                            while (hi - lo2 > 1) {
+                                const uint32_t mid = (lo2 + hi) >> 1;
+                                if (s.e_off[mid] <= h) lo2 = mid; else hi = mid;
+                            }
+                            lo = lo2;
                         }
                         q = q0 + s.e_q[lo];
                         uint32_t rl;
@@ -750,8 +774,8 @@ cudaError_t launch_coop(const FindParams &p, cudaStream_t s) {
 }
 
 cudaError_t launch_heavy(const FindParams &p, cudaStream_t s) {
-    if (p.rec8) pdl_launch(k_heavy<true>, num_sms() * 4, kT, 0, s, p);
-    else pdl_launch(k_heavy<false>, num_sms() * 4, kT, 0, s, p);
+    if (p.rec8) pdl_launch(k_heavy<true>, num_sms() * GM_HEAVY_CTAS, kT, 0, s, p);
+    else pdl_launch(k_heavy<false>, num_sms() * GM_HEAVY_CTAS, kT, 0, s, p);
     note_launch();
     return cudaGetLastError();
 }
