@@ -445,24 +445,37 @@ __global__ void __launch_bounds__(kT, GM_FIND_MINB) k_find(const FindParams P) {
     // L2 priorities: lookup tables stay, streamed data goes first (records only when
     // they cannot stay resident anyway, P.recs_stream)
 
-    for (;;) {
-        uint32_t grab = 0;
-        if (lane == 0) grab = atomicAdd(P.tile_ctr, 1u);
-        grab = __shfl_sync(0xffffffffu, grab, 0);
-        const uint64_t c_first = uint64_t(grab) * kGrab;
-        if (c_first >= P.n_tiles) break;
-        const uint64_t c_last = min(c_first + kGrab, P.n_tiles);
-        for (uint64_t c = c_first; c < c_last; ++c) {
+    // chunks in scheduler order; the next chunk (and, at a grab's end, the next grab) is
+    // claimed and its packed Q words loaded into a register before the current chunk is
+    // processed, so that load's latency hides behind the current chunk's work
+    auto grab_next = [&](uint64_t &c, uint64_t &c_end) {
+        uint32_t g = 0;
+        if (lane == 0) g = atomicAdd(P.tile_ctr, 1u);
+        g = __shfl_sync(0xffffffffu, g, 0);
+        c = uint64_t(g) * kGrab;
+        c_end = min(c + kGrab, P.n_tiles);
+    };
+    auto q_words = [&](uint64_t c) -> uint64_t {  // lane's staged word of chunk c
+        const uint32_t q0 = uint32_t(P.scan_lo + c * kChunk);
+        const uint32_t wb = (q0 >> 5) ? (q0 >> 5) - 1 : 0;
+        if (lane >= kQW || wb + lane >= P.nQw) return 0ull;
+        return kHints ? ld_first_u64(reinterpret_cast<const unsigned long long *>(P.Q) + wb + lane)
+                      : __ldg(P.Q + wb + lane);
+    };
+    uint64_t c, c_end;
+    grab_next(c, c_end);
+    uint64_t qpre = c < P.n_tiles ? q_words(c) : 0ull;
+    while (c < P.n_tiles) {
+        uint64_t cn = c + 1, cn_end = c_end;
+        if (cn >= c_end) grab_next(cn, cn_end);
+        {
             const uint32_t q0 = uint32_t(P.scan_lo + c * kChunk);
             // ---- stage the chunk's Q words (+ halo) in shared memory
             const uint32_t wb = (q0 >> 5) ? (q0 >> 5) - 1 : 0;
             qs.wbase = wb;
-            if (lane < kQW)
-                s.qw[lane] = (wb + lane < P.nQw)
-                                 ? (kHints ? ld_first_u64(reinterpret_cast<const unsigned long long *>(P.Q) + wb + lane)
-                                          : __ldg(P.Q + wb + lane))
-                                 : 0ull;
+            if (lane < kQW) s.qw[lane] = qpre;
             __syncwarp();
+            qpre = cn < P.n_tiles ? q_words(cn) : 0ull;  // the next chunk's words, in flight
 
             // ---- A5: seeds -> bitmap -> bucket ranges
             uint32_t beg[kQPT], cnt[kQPT];
@@ -659,6 +672,8 @@ __global__ void __launch_bounds__(kT, GM_FIND_MINB) k_find(const FindParams P) {
             }
             __syncwarp();
         }
+        c = cn;
+        c_end = cn_end;
     }
     if (nq) drain_deferred<kL>(P, s, nq, nbuf, nq);
     warp_emit(P, s, nbuf, false, Hit{0, 0}, true);
