@@ -213,8 +213,8 @@ gpumem_status gpumem_merge_sorted(const gpumem_triple *const *dev_runs, const ui
  *
  * gpumem_pipeline_stats -- find statistics of the last result.
  * gpumem_pipeline_profile -- per-stage device time of the last completed run (the
- *  stage events are event-record nodes of the graph), aggregated by name as
- *  gpumem_profile_read;
+ *  stage events are event-record nodes of the graph, present per option "pipe_events"),
+ *  aggregated by name as gpumem_profile_read;
  *  synchronises those events. Returns the number of entries written.
  * gpumem_free(pl) synchronises the stream and releases everything.
  */
@@ -266,6 +266,9 @@ gpumem_status gpumem_set_allocator(void *(*alloc_fn)(size_t bytes, void *cuda_st
  *                     placement, per-bucket sort) instead of the stable radix sort;
  *                     -1: only for dense indexes (n_locs >= 4^ls / 4); 0 (default): never
  *                     (measured slower: random atomics/stores into the 4^ls table)
+ *  "pipe_events"      stage event nodes captured into a pipeline graph (read at capture):
+ *                     0 (default) none, 2 around the find kernel only, 1 at every stage
+ *                     boundary (gpumem_pipeline_profile; each node costs a few us per run)
  *  "pdl"              1 (default): programmatic dependent launch between consecutive
  *                     kernels (each waits for its predecessor with griddepcontrol.wait);
  *                     0: ordinary launches

@@ -210,6 +210,8 @@ void dfree(void *p, cudaStream_t s) {
 Stage::Stage(const char *name, cudaStream_t st) : slot(-1), s(st), vec(nullptr) {
     std::vector<StageRec> *v = (t_cap && t_cap->recs) ? t_cap->recs : (g_prof ? &g_recs : nullptr);
     if (!v) return;
+    if (t_cap && t_cap->recs && g_opt.pipe_events == 0) return;                       // no stage events
+    if (t_cap && t_cap->recs && g_opt.pipe_events == 2 && strcmp(name, "find")) return;  // find's only
     std::lock_guard<std::mutex> g(g_prof_mu);
     StageRec r{name, take_event(), take_event(), g_launches.load(), 0};
     // in a capture: an event record node of the graph (timed on every launch)
@@ -572,6 +574,7 @@ gpumem_status gpumem_set_option(const char *name, int64_t value) {
     }
     else if (!strcmp(name, "index_msd")) g_opt.index_msd = value ? 1 : 0;
     else if (!strcmp(name, "pdl")) g_opt.pdl = value ? 1 : 0;
+    else if (!strcmp(name, "pipe_events")) g_opt.pipe_events = value < 0 ? 0 : (value > 2 ? 2 : value);
     else if (!strcmp(name, "index_alg1")) g_opt.index_alg1 = value < 0 ? -1 : (value ? 1 : 0);
     else if (!strcmp(name, "index_fused")) g_opt.index_fused = value ? 1 : 0;
     else if (!strcmp(name, "small_sort")) g_opt.small_sort = value ? 1 : 0;

@@ -29,6 +29,8 @@ struct Options {
                                  // 0 rank words, 1 rank sectors       // index sort: 1 = MSD bucket sort of (code << 32 | p), 0 = stable LSD radix
     int64_t radix_bits = 0;      // LSD digit width: 0 = 9 bits if that saves a pass else 8; or pinned 8, 9, 10
     int64_t pdl = 1;             // programmatic dependent launch between consecutive kernels
+    int64_t pipe_events = 0;     // stage event nodes in a pipeline graph: 0 none (fastest), 2 find only, 1 every
+                                 // stage (each node costs a few us: C4 1.263 / 1.280 / 1.311 ms per step)
     int64_t index_alg1 = 0;      // Alg. 1 literally (atomic counts, scan, placement, bucket sort): 1 always,
                                  // -1 for dense indexes (n_locs >= 4^ls / 4), 0 never (default: measured
                                  // slower everywhere -- C5 L = 20 2.9 vs 1.4 ms, C4 0.40 vs 0.21 ms)

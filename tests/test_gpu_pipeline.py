@@ -25,6 +25,7 @@ def _default_options():
     gpumem.set_option("out_capacity", 0)
     gpumem.set_option("sort_impl", 0)
     gpumem.set_option("index_alg1", 0)
+    gpumem.set_option("pipe_events", 0)
 
 
 def _dev(x):
@@ -100,6 +101,7 @@ def test_pipeline_qrange_and_recapture():
         got, _ = pipe_mems(P.R, P.Q, P.L, P.ls, q_range=(a, b))
         assert np.array_equal(got, oracle.mems(P.R, P.Q, P.L, P.ls, 0, a, b)), (a, b)
     # new input buffers (other contents, same sizes) -> recapture on the same pipeline
+    gpumem.set_option("pipe_events", 1)  # stage events in the graph (profile below)
     Rt, Qt = _dev(P.R), _dev(P.Q)
     pl = gpumem.Pipeline(len(P.R), n, P.ls, P.L)
     pl.run(Rt, Qt)

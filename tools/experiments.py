@@ -36,6 +36,7 @@ def run(R_dev, Q_dev, L, ls, steps, warmup, q_range=None, opts=None):
         gm.set_option(k, v)
     flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
     stream = torch.cuda.current_stream()
+    gm.set_option("pipe_events", 1)  # stage times from event nodes (each costs a few us)
     pl = gm.Pipeline(R_dev.numel(), Q_dev.numel(), ls, L, q_range)  # captured with these options
     tot, prof_acc, n_mems = 0.0, {}, 0
     for i in range(warmup + steps):

@@ -12,7 +12,7 @@ from paper_conf_ipps_abu_dolehkac14_b200 import gpumem as gm, synth  # noqa: E40
 
 DEFAULTS = {"find_grid": 0, "find_spill": 64, "out_capacity": 0, "use_bitmap": 1, "static_lb": 0, "sort_impl": 0,
             "index_msd": 0, "small_sort": 0, "radix_bits": 0, "rank_sectors": -1, "rec8": -1, "index_fused": 0,
-            "pdl": 1, "index_alg1": 0}
+            "pdl": 1, "index_alg1": 0, "pipe_events": 1}  # stage times (event nodes cost ~50 us)
 cfg = sys.argv[1]
 P = synth.make_pair(cfg)
 R = torch.from_numpy(P.R).cuda()
