@@ -6,7 +6,8 @@
 // the sampled-R hits of those positions. Every warp of a persistent grid is an
 // independent worker: it grabs kGrab chunks at a time from an atomic counter and
 // never waits on other warps (no CTA barriers). Per chunk:
-//  stage   the chunk's packed Q words (+ halo) go to the warp's shared memory;
+//  stage   the chunk's packed Q words (+ halo) go to the warp's shared memory (loaded
+//          into a register while the previous chunk was processed);
 //  A5      each lane cuts kQPT consecutive seeds out of one 64-bit window, probes
 //          the rank word of each seed (occupancy bit + running rank, 8 B per 32
 //          seeds, 16 MB at ls = 13, L2-resident) and, for occupied seeds, reads
@@ -21,9 +22,10 @@
 //          a global queue drained by k_heavy (reference-axis tiles of the hot
 //          seeds, Fig. 6 :268-270); the rest become (q, bucket) entries with a
 //          warp-scanned prefix of their hit counts;
-//  A6      the chunk's hits are dealt 32 at a time to the lanes (hit h -> entry by
-//          binary search), replacing Alg. 2's proactive load balancing (:120-149)
-//          and Alg. 3's combine (:155-169);
+//  A6      the chunk's hits are dealt 32 at a time to the lanes (hit h -> its entry
+//          from an OR-reduction of the entry starts inside the round), replacing
+//          Alg. 2's proactive load balancing (:120-149) and Alg. 3's combine
+//          (:155-169);
 //  A7      left extension capped at step. The seed record carries the 16 bases
 //          left of p and the 32 bases right of the seed (index.cu), so a random
 //          hit is decided without touching R. e == step means the sampled seed at
