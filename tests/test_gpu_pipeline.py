@@ -164,3 +164,28 @@ def test_pipeline_host_inputs():
         assert pl.result() == len(want), src
         assert np.array_equal(pl.numpy(), want), src
     pl.free()
+
+
+@pytest.mark.parametrize("events,want", [(0, set()), (2, {"find"}), (1, {"pack", "index.sort", "find", "sort"})])
+def test_pipeline_event_modes(events, want):
+    """pipe_events: no stage events (default), find's only (the timed bench graph), every
+    stage; the MEM set never depends on it."""
+    P = synth.make_pair("c1")
+    gpumem.set_option("pipe_events", events)
+    Rt, Qt = _dev(P.R), _dev(P.Q)
+    pl = gpumem.Pipeline(len(P.R), len(P.Q), P.ls, P.L)
+    pl.run(Rt, Qt)
+    pl.result()
+    prof = pl.profile()
+    assert want <= set(prof) and (events != 0 or not prof) and (events != 2 or set(prof) == {"find"})
+    assert np.array_equal(pl.numpy(), oracle.mems(P.R, P.Q, P.L, P.ls))
+    pl.free()
+
+
+def test_gather_ceiling_diag():
+    """The instrumentation kernel bench.py uses for k_find's ceiling runs and scales."""
+    a = gpumem.gather_ceiling(10_000_000, 16 << 20)
+    b = gpumem.gather_ceiling(40_000_000, 16 << 20)
+    assert 0 < a < b < 50 * a
+    with pytest.raises(gpumem.GpumemError):
+        gpumem.gather_ceiling(0, 16 << 20)
