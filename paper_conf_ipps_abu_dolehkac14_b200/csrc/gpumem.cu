@@ -96,6 +96,8 @@ struct CapCtx {
     unsigned long long *host = nullptr;   // pinned: [0, 8) find counters, [8] R flag, [9] Q flag
     uint64_t out_cap = 0, coop_cap = 0, spill_cap = 0, span = 0;
     uint64_t expect_n = 0;                // capture: the measuring run's MEM count (sort choice)
+    cudaStream_t side = nullptr;          // pipeline: the seed records are built here, next to the
+    cudaEvent_t ev_a = nullptr, ev_b = nullptr;  // directory fill on the main stream (fork / join)
     gpumem_mems *mems = nullptr;
 };
 thread_local CapCtx *t_cap = nullptr;
@@ -358,6 +360,7 @@ struct gpumem_pipeline {
     cudaStream_t user;                     // the caller's stream (runs are ordered on it by events)
     cudaStream_t stream;                   // the pipeline's own stream: capture, launches, fallback
     cudaStream_t side;                     // runs pack Q next to the index build
+    cudaStream_t side2;                    // runs the seed records next to the directory fill
     cudaEvent_t ev_in, ev_out, ev_join;
     uint64_t nR, nQ, q_begin, q_end;
     uint32_t ls, L;
@@ -367,6 +370,7 @@ struct gpumem_pipeline {
     cudaGraph_t graph;                     // the captured path (one launch per run)
     cudaGraphExec_t exec;
     cudaEvent_t ev_fork;                   // side-stream fork inside the graph
+    cudaEvent_t ev_ra, ev_rb;              // fork / join of the seed-record build (index)
     char *stage;                           // host-input runs: device copies of R and Q (nR + nQ bytes)
     cudaStream_t copy;                     // ... copied on this stream
     cudaEvent_t ev_r, ev_q;                // R / Q copied
@@ -449,6 +453,9 @@ gpumem_status pipeline_capture(gpumem_pipeline *pl, const char *R, const char *Q
     m.mode = 1;
     m.deferred = true;
     m.host = pl->host;
+    m.side = pl->side2;
+    m.ev_a = pl->ev_ra;
+    m.ev_b = pl->ev_rb;
     gpumem_seq *hR, *hQ;
     gpumem_index *hI;
     gpumem_mems *hM;
@@ -469,6 +476,9 @@ gpumem_status pipeline_capture(gpumem_pipeline *pl, const char *R, const char *Q
     c.cap = pl->arena_bytes;
     c.deferred = true;
     c.host = pl->host;
+    c.side = pl->side2;
+    c.ev_a = pl->ev_ra;
+    c.ev_b = pl->ev_rb;
     c.recs = &pl->recs;
     c.expect_n = pl->host[0];
     CK(cudaStreamBeginCapture(s, cudaStreamCaptureModeRelaxed), "begin capture");
@@ -662,9 +672,13 @@ void gpumem_free(void *handle) {
         cudaEventDestroy(pl->ev_r);
         cudaEventDestroy(pl->ev_q);
         cudaEventDestroy(pl->ev_fork);
+        cudaEventDestroy(pl->ev_ra);
+        cudaEventDestroy(pl->ev_rb);
         ws_release_stream(pl->device, pl->stream);
         cudaStreamSynchronize(pl->side);
         cudaStreamDestroy(pl->side);
+        cudaStreamSynchronize(pl->side2);
+        cudaStreamDestroy(pl->side2);
         cudaEventDestroy(pl->ev_join);
         cudaStreamDestroy(pl->stream);
         pl->magic = 0;
@@ -906,10 +920,24 @@ static gpumem_status index_build_impl(const gpumem_seq *R, uint32_t ls, uint32_t
         codes_sorted = alt ? codes1 : codes0;
         locs = alt ? locs1 : locs0;
     }
+    // the directory (from the sorted codes) and the seed records (from locs and R) are
+    // independent: in a pipeline the records are built on its side stream meanwhile
+    const bool fork = t_cap && t_cap->side && n_locs && !recs_done && !fill_done;
+    if (fork) {
+        CK(cudaEventRecord(t_cap->ev_a, s), "fork");
+        CK(cudaStreamWaitEvent(t_cap->side, t_cap->ev_a, 0), "fork");
+        {
+            Stage g("index.recs", t_cap->side);
+            CK(launch_seed_recs(R->words, ls, locs, n_locs, recs, rec8, t_cap->side), "seed records");
+        }
+        CK(cudaEventRecord(t_cap->ev_b, t_cap->side), "join");
+        recs_done = true;
+    }
     if (!fill_done) {
         Stage g("index.ptrs", s);
         CK(launch_ptrs_fill(codes_sorted, n_locs, ls, ptrs, rankw, rsect, buckets, fill_scratch, s), "ptrs fill");
     }
+    if (fork) CK(cudaStreamWaitEvent(s, t_cap->ev_b, 0), "join");
     if (n_locs && !recs_done) {
         Stage g("index.recs", s);
         CK(launch_seed_recs(R->words, ls, locs, n_locs, recs, rec8, s), "seed records");
@@ -1225,8 +1253,11 @@ gpumem_status gpumem_pipeline_create(uint64_t r_len, uint64_t q_len, uint32_t se
     // own, ordered after / before the caller's stream by events
     if (cudaStreamCreateWithFlags(&pl->stream, cudaStreamNonBlocking) != cudaSuccess ||
         cudaStreamCreateWithFlags(&pl->side, cudaStreamNonBlocking) != cudaSuccess ||
+        cudaStreamCreateWithFlags(&pl->side2, cudaStreamNonBlocking) != cudaSuccess ||
         cudaEventCreateWithFlags(&pl->ev_join, cudaEventDisableTiming) != cudaSuccess ||
         cudaEventCreateWithFlags(&pl->ev_fork, cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreateWithFlags(&pl->ev_ra, cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreateWithFlags(&pl->ev_rb, cudaEventDisableTiming) != cudaSuccess ||
         cudaEventCreateWithFlags(&pl->ev_r, cudaEventDisableTiming) != cudaSuccess ||
         cudaEventCreateWithFlags(&pl->ev_q, cudaEventDisableTiming) != cudaSuccess ||
         cudaEventCreateWithFlags(&pl->ev_in, cudaEventDisableTiming) != cudaSuccess ||
