@@ -252,16 +252,10 @@ gpumem_status gpumem_set_allocator(void *(*alloc_fn)(size_t bytes, void *cuda_st
  *  "use_bitmap"       1 (default) probe the rank words + bucket table, 0 probe ptrs only
  *  "static_lb"        1: no hit redistribution across lanes (load-balancing ablation)
  *  "sort_impl"        output sort: 0 (default) auto by size, 1 stable LSD radix sort,
- *                     2 MSD bucket sort, 3 hybrid (LSD passes over the top 16 key bits,
- *                     then shared-memory sorts of the equal-prefix runs); in a pipeline
- *                     0 picks MSD or LSD by the MEM count of its measuring run
- *  "index_msd"        index sort: 0 (default) stable LSD radix, 1 MSD bucket sort
- *  "index_fused"      1 (ls >= 9): group radix passes + one fused counting/placement
- *                     kernel; 0 (default): full radix sort, ptrs fill and record gather
+ *                     2 MSD bucket sort; in a pipeline 0 picks MSD or LSD by the MEM
+ *                     count of its measuring run
  *  "rec8"             seed records: -1 (default) auto (8-byte when step <= 8), 0 16-byte, 1 8-byte
  *  "rank_sectors"     lookup directory: -1 (default) auto, 0 rank words, 1 rank sectors
- *  "small_sort"       1: single-launch cooperative radix sorts (index and output) when
- *                     the input fits in shared memory; 0 (default): multi-launch
  *  "index_alg1"       1: PAPER.md Alg. 1 as written (atomic counts, prefix sums,
  *                     placement, per-bucket sort) instead of the stable radix sort;
  *                     -1: only for dense indexes (n_locs >= 4^ls / 4); 0 (default): never

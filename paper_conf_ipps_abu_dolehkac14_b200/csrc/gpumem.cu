@@ -289,7 +289,7 @@ gpumem_status check_device(int *dev) {
 // loop does no allocation at all once warm. gpumem_trim() releases everything.
 enum WsSlot {
     kWsCtr, kWsSpill, kWsKeys, kWsLens, kWsSortK, kWsSortL, kWsSortScratch, kWsCodes0, kWsCodes1,
-    kWsRadix, kWsFill, kWsMergeK, kWsMergeL, kWsPackTmp, kWsCoop, kWsMums, kWsSmall, kWsLocsTmp, kWsSlot, kWsAlg1,
+    kWsRadix, kWsFill, kWsMergeK, kWsMergeL, kWsPackTmp, kWsCoop, kWsMums, kWsAlg1,
     kWsCount
 };
 struct Workspace {
@@ -579,15 +579,12 @@ gpumem_status gpumem_set_option(const char *name, int64_t value) {
     else if (!strcmp(name, "use_bitmap")) g_opt.use_bitmap = value ? 1 : 0;
     else if (!strcmp(name, "static_lb")) g_opt.static_lb = value ? 1 : 0;
     else if (!strcmp(name, "sort_impl")) {
-        if (value < 0 || value > 3) return fail(GPUMEM_ERR_ARG, "sort_impl must be 0, 1, 2 or 3");
+        if (value < 0 || value > 2) return fail(GPUMEM_ERR_ARG, "sort_impl must be 0, 1 or 2");
         g_opt.sort_impl = value;
     }
-    else if (!strcmp(name, "index_msd")) g_opt.index_msd = value ? 1 : 0;
     else if (!strcmp(name, "pdl")) g_opt.pdl = value ? 1 : 0;
     else if (!strcmp(name, "pipe_events")) g_opt.pipe_events = value < 0 ? 0 : (value > 2 ? 2 : value);
     else if (!strcmp(name, "index_alg1")) g_opt.index_alg1 = value < 0 ? -1 : (value ? 1 : 0);
-    else if (!strcmp(name, "index_fused")) g_opt.index_fused = value ? 1 : 0;
-    else if (!strcmp(name, "small_sort")) g_opt.small_sort = value ? 1 : 0;
     else if (!strcmp(name, "rec8")) g_opt.rec8 = value < 0 ? -1 : (value ? 1 : 0);
     else if (!strcmp(name, "rank_sectors")) g_opt.rank_sectors = value < 0 ? -1 : (value ? 1 : 0);
     else if (!strcmp(name, "radix_bits")) {
@@ -831,57 +828,7 @@ static gpumem_status index_build_impl(const gpumem_seq *R, uint32_t ls, uint32_t
     void *recs = sc.get((n_locs ? n_locs : 1) * (rec8 ? sizeof(uint2) : sizeof(uint4)));
     if (!recs) return GPUMEM_ERR_NOMEM;
     bool recs_done = false, fill_done = false;
-    if (n_locs && ls >= 9 && g_opt.index_fused && !g_opt.index_msd && !g_opt.small_sort) {
-        // radix passes over the code bits above the 1024-seed groups, then one fused
-        // kernel: counts, ptrs, stable placement of locs + records, rank directory
-        auto *codes0 = static_cast<uint32_t *>(ws_get(kWsCodes0, n_locs * 4, s));
-        auto *codes1 = static_cast<uint32_t *>(ws_get(kWsCodes1, n_locs * 4, s));
-        auto *locs1 = static_cast<uint32_t *>(ws_get(kWsLocsTmp, n_locs * 4, s));
-        void *scratch = ws_get(kWsRadix, radix_scratch_bytes(n_locs), s);
-        void *lscratch = ws_get(kWsFill, index_local_scratch_bytes(ls), s);
-        if (!codes0 || !codes1 || !locs1 || !scratch || !lscratch) return GPUMEM_ERR_NOMEM;
-        {
-            Stage g("index.codes", s);
-            CK(launch_seed_codes(R->words, ls, step, k0, n_locs, codes0, locs1, s), "seed codes");
-        }
-        bool alt = false;
-        {
-            Stage g("index.sort", s);
-            CK(radix_sort_u32(codes0, locs1, codes1, locs0, n_locs, int(2 * ls), scratch, s, &alt, 10),
-               "seed group sort");
-        }
-        // the pairs are in (codes0, locs1) or, after an odd number of passes, (codes1, locs0);
-        // the final locs go to whichever of locs0 / locs1 is free, and that one is kept
-        const uint32_t *gc = alt ? codes1 : codes0;
-        const uint32_t *gp = alt ? locs0 : locs1;
-        uint32_t *out_locs = locs0;
-        if (alt) {  // locs0 holds the input: write into a fresh kept buffer
-            out_locs = static_cast<uint32_t *>(sc.get(n_locs * 4));
-            if (!out_locs) return GPUMEM_ERR_NOMEM;
-        }
-        {
-            Stage g("index.ptrs", s);
-            auto *slot = static_cast<uint32_t *>(ws_get(kWsSlot, index_local_slot_bytes(n_locs), s));
-            if (!slot) return GPUMEM_ERR_NOMEM;
-            CK(launch_index_local(gc, gp, n_locs, ls, R->words, ptrs, rankw, rsect, buckets, out_locs, recs, rec8,
-                                  slot, lscratch, s),
-               "index local");
-        }
-        locs = out_locs;
-        recs_done = fill_done = true;
-    } else if (n_locs && !rec8 && !g_opt.index_msd && g_opt.small_sort && n_locs <= small_sort_max_n(4)) {
-        // one cooperative launch: seed codes from R, stable sort, codes + locs + records
-        auto *codes1 = static_cast<uint32_t *>(ws_get(kWsCodes1, n_locs * 4, s));
-        void *scratch = ws_get(kWsSmall, small_sort_scratch_bytes(n_locs, 4), s);
-        if (!codes1 || !scratch) return GPUMEM_ERR_NOMEM;
-        {
-            Stage g("index.sort", s);
-            CK(small_sort_index(R->words, ls, step, k0, n_locs, codes1, locs0, static_cast<uint4 *>(recs), scratch, s), "seed sort");
-        }
-        codes_sorted = codes1;
-        recs_done = true;
-    } else if (n_locs && !g_opt.index_msd &&
-               (g_opt.index_alg1 > 0 || (g_opt.index_alg1 < 0 && n_locs * 4 >= nb))) {
+    if (n_locs && (g_opt.index_alg1 > 0 || (g_opt.index_alg1 < 0 && n_locs * 4 >= nb))) {
         // dense index: Alg. 1 literally (atomic counts, prefix sums, placement, bucket sort)
         void *scratch = ws_get(kWsAlg1, alg1_scratch_bytes(ls, n_locs), s);
         if (!scratch) return GPUMEM_ERR_NOMEM;
@@ -904,18 +851,8 @@ static gpumem_status index_build_impl(const gpumem_seq *R, uint32_t ls, uint32_t
         bool alt = false;
         {
             Stage g("index.sort", s);
-            if (g_opt.index_msd) {  // MSD sort of the unique keys (code << 32 | p)
-                auto *keys = static_cast<uint64_t *>(ws_get(kWsSortK, n_locs * 8, s));
-                void *ms = ws_get(kWsSortScratch, msd_scratch_bytes(n_locs), s);
-                if (!keys || !ms) return GPUMEM_ERR_NOMEM;
-                CK(launch_join_keys(codes0, locs0, n_locs, keys, s), "join keys");
-                CK(msd_sort(keys, nullptr, n_locs, int(2 * ls) + 32, ms, s), "seed sort");
-                CK(launch_split_keys(keys, n_locs, codes1, locs1, s), "split keys");
-                alt = true;
-            } else {
-                CK(radix_sort_u32(codes0, locs0, codes1, locs1, n_locs, int(2 * ls), scratch, s, &alt),
-                   "seed counting sort");
-            }
+            CK(radix_sort_u32(codes0, locs0, codes1, locs1, n_locs, int(2 * ls), scratch, s, &alt),
+               "seed counting sort");
         }
         codes_sorted = alt ? codes1 : codes0;
         locs = alt ? locs1 : locs0;
@@ -1009,18 +946,7 @@ static gpumem_status sort_into_triples(uint64_t *keys, uint32_t *lens, uint64_t 
         Stage g("sort", s);
         // MSD bucket sort (keys are unique): two passes over the data; measured faster than
         // the 7-pass LSD radix up to a few million keys, slower beyond (its 16K-way scatter)
-        if (g_opt.sort_impl == 0 && g_opt.small_sort && n <= small_sort_max_n(8)) {
-            void *scratch = ws_get(kWsSmall, small_sort_scratch_bytes(n, 8), s);
-            if (!scratch) return GPUMEM_ERR_NOMEM;
-            CK(small_sort_triples(keys, lens, n, int(key_bits), qbits, trip, scratch, s), "triple sort");
-        } else if (g_opt.sort_impl == 3) {  // hybrid: 2 LSD passes on the top 16 bits + local sorts
-            auto *k1 = static_cast<uint64_t *>(ws_get(kWsSortK, n * 8, s));
-            auto *l1 = static_cast<uint32_t *>(ws_get(kWsSortL, n * 4, s));
-            void *scratch = ws_get(kWsSortScratch, hybrid_scratch_bytes(), s);
-            if (!k1 || !l1 || !scratch) return GPUMEM_ERR_NOMEM;
-            CK(hybrid_sort_triples(keys, lens, k1, l1, nullptr, n, int(key_bits), scratch, s, trip, qbits),
-               "triple sort");
-        } else if (g_opt.sort_impl == 2 || (g_opt.sort_impl == 0 && n <= kMsdMaxN)) {
+        if (g_opt.sort_impl == 2 || (g_opt.sort_impl == 0 && n <= kMsdMaxN)) {
             void *scratch = ws_get(kWsSortScratch, msd_scratch_bytes(n), s);
             if (!scratch) return GPUMEM_ERR_NOMEM;
             CK(msd_sort(keys, lens, n, int(key_bits), scratch, s, trip, qbits), "triple sort");
@@ -1131,7 +1057,6 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
         int impl = int(g_opt.sort_impl);
         if (impl == 0) impl = (t_cap->mode == 2 && t_cap->expect_n > kMsdMaxN) ? 1 : 2;
         size_t sbytes = msd_scratch_bytes(cap);
-        if (hybrid_scratch_bytes() > sbytes) sbytes = hybrid_scratch_bytes();
         if (radix_scratch_bytes(cap) > sbytes) sbytes = radix_scratch_bytes(cap);
         void *scratch = ws_get(kWsSortScratch, sbytes, s);  // sized for every choice: the measuring
         auto *k1 = static_cast<uint64_t *>(ws_get(kWsSortK, cap * 8, s));  // run and the capture agree
@@ -1155,9 +1080,7 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
         {
             Stage g("sort", s);
             const int kb = int(bits_for(nR) + P.qbits);
-            if (impl == 3) {
-                CK(hybrid_sort_triples(keys, lens, k1, l1, ctr, cap, kb, scratch, s, trip, P.qbits), "triple sort");
-            } else if (impl == 2) {
+            if (impl == 2) {
                 CK(msd_sort_dev(keys, lens, ctr, cap, kb, scratch, s, trip, P.qbits), "triple sort");
             } else {
                 bool alt = false;

@@ -580,218 +580,6 @@ __global__ void __launch_bounds__(kCodeThreads) k_seed_recs(const uint64_t *__re
     else static_cast<uint4 *>(recs)[k] = make_uint4(p, left, uint32_t(right), uint32_t(right >> 32));
 }
 
-// ---------------------------------------------------------------- fused local pass
-// Decoupled look-back over chunks (warp 0): status word = flag | value, one 64-bit store.
-constexpr uint64_t kStAgg = 1ull << 62;
-constexpr uint64_t kStInc = 2ull << 62;
-constexpr uint64_t kStMask = (1ull << 62) - 1;
-
-__device__ __forceinline__ void chunk_publish(unsigned long long *status, uint64_t chunk, unsigned long long agg) {
-    volatile unsigned long long *st = status;
-    st[chunk] = (chunk == 0 ? kStInc : kStAgg) | agg;
-}
-
-// Exclusive prefix of the published aggregates over chunks 0..chunk-1 (warp 0 only;
-// 32 predecessors per step); publishes this chunk's inclusive value.
-__device__ __forceinline__ unsigned long long chunk_lookback(unsigned long long *status, uint64_t chunk,
-                                                             unsigned long long agg) {
-    const int lane = threadIdx.x & 31;
-    volatile unsigned long long *st = status;
-    if (chunk == 0) return 0;
-    unsigned long long excl = 0;
-    int64_t c = int64_t(chunk) - 1;
-    for (;;) {
-        const int64_t idx = c - lane;
-        const unsigned long long sv = idx >= 0 ? st[idx] : kStInc;
-        const unsigned long long f = sv & ~kStMask;
-        const unsigned inc_m = __ballot_sync(0xffffffffu, f == kStInc);
-        const unsigned zero_m = __ballot_sync(0xffffffffu, f == 0);
-        const int first_inc = inc_m ? __ffs(int(inc_m)) - 1 : 32;
-        const unsigned need = first_inc >= 31 ? 0xffffffffu : ((2u << first_inc) - 1u);
-        if (zero_m & need) continue;  // a predecessor has not published yet
-        unsigned long long part = (lane <= first_inc) ? (sv & kStMask) : 0ull;
-#pragma unroll
-        for (int o = 16; o; o >>= 1) part += __shfl_down_sync(0xffffffffu, part, o);
-        excl += __shfl_sync(0xffffffffu, part, 0);
-        if (first_inc < 32) break;
-        c -= 32;
-    }
-    if (lane == 0) st[chunk] = kStInc | (excl + agg);
-    return excl;
-}
-
-// Seed record of location p (16-byte or 8-byte layout, see k_seed_recs).
-template <bool kRec8>
-__device__ __forceinline__ void put_rec(const uint64_t *__restrict__ R, uint32_t ls, uint32_t p, void *recs,
-                                        uint64_t k) {
-    uint32_t left;
-    uint64_t right;
-    if (p >= 16) {
-        const uint64_t x = p - 16, w = x >> 5;
-        const uint64_t w0 = __ldg(R + w), w1 = __ldg(R + w + 1), w2 = __ldg(R + w + 2);
-        const uint32_t sx = uint32_t(x & 31) * 2;
-        left = uint32_t(((w0 << sx) | ((w1 >> 1) >> (63 - sx))) >> 32);
-        const uint32_t o = uint32_t(x & 31) + 16 + ls;
-        const uint32_t so = (o & 31) * 2;
-        const uint64_t a = o < 32 ? w0 : w1, b = o < 32 ? w1 : w2;
-        right = (a << so) | ((b >> 1) >> (63 - so));
-    } else {
-        left = uint32_t(win_back(R, p));
-        right = win_fwd(R, uint64_t(p) + ls);
-    }
-    if (kRec8) static_cast<uint2 *>(recs)[k] = make_uint2(p, (left & 0xffffu) | uint32_t(right >> 48) << 16);
-    else static_cast<uint4 *>(recs)[k] = make_uint4(p, left, uint32_t(right), uint32_t(right >> 32));
-}
-
-// The last step of the index build, one CTA per chunk of kChunk (16384) seeds, on
-// (code, p) pairs already sorted stably by code bits [10, 2 ls) -- i.e. grouped by
-// 1024-seed group, ascending p inside each group (radix passes over the top bits):
-//  count   the chunk's seeds (shared counters; lanes holding the same seed add once);
-//  scan    -> ptrs of the chunk (Alg. 1 steps 1-2), written coalesced;
-//  place   warp w takes group w of the chunk (the same slot range in input and output)
-//          and gives each pair the slot ptrs[s] + (equal seeds before it in p order):
-//          a stable counting sort, so `locs` is ascending inside every seed (Alg. 1
-//          step 4); then all threads move the pairs and write their seed records;
-//  finish  the counters now hold ptrs[s + 1]; with the chunk's first occupied rank
-//          (decoupled look-back over earlier chunks) they give the rank directory
-//          and the compact {first, count} table.
-// Replaces the last radix pass, the separate ptrs fill and the record gather.
-template <bool kSect, bool kRec8>
-__global__ void __launch_bounds__(kFillThreads) k_index_local(
-    const uint32_t *__restrict__ codes, const uint32_t *__restrict__ ps, uint64_t n, uint64_t n_buckets,
-    const uint64_t *__restrict__ R, uint32_t ls, const uint32_t *__restrict__ chunk_first, uint32_t *__restrict__ ptrs,
-    unsigned long long *__restrict__ rankw, uint4 *__restrict__ rsect, uint2 *__restrict__ buckets,
-    uint32_t *__restrict__ locs, void *__restrict__ recs, uint32_t *__restrict__ slot, unsigned long long *status,
-    unsigned int *ticket) {
-    pdl_wait();
-    extern __shared__ uint32_t cnt[];                // kChunk + kChunk / 32 (a pad word per 32 counters)
-    __shared__ uint32_t wsum[kFillThreads / 32];
-    __shared__ uint32_t wocc[kFillThreads / 32];
-    __shared__ uint32_t gstart[kFillThreads / 32 + 1];
-    __shared__ unsigned long long s_rank0;
-    __shared__ uint32_t s_chunk;
-    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
-    if (tid == 0) s_chunk = atomicAdd(ticket, 1u);  // chunks in launch order (look-back)
-    for (int i = tid; i < kChunk + kChunk / 32; i += kFillThreads) cnt[i] = 0;
-    __syncthreads();
-    const uint32_t c = s_chunk;
-    const uint64_t s0 = uint64_t(c) * kChunk;
-    const uint64_t lo = chunk_first[c], hi = chunk_first[c + 1];
-    // count
-    for (uint64_t base = lo; base < hi; base += kFillThreads) {
-        const uint64_t i = base + tid;
-        const uint32_t d = i < hi ? codes[i] - uint32_t(s0) : 0xffffffffu;
-        const unsigned peers = __match_any_sync(0xffffffffu, d);
-        if (i < hi && lane == __ffs(int(peers)) - 1) atomicAdd(&cnt[d + (d >> 5)], uint32_t(__popc(peers)));
-    }
-    __syncthreads();
-    // scan: thread t owns seeds [32t, 32t + 32) of the chunk
-    uint32_t sum = 0, occ = 0;
-#pragma unroll
-    for (int j = 0; j < kPer; ++j) {
-        const uint32_t x = cnt[tid * (kPer + 1) + j];
-        sum += x;
-        occ |= (x ? 1u : 0u) << j;
-    }
-    const uint32_t nocc = __popc(occ);
-    uint32_t inc = sum, inco = nocc;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        const uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
-        const uint32_t z = __shfl_up_sync(0xffffffffu, inco, o);
-        if (lane >= o) {
-            inc += y;
-            inco += z;
-        }
-    }
-    if (lane == 31) {
-        wsum[w] = inc;
-        wocc[w] = inco;
-    }
-    __syncthreads();
-    uint32_t pre = uint32_t(lo), preo = 0, tot_occ = 0;
-    for (int i = 0; i < kFillThreads / 32; ++i) {
-        if (i < w) {
-            pre += wsum[i];
-            preo += wocc[i];
-        }
-        tot_occ += wocc[i];
-    }
-    pre += inc - sum;
-    preo += inco - nocc;
-    if (tid == 0) chunk_publish(status, c, tot_occ);
-    const uint32_t first_pre = pre;
-#pragma unroll 4
-    for (int j = 0; j < kPer; ++j) {  // counts -> exclusive prefix (= ptrs) in place
-        const uint32_t x = cnt[tid * (kPer + 1) + j];
-        cnt[tid * (kPer + 1) + j] = pre;
-        pre += x;
-    }
-    if ((tid & 31) == 0) gstart[w] = first_pre;  // group w = seeds [1024 w, 1024 w + 1024) starts here
-    if (tid == 0) gstart[kFillThreads / 32] = uint32_t(hi);
-    __syncthreads();
-    // ptrs out, 16 bytes per store (skipped without a dense table)
-    const uint64_t lim = n_buckets - s0 < uint64_t(kChunk) ? n_buckets - s0 : uint64_t(kChunk);
-    if (!ptrs) {
-    } else if (lim == uint64_t(kChunk)) {
-        uint4 *dst = reinterpret_cast<uint4 *>(ptrs + s0);
-        for (int i = tid; i < kChunk / 4; i += kFillThreads) {
-            const int b = 4 * i;
-            const int sp = b + (b >> 5);
-            dst[i] = make_uint4(cnt[sp], cnt[sp + 1], cnt[sp + 2], cnt[sp + 3]);
-        }
-    } else {
-        for (int i = tid; i < int(lim); i += kFillThreads) ptrs[s0 + i] = cnt[i + (i >> 5)];
-    }
-    if (ptrs && s0 == 0 && tid == 0) ptrs[n_buckets] = uint32_t(n);
-    __syncthreads();
-    // place: warp w walks group w in p order; counters advance as cursors. Only the
-    // slots are computed here (shared memory only, so a hot group's long walk stays
-    // short); the moves and record gathers follow with all threads.
-    {
-        const uint32_t g0 = gstart[w], g1 = gstart[w + 1];
-        for (uint32_t base = g0; base < g1; base += 32) {
-            const uint32_t i = base + lane;
-            const bool valid = i < g1;
-            const uint32_t d = valid ? codes[i] - uint32_t(s0) : 0xffffffffu - lane;
-            const unsigned peers = __match_any_sync(0xffffffffu, d);
-            const uint32_t at = valid ? cnt[d + (d >> 5)] : 0u;
-            __syncwarp();
-            if (valid && lane == __ffs(int(peers)) - 1) cnt[d + (d >> 5)] = at + __popc(peers);
-            __syncwarp();
-            if (valid) slot[i] = at + __popc(peers & lanemask_lt());
-        }
-    }
-    __syncthreads();  // slot[] of the whole chunk written (global, read back by other warps)
-    for (uint64_t i = lo + tid; i < hi; i += kFillThreads) {
-        const uint32_t pos = __ldcg(slot + i), p = ps[i];
-        locs[pos] = p;
-        put_rec<kRec8>(R, ls, p, recs, pos);
-    }
-    // finish: counters hold ptrs[s + 1]; counts = differences
-    if (w == 0) {
-        const unsigned long long r0 = chunk_lookback(status, c, tot_occ);
-        if (lane == 0) s_rank0 = r0;
-    }
-    __syncthreads();
-    const uint64_t rank = s_rank0 + preo;
-    uint64_t r = rank;
-    uint32_t prev = first_pre;  // ptrs[first seed of this thread]
-    uint64_t c2 = 0;
-#pragma unroll 4
-    for (int j = 0; j < kPer; ++j) {
-        const uint32_t end = cnt[tid * (kPer + 1) + j];
-        const uint32_t x = end - prev;
-        if (x) buckets[r++] = make_uint2(prev, x);
-        if (kSect) c2 |= uint64_t(x < 3 ? x : 3u) << (2 * j);
-        prev = end;
-    }
-    if (s0 + uint64_t(tid) * kPer < n_buckets) {
-        if (kSect) rsect[(s0 >> 5) + tid] = make_uint4(first_pre, uint32_t(rank), uint32_t(c2), uint32_t(c2 >> 32));
-        else rankw[(s0 >> 5) + tid] = (rank << 32) | occ;
-    }
-}
-
 }  // namespace
 
 cudaError_t launch_seed_recs(const uint64_t *R, uint32_t ls, const uint32_t *locs, uint64_t n_locs, void *recs,
@@ -977,48 +765,5 @@ cudaError_t launch_ptrs_fill(const uint32_t *sorted_codes, uint64_t n_locs, uint
     return cudaGetLastError();
 }
 
-
-size_t index_local_scratch_bytes(uint32_t ls) {
-    const uint64_t nb = 1ull << (2 * ls);
-    const uint64_t chunks = (nb + kChunk - 1) / kChunk;
-    return (chunks + 1) * 4 + chunks * 8 + 3 * 256;
-}
-
-size_t index_local_slot_bytes(uint64_t n_locs) { return (n_locs ? n_locs : 1) * 4; }
-
-cudaError_t launch_index_local(const uint32_t *codes, const uint32_t *ps, uint64_t n_locs, uint32_t ls,
-                               const uint64_t *R, uint32_t *ptrs, unsigned long long *rankw, uint4 *rsect,
-                               uint2 *buckets, uint32_t *locs, void *recs, int rec8, uint32_t *slot, void *scratch,
-                               cudaStream_t s) {
-    const uint64_t nb = 1ull << (2 * ls);
-    const uint64_t chunks = (nb + kChunk - 1) / kChunk;
-    auto align = [](uintptr_t p) { return (p + 255) & ~uintptr_t(255); };
-    uintptr_t a = align(reinterpret_cast<uintptr_t>(scratch));
-    auto *first = reinterpret_cast<uint32_t *>(a);
-    a = align(a + (chunks + 1) * 4);
-    auto *status = reinterpret_cast<unsigned long long *>(a);
-    a = align(a + chunks * 8);
-    auto *ticket = reinterpret_cast<unsigned int *>(a);
-    cudaError_t e = cudaMemsetAsync(status, 0, (chunks * 8 + 255) / 256 * 256 + 4, s);
-    if (e != cudaSuccess) return e;
-    pdl_launch(k_chunk_bounds, unsigned((n_locs + 1 + kCodeThreads - 1) / kCodeThreads), kCodeThreads, 0, s, codes, n_locs,
-                                                                                                    chunks, first);
-    constexpr int smem = (kChunk + kChunk / 32) * 4;
-    static bool attr = false;
-    if (!attr) {
-        for (auto f : {k_index_local<false, false>, k_index_local<false, true>, k_index_local<true, false>,
-                       k_index_local<true, true>}) {
-            e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-            if (e != cudaSuccess) return e;
-        }
-        attr = true;
-    }
-    auto kern = rsect ? (rec8 ? k_index_local<true, true> : k_index_local<true, false>)
-                      : (rec8 ? k_index_local<false, true> : k_index_local<false, false>);
-    pdl_launch(kern, unsigned(chunks), kFillThreads, smem, s, codes, ps, n_locs, nb, R, ls, first, ptrs, rankw, rsect, buckets,
-                                                     locs, recs, slot, status, ticket);
-    note_launch(2);
-    return cudaGetLastError();
-}
 
 }  // namespace gm

@@ -17,16 +17,10 @@ struct Options {
     int64_t use_bitmap = 1;      // 1: rank-word probe + compact bucket table; 0: read the dense ptrs
     int64_t static_lb = 0;       // 1: each lane processes its own positions' hits (LB ablation)
     int64_t sort_impl = 0;       // output sort: 0 = auto (MSD below kMsdMaxN keys, else LSD), 1 = stable LSD radix
-                                 // (radix.cu), 2 = MSD bucket sort (msd.cu), 3 = hybrid (msd.cu)
-    int64_t small_sort = 0;      // 1: single-launch cooperative sorts when the input fits (small_sort.cu;
-                                 // measured slower at C4: its scattered global writes are not coalesced)
-    int64_t index_msd = 0;
-    int64_t index_fused = 0;     // 1: radix passes over the code bits above 1024-seed groups + the fused
-                                 // local kernel (ls >= 9; measured slower: 0.25 vs 0.20 ms at C4);
-                                 // 0: full radix sort + ptrs fill + record gather
+                                 // (radix.cu), 2 = MSD bucket sort (msd.cu)
     int64_t rec8 = -1;           // seed records: -1 auto (8-byte when step <= 8), 0 16-byte, 1 8-byte
     int64_t rank_sectors = -1;   // lookup directory: -1 auto (sectors when the compact table exceeds L2/4),
-                                 // 0 rank words, 1 rank sectors       // index sort: 1 = MSD bucket sort of (code << 32 | p), 0 = stable LSD radix
+                                 // 0 rank words, 1 rank sectors
     int64_t radix_bits = 0;      // LSD digit width: 0 = 9 bits if that saves a pass else 8; or pinned 8, 9, 10
     int64_t pdl = 1;             // programmatic dependent launch between consecutive kernels
     int64_t pipe_events = 0;     // stage event nodes in a pipeline graph: 0 none (fastest), 2 find only, 1 every
@@ -100,16 +94,6 @@ cudaError_t radix_sort_u64(uint64_t *k0, uint32_t *v0, uint64_t *k1, uint32_t *v
                            const unsigned long long *dn = nullptr);
 size_t radix_scratch_bytes(uint64_t n);
 
-// Single-launch (cooperative) stable LSD radix sorts for small inputs (small_sort.cu):
-// n <= small_sort_max_n(key bytes). The index variant computes the seed codes of the
-// sampled locations from packed R itself and writes sorted codes, locs and seed records.
-uint64_t small_sort_max_n(int key_bytes);
-size_t small_sort_scratch_bytes(uint64_t n, int key_bytes);
-cudaError_t small_sort_index(const uint64_t *R, uint32_t ls, uint32_t step, uint64_t k0, uint64_t n_locs,
-                             uint32_t *codes, uint32_t *locs, uint4 *recs, void *scratch, cudaStream_t s);
-cudaError_t small_sort_triples(const uint64_t *keys, const uint32_t *lens, uint64_t n, int bits, uint32_t qbits,
-                               gpumem_triple *out, void *scratch, cudaStream_t s);
-
 // MSD bucket sort of unique u64 keys (+ optional u32 values), in place, or written as
 // triples {key >> qbits, key & qmask, val} when trip != null (msd.cu).
 size_t msd_scratch_bytes(uint64_t n);
@@ -118,17 +102,6 @@ cudaError_t msd_sort(uint64_t *keys, uint32_t *vals, uint64_t n, int bits, void 
 // The same with the key count in device memory (n = min(*d_n, cap)); capturable.
 cudaError_t msd_sort_dev(uint64_t *keys, uint32_t *vals, const unsigned long long *d_n, uint64_t cap, int bits,
                          void *scratch, cudaStream_t s, gpumem_triple *trip, uint32_t qbits);
-// Output sort for large key sets: stable LSD passes over the top 16 key bits, then
-// every run of equal 16-bit prefix sorted in shared memory and written as triples
-// (msd.cu). (k1, v1): ping-pong buffers of cap entries. d_n: device count or null.
-size_t hybrid_scratch_bytes();
-cudaError_t hybrid_sort_triples(uint64_t *keys, uint32_t *vals, uint64_t *k1, uint32_t *v1,
-                                const unsigned long long *d_n, uint64_t cap, int bits, void *scratch,
-                                cudaStream_t s, gpumem_triple *trip, uint32_t qbits);
-// keys[i] = (codes[i] << 32) | locs[i] and back (sort.cu)
-cudaError_t launch_join_keys(const uint32_t *codes, const uint32_t *locs, uint64_t n, uint64_t *keys, cudaStream_t s);
-cudaError_t launch_split_keys(const uint64_t *keys, uint64_t n, uint32_t *codes, uint32_t *locs, cudaStream_t s);
-
 // Index (index.cu)
 // sampled locations p = (k0 + k) * step for k in [0, n_locs)
 cudaError_t launch_seed_codes(const uint64_t *R, uint32_t ls, uint32_t step, uint64_t k0, uint64_t n_locs,
@@ -146,14 +119,6 @@ cudaError_t launch_ptrs_fill(const uint32_t *sorted_codes, uint64_t n_locs, uint
 // Dense ptrs[0 .. 4^ls] from the rank directory (rankw or rsect) + compact table (index.cu).
 cudaError_t launch_ptrs_expand(const unsigned long long *rankw, const uint4 *rsect, const uint2 *buckets, uint32_t ls,
                                uint64_t n_locs, uint32_t *ptrs, cudaStream_t s);
-// Fused last step of the index (index.cu): (code, p) pairs sorted stably by code bits
-// [10, 2 ls) -> ptrs, rank directory, compact table, final locs and seed records.
-size_t index_local_scratch_bytes(uint32_t ls);
-size_t index_local_slot_bytes(uint64_t n_locs);
-cudaError_t launch_index_local(const uint32_t *codes, const uint32_t *ps, uint64_t n_locs, uint32_t ls,
-                               const uint64_t *R, uint32_t *ptrs, unsigned long long *rankw, uint4 *rsect,
-                               uint2 *buckets, uint32_t *locs, void *recs, int rec8, uint32_t *slot, void *scratch,
-                               cudaStream_t s);
 // Seed records for the lookup: rec[k] = {locs[k], 16 bases left of it, 32 bases right of its seed}
 // (uint4), or with rec8 {locs[k], 8 bases left | 8 bases right << 16} (uint2).
 cudaError_t launch_seed_recs(const uint64_t *R, uint32_t ls, const uint32_t *locs, uint64_t n_locs, void *recs,

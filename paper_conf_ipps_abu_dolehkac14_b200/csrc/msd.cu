@@ -65,8 +65,7 @@ struct NSpec {
     const unsigned long long *dn;
     uint64_t cap;
     int bits;                                    // significant key bits
-    int fixed_b;                                 // bucket = the top fixed_b bits (hybrid sort), else chosen by n
-    __device__ __forceinline__ int B(uint64_t n) const { return fixed_b ? fixed_b : choose_b(n, bits); }
+    __device__ __forceinline__ int B(uint64_t n) const { return choose_b(n, bits); }
     __device__ __forceinline__ uint64_t n() const {
         if (!dn) return cap;
         const unsigned long long x = *dn;
@@ -529,7 +528,7 @@ static cudaError_t msd_run(uint64_t *keys, uint32_t *vals, NSpec ns, void *scrat
 cudaError_t msd_sort(uint64_t *keys, uint32_t *vals, uint64_t n, int bits, void *scratch, cudaStream_t s,
                      gpumem_triple *trip, uint32_t qbits) {
     if (n == 0) return cudaSuccess;
-    return msd_run(keys, vals, NSpec{nullptr, n, bits < 1 ? 1 : bits, 0}, scratch, s, trip, qbits);
+    return msd_run(keys, vals, NSpec{nullptr, n, bits < 1 ? 1 : bits}, scratch, s, trip, qbits);
 }
 
 // The same with the key count in device memory: n = min(*d_n, cap); nothing is read on
@@ -537,70 +536,7 @@ cudaError_t msd_sort(uint64_t *keys, uint32_t *vals, uint64_t n, int bits, void 
 cudaError_t msd_sort_dev(uint64_t *keys, uint32_t *vals, const unsigned long long *d_n, uint64_t cap, int bits,
                          void *scratch, cudaStream_t s, gpumem_triple *trip, uint32_t qbits) {
     if (cap == 0) return cudaSuccess;
-    return msd_run(keys, vals, NSpec{d_n, cap, bits < 1 ? 1 : bits, 0}, scratch, s, trip, qbits);
-}
-
-// offs[b] = the first slot whose key prefix (key >> shift) is >= b, b in [0, nb] (keys
-// already ordered by that prefix): one binary search per bucket.
-__global__ void __launch_bounds__(256) k_prefix_bounds(const uint64_t *__restrict__ keys, NSpec ns, int shift,
-                                                       uint32_t nb, uint32_t *__restrict__ offs) {
-    pdl_wait();
-    const uint64_t n = ns.n();
-    for (uint32_t b = blockIdx.x * 256 + threadIdx.x; b <= nb; b += gridDim.x * 256) {
-        uint64_t lo = 0, hi = n;
-        while (lo < hi) {
-            const uint64_t mid = (lo + hi) >> 1;
-            if ((keys[mid] >> shift) < b) lo = mid + 1; else hi = mid;
-        }
-        offs[b] = uint32_t(lo);
-    }
-}
-
-size_t hybrid_scratch_bytes() { return radix_scratch_bytes(0) + (1u << 16) * 8 + 4096; }
-
-// Hybrid sort for large outputs: two stable LSD passes (8-bit
-// digits, radix.cu: coalesced tile-reordered scatter) order the keys by their top 16
-// bits; each run of equal prefix (65536 buckets, ~200 keys each at 1.3e7 MEMs) is then
-// a contiguous segment sorted in shared memory by k_bs_local and written as triples.
-// Three passes over the data instead of the LSD sort's seven, and no 16K-way scatter.
-cudaError_t hybrid_sort_triples(uint64_t *keys, uint32_t *vals, uint64_t *k1, uint32_t *v1,
-                                const unsigned long long *d_n, uint64_t cap, int bits, void *scratch,
-                                cudaStream_t s, gpumem_triple *trip, uint32_t qbits) {
-    if (cap == 0) return cudaSuccess;
-    if (bits < 1) bits = 1;
-    const int T = bits < 16 ? bits : 16;
-    const int lo = bits - T;
-    const uint32_t nb = 1u << T;
-    auto align = [](uintptr_t p) { return (p + 255) & ~uintptr_t(255); };
-    uintptr_t c = align(reinterpret_cast<uintptr_t>(scratch));
-    void *rscratch = reinterpret_cast<void *>(c);
-    c = align(c + radix_scratch_bytes(0));
-    uint32_t *offs = reinterpret_cast<uint32_t *>(c);
-    c = align(c + (nb + 1) * 4);
-    uint32_t *big = reinterpret_cast<uint32_t *>(c);
-    c = align(c + nb * 4);
-    unsigned int *n_big = reinterpret_cast<unsigned int *>(c);
-    bool alt = false;
-    cudaError_t e = radix_sort_u64(keys, vals, k1, v1, cap, bits, rscratch, s, &alt, lo, d_n);
-    if (e != cudaSuccess) return e;
-    uint64_t *tk = alt ? k1 : keys, *xk = alt ? keys : k1;
-    uint32_t *tv = alt ? v1 : vals, *xv = alt ? vals : v1;
-    const NSpec ns{d_n, cap, bits, T};
-    e = cudaMemsetAsync(n_big, 0, 4, s);
-    if (e != cudaSuccess) return e;
-    static bool attr = false;
-    if (!attr) {
-        cudaFuncSetAttribute(k_bs_local, cudaFuncAttributeMaxDynamicSharedMemorySize, int(sizeof(LocalSmem)));
-        attr = true;
-    }
-    pdl_launch(k_prefix_bounds, (nb + 256) / 256, 256, 0, s, tk, ns, lo, nb, offs);
-    uint64_t segs = (cap + kSeg - 1) / kSeg;
-    if (segs > uint64_t(kLocalCtas * num_sms())) segs = kLocalCtas * num_sms();  // blocks loop over the segments
-    Out out{keys, vals, trip, qbits};
-    pdl_launch(k_bs_local, unsigned(segs), kLT, sizeof(LocalSmem), s, offs, ns, tk, tv, out, big, n_big);
-    pdl_launch(k_bs_big, num_sms(), kT, 0, s, offs, big, n_big, tk, tv, xk, xv, ns, out);
-    note_launch(3);
-    return cudaGetLastError();
+    return msd_run(keys, vals, NSpec{d_n, cap, bits < 1 ? 1 : bits}, scratch, s, trip, qbits);
 }
 
 }  // namespace gm

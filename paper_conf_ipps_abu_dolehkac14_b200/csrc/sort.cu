@@ -39,38 +39,7 @@ __global__ void __launch_bounds__(kT) k_triples_to_keys(const gpumem_triple *__r
     lens[i] = t.len;
 }
 
-__global__ void __launch_bounds__(kT) k_join(const uint32_t *__restrict__ codes, const uint32_t *__restrict__ locs,
-                                             uint64_t n, uint64_t *__restrict__ keys) {
-    pdl_wait();
-    const uint64_t i = uint64_t(blockIdx.x) * kT + threadIdx.x;
-    if (i < n) keys[i] = (uint64_t(codes[i]) << 32) | locs[i];
-}
-
-__global__ void __launch_bounds__(kT) k_split(const uint64_t *__restrict__ keys, uint64_t n,
-                                              uint32_t *__restrict__ codes, uint32_t *__restrict__ locs) {
-    pdl_wait();
-    const uint64_t i = uint64_t(blockIdx.x) * kT + threadIdx.x;
-    if (i >= n) return;
-    const uint64_t k = keys[i];
-    codes[i] = uint32_t(k >> 32);
-    locs[i] = uint32_t(k);
-}
-
 }  // namespace
-
-cudaError_t launch_join_keys(const uint32_t *codes, const uint32_t *locs, uint64_t n, uint64_t *keys, cudaStream_t s) {
-    if (!n) return cudaSuccess;
-    pdl_launch(k_join, unsigned((n + kT - 1) / kT), kT, 0, s, codes, locs, n, keys);
-    note_launch();
-    return cudaGetLastError();
-}
-
-cudaError_t launch_split_keys(const uint64_t *keys, uint64_t n, uint32_t *codes, uint32_t *locs, cudaStream_t s) {
-    if (!n) return cudaSuccess;
-    pdl_launch(k_split, unsigned((n + kT - 1) / kT), kT, 0, s, keys, n, codes, locs);
-    note_launch();
-    return cudaGetLastError();
-}
 
 cudaError_t launch_keys_to_triples(const uint64_t *keys, const uint32_t *lens, uint64_t n, uint32_t qbits,
                                    gpumem_triple *out, cudaStream_t s, const unsigned long long *dn) {

@@ -23,8 +23,8 @@ from paper_conf_ipps_abu_dolehkac14_b200 import gpumem  # noqa: E402
 def _default_options():
     yield
     for k, v in (("find_grid", 0), ("find_spill", 64), ("out_capacity", 0), ("use_bitmap", 1), ("static_lb", 0),
-                 ("sort_impl", 0), ("index_msd", 0), ("small_sort", 0), ("radix_bits", 0),
-                 ("rank_sectors", -1), ("rec8", -1), ("index_fused", 0), ("pdl", 1), ("index_alg1", 0)):
+                 ("sort_impl", 0), ("radix_bits", 0),
+                 ("rank_sectors", -1), ("rec8", -1), ("pdl", 1), ("index_alg1", 0)):
         gpumem.set_option(k, v)
 
 
@@ -143,12 +143,12 @@ def test_index_hot_seed_chunks():
                 assert np.array_equal(p, op) and np.array_equal(l, ol), (ls, step, sect, alg1)
 
 
-@pytest.mark.parametrize("opts", [{"small_sort": 1}, {"radix_bits": 8}, {"index_msd": 1}, {"index_fused": 1},
+@pytest.mark.parametrize("opts", [{"radix_bits": 8}, {"radix_bits": 10},
                                   {"index_alg1": 1}, {"index_alg1": 1, "rank_sectors": 1}, {"index_alg1": 0},
-                                  {"index_fused": 1, "rank_sectors": 1, "rec8": 1}])
+                                  {"rank_sectors": 1, "rec8": 1}])
 def test_index_sort_paths(opts):
-    """Every index sort path (single-launch cooperative, multi-launch LSD, MSD) gives
-    Alg. 1's ptrs/locs word for word."""
+    """Every index path (stable LSD radix sort at each digit width, Alg. 1 as written)
+    gives the oracle's Alg. 1 ptrs/locs word for word."""
     P = synth.make_pair("c3", scale=0.05)
     op, ol = oracle.index(P.R.tobytes(), 13, 38)
     for k, v in opts.items():
@@ -196,15 +196,13 @@ def test_homopolymer_closed_form(n, m):
         assert np.array_equal(got, want), (n, m, L, ls)
 
 
-@pytest.mark.parametrize("impl", [0, 1, 2, 3, 4])
+@pytest.mark.parametrize("impl", [0, 1, 2])
 @pytest.mark.parametrize("n,m,L", [(300, 20000, 20), (20000, 300, 20), (9000, 9000, 8000), (2, 50000, 1)])
 def test_sort_skewed_buckets(impl, n, m, L):
     """Output sort on skewed key sets: most MEMs share r = 0 (one MSD bucket far past
     shared memory -> the global LSD fallback) or q = 0 (many small buckets), checked
-    against the homopolymer closed form, under every output sort path (auto, LSD, MSD,
-    hybrid, single-launch)."""
-    gpumem.set_option("sort_impl", impl % 4)
-    gpumem.set_option("small_sort", int(impl == 4))
+    against the homopolymer closed form, under every output sort path (auto, LSD, MSD)."""
+    gpumem.set_option("sort_impl", impl)
     want = np.array(pyoracle.homopolymer(n, m, L), dtype=np.uint32).reshape(-1, 3)
     got = gpu_mems("A" * n, "A" * m, L, 1 if L < 13 else 13)
     assert np.array_equal(got, want), (impl, n, m, L)
@@ -252,15 +250,15 @@ def test_overflow_retry_grid_spill_and_bitmap_invariance():
     base = gpu_mems(P.R, P.Q, P.L, P.ls)
     assert np.array_equal(base, want)
     for opt, vals in (("out_capacity", [1, 100]), ("find_grid", [1, 3, 148]), ("find_spill", [1, 2, 10**9]),
-                      ("use_bitmap", [0]), ("static_lb", [1]), ("sort_impl", [1, 2, 3]), ("index_msd", [1]), ("small_sort", [1]),
-                      ("rank_sectors", [0, 1]), ("rec8", [0, 1]), ("index_fused", [1]),
+                      ("use_bitmap", [0]), ("static_lb", [1]), ("sort_impl", [1, 2]),
+                      ("rank_sectors", [0, 1]), ("rec8", [0, 1]),
                       ("radix_bits", [8, 9, 10]), ("pdl", [0]), ("index_alg1", [1, -1])):
         for v in vals:
             gpumem.set_option(opt, v)
             assert np.array_equal(gpu_mems(P.R, P.Q, P.L, P.ls), want), (opt, v)
         gpumem.set_option(opt, {"out_capacity": 0, "find_grid": 0, "find_spill": 64, "use_bitmap": 1,
-                                "static_lb": 0, "sort_impl": 0, "index_msd": 0, "small_sort": 0, "rank_sectors": -1,
-                                "rec8": -1, "index_fused": 0,
+                                "static_lb": 0, "sort_impl": 0, "rank_sectors": -1,
+                                "rec8": -1,
                                 "radix_bits": 0, "pdl": 1, "index_alg1": 0}[opt])
 
 
