@@ -53,6 +53,7 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=5)
+    ap.add_argument("--no-d9", action="store_true")
     return ap.parse_args()
 
 
@@ -134,7 +135,8 @@ def run_reference(args, P):
     v = q_end / 1e6 / t
     desc = (f"full hash index of R ({len(P.R)} bp) + lookup/extension/sort-unique of MEMs starting in "
             f"Q[0:{q_end}] ({q_end / len(P.Q):.1%} of Q)")
-    line = {"impl": "reference", "metric": METRIC, "value": round(v, 3), "unit": "Mbp/s", "n_gpus": args.gpus,
+    line = {"impl": "reference", "metric": METRIC, "value": round(v, 3), "unit": "Mbp/s",
+            "n_gpus": int(os.environ.get("WORLD_SIZE", "1")),
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(t * 1e3, 3),
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u8 (ASCII chars)",
             "data": "synthetic", "config": {"workload": WORKLOAD_DESC[args.config], "sample": desc},
@@ -145,37 +147,96 @@ def run_reference(args, P):
 
 
 # ------------------------------------------------------------------ roofline bookkeeping
-def algorithmic_bytes(nR, nQ, ls, L, stats, world):
-    """Algorithmic (useful) HBM bytes per step of each stage on one rank:
-    what the method must move, not sector over-fetch."""
+def radix_passes(key_bits, n):
+    """LSD passes the library's radix sort runs (radix.cu pick_digit_bits): 8-bit digits
+    above 16 M keys, else 9-bit digits when that saves a pass, else 8-bit."""
+    if n > (16 << 20):
+        return (key_bits + 7) // 8
+    return min((key_bits + 8) // 9, (key_bits + 7) // 8)
+
+
+def d7_bytes(nR, nQ, ls, L, stats, mean_len):
+    """SURVEY.md §8(d) D7's algorithmic bytes per step of each stage (what the method
+    itself must move): pack 1.25 B per base; find per query position 0.25 B (packed Q)
+    + 8 B (ptrs[s], ptrs[s+1]), per hit 4 B (locs) + 16 B (R window), per MEM
+    mean_len/2 B (extension, R + Q) + 12 B (output); sort 12 B x 2 x passes per MEM."""
+    pos, hits, mems = stats["positions"], stats["hits"], stats["mems"]
+    kb = (max(nR, 1) - 1).bit_length() + (max(nQ, 1) - 1).bit_length()
+    return {"pack": 1.25 * (nR + nQ),
+            "find": (0.25 + 8) * pos + 20 * hits + (mean_len / 2 + 12) * mems,
+            "sort": 24 * radix_passes(kb, mems) * mems}
+
+
+def impl_bytes(nR, nQ, ls, L, stats):
+    """Bytes this implementation's data structures must move per step,
+    stage by stage; the find row is narrower than D7's (an occupancy bit and an 8-byte
+    {first, count} entry per occupied seed instead of two ptrs reads per position; one
+    seed record per hit instead of locs + an R window)."""
     step = L - ls + 1
     n_locs = (nR - ls) // step + 1 if nR >= ls else 0
     nb = 1 << (2 * ls)
-    passes = (2 * ls + 8) // 9                # LSD passes of 9-bit digits over the 2*ls-bit codes
+    passes = radix_passes(2 * ls, n_locs)
     rec = 8 if step <= 8 else 16              # seed record bytes (index.cu)
     pos, occ, hits, mems = stats["positions"], stats["occupied"], stats["hits"], stats["mems"]
+    sect = n_locs * 8 > (126 << 20) // 4      # rank sectors (16 B / 32 seeds) vs rank words (8 B)
+    cap = pos // 8 + 4096                     # output capacity the pipeline sizes its sort for
+    kb = (max(nR, 1) - 1).bit_length() + (max(nQ, 1) - 1).bit_length()
+    sort = (mems * 56 if mems <= (2 << 20)    # MSD: histogram 8, scatter 24, local sort + triples 24
+            else radix_passes(kb, cap) * mems * 32 + mems * 24)  # LSD: (8 + 4) x 2 + 8 per pass + triples
     return {
-        # 1 B ASCII read + 0.25 B packed write per base, R and Q
         "pack": 1.25 * (nR + nQ),
-        # per sampled seed: one 8-byte R window read, code + location written
         "index.codes": n_locs * (8 + 8),
-        # stable counting sort by seed code: per digit pass the (code, location) pair is
-        # read and written once, plus one code read for the chunk histogram
         "index.sort": passes * n_locs * (16 + 4),
-        # sorted codes read once; the rank directory (8 B per 32 seeds, 16 B for rank
-        # sectors) and the compact {first, count} table (8 B per occupied seed) written
-        # (the dense ptrs are not built on the hot path)
-        "index.ptrs": n_locs * 4 + (nb / 2 if n_locs * 8 > (126 << 20) // 4 else nb / 4) + 8 * min(n_locs, nb),
-        # per slot: location read, 3 words of R read, the seed record written
+        "index.ptrs": n_locs * 4 + (nb / 2 if sect else nb / 4) + 8 * min(n_locs, nb),
         "index.recs": n_locs * (4 + 24 + rec),
-        # per query position: packed Q (0.25 B) + its occupancy bit (1/8 B); per occupied
-        # position the {first, count} entry (8 B); per hit one seed record; per MEM the
-        # 12-byte (key, len) record written
         "find": 0.25 * pos + pos / 8 + 8 * occ + rec * hits + 12 * mems,
-        # output MSD sort: key read (histogram), key + len read and written (scatter),
-        # read again and written as a triple (local sort): 8 + 24 + 24 B per MEM
-        "sort": mems * 56,
+        "sort": sort,
     }
+
+
+# ------------------------------------------------------------------ D9 generator diagnostics
+def d9_diagnostics(P, dev):
+    """input SHA-256s, the Fig. 6 analogue (how many
+    seeds have k = 1, 2, 3, ... sampled locations, and the largest bucket) and the
+    distribution of hits per query position -- from the library's own index (the
+    paper's dense ptrs, expanded on demand), outside the timed region."""
+    import torch
+    from paper_conf_ipps_abu_dolehkac14_b200 import gpumem as gm
+    shaR, shaQ = P.sha256()
+    Rs = gm.pack(torch.from_numpy(P.R).to(dev))
+    idx = gm.index_build(Rs, P.ls, P.L)
+    ptrs, locs = idx.view()
+    n_locs = locs.numel()
+    cnt = (ptrs[1:].to(torch.int64) - ptrs[:-1].to(torch.int64))
+    edges = [1, 2, 3, 4, 5, 8, 16, 32, 64, 128, 256, 1024, 4096]
+    occupied = cnt[cnt > 0]
+    fig6 = {"seeds_with_k_locs": {}, "occupied_seeds": int(occupied.numel()),
+            "largest_bucket": int(occupied.max().item()) if occupied.numel() else 0}
+    for a, b in zip(edges, edges[1:] + [None]):
+        m = (occupied >= a) if b is None else ((occupied >= a) & (occupied < b))
+        fig6["seeds_with_k_locs"][f"{a}+" if b is None else (str(a) if b == a + 1 else f"{a}-{b - 1}")] = \
+            int(m.sum().item())
+    # hits per query position = the bucket size of the position's seed (first base most significant)
+    q = torch.from_numpy(P.Q).to(dev)
+    c = ((q >> 1) ^ (q >> 2)) & 3  # A0 C1 G2 T3 (both cases)
+    n = q.numel() - P.ls + 1
+    hist = {}
+    if n > 0:
+        code = torch.zeros(n, dtype=torch.int64, device=dev)
+        for i in range(P.ls):
+            code = (code << 2) | c[i:i + n].to(torch.int64)
+        h = cnt[code]
+        for a, b in ((0, 1), (1, 2), (2, 4), (4, 16), (16, 64), (64, 256), (256, 1024), (1024, None)):
+            m = (h >= a) if b is None else ((h >= a) & (h < b))
+            hist[f"{a}+" if b is None else (str(a) if b == a + 1 else f"{a}-{b - 1}")] = int(m.sum().item())
+        hist["mean"] = round(float(h.double().mean().item()), 4)
+        hist["max"] = int(h.max().item())
+        del code, h
+    del cnt, occupied, ptrs, locs
+    idx.free()
+    Rs.free()
+    return {"sha256_R": shaR, "sha256_Q": shaQ, "n_locs": int(n_locs), "fig6_bucket_sizes": fig6,
+            "hits_per_position": hist}
 
 
 # ------------------------------------------------------------------ our arm
@@ -244,7 +305,8 @@ def run_ours(args, P):
                 prof[k] = (a0[0] + t, a0[1] + nl)
         torch.cuda.synchronize()
     launches = gm.launch_count() - l0
-    gpu_result = sp.pl.numpy() if world == 1 else None  # the last timed step's MEMs
+    # the last timed step's MEMs (rank 0's merged set for N > 1)
+    gpu_result = sp.pl.numpy() if world == 1 else (sp.merged.numpy() if rank == 0 else None)
     if world > 1:
         dist.barrier()
     step_ms = [a.elapsed_time(b) for a, b in ev]
@@ -285,11 +347,16 @@ def run_ours(args, P):
     peak_src = "measured" if "hbm_gbs" in peaks else "fallback"
     nQ, nR, ls, L = len(P.Q), len(P.R), P.ls, P.L
     step_ = L - ls + 1
-    alg = algorithmic_bytes(nR, nQ, ls, L, stats, world)
+    mean_len = float(gpu_result[:, 2].astype(np.float64).mean()) if gpu_result is not None and len(gpu_result) else \
+        float(L)
+    d7 = d7_bytes(nR, nQ, ls, L, stats, mean_len)
+    alg = impl_bytes(nR, nQ, ls, L, stats)
     roof = None
-    if dom in alg:
+    if dom in d7:
         n_launch = prof[dom][1] / args.steps
-        achieved = alg[dom] / (kernel_ms[dom] / 1e3) / 1e9
+        sec = kernel_ms[dom] / 1e3
+        achieved = d7[dom] / sec / 1e9
+        achieved_impl = alg[dom] / sec / 1e9
         traffic, sectors = None, None
         try:  # dram read+write bytes of that kernel from the committed ncu --set full capture
             t = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json"))).get(args.config)
@@ -300,8 +367,17 @@ def run_ours(args, P):
             pass
         roof = {"bound": "hbm", "kernel": dom, "achieved": round(achieved, 1), "peak": peak,
                 "peak_source": peak_src, "unit": "GB/s", "frac": round(achieved / peak, 4), "traffic": traffic,
-                "algorithmic_bytes_per_step": int(alg[dom]), "launches_per_step": n_launch,
-                "ms_per_step": round(kernel_ms[dom], 4)}
+                "bytes_model": "SURVEY.md §8(d) D7: 8.25 B per query position + 20 B per hit + "
+                               "(mean_len/2 + 12) B per MEM",
+                "algorithmic_bytes_per_step": int(d7[dom]), "mean_mem_len": round(mean_len, 2),
+                "frac_d7": round(achieved / peak, 4),
+                "impl_bytes_per_step": int(alg[dom]), "achieved_impl": round(achieved_impl, 1),
+                "frac_impl": round(achieved_impl / peak, 4),
+                "impl_bytes_model": "DESIGN.md §7: this build's structures (occupancy bit per position, "
+                                    "8 B entry per occupied seed, one seed record per hit, 12 B per MEM)",
+                "launches_per_step": n_launch, "ms_per_step": round(kernel_ms[dom], 4)}
+        if traffic:
+            roof["traffic_over_d7"] = round(traffic / d7[dom], 3)
         if sectors:  # what bounds k_find: 32-byte sector requests L1 -> L2, ceiling
             # ~1 sector per SM clock; ncu's sector count over the live kernel time and SM clock
             clk_mhz = (clk.summary().get("sm_mhz") or 1965.0)
@@ -325,6 +401,7 @@ def run_ours(args, P):
             except Exception as e:  # pragma: no cover
                 roof["gather_ceiling"] = {"error": repr(e)}
     stage_frac = {k: round(alg[k] / (stage_ms_all[k] / 1e3) / 1e9 / peak, 4) for k in alg if k in stage_ms_all}
+    stage_frac_d7 = {k: round(d7[k] / (stage_ms_all[k] / 1e3) / 1e9 / peak, 4) for k in d7 if k in stage_ms_all}
 
     line = {"metric": METRIC, "value": round(value, 2), "unit": "Mbp/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": round(ms, 4), "higher_is_better": True, "scaling": "strong",
@@ -337,7 +414,7 @@ def run_ours(args, P):
             "stage_ms": {k: round(v, 4) for k, v in sorted(stage_ms_all.items())},
             "stage_ms_note": "separate 5-step run with an event node at every stage boundary (not the timed region)",
             "find_ms_live": round(kernel_ms.get("find", 0.0), 4),
-            "stage_hbm_frac": stage_frac, "find_stats": stats, "gpu_launches": int(launches),
+            "stage_hbm_frac": stage_frac, "stage_hbm_frac_d7": stage_frac_d7, "find_stats": stats, "gpu_launches": int(launches),
             "clocks": clk.summary(), "roofline": roof,
             "host_ms_per_step": round(statistics.mean(host_ms), 4), "capacity_fallbacks": fallbacks,
             "launch_mode": "one CUDA graph per step (gpumem_pipeline_run)",
@@ -374,6 +451,13 @@ def run_ours(args, P):
                        "steps": args.e2e_steps,
                        "path": "gpumem_pipeline_run_host (pinned host R, Q) + result + D2H of the triples"}
 
+    # ---- D9 generator diagnostics (input digests, Fig. 6 bucket sizes, hits per position)
+    if rank == 0 and not args.no_d9:
+        try:
+            line["d9"] = d9_diagnostics(P, dev)
+        except Exception as e:  # pragma: no cover
+            line["d9"] = {"error": repr(e)}
+
     # ---- CPU oracle on a bounded sample (rank 0, N = 1 only)
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         dt, q_end, nm_cpu, cores = oracle_sample(P, ORACLE_SAMPLE_BP["ours"])
@@ -400,8 +484,27 @@ def run_ours(args, P):
         dist.destroy_process_group()
 
 
+def relaunch_under_torchrun(args):
+    """`bench.py --gpus N` (N > 1) outside a launcher: run the same command as N ranks,
+    one per GPU, under torch.distributed.run (the driver's own launch), and exit with
+    its status."""
+    import socket
+    import subprocess
+    with socket.socket() as so:
+        so.bind(("127.0.0.1", 0))
+        port = so.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__), *sys.argv[1:]]
+    sys.exit(subprocess.call(cmd))
+
+
 def main():
     args = parse()
+    world = int(os.environ.get("WORLD_SIZE", "0"))
+    if world == 0 and args.gpus > 1:
+        relaunch_under_torchrun(args)
+    if world and world != args.gpus:
+        sys.exit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world} ranks were launched")
     P = synth.make_pair(args.config)
     if args.impl == "reference":
         run_reference(args, P)

@@ -168,9 +168,18 @@ gpumem_status gpumem_mems_view(const gpumem_mems *m, const gpumem_triple **dev_p
 gpumem_status gpumem_mems_to_host(const gpumem_mems *m, gpumem_triple *host_buf, uint64_t capacity);
 
 /*
- * gpumem_merge_sorted -- merge n_runs device arrays of triples, each sorted by (r, q), into
- *  one sorted set (multi-GPU rank-0 merge of query shards; shards are disjoint by the
- *  ownership rule so no duplicates arise). Runs are read, not modified. Synchronises once.
+ * gpumem_merge_sorted -- K9, the rank-0 merge of the query shards (it
+ *  replaces the host merge-sort of out-tile triplets, §III-C2).
+ *  dev_runs[i]: device pointer to counts[i] triples (host array of n_runs <= 64
+ *  pointers / host counts), each run sorted by (r, q) and no (r, q) in two runs (the
+ *  query shards are disjoint by the ownership rule). The runs may be peer memory
+ *  mapped with gpumem_ipc_open: the kernel then reads them over NVLink directly, the
+ *  gather and the merge in one pass. *out: the union sorted by (r, q) (one read and
+ *  one write per triple: bucketed by r, each bucket ranked in shared memory).
+ *  Asynchronous on cuda_stream (the runs must stay valid until it completes).
+ *  Errors: n_runs > 64 or a NULL run with a count -> GPUMEM_ERR_ARG; a run of 2^32 or
+ *  more triples -> GPUMEM_ERR_RANGE. Runs that are unsorted or overlap give an
+ *  unspecified order (not checked).
  */
 gpumem_status gpumem_merge_sorted(const gpumem_triple *const *dev_runs, const uint64_t *counts,
                                   int n_runs, void *cuda_stream, gpumem_mems **out);
@@ -226,6 +235,26 @@ gpumem_status gpumem_pipeline_result(gpumem_pipeline *pl, const gpumem_triple **
 gpumem_status gpumem_pipeline_stats(const gpumem_pipeline *pl, gpumem_find_stats *out);
 int gpumem_pipeline_profile(const gpumem_pipeline *pl, const char **names, double *ms, uint64_t *launches,
                             int max_stages);
+
+/*
+ * Multi-GPU export of a pipeline's result (dist.py's fused gather + merge):
+ * gpumem_pipeline_set_exportable(pl, 1) -- before the first run (or it recaptures):
+ *  the arena is allocated with cudaMalloc (IPC-capable; bypasses the allocator hook).
+ * gpumem_pipeline_export -- after a run: a CUDA IPC handle of the arena, the byte
+ *  offset of the result triples inside it, and the capture generation (a recapture,
+ *  e.g. on new input pointers, moves the arena: re-export; handle may be NULL to read
+ *  only offset and generation). The triples there are the
+ *  graph's result; after an overflow fallback (stats.attempts > 1) they are not.
+ * gpumem_ipc_open / gpumem_ipc_close -- map / unmap another process's exported arena
+ *  on the current device (peer access enabled lazily); dev_base + offset are the
+ *  triples. The exporting pipeline must outlive the mapping.
+ */
+typedef struct { unsigned char bytes[64]; } gpumem_ipc_handle;
+gpumem_status gpumem_pipeline_set_exportable(gpumem_pipeline *pl, int on);
+gpumem_status gpumem_pipeline_export(const gpumem_pipeline *pl, gpumem_ipc_handle *handle, uint64_t *offset,
+                                     uint64_t *generation);
+gpumem_status gpumem_ipc_open(const gpumem_ipc_handle *handle, void **dev_base);
+gpumem_status gpumem_ipc_close(void *dev_base);
 
 /* Release any handle above (seq, index, mems, pipeline). NULL is a no-op. */
 void gpumem_free(void *handle);

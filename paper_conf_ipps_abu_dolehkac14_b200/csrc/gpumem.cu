@@ -99,6 +99,11 @@ struct CapCtx {
     cudaStream_t side = nullptr;          // pipeline: the seed records are built here, next to the
     cudaEvent_t ev_a = nullptr, ev_b = nullptr;  // directory fill on the main stream (fork / join)
     gpumem_mems *mems = nullptr;
+    // The pipeline's own workspaces (never the per-stream global ones, which ordinary
+    // calls and gpumem_trim may grow or free while the graph still points into them):
+    // the measuring run allocates and sizes them (ws_need), the capture bump-allocates
+    // each from the arena at that size, so they live and die with the arena.
+    void *ws_priv = nullptr;              // WsSet *
 };
 thread_local CapCtx *t_cap = nullptr;
 thread_local bool t_ws_alloc = false;     // workspace growth: never from the arena
@@ -289,7 +294,7 @@ gpumem_status check_device(int *dev) {
 // loop does no allocation at all once warm. gpumem_trim() releases everything.
 enum WsSlot {
     kWsCtr, kWsSpill, kWsKeys, kWsLens, kWsSortK, kWsSortL, kWsSortScratch, kWsCodes0, kWsCodes1,
-    kWsRadix, kWsFill, kWsMergeK, kWsMergeL, kWsPackTmp, kWsCoop, kWsMums, kWsAlg1,
+    kWsRadix, kWsFill, kWsMergeK, kWsPackTmp, kWsCoop, kWsMums, kWsAlg1,
     kWsCount
 };
 struct Workspace {
@@ -299,7 +304,50 @@ struct Workspace {
 std::mutex g_ws_mu;
 std::vector<std::pair<std::pair<int, cudaStream_t>, Workspace *>> g_ws;
 
+// A pipeline's private workspaces, per stream of its path.
+struct WsSet {
+    std::vector<std::pair<cudaStream_t, Workspace>> w;
+    Workspace &of(cudaStream_t s) {
+        for (auto &e : w)
+            if (e.first == s) return e.second;
+        w.push_back({s, Workspace{}});
+        return w.back().second;
+    }
+    size_t bytes() const {  // arena bytes the capture will bump-allocate for them
+        size_t t = 0;
+        for (auto &e : w)
+            for (int k = 0; k < kWsCount; ++k) t += (e.second.sz[k] + 255) & ~size_t(255);
+        return t;
+    }
+    void release() {  // measuring run only (capture workspaces are arena memory)
+        for (auto &e : w)
+            for (int k = 0; k < kWsCount; ++k)
+                if (e.second.p[k]) dfree(e.second.p[k], e.first);
+        w.clear();
+    }
+};
+
+void *ws_get_priv(WsSet &set, int slot, size_t bytes, cudaStream_t s) {
+    Workspace &w = set.of(s);
+    if (w.sz[slot] >= bytes && w.p[slot]) return w.p[slot];
+    if (t_cap->mode == 2) {  // one arena slice per workspace, at the measured size
+        if (w.p[slot] || bytes > w.sz[slot]) {
+            fail(GPUMEM_ERR_NOMEM, "workspace %d would grow during a pipeline capture", slot);
+            return nullptr;
+        }
+        w.p[slot] = dalloc(w.sz[slot], s);  // bump allocation from the arena
+        return w.p[slot];
+    }
+    t_ws_alloc = true;  // measuring run: real allocations, not counted as handle bytes
+    if (w.p[slot]) dfree(w.p[slot], s);
+    w.p[slot] = dalloc(bytes, s);
+    w.sz[slot] = w.p[slot] ? bytes : 0;
+    t_ws_alloc = false;
+    return w.p[slot];
+}
+
 void *ws_get(int slot, size_t bytes, cudaStream_t s) {
+    if (t_cap && t_cap->ws_priv) return ws_get_priv(*static_cast<WsSet *>(t_cap->ws_priv), slot, bytes, s);
     int d = 0;
     cudaGetDevice(&d);
     std::lock_guard<std::mutex> g(g_ws_mu);
@@ -311,10 +359,6 @@ void *ws_get(int slot, size_t bytes, cudaStream_t s) {
         g_ws.push_back({{d, s}, w});
     }
     if (w->sz[slot] < bytes) {
-        if (t_cap && t_cap->mode == 2) {  // the measuring run sized every workspace
-            fail(GPUMEM_ERR_NOMEM, "workspace %d would grow during a pipeline capture", slot);
-            return nullptr;
-        }
         t_ws_alloc = true;
         if (w->p[slot]) dfree(w->p[slot], s);
         const size_t want = bytes + bytes / 8 + 4096;
@@ -365,8 +409,9 @@ struct gpumem_pipeline {
     uint64_t nR, nQ, q_begin, q_end;
     uint32_t ls, L;
     const char *inR, *inQ;                 // the device inputs the graph was captured with
-    char *arena;
+    char *arena;                           // every allocation of the captured path (allocator hook)
     size_t arena_bytes;
+    WsSet *ws;                             // the graph's workspaces, slices of the arena
     cudaGraph_t graph;                     // the captured path (one launch per run)
     cudaGraphExec_t exec;
     cudaEvent_t ev_fork;                   // side-stream fork inside the graph
@@ -382,6 +427,8 @@ struct gpumem_pipeline {
     uint64_t out_cap, coop_cap, spill_cap, span;
     std::vector<StageRec> recs;
     uint64_t launches;                     // kernels per graph launch
+    int exportable;                        // arena from cudaMalloc, so its IPC handle can be exported
+    uint64_t generation;                   // captures so far (an exported handle is valid for one)
     int ran;
     gpumem_find_stats stats;
 };
@@ -429,9 +476,14 @@ void pipeline_release(gpumem_pipeline *pl) {  // graph, arena and the arena-back
     pl->R = pl->Q = nullptr;
     pl->idx = nullptr;
     pl->mems = nullptr;
-    if (pl->arena) cudaFree(pl->arena);
+    if (pl->arena) {
+        if (pl->exportable) cudaFree(pl->arena);
+        else dfree(pl->arena, pl->stream);
+    }
     pl->arena = nullptr;
     pl->arena_bytes = 0;
+    delete pl->ws;  // its buffers were arena slices
+    pl->ws = nullptr;
     {
         std::lock_guard<std::mutex> g(g_prof_mu);
         for (auto &r : pl->recs) {
@@ -449,8 +501,10 @@ gpumem_status pipeline_capture(gpumem_pipeline *pl, const char *R, const char *Q
     CK(cudaStreamSynchronize(s), "sync");
     pipeline_release(pl);
     // 1) measuring run: sizes every workspace, sums the handle/scratch bytes
+    WsSet mws;
     CapCtx m;
     m.mode = 1;
+    m.ws_priv = &mws;
     m.deferred = true;
     m.host = pl->host;
     m.side = pl->side2;
@@ -464,14 +518,35 @@ gpumem_status pipeline_capture(gpumem_pipeline *pl, const char *R, const char *Q
     t_cap = nullptr;
     const cudaError_t se = cudaStreamSynchronize(s);
     for (void *h : {(void *)hM, (void *)hI, (void *)hQ, (void *)hR}) gpumem_free(h);
+    pl->ws = new WsSet();  // the capture's workspaces: the measured sizes, no memory yet
+    for (auto &e : mws.w) {
+        Workspace &w = pl->ws->of(e.first);
+        for (int k = 0; k < kWsCount; ++k) w.sz[k] = e.second.sz[k];
+    }
+    mws.release();
     if (st) return st;
     CK(se, "measuring run");
     CK(cudaStreamSynchronize(s), "sync");
-    // 2) capture into the arena
-    pl->arena_bytes = m.need + (1u << 20);
-    CK(cudaMalloc(&pl->arena, pl->arena_bytes), "pipeline arena");
+    // 2) capture into the arena (one allocation, through the allocator hook if set)
+    pl->arena_bytes = m.need + pl->ws->bytes() + (1u << 20);
+    if (pl->exportable) {  // IPC-capable memory (stream-ordered pool memory cannot be exported)
+        if (cudaMalloc(&pl->arena, pl->arena_bytes) != cudaSuccess) {
+            cudaGetLastError();
+            fail(GPUMEM_ERR_NOMEM, "cudaMalloc");
+            pl->arena = nullptr;
+        }
+    } else {
+        pl->arena = static_cast<char *>(dalloc(pl->arena_bytes, s));
+    }
+    if (!pl->arena) {
+        const std::string why = t_err;
+        const size_t want = pl->arena_bytes;
+        pipeline_release(pl);
+        return fail(GPUMEM_ERR_NOMEM, "pipeline arena of %zu bytes: %s", want, why.c_str());
+    }
     CapCtx c;
     c.mode = 2;
+    c.ws_priv = pl->ws;
     c.arena = pl->arena;
     c.cap = pl->arena_bytes;
     c.deferred = true;
@@ -508,6 +583,7 @@ gpumem_status pipeline_capture(gpumem_pipeline *pl, const char *R, const char *Q
     pl->span = c.span;
     pl->inR = R;
     pl->inQ = Q;
+    ++pl->generation;
     return GPUMEM_OK;
 }
 
@@ -661,9 +737,11 @@ void gpumem_free(void *handle) {
         cudaFreeHost(pl->host);
         cudaEventDestroy(pl->ev_in);
         cudaEventDestroy(pl->ev_out);
-        if (pl->stage) {
+        if (pl->copy) {
             cudaStreamSynchronize(pl->copy);
-            cudaFree(pl->stage);
+            if (pl->stage) dfree(pl->stage, pl->copy);
+            cudaStreamSynchronize(pl->copy);
+            ws_release_stream(pl->device, pl->copy);
             cudaStreamDestroy(pl->copy);
         }
         cudaEventDestroy(pl->ev_r);
@@ -672,10 +750,11 @@ void gpumem_free(void *handle) {
         cudaEventDestroy(pl->ev_ra);
         cudaEventDestroy(pl->ev_rb);
         ws_release_stream(pl->device, pl->stream);
-        cudaStreamSynchronize(pl->side);
-        cudaStreamDestroy(pl->side);
-        cudaStreamSynchronize(pl->side2);
-        cudaStreamDestroy(pl->side2);
+        for (cudaStream_t x : {pl->side, pl->side2}) {
+            cudaStreamSynchronize(x);
+            ws_release_stream(pl->device, x);
+            cudaStreamDestroy(x);
+        }
         cudaEventDestroy(pl->ev_join);
         cudaStreamDestroy(pl->stream);
         pl->magic = 0;
@@ -1106,7 +1185,7 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
     int attempts = 0;
     uint64_t *keys = nullptr;
     uint32_t *lens = nullptr;
-    for (int attempt = 0; attempt < 2; ++attempt) {
+    for (int attempt = 0; attempt < 3; ++attempt) {
         keys = static_cast<uint64_t *>(ws_get(kWsKeys, cap * 8, s));
         lens = static_cast<uint32_t *>(ws_get(kWsLens, cap * 4, s));
         if (!keys || !lens) return GPUMEM_ERR_NOMEM;
@@ -1135,10 +1214,13 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
         if (h[9] != ~0ull) return fail(GPUMEM_ERR_ALPHABET, "Q: byte at position %llu is not in {A,C,G,T,a,c,g,t}", h[9]);
         count = h[0];
         if (count <= cap && h[7] <= coop_cap) break;
-        if (attempt == 1) return fail(GPUMEM_ERR_CUDA, "output count changed between runs (%llu > %llu)",
+        if (attempt == 2) return fail(GPUMEM_ERR_CUDA, "output count changed between runs (%llu > %llu)",
                                       (unsigned long long)count, (unsigned long long)cap);
-        if (count > cap) cap = count;            // overflow: rerun with the exact capacity
-        if (h[7] > coop_cap) coop_cap = h[7];    // coop queue overflow: likewise
+        // overflow: rerun with exact capacities. The count of a run whose coop queue
+        // overflowed leaves out the dropped entries' MEMs (each entry yields at most one)
+        const uint64_t dropped = h[7] > coop_cap ? h[7] - coop_cap : 0;
+        if (count + dropped > cap) cap = count + dropped;
+        if (h[7] > coop_cap) coop_cap = h[7];
     }
     gpumem_find_stats fs{};
     fs.positions = span;
@@ -1238,9 +1320,11 @@ gpumem_status gpumem_pipeline_run_host(gpumem_pipeline *pl, const char *r_bases_
         gpumem_free(pl->fallback);
         pl->fallback = nullptr;
     }
-    if (!pl->stage) {
-        CK(cudaMalloc(&pl->stage, pl->nR + pl->nQ + 256), "input staging");
-        CK(cudaStreamCreateWithFlags(&pl->copy, cudaStreamNonBlocking), "copy stream");
+    if (!pl->copy) CK(cudaStreamCreateWithFlags(&pl->copy, cudaStreamNonBlocking), "copy stream");
+    if (!pl->stage) {  // device copies of R and Q (allocator hook if set)
+        pl->stage = static_cast<char *>(dalloc(pl->nR + pl->nQ + 256, pl->copy));
+        if (!pl->stage) return GPUMEM_ERR_NOMEM;
+        CK(cudaStreamSynchronize(pl->copy), "input staging");
     }
     char *dR = pl->stage, *dQ = pl->stage + pl->nR;
     // the copies start after the caller's prior work and after the previous run (which
@@ -1336,6 +1420,53 @@ int gpumem_pipeline_profile(const gpumem_pipeline *pl, const char **names, doubl
     return n;
 }
 
+gpumem_status gpumem_pipeline_set_exportable(gpumem_pipeline *pl, int on) {
+    if (!pl || pl->magic != kMagicPipe) return fail(GPUMEM_ERR_ARG, "not a gpumem_pipeline");
+    if ((on != 0) != (pl->exportable != 0)) {
+        CK(cudaStreamSynchronize(pl->stream), "sync");
+        pipeline_release(pl);  // the next run recaptures into the other kind of arena
+        pl->exportable = on != 0;
+        pl->ran = 0;
+    }
+    return GPUMEM_OK;
+}
+
+gpumem_status gpumem_pipeline_export(const gpumem_pipeline *pl, gpumem_ipc_handle *handle, uint64_t *offset,
+                                     uint64_t *generation) {
+    if (!pl || pl->magic != kMagicPipe) return fail(GPUMEM_ERR_ARG, "not a gpumem_pipeline");
+    if (!offset) return fail(GPUMEM_ERR_ARG, "offset is NULL");
+    if (!pl->exportable) return fail(GPUMEM_ERR_ARG, "pipeline is not exportable (gpumem_pipeline_set_exportable)");
+    if (!pl->exec || !pl->mems) return fail(GPUMEM_ERR_ARG, "pipeline has not run yet");
+    static_assert(sizeof(cudaIpcMemHandle_t) <= sizeof(gpumem_ipc_handle), "IPC handle size");
+    if (handle) {  // NULL: offset and generation only
+        cudaIpcMemHandle_t h;
+        CK(cudaIpcGetMemHandle(&h, pl->arena), "IPC handle");
+        memset(handle, 0, sizeof *handle);
+        memcpy(handle->bytes, &h, sizeof h);
+    }
+    *offset = uint64_t(reinterpret_cast<char *>(pl->mems->dev) - pl->arena);
+    if (generation) *generation = pl->generation;
+    return GPUMEM_OK;
+}
+
+gpumem_status gpumem_ipc_open(const gpumem_ipc_handle *handle, void **dev_base) {
+    if (!handle || !dev_base) return fail(GPUMEM_ERR_ARG, "handle / dev_base is NULL");
+    *dev_base = nullptr;
+    int dev;
+    gpumem_status st = check_device(&dev);
+    if (st) return st;
+    cudaIpcMemHandle_t h;
+    memcpy(&h, handle->bytes, sizeof h);
+    CK(cudaIpcOpenMemHandle(dev_base, h, cudaIpcMemLazyEnablePeerAccess), "IPC open");
+    return GPUMEM_OK;
+}
+
+gpumem_status gpumem_ipc_close(void *dev_base) {
+    if (!dev_base) return GPUMEM_OK;
+    CK(cudaIpcCloseMemHandle(dev_base), "IPC close");
+    return GPUMEM_OK;
+}
+
 gpumem_status gpumem_mums(const gpumem_mems *m, void *cuda_stream, gpumem_mems **out) {
     if (!out) return fail(GPUMEM_ERR_ARG, "out is NULL");
     *out = nullptr;
@@ -1395,22 +1526,25 @@ gpumem_status gpumem_merge_sorted(const gpumem_triple *const *dev_runs, const ui
     gpumem_status st = check_device(&dev);
     if (st) return st;
     cudaStream_t s = static_cast<cudaStream_t>(cuda_stream);
+    if (n_runs > kMergeMaxRuns) return fail(GPUMEM_ERR_ARG, "at most %d runs (got %d)", kMergeMaxRuns, n_runs);
     uint64_t total = 0;
-    for (int i = 0; i < n_runs; ++i) total += counts[i];
-    Scratch sc(s);
-    auto *keys = static_cast<uint64_t *>(ws_get(kWsMergeK, (total ? total : 1) * 8, s));
-    auto *lens = static_cast<uint32_t *>(ws_get(kWsMergeL, (total ? total : 1) * 4, s));
-    if (!keys || !lens) return GPUMEM_ERR_NOMEM;
-    {
-        Stage g("merge", s);
-        uint64_t off = 0;
-        for (int i = 0; i < n_runs; ++i) {
-            if (counts[i] && !dev_runs[i]) return fail(GPUMEM_ERR_ARG, "run %d is NULL", i);
-            CK(launch_triples_to_keys(dev_runs[i], counts[i], 32, keys + off, lens + off, s), "merge keys");
-            off += counts[i];
-        }
+    for (int i = 0; i < n_runs; ++i) {
+        if (counts[i] && !dev_runs[i]) return fail(GPUMEM_ERR_ARG, "run %d is NULL", i);
+        if (counts[i] >= (1ull << 32)) return fail(GPUMEM_ERR_RANGE, "run %d holds 2^32 or more triples", i);
+        total += counts[i];
     }
-    return sort_into_triples(keys, lens, total, 64, 32, dev, s, out);
+    Scratch sc(s);
+    auto *trip = static_cast<gpumem_triple *>(sc.get((total ? total : 1) * sizeof(gpumem_triple)));
+    void *scratch = ws_get(kWsMergeK, merge_scratch_bytes(n_runs > 0 ? n_runs : 1, total), s);
+    if (!trip || !scratch) return GPUMEM_ERR_NOMEM;
+    if (total) {
+        Stage g("merge", s);
+        CK(merge_runs(dev_runs, counts, n_runs, trip, scratch, s), "merge kernel");
+    }
+    sc.keep(trip);
+    *out = new gpumem_mems{kMagicMems, dev, s, total, trip, gpumem_find_stats{}};
+    (*out)->stats.mems = total;
+    return GPUMEM_OK;
 }
 
 }  // extern "C"

@@ -175,6 +175,13 @@ size_t mum_scratch_bytes(uint64_t n);
 cudaError_t mum_filter(const gpumem_triple *in, uint64_t n, gpumem_triple *out, unsigned long long *d_count,
                        void *scratch, cudaStream_t s);
 
+// K9 merge (merge.cu): G <= kMergeMaxRuns runs, each sorted by (r, q), pairwise disjoint
+// -> out (sum of counts triples) sorted by (r, q). The runs may be peer (IPC) memory.
+constexpr int kMergeMaxRuns = 64;
+size_t merge_scratch_bytes(int n_runs, uint64_t total);
+cudaError_t merge_runs(const gpumem_triple *const *runs, const uint64_t *counts, int n_runs, gpumem_triple *out,
+                       void *scratch, cudaStream_t s);
+
 // Triples (sort.cu)
 cudaError_t launch_keys_to_triples(const uint64_t *keys, const uint32_t *lens, uint64_t n, uint32_t qbits,
                                    gpumem_triple *out, cudaStream_t s, const unsigned long long *dn = nullptr);

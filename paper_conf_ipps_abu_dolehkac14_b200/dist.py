@@ -1,15 +1,26 @@
-"""One process per GPU: query-sharded MEM extraction with a gather to rank 0.
+"""One process per GPU: query-sharded MEM extraction with a gather + merge on rank 0.
 
 Partition: rank g owns the MEMs whose query start q lies in
 [a_g, b_g) = [g*|Q|//G, (g+1)*|Q|//G). Every rank packs R and Q itself and builds
 the (deterministic) index of R locally -- recomputing it is cheaper than
-broadcasting the 4^ls-entry table -- then runs gpumem_find_mems on its own range
-(the library scans query positions up to b_g + step - 2 and keeps only starts in
-[a_g, b_g), so the shards are disjoint and their union is the whole MEM set).
-The only exchange is the final gather: an all_gather of the per-rank counts and
-point-to-point sends of each rank's sorted triples to rank 0 (NCCL over NVLink on
-the GPU box; gloo in the CPU tests), followed by rank 0's merge kernel
-(gpumem_merge_sorted). No collective touches the data path before that.
+broadcasting the index -- then finds the MEMs of its own range (the library scans
+query positions up to b_g + step - 2 and keeps only starts in [a_g, b_g), so the
+shards are disjoint and their union is the whole MEM set). The only exchange is the
+final gather to rank 0 and its merge (K9, gpumem_merge_sorted), which replaces the
+paper's host merge-sort of out-tile triplets (§III-C2).
+
+Two gathers:
+ * ShardedPipeline (what bench.py times): every rank's result stays in its own HBM,
+   in an IPC-exportable pipeline arena. Rank 0 maps the peers' arenas once
+   (cudaIpcOpenMemHandle over NVLink/NVSwitch) and its merge kernel reads the peers'
+   sorted runs directly -- gather and merge are one kernel, each triple crossing
+   NVLink once. Per step the process group carries only 24 bytes per rank (count,
+   "result is in the exported buffer", capture generation) and one barrier that
+   keeps the peers from overwriting their results before rank 0 has merged them.
+   A rank whose graph overflowed (result recomputed elsewhere) sends its triples
+   point-to-point instead.
+ * gather_to_root (direct calls, find_mems_sharded): count all_gather + point-to-point
+   sends of each rank's triples to rank 0 (NCCL send/recv on the GPU box).
 """
 from __future__ import annotations
 
@@ -22,16 +33,20 @@ def shard_range(n_q: int, rank: int, world: int):
     return (n_q * rank) // world, (n_q * (rank + 1)) // world
 
 
-def gather_to_root(local: torch.Tensor, group=None):
-    """Gather variable-length (N_g, 3) int32 tensors to rank 0.
+def _ctrl_device(group=None):
+    """Device of the small control tensors: the process group's (NCCL moves device
+    tensors, gloo -- the CPU tests -- host tensors)."""
+    return torch.device("cuda", torch.cuda.current_device()) if dist.get_backend(group) == "nccl" \
+        else torch.device("cpu")
 
-    Returns the list of per-rank tensors on rank 0 (rank order) and None elsewhere.
-    Works with any backend that has all_gather/send/recv (NCCL, gloo)."""
+
+def gather_to_root(local: torch.Tensor, group=None):
+    """Gather variable-length (N_g, 3) int32 tensors to rank 0 (all_gather of the counts,
+    then point-to-point sends). Returns the list of per-rank tensors on rank 0 (rank
+    order) and None elsewhere. `local` lives where the group's backend moves data
+    (CUDA tensors for NCCL)."""
     world = dist.get_world_size(group)
     rank = dist.get_rank(group)
-    if local.is_cuda and dist.get_backend(group) == "gloo":  # gloo moves host tensors only
-        runs = gather_to_root(local.cpu(), group)
-        return None if runs is None else [r.to(local.device) for r in runs]
     dev = local.device
     cnt = torch.tensor([local.shape[0]], dtype=torch.int64, device=dev)
     counts = [torch.zeros_like(cnt) for _ in range(world)]
@@ -50,10 +65,11 @@ def gather_to_root(local: torch.Tensor, group=None):
     return None
 
 
-def find_mems_sharded(R_dev: torch.Tensor, Q_dev: torch.Tensor, min_len: int, seed_len: int, group=None):
-    """Whole multi-GPU step on this rank: pack, index, find own shard, gather,
-    merge on rank 0. Returns the merged gpumem.Mems on rank 0, None elsewhere.
-    Also returns the local (unmerged) Mems so callers can keep it alive."""
+def find_mems_sharded(R_dev: torch.Tensor, Q_dev: torch.Tensor, min_len: int, seed_len: int, group=None,
+                      gather=gather_to_root):
+    """Whole multi-GPU step on this rank with direct calls: pack, index, find own shard,
+    gather, merge on rank 0. Returns (merged Mems on rank 0 / None elsewhere, the
+    local Mems, kept alive by the caller)."""
     from . import gpumem as gm
     world = dist.get_world_size(group) if dist.is_initialized() else 1
     rank = dist.get_rank(group) if dist.is_initialized() else 0
@@ -64,7 +80,7 @@ def find_mems_sharded(R_dev: torch.Tensor, Q_dev: torch.Tensor, min_len: int, se
     local = gm.find_mems(idx, Q, (a, b))
     if world == 1:
         return local, local
-    runs = gather_to_root(local.view_u32().view(torch.int32), group)
+    runs = gather(local.view_u32().view(torch.int32), group)
     if rank == 0:
         return gm.merge_sorted(runs), local
     return None, local
@@ -73,8 +89,8 @@ def find_mems_sharded(R_dev: torch.Tensor, Q_dev: torch.Tensor, min_len: int, se
 class ShardedPipeline:
     """This rank's share of the whole step as a CUDA-graph pipeline (gpumem_pipeline_*):
     pack, index, find over the rank's MEM-start range [a_g, b_g) and the output sort in
-    one graph launch; `finish` checks the result and, for world > 1, gathers the sorted
-    runs to rank 0 and merges them there (the only exchange, as in find_mems_sharded)."""
+    one graph launch; `finish` checks the result and, for world > 1, runs the fused
+    gather + merge on rank 0 (module docstring)."""
 
     def __init__(self, n_r: int, n_q: int, min_len: int, seed_len: int, group=None):
         from . import gpumem as gm
@@ -84,7 +100,13 @@ class ShardedPipeline:
         self.rank = dist.get_rank(group) if dist.is_initialized() else 0
         self.q_range = shard_range(n_q, self.rank, self.world)
         self.pl = gm.Pipeline(n_r, n_q, seed_len, min_len, self.q_range)
+        if self.world > 1:
+            self.pl.set_exportable(True)
         self.merged = None
+        self.peer_gen = [None] * self.world   # capture generation of each peer's mapping
+        self.peer_ptr = [None] * self.world   # rank 0: device address of each peer's result
+        self.peer_base = [None] * self.world
+        self.p2p_ranks = 0                    # ranks that sent point-to-point in the last step
 
     def run(self, R_dev: torch.Tensor, Q_dev: torch.Tensor):
         """Async: one graph launch on the current stream's pipeline."""
@@ -93,20 +115,73 @@ class ShardedPipeline:
             self.merged = None
         self.pl.run(R_dev, Q_dev)
 
+    def _remap(self):
+        """(Re)exchange the IPC handles of every rank whose capture generation changed
+        (first step, or a recapture on new input pointers)."""
+        handle, off, gen = self.pl.export()
+        objs = [None] * self.world
+        dist.all_gather_object(objs, (handle, off, gen), group=self.group)
+        for g in range(1, self.world):
+            if self.rank == 0 and self.peer_base[g] is not None:
+                self.gm.ipc_close(self.peer_base[g])
+                self.peer_base[g] = self.peer_ptr[g] = None
+            h, o, gg = objs[g]
+            if self.rank == 0:
+                self.peer_base[g] = self.gm.ipc_open(h)
+                self.peer_ptr[g] = self.peer_base[g] + o
+            self.peer_gen[g] = gg
+        self.peer_gen[0] = gen
+
     def finish(self):
-        """Synchronise, check (alphabet, capacity fallback), gather + merge for world > 1.
-        Returns the number of MEMs on rank 0 (this rank's count when world == 1), None
-        on other ranks."""
+        """Synchronise, check (alphabet, capacity fallback); for world > 1 gather + merge
+        on rank 0. Returns the number of MEMs on rank 0 (this rank's count when
+        world == 1), None on other ranks."""
         n = self.pl.result()
         if self.world == 1:
             return n
-        runs = gather_to_root(self.pl.view_u32().view(torch.int32), self.group)
+        exported = self.pl.stats()["attempts"] == 1  # the result is the graph's, in the arena
+        gen = self.pl.export(handle=False)[2]
+        dev = _ctrl_device(self.group)
+        meta = torch.tensor([n, int(exported), gen], dtype=torch.int64, device=dev)
+        metas = [torch.empty_like(meta) for _ in range(self.world)]
+        dist.all_gather(metas, meta, group=self.group)
+        metas = torch.stack(metas).tolist()
+        if any(metas[g][2] != self.peer_gen[g] for g in range(self.world)):
+            self._remap()
+        p2p = [g for g in range(1, self.world) if not metas[g][1] and metas[g][0]]
+        self.p2p_ranks = len(p2p)
+        out = None
         if self.rank == 0:
-            self.merged = self.gm.merge_sorted(runs)
-            return len(self.merged)
-        return None
+            ptrs, counts, keep = [], [], []
+            ptrs.append(self.pl._ptr)
+            counts.append(n)
+            for g in range(1, self.world):
+                cnt = metas[g][0]
+                if g in p2p:  # overflow fallback on that rank: its triples come point-to-point
+                    buf = torch.empty((cnt, 3), dtype=torch.int32, device="cuda")
+                    dist.recv(buf, src=g, group=self.group)
+                    keep.append(buf)
+                    ptrs.append(buf.data_ptr())
+                else:
+                    ptrs.append(self.peer_ptr[g])
+                counts.append(cnt)
+            self.merged = self.gm.merge_runs(ptrs, counts)
+            torch.cuda.current_stream().synchronize()  # the peers' runs have been read
+            out = len(self.merged)
+        elif self.rank in p2p:
+            dist.send(self.pl.view_u32().view(torch.int32).contiguous(), dst=0, group=self.group)
+        # peers keep their results untouched until rank 0 has merged them
+        dist.barrier(group=self.group)
+        return out
 
     def free(self):
         if self.merged is not None:
             self.merged.free()
+            self.merged = None
+        for g in range(1, self.world):
+            if self.peer_base[g] is not None:
+                self.gm.ipc_close(self.peer_base[g])
+                self.peer_base[g] = None
+        if self.world > 1 and dist.is_initialized():
+            dist.barrier(group=self.group)  # no rank frees an arena a peer still maps
         self.pl.free()

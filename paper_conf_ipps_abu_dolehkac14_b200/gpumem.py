@@ -54,6 +54,10 @@ SYMBOLS = {
     "gpumem_pipeline_stats": (ctypes.c_int, [_vp, _vp]),
     "gpumem_pipeline_profile": (ctypes.c_int, [_vp, _P(ctypes.c_char_p), _P(ctypes.c_double), _P(_c_u64),
                                                ctypes.c_int]),
+    "gpumem_pipeline_set_exportable": (ctypes.c_int, [_vp, ctypes.c_int]),
+    "gpumem_pipeline_export": (ctypes.c_int, [_vp, _vp, _P(_c_u64), _P(_c_u64)]),
+    "gpumem_ipc_open": (ctypes.c_int, [_vp, _P(_vp)]),
+    "gpumem_ipc_close": (ctypes.c_int, [_vp]),
     "gpumem_free": (None, [_vp]),
     "gpumem_trim": (ctypes.c_int, []),
     "gpumem_last_error": (ctypes.c_char_p, []),
@@ -269,6 +273,28 @@ def mums(m: Mems, stream=None) -> Mems:
     return Mems(h.value, m)
 
 
+def ipc_open(handle: bytes) -> int:
+    """Map another process's exported pipeline arena; returns its device base address."""
+    h = (ctypes.c_ubyte * 64).from_buffer_copy(handle)
+    base = _vp()
+    _check(_lib.gpumem_ipc_open(ctypes.byref(h), ctypes.byref(base)))
+    return base.value
+
+
+def ipc_close(base: int):
+    _check(_lib.gpumem_ipc_close(_vp(base)))
+
+
+def merge_runs(ptrs, counts, stream=None) -> Mems:
+    """K9 merge of raw device runs (pointers to counts[i] triples, e.g. IPC-mapped peer
+    memory), each sorted by (r, q) and pairwise disjoint."""
+    p = (_vp * max(1, len(ptrs)))(*[_vp(int(x)) for x in ptrs])
+    c = (_c_u64 * max(1, len(ptrs)))(*[int(x) for x in counts])
+    h = _vp()
+    _check(_lib.gpumem_merge_sorted(p, c, len(ptrs), _stream(stream), ctypes.byref(h)))
+    return Mems(h.value)
+
+
 def merge_sorted(runs, stream=None) -> Mems:
     """Merge device runs of triples, each sorted by (r, q). `runs`: list of (N_i, 3) uint32/int32 CUDA tensors."""
     ptrs = (_vp * max(1, len(runs)))(*[_vp(r.data_ptr()) for r in runs])
@@ -345,6 +371,18 @@ class Pipeline(_Handle):
     def numpy(self):
         return self.view_u32().cpu().numpy()
 
+    def set_exportable(self, on=True):
+        """IPC-capable arena (cudaMalloc), so other processes can map the result."""
+        _check(_lib.gpumem_pipeline_set_exportable(self.handle, 1 if on else 0))
+
+    def export(self, handle=True):
+        """(64-byte IPC handle or None, byte offset of the result triples, capture generation)."""
+        h = (ctypes.c_ubyte * 64)()
+        off, gen = _c_u64(), _c_u64()
+        _check(_lib.gpumem_pipeline_export(self.handle, ctypes.byref(h) if handle else None, ctypes.byref(off),
+                                           ctypes.byref(gen)))
+        return (bytes(h) if handle else None), off.value, gen.value
+
     def stats(self):
         s = FindStats()
         _check(_lib.gpumem_pipeline_stats(self.handle, ctypes.byref(s)))
@@ -373,6 +411,42 @@ def profile_read(max_stages=32):
     nl = (_c_u64 * max_stages)()
     n = _lib.gpumem_profile_read(names, ms, nl, max_stages)
     return {names[i].decode(): (ms[i], nl[i]) for i in range(n)}
+
+
+ALLOC_FN = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, ctypes.c_void_p)
+FREE_FN = ctypes.CFUNCTYPE(None, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p)
+_allocator_refs = None  # the ctypes callbacks must outlive their registration
+
+
+def set_allocator(alloc=None, free=None):
+    """Route every device allocation of the library through alloc(bytes, stream) -> ptr
+    (0 = out of memory) and free(ptr, stream) (gpumem_set_allocator); no arguments
+    restores the default stream-ordered pool. Handles allocated under one allocator
+    must be freed under the same one."""
+    global _allocator_refs
+    if (alloc is None) != (free is None):
+        raise ValueError("set both alloc and free, or neither")
+    if alloc is None:
+        _check(_lib.gpumem_set_allocator(None, None, None))
+        _allocator_refs = None
+        return
+    a = ALLOC_FN(lambda n, s, ctx: alloc(int(n), s or 0) or None)
+    f = FREE_FN(lambda ptr, s, ctx: free(ptr or 0, s or 0))
+    _check(_lib.gpumem_set_allocator(ctypes.cast(a, _vp), ctypes.cast(f, _vp), None))
+    _allocator_refs = (a, f)
+
+
+def use_torch_allocator():
+    """Allocate through torch's caching allocator (stream-ordered, on the calling stream)."""
+    import torch
+
+    def alloc(n, s):
+        try:
+            return torch.cuda.caching_allocator_alloc(n, stream=torch.cuda.ExternalStream(s) if s else None)
+        except RuntimeError:  # torch.OutOfMemoryError
+            return 0
+
+    set_allocator(alloc, lambda p, s: torch.cuda.caching_allocator_delete(p))
 
 
 def trim():

@@ -284,6 +284,57 @@ def test_qrange_shards_union_to_whole():
         assert np.array_equal(cat, whole)
 
 
+def _random_runs(rng, n, G, r_max, q_max, skew):
+    """n unique (r, q) keys with a length each, dealt to G runs at random, each run
+    sorted by (r, q) (lexsort), plus the whole set sorted -- the merge's expected output."""
+    if skew == "one_r":  # every key on one r: one bucket far past shared memory
+        r = np.zeros(n, np.uint64)
+        q = rng.choice(q_max, size=n, replace=False).astype(np.uint64)
+    elif skew == "hot":  # half the keys on a handful of r values
+        r = np.where(rng.random(n) < 0.5, rng.integers(0, 4, n), rng.integers(0, r_max, n)).astype(np.uint64)
+        q = rng.integers(0, q_max, n).astype(np.uint64)
+    else:
+        r = rng.integers(0, r_max, n).astype(np.uint64)
+        q = rng.integers(0, q_max, n).astype(np.uint64)
+    keys = np.unique((r << np.uint64(32)) | q)
+    t = np.stack([(keys >> np.uint64(32)).astype(np.uint32), (keys & np.uint64(0xffffffff)).astype(np.uint32),
+                  rng.integers(20, 1000, len(keys)).astype(np.uint32)], axis=1)
+    owner = rng.integers(0, G, len(t))
+    return [t[owner == g] for g in range(G)], t
+
+
+@pytest.mark.parametrize("G", [1, 2, 3, 8, 64])
+@pytest.mark.parametrize("n,skew", [(0, "uniform"), (1, "uniform"), (5000, "uniform"), (2_000_000, "uniform"),
+                                    (300_000, "hot"), (20_000, "one_r")])
+def test_merge_kernel(G, n, skew):
+    """K9 merge (merge.cu): G sorted disjoint runs -> one (r, q)-sorted run, against a
+    plain lexicographic sort of the union; empty runs, tiny runs, 2M triples, a hot-r
+    skew and one bucket far past shared memory (all keys on r = 0)."""
+    rng = np.random.default_rng(1000 * G + n)
+    runs, want = _random_runs(rng, n, G, 250_000_000, 150_000_000, skew)
+    dev = [torch.from_numpy(r.copy()).cuda().view(torch.int32) for r in runs]
+    m = gpumem.merge_sorted(dev)
+    got = m.numpy()
+    m.free()
+    assert got.shape == want.shape and np.array_equal(got, want)
+
+
+def test_merge_of_query_shards():
+    """The merge's real input: per-shard find_mems results (disjoint by the ownership
+    rule, sorted) merged == the whole set == the oracle."""
+    P = synth.make_pair("c3", scale=0.05)
+    want = oracle.mems(P.R, P.Q, P.L, P.ls)
+    for G in (2, 5, 8):
+        cuts = [len(P.Q) * g // G for g in range(G + 1)]
+        R, Q = gpumem.pack(P.R), gpumem.pack(P.Q)
+        idx = gpumem.index_build(R, P.ls, P.L)
+        parts = [gpumem.find_mems(idx, Q, (a, b)) for a, b in zip(cuts[:-1], cuts[1:])]
+        m = gpumem.merge_sorted([p.view_u32().view(torch.int32) for p in parts])
+        assert np.array_equal(m.numpy(), want), G
+        for h in [m, *parts, idx, Q, R]:
+            h.free()
+
+
 def test_swap_symmetry():
     P = synth.make_pair("c1", scale=0.2)
     a = gpu_mems(P.R, P.Q, 20, 10)
