@@ -176,7 +176,7 @@ def test_coop_queue_overflow_recovers(n, L, ls):
     The retry must size the output for the dropped entries too; checked against the
     homopolymer closed form, through direct calls and the pipeline."""
     want = np.array(pyoracle.homopolymer(n, n, L), dtype=np.uint32).reshape(-1, 3)
-    assert len(want) > 150_000
+    assert len(want) > 100_000
     got = gpumem.mems("A" * n, "A" * n, L, ls)
     assert np.array_equal(got, want)
     R = _dev(b"A" * n)
