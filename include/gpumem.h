@@ -161,6 +161,17 @@ gpumem_status gpumem_mems_stats(const gpumem_mems *m, gpumem_find_stats *out);
  */
 gpumem_status gpumem_mums(const gpumem_mems *m, void *cuda_stream, gpumem_mems **out);
 
+/*
+ * gpumem_rare -- maximal rare matches (NEXT-F3; PAPER.md:23 "maximal rare matches", :286
+ *  "unique and rare exact match extraction" as future work): the MEMs of `m` whose
+ *  string occurs (overlapping occurrences counted) at most k times in R and at most k
+ *  times in Q (reading R23), in the same (r, q) order; k = 1 is gpumem_mums.
+ *  1 <= k <= 15, else GPUMEM_ERR_ARG. `m` must be a complete MEM set of (R, Q, L): the
+ *  counts come from the containment of the MEMs' query / reference intervals. New
+ *  handle on *out (NULL on error). Synchronises once (the result size is data-dependent).
+ */
+gpumem_status gpumem_rare(const gpumem_mems *m, uint32_t k, void *cuda_stream, gpumem_mems **out);
+
 /* Borrowed device pointer to the sorted triples and their count. */
 gpumem_status gpumem_mems_view(const gpumem_mems *m, const gpumem_triple **dev_ptr, uint64_t *count);
 
@@ -256,7 +267,46 @@ gpumem_status gpumem_pipeline_export(const gpumem_pipeline *pl, gpumem_ipc_handl
 gpumem_status gpumem_ipc_open(const gpumem_ipc_handle *handle, void **dev_base);
 gpumem_status gpumem_ipc_close(void *dev_base);
 
-/* Release any handle above (seq, index, mems, pipeline). NULL is a no-op. */
+/*
+ * Multi-FASTA input and MUMmer-style output (NEXT-F4; PAPER.md:64 §II-A MUMmer, :226
+ * §IV-B: I/O is outside the paper's timings). Host-side parsing and formatting; the
+ * record-boundary split runs on the GPU.
+ *
+ * gpumem_fasta_parse -- text[0, n): one or more records ">name[ description]\n" + sequence
+ *  lines (whitespace ignored; a leading run of blank lines allowed). The records are
+ *  concatenated with ONE masked separator base between consecutive records, and every
+ *  letter outside {A,C,G,T,a,c,g,t} (N, IUPAC codes) becomes a masked 'A' (DESIGN.md
+ *  reading R24: a masked position matches nothing). Errors: no '>' where a header must
+ *  start -> GPUMEM_ERR_ARG; a non-printable byte -> GPUMEM_ERR_ALPHABET; more than
+ *  2^32-1 bases in total -> GPUMEM_ERR_RANGE. *out: new handle (gpumem_free), NULL on error.
+ * gpumem_fasta_info -- the record count, the concatenated sequence (host, borrowed; pass
+ *  it to gpumem_pack / a pipeline), its length, the number of masked intervals.
+ * gpumem_fasta_record -- record i's name (borrowed) and its [start, start + len) in the
+ *  concatenated sequence.
+ * gpumem_split_masked -- the MEMs of the multi-record problem from the MEMs `m` of the
+ *  concatenated sequences (same L): every MEM cut at the masked positions of R and of Q,
+ *  the pieces of length >= min_len kept, sorted by (r, q) in concatenated coordinates.
+ *  q_reverse = 1 when m was computed against gpumem_revcomp(Q) (Q's masks mirrored).
+ *  Synchronises once. New handle on *out.
+ * gpumem_write_mummer -- writes host triples (concatenated coordinates, from
+ *  gpumem_split_masked: no match may cross a record, else GPUMEM_ERR_ARG) as MUMmer text to
+ *  `path`: per query record in input order "> qname" then "  rname\trpos\tqpos\tlen"
+ *  lines (1-based positions inside the records), ordered by query position, reference
+ *  record, reference position; if rev != NULL also "> qname Reverse" and the reverse-strand
+ *  matches (query positions relative to the reverse complement of the query record).
+ */
+typedef struct gpumem_fasta gpumem_fasta;
+gpumem_status gpumem_fasta_parse(const char *text, uint64_t n, gpumem_fasta **out);
+gpumem_status gpumem_fasta_info(const gpumem_fasta *f, uint64_t *n_records, const char **seq, uint64_t *seq_len,
+                                uint64_t *n_masked);
+gpumem_status gpumem_fasta_record(const gpumem_fasta *f, uint64_t i, const char **name, uint64_t *start,
+                                  uint64_t *len);
+gpumem_status gpumem_split_masked(const gpumem_mems *m, const gpumem_fasta *R, const gpumem_fasta *Q, uint32_t min_len,
+                                  int q_reverse, void *cuda_stream, gpumem_mems **out);
+gpumem_status gpumem_write_mummer(const gpumem_triple *fwd, uint64_t n_fwd, const gpumem_triple *rev, uint64_t n_rev,
+                                  const gpumem_fasta *R, const gpumem_fasta *Q, const char *path);
+
+/* Release any handle above (seq, index, mems, pipeline, fasta). NULL is a no-op. */
 void gpumem_free(void *handle);
 
 /* Temporaries (find buffers, sort and index scratch) live in a grow-only workspace per

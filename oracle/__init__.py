@@ -63,6 +63,10 @@ def _load():
             lib.oracle_mums.argtypes = [ctypes.c_char_p, ctypes.c_uint64, ctypes.c_char_p, ctypes.c_uint64,
                                         ctypes.c_uint32, ctypes.c_uint32, ctypes.c_int, u32pp]
             lib.oracle_mums.restype = ctypes.c_int64
+            lib.oracle_rare.argtypes = [ctypes.c_char_p, ctypes.c_uint64, ctypes.c_char_p, ctypes.c_uint64,
+                                        ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint32, ctypes.c_int,
+                                        ctypes.POINTER(ctypes.POINTER(ctypes.c_uint32))]
+            lib.oracle_rare.restype = ctypes.c_int64
             lib.oracle_free.argtypes = [ctypes.c_void_p]
             lib.oracle_num_threads.argtypes = [ctypes.c_int]
             lib.oracle_num_threads.restype = ctypes.c_int
@@ -129,6 +133,38 @@ def mums(R, Q, L, ls, threads=0):
     out = ctypes.POINTER(ctypes.c_uint32)()
     n = lib.oracle_mums(Rb, len(Rb), Qb, len(Qb), int(L), int(ls), int(threads), ctypes.byref(out))
     return _take(n, out)
+
+
+def rare(R, Q, L, ls, k, threads=0):
+    """Rare MEMs: MEMs whose string occurs at most k times in R and in Q (oracle_rare)."""
+    lib = _load()
+    Rb, Qb = _bytes(R), _bytes(Q)
+    out = ctypes.POINTER(ctypes.c_uint32)()
+    n = lib.oracle_rare(Rb, len(Rb), Qb, len(Qb), int(L), int(ls), int(k), int(threads), ctypes.byref(out))
+    return _take(n, out)
+
+
+def mems_multi(R_text, Q_text, L, ls, threads=0):
+    """MEMs of multi-FASTA inputs (R24): oracle_mems on every pair of ACGT
+    segments (the maximal runs of A/C/G/T letters inside each record), shifted to record
+    coordinates. Sorted (r_record, r_pos, q_record, q_pos, len), 0-based."""
+    from . import pyoracle
+    import re
+
+    def segments(seq):
+        return [(m.start(), m.group()) for m in re.finditer(r"[ACGTacgt]+", seq)]
+
+    out = []
+    R, Q = pyoracle.fasta(R_text), pyoracle.fasta(Q_text)
+    for ri, (_, r) in enumerate(R):
+        for a, rs in segments(r):
+            for qi, (_, q) in enumerate(Q):
+                for b, qs in segments(q):
+                    if len(rs) < L or len(qs) < L:
+                        continue
+                    for t in mems(rs.encode(), qs.encode(), L, min(ls, L), threads=threads).tolist():
+                        out.append((ri, a + t[0], qi, b + t[1], t[2]))
+    return sorted(out)
 
 
 def index(R, ls, step):

@@ -272,3 +272,36 @@ extern "C" int64_t oracle_mums(const char* Rs, uint64_t nR, const char* Qs, uint
     *out = export_triples(keep);
     return *out ? int64_t(keep.size()) : -3;
 }
+
+// Rare MEMs (PAPER.md:23 "maximal rare matches"; :286 "unique and rare exact match
+// extraction", future work; reading R23): the MEMs of oracle_mems whose string
+// occurs at most k times in R and at most k times in Q, occurrences counted by plain
+// substring search (std::string::find from every position, overlapping occurrences).
+// k = 1 is oracle_mums. Pinned by the hand-worked W3 fixture (tests/golden/w3_rare.txt),
+// the homopolymer closed form and the Python twin.
+extern "C" int64_t oracle_rare(const char* Rs, uint64_t nR, const char* Qs, uint64_t nQ, uint32_t L,
+                               uint32_t ls, uint32_t k, int threads, uint32_t** out) {
+    uint32_t* mem = nullptr;
+    *out = nullptr;
+    if (k < 1) return -1;
+    const int64_t n = oracle_mems(Rs, nR, Qs, nQ, L, ls, 0, 0, nQ, threads, &mem);
+    if (n < 0) return n;
+    std::string R, Q;
+    normalise(Rs, nR, R);
+    normalise(Qs, nQ, Q);
+    auto at_most_k = [k](const std::string& T, const std::string& S) {
+        uint32_t c = 0;
+        for (size_t pos = T.find(S); pos != std::string::npos; pos = T.find(S, pos + 1))
+            if (++c > k) return false;
+        return true;
+    };
+    std::vector<Triple> keep;
+    for (int64_t i = 0; i < n; ++i) {
+        const Triple t{mem[3 * i], mem[3 * i + 1], mem[3 * i + 2]};
+        const std::string S = R.substr(t.r, t.len);
+        if (at_most_k(R, S) && at_most_k(Q, S)) keep.push_back(t);
+    }
+    std::free(mem);
+    *out = export_triples(keep);
+    return *out ? int64_t(keep.size()) : -3;
+}

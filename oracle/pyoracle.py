@@ -77,3 +77,50 @@ def mums(R, Q, L):
         return sum(1 for i in range(len(T) - len(S) + 1) if T[i:i + len(S)] == S)
 
     return [t for t in brute(R, Q, L) if count(R, R[t[0]:t[0] + t[2]]) == 1 and count(Q, R[t[0]:t[0] + t[2]]) == 1]
+
+
+def rare(R, Q, L, k):
+    """MEMs (by the definition) whose string occurs at most k times in R and in Q."""
+    R, Q = _s(R), _s(Q)
+
+    def count(T, S):
+        return sum(1 for i in range(len(T) - len(S) + 1) if T[i:i + len(S)] == S)
+
+    return [t for t in brute(R, Q, L) if count(R, R[t[0]:t[0] + t[2]]) <= k and count(Q, R[t[0]:t[0] + t[2]]) <= k]
+
+
+def fasta(text):
+    """Records [(name, sequence)] of a multi-FASTA text (name = first word of the header)."""
+    text = text.decode() if isinstance(text, (bytes, bytearray)) else text
+    out = []
+    for block in text.split(">")[1:]:
+        head, _, body = block.partition("\n")
+        out.append((head.split()[0] if head.split() else "", "".join(body.split())))
+    return out
+
+
+def multi_brute(R_text, Q_text, L):
+    """MEMs of multi-FASTA inputs by the definition (R24): for every pair of
+    records, every diagonal walked base by base; a position matches when both bases are
+    in ACGT (either case) and equal; maximal runs of length >= L. Sorted
+    (r_record, r_pos, q_record, q_pos, len), 0-based positions inside the records."""
+    out = []
+    R, Q = fasta(R_text), fasta(Q_text)
+    for ri, (_, r) in enumerate(R):
+        r = r.upper()
+        for qi, (_, q) in enumerate(Q):
+            q = q.upper()
+            for d in range(-len(q) + 1, len(r)):
+                i, j, run = max(d, 0), max(-d, 0), 0
+                while i < len(r) and j < len(q):
+                    if r[i] == q[j] and r[i] in "ACGT":
+                        run += 1
+                    else:
+                        if run >= L:
+                            out.append((ri, i - run, qi, j - run, run))
+                        run = 0
+                    i += 1
+                    j += 1
+                if run >= L:
+                    out.append((ri, i - run, qi, j - run, run))
+    return sorted(out)

@@ -294,7 +294,7 @@ gpumem_status check_device(int *dev) {
 // loop does no allocation at all once warm. gpumem_trim() releases everything.
 enum WsSlot {
     kWsCtr, kWsSpill, kWsKeys, kWsLens, kWsSortK, kWsSortL, kWsSortScratch, kWsCodes0, kWsCodes1,
-    kWsRadix, kWsFill, kWsMergeK, kWsPackTmp, kWsCoop, kWsMums, kWsAlg1,
+    kWsRadix, kWsFill, kWsMergeK, kWsFasta, kWsPackTmp, kWsCoop, kWsMums, kWsAlg1,
     kWsCount
 };
 struct Workspace {
@@ -759,6 +759,10 @@ void gpumem_free(void *handle) {
         cudaStreamDestroy(pl->stream);
         pl->magic = 0;
         delete pl;
+    } else if (magic == kMagicFasta) {
+        auto *f = static_cast<gpumem_fasta *>(handle);
+        f->magic = 0;
+        delete f;
     } else if (magic == kMagicMems) {
         auto *m = static_cast<gpumem_mems *>(handle);
         cudaSetDevice(m->device);
@@ -1467,28 +1471,84 @@ gpumem_status gpumem_ipc_close(void *dev_base) {
     return GPUMEM_OK;
 }
 
-gpumem_status gpumem_mums(const gpumem_mems *m, void *cuda_stream, gpumem_mems **out) {
+gpumem_status gpumem_rare(const gpumem_mems *m, uint32_t k, void *cuda_stream, gpumem_mems **out) {
     if (!out) return fail(GPUMEM_ERR_ARG, "out is NULL");
     *out = nullptr;
     if (!m || m->magic != kMagicMems) return fail(GPUMEM_ERR_ARG, "not a gpumem_mems");
+    if (k < 1 || k > uint32_t(kRareMaxK)) return fail(GPUMEM_ERR_ARG, "k = %u outside [1, %d]", k, kRareMaxK);
     int dev;
     gpumem_status st = check_device(&dev);
     if (st) return st;
     cudaStream_t s = static_cast<cudaStream_t>(cuda_stream);
-    Stage g("mums", s);
+    Stage g(k == 1 ? "mums" : "rare", s);
     Scratch sc(s);
     auto *res = static_cast<gpumem_triple *>(sc.get((m->count ? m->count : 1) * sizeof(gpumem_triple)));
-    void *scratch = ws_get(kWsMums, mum_scratch_bytes(m->count), s);
+    void *scratch = ws_get(kWsMums, rare_scratch_bytes(m->count), s);
     auto *dcount = static_cast<unsigned long long *>(ws_get(kWsCtr, 64, s));
     unsigned long long *h = pinned_slots();
     if (!res || !scratch || !dcount || !h) return GPUMEM_ERR_NOMEM;
-    CK(mum_filter(m->dev, m->count, res, dcount, scratch, s), "MUM filter");
+    CK(rare_filter(m->dev, m->count, k, res, dcount, scratch, s), "rare filter");
     CK(cudaMemcpyAsync(h, dcount, 8, cudaMemcpyDeviceToHost, s), "D2H count");
     CK(cudaStreamSynchronize(s), "sync");
     sc.keep(res);
     *out = new gpumem_mems{kMagicMems, dev, s, h[0], res, m->stats};
     (*out)->stats.mems = h[0];
     return GPUMEM_OK;
+}
+
+gpumem_status gpumem_mums(const gpumem_mems *m, void *cuda_stream, gpumem_mems **out) {
+    return gpumem_rare(m, 1, cuda_stream, out);
+}
+
+gpumem_status gpumem_split_masked(const gpumem_mems *m, const gpumem_fasta *R, const gpumem_fasta *Q, uint32_t L,
+                                  int q_reverse, void *cuda_stream, gpumem_mems **out) {
+    if (!out) return fail(GPUMEM_ERR_ARG, "out is NULL");
+    *out = nullptr;
+    if (!m || m->magic != kMagicMems) return fail(GPUMEM_ERR_ARG, "not a gpumem_mems");
+    if (!R || R->magic != kMagicFasta || !Q || Q->magic != kMagicFasta)
+        return fail(GPUMEM_ERR_ARG, "R and Q must be gpumem_fasta handles");
+    if (L < 1) return fail(GPUMEM_ERR_ARG, "min_len must be >= 1");
+    int dev;
+    gpumem_status st = check_device(&dev);
+    if (st) return st;
+    cudaStream_t s = static_cast<cudaStream_t>(cuda_stream);
+    Stage g("split", s);
+    const uint64_t n = m->count, nQ = Q->seq.size();
+    std::vector<uint64_t> mq = Q->mask;
+    if (q_reverse) {  // the path ran on the reverse complement of the concatenated query
+        const size_t k = mq.size() / 2;
+        for (size_t j = 0; j < k; ++j) {
+            mq[2 * j] = nQ - Q->mask[2 * (k - 1 - j) + 1];
+            mq[2 * j + 1] = nQ - Q->mask[2 * (k - 1 - j)];
+        }
+    }
+    const size_t mbytes = (R->mask.size() + mq.size() + 2) * 8;
+    auto *dm = static_cast<uint64_t *>(ws_get(kWsFasta, mbytes, s));
+    auto *cnt = static_cast<uint32_t *>(ws_get(kWsMergeK, (n + 1) * 8, s));
+    auto *ctr = static_cast<unsigned long long *>(ws_get(kWsCtr, 64, s));
+    unsigned long long *h = pinned_slots();
+    if (!dm || !cnt || !ctr || !h) return GPUMEM_ERR_NOMEM;
+    uint32_t *off = cnt + (n + 1);
+    if (!R->mask.empty())
+        CK(cudaMemcpyAsync(dm, R->mask.data(), R->mask.size() * 8, cudaMemcpyHostToDevice, s), "H2D masks");
+    if (!mq.empty())
+        CK(cudaMemcpyAsync(dm + R->mask.size(), mq.data(), mq.size() * 8, cudaMemcpyHostToDevice, s), "H2D masks");
+    const uint32_t qbits = bits_for(nQ ? nQ : 1);
+    const uint64_t nmr = R->mask.size() / 2, nmq = mq.size() / 2;
+    CK(split_masked(m->dev, n, dm, nmr, dm + R->mask.size(), nmq, L, qbits, cnt, off, ctr, nullptr, nullptr, s),
+       "split count");
+    CK(cudaMemcpyAsync(h, ctr, 8, cudaMemcpyDeviceToHost, s), "D2H count");
+    CK(cudaStreamSynchronize(s), "sync");
+    const uint64_t total = h[0];
+    auto *keys = static_cast<uint64_t *>(ws_get(kWsKeys, (total ? total : 1) * 8, s));
+    auto *lens = static_cast<uint32_t *>(ws_get(kWsLens, (total ? total : 1) * 4, s));
+    if (!keys || !lens) return GPUMEM_ERR_NOMEM;
+    CK(split_masked(m->dev, n, dm, nmr, dm + R->mask.size(), nmq, L, qbits, cnt, off, ctr, keys, lens, s),
+       "split emit");
+    const uint32_t key_bits = bits_for(R->seq.size() ? R->seq.size() : 1) + qbits;
+    st = sort_into_triples(keys, lens, total, key_bits, qbits, dev, s, out);
+    if (st == GPUMEM_OK) (*out)->stats = m->stats, (*out)->stats.mems = total;
+    return st;
 }
 
 gpumem_status gpumem_mems_view(const gpumem_mems *m, const gpumem_triple **dev_ptr, uint64_t *count) {

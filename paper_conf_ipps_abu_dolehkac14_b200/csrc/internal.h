@@ -2,12 +2,26 @@
 // Not part of the ABI (see include/gpumem.h). No torch types anywhere.
 #pragma once
 #include <cstdint>
+#include <string>
 #include <utility>
+#include <vector>
 #include <cuda_runtime.h>
 
 #include "gpumem.h"
 
+// A parsed multi-FASTA (fasta.cu): records concatenated with one masked separator base,
+// non-ACGT letters masked (read as 'A'); masked positions as sorted half-open intervals.
+struct gpumem_fasta {
+    uint32_t magic;
+    std::string seq;                          // concatenated ASCII (A C G T only)
+    std::vector<std::string> names;
+    std::vector<uint64_t> start, len;         // record i: seq[start[i], start[i] + len[i])
+    std::vector<uint64_t> mask;               // masked intervals [mask[2j], mask[2j+1])
+};
+
 namespace gm {
+
+constexpr uint32_t kMagicFasta = 0x47464153u;
 
 // ---------------------------------------------------------------- runtime
 struct Options {
@@ -169,11 +183,13 @@ int find_default_grid();
 // table_bytes (rounded down to a power of two), 8 independent probes per thread.
 cudaError_t gather_ceiling(uint64_t n_probes, uint64_t table_bytes, cudaStream_t s, float *best_ms);
 
-// MUM filter (variants.cu): the MEMs whose string is unique in R and in Q, order kept;
-// the kept count is written to *d_count (device).
-size_t mum_scratch_bytes(uint64_t n);
-cudaError_t mum_filter(const gpumem_triple *in, uint64_t n, gpumem_triple *out, unsigned long long *d_count,
-                       void *scratch, cudaStream_t s);
+// Rare-MEM filter (variants.cu): the MEMs whose string occurs at most k times in R and
+// at most k times in Q (1 <= k <= kRareMaxK; k = 1: MUMs), order kept; the kept count is
+// written to *d_count (device).
+constexpr int kRareMaxK = 15;
+size_t rare_scratch_bytes(uint64_t n);
+cudaError_t rare_filter(const gpumem_triple *in, uint64_t n, uint32_t k, gpumem_triple *out,
+                        unsigned long long *d_count, void *scratch, cudaStream_t s);
 
 // K9 merge (merge.cu): G <= kMergeMaxRuns runs, each sorted by (r, q), pairwise disjoint
 // -> out (sum of counts triples) sorted by (r, q). The runs may be peer (IPC) memory.
@@ -181,6 +197,15 @@ constexpr int kMergeMaxRuns = 64;
 size_t merge_scratch_bytes(int n_runs, uint64_t total);
 cudaError_t merge_runs(const gpumem_triple *const *runs, const uint64_t *counts, int n_runs, gpumem_triple *out,
                        void *scratch, cudaStream_t s);
+
+// Multi-record split (fasta.cu): the pieces (length >= L) of the MEMs `in` cut at the
+// masked intervals of R (mr, nmr intervals) and Q (mq, nmq), as keys (r << qbits | q) and
+// lengths at off[i] (exclusive scan of the per-MEM piece counts cnt); *d_total = pieces.
+// Two phases: count + scan, then (keys, lens sized by *d_total) emit -- keys == nullptr
+// runs the first phase only.
+cudaError_t split_masked(const gpumem_triple *in, uint64_t n, const uint64_t *mr, uint64_t nmr, const uint64_t *mq,
+                         uint64_t nmq, uint32_t L, uint32_t qbits, uint32_t *cnt, uint32_t *off,
+                         unsigned long long *d_total, uint64_t *keys, uint32_t *lens, cudaStream_t s);
 
 // Triples (sort.cu)
 cudaError_t launch_keys_to_triples(const uint64_t *keys, const uint32_t *lens, uint64_t n, uint32_t qbits,

@@ -13,9 +13,10 @@
 //          memory as 64-bit keys (r << 32 | q); each triple's place in the bucket is
 //          its index in its own slice + the number of smaller keys in every other
 //          slice (binary search in shared memory; keys are unique across runs); the
-//          bucket is written back coalesced. A bucket over kCap (many MEMs with one r:
-//          low-complexity repeats) is ranked the same way with the searches in global
-//          memory.
+//          bucket is written back coalesced. A bucket over kCap (many MEMs in a narrow
+//          r range: low-complexity repeats) is split evenly over its key range into
+//          sub-buckets merged the same way; one still over kCap (keys that do not
+//          spread) is ranked with the searches in global memory.
 //
 // The runs may live in other GPUs' memory (CUDA IPC mappings of the ranks' result
 // buffers, dist.py): then this kernel is the gather and the merge in one pass, each
@@ -26,8 +27,15 @@ namespace gm {
 namespace {
 
 constexpr int kT = 256;
-constexpr int kCap = 2048;            // triples per bucket held in shared memory
-constexpr int kAvg = 512;             // target mean bucket size (kCap / 4: headroom for skew)
+#ifndef GM_MERGE_BT
+#define GM_MERGE_BT 512
+#endif
+#ifndef GM_MERGE_CAP
+#define GM_MERGE_CAP 4096
+#endif
+constexpr int kBT = GM_MERGE_BT;      // threads of the bucket kernel
+constexpr int kCap = GM_MERGE_CAP;    // triples per bucket held in shared memory
+constexpr int kAvg = kCap / 4;        // target mean bucket size (headroom for skew)
 constexpr int kMaxLog = 20;           // at most 2^20 buckets
 
 struct MergeRuns {
@@ -68,12 +76,18 @@ __global__ void __launch_bounds__(kT) k_merge_dir(const MergeRuns runs, uint32_t
     }
 }
 
+constexpr int kSubB = 32;            // sub-buckets of an oversized bucket handled per batch
+
 struct BucketSmem {
     uint64_t key[kCap];
     uint32_t len[kCap];
-    gpumem_triple out[kCap];
-    uint32_t off[kMergeMaxRuns + 1];   // slice h of the bucket: [off[h], off[h+1]) in key[]
+    uint16_t perm[kCap];               // perm[rank] = the triple's slot in key[] / len[]
+    uint32_t off[kMergeMaxRuns + 1];   // the slices being merged: slice h is key[off[h], off[h+1])
     uint32_t lo[kMergeMaxRuns];        // ... = run h's [lo[h], lo[h] + off[h+1] - off[h])
+    uint32_t blo[kMergeMaxRuns];       // the bucket's slices (oversized buckets: split further)
+    uint32_t bhi[kMergeMaxRuns];
+    uint32_t sb[kMergeMaxRuns * (kSubB + 1)];  // sub-bucket boundaries, [h][j]
+    uint64_t kmin, kmax;
 };
 
 // number of keys < k in a[0, n)
@@ -87,58 +101,51 @@ __device__ __forceinline__ uint32_t count_less(F at, uint32_t n, uint64_t k) {
     return lo;
 }
 
-__global__ void __launch_bounds__(kT) k_merge_bucket(const MergeRuns runs, uint32_t nb, const uint32_t *__restrict__ D,
-                                                      gpumem_triple *__restrict__ out) {
-    pdl_wait();
-    extern __shared__ __align__(16) unsigned char smem_raw[];
-    BucketSmem &s = *reinterpret_cast<BucketSmem *>(smem_raw);
-    const uint32_t b = blockIdx.x;
+// Merge the slices in s.lo / s.off (n <= kCap triples together) into out[0, n): keys to
+// shared memory, each triple's rank = its index in its slice + the smaller keys of every
+// other slice (binary searches in shared memory), coalesced write-back. All threads.
+__device__ void merge_in_smem(BucketSmem &s, const MergeRuns &runs, gpumem_triple *__restrict__ out) {
     const int G = runs.g;
-    if (threadIdx.x == 0) {
-        uint32_t acc = 0;
-        for (int h = 0; h < G; ++h) {
-            const uint32_t a = D[uint64_t(h) * (nb + 1) + b], z = D[uint64_t(h) * (nb + 1) + b + 1];
-            s.lo[h] = a;
-            s.off[h] = acc;
-            acc += z - a;
-        }
-        s.off[G] = acc;
+    const uint32_t n = s.off[G];
+    for (uint32_t i = threadIdx.x; i < n; i += kBT) {
+        int g = 0;
+        while (s.off[g + 1] <= i) ++g;
+        const gpumem_triple t = runs.run[g][s.lo[g] + (i - s.off[g])];
+        s.key[i] = key_of(t);
+        s.len[i] = t.len;
     }
     __syncthreads();
-    uint64_t base = 0;  // the bucket's first output slot: triples of all runs in earlier buckets
-    for (int h = 0; h < G; ++h) base += D[uint64_t(h) * (nb + 1) + b];
-    const uint32_t nbk = s.off[G];
-    if (nbk == 0) return;
-    if (nbk <= uint32_t(kCap)) {
-        for (uint32_t i = threadIdx.x; i < nbk; i += kT) {
-            int g = 0;
-            while (s.off[g + 1] <= i) ++g;
-            const gpumem_triple t = runs.run[g][s.lo[g] + (i - s.off[g])];
-            s.key[i] = key_of(t);
-            s.len[i] = t.len;
+    // rank of a triple = its index in its slice + the smaller keys of every other slice
+    for (uint32_t i = threadIdx.x; i < n; i += kBT) {
+        int g = 0;
+        while (s.off[g + 1] <= i) ++g;
+        const uint64_t k = s.key[i];
+        uint32_t rank = i - s.off[g];
+        for (int h = 0; h < G; ++h) {
+            if (h == g) continue;
+            const uint32_t o = s.off[h];
+            rank += count_less([&](uint32_t j) { return s.key[o + j]; }, s.off[h + 1] - o, k);
         }
-        __syncthreads();
-        for (uint32_t i = threadIdx.x; i < nbk; i += kT) {
-            int g = 0;
-            while (s.off[g + 1] <= i) ++g;
-            const uint64_t k = s.key[i];
-            uint32_t rank = i - s.off[g];
-            for (int h = 0; h < G; ++h) {
-                if (h == g) continue;
-                const uint32_t o = s.off[h];
-                rank += count_less([&](uint32_t j) { return s.key[o + j]; }, s.off[h + 1] - o, k);
-            }
-            s.out[rank] = gpumem_triple{uint32_t(k >> 32), uint32_t(k), s.len[i]};
-        }
-        __syncthreads();
-        // coalesced write-back: the bucket's triples as 32-bit words
-        const uint32_t *src = reinterpret_cast<const uint32_t *>(s.out);
-        uint32_t *dst = reinterpret_cast<uint32_t *>(out + base);
-        for (uint32_t w = threadIdx.x; w < nbk * 3; w += kT) dst[w] = src[w];
-        return;
+        s.perm[rank] = uint16_t(i);
     }
-    // oversized bucket: the same ranks, searched in global memory
-    for (uint32_t i = threadIdx.x; i < nbk; i += kT) {
+    __syncthreads();
+    uint32_t *dst = reinterpret_cast<uint32_t *>(out);  // coalesced write-back: consecutive triples
+    for (uint32_t e = threadIdx.x; e < n; e += kBT) {
+        const uint32_t src = s.perm[e];
+        const uint64_t k = s.key[src];
+        dst[3 * e] = uint32_t(k >> 32);
+        dst[3 * e + 1] = uint32_t(k);
+        dst[3 * e + 2] = s.len[src];
+    }
+    __syncthreads();
+}
+
+// The same ranks with the searches in global memory (a slice set over kCap whose keys
+// could not be split further). All threads.
+__device__ void merge_in_global(BucketSmem &s, const MergeRuns &runs, gpumem_triple *__restrict__ out) {
+    const int G = runs.g;
+    const uint32_t n = s.off[G];
+    for (uint32_t i = threadIdx.x; i < n; i += kBT) {
         int g = 0;
         while (s.off[g + 1] <= i) ++g;
         const gpumem_triple t = runs.run[g][s.lo[g] + (i - s.off[g])];
@@ -149,7 +156,91 @@ __global__ void __launch_bounds__(kT) k_merge_bucket(const MergeRuns runs, uint3
             const gpumem_triple *th = runs.run[h] + s.lo[h];
             rank += count_less([&](uint32_t j) { return key_of(th[j]); }, s.off[h + 1] - s.off[h], k);
         }
-        out[base + rank] = t;
+        out[rank] = t;
+    }
+    __syncthreads();
+}
+
+__global__ void __launch_bounds__(kBT) k_merge_bucket(const MergeRuns runs, uint32_t nb, const uint32_t *__restrict__ D,
+                                                       gpumem_triple *__restrict__ out) {
+    pdl_wait();
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    BucketSmem &s = *reinterpret_cast<BucketSmem *>(smem_raw);
+    const uint32_t b = blockIdx.x;
+    const int G = runs.g;
+    if (int(threadIdx.x) < G) {  // the bucket's slice of every run, loaded in parallel
+        const uint64_t r0 = uint64_t(threadIdx.x) * (nb + 1) + b;
+        s.lo[threadIdx.x] = s.blo[threadIdx.x] = D[r0];
+        s.bhi[threadIdx.x] = D[r0 + 1];
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        uint32_t acc = 0;
+        for (int h = 0; h < G; ++h) {
+            s.off[h] = acc;
+            acc += s.bhi[h] - s.blo[h];
+        }
+        s.off[G] = acc;
+    }
+    __syncthreads();
+    uint64_t base = 0;  // the bucket's first output slot: triples of all runs in earlier buckets
+    for (int h = 0; h < G; ++h) base += s.blo[h];
+    const uint32_t nbk = s.off[G];
+    if (nbk == 0) return;
+    if (nbk <= uint32_t(kCap)) {
+        merge_in_smem(s, runs, out + base);
+        return;
+    }
+    // Oversized bucket (many MEMs in a narrow r range: low-complexity repeats): split its
+    // key range [kmin, kmax] evenly into sub-buckets of ~kCap/2 expected triples, slice
+    // boundaries by binary search in each run, each sub-bucket merged like a bucket.
+    if (threadIdx.x == 0) {
+        uint64_t mn = ~0ull, mx = 0;
+        for (int h = 0; h < G; ++h) {
+            if (s.bhi[h] == s.blo[h]) continue;
+            mn = min(mn, key_of(runs.run[h][s.blo[h]]));
+            mx = max(mx, key_of(runs.run[h][s.bhi[h] - 1]));
+        }
+        s.kmin = mn;
+        s.kmax = mx;
+    }
+    __syncthreads();
+    const uint64_t kmin = s.kmin, span = s.kmax - s.kmin;  // keys in [kmin, kmin + span]
+    uint32_t nsub = (nbk + kCap / 2 - 1) / (kCap / 2);
+    if (uint64_t(nsub) > span + 1) nsub = uint32_t(span + 1);
+    const uint64_t w = span / nsub + 1;                       // nsub * w > span
+    uint64_t sbase = base;
+    for (uint32_t j0 = 0; j0 < nsub; j0 += kSubB) {
+        const uint32_t jn = min(uint32_t(kSubB), nsub - j0);
+        for (uint32_t x = threadIdx.x; x < uint32_t(G) * (jn + 1); x += kBT) {
+            const int h = int(x / (jn + 1));
+            const uint32_t j = x % (jn + 1);
+            uint32_t v = s.bhi[h];
+            if (j0 + j < nsub) {  // first index of run h's slice with key >= kmin + (j0 + j) * w
+                const gpumem_triple *th = runs.run[h] + s.blo[h];
+                v = s.blo[h] + count_less([&](uint32_t i) { return key_of(th[i]); }, s.bhi[h] - s.blo[h],
+                                          kmin + uint64_t(j0 + j) * w);
+            }
+            s.sb[h * (kSubB + 1) + j] = v;
+        }
+        __syncthreads();
+        for (uint32_t j = 0; j < jn; ++j) {
+            if (threadIdx.x == 0) {
+                uint32_t acc = 0;
+                for (int h = 0; h < G; ++h) {
+                    const uint32_t a = s.sb[h * (kSubB + 1) + j], z = s.sb[h * (kSubB + 1) + j + 1];
+                    s.lo[h] = a;
+                    s.off[h] = acc;
+                    acc += z - a;
+                }
+                s.off[G] = acc;
+            }
+            __syncthreads();
+            const uint32_t n = s.off[G];
+            if (n && n <= uint32_t(kCap)) merge_in_smem(s, runs, out + sbase);
+            else if (n) merge_in_global(s, runs, out + sbase);
+            sbase += n;
+        }
     }
 }
 
@@ -193,7 +284,7 @@ cudaError_t merge_runs(const gpumem_triple *const *runs, const uint64_t *counts,
     const uint64_t dir_blocks = (dir_n + kT - 1) / kT;
     pdl_launch(k_merge_dir, unsigned(dir_blocks < 4096 ? dir_blocks : 4096), kT, 0, s, mr, nb,
                static_cast<const uint32_t *>(shift), D);
-    pdl_launch(k_merge_bucket, nb, kT, sizeof(BucketSmem), s, mr, nb, static_cast<const uint32_t *>(D), out);
+    pdl_launch(k_merge_bucket, nb, kBT, sizeof(BucketSmem), s, mr, nb, static_cast<const uint32_t *>(D), out);
     note_launch(3);
     return cudaGetLastError();
 }

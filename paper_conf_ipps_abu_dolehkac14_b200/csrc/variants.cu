@@ -1,23 +1,25 @@
-// variants.cu -- NEXT-F3: maximal unique matches (MUMs) from the MEM set.
+// variants.cu -- NEXT-F3: maximal rare matches (MEMs whose string occurs at most k times
+// in R and at most k times in Q) and, as k = 1, maximal unique matches (MUMs).
 //
-// PAPER.md:23 defines a MUM as a match that "appears only once in both sequences
-// (i.e., unique) and cannot be extended to either directions" -- the paper's future
-// work (:286). Reading used here (R21): a MUM is a MEM (r, q, len) whose
-// string S = R[r, r+len) occurs exactly once in R and exactly once in Q.
+// PAPER.md:23 defines a MUM as a match that "appears only once in both sequences (i.e.,
+// unique) and cannot be extended to either directions" and mentions "maximal rare
+// matches"; :286 lists "unique and rare exact match extraction" as future work.
+// Reading used here (R21/R23): a rare MEM for k >= 1 is a MEM (r, q, len)
+// whose string S = R[r, r+len) occurs (overlapping occurrences counted) at most k times
+// in R and at most k times in Q; k = 1 gives the MUMs.
 //
-// From the MEM set alone: if S also occurs in R at r' != r, the diagonal r' - q matches
-// Q[q, q+len) for len >= L bases, so the maximal run through those cells is a MEM
-// (r'', q'', len'') on a different diagonal with q'' <= q and q'' + len'' >= q + len.
-// Conversely such a MEM yields another occurrence. So S is unique in R iff no other MEM's
-// query interval contains [q, q+len), and unique in Q iff no other MEM's reference
-// interval contains [r, r+len). (Two MEMs on one diagonal never nest: maximal runs on a
-// diagonal are disjoint.)
-//
-// Per axis: sort (start asc, len desc) with the radix sort; interval i is contained in
-// another iff the running maximum of the ends of the intervals before it reaches its own
-// end, or the next interval is identical. Prefix maxima: per-block maxima, a scan of the
-// block maxima, then a block-wide exclusive max-scan. The kept MEMs are compacted in
-// their original (r, q) order.
+// Counting from the MEM set alone: an occurrence of S in R at r' != r is a match of
+// length len >= L on the diagonal r' - q covering the query interval [q, q+len), so the
+// maximal run through it is a MEM (r'', q'', len'') on that diagonal with q'' <= q and
+// q'' + len'' >= q + len; different occurrences lie on different diagonals, and a
+// diagonal's maximal runs are disjoint, so
+//     occ_R(S) = #MEMs whose query interval contains [q, q+len)   (itself included),
+//     occ_Q(S) = #MEMs whose reference interval contains [r, r+len).
+// Per axis: sort the intervals by (start asc, len desc) (radix.cu); the intervals that
+// contain interval i are exactly the earlier ones with end >= end_i plus the identical
+// ones after it. A prefix scan whose running value is the top-K ends seen so far (K a
+// power of two > k; the union-of-two-top-K merge is associative) gives, for every i,
+// min(K, #earlier ends >= end_i) exactly. The kept MEMs are compacted in (r, q) order.
 #include "internal.h"
 #include "device.cuh"
 
@@ -27,6 +29,64 @@ namespace {
 constexpr int kT = 256;
 constexpr int kPer = 8;
 constexpr int kBlock = kT * kPer;  // items per CTA in the scans
+
+// The K largest interval ends seen, descending; 0 = empty (every end is >= L >= 1).
+template <int K>
+struct TopK {
+    uint32_t v[K];
+};
+
+template <int K>
+__device__ __forceinline__ TopK<K> topk_empty() {
+    TopK<K> t;
+#pragma unroll
+    for (int i = 0; i < K; ++i) t.v[i] = 0;
+    return t;
+}
+
+// Top K of the union of two descending lists: max(a[i], b[K-1-i]) is a bitonic sequence
+// holding the K largest; a bitonic merge network sorts it descending.
+template <int K>
+__device__ __forceinline__ TopK<K> topk_merge(const TopK<K> &a, const TopK<K> &b) {
+    TopK<K> c;
+#pragma unroll
+    for (int i = 0; i < K; ++i) c.v[i] = max(a.v[i], b.v[K - 1 - i]);
+#pragma unroll
+    for (int j = K / 2; j > 0; j >>= 1) {
+#pragma unroll
+        for (int i = 0; i < K; ++i) {
+            if ((i & j) == 0) {
+                const uint32_t x = c.v[i], y = c.v[i + j];
+                c.v[i] = max(x, y);
+                c.v[i + j] = min(x, y);
+            }
+        }
+    }
+    return c;
+}
+
+template <int K>
+__device__ __forceinline__ TopK<K> topk_one(uint32_t x) {
+    TopK<K> t = topk_empty<K>();
+    t.v[0] = x;
+    return t;
+}
+
+template <int K>
+__device__ __forceinline__ TopK<K> topk_shfl_up(const TopK<K> &a, int o) {
+    TopK<K> t;
+#pragma unroll
+    for (int i = 0; i < K; ++i) t.v[i] = __shfl_up_sync(0xffffffffu, a.v[i], o);
+    return t;
+}
+
+template <int K>
+__device__ __forceinline__ uint32_t topk_count_ge(const TopK<K> &a, uint32_t e) {
+    uint32_t c = 0;
+#pragma unroll
+    for (int i = 0; i < K; ++i) c += a.v[i] >= e ? 1u : 0u;
+    return c;
+}
 
 __global__ void __launch_bounds__(kT) k_interval_keys(const gpumem_triple *__restrict__ t, uint64_t n, int axis,
                                                       uint64_t *__restrict__ keys, uint32_t *__restrict__ vals) {
@@ -39,110 +99,105 @@ __global__ void __launch_bounds__(kT) k_interval_keys(const gpumem_triple *__res
     vals[i] = uint32_t(i);
 }
 
-__device__ __forceinline__ uint64_t end_of(uint64_t key) {
-    return (key >> 32) + uint64_t(~uint32_t(key));  // start + len
+__device__ __forceinline__ uint32_t end_of(uint64_t key) {
+    return uint32_t(key >> 32) + ~uint32_t(key);  // start + len (< 2^32: a position in a sequence)
 }
 
-__global__ void __launch_bounds__(kT) k_block_max(const uint64_t *__restrict__ keys, uint64_t n,
-                                                  uint64_t *__restrict__ bmax) {
-    pdl_wait();
-    __shared__ uint64_t ws[kT / 32];
-    const uint64_t base = uint64_t(blockIdx.x) * kBlock;
-    uint64_t m = 0;
-    for (int j = 0; j < kPer; ++j) {
-        const uint64_t i = base + uint64_t(j) * kT + threadIdx.x;
-        if (i < n) m = max(m, end_of(keys[i]));
-    }
-#pragma unroll
-    for (int o = 16; o; o >>= 1) m = max(m, __shfl_down_sync(0xffffffffu, m, o));
-    if ((threadIdx.x & 31) == 0) ws[threadIdx.x >> 5] = m;
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        uint64_t r = 0;
-        for (int w = 0; w < kT / 32; ++w) r = max(r, ws[w]);
-        bmax[blockIdx.x] = r;
-    }
-}
-
-// exclusive running maximum of bmax[0..m) in place (single CTA, sequential over chunks)
-__global__ void __launch_bounds__(kT) k_scan_max(uint64_t *bmax, uint64_t m) {
-    pdl_wait();
-    __shared__ uint64_t ws[kT / 32];
-    __shared__ uint64_t carry;
-    if (threadIdx.x == 0) carry = 0;
-    __syncthreads();
+// Block-wide inclusive scan of per-thread top-K lists (warp shuffles, then the warp
+// totals through shared memory). Returns the exclusive prefix of this thread; *total =
+// the block's aggregate.
+template <int K>
+__device__ __forceinline__ TopK<K> block_excl_scan(const TopK<K> &mine, TopK<K> *ws, TopK<K> *total) {
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-    for (uint64_t base = 0; base < m; base += kT) {
-        const uint64_t i = base + threadIdx.x;
-        const uint64_t x = i < m ? bmax[i] : 0;
-        uint64_t inc = x;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            const uint64_t y = __shfl_up_sync(0xffffffffu, inc, o);
-            if (lane >= o) inc = max(inc, y);
-        }
-        if (lane == 31) ws[w] = inc;
-        __syncthreads();
-        uint64_t pre = carry;
-        for (int k = 0; k < w; ++k) pre = max(pre, ws[k]);
-        const uint64_t up = __shfl_up_sync(0xffffffffu, inc, 1);
-        const uint64_t excl = lane ? max(pre, up) : pre;
-        uint64_t tot = carry;
-        for (int k = 0; k < kT / 32; ++k) tot = max(tot, ws[k]);
-        __syncthreads();
-        if (i < m) bmax[i] = excl;
-        if (threadIdx.x == 0) carry = tot;
-        __syncthreads();
-    }
-}
-
-__global__ void __launch_bounds__(kT) k_contained(const uint64_t *__restrict__ keys, const uint32_t *__restrict__ vals,
-                                                  uint64_t n, const uint64_t *__restrict__ bprefix,
-                                                  uint8_t *__restrict__ flags) {
-    pdl_wait();
-    __shared__ uint64_t ws[kT / 32];
-    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-    const uint64_t base = uint64_t(blockIdx.x) * kBlock + uint64_t(threadIdx.x) * kPer;  // blocked
-    uint64_t e[kPer];
-    uint64_t m = 0;
-#pragma unroll
-    for (int j = 0; j < kPer; ++j) {
-        e[j] = base + j < n ? end_of(keys[base + j]) : 0;
-        m = max(m, e[j]);
-    }
-    uint64_t inc = m;
+    TopK<K> inc = mine;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
-        const uint64_t y = __shfl_up_sync(0xffffffffu, inc, o);
-        if (lane >= o) inc = max(inc, y);
+        const TopK<K> y = topk_shfl_up(inc, o);
+        if (lane >= o) inc = topk_merge(inc, y);
     }
     if (lane == 31) ws[w] = inc;
     __syncthreads();
-    uint64_t run = bprefix[blockIdx.x];
-    for (int k = 0; k < w; ++k) run = max(run, ws[k]);
-    const uint64_t up = __shfl_up_sync(0xffffffffu, inc, 1);
-    if (lane) run = max(run, up);
+    TopK<K> pre = topk_empty<K>(), tot = topk_empty<K>();
+    for (int k = 0; k < kT / 32; ++k) {
+        if (k < w) pre = topk_merge(pre, ws[k]);
+        tot = topk_merge(tot, ws[k]);
+    }
+    const TopK<K> up = topk_shfl_up(inc, 1);
+    if (lane) pre = topk_merge(pre, up);
+    *total = tot;
+    __syncthreads();
+    return pre;
+}
+
+template <int K>
+__global__ void __launch_bounds__(kT) k_block_topk(const uint64_t *__restrict__ keys, uint64_t n,
+                                                   TopK<K> *__restrict__ bagg) {
+    pdl_wait();
+    __shared__ TopK<K> ws[kT / 32];
+    const uint64_t base = uint64_t(blockIdx.x) * kBlock + uint64_t(threadIdx.x) * kPer;
+    TopK<K> m = topk_empty<K>();
+    for (int j = 0; j < kPer; ++j)
+        if (base + j < n) m = topk_merge(m, topk_one<K>(end_of(keys[base + j])));
+    TopK<K> tot;
+    block_excl_scan(m, ws, &tot);
+    if (threadIdx.x == 0) bagg[blockIdx.x] = tot;
+}
+
+// exclusive scan of the block aggregates in place (one CTA, kT blocks per round)
+template <int K>
+__global__ void __launch_bounds__(kT) k_scan_topk(TopK<K> *bagg, uint64_t m) {
+    pdl_wait();
+    __shared__ TopK<K> ws[kT / 32];
+    TopK<K> carry = topk_empty<K>();
+    for (uint64_t base = 0; base < m; base += kT) {
+        const uint64_t i = base + threadIdx.x;
+        const TopK<K> x = i < m ? bagg[i] : topk_empty<K>();
+        TopK<K> tot;
+        const TopK<K> pre = block_excl_scan(x, ws, &tot);
+        if (i < m) bagg[i] = topk_merge(carry, pre);
+        carry = topk_merge(carry, tot);
+    }
+}
+
+// occ[vals[i]] = min(255, 1 + #intervals containing interval i other than itself), exact
+// up to K: the earlier ends >= end_i (from the top-K prefix) + identical intervals after i.
+template <int K>
+__global__ void __launch_bounds__(kT) k_occurrences(const uint64_t *__restrict__ keys, const uint32_t *__restrict__ vals,
+                                                    uint64_t n, const TopK<K> *__restrict__ bprefix,
+                                                    uint8_t *__restrict__ occ) {
+    pdl_wait();
+    __shared__ TopK<K> ws[kT / 32];
+    const uint64_t base = uint64_t(blockIdx.x) * kBlock + uint64_t(threadIdx.x) * kPer;  // blocked
+    uint32_t e[kPer];
+    TopK<K> m = topk_empty<K>();
+#pragma unroll
+    for (int j = 0; j < kPer; ++j) {
+        e[j] = base + j < n ? end_of(keys[base + j]) : 0;
+        if (base + j < n) m = topk_merge(m, topk_one<K>(e[j]));
+    }
+    TopK<K> tot;
+    TopK<K> run = topk_merge(bprefix[blockIdx.x], block_excl_scan(m, ws, &tot));
 #pragma unroll
     for (int j = 0; j < kPer; ++j) {
         const uint64_t i = base + j;
         if (i < n) {
-            bool c = run >= e[j] && i > 0;
-            if (!c && i + 1 < n && keys[i + 1] == keys[i]) c = true;  // identical interval follows
-            if (c) flags[vals[i]] = 1;
-            run = max(run, e[j]);
+            uint32_t c = 1 + topk_count_ge(run, e[j]);
+            for (uint64_t x = i + 1; x < n && c <= uint32_t(K) && keys[x] == keys[i]; ++x) ++c;
+            occ[vals[i]] = uint8_t(c < 255 ? c : 255);
+            run = topk_merge(run, topk_one<K>(e[j]));
         }
     }
 }
 
-__global__ void __launch_bounds__(kT) k_count_kept(const uint8_t *__restrict__ fq, const uint8_t *__restrict__ fr,
-                                                   uint64_t n, uint32_t *__restrict__ counts) {
+__global__ void __launch_bounds__(kT) k_count_kept(const uint8_t *__restrict__ oq, const uint8_t *__restrict__ orr,
+                                                   uint64_t n, uint32_t k, uint32_t *__restrict__ counts) {
     pdl_wait();
     __shared__ uint32_t ws[kT / 32];
     const uint64_t base = uint64_t(blockIdx.x) * kBlock;
     uint32_t c = 0;
     for (int j = 0; j < kPer; ++j) {
         const uint64_t i = base + uint64_t(j) * kT + threadIdx.x;
-        if (i < n && !fq[i] && !fr[i]) ++c;
+        if (i < n && oq[i] <= k && orr[i] <= k) ++c;
     }
 #pragma unroll
     for (int o = 16; o; o >>= 1) c += __shfl_down_sync(0xffffffffu, c, o);
@@ -188,8 +243,8 @@ __global__ void __launch_bounds__(kT) k_scan_sum(uint32_t *counts, uint64_t m, u
 }
 
 // order-preserving compaction of the kept triples (same striped order as k_count_kept)
-__global__ void __launch_bounds__(kT) k_compact(const gpumem_triple *__restrict__ in, const uint8_t *__restrict__ fq,
-                                                const uint8_t *__restrict__ fr, uint64_t n,
+__global__ void __launch_bounds__(kT) k_compact(const gpumem_triple *__restrict__ in, const uint8_t *__restrict__ oq,
+                                                const uint8_t *__restrict__ orr, uint64_t n, uint32_t k,
                                                 const uint32_t *__restrict__ offs, gpumem_triple *__restrict__ out) {
     pdl_wait();
     __shared__ uint32_t ws[kT / 32];
@@ -200,14 +255,14 @@ __global__ void __launch_bounds__(kT) k_compact(const gpumem_triple *__restrict_
     const uint64_t base = uint64_t(blockIdx.x) * kBlock;
     for (int j = 0; j < kPer; ++j) {
         const uint64_t i = base + uint64_t(j) * kT + threadIdx.x;
-        const bool keep = i < n && !fq[i] && !fr[i];
+        const bool keep = i < n && oq[i] <= k && orr[i] <= k;
         const unsigned bal = __ballot_sync(0xffffffffu, keep);
         if (lane == 0) ws[w] = __popc(bal);
         __syncthreads();
         uint32_t pre = 0, tot = 0;
-        for (int k = 0; k < kT / 32; ++k) {
-            if (k < w) pre += ws[k];
-            tot += ws[k];
+        for (int x = 0; x < kT / 32; ++x) {
+            if (x < w) pre += ws[x];
+            tot += ws[x];
         }
         if (keep) out[s_base + pre + __popc(bal & lanemask_lt())] = in[i];
         __syncthreads();
@@ -218,16 +273,27 @@ __global__ void __launch_bounds__(kT) k_compact(const gpumem_triple *__restrict_
 
 unsigned nblk(uint64_t n, uint64_t per) { return unsigned((n + per - 1) / per); }
 
-}  // namespace
-
-size_t mum_scratch_bytes(uint64_t n) {
-    const uint64_t nb = (n + kBlock - 1) / kBlock + 1;
-    return n * 8 * 2 + n * 4 * 2 + n * 2 + nb * 8 + nb * 4 + radix_scratch_bytes(n) + 8 * 256;
+template <int K>
+void launch_occurrences(const uint64_t *ks, const uint32_t *vs, uint64_t n, void *bagg, uint8_t *occ, cudaStream_t s) {
+    const uint64_t nb = (n + kBlock - 1) / kBlock;
+    auto *b = static_cast<TopK<K> *>(bagg);
+    pdl_launch(k_block_topk<K>, unsigned(nb), kT, 0, s, ks, n, b);
+    pdl_launch(k_scan_topk<K>, 1, kT, 0, s, b, nb);
+    pdl_launch(k_occurrences<K>, unsigned(nb), kT, 0, s, ks, vs, n, static_cast<const TopK<K> *>(b), occ);
 }
 
-cudaError_t mum_filter(const gpumem_triple *in, uint64_t n, gpumem_triple *out, unsigned long long *d_count,
-                       void *scratch, cudaStream_t s) {
+}  // namespace
+
+size_t rare_scratch_bytes(uint64_t n) {
+    const uint64_t nb = (n + kBlock - 1) / kBlock + 1;
+    return n * 8 * 2 + n * 4 * 2 + n * 2 + nb * sizeof(TopK<kRareMaxK + 1>) + nb * 4 + radix_scratch_bytes(n) +
+           8 * 256;
+}
+
+cudaError_t rare_filter(const gpumem_triple *in, uint64_t n, uint32_t k, gpumem_triple *out,
+                        unsigned long long *d_count, void *scratch, cudaStream_t s) {
     cudaError_t e;
+    if (k < 1 || k > uint32_t(kRareMaxK)) return cudaErrorInvalidValue;
     if (n == 0) return cudaMemsetAsync(d_count, 0, 8, s);
     const uint64_t nb = (n + kBlock - 1) / kBlock;
     auto align = [](uintptr_t p) { return (p + 255) & ~uintptr_t(255); };
@@ -240,28 +306,29 @@ cudaError_t mum_filter(const gpumem_triple *in, uint64_t n, gpumem_triple *out, 
     c = align(c + n * 4);
     uint32_t *v1 = reinterpret_cast<uint32_t *>(c);
     c = align(c + n * 4);
-    uint8_t *flags = reinterpret_cast<uint8_t *>(c);  // [axis][n]
+    uint8_t *occ = reinterpret_cast<uint8_t *>(c);  // [axis][n]
     c = align(c + n * 2);
-    uint64_t *bmax = reinterpret_cast<uint64_t *>(c);
-    c = align(c + (nb + 1) * 8);
+    void *bagg = reinterpret_cast<void *>(c);
+    c = align(c + (nb + 1) * sizeof(TopK<kRareMaxK + 1>));
     uint32_t *counts = reinterpret_cast<uint32_t *>(c);
     c = align(c + (nb + 1) * 4);
     void *rs = reinterpret_cast<void *>(c);
-    if ((e = cudaMemsetAsync(flags, 0, n * 2, s)) != cudaSuccess) return e;
-    for (int axis = 0; axis < 2; ++axis) {  // 0: query intervals (uniqueness in R), 1: reference (in Q)
+    for (int axis = 0; axis < 2; ++axis) {  // 0: query intervals (occurrences in R), 1: reference (in Q)
         pdl_launch(k_interval_keys, nblk(n, kT), kT, 0, s, in, n, axis, k0, v0);
         bool alt = false;
         if ((e = radix_sort_u64(k0, v0, k1, v1, n, 64, rs, s, &alt)) != cudaSuccess) return e;
         const uint64_t *ks = alt ? k1 : k0;
         const uint32_t *vs = alt ? v1 : v0;
-        pdl_launch(k_block_max, unsigned(nb), kT, 0, s, ks, n, bmax);
-        pdl_launch(k_scan_max, 1, kT, 0, s, bmax, nb);
-        pdl_launch(k_contained, unsigned(nb), kT, 0, s, ks, vs, n, bmax, flags + uint64_t(axis) * n);
+        uint8_t *o = occ + uint64_t(axis) * n;
+        if (k + 1 <= 2) launch_occurrences<2>(ks, vs, n, bagg, o, s);
+        else if (k + 1 <= 4) launch_occurrences<4>(ks, vs, n, bagg, o, s);
+        else if (k + 1 <= 8) launch_occurrences<8>(ks, vs, n, bagg, o, s);
+        else launch_occurrences<16>(ks, vs, n, bagg, o, s);
         note_launch(4);
     }
-    pdl_launch(k_count_kept, unsigned(nb), kT, 0, s, flags, flags + n, n, counts);
+    pdl_launch(k_count_kept, unsigned(nb), kT, 0, s, occ, occ + n, n, k, counts);
     pdl_launch(k_scan_sum, 1, kT, 0, s, counts, nb, d_count);
-    pdl_launch(k_compact, unsigned(nb), kT, 0, s, in, flags, flags + n, n, counts, out);
+    pdl_launch(k_compact, unsigned(nb), kT, 0, s, in, occ, occ + n, n, k, counts, out);
     note_launch(3);
     return cudaGetLastError();
 }

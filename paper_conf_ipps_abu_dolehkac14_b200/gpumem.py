@@ -46,6 +46,7 @@ SYMBOLS = {
     "gpumem_mems_to_host": (ctypes.c_int, [_vp, _vp, _c_u64]),
     "gpumem_mems_stats": (ctypes.c_int, [_vp, _vp]),
     "gpumem_mums": (ctypes.c_int, [_vp, _vp, _P(_vp)]),
+    "gpumem_rare": (ctypes.c_int, [_vp, _c_u32, _vp, _P(_vp)]),
     "gpumem_merge_sorted": (ctypes.c_int, [_P(_vp), _P(_c_u64), ctypes.c_int, _vp, _P(_vp)]),
     "gpumem_pipeline_create": (ctypes.c_int, [_c_u64, _c_u64, _c_u32, _c_u32, _c_u64, _c_u64, _vp, _P(_vp)]),
     "gpumem_pipeline_run": (ctypes.c_int, [_vp, _vp, _vp]),
@@ -58,6 +59,11 @@ SYMBOLS = {
     "gpumem_pipeline_export": (ctypes.c_int, [_vp, _vp, _P(_c_u64), _P(_c_u64)]),
     "gpumem_ipc_open": (ctypes.c_int, [_vp, _P(_vp)]),
     "gpumem_ipc_close": (ctypes.c_int, [_vp]),
+    "gpumem_fasta_parse": (ctypes.c_int, [ctypes.c_char_p, _c_u64, _P(_vp)]),
+    "gpumem_fasta_info": (ctypes.c_int, [_vp, _P(_c_u64), _P(_vp), _P(_c_u64), _P(_c_u64)]),
+    "gpumem_fasta_record": (ctypes.c_int, [_vp, _c_u64, _P(ctypes.c_char_p), _P(_c_u64), _P(_c_u64)]),
+    "gpumem_split_masked": (ctypes.c_int, [_vp, _vp, _vp, _c_u32, ctypes.c_int, _vp, _P(_vp)]),
+    "gpumem_write_mummer": (ctypes.c_int, [_vp, _c_u64, _vp, _c_u64, _vp, _vp, ctypes.c_char_p]),
     "gpumem_free": (None, [_vp]),
     "gpumem_trim": (ctypes.c_int, []),
     "gpumem_last_error": (ctypes.c_char_p, []),
@@ -293,6 +299,63 @@ def merge_runs(ptrs, counts, stream=None) -> Mems:
     h = _vp()
     _check(_lib.gpumem_merge_sorted(p, c, len(ptrs), _stream(stream), ctypes.byref(h)))
     return Mems(h.value)
+
+
+class Fasta(_Handle):
+    """A parsed multi-FASTA (gpumem_fasta_parse): records concatenated with one masked
+    separator base, non-ACGT letters masked."""
+
+    def info(self):
+        nrec, ptr, n, nm = _c_u64(), _vp(), _c_u64(), _c_u64()
+        _check(_lib.gpumem_fasta_info(self.handle, ctypes.byref(nrec), ctypes.byref(ptr), ctypes.byref(n),
+                                      ctypes.byref(nm)))
+        return nrec.value, ptr.value, n.value, nm.value
+
+    def seq(self) -> np.ndarray:
+        """The concatenated ASCII sequence (a copy)."""
+        _, ptr, n, _ = self.info()
+        return np.ctypeslib.as_array((ctypes.c_uint8 * n).from_address(ptr)).copy() if n else \
+            np.zeros(0, np.uint8)
+
+    def records(self):
+        """[(name, start, length)] in input order."""
+        out = []
+        for i in range(self.info()[0]):
+            nm, st, ln = ctypes.c_char_p(), _c_u64(), _c_u64()
+            _check(_lib.gpumem_fasta_record(self.handle, i, ctypes.byref(nm), ctypes.byref(st), ctypes.byref(ln)))
+            out.append((nm.value.decode(), st.value, ln.value))
+        return out
+
+
+def fasta_parse(text) -> Fasta:
+    b = text.encode() if isinstance(text, str) else bytes(text)
+    h = _vp()
+    _check(_lib.gpumem_fasta_parse(b, len(b), ctypes.byref(h)))
+    return Fasta(h.value)
+
+
+def split_masked(m: Mems, R: Fasta, Q: Fasta, min_len: int, q_reverse=False, stream=None) -> Mems:
+    """The multi-record MEMs: m (MEMs of the concatenations) cut at masked positions."""
+    h = _vp()
+    _check(_lib.gpumem_split_masked(m.handle, R.handle, Q.handle, int(min_len), 1 if q_reverse else 0,
+                                    _stream(stream), ctypes.byref(h)))
+    return Mems(h.value, (m, R, Q))
+
+
+def write_mummer(path, fwd, R: Fasta, Q: Fasta, rev=None):
+    """MUMmer-style text (1-based, per query record) from host (N, 3) uint32 triples."""
+    f = np.ascontiguousarray(fwd, dtype=np.uint32)
+    r = None if rev is None else np.ascontiguousarray(rev, dtype=np.uint32)
+    _check(_lib.gpumem_write_mummer(f.ctypes.data_as(_vp) if len(f) else None, len(f),
+                                    (r.ctypes.data_as(_vp) if len(r) else _vp(1)) if r is not None else None,
+                                    0 if r is None else len(r), R.handle, Q.handle, str(path).encode()))
+
+
+def rare(m: Mems, k: int, stream=None) -> Mems:
+    """MEMs whose string occurs at most k times in R and in Q (k = 1: MUMs), (r, q) order."""
+    h = _vp()
+    _check(_lib.gpumem_rare(m.handle, int(k), _stream(stream), ctypes.byref(h)))
+    return Mems(h.value, m)
 
 
 def merge_sorted(runs, stream=None) -> Mems:

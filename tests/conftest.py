@@ -32,6 +32,8 @@ def read_golden(name):
                 d[k] = v[0]
             elif k in ("ptrs", "locs"):
                 d[k] = [int(x) for x in v]
+            elif k[0] == "k" and k[1:].isdigit():  # expected triples at a parameter k (rare MEMs)
+                d.setdefault(k, []).append(tuple(int(x) for x in v))
             else:
                 d[k] = int(v[0])
     return d

@@ -387,19 +387,25 @@ def test_full_size_c4_c5(c4_full, L):
 
 
 @pytest.mark.slow
-def test_full_size_shards_byte_identical(c4_full):
-    """SURVEY.md §8(e) check at the full C4 size: the query-sharded runs of G = 1, 2, 4, 8
-    ranks (one pipeline per rank's MEM-start range, as bench.py --gpus G runs them;
-    here all on one device) concatenate, after the rank-0 merge kernel, to the byte-
-    identical whole set."""
+@pytest.mark.parametrize("L", [100, 20])
+def test_full_size_shards_byte_identical(c4_full, L):
+    """SURVEY.md §8(e) check at the full C4 / C5 L = 20 size: the query-sharded runs of
+    G = 1, 2, 4, 8 ranks (one pipeline per rank's MEM-start range, as bench.py --gpus G
+    runs them; here all on one device) merge (K9, merge.cu) to the byte-identical whole
+    set of the single pipeline."""
     P = c4_full
     Rt, Qt = torch.from_numpy(P.R).cuda(), torch.from_numpy(P.Q).cuda()
     from paper_conf_ipps_abu_dolehkac14_b200.dist import shard_range
-    whole = None
-    for G in (1, 2, 4, 8):
+    pl = gpumem.Pipeline(len(P.R), len(P.Q), P.ls, L)
+    pl.run(Rt, Qt)
+    pl.result()
+    whole = pl.numpy()
+    pl.free()
+    assert len(whole) == {100: 811662, 20: 13420345}[L]
+    for G in (2, 4, 8):
         runs = []
         for g in range(G):
-            pl = gpumem.Pipeline(len(P.R), len(P.Q), P.ls, P.L, shard_range(len(P.Q), g, G))
+            pl = gpumem.Pipeline(len(P.R), len(P.Q), P.ls, L, shard_range(len(P.Q), g, G))
             pl.run(Rt, Qt)
             pl.result()
             runs.append(pl.view_u32().clone())
@@ -407,9 +413,6 @@ def test_full_size_shards_byte_identical(c4_full):
         merged = gpumem.merge_sorted([r.view(torch.int32) for r in runs])
         got = merged.numpy()
         merged.free()
-        if whole is None:
-            whole = got
-            assert len(whole) == 811662
         assert got.tobytes() == whole.tobytes(), G
 
 
@@ -474,6 +477,45 @@ def test_mums_tiny_random():
         ls = int(rng.integers(1, L + 1))
         m = gpumem.find_mems(gpumem.index_build(gpumem.pack(R.tobytes()), min(ls, 15), L), gpumem.pack(Q.tobytes()))
         assert np.array_equal(gpumem.mums(m).numpy(), oracle.mums(R, Q, L, min(ls, 15))), trial
+
+
+@pytest.mark.parametrize("cfg,scale,L", [("c1", 1.0, 20), ("c3", 0.01, 30), ("c4", 0.005, 30)])
+@pytest.mark.parametrize("k", [1, 2, 5, 15])
+def test_rare(cfg, scale, L, k):
+    """F3: rare MEMs (string occurs <= k times in R and in Q; R23) vs the
+    substring-count oracle; k = 1 equals gpumem_mums."""
+    P = synth.make_pair(cfg, scale=scale)
+    ls = min(P.ls, L)
+    m = gpumem.find_mems(gpumem.index_build(gpumem.pack(P.R), ls, L), gpumem.pack(P.Q))
+    got = gpumem.rare(m, k).numpy()
+    want = oracle.rare(P.R, P.Q, L, ls, k)
+    assert np.array_equal(got, want)
+    if k == 1:
+        assert np.array_equal(got, gpumem.mums(m).numpy())
+
+
+def test_rare_golden_homopolymer_and_tiny():
+    g = read_golden("w3_rare.txt")
+    for k in (1, 2):
+        m = gpumem.find_mems(gpumem.index_build(gpumem.pack(g["R"]), 2, g["L"]), gpumem.pack(g["Q"]))
+        assert [tuple(t) for t in gpumem.rare(m, k).numpy().tolist()] == sorted(g[f"k{k}"])
+    for n, mm, L, k in ((300, 200, 20, 1), (300, 200, 20, 100 // 10), (500, 520, 480, 15), (64, 64, 8, 7)):
+        m = gpumem.find_mems(gpumem.index_build(gpumem.pack("A" * n), min(L, 13), L), gpumem.pack("A" * mm))
+        want = [t for t in pyoracle.homopolymer(n, mm, L) if n - t[2] + 1 <= k and mm - t[2] + 1 <= k]
+        assert [tuple(t) for t in gpumem.rare(m, k).numpy().tolist()] == want, (n, mm, L, k)
+    rng = np.random.default_rng(6)
+    for trial in range(80):
+        R, Q = synth.random_pair(rng, int(rng.integers(2, 150)), int(rng.integers(2, 150)),
+                                 [b"AC", b"ACG", b"ACGT"][trial % 3])
+        L = int(rng.integers(2, 12))
+        ls = min(int(rng.integers(1, L + 1)), 15)
+        k = int(rng.integers(1, 16))
+        m = gpumem.find_mems(gpumem.index_build(gpumem.pack(R.tobytes()), ls, L), gpumem.pack(Q.tobytes()))
+        assert np.array_equal(gpumem.rare(m, k).numpy(), oracle.rare(R, Q, L, ls, k)), trial
+    with pytest.raises(gpumem.GpumemError):
+        gpumem.rare(m, 0)
+    with pytest.raises(gpumem.GpumemError):
+        gpumem.rare(m, 16)
 
 
 @pytest.mark.slow

@@ -217,3 +217,33 @@ def test_mums_random_vs_python_twin():
         L = int(rng.integers(2, 10))
         want = set(pyoracle.mums(R.tobytes(), Q.tobytes(), L))
         assert as_set(oracle.mums(R, Q, L, min(L, 3))) == want
+
+
+def test_golden_rare_w3():
+    """Rare MEMs (R23) of the hand-worked W3 fixture at k = 1 and k = 2, both oracles."""
+    g = read_golden("w3_rare.txt")
+    for k in (1, 2):
+        want = set(g[f"k{k}"])
+        assert set(pyoracle.rare(g["R"], g["Q"], g["L"], k)) == want
+        for ls in (1, 2, 4):
+            assert as_set(oracle.rare(g["R"], g["Q"], g["L"], ls, k)) == want
+    assert as_set(oracle.rare(g["R"], g["Q"], g["L"], 4, 1)) == as_set(oracle.mums(g["R"], g["Q"], g["L"], 4))
+
+
+@pytest.mark.parametrize("n,m,L,k", [(30, 20, 5, 1), (30, 20, 5, 3), (25, 25, 4, 7), (12, 40, 2, 15)])
+def test_rare_homopolymer_closed_form(n, m, L, k):
+    """A^n vs A^m: the MEM of length len has A^len, which occurs n - len + 1 times in R and
+    m - len + 1 times in Q; it is rare iff both counts are <= k."""
+    want = {t for t in pyoracle.homopolymer(n, m, L) if n - t[2] + 1 <= k and m - t[2] + 1 <= k}
+    assert set(pyoracle.rare("A" * n, "A" * m, L, k)) == want
+    assert as_set(oracle.rare("A" * n, "A" * m, L, min(L, 3), k)) == want
+
+
+def test_rare_random_vs_python_twin():
+    rng = np.random.default_rng(78)
+    for trial in range(60):
+        R, Q = synth.random_pair(rng, int(rng.integers(5, 120)), int(rng.integers(5, 120)), ALPHABETS[trial % 4])
+        L = int(rng.integers(2, 10))
+        k = int(rng.integers(1, 6))
+        want = set(pyoracle.rare(R.tobytes(), Q.tobytes(), L, k))
+        assert as_set(oracle.rare(R, Q, L, min(L, 3), k)) == want
