@@ -123,6 +123,28 @@ gpumem_status gpumem_index_build_range(const gpumem_seq *R, uint32_t seed_len, u
                                        uint64_t r_begin, uint64_t r_end, void *cuda_stream,
                                        gpumem_index **out);
 
+/*
+ * gpumem_find_mems_banded -- the paper's reference row sweep (NEXT-F2; PAPER.md:76-80
+ *  §III "only a partial index is created for l_tile base pairs of reference", :92 §III-A)
+ *  for an R that need not fit in device memory: r_bases_host (ASCII, host, r_len bases)
+ *  is processed in bands of band_len bases (0 = one band; rounded up to a multiple of the
+ *  step). Only one window of R is resident at a time: the band plus `step` bases before
+ *  it and max(L, 1024) after it, copied, packed and indexed over the band's sampled seeds
+ *  (gpumem_index_build_range on the window), then searched against all of Q (resident,
+ *  packed). A MEM cut by its window's right end is carried to the next band and its
+ *  extension continued there (replacing the out-tile combining of PAPER.md:179-185).
+ *  *out: the same set as gpumem_find_mems on the whole of R, sorted by (r, q). stats
+ *  (optional): bands, band_len used, largest window in bytes, MEMs carried across
+ *  windows, MEMs. Synchronises once per band. Errors as gpumem_index_build /
+ *  gpumem_find_mems; *out NULL on error, nothing leaked.
+ */
+typedef struct {
+    uint64_t bands, band_len, window_bytes, carried, mems;
+} gpumem_band_stats;
+gpumem_status gpumem_find_mems_banded(const char *r_bases_host, uint64_t r_len, const gpumem_seq *Q, uint32_t seed_len,
+                                      uint32_t min_len, uint64_t band_len, void *cuda_stream, gpumem_mems **out,
+                                      gpumem_band_stats *stats);
+
 /* Borrowed device pointers to ptrs (4^ls + 1 entries) and locs (n_locs entries). The first
  * request for ptrs expands it on the index's stream and synchronises that stream. */
 gpumem_status gpumem_index_view(const gpumem_index *idx, const uint32_t **dev_ptrs,

@@ -1551,6 +1551,117 @@ gpumem_status gpumem_split_masked(const gpumem_mems *m, const gpumem_fasta *R, c
     return st;
 }
 
+gpumem_status gpumem_find_mems_banded(const char *r_bases_host, uint64_t r_len, const gpumem_seq *Q, uint32_t seed_len,
+                                      uint32_t min_len, uint64_t band_len, void *cuda_stream, gpumem_mems **out,
+                                      gpumem_band_stats *stats) {
+    if (!out) return fail(GPUMEM_ERR_ARG, "out is NULL");
+    *out = nullptr;
+    if (!r_bases_host && r_len) return fail(GPUMEM_ERR_ARG, "r_bases_host is NULL");
+    if (!Q || Q->magic != kMagicSeq) return fail(GPUMEM_ERR_ARG, "Q is not a gpumem_seq");
+    if (seed_len < 1 || seed_len > 15 || min_len < seed_len)
+        return fail(GPUMEM_ERR_ARG, "need 1 <= seed_len <= 15 and seed_len <= min_len (got %u, %u)", seed_len, min_len);
+    if (r_len >= (1ull << 32)) return fail(GPUMEM_ERR_RANGE, "sequences must be shorter than 2^32 bases");
+    int dev;
+    gpumem_status st = check_device(&dev);
+    if (st) return st;
+    if (Q->device != dev) return fail(GPUMEM_ERR_ARG, "Q lives on another device");
+    cudaStream_t s = static_cast<cudaStream_t>(cuda_stream);
+    const uint64_t step = min_len - seed_len + 1;
+    if (band_len == 0 || band_len > r_len) band_len = r_len ? r_len : 1;
+    band_len = (band_len + step - 1) / step * step;        // bands start on the sampling grid
+    const uint64_t halo = min_len > 1024 ? min_len : 1024;  // >= L: a cut MEM is still reported
+    uint64_t max_w = 0;
+    for (uint64_t b0 = 0; b0 < r_len; b0 += band_len) {
+        const uint64_t w0 = b0 >= step ? b0 - step : 0, b1 = min(b0 + band_len, r_len);
+        max_w = max(max_w, min(b1 + halo, r_len) - w0);
+    }
+    Scratch sc(s);
+    char *dwin = static_cast<char *>(sc.get(max_w ? max_w : 1));
+    auto *ctr = static_cast<unsigned long long *>(sc.get(64));
+    unsigned long long *h = pinned_slots();
+    if (!dwin || !ctr || !h) return GPUMEM_ERR_NOMEM;
+    std::vector<std::pair<gpumem_triple *, uint64_t>> chunks;  // closed MEMs per band (global r)
+    gpumem_triple *open = nullptr;
+    uint64_t n_open = 0, bands = 0, carried = 0;
+    auto release = [&]() {
+        for (auto &c : chunks) dfree(c.first, s);
+        chunks.clear();
+        if (open) dfree(open, s);
+        open = nullptr;
+    };
+    for (uint64_t b0 = 0; b0 < r_len; b0 += band_len, ++bands) {
+        const uint64_t b1 = min(b0 + band_len, r_len);
+        const uint64_t w0 = b0 >= step ? b0 - step : 0, w1 = min(b1 + halo, r_len), wlen = w1 - w0;
+        const int more = w1 < r_len ? 1 : 0;
+        Stage g("band", s);
+        if (cudaMemcpyAsync(dwin, r_bases_host + w0, wlen, cudaMemcpyHostToDevice, s) != cudaSuccess) {
+            release();
+            return cuda_fail(cudaGetLastError(), "H2D band window");
+        }
+        gpumem_seq *W = nullptr;
+        gpumem_index *idx = nullptr;
+        gpumem_mems *m = nullptr;
+        st = gpumem_pack(dwin, wlen, 1, s, &W);
+        if (!st) st = gpumem_index_build_range(W, seed_len, min_len, b0 - w0, b1 - w0, s, &idx);
+        if (!st) st = gpumem_find_mems(idx, Q, 0, UINT64_MAX, s, &m);
+        const uint64_t cap = (m ? m->count : 0) + n_open;
+        gpumem_triple *closed = st ? nullptr : static_cast<gpumem_triple *>(dalloc((cap ? cap : 1) * 12, s));
+        gpumem_triple *open2 = st ? nullptr : static_cast<gpumem_triple *>(dalloc((cap ? cap : 1) * 12, s));
+        if (!st && (!closed || !open2)) st = GPUMEM_ERR_NOMEM;
+        cudaError_t e = cudaSuccess;
+        if (!st) e = cudaMemsetAsync(ctr, 0, 16, s);
+        if (!st && e == cudaSuccess)  // carried MEMs first: continue their right extension here
+            e = band_continue(open, n_open, W->words, w0, wlen, more, Q->words, Q->n, closed, ctr, open2, ctr + 1, s);
+        if (!st && e == cudaSuccess) e = band_place(m->dev, m->count, w0, wlen, more, closed, ctr, open2, ctr + 1, s);
+        if (!st && e == cudaSuccess) e = cudaMemcpyAsync(h, ctr, 16, cudaMemcpyDeviceToHost, s);
+        if (!st && e == cudaSuccess) e = cudaStreamSynchronize(s);
+        for (void *x : {(void *)m, (void *)idx, (void *)W}) gpumem_free(x);
+        if (!st && e != cudaSuccess) st = cuda_fail(e, "band");
+        if (st) {
+            if (closed) dfree(closed, s);
+            if (open2) dfree(open2, s);
+            release();
+            return st;
+        }
+        carried += n_open;
+        if (open) dfree(open, s);
+        open = open2;
+        n_open = h[1];
+        chunks.push_back({closed, h[0]});
+    }
+    // every MEM is closed after the last band (no R follows it)
+    uint64_t total = 0;
+    for (auto &c : chunks) total += c.second;
+    const uint32_t qbits = bits_for(Q->n ? Q->n : 1);
+    auto *keys = static_cast<uint64_t *>(ws_get(kWsKeys, (total ? total : 1) * 8, s));
+    auto *lens = static_cast<uint32_t *>(ws_get(kWsLens, (total ? total : 1) * 4, s));
+    if (!keys || !lens) {
+        release();
+        return GPUMEM_ERR_NOMEM;
+    }
+    uint64_t off = 0;
+    for (auto &c : chunks) {
+        const cudaError_t e = launch_triples_to_keys(c.first, c.second, qbits, keys + off, lens + off, s);
+        if (e != cudaSuccess) {
+            release();
+            return cuda_fail(e, "band keys");
+        }
+        off += c.second;
+    }
+    st = sort_into_triples(keys, lens, total, bits_for(r_len ? r_len : 1) + qbits, qbits, dev, s, out);
+    release();
+    if (st) return st;
+    (*out)->stats.mems = total;
+    if (stats) {
+        stats->bands = bands;
+        stats->band_len = band_len;
+        stats->window_bytes = max_w;
+        stats->carried = carried;
+        stats->mems = total;
+    }
+    return GPUMEM_OK;
+}
+
 gpumem_status gpumem_mems_view(const gpumem_mems *m, const gpumem_triple **dev_ptr, uint64_t *count) {
     if (!m || m->magic != kMagicMems) return fail(GPUMEM_ERR_ARG, "not a gpumem_mems");
     if (dev_ptr) *dev_ptr = m->dev;

@@ -207,6 +207,16 @@ cudaError_t split_masked(const gpumem_triple *in, uint64_t n, const uint64_t *mr
                          uint64_t nmq, uint32_t L, uint32_t qbits, uint32_t *cnt, uint32_t *off,
                          unsigned long long *d_total, uint64_t *keys, uint32_t *lens, cudaStream_t s);
 
+// Band sweep (band.cu): place a band's local triples (global r = r + w0) into the closed
+// or open list, and continue carried open MEMs in the next window.
+cudaError_t band_place(const gpumem_triple *in, uint64_t n, uint64_t w0, uint64_t wlen, int more,
+                       gpumem_triple *closed, unsigned long long *n_closed, gpumem_triple *open,
+                       unsigned long long *n_open, cudaStream_t s);
+cudaError_t band_continue(const gpumem_triple *in, uint64_t n, const uint64_t *W, uint64_t w0, uint64_t wlen,
+                          int more, const uint64_t *Q, uint64_t nQ, gpumem_triple *closed,
+                          unsigned long long *n_closed, gpumem_triple *open, unsigned long long *n_open,
+                          cudaStream_t s);
+
 // Triples (sort.cu)
 cudaError_t launch_keys_to_triples(const uint64_t *keys, const uint32_t *lens, uint64_t n, uint32_t qbits,
                                    gpumem_triple *out, cudaStream_t s, const unsigned long long *dn = nullptr);

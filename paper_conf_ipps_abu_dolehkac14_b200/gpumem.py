@@ -64,6 +64,7 @@ SYMBOLS = {
     "gpumem_fasta_record": (ctypes.c_int, [_vp, _c_u64, _P(ctypes.c_char_p), _P(_c_u64), _P(_c_u64)]),
     "gpumem_split_masked": (ctypes.c_int, [_vp, _vp, _vp, _c_u32, ctypes.c_int, _vp, _P(_vp)]),
     "gpumem_write_mummer": (ctypes.c_int, [_vp, _c_u64, _vp, _c_u64, _vp, _vp, ctypes.c_char_p]),
+    "gpumem_find_mems_banded": (ctypes.c_int, [_vp, _c_u64, _vp, _c_u32, _c_u32, _c_u64, _vp, _P(_vp), _vp]),
     "gpumem_free": (None, [_vp]),
     "gpumem_trim": (ctypes.c_int, []),
     "gpumem_last_error": (ctypes.c_char_p, []),
@@ -349,6 +350,27 @@ def write_mummer(path, fwd, R: Fasta, Q: Fasta, rev=None):
     _check(_lib.gpumem_write_mummer(f.ctypes.data_as(_vp) if len(f) else None, len(f),
                                     (r.ctypes.data_as(_vp) if len(r) else _vp(1)) if r is not None else None,
                                     0 if r is None else len(r), R.handle, Q.handle, str(path).encode()))
+
+
+class BandStats(ctypes.Structure):
+    _fields_ = [("bands", _c_u64), ("band_len", _c_u64), ("window_bytes", _c_u64), ("carried", _c_u64),
+                ("mems", _c_u64)]
+
+    def as_dict(self):
+        return {k: int(getattr(self, k)) for k, _ in self._fields_}
+
+
+def find_mems_banded(R_host, Q: Seq, seed_len: int, min_len: int, band_len: int, stream=None):
+    """Row sweep over bands of a host-resident R (only one window of R on the device);
+    returns (Mems, stats dict). Same MEM set as find_mems on the whole of R."""
+    a = np.ascontiguousarray(np.frombuffer(R_host.encode(), np.uint8) if isinstance(R_host, str)
+                             else (np.frombuffer(bytes(R_host), np.uint8)
+                                   if isinstance(R_host, (bytes, bytearray)) else R_host), dtype=np.uint8)
+    h = _vp()
+    st = BandStats()
+    _check(_lib.gpumem_find_mems_banded(a.ctypes.data_as(_vp), a.size, Q.handle, int(seed_len), int(min_len),
+                                        int(band_len), _stream(stream), ctypes.byref(h), ctypes.byref(st)))
+    return Mems(h.value, Q), st.as_dict()
 
 
 def rare(m: Mems, k: int, stream=None) -> Mems:

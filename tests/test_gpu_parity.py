@@ -437,6 +437,35 @@ def test_band_index_union_is_whole(cfg, scale, bands):
     assert np.array_equal(whole, oracle.mems(P.R, P.Q, P.L, P.ls))
 
 
+@pytest.mark.parametrize("cfg,scale,band", [("c1", 1.0, 7000), ("c1", 1.0, 0), ("c2", 0.1, 50_000),
+                                            ("c4", 0.02, 1_000_000), ("c5_l20", 0.02, 333_333), ("c3", 0.03, 80_000)])
+def test_band_sweep_equals_whole(cfg, scale, band):
+    """F2 row sweep with a band-local R window: only one window of
+    R on the device, MEMs cut at a window's end carried to the next band -- the same set
+    as the whole-R path and the oracle."""
+    P = synth.make_pair(cfg, scale=scale)
+    want = oracle.mems(P.R, P.Q, P.L, P.ls)
+    Q = gpumem.pack(P.Q)
+    m, st = gpumem.find_mems_banded(P.R, Q, P.ls, P.L, band)
+    assert np.array_equal(m.numpy(), want), st
+    if band:
+        assert st["bands"] == -(-len(P.R) // st["band_len"]) and st["window_bytes"] < len(P.R)
+
+
+def test_band_sweep_long_matches_cross_many_windows():
+    """Homopolymers and a self-match: MEMs far longer than a band run through many
+    windows (carried and continued band after band), against the closed form."""
+    for n, m_, L, ls, band in ((20_000, 9_000, 30, 10, 2_100), (5_000, 5_000, 20, 13, 800), (3_000, 40_000, 1, 1, 64)):
+        want = np.array(pyoracle.homopolymer(n, m_, L), dtype=np.uint32).reshape(-1, 3)
+        got, st = gpumem.find_mems_banded("A" * n, gpumem.pack("A" * m_), ls, L, band)
+        assert np.array_equal(got.numpy(), want), (n, m_, L, band)
+        assert st["carried"] > 0
+    P = synth.make_pair("c1", scale=0.5)
+    got, st = gpumem.find_mems_banded(P.R, gpumem.pack(P.R), P.ls, P.L, 3000)
+    assert (0, 0, len(P.R)) in {tuple(t) for t in got.numpy().tolist()} and st["carried"] > 0
+    assert np.array_equal(got.numpy(), oracle.mems(P.R, P.R, P.L, P.ls))
+
+
 @pytest.mark.parametrize("n", [1, 31, 32, 33, 100, 4097])
 def test_revcomp_words(n):
     rng = np.random.default_rng(n)
