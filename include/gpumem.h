@@ -243,9 +243,14 @@ gpumem_status gpumem_merge_sorted(const gpumem_triple *const *dev_runs, const ui
  *
  * gpumem_pipeline_run_host -- the same from host memory (pinned for full speed): R and Q
  *  are copied on a copy stream into pipeline-owned device buffers (allocated on the
- *  first call), R first; the graph packs and indexes R while Q is still in flight (its
- *  external event-wait nodes make each branch wait only for the copy it reads). Async: the host buffers must stay
- *  valid and unmodified until the run completes (gpumem_pipeline_result).
+ *  first call, through the allocator hook), R first; the graph packs and indexes R while
+ *  Q is still in flight. Q crosses PCIe in q_chunks pieces (option "q_chunks", read at
+ *  gpumem_pipeline_create; pieces >= max(1 Mbp, 4 L) bases; whole-Q pipelines only):
+ *  piece j is packed as soon as it has arrived and the MEMs starting in piece i are
+ *  searched once pieces <= i + 1 are present, extensions stopping at the data present;
+ *  the few matches cut there are finished after the last piece. Same
+ *  result as gpumem_pipeline_run. Async: the host buffers must stay valid and
+ *  unmodified until the run completes (gpumem_pipeline_result).
  *
  * gpumem_pipeline_result -- synchronises the stream, then checks the alphabet flags
  *  (GPUMEM_ERR_ALPHABET as gpumem_find_mems) and the output capacity: on overflow the
@@ -367,6 +372,8 @@ gpumem_status gpumem_set_allocator(void *(*alloc_fn)(size_t bytes, void *cuda_st
  *  "pdl"              1 (default): programmatic dependent launch between consecutive
  *                     kernels (each waits for its predecessor with griddepcontrol.wait);
  *                     0: ordinary launches
+ *  "q_chunks"         host-input pipelines: pieces Q is copied, packed and searched in
+ *                     (default 8; 1 = search after the whole Q has arrived); read at create
  *  "radix_bits"       LSD digit width: 0 (default) = 9 bits when that saves a pass, else 8;
  *                     or pinned to 8, 9, 10; anything else is GPUMEM_ERR_ARG
  * Unknown names are GPUMEM_ERR_ARG. */

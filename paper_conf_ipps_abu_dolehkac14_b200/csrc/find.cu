@@ -176,6 +176,16 @@ __device__ __forceinline__ uint32_t ext_left(const uint64_t *__restrict__ R, con
     return min(e, lim);
 }
 
+// Streamed query (host-input pipeline, Q arriving in chunks): extensions stop at the
+// end of the query data present, q_avail. A match whose right extension was cut there
+// (more of Q follows, R does not end at the same point) is emitted with kOpenBit set in
+// its length and finished by k_open_fix once all of Q is present. Its length is already
+// >= L: its start lies a whole chunk (>= L bases) before q_avail.
+constexpr uint32_t kOpenBit = 0x80000000u;
+__device__ __forceinline__ uint32_t open_bit(const FindParams &P, uint32_t a, uint32_t b, uint32_t f) {
+    return (uint64_t(b) + f == P.q_avail && P.q_avail < P.nQ && uint64_t(a) + f < P.nR) ? kOpenBit : 0u;
+}
+
 // The record-only part of decide(): kDrop / kEmit when the kL + kR flank bases of the
 // record (16 + 32 for 16-byte records, 8 + 8 for 8-byte records) settle the hit, else
 // kExt with e_out = the left extension if the record settled it, or kUnresolved. kExt
@@ -201,7 +211,7 @@ __device__ __forceinline__ int decide_rec(const FindParams &P, uint32_t p, uint3
     const uint32_t qs = q - e;
     if (qs < P.own_lo || qs >= P.own_hi) return kDrop;
     const uint32_t a = p + P.ls, b = q + P.ls;
-    const uint32_t lim_r = min(uint32_t(P.nR) - a, uint32_t(P.nQ) - b);
+    const uint32_t lim_r = min(uint32_t(P.nR) - a, uint32_t(P.q_avail) - b);
     const uint64_t rmask = kR >= 32 ? ~0ull : ~(~0ull >> (2 * kR));  // kR bases, first base highest
     const uint64_t xr = (rright ^ qright) & rmask;
     uint32_t f = xr ? uint32_t(__clzll(xr)) >> 1 : uint32_t(kR);
@@ -214,7 +224,7 @@ __device__ __forceinline__ int decide_rec(const FindParams &P, uint32_t p, uint3
     const uint32_t lam = e + P.ls + f;
     if (lam < P.L) return kDrop;
     out.key = (uint64_t(p - e) << P.qbits) | qs;
-    out.len = lam;
+    out.len = lam | open_bit(P, a, b, f);
     return kEmit;
 }
 
@@ -234,13 +244,13 @@ __device__ __forceinline__ int decide_deferred(const FindParams &P, uint32_t p, 
     const uint32_t qs = q - e;
     if (qs < P.own_lo || qs >= P.own_hi) return kDrop;
     const uint32_t a = p + P.ls, b = q + P.ls;
-    const uint32_t lim_r = min(uint32_t(P.nR) - a, uint32_t(P.nQ) - b);
+    const uint32_t lim_r = min(uint32_t(P.nR) - a, uint32_t(P.q_avail) - b);
     uint32_t f = ext_right(P.R, P.Q, a, b, f0, lim_r, kLaneCap);
     if (f == kUnresolved) return kDefer;
     const uint32_t lam = e + P.ls + f;
     if (lam < P.L) return kDrop;
     out.key = (uint64_t(p - e) << P.qbits) | qs;
-    out.len = lam;
+    out.len = lam | open_bit(P, a, b, f);
     return kEmit;
 }
 
@@ -322,7 +332,7 @@ __device__ __forceinline__ bool resolve_deferred(const FindParams &P, bool valid
     alive = alive && qs >= P.own_lo && qs < P.own_hi;
     // ---- right
     const uint32_t a = p + P.ls, b = q + P.ls;
-    const uint32_t lim_r = alive ? min(uint32_t(P.nR) - a, uint32_t(P.nQ) - b) : 0u;
+    const uint32_t lim_r = alive ? min(uint32_t(P.nR) - a, uint32_t(P.q_avail) - b) : 0u;
     uint32_t f = 0;
     need = false;
     if (alive) {
@@ -349,7 +359,7 @@ __device__ __forceinline__ bool resolve_deferred(const FindParams &P, bool valid
     const uint32_t lam = e + P.ls + f;
     if (!alive || lam < P.L) return false;
     out.key = (uint64_t(p - e) << P.qbits) | qs;
-    out.len = lam;
+    out.len = lam | open_bit(P, a, b, f);
     return true;
 }
 
@@ -741,6 +751,32 @@ __global__ void __launch_bounds__(kT) k_coop(const FindParams P) {
     warp_emit(P, s, nbuf, false, Hit{0, 0}, true);
 }
 
+// Finish the right extension of the matches emitted open (kOpenBit) while Q was still
+// arriving: all of Q is present now. One thread per output slot; open matches are rare
+// (those reaching a chunk end), a long one is walked 32 bases per step.
+__global__ void __launch_bounds__(kT) k_open_fix(uint64_t *__restrict__ keys, uint32_t *__restrict__ lens,
+                                                 const unsigned long long *__restrict__ count, uint64_t cap,
+                                                 const uint64_t *__restrict__ R, uint64_t nR,
+                                                 const uint64_t *__restrict__ Q, uint64_t nQ, uint32_t qbits) {
+    pdl_wait();
+    const unsigned long long c = *count;
+    const uint64_t n = c < cap ? c : cap;
+    for (uint64_t i = uint64_t(blockIdx.x) * kT + threadIdx.x; i < n; i += uint64_t(gridDim.x) * kT) {
+        const uint32_t l0 = lens[i];
+        if (!(l0 & kOpenBit)) continue;
+        const uint64_t k = keys[i];
+        const uint64_t r = k >> qbits, q = k & ((1ull << qbits) - 1);
+        uint64_t f = l0 & ~kOpenBit;
+        const uint64_t lim = min(nR - r, nQ - q);
+        while (f < lim) {
+            const uint32_t run = lead_eq(win_fwd(R, r + f) ^ win_fwd(Q, q + f));
+            f += run;
+            if (run < 32) break;
+        }
+        lens[i] = uint32_t(min(f, lim));
+    }
+}
+
 int g_default_grid = 0;
 
 }  // namespace
@@ -780,6 +816,13 @@ cudaError_t launch_find(const FindParams &p, int grid, cudaStream_t s) {
     else if (p.recs_stream) GM_FIND_LAUNCH(false, true);
     else GM_FIND_LAUNCH(false, false);
 #undef GM_FIND_LAUNCH
+    note_launch();
+    return cudaGetLastError();
+}
+
+cudaError_t launch_open_fix(const FindParams &p, cudaStream_t s) {
+    pdl_launch(k_open_fix, num_sms() * 4, kT, 0, s, p.out_key, p.out_len, static_cast<const unsigned long long *>(p.out_count),
+               p.capacity, p.R, p.nR, p.Q, p.nQ, p.qbits);
     note_launch();
     return cudaGetLastError();
 }

@@ -2,6 +2,7 @@
 // streams, status codes, the overflow-and-retry protocol of find, and stage
 // instrumentation. All compute is in pack.cu / index.cu / radix.cu / find.cu /
 // sort.cu; this file only orchestrates launches.
+#include <algorithm>
 #include <atomic>
 #include <cstdarg>
 #include <cstdio>
@@ -104,6 +105,12 @@ struct CapCtx {
     // the measuring run allocates and sizes them (ws_need), the capture bump-allocates
     // each from the arena at that size, so they live and die with the arena.
     void *ws_priv = nullptr;              // WsSet *
+    // streamed query (host-input pipeline): Q in q_chunks pieces at q_bnd[0..q_chunks]
+    // (multiples of 32); piece j is packed once its copy has arrived and q_packed[j] is
+    // recorded; find over the MEM starts of piece i runs once pieces <= i + 1 are packed
+    int q_chunks = 1;
+    const uint64_t *q_bnd = nullptr;
+    const cudaEvent_t *q_packed = nullptr;
 };
 thread_local CapCtx *t_cap = nullptr;
 thread_local bool t_ws_alloc = false;     // workspace growth: never from the arena
@@ -398,6 +405,7 @@ unsigned long long *pinned_slots() {  // 16 per thread, never freed
 }  // namespace
 
 // ---------------------------------------------------------------- pipeline (CUDA graph)
+constexpr int kMaxQChunks = 16;
 struct gpumem_pipeline {
     uint32_t magic;
     int device;
@@ -427,6 +435,11 @@ struct gpumem_pipeline {
     uint64_t out_cap, coop_cap, spill_cap, span;
     std::vector<StageRec> recs;
     uint64_t launches;                     // kernels per graph launch
+    int q_chunks;                          // host-input runs: Q copied, packed, searched in this many pieces
+    uint64_t q_bnd[kMaxQChunks + 1];       // ... at these boundaries (multiples of 32)
+    int cap_chunks;                        // pieces of the captured graph (1 = whole Q at once)
+    cudaEvent_t ev_qc[kMaxQChunks];        // piece j copied (recorded on `copy`, waited on by the graph)
+    cudaEvent_t ev_pk[kMaxQChunks];        // piece j packed (inside the graph)
     int exportable;                        // arena from cudaMalloc, so its IPC handle can be exported
     uint64_t generation;                   // captures so far (an exported handle is valid for one)
     int ran;
@@ -443,6 +456,32 @@ void pipeline_wait_mark(gpumem_pipeline *pl, cudaStream_t s, int which) {
     if (t_cap && t_cap->recs) cudaStreamWaitEvent(s, which == 1 ? pl->ev_r : pl->ev_q, cudaEventWaitExternal);
 }
 
+// Q in pieces (host-input pipeline, cap_chunks > 1): piece j is packed on stream s once
+// its copy has arrived (external event wait in the graph), into one packed sequence;
+// ev_pk[j] marks it packed for the find launches of gpumem_find_mems.
+gpumem_status pack_q_pieces(gpumem_pipeline *pl, const char *Q, cudaStream_t s, gpumem_seq **out) {
+    *out = nullptr;
+    const uint64_t n = pl->nQ, n_words = (n + 31) / 32 + 4;
+    Scratch sc(s);
+    auto *words = static_cast<uint64_t *>(sc.get(n_words * 8));
+    auto *bad = static_cast<unsigned long long *>(sc.get(8));
+    if (!words || !bad) return GPUMEM_ERR_NOMEM;
+    CK(cudaMemsetAsync(bad, 0xff, 8, s), "memset");
+    const int K = pl->cap_chunks;
+    for (int j = 0; j < K; ++j) {
+        const uint64_t a = pl->q_bnd[j], b = pl->q_bnd[j + 1];
+        if (t_cap && t_cap->recs) CK(cudaStreamWaitEvent(s, pl->ev_qc[j], cudaEventWaitExternal), "wait piece");
+        const uint64_t nw = j + 1 < K ? (b - a) / 32 : n_words - a / 32;
+        Stage stage("pack", s);
+        CK(launch_pack(reinterpret_cast<const uint8_t *>(Q) + a, b - a, words + a / 32, nw, bad, s, a), "pack piece");
+        CK(cudaEventRecord(pl->ev_pk[j], s), "piece packed");
+    }
+    sc.keep(words);
+    sc.keep(bad);
+    *out = new gpumem_seq{kMagicSeq, pl->device, s, n, n_words, words, bad};
+    return GPUMEM_OK;
+}
+
 gpumem_status pipeline_path(gpumem_pipeline *pl, const char *R, const char *Q, gpumem_seq **hR, gpumem_seq **hQ,
                             gpumem_index **hI, gpumem_mems **hM) {
     *hR = *hQ = nullptr;
@@ -453,6 +492,14 @@ gpumem_status pipeline_path(gpumem_pipeline *pl, const char *R, const char *Q, g
     gpumem_status st = GPUMEM_OK;
     if (cudaEventRecord(pl->ev_fork, pl->stream) != cudaSuccess) st = cuda_fail(cudaGetLastError(), "fork");
     if (!st && cudaStreamWaitEvent(pl->side, pl->ev_fork, 0) != cudaSuccess) st = cuda_fail(cudaGetLastError(), "fork");
+    if (pl->cap_chunks > 1) {  // streamed query: pieces packed as they arrive; find joins per piece
+        if (!st) st = pack_q_pieces(pl, Q, pl->side, hQ);
+        if (!st) pipeline_wait_mark(pl, pl->stream, 1);
+        if (!st) st = gpumem_pack(R, pl->nR, 1, pl->stream, hR);
+        if (!st) st = gpumem_index_build(*hR, pl->ls, pl->L, pl->stream, hI);
+        if (!st) st = gpumem_find_mems(*hI, *hQ, pl->q_begin, pl->q_end, pl->stream, hM);
+        return st;
+    }
     if (!st) pipeline_wait_mark(pl, pl->side, 2);
     if (!st) st = gpumem_pack(Q, pl->nQ, 1, pl->side, hQ);
     if (!st && cudaEventRecord(pl->ev_join, pl->side) != cudaSuccess) st = cuda_fail(cudaGetLastError(), "join");
@@ -496,16 +543,20 @@ void pipeline_release(gpumem_pipeline *pl) {  // graph, arena and the arena-back
     cudaGetLastError();
 }
 
-gpumem_status pipeline_capture(gpumem_pipeline *pl, const char *R, const char *Q) {
+gpumem_status pipeline_capture(gpumem_pipeline *pl, const char *R, const char *Q, bool host_inputs) {
     cudaStream_t s = pl->stream;
     CK(cudaStreamSynchronize(s), "sync");
     pipeline_release(pl);
+    pl->cap_chunks = host_inputs ? pl->q_chunks : 1;
     // 1) measuring run: sizes every workspace, sums the handle/scratch bytes
     WsSet mws;
     CapCtx m;
     m.mode = 1;
     m.ws_priv = &mws;
     m.deferred = true;
+    m.q_chunks = pl->cap_chunks;
+    m.q_bnd = pl->q_bnd;
+    m.q_packed = pl->ev_pk;
     m.host = pl->host;
     m.side = pl->side2;
     m.ev_a = pl->ev_ra;
@@ -547,6 +598,9 @@ gpumem_status pipeline_capture(gpumem_pipeline *pl, const char *R, const char *Q
     CapCtx c;
     c.mode = 2;
     c.ws_priv = pl->ws;
+    c.q_chunks = pl->cap_chunks;
+    c.q_bnd = pl->q_bnd;
+    c.q_packed = pl->ev_pk;
     c.arena = pl->arena;
     c.cap = pl->arena_bytes;
     c.deferred = true;
@@ -594,6 +648,7 @@ cudaError_t pipeline_launch(gpumem_pipeline *pl, bool host_inputs) {
     if (!host_inputs) {
         e = cudaEventRecord(pl->ev_r, pl->stream);
         if (e == cudaSuccess) e = cudaEventRecord(pl->ev_q, pl->stream);
+        for (int j = 0; j < pl->cap_chunks && e == cudaSuccess; ++j) e = cudaEventRecord(pl->ev_qc[j], pl->stream);
         if (e != cudaSuccess) return e;
     }
     return cudaGraphLaunch(pl->exec, pl->stream);
@@ -659,6 +714,7 @@ gpumem_status gpumem_set_option(const char *name, int64_t value) {
         g_opt.sort_impl = value;
     }
     else if (!strcmp(name, "pdl")) g_opt.pdl = value ? 1 : 0;
+    else if (!strcmp(name, "q_chunks")) g_opt.q_chunks = value < 1 ? 1 : value;
     else if (!strcmp(name, "pipe_events")) g_opt.pipe_events = value < 0 ? 0 : (value > 2 ? 2 : value);
     else if (!strcmp(name, "index_alg1")) g_opt.index_alg1 = value < 0 ? -1 : (value ? 1 : 0);
     else if (!strcmp(name, "rec8")) g_opt.rec8 = value < 0 ? -1 : (value ? 1 : 0);
@@ -746,6 +802,10 @@ void gpumem_free(void *handle) {
         }
         cudaEventDestroy(pl->ev_r);
         cudaEventDestroy(pl->ev_q);
+        for (int j = 0; j < kMaxQChunks; ++j) {
+            cudaEventDestroy(pl->ev_qc[j]);
+            cudaEventDestroy(pl->ev_pk[j]);
+        }
         cudaEventDestroy(pl->ev_fork);
         cudaEventDestroy(pl->ev_ra);
         cudaEventDestroy(pl->ev_rb);
@@ -1075,6 +1135,7 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
     P.Q = Q->words;
     P.nQ = nQ;
     P.nQw = Q->n_words;
+    P.q_avail = nQ;
     if (!g_opt.use_bitmap) {  // the paper's lookup reads the dense ptrs
         st = index_ptrs(idx, s);
         if (st) return st;
@@ -1112,7 +1173,7 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
     uint64_t cap = g_opt.out_capacity ? uint64_t(g_opt.out_capacity) : (span / 8 + 4096);
 
     Scratch sc(s);
-    auto *ctr = static_cast<unsigned long long *>(ws_get(kWsCtr, 64, s));
+    auto *ctr = static_cast<unsigned long long *>(ws_get(kWsCtr, 256, s));  // [16..]: per-piece tile counters
     const uint64_t spill_cap = span / 8 + 4096;
     auto *spill = static_cast<uint4 *>(ws_get(kWsSpill, spill_cap * sizeof(uint4), s));
     uint64_t coop_cap = span / 64 + 4096;
@@ -1150,15 +1211,38 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
         P.out_len = lens;
         P.capacity = cap;
         P.coop_cap = coop_cap;
-        CK(cudaMemsetAsync(ctr, 0, 64, s), "memset counters");
-        {
+        CK(cudaMemsetAsync(ctr, 0, 256, s), "memset counters");
+        const int K = t_cap->q_chunks > 1 && q_begin == 0 && q_end == nQ ? t_cap->q_chunks : 1;
+        if (K == 1) {
             Stage g("find", s);
             CK(launch_find(P, int(g_opt.find_grid), s), "find kernel");
+        } else {
+            // streamed query: find over the MEM starts of piece i once pieces <= i + 1 are
+            // packed; extensions stop at the data present (q_avail), cut matches are open
+            const uint64_t *B = t_cap->q_bnd;
+            Stage g("find", s);
+            for (int i = 0; i < K && P.n_tiles; ++i) {
+                const int need = i + 1 < K ? i + 1 : K - 1;
+                CK(cudaStreamWaitEvent(s, t_cap->q_packed[need], 0), "wait for query piece");
+                FindParams Pi = P;
+                Pi.q_avail = B[need + 1];
+                Pi.own_lo = B[i];
+                Pi.own_hi = B[i + 1];
+                Pi.scan_lo = B[i];
+                const uint64_t hi = B[i + 1] + step - 1;
+                Pi.scan_hi = hi < nQ - ls + 1 ? hi : nQ - ls + 1;
+                if (Pi.scan_hi < Pi.scan_lo) Pi.scan_hi = Pi.scan_lo;
+                Pi.n_tiles = (Pi.scan_hi - Pi.scan_lo + tile - 1) / tile;
+                Pi.tile_ctr = reinterpret_cast<unsigned int *>(ctr + 16) + i;
+                CK(launch_find(Pi, int(g_opt.find_grid), s), "find kernel");
+            }
+            CK(cudaStreamWaitEvent(s, t_cap->q_packed[K - 1], 0), "join the query pieces");
         }
         if (P.n_tiles) {
             Stage g("find.heavy", s);
             CK(launch_heavy(P, s), "heavy kernel");
             CK(launch_coop(P, s), "coop kernel");
+            if (K > 1) CK(launch_open_fix(P, s), "open-match fix");
         }
         {
             Stage g("sort", s);
@@ -1281,6 +1365,25 @@ gpumem_status gpumem_pipeline_create(uint64_t r_len, uint64_t q_len, uint32_t se
     pl->q_end = q_end;
     pl->ls = seed_len;
     pl->L = min_len;
+    // streamed query for host-input runs (option q_chunks): pieces of >= max(1 MB, 4 L)
+    // bases on 32-base boundaries (a cut match is then already >= L long)
+    {
+        int K = int(g_opt.q_chunks < 1 ? 1 : (g_opt.q_chunks > kMaxQChunks ? kMaxQChunks : g_opt.q_chunks));
+        const uint64_t min_piece = std::max<uint64_t>(uint64_t(1) << 20, 4ull * min_len + 64);
+        while (K > 1 && q_len / uint64_t(K) < min_piece) --K;
+        if (q_begin != 0 || q_end < q_len) K = 1;  // a sharded pipeline keeps the whole-Q path
+        pl->q_chunks = K;
+        for (int j = 0; j <= K; ++j) pl->q_bnd[j] = j == K ? q_len : (q_len * uint64_t(j) / uint64_t(K)) / 32 * 32;
+        pl->cap_chunks = 1;
+        for (int j = 0; j < kMaxQChunks; ++j) {
+            if (cudaEventCreateWithFlags(&pl->ev_qc[j], cudaEventDisableTiming) != cudaSuccess ||
+                cudaEventCreateWithFlags(&pl->ev_pk[j], cudaEventDisableTiming) != cudaSuccess) {
+                cudaGetLastError();
+                gpumem_free(pl);
+                return fail(GPUMEM_ERR_CUDA, "pipeline events");
+            }
+        }
+    }
     if (cudaMallocHost(&pl->host, 16 * sizeof(unsigned long long)) != cudaSuccess) {
         cudaGetLastError();
         delete pl;
@@ -1303,7 +1406,7 @@ gpumem_status gpumem_pipeline_run(gpumem_pipeline *pl, const char *r_bases_dev, 
     CK(cudaEventRecord(pl->ev_in, pl->user), "event");  // inputs written on the caller's stream
     CK(cudaStreamWaitEvent(pl->stream, pl->ev_in, 0), "wait");
     if (!pl->exec || pl->inR != r_bases_dev || pl->inQ != q_bases_dev) {
-        const gpumem_status st = pipeline_capture(pl, r_bases_dev, q_bases_dev);
+        const gpumem_status st = pipeline_capture(pl, r_bases_dev, q_bases_dev, false);
         if (st) return st;
     }
     CK(pipeline_launch(pl, false), "graph launch");
@@ -1338,12 +1441,16 @@ gpumem_status gpumem_pipeline_run_host(gpumem_pipeline *pl, const char *r_bases_
     CK(cudaStreamWaitEvent(pl->copy, pl->ev_out, 0), "wait");
     if (pl->nR) CK(cudaMemcpyAsync(dR, r_bases_host, pl->nR, cudaMemcpyHostToDevice, pl->copy), "H2D R");
     CK(cudaEventRecord(pl->ev_r, pl->copy), "event");
-    if (pl->nQ) CK(cudaMemcpyAsync(dQ, q_bases_host, pl->nQ, cudaMemcpyHostToDevice, pl->copy), "H2D Q");
+    for (int j = 0; j < pl->q_chunks; ++j) {  // Q in pieces, each announced by its event
+        const uint64_t a = pl->q_bnd[j], b = pl->q_bnd[j + 1];
+        if (b > a) CK(cudaMemcpyAsync(dQ + a, q_bases_host + a, b - a, cudaMemcpyHostToDevice, pl->copy), "H2D Q");
+        CK(cudaEventRecord(pl->ev_qc[j], pl->copy), "event");
+    }
     CK(cudaEventRecord(pl->ev_q, pl->copy), "event");
     CK(cudaStreamWaitEvent(pl->stream, pl->ev_in, 0), "wait");
     if (!pl->exec || pl->inR != dR || pl->inQ != dQ) {
         CK(cudaStreamWaitEvent(pl->stream, pl->ev_q, 0), "wait");  // the measuring run reads both
-        const gpumem_status st = pipeline_capture(pl, dR, dQ);
+        const gpumem_status st = pipeline_capture(pl, dR, dQ, true);
         if (st) return st;
     }
     CK(pipeline_launch(pl, true), "graph launch");

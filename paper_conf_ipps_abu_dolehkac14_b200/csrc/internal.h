@@ -37,6 +37,8 @@ struct Options {
                                  // 0 rank words, 1 rank sectors
     int64_t radix_bits = 0;      // LSD digit width: 0 = 9 bits if that saves a pass else 8; or pinned 8, 9, 10
     int64_t pdl = 1;             // programmatic dependent launch between consecutive kernels
+    int64_t q_chunks = 8;        // host-input pipelines: Q copied, packed and searched in this many pieces
+                                 // (read at gpumem_pipeline_create; 1 = the whole Q after its copy)
     int64_t pipe_events = 0;     // stage event nodes in a pipeline graph: 0 none (fastest), 2 find only, 1 every
                                  // stage (each node costs a few us: C4 1.263 / 1.280 / 1.311 ms per step)
     int64_t index_alg1 = 0;      // Alg. 1 literally (atomic counts, scan, placement, bucket sort): 1 always,
@@ -90,9 +92,11 @@ struct Stage {
 };
 
 // ---------------------------------------------------------------- kernels (launchers)
-// K1: ASCII -> 2-bit words (pack.cu). words must hold ceil(n/32) + 2 entries.
+// K1: ASCII -> 2-bit words (pack.cu): in[0, n) into words[0, n_words_alloc) (words past
+// the data zero); an invalid byte at in[i] records pos_base + i (atomicMin) in *bad_pos.
+// A chunk of a longer sequence starting at base 32j: in + 32j, words + j, pos_base 32j.
 cudaError_t launch_pack(const uint8_t *in, uint64_t n, uint64_t *words, uint64_t n_words_alloc,
-                        unsigned long long *bad_pos, cudaStream_t s);
+                        unsigned long long *bad_pos, cudaStream_t s, uint64_t pos_base = 0);
 
 // Reverse complement of packed words (pack.cu).
 cudaError_t launch_revcomp(const uint64_t *in, uint64_t n, uint64_t *out, uint64_t n_words_alloc, cudaStream_t s);
@@ -145,6 +149,7 @@ struct FindParams {
     const uint64_t *Q;
     uint64_t nQ;
     uint64_t nQw;                // allocated words of Q (incl. padding)
+    uint64_t q_avail;            // Q bases present (== nQ unless Q is streamed in chunks)
     const uint32_t *ptrs;
     const void *recs;            // seed records, parallel to locs: uint4 {p, R[p-16,p), R[p+ls,p+ls+32)}, or
     int rec8;                    // (rec8) uint2 {p, R[p-8,p) | R[p+ls,p+ls+8) << 16}
@@ -177,6 +182,7 @@ uint64_t find_tile_positions();
 cudaError_t launch_find(const FindParams &p, int grid, cudaStream_t s);
 cudaError_t launch_heavy(const FindParams &p, cudaStream_t s);
 cudaError_t launch_coop(const FindParams &p, cudaStream_t s);
+cudaError_t launch_open_fix(const FindParams &p, cudaStream_t s);  // after streamed-Q finds
 int find_default_grid();
 
 // Instrumentation (diag.cu): best-of-4 time of n random 8-byte probes into a table of

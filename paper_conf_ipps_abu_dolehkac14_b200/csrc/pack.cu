@@ -26,7 +26,7 @@ __device__ __forceinline__ uint32_t pack4(uint32_t x, bool &ok) {
 
 // word w from 32 ASCII bytes (the scalar path handles unaligned input and the tail)
 __device__ __forceinline__ uint64_t pack_word_scalar(const uint8_t *__restrict__ in, uint64_t n, uint64_t w,
-                                                     unsigned long long *bad_pos) {
+                                                     unsigned long long *bad_pos, uint64_t pos_base) {
     uint64_t word = 0;
     const uint64_t base = w * 32;
     for (int i = 0; i < 32; ++i) {
@@ -35,17 +35,18 @@ __device__ __forceinline__ uint64_t pack_word_scalar(const uint8_t *__restrict__
         const uint32_t ch = in[pos];
         const uint32_t c = ((ch >> 1) ^ (ch >> 2)) & 3u;
         const uint32_t up = ch & 0xDFu;
-        if (up != 'A' && up != 'C' && up != 'G' && up != 'T') atomicMin(bad_pos, (unsigned long long)pos);
+        if (up != 'A' && up != 'C' && up != 'G' && up != 'T') atomicMin(bad_pos, (unsigned long long)(pos_base + pos));
         word |= uint64_t(c) << (62 - 2 * i);
     }
     return word;
 }
 
-__device__ __noinline__ void report_bad(const uint8_t *__restrict__ in, uint64_t w, unsigned long long *bad_pos) {
+__device__ __noinline__ void report_bad(const uint8_t *__restrict__ in, uint64_t w, unsigned long long *bad_pos,
+                                       uint64_t pos_base) {
     for (int i = 0; i < 32; ++i) {  // locate the first bad byte of this word
         const uint32_t up = in[w * 32 + i] & 0xDFu;
         if (up != 'A' && up != 'C' && up != 'G' && up != 'T') {
-            atomicMin(bad_pos, (unsigned long long)(w * 32 + i));
+            atomicMin(bad_pos, (unsigned long long)(pos_base + w * 32 + i));
             break;
         }
     }
@@ -69,7 +70,7 @@ __device__ __forceinline__ uint32_t pack16(const uint4 v, bool &ok) {
 __global__ void __launch_bounds__(kPackThreads) k_pack(const uint8_t *__restrict__ in, uint64_t n,
                                                        uint64_t *__restrict__ words, uint64_t n_full,
                                                        uint64_t n_words_alloc, unsigned long long *bad_pos,
-                                                       int aligned) {
+                                                       int aligned, uint64_t pos_base) {
     pdl_wait();
     const int lane = threadIdx.x & 31;
     if (aligned) {
@@ -88,7 +89,7 @@ __global__ void __launch_bounds__(kPackThreads) k_pack(const uint8_t *__restrict
             const uint32_t half = h < n_halves ? pack16(v[k], ok) : 0u;
             const uint32_t odd = __shfl_down_sync(0xffffffffu, half, 1);
             if (h < n_halves) {
-                if (!ok) report_bad(in, h >> 1, bad_pos);  // the word's first bad byte (either half)
+                if (!ok) report_bad(in, h >> 1, bad_pos, pos_base);  // the word's first bad byte (either half)
                 if (!(lane & 1)) words[h >> 1] = (uint64_t(half) << 32) | odd;
             }
         }
@@ -98,7 +99,7 @@ __global__ void __launch_bounds__(kPackThreads) k_pack(const uint8_t *__restrict
     const uint64_t tail = n_words_alloc - first;
     const uint64_t per_cta = uint64_t(kPackThreads);
     for (uint64_t i = uint64_t(blockIdx.x) * per_cta + threadIdx.x; i < tail; i += uint64_t(gridDim.x) * per_cta)
-        words[first + i] = pack_word_scalar(in, n, first + i, bad_pos);
+        words[first + i] = pack_word_scalar(in, n, first + i, bad_pos, pos_base);
 }
 
 // Reverse complement of a packed sequence (NEXT-F4): rc[i] = 3 - s[n-1-i] (A<->T, C<->G
@@ -141,13 +142,14 @@ cudaError_t launch_revcomp(const uint64_t *in, uint64_t n, uint64_t *out, uint64
 }
 
 cudaError_t launch_pack(const uint8_t *in, uint64_t n, uint64_t *words, uint64_t n_words_alloc,
-                        unsigned long long *bad_pos, cudaStream_t s) {
+                        unsigned long long *bad_pos, cudaStream_t s, uint64_t pos_base) {
     const int aligned = (reinterpret_cast<uintptr_t>(in) & 15) == 0;
     const uint64_t n_full = n / 32;
     const uint64_t per = uint64_t(kPackThreads) * kHPT;  // halves per CTA
     uint64_t blocks = aligned ? (2 * n_full + per - 1) / per : (n_words_alloc + kPackThreads - 1) / kPackThreads;
     if (blocks == 0) blocks = 1;
-    pdl_launch(k_pack, unsigned(blocks), kPackThreads, 0, s, in, n, words, n_full, n_words_alloc, bad_pos, aligned);
+    pdl_launch(k_pack, unsigned(blocks), kPackThreads, 0, s, in, n, words, n_full, n_words_alloc, bad_pos, aligned,
+               pos_base);
     note_launch();
     return cudaGetLastError();
 }

@@ -166,6 +166,48 @@ def test_pipeline_host_inputs():
     pl.free()
 
 
+@pytest.mark.parametrize("chunks", [1, 2, 5, 16])
+@pytest.mark.parametrize("cfg,scale", [("c4", 0.03), ("c5_l20", 0.03), ("c3", 0.1)])
+def test_pipeline_streamed_query(cfg, scale, chunks):
+    """Host-input runs with Q streamed in pieces (option q_chunks): MEMs cut at the data
+    present are finished after the last piece; the set equals the oracle's and the
+    whole-Q (q_chunks = 1) result, relaunch after relaunch."""
+    gpumem.set_option("q_chunks", chunks)
+    try:
+        P = synth.make_pair(cfg, scale=scale)
+        want = oracle.mems(P.R, P.Q, P.L, P.ls)
+        pl = gpumem.Pipeline(len(P.R), len(P.Q), P.ls, P.L)
+        Rh, Qh = torch.from_numpy(P.R).pin_memory(), torch.from_numpy(P.Q).pin_memory()
+        for _ in range(3):
+            pl.run_host(Rh, Qh)
+            assert pl.result() == len(want)
+            assert np.array_equal(pl.numpy(), want)
+            assert pl.stats()["attempts"] == 1
+        pl.free()
+    finally:
+        gpumem.set_option("q_chunks", 8)
+
+
+def test_pipeline_streamed_query_long_matches():
+    """Matches far longer than a piece run through every piece boundary: the self-match
+    of a 5 Mbp sequence (one MEM of 5 Mbp) and poly-A arrays across piece boundaries."""
+    gpumem.set_option("q_chunks", 5)
+    try:
+        rng = np.random.default_rng(11)
+        S = np.frombuffer(b"ACGT", np.uint8)[rng.integers(0, 4, 5_000_000)].copy()
+        for a in (1_000_000 - 3000, 2_000_000 - 17, 3_999_990):  # poly-A runs over piece boundaries
+            S[a:a + 6000] = ord("A")
+        want = oracle.mems(S, S, 50, 13)
+        assert (0, 0, len(S)) in {tuple(t) for t in want.tolist()}
+        pl = gpumem.Pipeline(len(S), len(S), 13, 50)
+        pl.run_host(torch.from_numpy(S).pin_memory(), torch.from_numpy(S).pin_memory())
+        pl.result()
+        assert np.array_equal(pl.numpy(), want)
+        pl.free()
+    finally:
+        gpumem.set_option("q_chunks", 8)
+
+
 @pytest.mark.parametrize("events,want", [(0, set()), (2, {"find"}), (1, {"pack", "index.sort", "find", "sort"})])
 def test_pipeline_event_modes(events, want):
     """pipe_events: no stage events (default), find's only (the timed bench graph), every
