@@ -245,9 +245,9 @@ gpumem_status gpumem_merge_sorted(const gpumem_triple *const *dev_runs, const ui
  *  are copied on a copy stream into pipeline-owned device buffers (allocated on the
  *  first call, through the allocator hook), R first; the graph packs and indexes R while
  *  Q is still in flight. Q crosses PCIe in q_chunks pieces (option "q_chunks", read at
- *  gpumem_pipeline_create; pieces >= max(1 Mbp, 4 L) bases; whole-Q pipelines only):
- *  piece j is packed as soon as it has arrived and the MEMs starting in piece i are
- *  searched once pieces <= i + 1 are present, extensions stopping at the data present;
+ *  gpumem_pipeline_create; pieces >= max(1 Mbp, 8 L) bases; whole-Q pipelines only):
+ *  piece j is packed as soon as it has arrived and searched for the MEMs starting in it
+ *  (shifted back by max(L, step + ls) + 64 bases), extensions stopping at the data present;
  *  the few matches cut there are finished after the last piece. Same
  *  result as gpumem_pipeline_run. Async: the host buffers must stay valid and
  *  unmodified until the run completes (gpumem_pipeline_result).

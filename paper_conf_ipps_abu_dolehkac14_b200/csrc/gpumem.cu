@@ -1173,7 +1173,8 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
     uint64_t cap = g_opt.out_capacity ? uint64_t(g_opt.out_capacity) : (span / 8 + 4096);
 
     Scratch sc(s);
-    auto *ctr = static_cast<unsigned long long *>(ws_get(kWsCtr, 256, s));  // [16..]: per-piece tile counters
+    // [16, 24): per-piece tile counters (u32), [24, 40): per-piece heavy-queue counters
+    auto *ctr = static_cast<unsigned long long *>(ws_get(kWsCtr, 320, s));
     const uint64_t spill_cap = span / 8 + 4096;
     auto *spill = static_cast<uint4 *>(ws_get(kWsSpill, spill_cap * sizeof(uint4), s));
     uint64_t coop_cap = span / 64 + 4096;
@@ -1211,36 +1212,42 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
         P.out_len = lens;
         P.capacity = cap;
         P.coop_cap = coop_cap;
-        CK(cudaMemsetAsync(ctr, 0, 256, s), "memset counters");
+        CK(cudaMemsetAsync(ctr, 0, 320, s), "memset counters");
         const int K = t_cap->q_chunks > 1 && q_begin == 0 && q_end == nQ ? t_cap->q_chunks : 1;
         if (K == 1) {
             Stage g("find", s);
             CK(launch_find(P, int(g_opt.find_grid), s), "find kernel");
         } else {
-            // streamed query: find over the MEM starts of piece i once pieces <= i + 1 are
-            // packed; extensions stop at the data present (q_avail), cut matches are open
+            // streamed query: piece i's search starts once piece i is packed. It owns the MEM
+            // starts [B[i] - X, B[i+1] - X) (X = 0 at the ends of Q), so its seeds (up to
+            // step - 1 bases past a start, ls long) lie in the data present; extensions
+            // stop at q_avail = B[i+1], and a match cut there starts >= X >= L before it
             const uint64_t *B = t_cap->q_bnd;
+            const uint64_t X = std::max<uint64_t>(L, step + ls) + 64;
             Stage g("find", s);
             for (int i = 0; i < K && P.n_tiles; ++i) {
-                const int need = i + 1 < K ? i + 1 : K - 1;
-                CK(cudaStreamWaitEvent(s, t_cap->q_packed[need], 0), "wait for query piece");
+                CK(cudaStreamWaitEvent(s, t_cap->q_packed[i], 0), "wait for query piece");
                 FindParams Pi = P;
-                Pi.q_avail = B[need + 1];
-                Pi.own_lo = B[i];
-                Pi.own_hi = B[i + 1];
-                Pi.scan_lo = B[i];
-                const uint64_t hi = B[i + 1] + step - 1;
+                Pi.q_avail = B[i + 1];
+                Pi.own_lo = i == 0 ? 0 : B[i] - X;
+                Pi.own_hi = i + 1 == K ? nQ : B[i + 1] - X;
+                Pi.scan_lo = Pi.own_lo;
+                const uint64_t hi = Pi.own_hi + step - 1;
                 Pi.scan_hi = hi < nQ - ls + 1 ? hi : nQ - ls + 1;
                 if (Pi.scan_hi < Pi.scan_lo) Pi.scan_hi = Pi.scan_lo;
                 Pi.n_tiles = (Pi.scan_hi - Pi.scan_lo + tile - 1) / tile;
                 Pi.tile_ctr = reinterpret_cast<unsigned int *>(ctr + 16) + i;
+                // the piece's own heavy queue (its counter; the buffer is reused piece after
+                // piece): its hits are decided with the piece's ownership range and data end
+                Pi.spill_count = ctr + 24 + i;
                 CK(launch_find(Pi, int(g_opt.find_grid), s), "find kernel");
+                CK(launch_heavy(Pi, s), "heavy kernel");
             }
             CK(cudaStreamWaitEvent(s, t_cap->q_packed[K - 1], 0), "join the query pieces");
         }
         if (P.n_tiles) {
             Stage g("find.heavy", s);
-            CK(launch_heavy(P, s), "heavy kernel");
+            if (K == 1) CK(launch_heavy(P, s), "heavy kernel");
             CK(launch_coop(P, s), "coop kernel");
             if (K > 1) CK(launch_open_fix(P, s), "open-match fix");
         }
@@ -1365,13 +1372,16 @@ gpumem_status gpumem_pipeline_create(uint64_t r_len, uint64_t q_len, uint32_t se
     pl->q_end = q_end;
     pl->ls = seed_len;
     pl->L = min_len;
-    // streamed query for host-input runs (option q_chunks): pieces of >= max(1 MB, 4 L)
-    // bases on 32-base boundaries (a cut match is then already >= L long)
+    // streamed query for host-input runs (option q_chunks): pieces of >= max(1 Mbp, 8 L)
+    // bases on 32-base boundaries (a piece's search then owns a non-empty start range and
+    // a cut match is already >= L long)
     {
         int K = int(g_opt.q_chunks < 1 ? 1 : (g_opt.q_chunks > kMaxQChunks ? kMaxQChunks : g_opt.q_chunks));
-        const uint64_t min_piece = std::max<uint64_t>(uint64_t(1) << 20, 4ull * min_len + 64);
+        const uint64_t min_piece = std::max<uint64_t>(uint64_t(1) << 20, 8ull * min_len + 256);
         while (K > 1 && q_len / uint64_t(K) < min_piece) --K;
         if (q_begin != 0 || q_end < q_len) K = 1;  // a sharded pipeline keeps the whole-Q path
+        if (min_len - seed_len + 1 > 4000) K = 1;   // left extensions past one lane's reach defer
+                                                    // before their ownership is known
         pl->q_chunks = K;
         for (int j = 0; j <= K; ++j) pl->q_bnd[j] = j == K ? q_len : (q_len * uint64_t(j) / uint64_t(K)) / 32 * 32;
         pl->cap_chunks = 1;

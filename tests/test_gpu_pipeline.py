@@ -166,13 +166,17 @@ def test_pipeline_host_inputs():
     pl.free()
 
 
+@pytest.mark.parametrize("spill", [64, 1])
 @pytest.mark.parametrize("chunks", [1, 2, 5, 16])
 @pytest.mark.parametrize("cfg,scale", [("c4", 0.03), ("c5_l20", 0.03), ("c3", 0.1)])
-def test_pipeline_streamed_query(cfg, scale, chunks):
+def test_pipeline_streamed_query(cfg, scale, chunks, spill):
     """Host-input runs with Q streamed in pieces (option q_chunks): MEMs cut at the data
     present are finished after the last piece; the set equals the oracle's and the
-    whole-Q (q_chunks = 1) result, relaunch after relaunch."""
+    whole-Q (q_chunks = 1) result, relaunch after relaunch. find_spill = 1 sends every
+    hit through the heavy queue, whose pieces must keep their piece's ownership range
+    (seed positions within step of a piece end are scanned by both pieces)."""
     gpumem.set_option("q_chunks", chunks)
+    gpumem.set_option("find_spill", spill)
     try:
         P = synth.make_pair(cfg, scale=scale)
         want = oracle.mems(P.R, P.Q, P.L, P.ls)
@@ -186,6 +190,7 @@ def test_pipeline_streamed_query(cfg, scale, chunks):
         pl.free()
     finally:
         gpumem.set_option("q_chunks", 8)
+        gpumem.set_option("find_spill", 64)
 
 
 def test_pipeline_streamed_query_long_matches():
