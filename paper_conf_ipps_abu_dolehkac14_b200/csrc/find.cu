@@ -504,14 +504,37 @@ __global__ void __launch_bounds__(kT, GM_FIND_MINB) k_find(const FindParams P) {
                     occ[j] = qa + j < P.scan_hi;
                 }
                 if (P.use_bitmap && !kSect) {
-                    // rank-word probe (occupancy bit + rank), then the compact {first, count}
+                    // rank-word probes in pairs (q, q+1): one 16-byte entry of group code(q+1) >> 5
+                    // holds q+1's rank word and the occupancy of the rotated code of q (same
+                    // group, index.cu); q's own rank word only when it is occupied. Then the
+                    // compact {first, count} of each occupied seed.
+                    const uint32_t nbits = 2 * P.ls;
+                    const uint32_t cmask = nbits >= 32 ? 0xffffffffu : ((1u << nbits) - 1u);
                     uint32_t rank[kQPT];
+                    bool own[kQPT];  // rank word of the position's own group still needed
 #pragma unroll
-                    for (int j = 0; j < kQPT; ++j) {
-                        rank[j] = 0;
-                        if (occ[j]) {
-                            const unsigned long long rw = kHints ? ld_last_u64(P.rankw + (code[j] >> 5))
-                                                                      : __ldg(P.rankw + (code[j] >> 5));
+                    for (int j = 0; j < kQPT; j += 2) {
+                        rank[j] = rank[j + 1] = 0;
+                        own[j] = false;
+                        own[j + 1] = false;
+                        if (occ[j + 1]) {  // both positions in range
+                            const uint4 *ep = reinterpret_cast<const uint4 *>(P.rankw + 2 * (code[j + 1] >> 5));
+                            const uint4 e = kHints ? ld_last_u4(ep) : __ldg(ep);
+                            const uint32_t b1 = code[j + 1] & 31;
+                            occ[j + 1] = (e.x >> b1) & 1u;
+                            rank[j + 1] = e.y + __popc(e.x & ((1u << b1) - 1u));
+                            const uint32_t rot = ((code[j] << 2) | (code[j] >> (nbits - 2))) & cmask;
+                            occ[j] = (e.z >> (rot & 31)) & 1u;
+                            own[j] = occ[j];
+                        } else if (occ[j]) {
+                            own[j] = true;
+                        }
+                    }
+#pragma unroll
+                    for (int j = 0; j < kQPT; j += 2) {
+                        if (own[j]) {
+                            const unsigned long long rw = kHints ? ld_last_u64(P.rankw + 2 * (code[j] >> 5))
+                                                                 : __ldg(P.rankw + 2 * (code[j] >> 5));
                             const uint32_t bit = code[j] & 31, bits = uint32_t(rw);
                             occ[j] = (bits >> bit) & 1u;
                             rank[j] = uint32_t(rw >> 32) + __popc(bits & ((1u << bit) - 1u));

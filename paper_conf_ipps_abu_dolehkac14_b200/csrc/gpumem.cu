@@ -42,7 +42,7 @@ struct gpumem_index {
     uint64_t n_locs;
     uint32_t *ptrs;
     uint32_t *locs;
-    unsigned long long *rankw;   // rank words, 8 B per 32 seeds, or
+    unsigned long long *rankw;   // rank words + rotated occupancy, 16 B per 32 seeds (index.cu), or
     uint4 *rsect;                // rank sectors, 16 B per 32 seeds (index.cu); one of the two is null
     uint2 *buckets;
     void *recs;                  // uint4 records, or uint2 when rec8
@@ -714,6 +714,7 @@ gpumem_status gpumem_set_option(const char *name, int64_t value) {
         g_opt.sort_impl = value;
     }
     else if (!strcmp(name, "pdl")) g_opt.pdl = value ? 1 : 0;
+    else if (!strcmp(name, "find_hints")) g_opt.find_hints = value < 0 ? -1 : (value ? 1 : 0);
     else if (!strcmp(name, "q_chunks")) g_opt.q_chunks = value < 1 ? 1 : value;
     else if (!strcmp(name, "pipe_events")) g_opt.pipe_events = value < 0 ? 0 : (value > 2 ? 2 : value);
     else if (!strcmp(name, "index_alg1")) g_opt.index_alg1 = value < 0 ? -1 : (value ? 1 : 0);
@@ -958,7 +959,7 @@ static gpumem_status index_build_impl(const gpumem_seq *R, uint32_t ls, uint32_t
     unsigned long long *rankw = nullptr;
     uint4 *rsect = nullptr;
     if (use_sect) rsect = static_cast<uint4 *>(sc.get(((nb + 31) / 32) * 16));
-    else rankw = static_cast<unsigned long long *>(sc.get(((nb + 31) / 32) * 8));
+    else rankw = static_cast<unsigned long long *>(sc.get(((nb + 31) / 32) * 16));  // + rotated occupancy
     const uint64_t max_occ = (n_locs < nb ? n_locs : nb) + 1;
     auto *buckets = static_cast<uint2 *>(sc.get(max_occ * sizeof(uint2)));
     void *fill_scratch = ws_get(kWsFill, ptrs_fill_scratch_bytes(ls), s);
@@ -1169,6 +1170,7 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
         int l2 = 0;
         cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, dev);
         P.recs_stream = idx->n_locs * (idx->rec8 ? 8 : 16) > uint64_t(l2) / 2 ? 1 : 0;
+        if (g_opt.find_hints >= 0) P.recs_stream = int(g_opt.find_hints);
     }
     uint64_t cap = g_opt.out_capacity ? uint64_t(g_opt.out_capacity) : (span / 8 + 4096);
 

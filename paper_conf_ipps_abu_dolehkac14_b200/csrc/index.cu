@@ -113,6 +113,20 @@ __global__ void __launch_bounds__(1024) k_occ_scan(const uint32_t *__restrict__ 
     }
 }
 
+// Rank-word directory entries are 16 bytes per group g of 32 seeds: word 2g = {occupancy
+// bits, occupied seeds before the group} (the rank word), word 2g+1 = occupancy of the 32
+// seeds whose codes ROTATED left by one base (the first base moved to the end) fall in
+// group g. Rotating code(Q, q) gives the same top bits as code(Q, q+1) (both start with
+// bases q+1 ...), so one 16-byte probe of group code(q+1) >> 5 answers "is the seed at q
+// occupied?" and "at q+1?" -- k_find probes query positions in pairs.
+// The rotated bits are ORed in here (the directory is zeroed first) for every occupied seed.
+__device__ __forceinline__ void set_rot_occ(unsigned long long *rankw, uint32_t code, uint32_t ls) {
+    const uint32_t nbits = 2 * ls;
+    const uint32_t mask = nbits >= 32 ? 0xffffffffu : ((1u << nbits) - 1u);
+    const uint32_t rot = ((code << 2) | (code >> (nbits - 2))) & mask;
+    atomicOr(reinterpret_cast<unsigned int *>(rankw + 2 * (rot >> 5) + 1), 1u << (rot & 31));
+}
+
 // kCounts: `codes` is instead the dense per-seed count array (Alg. 1 step 1 done with
 // atomics by k_alg1_count) and chunk_first the records before each chunk.
 template <bool kSect, bool kCounts = false>
@@ -122,7 +136,7 @@ __global__ void __launch_bounds__(kFillThreads) k_ptrs_fill(const uint32_t *__re
                                                             uint4 *__restrict__ rsect,
                                                             uint2 *__restrict__ buckets,
                                                             const uint32_t *__restrict__ chunk_first,
-                                                            const uint32_t *__restrict__ rank0) {
+                                                            const uint32_t *__restrict__ rank0, uint32_t rot_ls) {
     pdl_wait();
     extern __shared__ uint32_t cnt[];                // kChunk + kChunk / 32: a pad word per 32 (conflict-free rows)
     __shared__ uint32_t wsum[kFillThreads / 32];
@@ -198,12 +212,13 @@ __global__ void __launch_bounds__(kFillThreads) k_ptrs_fill(const uint32_t *__re
         const uint32_t x = cnt[tid * (kPer + 1) + j];
         cnt[tid * (kPer + 1) + j] = pre;
         if (x) buckets[r++] = make_uint2(pre, x);
+        if (!kSect && x) set_rot_occ(rankw, uint32_t(s0) + uint32_t(tid) * kPer + j, rot_ls);
         if (kSect) c2 |= uint64_t(x < 3 ? x : 3u) << (2 * j);
         pre += x;
     }
     if (s0 + uint64_t(tid) * kPer < n_buckets) {
         if (kSect) rsect[(s0 >> 5) + tid] = make_uint4(group_first, uint32_t(rank), uint32_t(c2), uint32_t(c2 >> 32));
-        else rankw[(s0 >> 5) + tid] = (rank << 32) | occ;
+        else rankw[2 * ((s0 >> 5) + tid)] = (rank << 32) | occ;
     }
     __syncthreads();
     // coalesced write-out of the chunk's ptrs, 16 bytes per store (skipped when the dense
@@ -245,7 +260,7 @@ __global__ void __launch_bounds__(kDirThreads) k_dir_fill(const uint32_t *__rest
                                                           unsigned long long *__restrict__ rankw,
                                                           uint4 *__restrict__ rsect, uint2 *__restrict__ buckets,
                                                           const uint32_t *__restrict__ chunk_first,
-                                                          const uint32_t *__restrict__ rank0) {
+                                                          const uint32_t *__restrict__ rank0, uint32_t rot_ls) {
     pdl_wait();
     __shared__ uint32_t occ[kGroups], ecnt[kGroups], c2lo[kGroups], c2hi[kGroups];
     __shared__ uint32_t hpos[kDirThreads + 1];
@@ -272,6 +287,7 @@ __global__ void __launch_bounds__(kDirThreads) k_dir_fill(const uint32_t *__rest
         buckets[r0 + rank] = make_uint2(first, count);
         const uint32_t sd = code - uint32_t(s0), g = sd >> 5, b = sd & 31;
         atomicOr(&occ[g], 1u << b);
+        if (!kSect) set_rot_occ(rankw, code, rot_ls);
         if (kSect) {
             atomicAdd(&ecnt[g], count);
             const uint32_t sat = count < 3 ? count : 3u;
@@ -349,7 +365,7 @@ __global__ void __launch_bounds__(kDirThreads) k_dir_fill(const uint32_t *__rest
     if (s0 + uint64_t(tid) * 32 < n_buckets) {
         const uint64_t g = (s0 >> 5) + tid;
         if (kSect) rsect[g] = make_uint4(lo + pe, r0 + po, c2lo[tid], c2hi[tid]);
-        else rankw[g] = (uint64_t(r0 + po) << 32) | o;
+        else rankw[2 * g] = (uint64_t(r0 + po) << 32) | o;
     }
 }
 
@@ -441,7 +457,7 @@ __global__ void __launch_bounds__(kCodeThreads) k_alg1_place(const uint32_t *__r
             first = __ldg(buckets + rs.y + __popcll((below | (below >> 1)) & kLo)).x;
         }
     } else {
-        const unsigned long long rw = __ldg(rankw + (code >> 5));
+        const unsigned long long rw = __ldg(rankw + 2 * (code >> 5));
         const uint32_t rank = uint32_t(rw >> 32) + __popc(uint32_t(rw) & ((1u << b) - 1u));
         first = __ldg(buckets + rank).x;
     }
@@ -465,7 +481,7 @@ __global__ void __launch_bounds__(kCodeThreads) k_bucket_fix(const uint2 *__rest
         const uint64_t c2 = (uint64_t(rs.w) << 32) | rs.z;
         n_occ = rs.y + __popcll((c2 | (c2 >> 1)) & 0x5555555555555555ull);
     } else {
-        const unsigned long long rw = rankw[g];
+        const unsigned long long rw = rankw[2 * g];
         n_occ = uint32_t(rw >> 32) + __popc(uint32_t(rw));
     }
     for (uint64_t r = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; r < n_occ; r += uint64_t(gridDim.x) * blockDim.x) {
@@ -621,7 +637,7 @@ __global__ void __launch_bounds__(256) k_ptrs_expand(const unsigned long long *_
             in = ((c2 >> (2 * b)) & 3u) != 0;
             return r.y + __popcll((below | (below >> 1)) & kLo);
         }
-        const unsigned long long r = rankw[s >> 5];
+        const unsigned long long r = rankw[2 * (s >> 5)];
         const uint32_t bits = uint32_t(r);
         in = (bits >> b) & 1u;
         return uint32_t(r >> 32) + __popc(bits & ((1u << b) - 1u));
@@ -683,6 +699,7 @@ cudaError_t launch_index_alg1(const uint64_t *R, uint32_t ls, uint32_t step, uin
     auto *big = reinterpret_cast<uint32_t *>(a);  // occupied seeds over kFixMax (<= n_locs / kFixMax)
     cudaError_t e = cudaMemsetAsync(cnt, 0, nb * 4, s);
     if (e == cudaSuccess) e = cudaMemsetAsync(n_big, 0, 4, s);
+    if (e == cudaSuccess && rankw) e = cudaMemsetAsync(rankw, 0, ((nb + 31) / 32) * 16, s);
     if (e != cudaSuccess) return e;
     const unsigned grid_k = unsigned((n_locs + kCodeThreads - 1) / kCodeThreads);
     pdl_launch(k_alg1_count, grid_k, kCodeThreads, 0, s, R, ls, step, k0, n_locs, cnt, codes, arr);
@@ -700,10 +717,10 @@ cudaError_t launch_index_alg1(const uint64_t *R, uint32_t ls, uint32_t step, uin
     }
     if (rsect)
         pdl_launch(k_ptrs_fill<true, true>, unsigned(chunks), kFillThreads, smem, s, cnt, n_locs, nb, (uint32_t *)nullptr,
-                   rankw, rsect, buckets, first, rank0);
+                   rankw, rsect, buckets, first, rank0, ls);
     else
         pdl_launch(k_ptrs_fill<false, true>, unsigned(chunks), kFillThreads, smem, s, cnt, n_locs, nb, (uint32_t *)nullptr,
-                   rankw, rsect, buckets, first, rank0);
+                   rankw, rsect, buckets, first, rank0, ls);
     if (rsect) pdl_launch(k_alg1_place<true>, grid_k, kCodeThreads, 0, s, codes, arr, n_locs, k0, step, rankw, rsect, buckets, locs);
     else pdl_launch(k_alg1_place<false>, grid_k, kCodeThreads, 0, s, codes, arr, n_locs, k0, step, rankw, rsect, buckets, locs);
     pdl_launch(k_bucket_fix, unsigned(num_sms() * 8), kCodeThreads, 0, s, buckets, rankw, rsect, nb, locs, big, n_big);
@@ -731,6 +748,10 @@ cudaError_t launch_ptrs_fill(const uint32_t *sorted_codes, uint64_t n_locs, uint
     a = align(a + (chunks + 1) * 4);
     auto *rank0 = reinterpret_cast<uint32_t *>(a);
     cudaError_t e = cudaSuccess;
+    if (rankw) {  // 16 B per group: rank word + rotated occupancy (ORed in by the fill)
+        e = cudaMemsetAsync(rankw, 0, ((nb + 31) / 32) * 16, s);
+        if (e != cudaSuccess) return e;
+    }
     pdl_launch(k_chunk_bounds, unsigned((n_locs + 1 + kCodeThreads - 1) / kCodeThreads), kCodeThreads, 0, s, 
         sorted_codes, n_locs, chunks, first);
     pdl_launch(k_occ_count, unsigned(chunks), kCodeThreads, 0, s, sorted_codes, first, occ);
@@ -750,16 +771,16 @@ cudaError_t launch_ptrs_fill(const uint32_t *sorted_codes, uint64_t n_locs, uint
     if (!ptrs && n_locs * 4 < nb) {
         if (rsect)
             pdl_launch(k_dir_fill<true>, unsigned(chunks), kDirThreads, 0, s, sorted_codes, nb, rankw, rsect, buckets, first,
-                                                                      rank0);
+                       rank0, ls);
         else
             pdl_launch(k_dir_fill<false>, unsigned(chunks), kDirThreads, 0, s, sorted_codes, nb, rankw, rsect, buckets, first,
-                                                                       rank0);
+                       rank0, ls);
     } else if (rsect) {
         pdl_launch(k_ptrs_fill<true>, unsigned(chunks), kFillThreads, smem, s, sorted_codes, n_locs, nb, ptrs, rankw, rsect,
-                                                                       buckets, first, rank0);
+                   buckets, first, rank0, ls);
     } else {
         pdl_launch(k_ptrs_fill<false>, unsigned(chunks), kFillThreads, smem, s, sorted_codes, n_locs, nb, ptrs, rankw, rsect,
-                                                                        buckets, first, rank0);
+                   buckets, first, rank0, ls);
     }
     note_launch(4);
     return cudaGetLastError();

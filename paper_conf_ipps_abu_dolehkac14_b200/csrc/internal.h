@@ -37,6 +37,7 @@ struct Options {
                                  // 0 rank words, 1 rank sectors
     int64_t radix_bits = 0;      // LSD digit width: 0 = 9 bits if that saves a pass else 8; or pinned 8, 9, 10
     int64_t pdl = 1;             // programmatic dependent launch between consecutive kernels
+    int64_t find_hints = -1;     // k_find L2 cache-policy loads: -1 auto (seed records > L2 / 2), 0 off, 1 on
     int64_t q_chunks = 8;        // host-input pipelines: Q copied, packed and searched in this many pieces
                                  // (read at gpumem_pipeline_create; 1 = the whole Q after its copy)
     int64_t pipe_events = 0;     // stage event nodes in a pipeline graph: 0 none (fastest), 2 find only, 1 every

@@ -51,6 +51,6 @@ for st in settings:
     pl.free()
     for k in opts:
         gm.set_option(k, {"heavy_tail": 1, "pdl": 1, "find_spill": 64, "sort_impl": 0, "radix_bits": 0,
-                          "rank_sectors": -1, "rec8": -1, "find_grid": 0}.get(k, 0))
+                          "rank_sectors": -1, "rec8": -1, "find_grid": 0, "find_hints": -1}.get(k, 0))
     gm.set_option("pipe_events", 0)
 print(json.dumps(out))
