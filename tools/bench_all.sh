@@ -1,3 +1,4 @@
+#!/bin/bash
 # Bench every config on one GPU (bench.py lines -> gpurun_out/bench_<cfg>_<tag>.json): bench_all.sh TAG
 TAG=${1:-x}
 mkdir -p gpurun_out
