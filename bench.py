@@ -389,11 +389,14 @@ def run_ours(args, P):
             # the rank directory, nothing else (gpumem_gather_ceiling), measured here: the
             # practical peak of k_find's access pattern on this GPU
             try:
-                table = (1 << (2 * ls)) // 32 * 8
+                table = (1 << (2 * ls)) // 32 * 16  # the directory: 16 B per group of 32 seeds
                 ceil_ms = gm.gather_ceiling(int(sectors), table)
                 find_ms = kernel_ms[dom] / n_launch
-                roof["note"] = ("at C4 k_find is bound by random 32-B sector requests to L2, not HBM "
-                                "bandwidth: see gather_ceiling (DESIGN.md §7)")
+                dram_gbs = traffic / (find_ms / 1e3) / 1e9 if traffic else 0.0
+                roof["note"] = ("k_find is DRAM-bound here (random seed-record gathers at 64-B DRAM granularity)"
+                                if dram_gbs > 0.4 * peak else
+                                "k_find is bound by random L1->L2 requests and their latency chain (directory "
+                                "probe -> bucket entry -> seed record), not HBM bandwidth (DESIGN.md §7)")
                 roof["gather_ceiling"] = {
                     "what": f"{int(sectors)} random 8-B loads into a {table >> 20} MB table, 8 per thread",
                     "unit": "Gsector/s", "peak": round(sectors / ceil_ms / 1e6, 1),
