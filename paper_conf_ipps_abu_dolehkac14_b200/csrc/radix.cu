@@ -293,15 +293,29 @@ __global__ void __launch_bounds__(kST, GM_RADIX_MINB) k_scatter(const K *__restr
 #pragma unroll
         for (int j = 0; j < kItems; ++j)
             peers[j] = match_digit<RB>(uint32_t(k[j] >> shift) & dmask, wofs + j * 32 + lane < tile_n, bits);
+#ifndef GM_RADIX_ATOMIC_RANK
+#define GM_RADIX_ATOMIC_RANK 1
+#endif
 #pragma unroll
         for (int j = 0; j < kItems; ++j) {
             const bool valid = wofs + j * 32 + lane < tile_n;
             const uint32_t d = uint32_t(k[j] >> shift) & dmask;
+#if GM_RADIX_ATOMIC_RANK
+            // the leader of each digit group reserves the group's slots with one shared
+            // atomicAdd (rounds of one warp issue in program order: ranks stay stable) and
+            // hands the base to its peers
+            const int leader = __ffs(peers[j]) - 1;
+            uint32_t b0 = 0;
+            if (valid && lane == leader) b0 = atomicAdd(&S.wcnt[w][d], uint32_t(__popc(peers[j])));
+            b0 = __shfl_sync(0xffffffffu, b0, valid ? leader : lane);
+            rank[j] = b0 + __popc(peers[j] & lanemask_lt());
+#else
             const uint32_t b0 = valid ? S.wcnt[w][d] : 0u;
             rank[j] = b0 + __popc(peers[j] & lanemask_lt());
             __syncwarp();
             if (valid && lane == __ffs(peers[j]) - 1) S.wcnt[w][d] = b0 + __popc(peers[j]);
             __syncwarp();
+#endif
         }
         __syncthreads();
 
