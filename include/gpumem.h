@@ -207,8 +207,8 @@ gpumem_status gpumem_mems_to_host(const gpumem_mems *m, gpumem_triple *host_buf,
  *  pointers / host counts), each run sorted by (r, q) and no (r, q) in two runs (the
  *  query shards are disjoint by the ownership rule). The runs may be peer memory
  *  mapped with gpumem_ipc_open: the kernel then reads them over NVLink directly, the
- *  gather and the merge in one pass. *out: the union sorted by (r, q) (one read and
- *  one write per triple: bucketed by r, each bucket ranked in shared memory).
+ *  gather and the merge in one pass. *out: the union sorted by (r, q) (a tree of
+ *  two-way merge-path merges: one read and one write per triple per level).
  *  Asynchronous on cuda_stream (the runs must stay valid until it completes).
  *  Errors: n_runs > 64 or a NULL run with a count -> GPUMEM_ERR_ARG; a run of 2^32 or
  *  more triples -> GPUMEM_ERR_RANGE. Runs that are unsorted or overlap give an
