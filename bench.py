@@ -454,6 +454,40 @@ def run_ours(args, P):
                        "steps": args.e2e_steps,
                        "path": "gpumem_pipeline_run_host (pinned host R, Q) + result + D2H of the triples"}
 
+    if not args.no_e2e and world > 1:
+        # every rank: its shard's pipeline from pinned host R and Q (the whole of both: a
+        # shard's extensions read all of Q), the fused gather + merge, and on rank 0 the
+        # D2H of the merged triples; the max over ranks of the mean wall time
+        R_h = torch.from_numpy(P.R).pin_memory()
+        Q_h = torch.from_numpy(P.Q).pin_memory()
+        se = ShardedPipeline(nR, nQ, L, ls)
+        host_out, times, nm = None, [], 0
+        for i in range(args.e2e_steps + 2):
+            flush.zero_()
+            torch.cuda.synchronize()
+            dist.barrier()
+            t = time.perf_counter()
+            se.run_host(R_h, Q_h)
+            nm = se.finish() or 0
+            if rank == 0:
+                if host_out is None or host_out.shape[0] < nm:
+                    host_out = torch.empty((max(nm, 1) * 5 // 4, 3), dtype=torch.uint32, pin_memory=True)
+                if nm:
+                    host_out[:nm].copy_(se.merged.view_u32(), non_blocking=True)
+            torch.cuda.current_stream().synchronize()
+            if i >= 2:
+                times.append(time.perf_counter() - t)
+        te_t = torch.tensor([statistics.mean(times)], dtype=torch.float64, device=dev)
+        dist.all_reduce(te_t, op=dist.ReduceOp.MAX)
+        te = te_t.item()
+        se.free()
+        line["e2e"] = {"value": round(nQ / 1e6 / te, 2), "unit": "Mbp/s", "h2d_bytes_per_step": world * (nR + nQ),
+                       "d2h_bytes_per_step": 12 * nm + 128 * world, "ms_per_step": round(te * 1e3, 3),
+                       "steps": args.e2e_steps,
+                       "path": "per rank: gpumem_pipeline_run_host (pinned host R, Q) of its shard; fused gather + "
+                               "merge on rank 0 (dist.ShardedPipeline); D2H of the merged triples on rank 0; "
+                               "max over ranks"}
+
     # ---- D9 generator diagnostics (input digests, Fig. 6 bucket sizes, hits per position)
     if rank == 0 and not args.no_d9:
         try:

@@ -115,6 +115,13 @@ class ShardedPipeline:
             self.merged = None
         self.pl.run(R_dev, Q_dev)
 
+    def run_host(self, R_host, Q_host):
+        """The same from (pinned) host memory: the copies overlap the R half of the graph."""
+        if self.merged is not None:
+            self.merged.free()
+            self.merged = None
+        self.pl.run_host(R_host, Q_host)
+
     def _remap(self):
         """(Re)exchange the IPC handles of every rank whose capture generation changed
         (first step, or a recapture on new input pointers)."""
