@@ -249,10 +249,15 @@ def run_ours(args, P):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
-    torch.cuda.set_device(local)
+    # NCCL, one rank per GPU. GM_BENCH_BACKEND=gloo with GM_BENCH_SAME_DEVICE=1 runs the
+    # N > 1 code path with every rank on cuda:0 (tests/test_gpu_bench.py: one GPU box)
+    backend = os.environ.get("GM_BENCH_BACKEND", "nccl")
+    gpu = 0 if os.environ.get("GM_BENCH_SAME_DEVICE") == "1" else local
+    torch.cuda.set_device(gpu)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    dev = torch.device("cuda", local)
+        dist.init_process_group(backend, device_id=torch.device("cuda", gpu) if backend == "nccl" else None)
+    dev = torch.device("cuda", gpu)
+    red_dev = dev if backend == "nccl" else torch.device("cpu")  # where the max-over-ranks reductions run
     stream = torch.cuda.current_stream()
 
     # inputs resident in HBM before timing
@@ -283,7 +288,7 @@ def run_ours(args, P):
     torch.cuda.synchronize()
     l0 = gm.launch_count()
     host_ms = []
-    with ClockSampler(local) as clk:
+    with ClockSampler(gpu) as clk:
         for i in range(args.steps):
             flush.zero_()
             ev[i][0].record(stream)
@@ -310,7 +315,7 @@ def run_ours(args, P):
     if world > 1:
         dist.barrier()
     step_ms = [a.elapsed_time(b) for a, b in ev]
-    tot = torch.tensor([sum(step_ms)], dtype=torch.float64, device=dev)
+    tot = torch.tensor([sum(step_ms)], dtype=torch.float64, device=red_dev)
     if world > 1:
         dist.all_reduce(tot, op=dist.ReduceOp.MAX)
     ms = tot.item() / args.steps
@@ -477,7 +482,7 @@ def run_ours(args, P):
             torch.cuda.current_stream().synchronize()
             if i >= 2:
                 times.append(time.perf_counter() - t)
-        te_t = torch.tensor([statistics.mean(times)], dtype=torch.float64, device=dev)
+        te_t = torch.tensor([statistics.mean(times)], dtype=torch.float64, device=red_dev)
         dist.all_reduce(te_t, op=dist.ReduceOp.MAX)
         te = te_t.item()
         se.free()
