@@ -69,14 +69,18 @@ constexpr uint32_t kLaneCap = 4096;       // bases one lane extends before the w
 
 constexpr int kDQ = 64;                   // deferred-extension queue entries per warp
 
-struct WarpSmem {
+// per-warp shared memory for chunks of kC query positions (k_heavy / k_coop use only the
+// deferred queue and the output buffer: kC = 32 keeps their footprint small, and shared
+// memory the find path does not need is L1 its record and window loads rely on)
+template <int kC>
+struct WarpSmemT {
     uint4 dq[kDQ];                        // {p, q, e (or kUnresolved), known right}: hits needing global extension
-    uint64_t qw[kQW];
-    uint32_t e_beg[kChunk];
-    uint32_t e_off[kChunk + 1];
+    uint64_t qw[kC / 32 + 6];
+    uint32_t e_beg[kC];
+    uint32_t e_off[kC + 1];
     uint64_t okey[kOutBuf];
     uint32_t olen[kOutBuf];
-    uint8_t e_q[kChunk];
+    uint8_t e_q[kC];
 };
 
 // staged Q: word i of the smem copy is Q word (wbase + i)
@@ -373,6 +377,7 @@ __device__ __forceinline__ void push_coop(const FindParams &P, int &verdict, uin
 }
 
 // A10: warp-aggregated append into the warp's buffer; flush when >= 32 are pending.
+template <class WarpSmem>
 __device__ __forceinline__ void warp_emit(const FindParams &P, WarpSmem &s, uint32_t &nbuf, bool emit,
                                           const Hit &h, bool force_flush) {
     const int lane = threadIdx.x & 31;
@@ -421,7 +426,7 @@ __device__ __forceinline__ void load_rec(const FindParams &P, uint64_t k, uint32
 }
 
 // One converged extension round: the last `take` (<= 32) queued hits, one per lane.
-template <int kL>
+template <int kL, class WarpSmem>
 __device__ __forceinline__ void drain_deferred(const FindParams &P, WarpSmem &s, uint32_t &nq, uint32_t &nbuf,
                                                uint32_t take) {
     const int lane = threadIdx.x & 31;
@@ -443,9 +448,29 @@ __device__ __forceinline__ void drain_deferred(const FindParams &P, WarpSmem &s,
 #ifndef GM_FIND_MINB
 #define GM_FIND_MINB 4
 #endif
+#ifndef GM_FIND_MINB_SECT
+#define GM_FIND_MINB_SECT 6
+#endif
+#ifndef GM_FIND_QPT_SECT
+#define GM_FIND_QPT_SECT 4
+#endif
+// Rank-sector indexes (large: C5 at L = 20, 50) run 4 positions per lane and 6 CTAs per SM
+// (their find is DRAM-bound: more warps in flight, C5 L = 20 2.66 -> 2.53 ms); rank-word
+// indexes 8 positions per lane and 4 CTAs per SM (probe pairs; C4 0.78 vs 0.81 ms).
+template <bool kSect>
+struct FindShape {
+    static constexpr int kQPT = kSect ? GM_FIND_QPT_SECT : GM_FIND_QPT;
+    static constexpr int kChunk = 32 * kQPT;
+    static constexpr int kQW = kChunk / 32 + 6;
+    static constexpr int kMinB = kSect ? GM_FIND_MINB_SECT : GM_FIND_MINB;
+};
+static_assert(FindShape<true>::kChunk <= 256 && FindShape<false>::kChunk <= 256, "e_q holds 8-bit slots");
+
 template <bool kStatic, bool kHints, bool kSect, bool kRec8>
-__global__ void __launch_bounds__(kT, GM_FIND_MINB) k_find(const FindParams P) {
+__global__ void __launch_bounds__(kT, FindShape<kSect>::kMinB) k_find(const FindParams P) {
     pdl_wait();
+    constexpr int kQPT = FindShape<kSect>::kQPT, kChunk = FindShape<kSect>::kChunk, kQW = FindShape<kSect>::kQW;
+    using WarpSmem = WarpSmemT<kChunk>;
     constexpr int kL = kRec8 ? 8 : 16, kR = kRec8 ? 8 : 32;  // record flank widths (bases)
     __shared__ WarpSmem smem[kWarps];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
@@ -723,9 +748,9 @@ template <bool kRec8>
 __global__ void __launch_bounds__(kT) k_heavy(const FindParams P) {
     pdl_wait();
     constexpr int kL = kRec8 ? 8 : 16, kR = kRec8 ? 8 : 32;
-    __shared__ WarpSmem smem[kWarps];
+    __shared__ WarpSmemT<32> smem[kWarps];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    WarpSmem &s = smem[wid];
+    WarpSmemT<32> &s = smem[wid];
     uint32_t nbuf = 0;
     const unsigned long long sc = *P.spill_count;
     const unsigned long long n = sc < P.spill_cap ? sc : P.spill_cap;
@@ -755,9 +780,9 @@ __global__ void __launch_bounds__(kT) k_heavy(const FindParams P) {
 // with per-lane extension up to kLaneCap and warp-cooperative extension beyond.
 __global__ void __launch_bounds__(kT) k_coop(const FindParams P) {
     pdl_wait();
-    __shared__ WarpSmem smem[kWarps];
+    __shared__ WarpSmemT<32> smem[kWarps];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    WarpSmem &s = smem[wid];
+    WarpSmemT<32> &s = smem[wid];
     uint32_t nbuf = 0;
     const unsigned long long cc = *P.coop_count;
     const unsigned long long n = cc < P.coop_cap ? cc : P.coop_cap;
@@ -800,25 +825,27 @@ __global__ void __launch_bounds__(kT) k_open_fix(uint64_t *__restrict__ keys, ui
     }
 }
 
-int g_default_grid = 0;
+int g_default_grid[2] = {0, 0};
 
 }  // namespace
 
-uint64_t find_tile_positions() { return kChunk; }
+uint64_t find_tile_positions(bool sect) { return sect ? FindShape<true>::kChunk : FindShape<false>::kChunk; }
 
-int find_default_grid() {
-    if (!g_default_grid) {
+int find_default_grid(bool sect) {
+    int &g = g_default_grid[sect ? 1 : 0];
+    if (!g) {
         int per_sm = 0;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_find<false, false, false, false>, kT, 0);
+        if (sect) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_find<false, false, true, false>, kT, 0);
+        else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_find<false, false, false, false>, kT, 0);
         if (per_sm < 1) per_sm = 1;
-        g_default_grid = per_sm * num_sms();
+        g = per_sm * num_sms();
     }
-    return g_default_grid;
+    return g;
 }
 
 cudaError_t launch_find(const FindParams &p, int grid, cudaStream_t s) {
     if (p.n_tiles == 0) return cudaSuccess;
-    if (grid <= 0) grid = find_default_grid();
+    if (grid <= 0) grid = find_default_grid(p.rsect != nullptr);
     const uint64_t max_useful = (p.n_tiles + kGrab - 1) / kGrab;
     if (uint64_t(grid) * kWarps > max_useful) grid = int((max_useful + kWarps - 1) / kWarps);
     if (grid < 1) grid = 1;

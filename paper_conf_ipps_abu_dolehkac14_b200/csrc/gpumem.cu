@@ -1161,7 +1161,7 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
         if (P.scan_hi < P.scan_lo) P.scan_hi = P.scan_lo;
     }
     const uint64_t span = P.scan_hi - P.scan_lo;
-    const uint64_t tile = find_tile_positions();
+    const uint64_t tile = find_tile_positions(idx->rsect != nullptr);
     P.n_tiles = (span + tile - 1) / tile;
     P.spill_t = uint32_t(g_opt.find_spill);
     P.use_bitmap = int(g_opt.use_bitmap);

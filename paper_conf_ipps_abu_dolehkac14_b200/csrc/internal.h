@@ -179,12 +179,12 @@ struct FindParams {
     int static_lb;               // ablation: no hit redistribution across lanes
     int recs_stream;             // seed records too large to stay in L2: load them evict_first
 };
-uint64_t find_tile_positions();
+uint64_t find_tile_positions(bool rank_sectors);  // query positions per scheduler chunk
 cudaError_t launch_find(const FindParams &p, int grid, cudaStream_t s);
 cudaError_t launch_heavy(const FindParams &p, cudaStream_t s);
 cudaError_t launch_coop(const FindParams &p, cudaStream_t s);
 cudaError_t launch_open_fix(const FindParams &p, cudaStream_t s);  // after streamed-Q finds
-int find_default_grid();
+int find_default_grid(bool rank_sectors);
 
 // Instrumentation (diag.cu): best-of-4 time of n random 8-byte probes into a table of
 // table_bytes (rounded down to a power of two), 8 independent probes per thread.
