@@ -69,9 +69,8 @@ constexpr uint32_t kLaneCap = 4096;       // bases one lane extends before the w
 
 constexpr int kDQ = 64;                   // deferred-extension queue entries per warp
 
-// per-warp shared memory for chunks of kC query positions (k_heavy / k_coop use only the
-// deferred queue and the output buffer: kC = 32 keeps their footprint small, and shared
-// memory the find path does not need is L1 its record and window loads rely on)
+// per-warp shared memory of k_find for chunks of kC query positions (sized to the chunk:
+// shared memory the kernel does not need is L1 its record and window loads rely on)
 template <int kC>
 struct WarpSmemT {
     uint4 dq[kDQ];                        // {p, q, e (or kUnresolved), known right}: hits needing global extension
@@ -81,6 +80,12 @@ struct WarpSmemT {
     uint64_t okey[kOutBuf];
     uint32_t olen[kOutBuf];
     uint8_t e_q[kC];
+};
+
+// k_heavy / k_coop: only the output buffer of warp_emit
+struct EmitSmem {
+    uint64_t okey[kOutBuf];
+    uint32_t olen[kOutBuf];
 };
 
 // staged Q: word i of the smem copy is Q word (wbase + i)
@@ -748,9 +753,9 @@ template <bool kRec8>
 __global__ void __launch_bounds__(kT) k_heavy(const FindParams P) {
     pdl_wait();
     constexpr int kL = kRec8 ? 8 : 16, kR = kRec8 ? 8 : 32;
-    __shared__ WarpSmemT<32> smem[kWarps];
+    __shared__ EmitSmem smem[kWarps];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    WarpSmemT<32> &s = smem[wid];
+    EmitSmem &s = smem[wid];
     uint32_t nbuf = 0;
     const unsigned long long sc = *P.spill_count;
     const unsigned long long n = sc < P.spill_cap ? sc : P.spill_cap;
@@ -780,9 +785,9 @@ __global__ void __launch_bounds__(kT) k_heavy(const FindParams P) {
 // with per-lane extension up to kLaneCap and warp-cooperative extension beyond.
 __global__ void __launch_bounds__(kT) k_coop(const FindParams P) {
     pdl_wait();
-    __shared__ WarpSmemT<32> smem[kWarps];
+    __shared__ EmitSmem smem[kWarps];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    WarpSmemT<32> &s = smem[wid];
+    EmitSmem &s = smem[wid];
     uint32_t nbuf = 0;
     const unsigned long long cc = *P.coop_count;
     const unsigned long long n = cc < P.coop_cap ? cc : P.coop_cap;
