@@ -761,8 +761,10 @@ __global__ void __launch_bounds__(kT) k_heavy(const FindParams P) {
     const unsigned long long n = sc < P.spill_cap ? sc : P.spill_cap;
     const unsigned long long gw = (unsigned long long)blockIdx.x * kWarps + wid;
     const unsigned long long nw = (unsigned long long)gridDim.x * kWarps;
+    uint4 next = gw < n ? P.spill[gw] : make_uint4(0u, 0u, 0u, 0u);
     for (unsigned long long c = gw; c < n; c += nw) {
-        const uint4 piece = P.spill[c];
+        const uint4 piece = next;
+        if (c + nw < n) next = P.spill[c + nw];  // the warp's next piece, in flight meanwhile
         int verdict = kDrop;
         Hit out{0, 0};
         uint32_t p = 0;
