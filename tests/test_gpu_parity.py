@@ -436,6 +436,44 @@ def test_full_size_shards_byte_identical(c4_full, L):
         assert got.tobytes() == whole.tobytes(), G
 
 
+@pytest.mark.slow
+@pytest.mark.parametrize("L,band", [(100, 64_000_000), (20, 16_000_000)])
+def test_full_size_band_sweep(c4_full, L, band):
+    """F2 at the full C4 / C5 L = 20 size: the row sweep over a host-resident R with a
+    16-64 Mbp window equals the whole-R pipeline result (itself bit-exact against the
+    oracle in test_full_size_c4_c5)."""
+    P = c4_full
+    Rt, Qt = torch.from_numpy(P.R).cuda(), torch.from_numpy(P.Q).cuda()
+    pl = gpumem.Pipeline(len(P.R), len(P.Q), P.ls, L)
+    pl.run(Rt, Qt)
+    pl.result()
+    whole = pl.numpy()
+    pl.free()
+    m, st = gpumem.find_mems_banded(P.R, gpumem.pack(Qt), P.ls, L, band)
+    assert st["bands"] > 1 and st["window_bytes"] < len(P.R) // 3
+    assert m.numpy().tobytes() == whole.tobytes()
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("L", [100, 20])
+def test_full_size_streamed_query(c4_full, L):
+    """The host-input pipeline with Q streamed in 8 pieces at the full C4 / C5 L = 20 size
+    equals the device-input pipeline byte for byte."""
+    P = c4_full
+    Rt, Qt = torch.from_numpy(P.R).cuda(), torch.from_numpy(P.Q).cuda()
+    pl = gpumem.Pipeline(len(P.R), len(P.Q), P.ls, L)
+    pl.run(Rt, Qt)
+    pl.result()
+    whole = pl.numpy()
+    pl.free()
+    pl = gpumem.Pipeline(len(P.R), len(P.Q), P.ls, L)
+    for _ in range(2):
+        pl.run_host(torch.from_numpy(P.R).pin_memory(), torch.from_numpy(P.Q).pin_memory())
+        pl.result()
+        assert pl.numpy().tobytes() == whole.tobytes()
+    pl.free()
+
+
 # ------------------------------------------------------------------ NEXT rows (SURVEY.md §8(f))
 def _rc(b):
     return bytes(b)[::-1].translate(bytes.maketrans(b"ACGTacgt", b"TGCAtgca"))
