@@ -1695,10 +1695,46 @@ gpumem_status gpumem_find_mems_banded(const char *r_bases_host, uint64_t r_len, 
         max_w = max(max_w, min(b1 + halo, r_len) - w0);
     }
     Scratch sc(s);
-    char *dwin = static_cast<char *>(sc.get(max_w ? max_w : 1));
+    // two window buffers: the next band's window crosses PCIe on a copy stream while the
+    // current band is searched (double buffering; full overlap needs pinned host memory)
+    char *dwin[2] = {static_cast<char *>(sc.get(max_w ? max_w : 1)), static_cast<char *>(sc.get(max_w ? max_w : 1))};
     auto *ctr = static_cast<unsigned long long *>(sc.get(64));
     unsigned long long *h = pinned_slots();
-    if (!dwin || !ctr || !h) return GPUMEM_ERR_NOMEM;
+    if (!dwin[0] || !dwin[1] || !ctr || !h) return GPUMEM_ERR_NOMEM;
+    struct CopyLane {  // copy stream + "window copied" / "window consumed" events, released on exit
+        cudaStream_t cs = nullptr;
+        cudaEvent_t copied[2] = {nullptr, nullptr}, freed[2] = {nullptr, nullptr};
+        bool ok = true;
+        CopyLane() {
+            ok = cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking) == cudaSuccess;
+            for (int i = 0; i < 2 && ok; ++i)
+                ok = cudaEventCreateWithFlags(&copied[i], cudaEventDisableTiming) == cudaSuccess &&
+                     cudaEventCreateWithFlags(&freed[i], cudaEventDisableTiming) == cudaSuccess;
+        }
+        ~CopyLane() {
+            if (cs) cudaStreamSynchronize(cs);
+            for (int i = 0; i < 2; ++i) {
+                if (copied[i]) cudaEventDestroy(copied[i]);
+                if (freed[i]) cudaEventDestroy(freed[i]);
+            }
+            if (cs) cudaStreamDestroy(cs);
+        }
+    } lane;
+    if (!lane.ok) return cuda_fail(cudaGetLastError(), "band copy stream");
+    auto window = [&](uint64_t b0, uint64_t &w0, uint64_t &w1) {
+        const uint64_t b1 = min(b0 + band_len, r_len);
+        w0 = b0 >= step ? b0 - step : 0;
+        w1 = min(b1 + halo, r_len);
+    };
+    auto issue_copy = [&](uint64_t b0, int buf, bool wait_free) -> cudaError_t {
+        uint64_t w0, w1;
+        window(b0, w0, w1);
+        cudaError_t e = wait_free ? cudaStreamWaitEvent(lane.cs, lane.freed[buf], 0) : cudaSuccess;
+        if (e == cudaSuccess) e = cudaMemcpyAsync(dwin[buf], r_bases_host + w0, w1 - w0, cudaMemcpyHostToDevice, lane.cs);
+        if (e == cudaSuccess) e = cudaEventRecord(lane.copied[buf], lane.cs);
+        return e;
+    };
+    if (r_len && issue_copy(0, 0, false) != cudaSuccess) return cuda_fail(cudaGetLastError(), "H2D band window");
     std::vector<std::pair<gpumem_triple *, uint64_t>> chunks;  // closed MEMs per band (global r)
     gpumem_triple *open = nullptr;
     uint64_t n_open = 0, bands = 0, carried = 0;
@@ -1713,14 +1749,19 @@ gpumem_status gpumem_find_mems_banded(const char *r_bases_host, uint64_t r_len, 
         const uint64_t w0 = b0 >= step ? b0 - step : 0, w1 = min(b1 + halo, r_len), wlen = w1 - w0;
         const int more = w1 < r_len ? 1 : 0;
         Stage g("band", s);
-        if (cudaMemcpyAsync(dwin, r_bases_host + w0, wlen, cudaMemcpyHostToDevice, s) != cudaSuccess) {
+        const int buf = int(bands & 1);
+        cudaError_t ce = cudaSuccess;
+        if (b0 + band_len < r_len) ce = issue_copy(b0 + band_len, buf ^ 1, bands >= 1);  // the next window
+        if (ce == cudaSuccess) ce = cudaStreamWaitEvent(s, lane.copied[buf], 0);
+        if (ce != cudaSuccess) {
             release();
-            return cuda_fail(cudaGetLastError(), "H2D band window");
+            return cuda_fail(ce, "H2D band window");
         }
         gpumem_seq *W = nullptr;
         gpumem_index *idx = nullptr;
         gpumem_mems *m = nullptr;
-        st = gpumem_pack(dwin, wlen, 1, s, &W);
+        st = gpumem_pack(dwin[buf], wlen, 1, s, &W);
+        if (!st && cudaEventRecord(lane.freed[buf], s) != cudaSuccess) st = cuda_fail(cudaGetLastError(), "event");
         if (!st) st = gpumem_index_build_range(W, seed_len, min_len, b0 - w0, b1 - w0, s, &idx);
         if (!st) st = gpumem_find_mems(idx, Q, 0, UINT64_MAX, s, &m);
         const uint64_t cap = (m ? m->count : 0) + n_open;
