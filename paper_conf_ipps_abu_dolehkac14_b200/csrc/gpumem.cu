@@ -1380,12 +1380,17 @@ gpumem_status gpumem_pipeline_create(uint64_t r_len, uint64_t q_len, uint32_t se
     {
         int K = int(g_opt.q_chunks < 1 ? 1 : (g_opt.q_chunks > kMaxQChunks ? kMaxQChunks : g_opt.q_chunks));
         const uint64_t min_piece = std::max<uint64_t>(uint64_t(1) << 20, 8ull * min_len + 256);
-        while (K > 1 && q_len / uint64_t(K) < min_piece) --K;
+        while (K > 1 && q_len / uint64_t(K) < 2 * min_piece) --K;
         if (q_begin != 0 || q_end < q_len) K = 1;  // a sharded pipeline keeps the whole-Q path
         if (min_len - seed_len + 1 > 4000) K = 1;   // left extensions past one lane's reach defer
                                                     // before their ownership is known
         pl->q_chunks = K;
-        for (int j = 0; j <= K; ++j) pl->q_bnd[j] = j == K ? q_len : (q_len * uint64_t(j) / uint64_t(K)) / 32 * 32;
+        // the last piece small (its search is the part of the run after the copy): the
+        // first K-1 pieces share the rest evenly
+        const uint64_t last = K > 1 ? std::max<uint64_t>(min_piece, q_len / 32) : q_len;
+        const uint64_t head = q_len - last;
+        for (int j = 0; j < K; ++j) pl->q_bnd[j] = K > 1 ? (head * uint64_t(j) / uint64_t(K - 1)) / 32 * 32 : 0;
+        pl->q_bnd[K] = q_len;
         pl->cap_chunks = 1;
         for (int j = 0; j < kMaxQChunks; ++j) {
             if (cudaEventCreateWithFlags(&pl->ev_qc[j], cudaEventDisableTiming) != cudaSuccess ||
