@@ -13,7 +13,7 @@
 
 #include "internal.h"
 
-#define GPUMEM_VERSION "0.1.0"
+#define GPUMEM_VERSION "0.2.0"
 
 // output sort: the MSD bucket sort up to this many MEMs, the LSD radix sort beyond
 // (measured in the pipeline: MSD 0.115 vs LSD 0.173 ms at 0.81 M keys (C4), 0.50 vs 0.31 ms
