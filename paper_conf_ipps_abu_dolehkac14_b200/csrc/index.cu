@@ -41,16 +41,33 @@ constexpr int kFillThreads = 512;
 constexpr int kChunk = 16384;                   // buckets per CTA in k_ptrs_fill
 constexpr int kPer = kChunk / kFillThreads;     // 32 consecutive buckets per thread
 
+// four consecutive sampled locations per thread (16-byte stores), grid-stride: one
+// thread per location left the GPU block-scheduling-bound (C5 L = 20: 31 M locations)
 __global__ void __launch_bounds__(kCodeThreads) k_seed_codes(const uint64_t *__restrict__ R, uint32_t ls,
                                                              uint32_t step, uint64_t k0, uint64_t n_locs,
                                                              uint32_t *__restrict__ codes,
                                                              uint32_t *__restrict__ locs) {
     pdl_wait();
-    const uint64_t k = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
-    if (k >= n_locs) return;
-    const uint64_t p = (k0 + k) * step;
-    codes[k] = uint32_t(win_fwd(R, p) >> (64 - 2 * ls));
-    locs[k] = uint32_t(p);
+    const uint32_t sh = 64 - 2 * ls;
+    const uint64_t n4 = (n_locs + 3) / 4;
+    for (uint64_t g = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; g < n4; g += uint64_t(gridDim.x) * blockDim.x) {
+        const uint64_t k = 4 * g;
+        uint32_t c[4], p[4];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            p[j] = uint32_t((k0 + k + j) * step);
+            c[j] = k + j < n_locs ? uint32_t(win_fwd(R, p[j]) >> sh) : 0u;
+        }
+        if (k + 4 <= n_locs) {
+            reinterpret_cast<uint4 *>(codes)[g] = make_uint4(c[0], c[1], c[2], c[3]);
+            reinterpret_cast<uint4 *>(locs)[g] = make_uint4(p[0], p[1], p[2], p[3]);
+        } else {
+            for (int j = 0; j < 4 && k + j < n_locs; ++j) {
+                codes[k + j] = c[j];
+                locs[k + j] = p[j];
+            }
+        }
+    }
 }
 
 // chunk_first[c] = first index i of the sorted codes with codes[i] >= c * kChunk, for
@@ -58,11 +75,19 @@ __global__ void __launch_bounds__(kCodeThreads) k_seed_codes(const uint64_t *__r
 __global__ void __launch_bounds__(kCodeThreads) k_chunk_bounds(const uint32_t *__restrict__ codes, uint64_t n,
                                                                uint64_t n_chunks, uint32_t *__restrict__ first) {
     pdl_wait();
-    const uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
-    if (i > n) return;
-    const uint64_t c_prev = i == 0 ? 0 : uint64_t(codes[i - 1]) / kChunk + 1;  // chunks after codes[i-1]'s
-    const uint64_t c_this = i == n ? n_chunks : uint64_t(codes[i]) / kChunk;    // ... up to codes[i]'s
-    for (uint64_t c = (i == 0 ? 0 : c_prev); c <= c_this && c <= n_chunks; ++c) first[c] = uint32_t(i);
+    // element i in [0, n]: four per thread, grid-stride
+    for (uint64_t g = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; 4 * g <= n;
+         g += uint64_t(gridDim.x) * blockDim.x) {
+        const uint64_t i0 = 4 * g;
+        uint32_t prev = i0 ? codes[i0 - 1] : 0u;
+        for (uint64_t i = i0; i < i0 + 4 && i <= n; ++i) {
+            const uint32_t cur = i < n ? codes[i] : 0u;
+            const uint64_t c_prev = i == 0 ? 0 : uint64_t(prev) / kChunk + 1;  // chunks after codes[i-1]'s
+            const uint64_t c_this = i == n ? n_chunks : uint64_t(cur) / kChunk;  // ... up to codes[i]'s
+            for (uint64_t c = (i == 0 ? 0 : c_prev); c <= c_this && c <= n_chunks; ++c) first[c] = uint32_t(i);
+            prev = cur;
+        }
+    }
 }
 
 // occ[c] = number of distinct codes in chunk c (one CTA per chunk, block reduction of
@@ -611,7 +636,8 @@ cudaError_t launch_seed_recs(const uint64_t *R, uint32_t ls, const uint32_t *loc
 cudaError_t launch_seed_codes(const uint64_t *R, uint32_t ls, uint32_t step, uint64_t k0, uint64_t n_locs,
                               uint32_t *codes, uint32_t *locs, cudaStream_t s) {
     if (n_locs == 0) return cudaSuccess;
-    const uint64_t blocks = (n_locs + kCodeThreads - 1) / kCodeThreads;
+    uint64_t blocks = ((n_locs + 3) / 4 + kCodeThreads - 1) / kCodeThreads;
+    if (blocks > uint64_t(num_sms()) * 16) blocks = uint64_t(num_sms()) * 16;
     pdl_launch(k_seed_codes, unsigned(blocks), kCodeThreads, 0, s, R, ls, step, k0, n_locs, codes, locs);
     note_launch();
     return cudaGetLastError();
@@ -752,8 +778,9 @@ cudaError_t launch_ptrs_fill(const uint32_t *sorted_codes, uint64_t n_locs, uint
         e = cudaMemsetAsync(rankw, 0, ((nb + 31) / 32) * 16, s);
         if (e != cudaSuccess) return e;
     }
-    pdl_launch(k_chunk_bounds, unsigned((n_locs + 1 + kCodeThreads - 1) / kCodeThreads), kCodeThreads, 0, s, 
-        sorted_codes, n_locs, chunks, first);
+    uint64_t bblocks = ((n_locs + 1 + 3) / 4 + kCodeThreads - 1) / kCodeThreads;
+    if (bblocks > uint64_t(num_sms()) * 16) bblocks = uint64_t(num_sms()) * 16;
+    pdl_launch(k_chunk_bounds, unsigned(bblocks), kCodeThreads, 0, s, sorted_codes, n_locs, chunks, first);
     pdl_launch(k_occ_count, unsigned(chunks), kCodeThreads, 0, s, sorted_codes, first, occ);
     pdl_launch(k_occ_scan, 1, 1024, 0, s, occ, uint32_t(chunks), rank0);
     constexpr int smem = (kChunk + kChunk / 32) * 4;
