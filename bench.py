@@ -422,7 +422,14 @@ def run_ours(args, P):
             "stage_ms": {k: round(v, 4) for k, v in sorted(stage_ms_all.items())},
             "stage_ms_note": "separate 5-step run with an event node at every stage boundary (not the timed region)",
             "find_ms_live": round(kernel_ms.get("find", 0.0), 4),
-            "stage_hbm_frac": stage_frac, "stage_hbm_frac_d7": stage_frac_d7, "find_stats": stats, "gpu_launches": int(launches),
+            "stage_hbm_frac": stage_frac, "stage_hbm_frac_d7": stage_frac_d7, "find_stats": stats,
+            "work_balance": {  # the tile scheduler's balance
+                "what": "hits dealt by the busiest warp of k_find vs the mean over its warps (heavy-queue hits, "
+                        "drained by k_heavy, are not a warp's own)",
+                "max_warp_hits": stats.get("max_warp_hits"), "warps": stats.get("warps"),
+                "max_over_mean": round(stats["max_warp_hits"] * stats["warps"] / max(1, stats["hits"]), 3)
+                if stats.get("warps") else None},
+            "gpu_launches": int(launches),
             "clocks": clk.summary(), "roofline": roof,
             "host_ms_per_step": round(statistics.mean(host_ms), 4), "capacity_fallbacks": fallbacks,
             "launch_mode": "one CUDA graph per step (gpumem_pipeline_run)",

@@ -171,6 +171,8 @@ typedef struct {
     uint64_t spilled_chunks; /* heavy-bucket chunks drained by the heavy kernel               */
     uint64_t mems;           /* MEMs reported                                                */
     uint32_t attempts;       /* 1, or 2 after an output-capacity overflow                     */
+    uint64_t max_warp_hits;  /* D5 balance: the most hits one warp of the search dealt itself  */
+    uint64_t warps;          /* ... over this many warps (mean = (hits - spilled hits) / warps) */
 } gpumem_find_stats;
 gpumem_status gpumem_mems_stats(const gpumem_mems *m, gpumem_find_stats *out);
 

@@ -746,6 +746,10 @@ __global__ void __launch_bounds__(kT, FindShape<kSect>::kMinB) k_find(const Find
         atomicAdd(&P.stats[0], st_e);
         atomicAdd(&P.stats[1], st_h);
     }
+    if (lane == 0 && P.work) {  // D5: the tile scheduler's balance -- the busiest warp's hits
+        atomicMax(P.work, st_h);
+        atomicAdd(P.work + 1, 1ull);
+    }
 }
 
 // K7: drain the heavy-bucket queue, one 32-hit piece per warp iteration.

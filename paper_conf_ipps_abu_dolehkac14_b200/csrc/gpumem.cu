@@ -1186,6 +1186,7 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
     P.tile_ctr = reinterpret_cast<unsigned int *>(ctr + 2);
     P.stats = ctr + 3;
     P.coop_count = ctr + 7;
+    P.work = ctr + 8;  // [8] max hits per warp, [9] warps
     P.spill = spill;
     P.spill_cap = spill_cap;
     unsigned long long *h = pinned_slots();
@@ -1266,6 +1267,7 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
             }
         }
         CK(cudaMemcpyAsync(t_cap->host, ctr, 64, cudaMemcpyDeviceToHost, s), "D2H counters");
+        CK(cudaMemcpyAsync(t_cap->host + 10, ctr + 8, 16, cudaMemcpyDeviceToHost, s), "D2H balance");
         CK(cudaMemcpyAsync(t_cap->host + 8, R->bad, 8, cudaMemcpyDeviceToHost, s), "D2H flag");
         CK(cudaMemcpyAsync(t_cap->host + 9, Q->bad, 8, cudaMemcpyDeviceToHost, s), "D2H flag");
         sc.keep(trip);
@@ -1292,7 +1294,7 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
         P.coopq = static_cast<uint2 *>(ws_get(kWsCoop, coop_cap * sizeof(uint2), s));
         P.coop_cap = coop_cap;
         if (!P.coopq) return GPUMEM_ERR_NOMEM;
-        CK(cudaMemsetAsync(ctr, 0, 64, s), "memset counters");
+        CK(cudaMemsetAsync(ctr, 0, 128, s), "memset counters");
         {
             Stage g("find", s);
             CK(launch_find(P, int(g_opt.find_grid), s), "find kernel");
@@ -1304,6 +1306,7 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
         }
         ++attempts;
         CK(cudaMemcpyAsync(h, ctr, 64, cudaMemcpyDeviceToHost, s), "D2H counters");
+        CK(cudaMemcpyAsync(h + 10, ctr + 8, 16, cudaMemcpyDeviceToHost, s), "D2H balance");
         CK(cudaMemcpyAsync(h + 8, R->bad, 8, cudaMemcpyDeviceToHost, s), "D2H flag");
         CK(cudaMemcpyAsync(h + 9, Q->bad, 8, cudaMemcpyDeviceToHost, s), "D2H flag");
         CK(cudaStreamSynchronize(s), "find sync");
@@ -1325,6 +1328,8 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
     fs.hits = h[4] + h[5];
     fs.spilled_chunks = h[1] < spill_cap ? h[1] : spill_cap;
     fs.attempts = uint32_t(attempts);
+    fs.max_warp_hits = h[10];
+    fs.warps = h[11];
     const uint32_t key_bits = bits_for(nR) + P.qbits;
     const gpumem_status st2 = sort_into_triples(keys, lens, count, key_bits, P.qbits, dev, s, out);
     if (st2 == GPUMEM_OK) {
@@ -1491,6 +1496,8 @@ gpumem_status gpumem_pipeline_result(gpumem_pipeline *pl, const gpumem_triple **
     fs.hits = h[4] + h[5];
     fs.spilled_chunks = h[1] < pl->spill_cap ? h[1] : pl->spill_cap;
     fs.attempts = 1;
+    fs.max_warp_hits = h[10];
+    fs.warps = h[11];
     const gpumem_mems *res = pl->mems;
     uint64_t n = h[0];
     if (!pl->fallback && (h[0] > pl->out_cap || h[7] > pl->coop_cap)) {

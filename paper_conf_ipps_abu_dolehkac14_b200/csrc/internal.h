@@ -178,6 +178,7 @@ struct FindParams {
     int use_bitmap;
     int static_lb;               // ablation: no hit redistribution across lanes
     int recs_stream;             // seed records too large to stay in L2: load them evict_first
+    unsigned long long *work;    // [0] most hits one warp dealt locally, [1] warps (D5 balance)
 };
 uint64_t find_tile_positions(bool rank_sectors);  // query positions per scheduler chunk
 cudaError_t launch_find(const FindParams &p, int grid, cudaStream_t s);

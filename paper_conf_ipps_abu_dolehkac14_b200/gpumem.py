@@ -87,7 +87,7 @@ STATUS = {0: "OK", 1: "ERR_ARG", 2: "ERR_ALPHABET", 3: "ERR_RANGE", 4: "ERR_NOME
 
 class FindStats(ctypes.Structure):
     _fields_ = [("positions", _c_u64), ("occupied", _c_u64), ("hits", _c_u64), ("spilled_chunks", _c_u64),
-                ("mems", _c_u64), ("attempts", _c_u32)]
+                ("mems", _c_u64), ("attempts", _c_u32), ("max_warp_hits", _c_u64), ("warps", _c_u64)]
 
     def as_dict(self):
         return {k: int(getattr(self, k)) for k, _ in self._fields_}
