@@ -378,6 +378,14 @@ gpumem_status gpumem_set_allocator(void *(*alloc_fn)(size_t bytes, void *cuda_st
  *                     (default 8; 1 = search after the whole Q has arrived); read at create
  *  "radix_bits"       LSD digit width: 0 (default) = 9 bits when that saves a pass, else 8;
  *                     or pinned to 8, 9, 10; anything else is GPUMEM_ERR_ARG
+ *  "l2_persist"       MB of L2 set aside for persisting lines (device-wide
+ *                     cudaLimitPersistingL2CacheSize, clamped to the device maximum);
+ *                     0 (default) none. Not a stream operation: set outside capture
+ *  "l2_window"        access-policy window of k_find / k_heavy (with l2_persist > 0):
+ *                     0 (default) none, 1 the lookup directory, 2 the compact table,
+ *                     3 the seed records; hit ratio = set-aside / window bytes.
+ *                     Measured no gain (profiles/r2_l2_persist.json), kept as the probe
+ *                     of SURVEY.md §7's persisting-window suggestion
  * Unknown names are GPUMEM_ERR_ARG. */
 gpumem_status gpumem_set_option(const char *name, int64_t value);
 

@@ -860,6 +860,7 @@ cudaError_t launch_find(const FindParams &p, int grid, cudaStream_t s) {
     const uint64_t max_useful = (p.n_tiles + kGrab - 1) / kGrab;
     if (uint64_t(grid) * kWarps > max_useful) grid = int((max_useful + kWarps - 1) / kWarps);
     if (grid < 1) grid = 1;
+    g_l2win = p.l2win;
     // kHints: the seed records exceed half of L2 -> cache-policy loads (lookup tables
     // evict_last, streams evict_first); otherwise plain loads (measured faster there)
     const bool sect = p.rsect != nullptr;
@@ -877,6 +878,7 @@ cudaError_t launch_find(const FindParams &p, int grid, cudaStream_t s) {
     else if (p.recs_stream) GM_FIND_LAUNCH(false, true);
     else GM_FIND_LAUNCH(false, false);
 #undef GM_FIND_LAUNCH
+    g_l2win = cudaAccessPolicyWindow{};
     note_launch();
     return cudaGetLastError();
 }
@@ -895,8 +897,10 @@ cudaError_t launch_coop(const FindParams &p, cudaStream_t s) {
 }
 
 cudaError_t launch_heavy(const FindParams &p, cudaStream_t s) {
+    g_l2win = p.l2win;
     if (p.rec8) pdl_launch(k_heavy<true>, num_sms() * GM_HEAVY_CTAS, kT, 0, s, p);
     else pdl_launch(k_heavy<false>, num_sms() * GM_HEAVY_CTAS, kT, 0, s, p);
+    g_l2win = cudaAccessPolicyWindow{};
     note_launch();
     return cudaGetLastError();
 }

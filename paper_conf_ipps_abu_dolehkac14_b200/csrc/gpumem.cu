@@ -61,6 +61,7 @@ struct gpumem_mems {
 namespace gm {
 
 Options g_opt;
+thread_local cudaAccessPolicyWindow g_l2win = {};
 
 namespace {
 thread_local std::string t_err;
@@ -720,6 +721,21 @@ gpumem_status gpumem_set_option(const char *name, int64_t value) {
     else if (!strcmp(name, "index_alg1")) g_opt.index_alg1 = value < 0 ? -1 : (value ? 1 : 0);
     else if (!strcmp(name, "rec8")) g_opt.rec8 = value < 0 ? -1 : (value ? 1 : 0);
     else if (!strcmp(name, "rank_sectors")) g_opt.rank_sectors = value < 0 ? -1 : (value ? 1 : 0);
+    else if (!strcmp(name, "l2_window")) {
+        if (value < 0 || value > 3) return fail(GPUMEM_ERR_ARG, "l2_window must be 0..3");
+        g_opt.l2_window = value;
+    }
+    else if (!strcmp(name, "l2_persist")) {  // MB of persisting L2 (device-wide limit), clamped to the maximum
+        int dev = 0, mx = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&mx, cudaDevAttrMaxPersistingL2CacheSize, dev);
+        uint64_t b = value < 0 ? 0 : uint64_t(value) << 20;
+        if (b > uint64_t(mx)) b = uint64_t(mx);
+        const cudaError_t e = cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, size_t(b));
+        if (e != cudaSuccess) return cuda_fail(e, "persisting L2 limit");
+        if (!b) cudaCtxResetPersistingL2Cache();
+        g_opt.l2_persist = int64_t(b >> 20);
+    }
     else if (!strcmp(name, "radix_bits")) {
         if (value != 0 && (value < 8 || value > 10)) return fail(GPUMEM_ERR_ARG, "radix_bits must be 0 or 8..10");
         g_opt.radix_bits = value;
@@ -1171,6 +1187,33 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
         cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, dev);
         P.recs_stream = idx->n_locs * (idx->rec8 ? 8 : 16) > uint64_t(l2) / 2 ? 1 : 0;
         if (g_opt.find_hints >= 0) P.recs_stream = int(g_opt.find_hints);
+        // optional persisting-L2 window over one lookup structure (l2_window / l2_persist)
+        if (g_opt.l2_window && g_opt.l2_persist) {
+            const uint64_t groups = ((1ull << (2 * ls)) + 31) / 32;
+            void *base = nullptr;
+            uint64_t bytes = 0;
+            if (g_opt.l2_window == 1) {
+                base = idx->rsect ? static_cast<void *>(idx->rsect) : static_cast<void *>(idx->rankw);
+                bytes = groups * 16;
+            } else if (g_opt.l2_window == 2) {
+                base = idx->buckets;
+                bytes = idx->n_locs * sizeof(uint2);
+            } else {
+                base = idx->recs;
+                bytes = idx->n_locs * (idx->rec8 ? 8 : 16);
+            }
+            int wmax = 0;
+            cudaDeviceGetAttribute(&wmax, cudaDevAttrMaxAccessPolicyWindowSize, dev);
+            if (bytes > uint64_t(wmax)) bytes = uint64_t(wmax);
+            if (base && bytes) {
+                const double set_aside = double(g_opt.l2_persist) * (1 << 20);
+                P.l2win.base_ptr = base;
+                P.l2win.num_bytes = size_t(bytes);
+                P.l2win.hitRatio = float(set_aside >= double(bytes) ? 1.0 : set_aside / double(bytes));
+                P.l2win.hitProp = cudaAccessPropertyPersisting;
+                P.l2win.missProp = cudaAccessPropertyStreaming;
+            }
+        }
     }
     uint64_t cap = g_opt.out_capacity ? uint64_t(g_opt.out_capacity) : (span / 8 + 4096);
 

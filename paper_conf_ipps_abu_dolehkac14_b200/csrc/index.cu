@@ -587,14 +587,10 @@ __global__ void __launch_bounds__(1024) k_bucket_big(const uint2 *__restrict__ b
 // sector, so the find kernel decides a random seed hit without gathering R. With
 // step <= 8 the left extension never passes 8 bases, and 8-byte records {p, R[p-8, p)
 // | R[p+ls, p+ls+8) << 16} halve the record traffic of the (then numerous) hits.
+// the record of location p = locs[k] (16-byte or 8-byte layout, see above)
 template <bool kRec8>
-__global__ void __launch_bounds__(kCodeThreads) k_seed_recs(const uint64_t *__restrict__ R, uint32_t ls,
-                                                            const uint32_t *__restrict__ locs, uint64_t n_locs,
-                                                            void *__restrict__ recs) {
-    pdl_wait();
-    const uint64_t k = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
-    if (k >= n_locs) return;
-    const uint32_t p = locs[k];
+__device__ __forceinline__ void seed_rec(const uint64_t *__restrict__ R, uint32_t ls, uint32_t p, void *recs,
+                                         uint64_t k) {
     uint32_t left;
     uint64_t right;
     if (kRec8 && p >= 8) {  // bases [p - 8, p + ls + 8) (<= 31 bases) lie in the 2 words from (p - 8) / 32
@@ -621,12 +617,36 @@ __global__ void __launch_bounds__(kCodeThreads) k_seed_recs(const uint64_t *__re
     else static_cast<uint4 *>(recs)[k] = make_uint4(p, left, uint32_t(right), uint32_t(right >> 32));
 }
 
+// kRecsPT records per thread (their R gathers in flight together), grid-stride
+constexpr int kRecsPT = 4;
+template <bool kRec8>
+__global__ void __launch_bounds__(kCodeThreads) k_seed_recs(const uint64_t *__restrict__ R, uint32_t ls,
+                                                            const uint32_t *__restrict__ locs, uint64_t n_locs,
+                                                            void *__restrict__ recs) {
+    pdl_wait();
+    const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
+    for (uint64_t k0 = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; k0 < n_locs; k0 += stride * kRecsPT) {
+        uint32_t p[kRecsPT];
+#pragma unroll
+        for (int j = 0; j < kRecsPT; ++j) {
+            const uint64_t k = k0 + uint64_t(j) * stride;
+            p[j] = k < n_locs ? locs[k] : 0u;
+        }
+#pragma unroll
+        for (int j = 0; j < kRecsPT; ++j) {
+            const uint64_t k = k0 + uint64_t(j) * stride;
+            if (k < n_locs) seed_rec<kRec8>(R, ls, p[j], recs, k);
+        }
+    }
+}
+
 }  // namespace
 
 cudaError_t launch_seed_recs(const uint64_t *R, uint32_t ls, const uint32_t *locs, uint64_t n_locs, void *recs,
                              int rec8, cudaStream_t s) {
     if (n_locs == 0) return cudaSuccess;
-    const uint64_t blocks = (n_locs + kCodeThreads - 1) / kCodeThreads;
+    uint64_t blocks = (n_locs + kCodeThreads * kRecsPT - 1) / (kCodeThreads * kRecsPT);
+    if (blocks > uint64_t(num_sms()) * 16) blocks = uint64_t(num_sms()) * 16;
     if (rec8) pdl_launch(k_seed_recs<true>, unsigned(blocks), kCodeThreads, 0, s, R, ls, locs, n_locs, recs);
     else pdl_launch(k_seed_recs<false>, unsigned(blocks), kCodeThreads, 0, s, R, ls, locs, n_locs, recs);
     note_launch();

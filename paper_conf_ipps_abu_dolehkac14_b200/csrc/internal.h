@@ -45,8 +45,15 @@ struct Options {
     int64_t index_alg1 = 0;      // Alg. 1 literally (atomic counts, scan, placement, bucket sort): 1 always,
                                  // -1 for dense indexes (n_locs >= 4^ls / 4), 0 never (default: measured
                                  // slower everywhere -- C5 L = 20 2.9 vs 1.4 ms, C4 0.40 vs 0.21 ms)
+    int64_t l2_persist = 0;      // MB of L2 set aside for persisting lines (cudaLimitPersistingL2CacheSize);
+                                 // 0 = none (default)
+    int64_t l2_window = 0;       // k_find / k_heavy access-policy window over: 0 nothing, 1 the lookup
+                                 // directory, 2 the compact table, 3 the seed records (hit ratio = set-aside
+                                 // / window bytes)
 };
 extern Options g_opt;
+// L2 access-policy window of the launches being issued (num_bytes == 0: none)
+extern thread_local cudaAccessPolicyWindow g_l2win;
 
 // Kernel launch with programmatic dependent launch (PDL): the next kernel on the stream
 // may be scheduled while this one drains (its CTAs fill the SMs freed by finished
@@ -62,11 +69,16 @@ inline cudaError_t pdl_launch(void (*kernel)(KArgs...), dim3 grid, dim3 block, s
     cfg.blockDim = block;
     cfg.dynamicSmemBytes = smem;
     cfg.stream = s;
-    cudaLaunchAttribute attr[1];
+    cudaLaunchAttribute attr[2];
     attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
     attr[0].val.programmaticStreamSerializationAllowed = g_opt.pdl ? 1 : 0;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
+    if (g_l2win.num_bytes) {  // set around the find launches only (launch_find / launch_heavy)
+        attr[1].id = cudaLaunchAttributeAccessPolicyWindow;
+        attr[1].val.accessPolicyWindow = g_l2win;
+        cfg.numAttrs = 2;
+    }
     return cudaLaunchKernelEx(&cfg, kernel, std::forward<Args>(args)...);
 }
 #ifdef __CUDACC__
@@ -179,6 +191,7 @@ struct FindParams {
     int static_lb;               // ablation: no hit redistribution across lanes
     int recs_stream;             // seed records too large to stay in L2: load them evict_first
     unsigned long long *work;    // [0] most hits one warp dealt locally, [1] warps (D5 balance)
+    cudaAccessPolicyWindow l2win;  // persisting-L2 window of k_find / k_heavy (num_bytes 0: none)
 };
 uint64_t find_tile_positions(bool rank_sectors);  // query positions per scheduler chunk
 cudaError_t launch_find(const FindParams &p, int grid, cudaStream_t s);

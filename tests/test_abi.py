@@ -86,5 +86,7 @@ def test_errors_without_gpu_are_clean(lib_path):
     assert lib.gpumem_set_option(b"find_spill", 64) == 0
     assert lib.gpumem_set_option(b"radix_bits", 7) == 1 and lib.gpumem_set_option(b"radix_bits", 11) == 1
     assert lib.gpumem_set_option(b"radix_bits", 0) == 0
+    assert lib.gpumem_set_option(b"l2_window", 4) == 1 and lib.gpumem_set_option(b"l2_window", -1) == 1
+    assert lib.gpumem_set_option(b"l2_window", 0) == 0
     lib.gpumem_free(None)
     assert gpumem.version()

@@ -262,6 +262,23 @@ def test_overflow_retry_grid_spill_and_bitmap_invariance():
                                 "radix_bits": 0, "pdl": 1, "index_alg1": 0}[opt])
 
 
+def test_l2_persisting_window_invariance():
+    """The persisting-L2 access-policy window (options l2_persist / l2_window) changes
+    only cache placement: every window choice, partial hit ratios and the reset are exact."""
+    P = synth.make_pair("c1")
+    want = oracle.mems(P.R, P.Q, P.L, P.ls)
+    try:
+        for persist, window in ((32, 1), (1, 1), (8, 2), (64, 3), (0, 1)):
+            gpumem.set_option("l2_persist", persist)
+            gpumem.set_option("l2_window", window)
+            for sect in (0, 1):
+                gpumem.set_option("rank_sectors", sect)
+                assert np.array_equal(gpu_mems(P.R, P.Q, P.L, P.ls), want), (persist, window, sect)
+    finally:
+        gpumem.set_option("l2_window", 0)
+        gpumem.set_option("l2_persist", 0)
+
+
 def test_seed_length_and_step_invariance():
     P = synth.make_pair("c1", scale=0.5)
     want = oracle.mems(P.R, P.Q, 20, 10)
