@@ -1,5 +1,3 @@
 mkdir -p gpurun_out
-for c in c4 c3 c5_l300 c5_l50; do
-timeout 600 python tools/ab.py $c pdl=1 l2_persist=8,l2_window=1 l2_persist=16,l2_window=1 l2_persist=24,l2_window=1 l2_persist=32,l2_window=1 l2_persist=48,l2_window=1 pdl=1 > gpurun_out/l2_$c.json 2>gpurun_out/l2_$c.err; python -c "
-import json,sys; d=json.load(open('gpurun_out/l2_$c.json')); print(d.pop('config'), {k:(v['ms'],v['find_ms'],v['identical']) for k,v in d.items()})"; tail -2 gpurun_out/l2_$c.err
-done
+timeout 600 ncu --set full --clock-control none --import-source on --profile-from-start off -k regex:k_scatter -s 1 -c 1 -o gpurun_out/prof_scat32 python tools/prof_step.py c5_l20 > gpurun_out/p1.log 2>&1; tail -2 gpurun_out/p1.log
+timeout 600 ncu --set full --clock-control none --import-source on --profile-from-start off -k regex:k_scatter -s 5 -c 1 -o gpurun_out/prof_scat64 python tools/prof_step.py c5_l20 > gpurun_out/p2.log 2>&1; tail -2 gpurun_out/p2.log
