@@ -226,12 +226,83 @@ __device__ __forceinline__ unsigned match8(uint32_t d, bool valid) {
     return peers;
 }
 
+// One stable LSD pass in shared memory over the 8-bit digit at `sh`: buffer cur -> cur ^ 1
+// (stable ranks from per-warp digit counters + ballot peers). Rows of 32 slots wholly past
+// m are skipped warp-uniformly (a segment rarely fills the CTA's kLocal slots).
+__device__ __forceinline__ void smem_pass(LocalSmem &S, uint32_t m, int sh, int &cur) {
+    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+    const uint32_t wofs = uint32_t(w) * 32 * kItems;  // warp w owns slots [wofs, wofs + 32 kItems)
+#pragma unroll
+    for (int ww = 0; ww < kLWarps; ++ww) S.wcnt[ww][tid & 255] = 0;
+    __syncthreads();
+    uint64_t k[kItems];
+    uint32_t v[kItems], rank[kItems];
+    unsigned peers[kItems];
+#pragma unroll
+    for (int j = 0; j < kItems; ++j) {
+        const uint32_t i = wofs + j * 32 + lane;
+        const bool valid = i < m;
+        k[j] = valid ? S.k[cur][i] : 0ull;
+        v[j] = valid ? S.v[cur][i] : 0u;
+        peers[j] = wofs + j * 32 < m ? match8(uint32_t(k[j] >> sh) & 255u, valid) : 0u;
+    }
+#pragma unroll
+    for (int j = 0; j < kItems; ++j) {
+        if (wofs + j * 32 >= m) break;  // warp-uniform
+        const bool valid = wofs + j * 32 + lane < m;
+        const uint32_t d = uint32_t(k[j] >> sh) & 255u;
+        const uint32_t b0 = valid ? S.wcnt[w][d] : 0u;
+        rank[j] = b0 + __popc(peers[j] & lanemask_lt());
+        __syncwarp();
+        if (valid && lane == __ffs(peers[j]) - 1) S.wcnt[w][d] = b0 + __popc(peers[j]);
+        __syncwarp();
+    }
+    __syncthreads();
+    // digit-major, warp-minor exclusive offsets (thread tid < 256 owns digit tid)
+    uint32_t xw[kLWarps], c = 0;
+    if (tid < 256) {
+#pragma unroll
+        for (int ww = 0; ww < kLWarps; ++ww) {
+            xw[ww] = S.wcnt[ww][tid];
+            c += xw[ww];
+        }
+    }
+    uint32_t inc = c;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
+        if (lane >= o) inc += y;
+    }
+    if (lane == 31) S.ws[w] = inc;
+    __syncthreads();
+    if (tid < 256) {
+        uint32_t run = inc - c;
+        for (int i = 0; i < w; ++i) run += S.ws[i];
+#pragma unroll
+        for (int ww = 0; ww < kLWarps; ++ww) {
+            S.wcnt[ww][tid] = run;
+            run += xw[ww];
+        }
+    }
+    __syncthreads();
+#pragma unroll
+    for (int j = 0; j < kItems; ++j) {
+        if (wofs + j * 32 + lane < m) {
+            const uint32_t pos = S.wcnt[w][uint32_t(k[j] >> sh) & 255u] + rank[j];
+            S.k[cur ^ 1][pos] = k[j];
+            S.v[cur ^ 1][pos] = v[j];
+        }
+    }
+    cur ^= 1;
+    __syncthreads();
+}
+
 // Sorts the m <= kLocal keys (with values) of [tk + lo, tk + lo + m) by their low `bits`
-// bits -- an LSD radix sort with 8-bit digits entirely in shared memory (stable ranks
-// from per-warp digit counters + ballot peers) -- and writes them to out[lo, lo + m).
+// bits with LSD passes in shared memory (digits equal in every key skipped) and writes
+// them to out[lo, lo + m).
 __device__ void smem_sort_write(LocalSmem &S, const uint64_t *__restrict__ tk, const uint32_t *__restrict__ tv,
                                 uint32_t lo, uint32_t m, int bits, const Out &out) {
-    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+    const int tid = threadIdx.x, lane = tid & 31;
     if (tid == 0) {
         S.kor = 0ull;
         S.kand = ~0ull;
@@ -257,72 +328,8 @@ __device__ void smem_sort_write(LocalSmem &S, const uint64_t *__restrict__ tk, c
     __syncthreads();
     const uint64_t diff = S.kor ^ S.kand;
     int cur = 0;
-    const uint32_t wofs = uint32_t(w) * 32 * kItems;  // warp w owns slots [wofs, wofs + 32 kItems)
-    for (int sh = 0; sh < bits; sh += 8) {
-        if (((diff >> sh) & 255u) == 0) continue;  // same digit in every key: the pass is the identity
-#pragma unroll
-        for (int ww = 0; ww < kLWarps; ++ww) S.wcnt[ww][tid & 255] = 0;
-        __syncthreads();
-        uint64_t k[kItems];
-        uint32_t v[kItems], rank[kItems];
-        unsigned peers[kItems];
-#pragma unroll
-        for (int j = 0; j < kItems; ++j) {
-            const uint32_t i = wofs + j * 32 + lane;
-            const bool valid = i < m;
-            k[j] = valid ? S.k[cur][i] : 0ull;
-            v[j] = valid ? S.v[cur][i] : 0u;
-            peers[j] = match8(uint32_t(k[j] >> sh) & 255u, valid);
-        }
-#pragma unroll
-        for (int j = 0; j < kItems; ++j) {
-            const bool valid = wofs + j * 32 + lane < m;
-            const uint32_t d = uint32_t(k[j] >> sh) & 255u;
-            const uint32_t b0 = valid ? S.wcnt[w][d] : 0u;
-            rank[j] = b0 + __popc(peers[j] & lanemask_lt());
-            __syncwarp();
-            if (valid && lane == __ffs(peers[j]) - 1) S.wcnt[w][d] = b0 + __popc(peers[j]);
-            __syncwarp();
-        }
-        __syncthreads();
-        // digit-major, warp-minor exclusive offsets (thread tid < 256 owns digit tid)
-        uint32_t xw[kLWarps], c = 0;
-        if (tid < 256) {
-#pragma unroll
-            for (int ww = 0; ww < kLWarps; ++ww) {
-                xw[ww] = S.wcnt[ww][tid];
-                c += xw[ww];
-            }
-        }
-        uint32_t inc = c;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            const uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
-            if (lane >= o) inc += y;
-        }
-        if (lane == 31) S.ws[w] = inc;
-        __syncthreads();
-        if (tid < 256) {
-            uint32_t run = inc - c;
-            for (int i = 0; i < w; ++i) run += S.ws[i];
-#pragma unroll
-            for (int ww = 0; ww < kLWarps; ++ww) {
-                S.wcnt[ww][tid] = run;
-                run += xw[ww];
-            }
-        }
-        __syncthreads();
-#pragma unroll
-        for (int j = 0; j < kItems; ++j) {
-            if (wofs + j * 32 + lane < m) {
-                const uint32_t pos = S.wcnt[w][uint32_t(k[j] >> sh) & 255u] + rank[j];
-                S.k[cur ^ 1][pos] = k[j];
-                S.v[cur ^ 1][pos] = v[j];
-            }
-        }
-        cur ^= 1;
-        __syncthreads();
-    }
+    for (int sh = 0; sh < bits; sh += 8)
+        if ((diff >> sh) & 255u) smem_pass(S, m, sh, cur);  // same digit in every key: the pass is the identity
     for (uint32_t i = tid; i < m; i += kLT) out.put(uint64_t(lo) + i, S.k[cur][i], S.v[cur][i]);
     __syncthreads();
 }

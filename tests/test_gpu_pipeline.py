@@ -73,6 +73,30 @@ def test_pipeline_sort_skewed(impl, n, m, L):
     assert np.array_equal(got, want)
 
 
+@pytest.mark.parametrize("impl", [0, 2])
+@pytest.mark.parametrize("copies", [2, 33, 70, 1100])
+def test_pipeline_sort_equal_r_runs(impl, copies):
+    """The MSD segment sort orders r's digits only and then ranks each key inside its run
+    of equal r; runs past 1024 keys take the full-digit fallback. Q holds `copies` copies
+    of several R segments, so each of their r has that many MEMs."""
+    rng = np.random.default_rng(copies)
+    R = rng.choice(np.frombuffer(b"ACGT", dtype=np.uint8), 20000)
+    parts = []
+    for c in range(copies):
+        for a in (1000, 5000, 12000):
+            parts.append(R[a:a + 300])
+            parts.append(rng.choice(np.frombuffer(b"ACGT", dtype=np.uint8), 40 + c % 7))
+    Q = np.concatenate(parts)
+    want = oracle.mems(R.tobytes(), Q.tobytes(), 100, 13)
+    assert len(want) >= 3 * copies
+    gpumem.set_option("sort_impl", impl)
+    try:
+        got, _ = pipe_mems(R.tobytes().decode(), Q.tobytes().decode(), 100, 13)
+        assert np.array_equal(got, want)
+    finally:
+        gpumem.set_option("sort_impl", 0)
+
+
 @pytest.mark.parametrize("alg1", [0, 1])
 def test_pipeline_index_paths(alg1):
     """Both index builds (stable radix sort / Alg. 1 as written) under the captured graph."""
