@@ -883,6 +883,26 @@ cudaError_t launch_find(const FindParams &p, int grid, cudaStream_t s) {
     return cudaGetLastError();
 }
 
+// The pipeline's end-of-run report, written straight into its pinned host buffer (mapped
+// under unified addressing) by one launch instead of four small D2H copy nodes:
+// host[0, 8) = counters, [8] / [9] = R / Q alphabet flags, [10, 12) = balance stats.
+__global__ void k_collect(const unsigned long long *__restrict__ ctr, const unsigned long long *__restrict__ rbad,
+                          const unsigned long long *__restrict__ qbad, unsigned long long *host) {
+    pdl_wait();
+    const int t = threadIdx.x;
+    if (t < 8) host[t] = ctr[t];
+    else if (t == 8) host[8] = *rbad;
+    else if (t == 9) host[9] = *qbad;
+    else if (t < 12) host[t] = ctr[t - 2];
+}
+
+cudaError_t launch_collect(const unsigned long long *ctr, const unsigned long long *rbad,
+                           const unsigned long long *qbad, unsigned long long *host, cudaStream_t s) {
+    pdl_launch(k_collect, 1, 32, 0, s, ctr, rbad, qbad, host);
+    note_launch();
+    return cudaGetLastError();
+}
+
 cudaError_t launch_open_fix(const FindParams &p, cudaStream_t s) {
     pdl_launch(k_open_fix, num_sms() * 4, kT, 0, s, p.out_key, p.out_len, static_cast<const unsigned long long *>(p.out_count),
                p.capacity, p.R, p.nR, p.Q, p.nQ, p.qbits);

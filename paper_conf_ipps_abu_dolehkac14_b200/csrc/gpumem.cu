@@ -467,7 +467,7 @@ gpumem_status pack_q_pieces(gpumem_pipeline *pl, const char *Q, cudaStream_t s, 
     auto *words = static_cast<uint64_t *>(sc.get(n_words * 8));
     auto *bad = static_cast<unsigned long long *>(sc.get(8));
     if (!words || !bad) return GPUMEM_ERR_NOMEM;
-    CK(cudaMemsetAsync(bad, 0xff, 8, s), "memset");
+    CK(fill_async(bad, 0xffffffffu, 8, s), "flag init");
     const int K = pl->cap_chunks;
     for (int j = 0; j < K; ++j) {
         const uint64_t a = pl->q_bnd[j], b = pl->q_bnd[j + 1];
@@ -868,7 +868,7 @@ gpumem_status gpumem_pack(const char *bases, uint64_t n, int bases_on_device, vo
     auto *words = static_cast<uint64_t *>(sc.get(n_words * 8));
     auto *bad = static_cast<unsigned long long *>(sc.get(8));
     if (!words || !bad) return GPUMEM_ERR_NOMEM;
-    CK(cudaMemsetAsync(bad, 0xff, 8, s), "memset");
+    CK(fill_async(bad, 0xffffffffu, 8, s), "flag init");
     const uint8_t *in = reinterpret_cast<const uint8_t *>(bases);
     if (!bases_on_device && n) {
         auto *tmp = static_cast<uint8_t *>(ws_get(kWsPackTmp, n, s));
@@ -1258,7 +1258,7 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
         P.out_len = lens;
         P.capacity = cap;
         P.coop_cap = coop_cap;
-        CK(cudaMemsetAsync(ctr, 0, 320, s), "memset counters");
+        CK(fill_async(ctr, 0u, 320, s), "zero counters");
         const int K = t_cap->q_chunks > 1 && q_begin == 0 && q_end == nQ ? t_cap->q_chunks : 1;
         if (K == 1) {
             Stage g("find", s);
@@ -1309,10 +1309,7 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
                    "keys to triples");
             }
         }
-        CK(cudaMemcpyAsync(t_cap->host, ctr, 64, cudaMemcpyDeviceToHost, s), "D2H counters");
-        CK(cudaMemcpyAsync(t_cap->host + 10, ctr + 8, 16, cudaMemcpyDeviceToHost, s), "D2H balance");
-        CK(cudaMemcpyAsync(t_cap->host + 8, R->bad, 8, cudaMemcpyDeviceToHost, s), "D2H flag");
-        CK(cudaMemcpyAsync(t_cap->host + 9, Q->bad, 8, cudaMemcpyDeviceToHost, s), "D2H flag");
+        CK(launch_collect(ctr, R->bad, Q->bad, t_cap->host, s), "report");
         sc.keep(trip);
         *out = new gpumem_mems{kMagicMems, dev, s, 0, trip, gpumem_find_stats{}};
         t_cap->out_cap = cap;
@@ -1337,7 +1334,7 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
         P.coopq = static_cast<uint2 *>(ws_get(kWsCoop, coop_cap * sizeof(uint2), s));
         P.coop_cap = coop_cap;
         if (!P.coopq) return GPUMEM_ERR_NOMEM;
-        CK(cudaMemsetAsync(ctr, 0, 128, s), "memset counters");
+        CK(fill_async(ctr, 0u, 128, s), "zero counters");
         {
             Stage g("find", s);
             CK(launch_find(P, int(g_opt.find_grid), s), "find kernel");

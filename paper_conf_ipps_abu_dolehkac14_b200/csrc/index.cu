@@ -795,7 +795,7 @@ cudaError_t launch_ptrs_fill(const uint32_t *sorted_codes, uint64_t n_locs, uint
     auto *rank0 = reinterpret_cast<uint32_t *>(a);
     cudaError_t e = cudaSuccess;
     if (rankw) {  // 16 B per group: rank word + rotated occupancy (ORed in by the fill)
-        e = cudaMemsetAsync(rankw, 0, ((nb + 31) / 32) * 16, s);
+        e = fill_async(rankw, 0u, ((nb + 31) / 32) * 16, s);
         if (e != cudaSuccess) return e;
     }
     uint64_t bblocks = ((n_locs + 1 + 3) / 4 + kCodeThreads - 1) / kCodeThreads;

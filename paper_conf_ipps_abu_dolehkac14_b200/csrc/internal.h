@@ -88,6 +88,8 @@ __device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;"
 void *dalloc(size_t bytes, cudaStream_t s);   // nullptr on failure (error text set)
 void dfree(void *p, cudaStream_t s);
 void note_launch(int n = 1);                  // launch counter
+// bytes / 4 words of value v at p, as a (PDL) kernel instead of a memset node (pack.cu)
+cudaError_t fill_async(void *p, uint32_t v, size_t bytes, cudaStream_t s);
 int num_sms();
 
 gpumem_status fail(gpumem_status st, const char *fmt, ...);
@@ -198,6 +200,9 @@ cudaError_t launch_find(const FindParams &p, int grid, cudaStream_t s);
 cudaError_t launch_heavy(const FindParams &p, cudaStream_t s);
 cudaError_t launch_coop(const FindParams &p, cudaStream_t s);
 cudaError_t launch_open_fix(const FindParams &p, cudaStream_t s);  // after streamed-Q finds
+// pipeline report: counters, alphabet flags and balance stats into pinned host memory
+cudaError_t launch_collect(const unsigned long long *ctr, const unsigned long long *rbad,
+                           const unsigned long long *qbad, unsigned long long *host, cudaStream_t s);
 int find_default_grid(bool rank_sectors);
 
 // Instrumentation (diag.cu): best-of-4 time of n random 8-byte probes into a table of

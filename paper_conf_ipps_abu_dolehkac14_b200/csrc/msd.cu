@@ -506,7 +506,7 @@ static cudaError_t msd_run(uint64_t *keys, uint32_t *vals, NSpec ns, void *scrat
     uint32_t *big = reinterpret_cast<uint32_t *>(c);
     c = align(c + nb_max * 4);
     unsigned int *n_big = reinterpret_cast<unsigned int *>(c);
-    cudaError_t e = cudaMemsetAsync(n_big, 0, 4, s);
+    cudaError_t e = fill_async(n_big, 0u, 4, s);
     if (e != cudaSuccess) return e;
     static bool attr = false;
     if (!attr) {

@@ -132,7 +132,33 @@ __global__ void __launch_bounds__(kPackThreads) k_revcomp(const uint64_t *__rest
     out[w] = y;
 }
 
+// Fill `words` 32-bit words with v (16-byte stores when aligned), grid-stride. A kernel
+// rather than a memset node, so it keeps the PDL chain between the kernels around it.
+__global__ void __launch_bounds__(256) k_fill(uint32_t *__restrict__ p, uint64_t words, uint32_t v) {
+    pdl_wait();
+    const uint64_t t0 = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x, nt = uint64_t(gridDim.x) * blockDim.x;
+    uint64_t head = 0;
+    if ((reinterpret_cast<uintptr_t>(p) & 15) == 0) {
+        const uint64_t n4 = words / 4;
+        uint4 *q = reinterpret_cast<uint4 *>(p);
+        for (uint64_t i = t0; i < n4; i += nt) q[i] = make_uint4(v, v, v, v);
+        head = n4 * 4;
+    }
+    for (uint64_t i = head + t0; i < words; i += nt) p[i] = v;
+}
+
 }  // namespace
+
+cudaError_t fill_async(void *p, uint32_t v, size_t bytes, cudaStream_t s) {
+    const uint64_t words = bytes / 4;
+    if (!words) return cudaSuccess;
+    uint64_t blocks = (words / 4 + 255) / 256;
+    if (blocks < 1) blocks = 1;
+    if (blocks > uint64_t(num_sms()) * 8) blocks = uint64_t(num_sms()) * 8;
+    pdl_launch(k_fill, unsigned(blocks), 256, 0, s, static_cast<uint32_t *>(p), words, v);
+    note_launch();
+    return cudaGetLastError();
+}
 
 cudaError_t launch_revcomp(const uint64_t *in, uint64_t n, uint64_t *out, uint64_t n_words_alloc, cudaStream_t s) {
     const uint64_t blocks = (n_words_alloc + kPackThreads - 1) / kPackThreads;

@@ -447,7 +447,7 @@ cudaError_t radix_sort_rb(K *k0, uint32_t *v0, K *k1, uint32_t *v1, uint64_t n, 
     uint32_t *totals = static_cast<uint32_t *>(scratch);  // [passes][kBins]
     uint32_t *counts = totals + size_t(passes) * kBins;     // [kBins][chunks]
     uint32_t *offs = counts + size_t(ch.chunks) * kBins;    // [kBins][chunks]
-    e = cudaMemsetAsync(totals, 0, size_t(passes) * kBins * sizeof(uint32_t), s);
+    e = fill_async(totals, 0u, size_t(passes) * kBins * sizeof(uint32_t), s);
     if (e != cudaSuccess) return e;
     K *ka = k0, *kb = k1;
     uint32_t *va = v0, *vb = v1;

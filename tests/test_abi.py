@@ -52,7 +52,7 @@ def test_library_holds_sm100a_code(lib_path):
     sass = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "-sass", lib_path], capture_output=True,
                           text=True).stdout
     for k in ("k_pack", "k_find", "k_heavy", "k_coop", "k_seed_codes", "k_ptrs_fill", "k_seed_recs",
-              "k_chunk_hist", "k_chunk_scan", "k_scatter", "k_revcomp", "k_occurrences", "k_merge_tile", "k_split_emit", "k_band_continue", "k_open_fix"):
+              "k_chunk_hist", "k_chunk_scan", "k_scatter", "k_revcomp", "k_occurrences", "k_merge_tile", "k_split_emit", "k_band_continue", "k_open_fix", "k_fill", "k_collect"):
         assert k in sass, k
 
 
