@@ -302,7 +302,7 @@ gpumem_status check_device(int *dev) {
 // loop does no allocation at all once warm. gpumem_trim() releases everything.
 enum WsSlot {
     kWsCtr, kWsSpill, kWsKeys, kWsLens, kWsSortK, kWsSortL, kWsSortScratch, kWsCodes0, kWsCodes1,
-    kWsRadix, kWsFill, kWsMergeK, kWsFasta, kWsPackTmp, kWsCoop, kWsMums, kWsAlg1,
+    kWsRadix, kWsFill, kWsMergeK, kWsFasta, kWsPackTmp, kWsCoop, kWsMums, kWsAlg1, kWsTiled,
     kWsCount
 };
 struct Workspace {
@@ -719,6 +719,7 @@ gpumem_status gpumem_set_option(const char *name, int64_t value) {
     else if (!strcmp(name, "q_chunks")) g_opt.q_chunks = value < 1 ? 1 : value;
     else if (!strcmp(name, "pipe_events")) g_opt.pipe_events = value < 0 ? 0 : (value > 2 ? 2 : value);
     else if (!strcmp(name, "index_alg1")) g_opt.index_alg1 = value < 0 ? -1 : (value ? 1 : 0);
+    else if (!strcmp(name, "index_tiled")) g_opt.index_tiled = value < 0 ? -1 : (value ? 1 : 0);
     else if (!strcmp(name, "rec8")) g_opt.rec8 = value < 0 ? -1 : (value ? 1 : 0);
     else if (!strcmp(name, "rank_sectors")) g_opt.rank_sectors = value < 0 ? -1 : (value ? 1 : 0);
     else if (!strcmp(name, "l2_window")) {
@@ -976,7 +977,11 @@ static gpumem_status index_build_impl(const gpumem_seq *R, uint32_t ls, uint32_t
     uint4 *rsect = nullptr;
     if (use_sect) rsect = static_cast<uint4 *>(sc.get(((nb + 31) / 32) * 16));
     else rankw = static_cast<unsigned long long *>(sc.get(((nb + 31) / 32) * 16));  // + rotated occupancy
-    const uint64_t max_occ = (n_locs < nb ? n_locs : nb) + 1;
+    const bool alg1 = n_locs && (g_opt.index_alg1 > 0 || (g_opt.index_alg1 < 0 && n_locs * 4 >= nb));
+    const bool tiled = g_opt.index_tiled > 0 || (g_opt.index_tiled < 0 && n_locs <= (1u << 20));
+    const TiledPlan tp = (tiled && !alg1) ? tiled_plan(ls, n_locs) : TiledPlan{};
+    // compact table: one entry per occupied seed, or (tiled build) per location, gapped per bin
+    const uint64_t max_occ = (tp.ok ? n_locs : (n_locs < nb ? n_locs : nb)) + 1;
     auto *buckets = static_cast<uint2 *>(sc.get(max_occ * sizeof(uint2)));
     void *fill_scratch = ws_get(kWsFill, ptrs_fill_scratch_bytes(ls), s);
     auto *locs0 = static_cast<uint32_t *>(sc.get((n_locs ? n_locs : 1) * 4));
@@ -988,7 +993,20 @@ static gpumem_status index_build_impl(const gpumem_seq *R, uint32_t ls, uint32_t
     void *recs = sc.get((n_locs ? n_locs : 1) * (rec8 ? sizeof(uint2) : sizeof(uint4)));
     if (!recs) return GPUMEM_ERR_NOMEM;
     bool recs_done = false, fill_done = false;
-    if (n_locs && (g_opt.index_alg1 > 0 || (g_opt.index_alg1 < 0 && n_locs * 4 >= nb))) {
+    if (tp.ok) {
+        // Alg. 1 tiled over the seed space: partition, then every bin in shared memory
+        void *scratch = ws_get(kWsTiled, tiled_scratch_bytes(tp, n_locs), s);
+        if (!scratch) return GPUMEM_ERR_NOMEM;
+        {
+            Stage g("index.tiled", s);
+            const bool side = t_cap && t_cap->side;  // hot bins beside the warps' bins
+            CK(launch_index_tiled(tp, R->words, ls, step, k0, n_locs, rankw, rsect, buckets, locs0, recs, rec8, scratch, s,
+                                  side ? t_cap->side : nullptr, side ? t_cap->ev_a : nullptr,
+                                  side ? t_cap->ev_b : nullptr),
+               "index (tiled Alg. 1)");
+        }
+        fill_done = recs_done = true;
+    } else if (alg1) {
         // dense index: Alg. 1 literally (atomic counts, prefix sums, placement, bucket sort)
         void *scratch = ws_get(kWsAlg1, alg1_scratch_bytes(ls, n_locs), s);
         if (!scratch) return GPUMEM_ERR_NOMEM;

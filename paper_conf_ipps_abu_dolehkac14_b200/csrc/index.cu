@@ -32,6 +32,7 @@
 
 #include "internal.h"
 #include "device.cuh"
+#include "index_common.cuh"
 
 namespace gm {
 namespace {
@@ -40,6 +41,7 @@ constexpr int kCodeThreads = 256;
 constexpr int kFillThreads = 512;
 constexpr int kChunk = 16384;                   // buckets per CTA in k_ptrs_fill
 constexpr int kPer = kChunk / kFillThreads;     // 32 consecutive buckets per thread
+static_assert(kPer == 32, "k_ptrs_fill: one seed group per thread");
 
 // four consecutive sampled locations per thread (16-byte stores), grid-stride: one
 // thread per location left the GPU block-scheduling-bound (C5 L = 20: 31 M locations)
@@ -138,20 +140,6 @@ __global__ void __launch_bounds__(1024) k_occ_scan(const uint32_t *__restrict__ 
     }
 }
 
-// Rank-word directory entries are 16 bytes per group g of 32 seeds: word 2g = {occupancy
-// bits, occupied seeds before the group} (the rank word), word 2g+1 = occupancy of the 32
-// seeds whose codes ROTATED left by one base (the first base moved to the end) fall in
-// group g. Rotating code(Q, q) gives the same top bits as code(Q, q+1) (both start with
-// bases q+1 ...), so one 16-byte probe of group code(q+1) >> 5 answers "is the seed at q
-// occupied?" and "at q+1?" -- k_find probes query positions in pairs.
-// The rotated bits are ORed in here (the directory is zeroed first) for every occupied seed.
-__device__ __forceinline__ void set_rot_occ(unsigned long long *rankw, uint32_t code, uint32_t ls) {
-    const uint32_t nbits = 2 * ls;
-    const uint32_t mask = nbits >= 32 ? 0xffffffffu : ((1u << nbits) - 1u);
-    const uint32_t rot = ((code << 2) | (code >> (nbits - 2))) & mask;
-    atomicOr(reinterpret_cast<unsigned int *>(rankw + 2 * (rot >> 5) + 1), 1u << (rot & 31));
-}
-
 // kCounts: `codes` is instead the dense per-seed count array (Alg. 1 step 1 done with
 // atomics by k_alg1_count) and chunk_first the records before each chunk.
 template <bool kSect, bool kCounts = false>
@@ -226,17 +214,15 @@ __global__ void __launch_bounds__(kFillThreads) k_ptrs_fill(const uint32_t *__re
     }
     pre += inc - sum;
     preo += inco - nocc;
-    // counts -> ptrs (in place), rank words {occupancy bits, occupied buckets before this
-    // word} and the compact {first slot, count} table, in bucket order
+    // counts -> ptrs (in place) and rank words {occupancy bits, occupied buckets before this
+    // word} (or rank sectors)
     const uint64_t rank = uint64_t(rank0[c]) + preo;
-    uint64_t r = rank;
     const uint32_t group_first = pre;
     uint64_t c2 = 0;  // 2-bit saturating count per seed of the group
 #pragma unroll 4
     for (int j = 0; j < kPer; ++j) {
         const uint32_t x = cnt[tid * (kPer + 1) + j];
         cnt[tid * (kPer + 1) + j] = pre;
-        if (x) buckets[r++] = make_uint2(pre, x);
         if (!kSect && x) set_rot_occ(rankw, uint32_t(s0) + uint32_t(tid) * kPer + j, rot_ls);
         if (kSect) c2 |= uint64_t(x < 3 ? x : 3u) << (2 * j);
         pre += x;
@@ -246,6 +232,24 @@ __global__ void __launch_bounds__(kFillThreads) k_ptrs_fill(const uint32_t *__re
         else rankw[2 * ((s0 >> 5) + tid)] = (rank << 32) | occ;
     }
     __syncthreads();
+    // the compact {first slot, count} table in seed order, coalesced: warp w's seeds (the 32
+    // groups of its lanes) take consecutive entries from its first lane's rank; lane j walks
+    // seed j of each group (consecutive seeds across the lanes, consecutive entries)
+    {
+        uint32_t chunk_end = uint32_t(lo);
+        for (int i = 0; i < kFillThreads / 32; ++i) chunk_end += wsum[i];
+        uint64_t wr = __shfl_sync(0xffffffffu, rank, 0);
+        const uint32_t wseed = uint32_t(w) * 32 * kPer;
+        for (int g = 0; g < 32; ++g) {  // group g of the warp = lane g's seeds
+            const uint32_t sl = wseed + uint32_t(g) * kPer + uint32_t(lane);  // chunk-local seed
+            const uint32_t f = cnt[sl + (sl >> 5)];
+            const uint32_t nx = sl + 1 < uint32_t(kChunk) ? cnt[(sl + 1) + ((sl + 1) >> 5)] : chunk_end;
+            const uint32_t x = s0 + sl < n_buckets ? nx - f : 0u;
+            const unsigned ob = __ballot_sync(0xffffffffu, x != 0);
+            if (x) buckets[wr + __popc(ob & lanemask_lt())] = make_uint2(f, x);
+            wr += __popc(ob);
+        }
+    }
     // coalesced write-out of the chunk's ptrs, 16 bytes per store (skipped when the dense
     // table is not wanted: the lookup uses the rank directory + compact table, and
     // gpumem_index_view expands ptrs from them on demand, k_ptrs_expand)
@@ -529,38 +533,9 @@ __global__ void __launch_bounds__(kCodeThreads) k_bucket_fix(const uint2 *__rest
     }
 }
 
-// One CTA per listed bucket: a bitonic-type sorting network with ascending
-// compare-exchanges only (the first stage of every merge pairs i with the mirror
-// element), so indices past the bucket act as +infinity and need no padding. In shared
-// memory up to kBigSmem locations, in place in global memory beyond.
 constexpr uint32_t kBigSmem = 16384;
-__device__ __forceinline__ void cmpswap(uint32_t *a, uint32_t i, uint32_t j) {
-    const uint32_t x = a[i], y = a[j];
-    if (x > y) {
-        a[i] = y;
-        a[j] = x;
-    }
-}
-__device__ void net_sort(uint32_t *a, uint32_t n) {
-    uint32_t N = 1;
-    while (N < n) N <<= 1;
-    for (uint32_t k = 2; k <= N; k <<= 1) {
-        for (uint32_t t = threadIdx.x; t < N / 2; t += blockDim.x) {  // mirror stage
-            const uint32_t blk = t / (k / 2), j = t % (k / 2);
-            const uint32_t i0 = blk * k + j, i1 = blk * k + k - 1 - j;
-            if (i1 < n) cmpswap(a, i0, i1);
-        }
-        __syncthreads();
-        for (uint32_t d = k / 4; d >= 1; d >>= 1) {  // half-cleaners
-            for (uint32_t t = threadIdx.x; t < N / 2; t += blockDim.x) {
-                const uint32_t blk = t / d, j = t % d;
-                const uint32_t i0 = blk * 2 * d + j, i1 = i0 + d;
-                if (i1 < n) cmpswap(a, i0, i1);
-            }
-            __syncthreads();
-        }
-    }
-}
+// One CTA per listed bucket: the sorting network net_sort (index_common.cuh), in shared
+// memory up to kBigSmem locations, in place in global memory beyond.
 __global__ void __launch_bounds__(1024) k_bucket_big(const uint2 *__restrict__ buckets, const uint32_t *__restrict__ big,
                                                      const unsigned int *__restrict__ n_big, uint32_t *__restrict__ locs) {
     pdl_wait();
@@ -579,42 +554,6 @@ __global__ void __launch_bounds__(1024) k_bucket_big(const uint2 *__restrict__ b
         }
         __syncthreads();
     }
-}
-
-// Seed records (lookup acceleration, not part of the paper's index): for each slot k
-// of locs, {p, bases R[p-16, p) with base p-1 in the low bits (00 before position 0),
-// bases R[p+ls, p+ls+32) first base highest (00 past the end)} -- 16 bytes, one
-// sector, so the find kernel decides a random seed hit without gathering R. With
-// step <= 8 the left extension never passes 8 bases, and 8-byte records {p, R[p-8, p)
-// | R[p+ls, p+ls+8) << 16} halve the record traffic of the (then numerous) hits.
-// the record of location p = locs[k] (16-byte or 8-byte layout, see above)
-template <bool kRec8>
-__device__ __forceinline__ void seed_rec(const uint64_t *__restrict__ R, uint32_t ls, uint32_t p, void *recs,
-                                         uint64_t k) {
-    uint32_t left;
-    uint64_t right;
-    if (kRec8 && p >= 8) {  // bases [p - 8, p + ls + 8) (<= 31 bases) lie in the 2 words from (p - 8) / 32
-        const uint64_t x = p - 8, w = x >> 5;
-        const uint64_t w0 = __ldg(R + w), w1 = __ldg(R + w + 1);
-        const uint32_t sx = uint32_t(x & 31) * 2;
-        const uint64_t win = sx ? (w0 << sx) | (w1 >> (64 - sx)) : w0;  // bases [p - 8, p + 24)
-        left = uint32_t(win >> 48);                                       // R[p - 8, p), base p-1 lowest
-        right = (win << (2 * (8 + ls))) & 0xffff000000000000ull;          // R[p + ls, p + ls + 8) on top
-    } else if (p >= 16) {  // bases [p - 16, p + ls + 32) lie in the 3 words from (p - 16) / 32: one gather
-        const uint64_t x = p - 16, w = x >> 5;
-        const uint64_t w0 = __ldg(R + w), w1 = __ldg(R + w + 1), w2 = __ldg(R + w + 2);
-        const uint32_t sx = uint32_t(x & 31) * 2;
-        left = uint32_t(((w0 << sx) | ((w1 >> 1) >> (63 - sx))) >> 32);
-        const uint32_t o = uint32_t(x & 31) + 16 + ls;  // right window start, bases from word w
-        const uint32_t so = (o & 31) * 2;
-        const uint64_t a = o < 32 ? w0 : w1, b = o < 32 ? w1 : w2;
-        right = (a << so) | ((b >> 1) >> (63 - so));
-    } else {
-        left = uint32_t(win_back(R, p));
-        right = win_fwd(R, uint64_t(p) + ls);
-    }
-    if (kRec8) static_cast<uint2 *>(recs)[k] = make_uint2(p, (left & 0xffffu) | uint32_t(right >> 48) << 16);
-    else static_cast<uint4 *>(recs)[k] = make_uint4(p, left, uint32_t(right), uint32_t(right >> 32));
 }
 
 // kRecsPT records per thread (their R gathers in flight together), grid-stride

@@ -45,6 +45,10 @@ struct Options {
     int64_t index_alg1 = 0;      // Alg. 1 literally (atomic counts, scan, placement, bucket sort): 1 always,
                                  // -1 for dense indexes (n_locs >= 4^ls / 4), 0 never (default: measured
                                  // slower everywhere -- C5 L = 20 2.9 vs 1.4 ms, C4 0.40 vs 0.21 ms)
+    int64_t index_tiled = -1;    // index build: 1 Alg. 1 tiled over the seed space (tindex.cu) where it
+                                 // applies (sparse, ls <= 13), 0 the radix-sort path (index.cu + radix.cu),
+                                 // -1 auto: tiled up to 1 M sampled locations (measured faster at C1/C2,
+                                 // slower at C3/C4: see DESIGN.md)
     int64_t l2_persist = 0;      // MB of L2 set aside for persisting lines (cudaLimitPersistingL2CacheSize);
                                  // 0 = none (default)
     int64_t l2_window = 0;       // k_find / k_heavy access-policy window over: 0 nothing, 1 the lookup
@@ -126,6 +130,7 @@ cudaError_t radix_sort_u64(uint64_t *k0, uint32_t *v0, uint64_t *k1, uint32_t *v
                            void *scratch, cudaStream_t s, bool *in_alt, int lo = 0,
                            const unsigned long long *dn = nullptr);
 size_t radix_scratch_bytes(uint64_t n);
+int radix_passes(int bits, uint64_t n);  // LSD passes a sort of `bits` key bits of n keys runs
 
 // MSD bucket sort of unique u64 keys (+ optional u32 values), in place, or written as
 // triples {key >> qbits, key & qmask, val} when trip != null (msd.cu).
@@ -140,6 +145,19 @@ cudaError_t msd_sort_dev(uint64_t *keys, uint32_t *vals, const unsigned long lon
 cudaError_t launch_seed_codes(const uint64_t *R, uint32_t ls, uint32_t step, uint64_t k0, uint64_t n_locs,
                               uint32_t *codes, uint32_t *locs, cudaStream_t s);
 size_t ptrs_fill_scratch_bytes(uint32_t ls);
+// Alg. 1 tiled over the seed space (tindex.cu): partition the sampled locations into 2^H
+// bins of 2^bbits seeds, then Alg. 1 steps 1-4 + directory + table + seed records per bin
+// in shared memory. ok == 0: not applicable (ls > 13), use the radix path.
+struct TiledPlan {
+    uint32_t ok, H, bbits, wcap;  // 2^H bins of 2^bbits seeds; locations a warp takes per bin
+};
+TiledPlan tiled_plan(uint32_t ls, uint64_t n_locs);
+size_t tiled_scratch_bytes(const TiledPlan &p, uint64_t n_locs);
+// buckets must hold n_locs + 1 entries (gapped per bin, see tindex.cu)
+cudaError_t launch_index_tiled(const TiledPlan &p, const uint64_t *R, uint32_t ls, uint32_t step, uint64_t k0,
+                               uint64_t n_locs, unsigned long long *rankw, uint4 *rsect, uint2 *buckets, uint32_t *locs,
+                               void *recs, int rec8, void *scratch, cudaStream_t s, cudaStream_t side = nullptr,
+                               cudaEvent_t ev_fork = nullptr, cudaEvent_t ev_join = nullptr);
 // Alg. 1 as written for dense indexes (index.cu): counts by atomics, prefix sums +
 // directory, placement, per-bucket sort -> locs, directory, compact table.
 size_t alg1_scratch_bytes(uint32_t ls, uint64_t n_locs);

@@ -483,6 +483,12 @@ cudaError_t radix_sort(K *k0, uint32_t *v0, K *k1, uint32_t *v1, uint64_t n, int
 
 }  // namespace
 
+int radix_passes(int bits, uint64_t n) {  // as radix_sort runs them (none for n <= 1)
+    if (bits <= 0 || n <= 1) return 0;
+    const int rb = pick_digit_bits(bits, n);
+    return (bits + rb - 1) / rb;
+}
+
 size_t radix_scratch_bytes(uint64_t n) {  // totals of every pass + counts + offsets, at the widest digit
     (void)n;
     return size_t(8 * 1024 + 2 * size_t(kMaxChunks) * 1024) * sizeof(uint32_t);

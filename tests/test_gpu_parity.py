@@ -24,7 +24,7 @@ def _default_options():
     yield
     for k, v in (("find_grid", 0), ("find_spill", 64), ("out_capacity", 0), ("use_bitmap", 1), ("static_lb", 0),
                  ("sort_impl", 0), ("radix_bits", 0),
-                 ("rank_sectors", -1), ("rec8", -1), ("pdl", 1), ("index_alg1", 0)):
+                 ("rank_sectors", -1), ("rec8", -1), ("pdl", 1), ("index_alg1", 0), ("index_tiled", -1)):
         gpumem.set_option(k, v)
 
 
@@ -122,11 +122,13 @@ def test_index_parity_word_for_word(cfg, ls, step, scale):
     and locs word for word against Alg. 1."""
     P = synth.make_pair(cfg, scale=scale)
     op, ol = oracle.index(P.R.tobytes(), ls, step)
-    for sect in (-1, 0, 1):
-        gpumem.set_option("rank_sectors", sect)
-        p, l = _index_gpu(P.R.tobytes(), ls, step)
-        assert np.array_equal(p, op), sect
-        assert np.array_equal(l, ol), sect
+    for tiled in (1, 0):  # Alg. 1 tiled over the seed space (tindex.cu) / the radix path
+        gpumem.set_option("index_tiled", tiled)
+        for sect in (-1, 0, 1):
+            gpumem.set_option("rank_sectors", sect)
+            p, l = _index_gpu(P.R.tobytes(), ls, step)
+            assert np.array_equal(p, op), (tiled, sect)
+            assert np.array_equal(l, ol), (tiled, sect)
 
 
 def test_index_hot_seed_chunks():
@@ -136,16 +138,20 @@ def test_index_hot_seed_chunks():
     for ls, step in ((13, 1), (12, 3), (5, 2)):
         op, ol = oracle.index(R, ls, step)
         for sect in (0, 1):
-            for alg1 in (0, 1):  # Alg. 1 path: buckets of 70 000 (global sorting network), 20 000, ...
+            # Alg. 1 as written (buckets of 70 000: global sorting network), the tiled Alg. 1
+            # (a bin of 70 000: beyond a CTA's shared memory, steps 3-4 in global memory),
+            # the radix path
+            for alg1, tiled in ((1, 0), (0, 1), (0, 0)):
                 gpumem.set_option("rank_sectors", sect)
                 gpumem.set_option("index_alg1", alg1)
+                gpumem.set_option("index_tiled", tiled)
                 p, l = _index_gpu(R, ls, step)
-                assert np.array_equal(p, op) and np.array_equal(l, ol), (ls, step, sect, alg1)
+                assert np.array_equal(p, op) and np.array_equal(l, ol), (ls, step, sect, alg1, tiled)
 
 
-@pytest.mark.parametrize("opts", [{"radix_bits": 8}, {"radix_bits": 10},
+@pytest.mark.parametrize("opts", [{"radix_bits": 8, "index_tiled": 0}, {"radix_bits": 10, "index_tiled": 0},
                                   {"index_alg1": 1}, {"index_alg1": 1, "rank_sectors": 1}, {"index_alg1": 0},
-                                  {"rank_sectors": 1, "rec8": 1}])
+                                  {"rank_sectors": 1, "rec8": 1}, {"rank_sectors": 1, "rec8": 1, "index_tiled": 0}])
 def test_index_sort_paths(opts):
     """Every index path (stable LSD radix sort at each digit width, Alg. 1 as written)
     gives the oracle's Alg. 1 ptrs/locs word for word."""
@@ -252,14 +258,14 @@ def test_overflow_retry_grid_spill_and_bitmap_invariance():
     for opt, vals in (("out_capacity", [1, 100]), ("find_grid", [1, 3, 148]), ("find_spill", [1, 2, 10**9]),
                       ("use_bitmap", [0]), ("static_lb", [1]), ("sort_impl", [1, 2]),
                       ("rank_sectors", [0, 1]), ("rec8", [0, 1]),
-                      ("radix_bits", [8, 9, 10]), ("pdl", [0]), ("index_alg1", [1, -1])):
+                      ("radix_bits", [8, 9, 10]), ("pdl", [0]), ("index_alg1", [1, -1]), ("index_tiled", [0, 1])):
         for v in vals:
             gpumem.set_option(opt, v)
             assert np.array_equal(gpu_mems(P.R, P.Q, P.L, P.ls), want), (opt, v)
         gpumem.set_option(opt, {"out_capacity": 0, "find_grid": 0, "find_spill": 64, "use_bitmap": 1,
                                 "static_lb": 0, "sort_impl": 0, "rank_sectors": -1,
                                 "rec8": -1,
-                                "radix_bits": 0, "pdl": 1, "index_alg1": 0}[opt])
+                                "radix_bits": 0, "pdl": 1, "index_alg1": 0, "index_tiled": -1}[opt])
 
 
 def test_l2_persisting_window_invariance():
@@ -381,8 +387,10 @@ def test_kernels_are_ours():
     assert kernels, "no kernel seen by the profiler"
     foreign = [k for k in kernels if "gm::" not in k]
     assert not foreign, foreign
-    for stage in ("k_pack", "k_seed_codes", "k_scatter", "k_dir_fill", "k_seed_recs", "k_find", "k_heavy", "k_bs_local"):
-        assert any(stage in k for k in kernels), (stage, sorted(set(kernels)))
+    for stage in ("k_pack", "k_seed_codes", "k_scatter", ("k_dir_fill", "k_tx_warp"), "k_seed_recs", "k_find",
+                  "k_heavy", "k_bs_local"):
+        alts = stage if isinstance(stage, tuple) else (stage,)  # radix / tiled index build
+        assert any(a in k for k in kernels for a in alts), (stage, sorted(set(kernels)))
     assert launched == len(kernels), (launched, len(kernels))
 
 

@@ -25,6 +25,7 @@ def _default_options():
     gpumem.set_option("out_capacity", 0)
     gpumem.set_option("sort_impl", 0)
     gpumem.set_option("index_alg1", 0)
+    gpumem.set_option("index_tiled", -1)
     gpumem.set_option("pipe_events", 0)
 
 
@@ -97,14 +98,16 @@ def test_pipeline_sort_equal_r_runs(impl, copies):
         gpumem.set_option("sort_impl", 0)
 
 
-@pytest.mark.parametrize("alg1", [0, 1])
-def test_pipeline_index_paths(alg1):
-    """Both index builds (stable radix sort / Alg. 1 as written) under the captured graph."""
+@pytest.mark.parametrize("alg1,tiled", [(0, 1), (0, 0), (1, 0)])
+def test_pipeline_index_paths(alg1, tiled):
+    """Every index build (tiled Alg. 1 / stable radix sort / Alg. 1 as written) under the
+    captured graph."""
     gpumem.set_option("index_alg1", alg1)
+    gpumem.set_option("index_tiled", tiled)
     for cfg, scale in (("c5_l20", 0.02), ("c1", 1.0)):
         P = synth.make_pair(cfg, scale=scale)
         got, _ = pipe_mems(P.R, P.Q, P.L, P.ls, runs=2)
-        assert np.array_equal(got, oracle.mems(P.R, P.Q, P.L, P.ls)), (cfg, alg1)
+        assert np.array_equal(got, oracle.mems(P.R, P.Q, P.L, P.ls)), (cfg, alg1, tiled)
 
 
 def test_pipeline_random_tiny_vs_brute_force():
@@ -237,7 +240,7 @@ def test_pipeline_streamed_query_long_matches():
         gpumem.set_option("q_chunks", 8)
 
 
-@pytest.mark.parametrize("events,want", [(0, set()), (2, {"find"}), (1, {"pack", "index.sort", "find", "sort"})])
+@pytest.mark.parametrize("events,want", [(0, set()), (2, {"find"}), (1, {"pack", "index.tiled", "find", "sort"})])
 def test_pipeline_event_modes(events, want):
     """pipe_events: no stage events (default), find's only (the timed bench graph), every
     stage; the MEM set never depends on it."""
