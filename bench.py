@@ -189,6 +189,11 @@ def impl_bytes(nR, nQ, ls, L, stats):
         "index.sort": passes * n_locs * (16 + 4),
         "index.ptrs": n_locs * 4 + (nb / 2 if sect else nb / 4) + 8 * min(n_locs, nb),
         "index.recs": n_locs * (4 + 24 + rec),
+        # tiled Alg. 1 (tindex.cu, sparse indexes up to 2^20 locations): codes + locations
+        # written, radix passes over the top 2 ls - 10 bits, the bins read once, locs +
+        # {first, count} entry per location, the directory, the seed records
+        "index.tiled": n_locs * (8 + radix_passes(max(2 * ls - 10, 0), n_locs) * 20 + 8 + 4 + 8 + 4 + 24 + rec)
+                       + (nb / 2 if sect else nb / 4),
         "find": 0.25 * pos + pos / 8 + 8 * occ + rec * hits + 12 * mems,
         "sort": sort,
     }

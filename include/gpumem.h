@@ -364,12 +364,12 @@ gpumem_status gpumem_set_allocator(void *(*alloc_fn)(size_t bytes, void *cuda_st
  *                     count of its measuring run
  *  "rec8"             seed records: -1 (default) auto (8-byte when step <= 8), 0 16-byte, 1 8-byte
  *  "rank_sectors"     lookup directory: -1 (default) auto, 0 rank words, 1 rank sectors
- *  "index_tiled"      1: the index is Alg. 1 tiled over the seed space (the sampled
- *                     locations partitioned into bins of 1024 consecutive seeds by a radix
- *                     sort of the top code bits, then Alg. 1 steps 1-4, the directory and
- *                     the table per bin on chip; sparse indexes with seed_len <= 13);
+ *  "index_tiled"      1: a sparse index (n_locs < 4^ls / 4, seed_len <= 13) is Alg. 1
+ *                     tiled over the seed space (the sampled locations put into bins of
+ *                     1024 consecutive seeds by a radix sort of the top code bits, then
+ *                     Alg. 1 steps 1-4, the directory and the table per bin on chip);
  *                     0: the stable LSD radix sort of all code bits; -1 (default): tiled
- *                     up to 2^20 sampled locations
+ *                     for sparse indexes up to 2^20 sampled locations
  *  "index_alg1"       1: PAPER.md Alg. 1 as written over the whole 4^ls table (atomic
  *                     counts, prefix sums, placement, per-bucket sort); -1: only for
  *                     dense indexes (n_locs >= 4^ls / 4); 0 (default): never (measured

@@ -46,9 +46,9 @@ struct Options {
                                  // -1 for dense indexes (n_locs >= 4^ls / 4), 0 never (default: measured
                                  // slower everywhere -- C5 L = 20 2.9 vs 1.4 ms, C4 0.40 vs 0.21 ms)
     int64_t index_tiled = -1;    // index build: 1 Alg. 1 tiled over the seed space (tindex.cu) where it
-                                 // applies (sparse, ls <= 13), 0 the radix-sort path (index.cu + radix.cu),
-                                 // -1 auto: tiled up to 1 M sampled locations (measured faster at C1/C2,
-                                 // slower at C3/C4: see DESIGN.md)
+                                 // applies (sparse: n_locs < 4^ls / 4, ls <= 13), 0 the radix-sort path
+                                 // (index.cu + radix.cu), -1 auto: tiled up to 2^20 locations (measured
+                                 // faster at C1/C2, slower at C3-C5: DESIGN.md)
     int64_t l2_persist = 0;      // MB of L2 set aside for persisting lines (cudaLimitPersistingL2CacheSize);
                                  // 0 = none (default)
     int64_t l2_window = 0;       // k_find / k_heavy access-policy window over: 0 nothing, 1 the lookup

@@ -6,21 +6,22 @@
 //  k_seed_codes  Eq. 1 sampling (p = (k0 + k) * step, :86-90) and the seed code of every
 //                sampled location (index.cu);
 //  radix sort    stable LSD passes over the top H code bits only (radix.cu; 2 passes for
-//                ls = 13 instead of 3-4 over all 2 ls bits): the locations grouped by bin,
+//                ls = 13 instead of 3 over all 2 ls bits): the locations grouped by bin,
 //                ascending inside each bin;
 //  k_tx_bounds   the first slot of every bin (one pass over the bin-sorted codes);
-//  k_tx_warp     one warp per bin of <= Cap locations (Cap 128-512 by the mean density):
-//                Alg. 1 step 1 (a shared counter per seed), step 2 (exclusive scan = the
-//                bin's slice of ptrs, :84), step 3 (placement through cursors), step 4 (each
-//                seed's locations ascending: a bucket of > kRunT locations is placed in
-//                input order, which is ascending; shorter ones are insertion-sorted by
-//                their lane); the directory groups, {first, count} entries, locs and seed
-//                records of the bin from the same counters, each written once;
+//  k_tx_warp     one warp per bin of <= Cap locations (Cap 128-512 by the mean density),
+//                Alg. 1 steps 1-4 for the bin (a count per seed, exclusive scan = the bin's
+//                slice of ptrs :84, placement, each seed's locations ascending): a bin of
+//                <= 32 locations (nearly all of a sparse index) by a radix rank from one
+//                ballot per seed bit; a larger one by two stable 5-bit counting passes
+//                (lane l = digit l). The bin's directory groups, {first, count} entries and
+//                locs come out of the same ranks, each written once;
 //  k_tx_bins     the same by a CTA (shared counters per seed, block scans) for the bins
 //                past Cap (hot seeds), concurrently with k_tx_warp; a bin past kBCap runs
 //                steps 3-4 in global memory;
 //  k_seed_recs   the seed records in slot order (index.cu).
-// Used for sparse indexes (n_locs < 4^ls / 4); dense ones take the radix path.
+// Used by default for sparse indexes up to 2^20 locations (measured faster there: C1,
+// C2); larger or dense ones take the radix path.
 //
 // The compact {first, count} table is indexed from each bin's FIRST SLOT: bin j's
 // occupied seeds take table entries [off_j, off_j + occupied_j), and entries up to
@@ -41,7 +42,7 @@
 namespace gm {
 namespace {
 
-constexpr int kMaxH = 16;         // at most 65536 bins (two radix passes)
+constexpr int kMaxH = 16;         // at most 2^16 bins (two radix passes)
 constexpr int kWT = 128;          // threads of k_tx_warp (4 warps, one bin each)
 constexpr int kBT = 512;          // threads of k_tx_bins
 constexpr uint32_t kBCap = 4096;  // locations a k_tx_bins CTA holds in shared memory
@@ -133,6 +134,73 @@ __device__ __forceinline__ Match5 match5(uint32_t d, bool valid) {
     return Match5{byl, byd};
 }
 
+// A bin of m <= 32 locations, one per lane (lane i: the i-th, ascending): Alg. 1 steps 1-4
+// as a radix rank over the bin-local seed bits (ballots from the top bit down keep the
+// lanes still equal to mine and count the smaller ones), so location i goes to slot
+// rank_i; the same rank over the run heads only (one per occupied seed) gives its
+// {first, count} entry, and over a lane's own number (as a group) the directory counts.
+constexpr int kTB = 10;  // bin-local seed bits at most (bins of <= 2^10 seeds)
+template <bool kSect>
+__device__ void bin_warp_round(uint32_t bin, uint32_t lo, uint32_t m, uint32_t *occw, uint32_t *c2lo,
+                               uint32_t *c2hi, const uint32_t *ic, const uint32_t *il, uint32_t bbits, uint32_t ls,
+                               uint32_t *__restrict__ locs, unsigned long long *__restrict__ rankw,
+                               uint4 *__restrict__ rsect, uint2 *__restrict__ buckets) {
+    const uint32_t lane = threadIdx.x & 31, lt = lanemask_lt();
+    const uint32_t bmask = (1u << bbits) - 1, ng = bbits >= 5 ? (1u << bbits) >> 5 : 1u;
+    const bool valid = lane < m;
+    const uint32_t c = valid ? ic[lane] & bmask : 0u;
+    const unsigned vm = __ballot_sync(0xffffffffu, valid);
+    unsigned bal[kTB];
+#pragma unroll
+    for (int b = 0; b < kTB; ++b) bal[b] = __ballot_sync(0xffffffffu, valid && ((c >> b) & 1u));
+    // rank of value v among the lanes of `set`: (lanes with a smaller value, lanes equal)
+    auto rank = [&](uint32_t v, unsigned set, int lowest, uint32_t &smaller) -> unsigned {
+        smaller = 0;
+#pragma unroll
+        for (int b = kTB - 1; b >= 0; --b) {
+            if (b < int(bbits) && b >= lowest) {
+                if ((v >> b) & 1u) {
+                    smaller += __popc(set & ~bal[b]);
+                    set &= bal[b];
+                } else {
+                    set &= ~bal[b];
+                }
+            }
+        }
+        return set;
+    };
+    uint32_t less, hless;
+    const unsigned eq = rank(c, vm, 0, less);             // my seed's locations
+    const bool head = valid && (eq & lt) == 0;            // the first of them
+    const unsigned hm = __ballot_sync(0xffffffffu, head);
+    rank(c, hm, 0, hless);                                // occupied seeds before mine
+    if (valid) locs[lo + less + __popc(eq & lt)] = il[lane];
+    const uint32_t g = c >> 5, bb = c & 31, len = __popc(eq);
+    if (head) {
+        buckets[lo + hless] = make_uint2(lo + less, len);
+        atomicOr(&occw[g], 1u << bb);
+        if (kSect) {
+            const uint32_t sat = len < 3 ? len : 3u;
+            if (bb < 16) atomicOr(&c2lo[g], sat << (2 * bb));
+            else atomicOr(&c2hi[g], sat << (2 * (bb - 16)));
+        } else {
+            set_rot_occ(rankw, uint32_t(((uint64_t(bin) << bbits) >> 5) << 5) + c, ls);
+        }
+    }
+    const uint32_t n_occ = __popc(hm);
+    if (lane >= n_occ && lane < m) buckets[lo + lane] = make_uint2(lo + m, 0u);  // gaps
+    __syncwarp();
+    // directory: lane q = group q; locations / occupied seeds in groups before it
+    uint32_t pe, po;
+    rank(lane << 5, vm, 5, pe);
+    rank(lane << 5, hm, 5, po);
+    if (lane < ng) {
+        const uint64_t gq = ((uint64_t(bin) << bbits) >> 5) + lane;
+        if (kSect) rsect[gq] = make_uint4(lo + pe, lo + po, c2lo[lane], c2hi[lane]);
+        else rankw[2 * gq] = (uint64_t(lo + po) << 32) | occw[lane];
+    }
+}
+
 template <bool kSect, uint32_t Cap>
 __device__ void bin_warp(uint32_t bin, uint32_t lo, uint32_t m, WarpSmem<Cap> &S, const uint32_t *ic, const uint32_t *il,
                          uint32_t bbits, uint32_t ls, uint32_t *__restrict__ locs,
@@ -145,6 +213,10 @@ __device__ void bin_warp(uint32_t bin, uint32_t lo, uint32_t m, WarpSmem<Cap> &S
     if (kSect) {
         S.c2lo[lane] = 0;
         S.c2hi[lane] = 0;
+    }
+    if (m <= 32) {  // one round: ranks straight from ballots (most bins of a sparse index)
+        bin_warp_round<kSect>(bin, lo, m, S.occ, S.c2lo, S.c2hi, ic, il, bbits, ls, locs, rankw, rsect, buckets);
+        return;
     }
     // pass 1 (low digit), from the staged bin: count sweep, scan, placement sweep
     uint32_t cnt = 0;
@@ -518,8 +590,9 @@ TiledPlan tiled_plan(uint32_t ls, uint64_t n_locs) {
     const int nbits = int(2 * ls);
     // sparse indexes only (dense ones: the radix path), < 2^32 locations
     if (n_locs == 0 || n_locs >= (1ull << 32) - 1 || n_locs * 4 >= (1ull << nbits)) return p;
-    // bins of 2^10 seeds = 32 groups of 32, one per lane of a warp (C4: ~43 locations per
-    // bin); tiny seed spaces: one bin
+    // bins of 2^10 seeds = 32 groups of 32 (C2: ~8 locations per bin, C4: ~43); tiny seed
+    // spaces: one bin. (2^9-seed bins, nearly all within one warp round at C4, measured
+    // slower: 2^17 bins' fetch latency)
     const int b = nbits < 10 ? nbits : 10;
     if (nbits - b > kMaxH) return p;
     p.bbits = uint32_t(b);
