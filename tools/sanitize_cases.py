@@ -28,7 +28,7 @@ def direct(R, Q, L, ls, **opts):
     finally:
         for k in opts:
             gpumem.set_option(k, {"index_alg1": 0, "sort_impl": 0, "find_spill": 64, "static_lb": 0,
-                                  "use_bitmap": 1, "rank_sectors": -1, "out_capacity": 0}[k])
+                                  "use_bitmap": 1, "rank_sectors": -1, "out_capacity": 0, "index_tiled": -1}[k])
 
 
 def piped(R, Q, L, ls):
@@ -60,7 +60,8 @@ R, Q = P.R.tobytes(), P.Q.tobytes()
 check(direct(R, Q, P.L, P.ls), want, "c1 direct")
 check(piped(R, Q, P.L, P.ls), want, "c1 pipeline")
 for opts in ({"index_alg1": 1}, {"sort_impl": 1}, {"sort_impl": 2}, {"find_spill": 1}, {"static_lb": 1},
-             {"use_bitmap": 0}, {"rank_sectors": 1}, {"out_capacity": 5}):
+             {"use_bitmap": 0}, {"rank_sectors": 1}, {"out_capacity": 5}, {"index_tiled": 0},
+             {"index_tiled": 1, "rank_sectors": 1}):
     check(direct(R, Q, P.L, P.ls, **opts), want, f"c1 {opts}")
 
 # adversarial tiny cases: homopolymers (heavy queue, coop extensions), (AC)^n, long
@@ -68,6 +69,15 @@ for opts in ({"index_alg1": 1}, {"sort_impl": 1}, {"sort_impl": 2}, {"find_spill
 for n, m, L, ls in ((300, 2000, 20, 10), (5000, 5000, 4500, 13), (2, 3000, 1, 1), (700, 700, 300, 13)):
     check(direct("A" * n, "A" * m, L, ls), pyoracle.homopolymer(n, m, L), f"homopolymer {n} {m} {L}")
 check(piped("A" * 3000, "A" * 3000, 20, 10), pyoracle.homopolymer(3000, 3000, 20), "homopolymer pipeline")
+# tiled index: a hot bin past the CTA's shared memory (global-memory steps 3-4), long
+# buckets placed in input order, rank sectors; the radix path on the same input
+check(direct("A" * 45000, "A" * 500, 20, 13, index_tiled=1), pyoracle.homopolymer(45000, 500, 20),
+      "tiled global-memory bin")
+hot = b"A" * 3000 + b"AC" * 1000 + b"ACGT" * 400 + b"T" * 300
+hot_want = oracle.mems(hot, hot[100:], 20, 13)
+for tiled, sect in ((1, 0), (1, 1), (0, 0)):
+    check(direct(hot, hot[100:], 20, 13, index_tiled=tiled, rank_sectors=sect), hot_want,
+          f"hot seeds tiled={tiled} sect={sect}")
 rng = np.random.default_rng(5)
 for trial in range(20 if quick else 60):
     R1, Q1 = synth.random_pair(rng, int(rng.integers(0, 300)), int(rng.integers(0, 300)), [b"AC", b"ACGT"][trial % 2])
