@@ -980,8 +980,9 @@ static gpumem_status index_build_impl(const gpumem_seq *R, uint32_t ls, uint32_t
     const bool alg1 = n_locs && (g_opt.index_alg1 > 0 || (g_opt.index_alg1 < 0 && n_locs * 4 >= nb));
     const bool tiled = g_opt.index_tiled > 0 || (g_opt.index_tiled < 0 && n_locs <= (1u << 20));
     const TiledPlan tp = (tiled && !alg1) ? tiled_plan(ls, n_locs) : TiledPlan{};
-    // compact table: one entry per occupied seed, or (tiled build) per location, gapped per bin
-    const uint64_t max_occ = (tp.ok ? n_locs : (n_locs < nb ? n_locs : nb)) + 1;
+    // compact table: per location, gapped per chunk / bin (radix and tiled builds), or one
+    // entry per occupied seed (Alg. 1 as written)
+    const uint64_t max_occ = (alg1 ? (n_locs < nb ? n_locs : nb) : n_locs) + 1;
     auto *buckets = static_cast<uint2 *>(sc.get(max_occ * sizeof(uint2)));
     void *fill_scratch = ws_get(kWsFill, ptrs_fill_scratch_bytes(ls), s);
     auto *locs0 = static_cast<uint32_t *>(sc.get((n_locs ? n_locs : 1) * 4));

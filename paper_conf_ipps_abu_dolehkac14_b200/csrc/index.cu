@@ -23,8 +23,11 @@
 //                occupied seeds before the group, a 2-bit saturating count per seed}:
 //                the probe alone gives {first, count} unless a count in the group up
 //                to the seed saturates (>= 3), so most HBM table reads disappear.
-//                A chunk's first rank comes from a scan of the per-chunk occupancy
-//                counts. Either replaces two reads of the HBM-resident 4^ls-entry ptrs.
+//                The table is gapped: a chunk's entries start at its first slot (entries
+//                past its occupied seeds are gaps {next chunk's first slot, 0}), so no
+//                scan of occupancy counts across chunks is needed (Alg. 1 as written,
+//                index_alg1, keeps the dense table). Either replaces two reads of the
+//                HBM-resident 4^ls-entry ptrs.
 // Algorithmic bytes: n_locs * (8 B codes/locs written + 16 B per radix pass read+
 // write) + 4 * (4^ls + 1) B ptrs written + 4^ls / 2 B rank sectors + 8 B per
 // occupied seed.
@@ -75,8 +78,10 @@ __global__ void __launch_bounds__(kCodeThreads) k_seed_codes(const uint64_t *__r
 // chunk_first[c] = first index i of the sorted codes with codes[i] >= c * kChunk, for
 // c in [0, n_chunks]; written by the element at each chunk boundary (no searches).
 __global__ void __launch_bounds__(kCodeThreads) k_chunk_bounds(const uint32_t *__restrict__ codes, uint64_t n,
-                                                               uint64_t n_chunks, uint32_t *__restrict__ first) {
+                                                               uint64_t n_chunks, uint32_t *__restrict__ first,
+                                                               uint2 *__restrict__ buckets) {
     pdl_wait();
+    if (blockIdx.x == 0 && threadIdx.x == 0) buckets[n] = make_uint2(uint32_t(n), 0u);  // the table's closing entry
     // element i in [0, n]: four per thread, grid-stride
     for (uint64_t g = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; 4 * g <= n;
          g += uint64_t(gridDim.x) * blockDim.x) {
@@ -89,28 +94,6 @@ __global__ void __launch_bounds__(kCodeThreads) k_chunk_bounds(const uint32_t *_
             for (uint64_t c = (i == 0 ? 0 : c_prev); c <= c_this && c <= n_chunks; ++c) first[c] = uint32_t(i);
             prev = cur;
         }
-    }
-}
-
-// occ[c] = number of distinct codes in chunk c (one CTA per chunk, block reduction of
-// the run heads; no global atomics -- sorted codes would hammer a few counters)
-__global__ void __launch_bounds__(kCodeThreads) k_occ_count(const uint32_t *__restrict__ codes,
-                                                            const uint32_t *__restrict__ first,
-                                                            uint32_t *__restrict__ occ) {
-    pdl_wait();
-    __shared__ uint32_t ws[kCodeThreads / 32];
-    const uint32_t c = blockIdx.x;
-    const uint64_t lo = first[c], hi = first[c + 1];
-    uint32_t h = 0;
-    for (uint64_t i = lo + threadIdx.x; i < hi; i += kCodeThreads) h += (i == 0 || codes[i - 1] != codes[i]) ? 1u : 0u;
-#pragma unroll
-    for (int o = 16; o; o >>= 1) h += __shfl_xor_sync(0xffffffffu, h, o);
-    if ((threadIdx.x & 31) == 0) ws[threadIdx.x >> 5] = h;
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        uint32_t t = 0;
-        for (int k = 0; k < kCodeThreads / 32; ++k) t += ws[k];
-        occ[c] = t;
     }
 }
 
@@ -249,6 +232,14 @@ __global__ void __launch_bounds__(kFillThreads) k_ptrs_fill(const uint32_t *__re
             if (x) buckets[wr + __popc(ob & lanemask_lt())] = make_uint2(f, x);
             wr += __popc(ob);
         }
+        // gapped table (the radix path): the chunk's entries start at its first slot and
+        // run up to the next chunk's as gaps {its first slot, 0} (see tindex.cu)
+        if (!kCounts) {
+            uint32_t nocc = 0;
+            for (int i = 0; i < kFillThreads / 32; ++i) nocc += wocc[i];
+            for (uint32_t i = uint32_t(lo) + nocc + tid; i < chunk_end; i += kFillThreads)
+                buckets[i] = make_uint2(chunk_end, 0u);
+        }
     }
     // coalesced write-out of the chunk's ptrs, 16 bytes per store (skipped when the dense
     // table is not wanted: the lookup uses the rank directory + compact table, and
@@ -368,6 +359,9 @@ __global__ void __launch_bounds__(kDirThreads) k_dir_fill(const uint32_t *__rest
     }
     if (tid == 0 && s_pend) run_out(s_pend_code, s_pend_first, hi - s_pend_first, s_pend_rank);
     __syncthreads();
+    // gapped table: entries from the chunk's first slot (rank0 = first), gaps {hi, 0} after
+    // its occupied seeds up to the next chunk's first slot (see tindex.cu)
+    for (uint32_t i = r0 + s_carry + tid; i < hi; i += kDirThreads) buckets[i] = make_uint2(hi, 0u);
     // group phase: thread tid owns group tid of the chunk
     const uint32_t o = occ[tid], no = __popc(o), ne = kSect ? ecnt[tid] : 0u;
     uint32_t inc = no, ince = ne;
@@ -728,10 +722,6 @@ cudaError_t launch_ptrs_fill(const uint32_t *sorted_codes, uint64_t n_locs, uint
     auto align = [](uintptr_t p) { return (p + 255) & ~uintptr_t(255); };
     uintptr_t a = align(reinterpret_cast<uintptr_t>(scratch));
     auto *first = reinterpret_cast<uint32_t *>(a);
-    a = align(a + (chunks + 1) * 4);
-    auto *occ = reinterpret_cast<uint32_t *>(a);
-    a = align(a + (chunks + 1) * 4);
-    auto *rank0 = reinterpret_cast<uint32_t *>(a);
     cudaError_t e = cudaSuccess;
     if (rankw) {  // 16 B per group: rank word + rotated occupancy (ORed in by the fill)
         e = fill_async(rankw, 0u, ((nb + 31) / 32) * 16, s);
@@ -739,9 +729,10 @@ cudaError_t launch_ptrs_fill(const uint32_t *sorted_codes, uint64_t n_locs, uint
     }
     uint64_t bblocks = ((n_locs + 1 + 3) / 4 + kCodeThreads - 1) / kCodeThreads;
     if (bblocks > uint64_t(num_sms()) * 16) bblocks = uint64_t(num_sms()) * 16;
-    pdl_launch(k_chunk_bounds, unsigned(bblocks), kCodeThreads, 0, s, sorted_codes, n_locs, chunks, first);
-    pdl_launch(k_occ_count, unsigned(chunks), kCodeThreads, 0, s, sorted_codes, first, occ);
-    pdl_launch(k_occ_scan, 1, 1024, 0, s, occ, uint32_t(chunks), rank0);
+    pdl_launch(k_chunk_bounds, unsigned(bblocks), kCodeThreads, 0, s, sorted_codes, n_locs, chunks, first, buckets);
+    // the compact table is gapped (indexed from each chunk's first slot), so a chunk's
+    // first entry is its first slot: no occupancy count and scan across chunks
+    const uint32_t *rank0 = first;
     constexpr int smem = (kChunk + kChunk / 32) * 4;
     static bool attr = false;
     if (!attr) {
@@ -768,7 +759,7 @@ cudaError_t launch_ptrs_fill(const uint32_t *sorted_codes, uint64_t n_locs, uint
         pdl_launch(k_ptrs_fill<false>, unsigned(chunks), kFillThreads, smem, s, sorted_codes, n_locs, nb, ptrs, rankw, rsect,
                    buckets, first, rank0, ls);
     }
-    note_launch(4);
+    note_launch(2);
     return cudaGetLastError();
 }
 
