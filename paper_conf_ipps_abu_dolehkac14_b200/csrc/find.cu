@@ -484,6 +484,7 @@ __global__ void __launch_bounds__(kT, FindShape<kSect>::kMinB) k_find(const Find
     uint32_t nbuf = 0, nq = 0;
     unsigned long long st_e = 0, st_h = 0;
     QStage qs{s.qw, 0};
+    const uint32_t hvn = P.hv_n ? *P.hv_n : 0u;  // heavy buckets with a minority prefix
     // L2 priorities: lookup tables stay, streamed data goes first (records only when
     // they cannot stay resident anyway, P.recs_stream)
 
@@ -623,15 +624,37 @@ __global__ void __launch_bounds__(kT, FindShape<kSect>::kMinB) k_find(const Find
 #pragma unroll
                 for (int j = 0; j < kQPT; ++j) {
                     if (cnt[j] > P.spill_t) {  // heavy bucket -> reference-axis pieces on the queue
-                        const uint32_t npc = (cnt[j] + kSpillHits - 1) / kSpillHits;
+                        // a bucket reordered minority-left-flank first (index.cu, k_hv_part): a
+                        // query position with the majority flank spills only the minority
+                        // (the others are non-canonical: equal flanks over >= step bases)
+                        uint32_t ncnt = cnt[j];
+                        if (hvn && qa + j >= P.step) {
+                            uint32_t lo2 = 0, hi2 = hvn;
+                            while (lo2 < hi2) {
+                                const uint32_t mid = (lo2 + hi2) >> 1;
+                                if (__ldg(&P.hv_info[mid].x) < beg[j]) lo2 = mid + 1; else hi2 = mid;
+                            }
+                            if (lo2 < hvn) {
+                                const uint4 hv = __ldg(P.hv_info + lo2);
+                                constexpr uint32_t lmask = kL >= 16 ? 0xffffffffu : ((1u << (2 * kL)) - 1u);
+                                if (hv.x == beg[j] && (qs.back16(qa + j) & lmask) == hv.z) ncnt = hv.w;
+                            }
+                        }
+                        if (ncnt == 0) {  // every location of the bucket is non-canonical here
+                            atomicAdd(&P.stats[2], (unsigned long long)cnt[j]);  // hits (decided here)
+                            atomicAdd(&P.stats[3], 1ull);
+                            cnt[j] = 0;
+                            continue;
+                        }
+                        const uint32_t npc = (ncnt + kSpillHits - 1) / kSpillHits;
                         const unsigned long long slot = atomicAdd(P.spill_count, (unsigned long long)npc);
                         if (slot + npc <= P.spill_cap) {
                             for (uint32_t c2 = 0; c2 < npc; ++c2) {
                                 const uint32_t off = c2 * kSpillHits;
-                                P.spill[slot + c2] = make_uint4(qa + j, beg[j] + off, min(kSpillHits, cnt[j] - off), 0u);
+                                P.spill[slot + c2] = make_uint4(qa + j, beg[j] + off, min(kSpillHits, ncnt - off), 0u);
                             }
-                            atomicAdd(&P.stats[2], (unsigned long long)cnt[j]);
-                            atomicAdd(&P.stats[3], 1ull);
+                            atomicAdd(&P.stats[2], (unsigned long long)cnt[j]);  // hits: the skipped majority
+                            atomicAdd(&P.stats[3], 1ull);                          // is decided here too
                             cnt[j] = 0;
                         } else {
                             for (unsigned long long s2 = slot; s2 < P.spill_cap; ++s2)

@@ -47,6 +47,9 @@ struct gpumem_index {
     uint2 *buckets;
     void *recs;                  // uint4 records, or uint2 when rec8
     int rec8;
+    uint4 *hv_info = nullptr;    // heavy buckets (index.cu k_hv_part), or null
+    unsigned int *hv_cnt = nullptr;  // [0] listed, [1] usable (sorted) entries of hv_info
+    uint2 *hv_list = nullptr;
 };
 
 struct gpumem_mems {
@@ -799,6 +802,9 @@ void gpumem_free(void *handle) {
         dfree(x->rsect, x->stream);
         dfree(x->buckets, x->stream);
         dfree(x->recs, x->stream);
+        if (x->hv_info) dfree(x->hv_info, x->stream);
+        if (x->hv_cnt) dfree(x->hv_cnt, x->stream);
+        if (x->hv_list) dfree(x->hv_list, x->stream);
         x->magic = 0;
         delete x;
     } else if (magic == kMagicPipe) {
@@ -993,6 +999,18 @@ static gpumem_status index_build_impl(const gpumem_seq *R, uint32_t ls, uint32_t
     const int rec8 = g_opt.rec8 < 0 ? (step <= 8 ? 1 : 0) : int(g_opt.rec8 != 0);
     void *recs = sc.get((n_locs ? n_locs : 1) * (rec8 ? sizeof(uint2) : sizeof(uint4)));
     if (!recs) return GPUMEM_ERR_NOMEM;
+    // heavy buckets reordered minority-left-flank first (k_hv_part) when the record's left
+    // flank decides canonicity (step <= its width); radix-path directory fills list them
+    const bool hv_ok = n_locs && !tp.ok && !alg1 && step <= (rec8 ? 8u : 16u);
+    uint2 *hv_list = nullptr;
+    uint4 *hv_info = nullptr;
+    unsigned int *hv_cnt = nullptr;
+    if (hv_ok) {
+        hv_list = static_cast<uint2 *>(sc.get(kHvCap * sizeof(uint2)));
+        hv_info = static_cast<uint4 *>(sc.get(kHvCap * sizeof(uint4)));
+        hv_cnt = static_cast<unsigned int *>(sc.get(2 * sizeof(unsigned int)));
+        if (!hv_list || !hv_info || !hv_cnt) return GPUMEM_ERR_NOMEM;
+    }
     bool recs_done = false, fill_done = false;
     if (tp.ok) {
         // Alg. 1 tiled over the seed space: partition, then every bin in shared memory
@@ -1051,12 +1069,20 @@ static gpumem_status index_build_impl(const gpumem_seq *R, uint32_t ls, uint32_t
     }
     if (!fill_done) {
         Stage g("index.ptrs", s);
-        CK(launch_ptrs_fill(codes_sorted, n_locs, ls, ptrs, rankw, rsect, buckets, fill_scratch, s), "ptrs fill");
+        CK(launch_ptrs_fill(codes_sorted, n_locs, ls, ptrs, rankw, rsect, buckets, fill_scratch, s, hv_list, hv_cnt),
+           "ptrs fill");
     }
     if (fork) CK(cudaStreamWaitEvent(s, t_cap->ev_b, 0), "join");
     if (n_locs && !recs_done) {
         Stage g("index.recs", s);
         CK(launch_seed_recs(R->words, ls, locs, n_locs, recs, rec8, s), "seed records");
+    }
+    if (hv_ok) {
+        Stage g("index.heavy", s);
+        CK(launch_heavy_prep(recs, rec8, step, hv_list, hv_cnt, hv_info, s), "heavy buckets");
+        sc.keep(hv_list);
+        sc.keep(hv_info);
+        sc.keep(hv_cnt);
     }
     if (rankw) sc.keep(rankw);
     if (rsect) sc.keep(rsect);
@@ -1064,6 +1090,9 @@ static gpumem_status index_build_impl(const gpumem_seq *R, uint32_t ls, uint32_t
     sc.keep(locs);
     sc.keep(recs);
     auto *h = new gpumem_index{kMagicIdx, dev, s, R, ls, L, step, n_locs, ptrs, locs, rankw, rsect, buckets, recs, rec8};
+    h->hv_info = hv_info;
+    h->hv_cnt = hv_cnt;
+    h->hv_list = hv_list;
     *out = h;
     return GPUMEM_OK;
 }
@@ -1182,6 +1211,8 @@ gpumem_status gpumem_find_mems(const gpumem_index *idx, const gpumem_seq *Q, uin
     P.rankw = idx->rankw;
     P.rsect = idx->rsect;
     P.buckets = idx->buckets;
+    P.hv_info = idx->hv_info;
+    P.hv_n = idx->hv_cnt ? idx->hv_cnt + 1 : nullptr;
     P.ls = ls;
     P.L = L;
     P.step = step;

@@ -32,6 +32,7 @@
 // write) + 4 * (4^ls + 1) B ptrs written + 4^ls / 2 B rank sectors + 8 B per
 // occupied seed.
 #include <algorithm>
+#include <type_traits>
 
 #include "internal.h"
 #include "device.cuh"
@@ -79,9 +80,12 @@ __global__ void __launch_bounds__(kCodeThreads) k_seed_codes(const uint64_t *__r
 // c in [0, n_chunks]; written by the element at each chunk boundary (no searches).
 __global__ void __launch_bounds__(kCodeThreads) k_chunk_bounds(const uint32_t *__restrict__ codes, uint64_t n,
                                                                uint64_t n_chunks, uint32_t *__restrict__ first,
-                                                               uint2 *__restrict__ buckets) {
+                                                               uint2 *__restrict__ buckets, unsigned int *hv_cnt) {
     pdl_wait();
-    if (blockIdx.x == 0 && threadIdx.x == 0) buckets[n] = make_uint2(uint32_t(n), 0u);  // the table's closing entry
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        buckets[n] = make_uint2(uint32_t(n), 0u);  // the table's closing entry
+        if (hv_cnt) hv_cnt[0] = 0;                 // the heavy-bucket list, filled by the directory fill
+    }
     // element i in [0, n]: four per thread, grid-stride
     for (uint64_t g = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; 4 * g <= n;
          g += uint64_t(gridDim.x) * blockDim.x) {
@@ -132,7 +136,8 @@ __global__ void __launch_bounds__(kFillThreads) k_ptrs_fill(const uint32_t *__re
                                                             uint4 *__restrict__ rsect,
                                                             uint2 *__restrict__ buckets,
                                                             const uint32_t *__restrict__ chunk_first,
-                                                            const uint32_t *__restrict__ rank0, uint32_t rot_ls) {
+                                                            const uint32_t *__restrict__ rank0, uint32_t rot_ls,
+                                                            uint2 *__restrict__ hv_list, unsigned int *hv_cnt) {
     pdl_wait();
     extern __shared__ uint32_t cnt[];                // kChunk + kChunk / 32: a pad word per 32 (conflict-free rows)
     __shared__ uint32_t wsum[kFillThreads / 32];
@@ -206,6 +211,10 @@ __global__ void __launch_bounds__(kFillThreads) k_ptrs_fill(const uint32_t *__re
     for (int j = 0; j < kPer; ++j) {
         const uint32_t x = cnt[tid * (kPer + 1) + j];
         cnt[tid * (kPer + 1) + j] = pre;
+        if (hv_cnt && x > kHvT) {  // a heavy bucket: listed for k_hv_part
+            const unsigned slot = atomicAdd(hv_cnt, 1u);
+            if (slot < kHvCap) hv_list[slot] = make_uint2(pre, x);
+        }
         if (!kSect && x) set_rot_occ(rankw, uint32_t(s0) + uint32_t(tid) * kPer + j, rot_ls);
         if (kSect) c2 |= uint64_t(x < 3 ? x : 3u) << (2 * j);
         pre += x;
@@ -280,7 +289,8 @@ __global__ void __launch_bounds__(kDirThreads) k_dir_fill(const uint32_t *__rest
                                                           unsigned long long *__restrict__ rankw,
                                                           uint4 *__restrict__ rsect, uint2 *__restrict__ buckets,
                                                           const uint32_t *__restrict__ chunk_first,
-                                                          const uint32_t *__restrict__ rank0, uint32_t rot_ls) {
+                                                          const uint32_t *__restrict__ rank0, uint32_t rot_ls,
+                                                          uint2 *__restrict__ hv_list, unsigned int *hv_cnt) {
     pdl_wait();
     __shared__ uint32_t occ[kGroups], ecnt[kGroups], c2lo[kGroups], c2hi[kGroups];
     __shared__ uint32_t hpos[kDirThreads + 1];
@@ -305,6 +315,10 @@ __global__ void __launch_bounds__(kDirThreads) k_dir_fill(const uint32_t *__rest
     // one finished run (code, first slot, count, in-chunk rank) into every structure
     auto run_out = [&](uint32_t code, uint32_t first, uint32_t count, uint32_t rank) {
         buckets[r0 + rank] = make_uint2(first, count);
+        if (hv_cnt && count > kHvT) {  // a heavy bucket: listed for k_hv_part
+            const unsigned slot = atomicAdd(hv_cnt, 1u);
+            if (slot < kHvCap) hv_list[slot] = make_uint2(first, count);
+        }
         const uint32_t sd = code - uint32_t(s0), g = sd >> 5, b = sd & 31;
         atomicOr(&occ[g], 1u << b);
         if (!kSect) set_rot_occ(rankw, code, rot_ls);
@@ -573,6 +587,99 @@ __global__ void __launch_bounds__(kCodeThreads) k_seed_recs(const uint64_t *__re
     }
 }
 
+// ---------------------------------------------------------------- heavy buckets
+// A hit whose record's left flank (kL bases before p) equals the query's (kL bases before
+// q) is non-canonical whenever step <= kL and p, q >= step (decide_rec drops it: the left
+// extension reaches step). A hot seed (poly-A, (AC)^n) has one left flank on nearly all
+// of its locations, so for a query position with that same flank only the other records
+// can give a MEM. k_hv_part finds each heavy bucket's majority flank (from 32 evenly
+// spaced records) and reorders the bucket's records minority first (the records of
+// p < step count as minority); k_find then spills only that prefix for such positions.
+// Only the records move (find never reads locs); the MEM set is unchanged.
+constexpr int kHvT_ = 512;  // threads of k_hv_part
+template <bool kRec8>
+__device__ __forceinline__ uint32_t rec_flank(const void *recs, uint64_t k) {
+    return kRec8 ? (static_cast<const uint2 *>(recs)[k].y & 0xffffu) : static_cast<const uint4 *>(recs)[k].y;
+}
+template <bool kRec8>
+__global__ void __launch_bounds__(kHvT_) k_hv_part(void *__restrict__ recs, uint32_t step,
+                                                   const uint2 *__restrict__ hv_list, const unsigned int *hv_cnt,
+                                                   uint4 *__restrict__ hv_info) {
+    pdl_wait();
+    using Rec = typename std::conditional<kRec8, uint2, uint4>::type;
+    extern __shared__ __align__(16) unsigned char hsm[];
+    Rec *buf = reinterpret_cast<Rec *>(hsm);
+    const uint32_t cap = (kRec8 ? 16384u : 8192u);
+    __shared__ uint32_t s_m, s_min, s_maj;
+    const uint32_t n = min(hv_cnt[0], kHvCap);
+    Rec *R = static_cast<Rec *>(recs);
+    for (uint32_t li = blockIdx.x; li < n; li += gridDim.x) {
+        const uint2 e = hv_list[li];  // {first slot, count}
+        if (threadIdx.x < 32) {       // the majority flank among 32 evenly spaced records
+            const uint32_t f = rec_flank<kRec8>(recs, e.x + uint64_t(e.y) * threadIdx.x / 32);
+            uint32_t votes = 0;
+            for (int k = 0; k < 32; ++k) votes += __shfl_sync(0xffffffffu, f, k) == f ? 1u : 0u;
+            uint32_t best = (votes << 5) | (31u - threadIdx.x);  // most votes, then the lowest lane
+#pragma unroll
+            for (int o = 16; o; o >>= 1) best = max(best, __shfl_xor_sync(0xffffffffu, best, o));
+            const uint32_t src = 31u - (best & 31u);
+            const uint32_t m = __shfl_sync(0xffffffffu, f, src);
+            if (threadIdx.x == 0) {
+                s_m = m;
+                s_min = 0;
+                s_maj = 0;
+            }
+        }
+        __syncthreads();
+        const uint32_t m = s_m;
+        if (e.y > cap) {  // too large to reorder here: no skipping for this bucket
+            if (threadIdx.x == 0) hv_info[li] = make_uint4(e.x, e.y, m, e.y);
+            __syncthreads();
+            continue;
+        }
+        for (uint32_t i = threadIdx.x; i < e.y; i += kHvT_) buf[i] = R[e.x + i];
+        __syncthreads();
+        for (uint32_t i = threadIdx.x; i < e.y; i += kHvT_) {
+            const Rec r = buf[i];
+            const uint32_t f = kRec8 ? (uint32_t(r.y) & 0xffffu) : uint32_t(r.y);
+            const bool minority = f != m || r.x < step;
+            const uint32_t pos = minority ? atomicAdd(&s_min, 1u) : e.y - 1u - atomicAdd(&s_maj, 1u);
+            R[e.x + pos] = r;
+        }
+        __syncthreads();
+        if (threadIdx.x == 0) hv_info[li] = make_uint4(e.x, e.y, m, s_min);
+        __syncthreads();
+    }
+}
+
+// one CTA: hv_info[0, n) sorted by first slot (a bitonic network in shared memory);
+// hv_cnt[1] = n, or 0 when the list overflowed kHvCap (no skipping at all then)
+__global__ void __launch_bounds__(1024) k_hv_sort(uint4 *__restrict__ hv_info, unsigned int *hv_cnt) {
+    pdl_wait();
+    __shared__ uint4 a[kHvCap];
+    const uint32_t raw = hv_cnt[0];
+    const uint32_t n = raw > kHvCap ? 0u : raw;
+    uint32_t N = 1;
+    while (N < n) N <<= 1;
+    for (uint32_t i = threadIdx.x; i < N; i += 1024) a[i] = i < n ? hv_info[i] : make_uint4(~0u, 0u, 0u, 0u);
+    __syncthreads();
+    for (uint32_t k = 2; k <= N; k <<= 1) {
+        for (uint32_t j = k >> 1; j > 0; j >>= 1) {
+            for (uint32_t t = threadIdx.x; t < N / 2; t += 1024) {
+                const uint32_t i = ((t & ~(j - 1)) << 1) | (t & (j - 1)), p = i + j;
+                const uint4 x = a[i], y = a[p];
+                if ((x.x > y.x) == ((i & k) == 0)) {
+                    a[i] = y;
+                    a[p] = x;
+                }
+            }
+            __syncthreads();
+        }
+    }
+    for (uint32_t i = threadIdx.x; i < n; i += 1024) hv_info[i] = a[i];
+    if (threadIdx.x == 0) hv_cnt[1] = n;
+}
+
 }  // namespace
 
 cudaError_t launch_seed_recs(const uint64_t *R, uint32_t ls, const uint32_t *locs, uint64_t n_locs, void *recs,
@@ -696,15 +803,33 @@ cudaError_t launch_index_alg1(const uint64_t *R, uint32_t ls, uint32_t step, uin
     }
     if (rsect)
         pdl_launch(k_ptrs_fill<true, true>, unsigned(chunks), kFillThreads, smem, s, cnt, n_locs, nb, (uint32_t *)nullptr,
-                   rankw, rsect, buckets, first, rank0, ls);
+                   rankw, rsect, buckets, first, rank0, ls, (uint2 *)nullptr, (unsigned int *)nullptr);
     else
         pdl_launch(k_ptrs_fill<false, true>, unsigned(chunks), kFillThreads, smem, s, cnt, n_locs, nb, (uint32_t *)nullptr,
-                   rankw, rsect, buckets, first, rank0, ls);
+                   rankw, rsect, buckets, first, rank0, ls, (uint2 *)nullptr, (unsigned int *)nullptr);
     if (rsect) pdl_launch(k_alg1_place<true>, grid_k, kCodeThreads, 0, s, codes, arr, n_locs, k0, step, rankw, rsect, buckets, locs);
     else pdl_launch(k_alg1_place<false>, grid_k, kCodeThreads, 0, s, codes, arr, n_locs, k0, step, rankw, rsect, buckets, locs);
     pdl_launch(k_bucket_fix, unsigned(num_sms() * 8), kCodeThreads, 0, s, buckets, rankw, rsect, nb, locs, big, n_big);
     pdl_launch(k_bucket_big, unsigned(num_sms()), 1024, size_t(kBigSmem * 4), s, buckets, big, n_big, locs);
     note_launch(9);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_heavy_prep(void *recs, int rec8, uint32_t step, const uint2 *hv_list, unsigned int *hv_cnt,
+                              uint4 *hv_info, cudaStream_t s) {
+    const size_t sm = rec8 ? 16384 * sizeof(uint2) : 8192 * sizeof(uint4);
+    static bool attr = false;
+    if (!attr) {
+        cudaError_t e = cudaFuncSetAttribute(k_hv_part<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(sm));
+        if (!e) e = cudaFuncSetAttribute(k_hv_part<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(sm));
+        if (e) return e;
+        attr = true;
+    }
+    const unsigned grid = unsigned(num_sms());
+    if (rec8) pdl_launch(k_hv_part<true>, grid, kHvT_, sm, s, recs, step, hv_list, hv_cnt, hv_info);
+    else pdl_launch(k_hv_part<false>, grid, kHvT_, sm, s, recs, step, hv_list, hv_cnt, hv_info);
+    pdl_launch(k_hv_sort, 1, 1024, 0, s, hv_info, hv_cnt);
+    note_launch(2);
     return cudaGetLastError();
 }
 
@@ -716,7 +841,7 @@ size_t ptrs_fill_scratch_bytes(uint32_t ls) {
 
 cudaError_t launch_ptrs_fill(const uint32_t *sorted_codes, uint64_t n_locs, uint32_t ls, uint32_t *ptrs,
                              unsigned long long *rankw, uint4 *rsect, uint2 *buckets, void *scratch,
-                             cudaStream_t s) {
+                             cudaStream_t s, uint2 *hv_list, unsigned int *hv_cnt) {
     const uint64_t nb = 1ull << (2 * ls);
     const uint64_t chunks = (nb + kChunk - 1) / kChunk;
     auto align = [](uintptr_t p) { return (p + 255) & ~uintptr_t(255); };
@@ -729,7 +854,8 @@ cudaError_t launch_ptrs_fill(const uint32_t *sorted_codes, uint64_t n_locs, uint
     }
     uint64_t bblocks = ((n_locs + 1 + 3) / 4 + kCodeThreads - 1) / kCodeThreads;
     if (bblocks > uint64_t(num_sms()) * 16) bblocks = uint64_t(num_sms()) * 16;
-    pdl_launch(k_chunk_bounds, unsigned(bblocks), kCodeThreads, 0, s, sorted_codes, n_locs, chunks, first, buckets);
+    pdl_launch(k_chunk_bounds, unsigned(bblocks), kCodeThreads, 0, s, sorted_codes, n_locs, chunks, first, buckets,
+               hv_cnt);
     // the compact table is gapped (indexed from each chunk's first slot), so a chunk's
     // first entry is its first slot: no occupancy count and scan across chunks
     const uint32_t *rank0 = first;
@@ -748,16 +874,16 @@ cudaError_t launch_ptrs_fill(const uint32_t *sorted_codes, uint64_t n_locs, uint
     if (!ptrs && n_locs * 4 < nb) {
         if (rsect)
             pdl_launch(k_dir_fill<true>, unsigned(chunks), kDirThreads, 0, s, sorted_codes, nb, rankw, rsect, buckets, first,
-                       rank0, ls);
+                       rank0, ls, hv_list, hv_cnt);
         else
             pdl_launch(k_dir_fill<false>, unsigned(chunks), kDirThreads, 0, s, sorted_codes, nb, rankw, rsect, buckets, first,
-                       rank0, ls);
+                       rank0, ls, hv_list, hv_cnt);
     } else if (rsect) {
         pdl_launch(k_ptrs_fill<true>, unsigned(chunks), kFillThreads, smem, s, sorted_codes, n_locs, nb, ptrs, rankw, rsect,
-                   buckets, first, rank0, ls);
+                   buckets, first, rank0, ls, hv_list, hv_cnt);
     } else {
         pdl_launch(k_ptrs_fill<false>, unsigned(chunks), kFillThreads, smem, s, sorted_codes, n_locs, nb, ptrs, rankw, rsect,
-                   buckets, first, rank0, ls);
+                   buckets, first, rank0, ls, hv_list, hv_cnt);
     }
     note_launch(2);
     return cudaGetLastError();

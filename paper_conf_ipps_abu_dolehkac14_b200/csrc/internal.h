@@ -166,7 +166,13 @@ cudaError_t launch_index_alg1(const uint64_t *R, uint32_t ls, uint32_t step, uin
                               cudaStream_t s);
 cudaError_t launch_ptrs_fill(const uint32_t *sorted_codes, uint64_t n_locs, uint32_t ls, uint32_t *ptrs,
                              unsigned long long *rankw, uint4 *rsect, uint2 *buckets, void *scratch,
-                             cudaStream_t s);
+                             cudaStream_t s, uint2 *hv_list = nullptr, unsigned int *hv_cnt = nullptr);
+// Heavy buckets (> kHvT locations), listed by the directory fill into hv_list (hv_cnt[0]):
+// each one's records reordered minority-left-flank first, hv_info sorted by first slot,
+// hv_cnt[1] = how many (0 if more than kHvCap). Valid when step <= the records' left flank.
+constexpr uint32_t kHvT = 64, kHvCap = 2048;
+cudaError_t launch_heavy_prep(void *recs, int rec8, uint32_t step, const uint2 *hv_list, unsigned int *hv_cnt,
+                              uint4 *hv_info, cudaStream_t s);
 // Dense ptrs[0 .. 4^ls] from the rank directory (rankw or rsect) + compact table (index.cu).
 cudaError_t launch_ptrs_expand(const unsigned long long *rankw, const uint4 *rsect, const uint2 *buckets, uint32_t ls,
                                uint64_t n_locs, uint32_t *ptrs, cudaStream_t s);
@@ -211,6 +217,9 @@ struct FindParams {
     int static_lb;               // ablation: no hit redistribution across lanes
     int recs_stream;             // seed records too large to stay in L2: load them evict_first
     unsigned long long *work;    // [0] most hits one warp dealt locally, [1] warps (D5 balance)
+    const uint4 *hv_info;        // heavy buckets sorted by first slot: {first, count, majority left flank,
+                                 // minority count}; their records minority first (index.cu, k_hv_part)
+    const unsigned int *hv_n;    // how many (null: none built)
     cudaAccessPolicyWindow l2win;  // persisting-L2 window of k_find / k_heavy (num_bytes 0: none)
 };
 uint64_t find_tile_positions(bool rank_sectors);  // query positions per scheduler chunk

@@ -163,6 +163,25 @@ def test_index_sort_paths(opts):
     assert np.array_equal(p, op) and np.array_equal(l, ol)
 
 
+@pytest.mark.parametrize("L,ls", [(20, 13), (28, 13), (12, 5)])
+def test_heavy_bucket_minority_skip(L, ls):
+    """Heavy buckets reordered minority-left-flank first (k_hv_part) and spilled as that
+    prefix for query positions with the majority flank (step <= record flank width):
+    poly-A / (AC)^n / (ACGT)^n hot seeds, run starts, p < step, both the heavy-queue
+    threshold and find_spill 1 (every bucket spilled), 8- and 16-byte records."""
+    rng = np.random.default_rng(11)
+    rnd = lambda n: bytes(rng.choice(list(b"ACGT"), n).tolist())
+    R = b"A" * 1500 + rnd(300) + b"AC" * 700 + rnd(200) + b"A" * 900 + b"ACGT" * 400 + rnd(500) + b"A" * 40
+    Q = rnd(100) + b"A" * 1200 + rnd(50) + b"AC" * 600 + b"A" * 30 + rnd(300) + b"ACGT" * 300 + b"A" * 700
+    want = oracle.mems(R, Q, L, ls)
+    for spill in (64, 1):
+        gpumem.set_option("index_tiled", 0)  # the radix path lists heavy buckets
+        gpumem.set_option("find_spill", spill)
+        got = gpu_mems(R, Q, L, ls)
+        assert np.array_equal(got, want), (L, ls, spill)
+    gpumem.set_option("find_spill", 64)
+
+
 def test_index_short_reference():
     p, l = _index_gpu(b"ACG", 4, 1)
     assert len(l) == 0 and not p.any()
