@@ -12,6 +12,22 @@
 
 namespace gm {
 
+// Bounds checks of the debug variant (tools/variants.py dbg=-DGM_DEBUG_BOUNDS=1): a failed
+// check traps the kernel (the call returns GPUMEM_ERR_CUDA); compiled out by default.
+#ifndef GM_DEBUG_BOUNDS
+#define GM_DEBUG_BOUNDS 0
+#endif
+#if GM_DEBUG_BOUNDS
+#define GM_CHECK(c) \
+    do {            \
+        if (!(c)) __trap(); \
+    } while (0)
+#else
+#define GM_CHECK(c) \
+    do {            \
+    } while (0)
+#endif
+
 // 32 bases starting at position i (i may be up to n; padding makes it safe).
 __device__ __forceinline__ uint64_t win_fwd(const uint64_t *__restrict__ W, uint64_t i) {
     const uint64_t wi = i >> 5;

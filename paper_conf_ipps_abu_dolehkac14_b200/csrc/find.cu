@@ -640,6 +640,7 @@ __global__ void __launch_bounds__(kT, FindShape<kSect>::kMinB) k_find(const Find
                                 if (hv.x == beg[j] && (qs.back16(qa + j) & lmask) == hv.z) ncnt = hv.w;
                             }
                         }
+                        GM_CHECK(ncnt <= cnt[j]);
                         if (ncnt == 0) {  // every location of the bucket is non-canonical here
                             atomicAdd(&P.stats[2], (unsigned long long)cnt[j]);  // hits (decided here)
                             atomicAdd(&P.stats[3], 1ull);

@@ -644,6 +644,7 @@ __global__ void __launch_bounds__(kHvT_) k_hv_part(void *__restrict__ recs, uint
             const uint32_t f = kRec8 ? (uint32_t(r.y) & 0xffffu) : uint32_t(r.y);
             const bool minority = f != m || r.x < step;
             const uint32_t pos = minority ? atomicAdd(&s_min, 1u) : e.y - 1u - atomicAdd(&s_maj, 1u);
+            GM_CHECK(pos < e.y);
             R[e.x + pos] = r;
         }
         __syncthreads();

@@ -62,6 +62,7 @@ __global__ void __launch_bounds__(256) k_tx_bounds(const uint32_t *__restrict__ 
     for (uint64_t i = g0; i <= n; i += uint64_t(gridDim.x) * blockDim.x) {
         const uint32_t cur = i < n ? codes[i] >> bbits : nbins;
         const uint32_t b0 = i ? (codes[i - 1] >> bbits) + 1 : 0u;
+        GM_CHECK(cur <= nbins);
         for (uint32_t b = b0; b <= cur; ++b) binoff[b] = uint32_t(i);
     }
 }
@@ -91,6 +92,7 @@ template <uint32_t Cap>
 __device__ __forceinline__ uint32_t bin_fetch(WarpSmem<Cap> &S, int st, const uint32_t *codes, const uint32_t *lin,
                                               uint32_t lo, uint32_t m) {
     const uint32_t a0 = lo & ~3u, a1 = (lo + m + 3) & ~3u, bytes = (a1 - a0) * 4;
+    GM_CHECK(a1 - a0 <= Cap + 8);
     if ((threadIdx.x & 31) == 0 && m) {
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
         asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_addr(&S.bar[st])), "r"(2 * bytes)
@@ -174,9 +176,11 @@ __device__ void bin_warp_round(uint32_t bin, uint32_t lo, uint32_t m, uint32_t *
     const bool head = valid && (eq & lt) == 0;            // the first of them
     const unsigned hm = __ballot_sync(0xffffffffu, head);
     rank(c, hm, 0, hless);                                // occupied seeds before mine
+    GM_CHECK(!valid || less + __popc(eq & lt) < m);
     if (valid) locs[lo + less + __popc(eq & lt)] = il[lane];
     const uint32_t g = c >> 5, bb = c & 31, len = __popc(eq);
     if (head) {
+        GM_CHECK(hless < m && g < 32);
         buckets[lo + hless] = make_uint2(lo + less, len);
         atomicOr(&occw[g], 1u << bb);
         if (kSect) {
@@ -240,6 +244,7 @@ __device__ void bin_warp(uint32_t bin, uint32_t lo, uint32_t m, WarpSmem<Cap> &S
         const uint32_t base = __shfl_sync(0xffffffffu, run, c & 31);
         if (valid) {
             const uint32_t pos = base + __popc(mt.peers & lt);
+            GM_CHECK(pos < m && m <= Cap);
             S.al[pos] = il[i];
             S.ac[pos] = uint16_t(c);
         }
@@ -271,6 +276,7 @@ __device__ void bin_warp(uint32_t bin, uint32_t lo, uint32_t m, WarpSmem<Cap> &S
         const uint32_t base = __shfl_sync(0xffffffffu, run, c >> 5);
         if (valid) {
             const uint32_t pos = base + __popc(mt.peers & lt);
+            GM_CHECK(pos < m);
             locs[lo + pos] = S.al[i];
             bc[pos] = uint16_t(c);
         }
@@ -300,6 +306,7 @@ __device__ void bin_warp(uint32_t bin, uint32_t lo, uint32_t m, WarpSmem<Cap> &S
                 rank = carry_rank - 1;
             }
             const uint32_t len = i - h + 1, g = c >> 5, b = c & 31;
+            GM_CHECK(rank < m && h <= i && g < 32);
             buckets[lo + rank] = make_uint2(lo + h, len);
             atomicOr(&S.occ[g], 1u << b);
             if (kSect) {
@@ -476,7 +483,11 @@ __device__ void bin_alg1(uint32_t bin, uint32_t lo, uint32_t m, uint32_t cap, co
     uint32_t *dst = in_smem ? S.out : locs + lo;
     for (uint32_t i = tid; i < m; i += kT) {
         const uint32_t k = pad(codes[lo + i] & bmask);
-        if (!(S.cnt[k] & kFlag)) dst[atomicAdd(&S.cnt[k], 1u)] = lin[lo + i];
+        if (!(S.cnt[k] & kFlag)) {
+            const uint32_t pos = atomicAdd(&S.cnt[k], 1u);
+            GM_CHECK(pos < m);
+            dst[pos] = lin[lo + i];
+        }
     }
     // long buckets: the bin's locations arrive ascending (stable radix passes), so each is
     // placed in input order -- rank = same-seed locations before it (block-wide ballot scan)
@@ -500,6 +511,7 @@ __device__ void bin_alg1(uint32_t bin, uint32_t lo, uint32_t m, uint32_t cap, co
                 before += k < w ? ws_e[k] : 0u;
                 tot += ws_e[k];
             }
+            GM_CHECK(!mine || first + run + before + __popc(bb & lanemask_lt()) < m);
             if (mine) dst[first + run + before + __popc(bb & lanemask_lt())] = lin[lo + i];
             run += tot;
             __syncthreads();
