@@ -97,9 +97,10 @@ gpumem_status gpumem_seq_info(const gpumem_seq *s, uint64_t *n_bases, const uint
  *  Eq. 1, :88-90). Indexed locations: p = 0, step, 2*step, ... <= |R| - ls (reading R6).
  *  Result: locs (n_locs uint32, sorted ascending inside each seed, Alg. 1 step 4) and the
  *  lookup directory: per 32 seeds an occupancy/rank word (or rank sector), plus the
- *  compact table {first slot, count} of the occupied seeds -- an exact, compressed form
- *  of the paper's ptrs (4^ls + 1 uint32, ptrs[s] = first slot of seed s, ptrs[4^ls] =
- *  n_locs, :84; 268 MB at ls = 13), which is expanded from it only on demand
+ *  compact table {first slot, count} of the occupied seeds (one entry per sampled
+ *  location at most: each chunk of seeds indexes its entries from its first slot) -- an
+ *  exact, compressed form of the paper's ptrs (4^ls + 1 uint32, ptrs[s] = first slot of
+ *  seed s, ptrs[4^ls] = n_locs, :84; 268 MB at ls = 13), which is expanded from it only on demand
  *  (gpumem_index_view, or find with option use_bitmap = 0). The index references R: R
  *  must outlive it. Async.
  */
