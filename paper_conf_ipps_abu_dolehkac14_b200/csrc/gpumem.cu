@@ -1041,14 +1041,18 @@ static gpumem_status index_build_impl(const gpumem_seq *R, uint32_t ls, uint32_t
         auto *locs1 = static_cast<uint32_t *>(sc.get(n_locs * 4));
         void *scratch = ws_get(kWsRadix, radix_scratch_bytes(n_locs), s);
         if (!codes0 || !codes1 || !locs1 || !scratch) return GPUMEM_ERR_NOMEM;
+        // the first radix pass generates the locations (p = (k0 + i) * step) instead of
+        // reading them: the codes pass writes them only when no pass runs
+        const bool gen = radix_passes(int(2 * ls), n_locs) > 0;
         {
             Stage g("index.codes", s);
-            CK(launch_seed_codes(R->words, ls, step, k0, n_locs, codes0, locs0, s), "seed codes");
+            CK(launch_seed_codes(R->words, ls, step, k0, n_locs, codes0, gen ? nullptr : locs0, s), "seed codes");
         }
         bool alt = false;
         {
             Stage g("index.sort", s);
-            CK(radix_sort_u32(codes0, locs0, codes1, locs1, n_locs, int(2 * ls), scratch, s, &alt),
+            CK(radix_sort_u32(codes0, locs0, codes1, locs1, n_locs, int(2 * ls), scratch, s, &alt, 0, gen ? k0 : 0,
+                              gen ? step : 0u),
                "seed counting sort");
         }
         codes_sorted = alt ? codes1 : codes0;

@@ -3,7 +3,8 @@
 // Built in three steps:
 //  k_seed_codes  for every sampled location p = k*step (Eq. 1, :86-90; reading R6):
 //                the seed integer s = code(R, p) (2*ls bits, first base most
-//                significant, A0 C1 G2 T3, :92) and the location itself.
+//                significant, A0 C1 G2 T3, :92); the location itself only when no radix
+//                pass runs (the first pass generates the locations from the key index).
 //  radix sort    the (s, p) pairs by s, stable (radix.cu): the counting sort of
 //                Alg. 1 steps 1-3 done digit by digit. Stability leaves each
 //                bucket in ascending p order = Alg. 1 step 4, so `locs` is the
@@ -66,11 +67,11 @@ __global__ void __launch_bounds__(kCodeThreads) k_seed_codes(const uint64_t *__r
         }
         if (k + 4 <= n_locs) {
             reinterpret_cast<uint4 *>(codes)[g] = make_uint4(c[0], c[1], c[2], c[3]);
-            reinterpret_cast<uint4 *>(locs)[g] = make_uint4(p[0], p[1], p[2], p[3]);
+            if (locs) reinterpret_cast<uint4 *>(locs)[g] = make_uint4(p[0], p[1], p[2], p[3]);
         } else {
             for (int j = 0; j < 4 && k + j < n_locs; ++j) {
                 codes[k + j] = c[j];
-                locs[k + j] = p[j];
+                if (locs) locs[k + j] = p[j];
             }
         }
     }

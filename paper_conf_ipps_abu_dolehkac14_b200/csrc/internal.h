@@ -123,8 +123,10 @@ cudaError_t launch_revcomp(const uint64_t *in, uint64_t n, uint64_t *out, uint64
 // Radix sort (radix.cu): stable LSD on bits [lo, bits) of the keys, values ride along.
 // Ping-pongs between (k0,v0) and (k1,v1); returns true when the result is in (k1,v1).
 // `scratch` must hold radix_scratch_bytes(n) bytes (digit counts + scan partials).
+// vg_step != 0: v0 is not read -- the values are generated, value of key i = (vg_base + i) * vg_step
 cudaError_t radix_sort_u32(uint32_t *k0, uint32_t *v0, uint32_t *k1, uint32_t *v1, uint64_t n, int bits,
-                           void *scratch, cudaStream_t s, bool *in_alt, int lo = 0);
+                           void *scratch, cudaStream_t s, bool *in_alt, int lo = 0, uint64_t vg_base = 0,
+                           uint32_t vg_step = 0);
 // radix_sort_u64 with dn != null: n is a capacity, the count is min(*dn, n) on the device.
 cudaError_t radix_sort_u64(uint64_t *k0, uint32_t *v0, uint64_t *k1, uint32_t *v1, uint64_t n, int bits,
                            void *scratch, cudaStream_t s, bool *in_alt, int lo = 0,

@@ -220,10 +220,13 @@ __device__ __forceinline__ void mbar_wait(unsigned long long *bar, uint32_t pari
                      : "=r"(ok) : "r"(smem_u32(bar)), "r"(parity) : "memory");
 }
 
-template <class K, class V, int RB>
+template <class K, class V, int RB, bool kGen = false>
 __global__ void __launch_bounds__(kST, GM_RADIX_MINB) k_scatter(const K *__restrict__ kin, const V *__restrict__ vin,
                                                   K *__restrict__ kout, V *__restrict__ vout, Chunking ch0,
-                                                  int shift, int bits, const uint32_t *__restrict__ offs) {
+                                                  int shift, int bits, const uint32_t *__restrict__ offs,
+                                                  uint64_t vg_base, uint32_t vg_step) {
+    // kGen: the values are generated, value of item i = (vg_base + i) * vg_step, vin unread
+    // (the index sort's first pass: the sampled locations in input order)
     pdl_wait();
     constexpr int kBins = 1 << RB;
     constexpr int DPT = (kBins + kST - 1) / kST;  // digits owned per thread: tid, tid + kST, ... (< kBins)
@@ -242,9 +245,10 @@ __global__ void __launch_bounds__(kST, GM_RADIX_MINB) k_scatter(const K *__restr
     auto issue = [&](uint32_t t, int stage) {  // thread 0
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
         asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;"
-                     :: "r"(smem_u32(&S.bar[stage])), "r"(uint32_t(kTile * (sizeof(K) + sizeof(V)))) : "memory");
+                     :: "r"(smem_u32(&S.bar[stage])), "r"(uint32_t(kTile * (sizeof(K) + (kGen ? 0 : sizeof(V)))))
+                     : "memory");
         bulk_g2s(S.k[stage], kin + cb + uint64_t(t) * kTile, kTile * sizeof(K), &S.bar[stage]);
-        bulk_g2s(S.v[stage], vin + cb + uint64_t(t) * kTile, kTile * sizeof(V), &S.bar[stage]);
+        if (!kGen) bulk_g2s(S.v[stage], vin + cb + uint64_t(t) * kTile, kTile * sizeof(V), &S.bar[stage]);
     };
     if (tid == 0) {
         asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" :: "r"(smem_u32(&S.bar[0])) : "memory");
@@ -275,14 +279,14 @@ __global__ void __launch_bounds__(kST, GM_RADIX_MINB) k_scatter(const K *__restr
 #pragma unroll
             for (int j = 0; j < kItems; ++j) {
                 k[j] = S.k[sg][wofs + j * 32 + lane];
-                v[j] = S.v[sg][wofs + j * 32 + lane];
+                v[j] = kGen ? V((vg_base + base + wofs + j * 32 + lane) * vg_step) : S.v[sg][wofs + j * 32 + lane];
             }
         } else {
 #pragma unroll
             for (int j = 0; j < kItems; ++j) {
                 const uint32_t li = wofs + j * 32 + lane;
                 k[j] = li < tile_n ? kin[base + li] : K(0);
-                v[j] = li < tile_n ? vin[base + li] : V(0);
+                v[j] = li < tile_n ? (kGen ? V((vg_base + base + li) * vg_step) : vin[base + li]) : V(0);
             }
         }
         __syncthreads();  // wcnt zeroed
@@ -416,7 +420,8 @@ constexpr int kMaxChunks = 148 * 8;  // >= SMs x resident scatter CTAs
 
 template <class K, int RB>
 cudaError_t radix_sort_rb(K *k0, uint32_t *v0, K *k1, uint32_t *v1, uint64_t n, int lo, int bits, void *scratch,
-                          cudaStream_t s, bool *in_alt, const unsigned long long *dn) {
+                          cudaStream_t s, bool *in_alt, const unsigned long long *dn, uint64_t vg_base = 0,
+                          uint32_t vg_step = 0) {
     constexpr int kBins = 1 << RB;
     const int passes = (bits - lo + RB - 1) / RB;
     const size_t smem = sizeof(ScatterSmem<K, uint32_t, RB>);
@@ -426,6 +431,11 @@ cudaError_t radix_sort_rb(K *k0, uint32_t *v0, K *k1, uint32_t *v1, uint64_t n, 
         e = cudaFuncSetAttribute(k_scatter<K, uint32_t, RB>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
         if (e != cudaSuccess) return e;
         e = cudaFuncSetAttribute(k_scatter<K, uint32_t, RB>, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+        if (e != cudaSuccess) return e;
+        e = cudaFuncSetAttribute(k_scatter<K, uint32_t, RB, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 int(smem));
+        if (e != cudaSuccess) return e;
+        e = cudaFuncSetAttribute(k_scatter<K, uint32_t, RB, true>, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
         if (e != cudaSuccess) return e;
         int per_sm = 0;
         e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_scatter<K, uint32_t, RB>, kST, smem);
@@ -457,7 +467,13 @@ cudaError_t radix_sort_rb(K *k0, uint32_t *v0, K *k1, uint32_t *v1, uint64_t n, 
         uint32_t *tot = totals + size_t(p) * kBins;
         pdl_launch(k_chunk_hist<K, RB>, ch.chunks, kT, 0, s, ka, ch, sh, dbits, counts, tot);
         pdl_launch(k_chunk_scan<RB>, kBins / kWarps, kT, 0, s, counts, tot, ch.chunks, offs);
-        pdl_launch(k_scatter<K, uint32_t, RB>, ch.chunks, kST, smem, s, ka, va, kb, vb, ch, sh, dbits, offs);
+        // pass 0 with generated values (vg_step != 0): v0 is not read
+        if (p == 0 && vg_step)
+            pdl_launch(k_scatter<K, uint32_t, RB, true>, ch.chunks, kST, smem, s, ka, va, kb, vb, ch, sh, dbits, offs,
+                       vg_base, vg_step);
+        else
+            pdl_launch(k_scatter<K, uint32_t, RB>, ch.chunks, kST, smem, s, ka, va, kb, vb, ch, sh, dbits, offs,
+                       vg_base, vg_step);
         note_launch(3);
         std::swap(ka, kb);
         std::swap(va, vb);
@@ -468,16 +484,17 @@ cudaError_t radix_sort_rb(K *k0, uint32_t *v0, K *k1, uint32_t *v1, uint64_t n, 
 
 template <class K>
 cudaError_t radix_sort(K *k0, uint32_t *v0, K *k1, uint32_t *v1, uint64_t n, int lo, int bits, void *scratch,
-                       cudaStream_t s, bool *in_alt, const unsigned long long *dn = nullptr) {
+                       cudaStream_t s, bool *in_alt, const unsigned long long *dn = nullptr, uint64_t vg_base = 0,
+                       uint32_t vg_step = 0) {
     *in_alt = false;
     if (bits > int(8 * sizeof(K))) bits = int(8 * sizeof(K));
     if ((n <= 1 && !dn) || n == 0 || bits <= lo) return cudaSuccess;
     if (!scratch) return cudaErrorInvalidValue;
     if (uint64_t(n) >= (uint64_t(1) << 32)) return cudaErrorInvalidValue;  // 32-bit offsets
     switch (pick_digit_bits(bits - lo, n)) {
-        case 9: return radix_sort_rb<K, 9>(k0, v0, k1, v1, n, lo, bits, scratch, s, in_alt, dn);
-        case 10: return radix_sort_rb<K, 10>(k0, v0, k1, v1, n, lo, bits, scratch, s, in_alt, dn);
-        default: return radix_sort_rb<K, 8>(k0, v0, k1, v1, n, lo, bits, scratch, s, in_alt, dn);
+        case 9: return radix_sort_rb<K, 9>(k0, v0, k1, v1, n, lo, bits, scratch, s, in_alt, dn, vg_base, vg_step);
+        case 10: return radix_sort_rb<K, 10>(k0, v0, k1, v1, n, lo, bits, scratch, s, in_alt, dn, vg_base, vg_step);
+        default: return radix_sort_rb<K, 8>(k0, v0, k1, v1, n, lo, bits, scratch, s, in_alt, dn, vg_base, vg_step);
     }
 }
 
@@ -495,8 +512,8 @@ size_t radix_scratch_bytes(uint64_t n) {  // totals of every pass + counts + off
 }
 
 cudaError_t radix_sort_u32(uint32_t *k0, uint32_t *v0, uint32_t *k1, uint32_t *v1, uint64_t n, int bits,
-                           void *scratch, cudaStream_t s, bool *in_alt, int lo) {
-    return radix_sort<uint32_t>(k0, v0, k1, v1, n, lo, bits, scratch, s, in_alt);
+                           void *scratch, cudaStream_t s, bool *in_alt, int lo, uint64_t vg_base, uint32_t vg_step) {
+    return radix_sort<uint32_t>(k0, v0, k1, v1, n, lo, bits, scratch, s, in_alt, nullptr, vg_base, vg_step);
 }
 
 cudaError_t radix_sort_u64(uint64_t *k0, uint32_t *v0, uint64_t *k1, uint32_t *v1, uint64_t n, int bits,

@@ -655,12 +655,16 @@ cudaError_t launch_index_tiled(const TiledPlan &p, const uint64_t *R, uint32_t l
     }
     // codes and locations, bins by radix; the first location buffer is picked so that the
     // bin-sorted locations do not land in locs (the final ones are written there)
-    const bool odd = radix_passes(int(2 * ls - p.bbits), n_locs) & 1;
+    const int np = radix_passes(int(2 * ls - p.bbits), n_locs);
+    const bool odd = np & 1;
     uint32_t *la = odd ? locs : l1, *lb = odd ? l1 : locs;  // the result: la after even passes, lb after odd
-    e = launch_seed_codes(R, ls, step, k0, n_locs, c0, la, s);
+    // the first pass generates the locations (p = (k0 + i) * step); written here only
+    // when no pass runs
+    e = launch_seed_codes(R, ls, step, k0, n_locs, c0, np ? nullptr : la, s);
     if (e) return e;
     bool alt = false;
-    e = radix_sort_u32(c0, la, c1, lb, n_locs, int(2 * ls), rscratch, s, &alt, int(p.bbits));
+    e = radix_sort_u32(c0, la, c1, lb, n_locs, int(2 * ls), rscratch, s, &alt, int(p.bbits), np ? k0 : 0,
+                       np ? step : 0u);
     if (e) return e;
     const uint32_t *codes = alt ? c1 : c0;
     const uint32_t *lin = alt ? lb : la;
