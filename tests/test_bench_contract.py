@@ -40,3 +40,23 @@ def test_gpus_must_match_world_size():
     r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--impl", "reference", "--gpus", "2",
                         "--config", "c1"], capture_output=True, text=True, timeout=120, cwd=ROOT, env=env)
     assert r.returncode != 0 and "WORLD_SIZE=3" in r.stderr
+
+
+def test_byte_models():
+    """bench.py's byte models: the LSD pass count follows the library's digit rule
+    (radix.cu pick_digit_bits: 8-bit digits above 16 M keys, else 9-bit when that saves a
+    pass), and every stage of both models is positive at C4's sizes (the tiled index stage
+    included)."""
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    import bench
+    assert bench.radix_passes(26, 2_840_909) == 3      # C4 index: 9 + 9 + 8
+    assert bench.radix_passes(26, 31_249_999) == 4     # C5 L=20 index: 8-bit digits
+    assert bench.radix_passes(16, 2_840_909) == 2
+    assert bench.radix_passes(56, 13_420_345) == 7     # C5 L=20 output keys
+    stats = {"positions": 149_997_216, "occupied": 12_000_000, "hits": 17_300_000, "mems": 811_662}
+    impl = bench.impl_bytes(250_000_000, 150_000_000, 13, 100, stats)
+    d7 = bench.d7_bytes(250_000_000, 150_000_000, 13, 100, stats, 151.5)
+    assert set(impl) >= {"pack", "index.codes", "index.sort", "index.ptrs", "index.recs", "index.tiled", "find", "sort"}
+    assert all(v > 0 for v in impl.values()) and all(v > 0 for v in d7.values())
+    # D7's find bytes: 8.25 B per position + 20 B per hit + (mean/2 + 12) B per MEM
+    assert abs(d7["find"] - (8.25 * 149_997_216 + 20 * 17_300_000 + (151.5 / 2 + 12) * 811_662)) < 1
