@@ -1,17 +1,14 @@
 // msd.cu -- MSD bucket sort for unique 64-bit keys (+ optional 32-bit values).
 //
-// Used where the keys are unique, so stability is irrelevant:
-//  * the output: keys (r << qbits | q) with len as value; the
-//    last kernel writes gpumem_triple {r, q, len} directly;
-//  * the index (sort_impl = 0 option): keys (seed code << 32 | location) -- sorting them
-//    groups the sampled locations by seed, ascending inside each seed, i.e. Alg. 1
-//    steps 1-4 in one sort.
+// Used where the keys are unique, so stability is irrelevant: the output, keys
+// (r << qbits | q) with len as value, up to 2 M MEMs; the last
+// kernel writes gpumem_triple {r, q, len} directly.
 // Two passes over the data:
 //  k_bp_hist     chunk c (one CTA per SM, a contiguous run of the input) counts the
 //                top B key bits (2^B <= 16384 buckets) in a shared-memory histogram;
 //  k_bp_colscan  per bucket: exclusive prefix over the chunks + the bucket total;
-//  k_bs_scan     one CTA: bucket offsets;
-//  k_bp_scatter  chunk c moves its keys to its private range of each bucket (order
+//  k_bp_scatter  every CTA scans the bucket totals (CTA 0 publishes the offsets); chunk c
+//                moves its keys to its private range of each bucket (order
 //                inside a chunk's range arbitrary: shared-memory atomic cursors; the
 //                keys are unique and get fully sorted next);
 //  k_bs_local    CTA s sorts the buckets that start in slots [s * kSeg, (s + 1) * kSeg)
@@ -75,8 +72,9 @@ struct NSpec {
 
 // chunk c = elements [c * cs, min((c + 1) * cs, n))
 __global__ void __launch_bounds__(kPT) k_bp_hist(const uint64_t *__restrict__ keys, NSpec ns,
-                                                 uint32_t *__restrict__ counts) {
+                                                 uint32_t *__restrict__ counts, unsigned int *__restrict__ n_big) {
     pdl_wait();
+    if (blockIdx.x == 0 && threadIdx.x == 0) *n_big = 0;  // k_bs_local's list of oversized buckets
     extern __shared__ uint32_t h[];
     const uint64_t n = ns.n();
     const int B = choose_b(n, ns.bits), shift = ns.bits - B;
@@ -123,48 +121,45 @@ __global__ void __launch_bounds__(256) k_bp_colscan(uint32_t *__restrict__ count
     if (lane == 31) totals[b] = inc;
 }
 
-// exclusive scan of totals[0..nb) -> offs[0..nb] (offs[nb] = the sum); each thread owns
-// a contiguous run of ceil(nb / 1024) entries
-__global__ void __launch_bounds__(1024) k_bs_scan(const uint32_t *__restrict__ totals, NSpec ns,
-                                                  uint32_t *__restrict__ offs) {
-    pdl_wait();
-    __shared__ uint32_t ws[32];
-    const uint32_t nb = 1u << choose_b(ns.n(), ns.bits);
-    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-    const uint32_t per = (nb + 1023) / 1024;
-    const uint32_t i0 = threadIdx.x * per, i1 = min(i0 + per, nb);
-    uint32_t sum = 0;
-    for (uint32_t i = i0; i < i1; ++i) sum += totals[i];
-    uint32_t inc = sum;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        const uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
-        if (lane >= o) inc += y;
-    }
-    if (lane == 31) ws[w] = inc;
-    __syncthreads();
-    uint32_t run = inc - sum;
-    for (int k = 0; k < w; ++k) run += ws[k];
-    for (uint32_t i = i0; i < i1; ++i) {
-        offs[i] = run;
-        run += totals[i];
-    }
-    if (threadIdx.x == 1023) offs[nb] = run;
-}
-
+// Every CTA scans the bucket totals itself (<= 16 K of them: one run of 16 per thread),
+// so no separate scan launch sits between the column scan and the scatter; CTA 0 writes
+// the bucket offsets (offs[0, nb]) for k_bs_local / k_bs_big.
 __global__ void __launch_bounds__(kPT) k_bp_scatter(const uint64_t *__restrict__ keys,
                                                     const uint32_t *__restrict__ vals, NSpec ns,
                                                     const uint32_t *__restrict__ rel,
-                                                    const uint32_t *__restrict__ offs, uint64_t *__restrict__ ok,
-                                                    uint32_t *__restrict__ ov) {
+                                                    const uint32_t *__restrict__ totals, uint32_t *__restrict__ offs,
+                                                    uint64_t *__restrict__ ok, uint32_t *__restrict__ ov) {
     pdl_wait();
     extern __shared__ uint32_t cur[];
+    __shared__ uint32_t ws[kPT / 32];
     const uint64_t n = ns.n();
     const int B = choose_b(n, ns.bits), shift = ns.bits - B;
     const uint32_t nb = 1u << B;
     const uint64_t cs = (n + gridDim.x - 1) / gridDim.x;
     const uint32_t *row = rel + uint64_t(blockIdx.x) * nb;
-    for (uint32_t i = threadIdx.x; i < nb; i += kPT) cur[i] = offs[i] + row[i];
+    {
+        const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+        const uint32_t per = (nb + kPT - 1) / kPT;
+        const uint32_t i0 = min(threadIdx.x * per, nb), i1 = min(i0 + per, nb);
+        uint32_t sum = 0;
+        for (uint32_t i = i0; i < i1; ++i) sum += totals[i];
+        uint32_t inc = sum;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
+            if (lane >= o) inc += y;
+        }
+        if (lane == 31) ws[w] = inc;
+        __syncthreads();
+        uint32_t run = inc - sum;
+        for (int k = 0; k < w; ++k) run += ws[k];
+        for (uint32_t i = i0; i < i1; ++i) {
+            if (blockIdx.x == 0) offs[i] = run;
+            cur[i] = run + row[i];
+            run += totals[i];
+        }
+        if (blockIdx.x == 0 && threadIdx.x == kPT - 1) offs[nb] = run;
+    }
     __syncthreads();
     const uint64_t b = uint64_t(blockIdx.x) * cs, e = min(b + cs, n);
     for (uint64_t i = b + threadIdx.x; i < e; i += kPT) {
@@ -506,8 +501,6 @@ static cudaError_t msd_run(uint64_t *keys, uint32_t *vals, NSpec ns, void *scrat
     uint32_t *big = reinterpret_cast<uint32_t *>(c);
     c = align(c + nb_max * 4);
     unsigned int *n_big = reinterpret_cast<unsigned int *>(c);
-    cudaError_t e = fill_async(n_big, 0u, 4, s);
-    if (e != cudaSuccess) return e;
     static bool attr = false;
     if (!attr) {
         cudaFuncSetAttribute(k_bp_hist, cudaFuncAttributeMaxDynamicSharedMemorySize, (1 << kMaxB) * 4);
@@ -515,17 +508,16 @@ static cudaError_t msd_run(uint64_t *keys, uint32_t *vals, NSpec ns, void *scrat
         cudaFuncSetAttribute(k_bs_local, cudaFuncAttributeMaxDynamicSharedMemorySize, int(sizeof(LocalSmem)));
         attr = true;
     }
-    pdl_launch(k_bp_hist, chunks, kPT, nb_max * 4, s, keys, ns, counts);
+    pdl_launch(k_bp_hist, chunks, kPT, nb_max * 4, s, keys, ns, counts, n_big);
     pdl_launch(k_bp_colscan, (nb_max + 7) / 8, 256, 0, s, counts, chunks, ns, totals);
-    pdl_launch(k_bs_scan, 1, 1024, 0, s, totals, ns, offs);
-    pdl_launch(k_bp_scatter, chunks, kPT, nb_max * 4, s, keys, vals, ns, counts, offs, tk, tv);
+    pdl_launch(k_bp_scatter, chunks, kPT, nb_max * 4, s, keys, vals, ns, counts, totals, offs, tk, tv);
     uint64_t segs = (cap + kSeg - 1) / kSeg;
     if (segs > uint64_t(kLocalCtas * num_sms())) segs = kLocalCtas * num_sms();  // blocks loop over the segments
     pdl_launch(k_bs_local, unsigned(segs ? segs : 1), kLT, sizeof(LocalSmem), s, offs, ns, tk, tv, out, big, n_big);
     // oversized buckets: ping-pong with the input's range of the bucket (free: the scatter
     // consumed it and the local pass wrote only other buckets' ranges)
     pdl_launch(k_bs_big, num_sms(), kT, 0, s, offs, big, n_big, tk, tv, keys, xv, ns, out);
-    note_launch(6);
+    note_launch(5);
     return cudaGetLastError();
 }
 
