@@ -433,6 +433,29 @@ def c4_full():
 
 
 @pytest.mark.slow
+@pytest.mark.parametrize("L", [100, 50])
+def test_full_size_index_builders_identical(c4_full, L):
+    """Both index builders at the full C4 / C5 L = 50 size (2.8 M / 6.6 M sampled
+    locations, 4^13 seeds): the tiled Alg. 1 (forced; by default it serves only indexes
+    up to 2^20 locations) and the radix path give the same locs and the same dense ptrs
+    (expanded from each one's gapped table) word for word, and the same MEMs."""
+    P = c4_full
+    Rt, Qt = torch.from_numpy(P.R).cuda(), torch.from_numpy(P.Q).cuda()
+    views, mems = {}, {}
+    for tiled in (0, 1):
+        gpumem.set_option("index_tiled", tiled)
+        Rs = gpumem.pack(Rt)
+        idx = gpumem.index_build(Rs, 13, L)
+        p, l = idx.view()
+        views[tiled] = (p.cpu().numpy().copy(), l.cpu().numpy().copy())
+        mems[tiled] = gpumem.find_mems(idx, gpumem.pack(Qt)).numpy()
+        del p, l, idx, Rs
+        torch.cuda.synchronize()
+    assert np.array_equal(views[0][0], views[1][0]) and np.array_equal(views[0][1], views[1][1])
+    assert np.array_equal(mems[0], mems[1]) and len(mems[0]) > 0
+
+
+@pytest.mark.slow
 @pytest.mark.parametrize("L", [100, 300, 50, 20])
 def test_full_size_c4_c5(c4_full, L):
     """BASELINE sizes (250 Mbp x 150 Mbp), bit-exact against the full oracle run."""
